@@ -1,0 +1,281 @@
+"""Tenant kernels K(B,T), executed block by block on the CPU  (test infrastructure only).
+
+The paper fixes *what* Slate must compute only by reference to the user kernel:
+"The kernel transformation must preserve the semantics of user kernels"
+(§III-A) and "K and K* are isomorphic".  So the oracle of every
+tenant is the tenant kernel itself, its blocks run one after another in linear
+order b = 0 .. B-1 with (x,y,z) = decode(b), each block's arithmetic
+written out in float64 from the tenant's plain definition.  Each block owns a
+disjoint slice of the output (no block reads another block's output), so the
+result does not depend on the order blocks run in -- the property Slate's
+out-of-order, multi-worker execution relies on.
+
+Tenants (BASELINE.json configs; geometry in
+DESIGN.md §Tenants):
+
+  triad        a[i] = b[i] + s*c[i]              STREAM triad (K9), E=1024 elems/block
+  copy         a[i] = b[i]                        STREAM copy (K9), E=4096 elems/block
+  sgemm_naive  C = A @ B, one thread per C elem   CUDA-sample naive SGEMM "MM" (K6), 16x16 blocks
+  spmv_csr     y = A x, CSR                       32 rows/block (K10)
+  blackscholes European call/put, mean over P volatility scenarios (K4, reading Q16),
+               1024 options/block; Phi(x) = erfc(-x/sqrt 2)/2 in double
+  stencil2d    5-point Jacobi sweep, Dirichlet boundary copied; 32x8 points/block (K11)
+  gemm_bf16    C = A @ B^T, A[MxK], B[NxK] bf16 K-major, C fp32; 128x128 tile/block (K12)
+
+Inputs are numpy arrays (fp32, int32, or uint16 bf16 bit patterns); outputs
+are float64 arrays of the same shape as the tenant's output.  Nothing here
+decides an integer from floating point, so no precision pairing is needed.
+"""
+import math
+
+import numpy as np
+from scipy.special import erfc
+
+from .decode import decode
+
+TRIAD_E = 1024
+COPY_E = 4096
+SGEMM_TILE = 16
+SPMV_ROWS = 32
+BS_E = 1024
+STENCIL_BX, STENCIL_BY = 32, 8
+GEMM_TILE = 128
+
+
+def cdiv(a, b):
+    return -(-a // b)
+
+
+def run_grid(grid, block, blocks=None):
+    """Execute ``block(x, y, z)`` for every original block in linear order.
+
+    ``blocks`` optionally restricts execution to a subset of linear indices
+    (used for bounded samples); the default is all of 0 .. B-1.
+    """
+    gx, gy, gz = grid
+    total = gx * gy * gz
+    for b in (range(total) if blocks is None else blocks):
+        block(*decode(b, grid))
+
+
+# ---------------------------------------------------------------- triad / copy
+def triad_grid(n):
+    return (cdiv(n, TRIAD_E), 1, 1)
+
+
+def triad(b, c, s, blocks=None):
+    """STREAM triad a = b + s*c (McCalpin's STREAM; the Stream app of)."""
+    n = b.shape[0]
+    a = np.zeros(n, dtype=np.float64)
+    b64 = b.astype(np.float64)
+    c64 = c.astype(np.float64)
+    s64 = float(s)
+
+    def block(x, y, z):
+        lo, hi = x * TRIAD_E, min((x + 1) * TRIAD_E, n)
+        a[lo:hi] = b64[lo:hi] + s64 * c64[lo:hi]
+
+    run_grid(triad_grid(n), block, blocks)
+    return a
+
+
+def copy_grid(n):
+    return (cdiv(n, COPY_E), 1, 1)
+
+
+def copy(b, blocks=None):
+    """STREAM copy a = b; the output is the input's exact bytes."""
+    n = b.shape[0]
+    a = np.zeros(n, dtype=b.dtype)
+
+    def block(x, y, z):
+        lo, hi = x * COPY_E, min((x + 1) * COPY_E, n)
+        a[lo:hi] = b[lo:hi]
+
+    run_grid(copy_grid(n), block, blocks)
+    return a
+
+
+# ---------------------------------------------------------------- naive SGEMM
+def sgemm_grid(m, n):
+    return (cdiv(n, SGEMM_TILE), cdiv(m, SGEMM_TILE), 1)
+
+
+def sgemm_naive(A, B, blocks=None):
+    """C = A @ B; A is MxK, B is KxN, row-major.  Block (x, y) owns rows
+    16y..16y+15 and columns 16x..16x+15 (thread (tx, ty) -> C[16y+ty][16x+tx])."""
+    m, k = A.shape
+    k2, n = B.shape
+    assert k == k2
+    A64 = A.astype(np.float64)
+    B64 = B.astype(np.float64)
+    C = np.zeros((m, n), dtype=np.float64)
+
+    def block(x, y, z):
+        r0, r1 = y * SGEMM_TILE, min((y + 1) * SGEMM_TILE, m)
+        c0, c1 = x * SGEMM_TILE, min((x + 1) * SGEMM_TILE, n)
+        # thread (tx, ty) computes the dot product of row 16y+ty and column 16x+tx
+        C[r0:r1, c0:c1] = A64[r0:r1, :] @ B64[:, c0:c1]
+
+    run_grid(sgemm_grid(m, n), block, blocks)
+    return C
+
+
+# ---------------------------------------------------------------- CSR SpMV
+def spmv_grid(n_rows):
+    return (cdiv(n_rows, SPMV_ROWS), 1, 1)
+
+
+def spmv_csr(rowptr, col, val, xvec, blocks=None):
+    """y[i] = sum_{j = rowptr[i]}^{rowptr[i+1]-1} val[j] * x[col[j]]."""
+    n_rows = rowptr.shape[0] - 1
+    y = np.zeros(n_rows, dtype=np.float64)
+    v64 = val.astype(np.float64)
+    x64 = xvec.astype(np.float64)
+
+    def block(x, yy, z):
+        for i in range(x * SPMV_ROWS, min((x + 1) * SPMV_ROWS, n_rows)):
+            lo, hi = int(rowptr[i]), int(rowptr[i + 1])
+            y[i] = float(np.sum(v64[lo:hi] * x64[col[lo:hi]]))
+
+    run_grid(spmv_grid(n_rows), block, blocks)
+    return y
+
+
+# ---------------------------------------------------------------- Black-Scholes
+def bs_sigmas(p_count, sigma0=0.30, dsigma=0.01):
+    """Volatility scenarios sigma_p = sigma0 + p*dsigma, p = 0..P-1 (reading Q16).
+    Computed in float32 -- the same float32 values the kernel is given."""
+    return (np.float32(sigma0) + np.float32(dsigma) * np.arange(p_count, dtype=np.float32)).astype(np.float32)
+
+
+def phi(x):
+    """Standard normal CDF, Phi(x) = erfc(-x / sqrt(2)) / 2, in double."""
+    return 0.5 * erfc(-x / math.sqrt(2.0))
+
+
+def bs_option(S, X, T, r, sigma):
+    """Black-Scholes European call and put (Black & Scholes 1973):
+       d1 = (ln(S/X) + (r + sigma^2/2) T) / (sigma sqrt T),  d2 = d1 - sigma sqrt T
+       C  = S Phi(d1) - X e^{-rT} Phi(d2),  P = X e^{-rT} Phi(-d2) - S Phi(-d1)."""
+    sqt = np.sqrt(T)
+    d1 = (np.log(S / X) + (r + 0.5 * sigma * sigma) * T) / (sigma * sqt)
+    d2 = d1 - sigma * sqt
+    disc = X * np.exp(-r * T)
+    call = S * phi(d1) - disc * phi(d2)
+    put = disc * phi(-d2) - S * phi(-d1)
+    return call, put
+
+
+def bs_grid(n):
+    return (cdiv(n, BS_E), 1, 1)
+
+
+def blackscholes(S, X, T, r, sigmas, blocks=None):
+    """Per option, the mean over the P scenarios of the call and put prices."""
+    n = S.shape[0]
+    call = np.zeros(n, dtype=np.float64)
+    put = np.zeros(n, dtype=np.float64)
+    S64, X64, T64 = (v.astype(np.float64) for v in (S, X, T))
+    r64 = float(np.float32(r))
+    sig64 = sigmas.astype(np.float64)
+
+    def block(x, y, z):
+        lo, hi = x * BS_E, min((x + 1) * BS_E, n)
+        cs = np.zeros(hi - lo)
+        ps = np.zeros(hi - lo)
+        for sg in sig64:
+            c, p = bs_option(S64[lo:hi], X64[lo:hi], T64[lo:hi], r64, sg)
+            cs += c
+            ps += p
+        call[lo:hi] = cs / len(sig64)
+        put[lo:hi] = ps / len(sig64)
+
+    run_grid(bs_grid(n), block, blocks)
+    return call, put
+
+
+# ---------------------------------------------------------------- 2-D stencil
+def stencil_grid(h, w):
+    return (cdiv(w, STENCIL_BX), cdiv(h, STENCIL_BY), 1)
+
+
+def stencil2d(field, blocks=None):
+    """One 5-point Jacobi sweep of an HxW field:
+       out[i][j] = (in[i-1][j] + in[i+1][j] + in[i][j-1] + in[i][j+1]) / 4
+    on the interior; boundary points (Dirichlet) are copied."""
+    h, w = field.shape
+    f = field.astype(np.float64)
+    out = np.zeros((h, w), dtype=np.float64)
+
+    def block(x, y, z):
+        i0, i1 = y * STENCIL_BY, min((y + 1) * STENCIL_BY, h)
+        j0, j1 = x * STENCIL_BX, min((x + 1) * STENCIL_BX, w)
+        i = np.arange(i0, i1)[:, None]
+        j = np.arange(j0, j1)[None, :]
+        boundary = (i == 0) | (j == 0) | (i == h - 1) | (j == w - 1)
+        if h < 3 or w < 3:      # every point is a boundary point
+            out[i0:i1, j0:j1] = f[i0:i1, j0:j1]
+            return
+        ic, jc = np.clip(i, 1, h - 2), np.clip(j, 1, w - 2)   # neighbour indices, valid for interior points
+        interior = 0.25 * (f[ic - 1, jc] + f[ic + 1, jc] + f[ic, jc - 1] + f[ic, jc + 1])
+        out[i0:i1, j0:j1] = np.where(boundary, f[i0:i1, j0:j1], interior)
+
+    run_grid(stencil_grid(h, w), block, blocks)
+    return out
+
+
+# ---------------------------------------------------------------- bf16 GEMM
+def bf16_to_f64(bits):
+    """bfloat16 bit patterns (uint16) -> float64.  A bf16 value is the float32
+    whose upper 16 bits are the pattern and whose lower 16 bits are zero."""
+    return (bits.astype(np.uint32) << np.uint32(16)).view(np.float32).astype(np.float64)
+
+
+def gemm_grid(m, n):
+    return (cdiv(n, GEMM_TILE), cdiv(m, GEMM_TILE), 1)
+
+
+def gemm_bf16_tile(A_bits, B_bits, x, y):
+    """One 128x128 output tile (x = column tile, y = row tile) of C = A @ B^T."""
+    m, _ = A_bits.shape
+    n, _ = B_bits.shape
+    r0, r1 = y * GEMM_TILE, min((y + 1) * GEMM_TILE, m)
+    c0, c1 = x * GEMM_TILE, min((x + 1) * GEMM_TILE, n)
+    return bf16_to_f64(A_bits[r0:r1]) @ bf16_to_f64(B_bits[c0:c1]).T
+
+
+def gemm_bf16(A_bits, B_bits, blocks=None):
+    """C[m][n] = sum_k A[m][k] * B[n][k], inputs bf16 widened exactly, summed in double."""
+    m, k = A_bits.shape
+    n, k2 = B_bits.shape
+    assert k == k2
+    C = np.zeros((m, n), dtype=np.float64)
+
+    def block(x, y, z):
+        r0, c0 = y * GEMM_TILE, x * GEMM_TILE
+        t = gemm_bf16_tile(A_bits, B_bits, x, y)
+        C[r0:r0 + t.shape[0], c0:c0 + t.shape[1]] = t
+
+    run_grid(gemm_grid(m, n), block, blocks)
+    return C
+
+
+# ---------------------------------------------------------------- coverage
+def expected_counters(total_blocks, iters):
+    """Deterministic counters of one complete slate launch.
+
+    Every original block runs exactly once (P:L79 isomorphism; P:L127 progress
+    carried in slateIdx), tasks are ``iters`` consecutive blocks, so
+    the task starts are 0, iters, 2*iters, ... < B and the last task is clamped
+    (P:L210).  ``next_clamped`` is the counter value once every task start has
+    been handed out, clamped to the first start >= B.
+    """
+    tasks = cdiv(total_blocks, iters)
+    return {
+        "coverage": np.ones(total_blocks, dtype=np.uint32),
+        "blocks_done": total_blocks,
+        "tasks_done": tasks,
+        "task_starts": list(range(0, total_blocks, iters)),
+        "next_clamped": tasks * iters,
+    }

@@ -1,0 +1,109 @@
+"""Seeded synthetic inputs for the tenant kernels.
+
+This module is the ONLY code shared by the CUDA path's harness (tests, bench)
+and the CPU oracle's harness: it draws random numbers and lays out arrays, and
+holds none of the method's arithmetic.  Recipes follow
+SURVEY.md §8(d): numpy PCG64, seed = 20190520 + 100*cfg + tenant; every tenant
+has an ``int`` mode (small integers: every fp32 result is exact, so GPU and
+oracle agree bit for bit) and a ``float`` mode (realistic values, tolerance).
+"""
+import numpy as np
+
+BASE_SEED = 20190520
+
+
+def seed_for(cfg, tenant):
+    return BASE_SEED + 100 * cfg + tenant
+
+
+def rng(seed):
+    return np.random.Generator(np.random.PCG64(seed))
+
+
+def _vec(g, n, mode, int_lo, int_hi):
+    if mode == "int":
+        return g.integers(int_lo, int_hi + 1, size=n).astype(np.float32)
+    return g.uniform(-1.0, 1.0, size=n).astype(np.float32)
+
+
+def triad_inputs(n, seed, mode="float"):
+    """b, c in U[-1,1) (float) or integers in [-2^10, 2^10] (int); s = 3."""
+    g = rng(seed)
+    return _vec(g, n, mode, -1024, 1024), _vec(g, n, mode, -1024, 1024), np.float32(3.0)
+
+
+def copy_inputs(n, seed, mode="float"):
+    return _vec(rng(seed), n, mode, -1024, 1024)
+
+
+def sgemm_inputs(m, n, k, seed, mode="float"):
+    """A (m x k), B (k x n) row-major fp32; U[-1,1) or integers in [-4, 4]."""
+    g = rng(seed)
+    A = _vec(g, m * k, mode, -4, 4).reshape(m, k)
+    B = _vec(g, k * n, mode, -4, 4).reshape(k, n)
+    return A, B
+
+
+def spmv_inputs(n_rows, seed, mode="float", nnz_per_row=16, band=4096, n_cols=None):
+    """CSR with ``nnz_per_row`` distinct sorted columns per row drawn from the
+    band [i - band, i + band] clipped to [0, n_cols) (fewer when the clipped band
+    is narrower than nnz_per_row).  int32 rowptr/col, fp32 val and x:
+    U[-1,1) or integers in [-2, 2]."""
+    n_cols = n_rows if n_cols is None else n_cols
+    g = rng(seed)
+    i = np.arange(n_rows, dtype=np.int64)
+    start = np.clip(i - band, 0, n_cols)
+    stop = np.clip(i + band + 1, 0, n_cols)
+    width = stop - start
+    per_row = np.minimum(width, nnz_per_row)
+    # k distinct sorted offsets in [0, width): sorted draws with replacement from
+    # [0, width - k] plus 0..k-1 (strictly increasing by construction)
+    k = nnz_per_row
+    draws = np.sort(g.integers(0, 1 << 62, size=(n_rows, k)) % np.maximum(width - per_row + 1, 1)[:, None], axis=1)
+    offs = draws + np.arange(k)[None, :]
+    mask = np.arange(k)[None, :] < per_row[:, None]
+    cols = (start[:, None] + offs)[mask].astype(np.int32)
+    rowptr = np.zeros(n_rows + 1, dtype=np.int64)
+    rowptr[1:] = np.cumsum(per_row)
+    nnz = int(rowptr[-1])
+    val = _vec(g, nnz, mode, -2, 2)
+    x = _vec(g, n_cols, mode, -2, 2)
+    return rowptr.astype(np.int32), cols, val, x
+
+
+def bs_inputs(n, seed):
+    """Option batch in the CUDA SDK BlackScholes sample's ranges: stock price
+    S ~ U[5, 30], strike X ~ U[1, 100], expiry T ~ U[0.25, 10] years; SoA fp32.
+    The riskless rate r = 0.02 is a constant of the workload."""
+    g = rng(seed)
+    S = g.uniform(5.0, 30.0, size=n).astype(np.float32)
+    X = g.uniform(1.0, 100.0, size=n).astype(np.float32)
+    T = g.uniform(0.25, 10.0, size=n).astype(np.float32)
+    return S, X, T, np.float32(0.02)
+
+
+def stencil_inputs(h, w, seed, mode="float"):
+    """HxW fp32 field: U[0,1) (float) or a random integer linear field
+    f = a*i + b*j + c with small integer a, b, c (int)."""
+    g = rng(seed)
+    if mode == "int":
+        a, b, c = (int(v) for v in g.integers(-3, 4, size=3))
+        i = np.arange(h, dtype=np.int64)[:, None]
+        j = np.arange(w, dtype=np.int64)[None, :]
+        return (a * i + b * j + c).astype(np.float32)
+    return g.uniform(0.0, 1.0, size=(h, w)).astype(np.float32)
+
+
+def to_bf16_bits(x):
+    """Round-toward-zero fp32 -> bf16 bit patterns (uint16): the input
+    distribution only; exact for values already representable in bf16."""
+    return (np.ascontiguousarray(x, dtype=np.float32).view(np.uint32) >> np.uint32(16)).astype(np.uint16)
+
+
+def gemm_inputs(m, n, k, seed, mode="float"):
+    """A (m x k) and B (n x k), both K-major bf16 bit patterns (uint16):
+    U[-1,1) or integers in [-2, 2]."""
+    g = rng(seed)
+    A = _vec(g, m * k, mode, -2, 2).reshape(m, k)
+    B = _vec(g, n * k, mode, -2, 2).reshape(n, k)
+    return to_bf16_bits(A), to_bf16_bits(B)

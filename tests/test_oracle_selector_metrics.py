@@ -1,0 +1,109 @@
+"""Pins for oracle/selector.py and oracle/metrics.py (CPU only).
+
+Tab I is compared against the printed table (tests/golden/table1_policy.txt);
+the classifier with the Q9 thresholds must reproduce every Tab II label; and
+Tab I + Tab II must reproduce the paper's statement of which pairs it co-ran
+("Slate concurrently runs RG with all the other kernels ... For all
+pairings for which Slate gains less than 10%, Slate runs the kernels
+consecutively").
+"""
+import itertools
+import os
+
+import pytest
+
+from oracle import metrics as M
+from oracle import selector as S
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _rows(name):
+    return [l.split() for l in open(os.path.join(GOLDEN, name)) if l.strip() and not l.startswith("#")]
+
+
+def test_table1_literal_matches_print():
+    rows = _rows("table1_policy.txt")
+    header = rows[0][1:]
+    for r in rows[1:]:
+        for c, v in zip(header, r[1:]):
+            assert S.TABLE1_LITERAL[(r[0], c)] == v
+
+
+def test_table1_symmetric_reading():
+    for a, b in itertools.product(S.CATEGORIES, repeat=2):
+        assert S.TABLE1[(a, b)] == S.TABLE1[(b, a)]
+    # the two cells the print has asymmetric (Q8) follow the H_C row
+    assert S.TABLE1[("M_M", "H_C")] == "solo" and S.TABLE1[("H_M", "H_C")] == "corun"
+    diff = [k for k in S.TABLE1 if S.TABLE1[k] != S.TABLE1_LITERAL[k]]
+    assert sorted(diff) == [("H_M", "H_C"), ("M_M", "H_C")]
+
+
+def _labels():
+    rows = _rows("table2_profiles.txt")
+    peak = [r for r in rows if r[0] == "peak"][0]
+    pk_bw, pk_fl = float(peak[1]), float(peak[2])
+    out = {}
+    for r in rows:
+        if r[0] == "peak":
+            continue
+        c, m, cat = S.classify(float(r[4]), float(r[3]), 0.0, pk_bw, pk_fl, 0.0)
+        out[r[0]] = (c, m, cat, r[1][0], r[2][0])
+    return out
+
+
+def test_classifier_reproduces_table2():
+    for name, (c, m, cat, c_paper, m_paper) in _labels().items():
+        assert (c, m) == (c_paper, m_paper), name
+    cats = {k: v[2] for k, v in _labels().items()}
+    assert cats == {"BS": "M_M", "GS": "M_M", "MM": "M_M", "RG": "L_C", "TR": "H_M"}
+
+
+@pytest.mark.parametrize("literal", [False, True])
+def test_pairings_reproduce_section_VE(literal):
+    cats = {k: v[2] for k, v in _labels().items()}
+    corun = set()
+    for a, b in itertools.combinations_with_replacement(sorted(cats), 2):
+        if S.policy(cats[a], cats[b], literal) == "corun":
+            corun.add(frozenset((a, b)))
+    assert corun == {frozenset(p) for p in [("RG",), ("RG", "BS"), ("RG", "GS"), ("RG", "MM"), ("RG", "TR")]}
+    assert len(list(itertools.combinations_with_replacement(cats, 2))) == 15
+
+
+def test_select_algorithm():
+    # next kernel first, then the rest of the queue, else solo
+    assert S.select("H_C", ["H_M", "L_C"]) == 0
+    assert S.select("H_C", ["M_M", "H_M"]) == 1
+    assert S.select("H_C", ["M_M", "H_C"]) is None
+    assert S.select("M_M", []) is None
+    # a head bypassed too often blocks look-ahead (Q13)
+    assert S.select("H_C", ["M_M", "H_M"], bypassed=[4, 0]) is None
+
+
+def test_split_fluid_model():
+    # A compute tenant scales linearly; B saturates memory at 1/4 of the SMs
+    n = 148
+    curve_a = {s: 148.0 / s for s in (18, 37, 74, 111, 148)}
+    curve_b = {s: max(1.0, 37.0 / s) for s in (18, 37, 74, 111, 148)}
+    s, t = S.choose_split(curve_a, curve_b, n)
+    assert 30 <= s <= 44
+    assert t < 2.0                          # solo sum is 2.0
+    # no gain possible when both scale linearly: best makespan equals the solo sum
+    lin = {k: 148.0 / k for k in (37, 74, 148)}
+    _, t2 = S.choose_split(lin, lin, n)
+    assert abs(t2 - 2.0) < 1e-9
+    assert S.interp_time(curve_a, 148) == 1.0 and S.interp_time(curve_a, 200) == 1.0
+
+
+def test_metrics_closed_forms():
+    # P10: perfect overlap of equal jobs, no slowdown -> G = 2, STP = 2, ANTT = 1
+    assert M.gain([1, 1], [1, 1]) == 2.0
+    assert M.stp([1, 1], [1, 1]) == 2.0 and M.antt([1, 1], [1, 1]) == 1.0
+    # fully serialised "co-run" -> G = 1, not complementary (P:L99 needs T' < T)
+    assert M.gain([1, 1], [1, 2]) == 1.0 and not M.complementary([1, 1], [1, 2])
+    # sequential schedule of equal jobs: turnarounds 1, 2 -> STP 1.5, ANTT 1.5
+    ta = M.sequential_turnarounds([1, 1])
+    assert ta == [1, 2] and M.stp([1, 1], ta) == 1.5 and M.antt([1, 1], ta) == 1.5
+    assert M.utilisation(6.5e12, 1.0, 6.5e12) == 1.0
+    # STP <= n for any schedule without super-linear speed-up
+    assert M.stp([2, 3, 5], [2, 3, 5]) == 3.0
