@@ -1,0 +1,298 @@
+/*
+ * slate.h -- C ABI of libslate, the B200 (sm_100a) runtime of the Slate
+ * slate-kernel path (Allen, Feng, Ge, "Slate: Enabling Workload-Aware
+ * Efficient Multiprocessing for Modern GPGPUs", IPDPS 2019).
+ *
+ * Citations "P:L<n> §<sec>" are lines of the paper text.
+ *
+ * What the library does (north star):
+ *   Client processes submit kernels to a single-context server (P:L133-139
+ *   §IV-A).  Every kernel K(B,T) is run as the transformed kernel
+ *   K*(B*,T) (§III-A-1): persistent worker CTAs bound to a per-queue SM
+ *   range (Lst1) pull original block indices from a device-side
+ *   atomic task counter (slateIdx, Lst2 P:L199-231), decode them to (x,y,z),
+ *   run the tenant body, and check a device-visible resize word at every task
+ *   boundary, so a kernel shrinks or grows its SM share on the fly with no
+ *   relaunch (§III-C).  A workload-aware selector (Tab I,
+ *   P:L99-121 §III-B) decides which kernels co-run.
+ *
+ * Conventions
+ *   - Every call returns slate_status: 0 = SLATE_OK, > 0 informational,
+ *     < 0 an error.  No exception or abort crosses the ABI.  After an error,
+ *     slate_last_error(session) holds a one-line message (CUDA's text kept).
+ *   - Device pointers are passed as uint64_t device addresses.  In-process
+ *     (endpoint == NULL) they are used as is.  Through a server endpoint every
+ *     pointer must lie inside a buffer registered with slate_share_buffer; the
+ *     server rewrites it to its own mapping of that buffer (the paper's
+ *     shared-buffer -> GPU-pointer table).
+ *   - Sessions are thread-safe (one mutex per session).  Handles
+ *     (slate_kernel, slate_launch_id) are never reused within a server's life.
+ *   - SM ranges are inclusive [sm_lo, sm_hi] in *rank* space (P:L185-186,
+ *     reading Q5): rank r is the r-th smallest %smid the server observed at
+ *     start-up (calibration), 0 <= r < slate_info.num_sms.
+ */
+#ifndef SLATE_H
+#define SLATE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SLATE_ABI_VERSION 1u
+
+/* ------------------------------------------------------------------ status */
+typedef int32_t slate_status;
+#define SLATE_OK            0
+#define SLATE_DONE          1   /* informational: the launch had already completed */
+#define SLATE_EINVAL       (-1) /* bad argument */
+#define SLATE_ENOMEM       (-2) /* out of device memory or control blocks */
+#define SLATE_ECUDA        (-3) /* a CUDA call failed (sticky kernel errors included) */
+#define SLATE_EIPC         (-4) /* no server at the endpoint / transport failure */
+#define SLATE_ETIMEDOUT    (-5) /* slate_sync timed out */
+#define SLATE_ENOTFOUND    (-6) /* unknown kernel or launch handle */
+#define SLATE_ESTATE       (-7) /* call not valid in the current state */
+#define SLATE_EUNSUPPORTED (-8) /* kind not built into this library */
+
+typedef struct slate_session slate_session;
+typedef uint64_t slate_kernel;   /* 0 is never a valid handle */
+typedef uint64_t slate_launch_id; /* monotonically increasing per server, 0 never valid */
+
+/* ------------------------------------------------------------------ kinds
+ * The tenant kernels built into this library.  The paper
+ * injects the Slate code into arbitrary user kernels at run time with a FLEX
+ * scanner + NVRTC; its static alternative ("OMP-like pragma",
+ * P:L157) is what this build does: each kind is compiled into the worker
+ * template at build time.  Block geometry T is fixed per kind. */
+typedef enum {
+  SLATE_KIND_TRIAD = 1,        /* a = b + s*c, fp32; 1024 elems/block, T = 256          */
+  SLATE_KIND_COPY = 2,         /* a = b, fp32; 4096 elems (16 KiB)/block, T = 128       */
+  SLATE_KIND_SGEMM_NAIVE = 3,  /* C = A B, fp32 row-major; 16x16 C tile/block, T = 256  */
+  SLATE_KIND_SPMV_CSR = 4,     /* y = A x, CSR int32/fp32; 32 rows/block, T = 256       */
+  SLATE_KIND_BLACKSCHOLES = 5, /* mean call/put over P sigmas; 1024 options/block, T=256 */
+  SLATE_KIND_STENCIL2D = 6,    /* 5-point Jacobi sweep; 32x8 points/block, T = 256      */
+  SLATE_KIND_GEMM_BF16 = 7,    /* C(fp32) = A B^T, bf16 K-major; 128x128 tile/block     */
+  SLATE_KIND_MAX_ = 8
+} slate_kind;
+
+/* Per-kind argument blocks (passed by value in slate_launch_desc.args).
+ * All arrays are densely packed, 16-byte aligned, row-major. */
+typedef struct { uint64_t a, b, c; uint64_t n; float s; uint32_t pad_; } slate_args_triad;
+typedef struct { uint64_t a, b; uint64_t n; } slate_args_copy;
+typedef struct { uint64_t A, B, C; uint32_t m, n, k, pad_; } slate_args_sgemm;      /* A m x k, B k x n */
+typedef struct { uint64_t rowptr, col, val, x, y; uint32_t n_rows, n_cols; } slate_args_spmv;
+typedef struct {
+  uint64_t S, X, T;        /* inputs [n] fp32: spot, strike, years to expiry */
+  uint64_t call, put;      /* outputs [n] fp32: mean over the P scenarios    */
+  uint64_t sigmas;         /* [n_scen] fp32 volatilities (reading Q16)       */
+  uint64_t n; float r; uint32_t n_scen;
+} slate_args_bs;
+typedef struct { uint64_t in, out; uint32_t h, w; } slate_args_stencil;
+typedef struct { uint64_t A, B, C; uint32_t m, n, k, pad_; } slate_args_gemm;       /* A m x k, B n x k bf16 */
+
+/* ------------------------------------------------------------------ attach */
+/* Open a session ("the daemon creates a session for each application
+ * process upon its first Slate API call").
+ *   endpoint  NULL -> an in-process server on CUDA device `device` (created on
+ *             first use, shared by every in-process session on that device);
+ *             otherwise the POSIX shared-memory name of a running `slated`
+ *             (e.g. "/slate-gpu0"); `device` is then ignored.
+ *   out       receives the session; the caller owns it until slate_detach.
+ * Errors: EINVAL (out == NULL, bad device), EIPC (no server answering at the
+ * endpoint), ECUDA (context creation / calibration failed). */
+slate_status slate_attach(const char* endpoint, int device, slate_session** out);
+
+/* Close a session: waits for all of its outstanding launches (watchdog 60 s),
+ * releases its queue's SMs, closes IPC imports, frees the session.
+ * Errors: ETIMEDOUT (a launch did not finish; the session is freed anyway). */
+slate_status slate_detach(slate_session* s);
+
+typedef struct {
+  uint32_t abi_version;
+  uint32_t num_sms;          /* N: ranks 0..N-1 (calibrated, see header) */
+  uint32_t max_smid;         /* largest %smid observed */
+  uint32_t device;
+  uint64_t server_pid;       /* 0 in-process */
+  double peak_hbm_gbps;      /* peaks the classifier uses (MEASURED_PEAKS.json or defaults) */
+  double peak_fp32_gflops;
+  double peak_tc_tflops;
+} slate_info;
+/* Static facts about the server behind a session.  Errors: EINVAL. */
+slate_status slate_get_info(slate_session* s, slate_info* out);
+
+/* ------------------------------------------------------------------ buffers */
+/* Make client-owned device memory [dev_ptr, dev_ptr+bytes) usable by the
+ * server (kernel IO data travels in buffers shared between
+ * client and daemon).  Through an endpoint: exports a cudaIpcMemHandle of the
+ * allocation, the server opens it once and caches base -> server pointer
+ * (the paper's hash table).  In-process: records the range (identity map).
+ *   handle  receives an opaque id (for slate_unshare_buffer).
+ * Ownership: the CLIENT owns the memory and must keep it alive until every
+ * launch that uses it has completed and the buffer is unshared/detached.
+ * Errors: EINVAL (null/zero range, not device memory), EIPC. */
+slate_status slate_share_buffer(slate_session* s, uint64_t dev_ptr, size_t bytes, uint64_t* handle);
+slate_status slate_unshare_buffer(slate_session* s, uint64_t handle);
+
+/* ------------------------------------------------------------------ kernels */
+#define SLATE_KFLAG_COVERAGE 1u   /* launches may pass a coverage log (debug) */
+
+typedef struct {
+  uint32_t abi_version;    /* SLATE_ABI_VERSION */
+  uint32_t kind;           /* slate_kind */
+  uint32_t iters;          /* SLATE_ITERS, blocks per task; 0 -> auto per launch (reading
+                              Q11): min(10, max(1, B / (4 * occ * N))); GEMM_BF16 -> 1 */
+  uint32_t flags;          /* SLATE_KFLAG_* */
+} slate_kernel_desc;
+
+/* Register a kernel kind (the injector's output).  Computes the
+ * worker's occupancy (the "maximum number of thread blocks that the
+ * designated SMs can support").  Idempotent per
+ * (kind, iters, flags): registering twice returns the same handle.
+ * Errors: EINVAL (bad abi_version / kind / flags), EUNSUPPORTED. */
+slate_status slate_register_kernel(slate_session* s, const slate_kernel_desc* d, slate_kernel* out);
+
+/* ------------------------------------------------------------------ launch */
+#define SLATE_PLACE_AUTO  0u  /* the selector decides co-run or solo (Tab I) */
+#define SLATE_PLACE_SOLO  1u  /* wait for a free GPU, run on all SMs */
+#define SLATE_PLACE_CORUN 2u  /* run now on [sm_lo, sm_hi] (resizes this queue's range) */
+
+#define SLATE_MODE_SLATE      0u  /* transformed kernel K*(B*,T): persistent workers */
+#define SLATE_MODE_STANDALONE 1u  /* the original K(B,T) on the hardware block
+                                     scheduler, same body code (bit-exact reference,
+                                     and the "vanilla CUDA" schedule) */
+
+typedef struct {
+  uint32_t grid[3];        /* original grid (Gx, Gy, Gz); must equal the grid the
+                              kind's args imply (e.g. triad: ceil(n/1024), 1, 1) */
+  uint32_t placement;      /* SLATE_PLACE_* */
+  uint32_t sm_lo, sm_hi;   /* CORUN: inclusive rank range */
+  uint32_t mode;           /* SLATE_MODE_* */
+  uint32_t args_size;      /* sizeof the kind's slate_args_* */
+  const void* args;        /* copied before the call returns */
+  uint64_t coverage;       /* 0, or device u32[Gx*Gy*Gz] zero-filled by the caller:
+                              every executed original block b does cov[b] += 1 */
+} slate_launch_desc;
+
+/* Submit one kernel launch, asynchronously (the API "wraps ... launch",
+ * P:L139).  Launches of one session run in submission order, one after
+ * another (one queue per process); launches of different sessions may
+ * run concurrently on disjoint SM ranges.  Returns once the launch is queued
+ * (it may already be running).
+ *   out  receives the launch id.
+ * Ordering: the server runs launches on its own non-blocking streams, which do
+ * not wait for the caller's streams: the caller must have finished writing the
+ * inputs (and zeroing a coverage log) before the call, and must slate_sync
+ * before reading the outputs.
+ * Errors: EINVAL (grid inconsistent with args, zero grid, B >= 2^31, a pointer
+ * outside every shared buffer through an endpoint, lo > hi, hi >= N),
+ * ENOTFOUND (kernel), ENOMEM (control-block pool exhausted), ECUDA. */
+slate_status slate_launch(slate_session* s, slate_kernel k, const slate_launch_desc* d, slate_launch_id* out);
+
+/* Resize the SM range of the queue that owns launch l to [sm_lo, sm_hi]
+ * (§III-C; the dispatcher's start_sm/end_sm, Lst3 P:L250-251).
+ * Publishes {epoch+1, lo, hi} to the device with a stream memory write that
+ * needs no SM; workers outside the range retire at their next task boundary
+ * (shrink), and ranks newly in range get workers (grow: waiting CTAs join, plus
+ * a top-up launch bound to the new ranks sharing the same task counter).  The
+ * running workers are never relaunched; progress is only in the counter.
+ * Returns once the write is enqueued; completion is visible in slate_query.
+ * Errors: EINVAL (lo > hi, hi >= N), ENOTFOUND.  SLATE_DONE (+1) if l had
+ * already completed (the queue's range is still updated). */
+slate_status slate_resize(slate_session* s, slate_launch_id l, uint32_t sm_lo, uint32_t sm_hi);
+
+/* Wait until launch l (0 = every launch of this session) has run every block
+ * and all its worker CTAs have exited.  timeout_us < 0 waits forever.
+ * Errors: ETIMEDOUT, ECUDA (sticky kernel error), ENOTFOUND. */
+slate_status slate_sync(slate_session* s, slate_launch_id l, int64_t timeout_us);
+
+/* ------------------------------------------------------------------ profile */
+#define SLATE_PROF_CURVE 1u  /* also time the kernel on N, 3N/4, N/2, N/3, N/4, N/8 SMs */
+#define SLATE_PROF_FORCE 2u  /* ignore the cached entry */
+
+typedef struct {
+  double solo_ms;          /* time on all SMs */
+  double hbm_gbps;         /* algorithmic bytes / solo time */
+  double fp32_gflops;      /* algorithmic fp32 flops / solo time */
+  double tc_tflops;        /* algorithmic tensor-core flops / solo time */
+  double hbm_frac, fp32_frac, tc_frac;   /* of the server's peaks (slate_info) */
+  uint32_t c_level, m_level;             /* 0 = L, 1 = M, 2 = H (reading Q9) */
+  uint32_t category;       /* 0 L_C, 1 M_C, 2 H_C, 3 M_M, 4 H_M (Tab I order) */
+  uint32_t n_curve;        /* points in curve_* */
+  uint32_t curve_sms[8];
+  double curve_ms[8];
+  double bytes, flops;     /* algorithmic bytes and flops of the sample launch */
+} slate_profile_t;
+
+/* Profile a kernel solo on a sample launch ("The daemon profiles
+ * kernels at their first time run, and saves the profile data in the kernel
+ * profile table").  Runs the sample through the worker on all SMs (and on
+ * fewer SMs with SLATE_PROF_CURVE), times it with CUDA events, and classifies
+ * it; the entry is cached per (kind, shape) and used by SLATE_PLACE_AUTO.
+ * The sample launch's outputs are written (the kernel really runs).
+ * Requires an idle GPU for this session's server (waits for it).
+ * Errors: EINVAL, ECUDA, ENOTFOUND. */
+slate_status slate_profile(slate_session* s, slate_kernel k, const slate_launch_desc* sample,
+                           uint32_t flags, slate_profile_t* out);
+
+/* ------------------------------------------------------------------ query */
+typedef struct {
+  uint32_t state;          /* 0 queued, 1 issued, 2 complete */
+  uint32_t blocks_done;    /* original blocks executed (== B when complete) */
+  uint32_t tasks_done;     /* tasks executed (== ceil(B/iters)) */
+  uint32_t total_blocks;   /* B */
+  uint32_t next_clamped;   /* min(slateIdx, ceil(B/iters)*iters) */
+  uint32_t next_raw;       /* raw slateIdx (overshoots; nondeterministic) */
+  uint32_t live_workers;   /* worker CTAs (or warps) still live */
+  uint32_t iters;
+  uint32_t sm_lo, sm_hi;   /* the queue's current range */
+  uint32_t n_resizes;      /* resizes applied while the launch ran */
+  uint32_t n_topups;       /* top-up worker launches (grow) */
+  uint32_t workers_started;/* worker CTAs/warps that ran at least one prologue */
+  uint32_t coverage_ok;    /* 1 if a coverage log was given and every entry is 1 */
+  uint32_t epoch;          /* the queue's resize-word epoch now */
+  uint32_t shrink_epoch;   /* last epoch whose shrink the device saw complete */
+  uint32_t join_epoch;     /* last epoch in which a worker joined (grow) */
+  uint32_t pad_;
+  uint64_t t_first_ns;     /* %globaltimer at the first task start (device clock) */
+  uint64_t t_last_ns;      /* %globaltimer when the last block finished */
+  double start_ms, end_ms; /* CUDA-event times of the launch relative to the server's epoch */
+  double resize_us[16];    /* host-observed latency of the first 16 resizes (shrink: until
+                              no worker is live outside the range; grow: until the first
+                              task starts on a new rank); -1 if not observed */
+} slate_launch_info;
+
+/* Counters and timing of a launch (copied out).  Errors: ENOTFOUND. */
+slate_status slate_query(slate_session* s, slate_launch_id l, slate_launch_info* out);
+
+/* ------------------------------------------------------------------ strings */
+const char* slate_status_string(slate_status st);     /* static string */
+const char* slate_last_error(slate_session* s);       /* session-owned, valid until the next call */
+
+/* ------------------------------------------------------------------ host logic
+ * The selector's pure functions, exported so they can be checked without a GPU.
+ * Categories: 0 L_C, 1 M_C, 2 H_C, 3 M_M, 4 H_M. */
+/* Classify fractions of peak (reading Q9). Returns the category;
+ * *c_level/*m_level receive 0 = L, 1 = M, 2 = H (may be NULL). */
+uint32_t slate_classify(double hbm_frac, double fp32_frac, double tc_frac, uint32_t* c_level, uint32_t* m_level);
+/* Tab I: 1 = corun, 0 = solo.  literal != 0 uses the table as
+ * printed, otherwise the symmetric reading (Q8). */
+int slate_policy(uint32_t cat_active, uint32_t cat_candidate, int literal);
+/* Selection algorithm (reading Q13): index of the first queued
+ * candidate to co-run with the active kernel, or -1 for solo.  bypassed may
+ * be NULL. */
+int slate_select(uint32_t cat_active, const uint32_t* queue_cats, const uint32_t* bypassed, uint32_t n,
+                 uint32_t max_bypass, int literal);
+/* SM split for a co-run (reading Q10): SMs for candidate B (A keeps n - s),
+ * minimising the fluid-model makespan with grow-on-completion, given solo
+ * time curves (sms ascending, ms).  Returns s (multiple of step) and the
+ * predicted makespan in *makespan_ms (may be NULL). */
+uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t n_a,
+                            const uint32_t* sms_b, const double* ms_b, uint32_t n_b,
+                            uint32_t n_sms, uint32_t step, double* makespan_ms);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SLATE_H */

@@ -1,0 +1,211 @@
+// capi.cu -- the extern "C" boundary of libslate (include/slate.h).
+// In-process sessions talk to a per-device Server directly; sessions attached
+// to an endpoint go through the shared-memory transport (ipc.cu).
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "ipc.h"
+#include "server.h"
+
+using slate::Server;
+
+struct slate_session {
+  Server* srv = nullptr;                 // in-process
+  std::unique_ptr<slate::RemoteClient> remote;   // through an endpoint
+  uint32_t queue = 0;
+  std::mutex mu;
+  std::string last_error;
+  struct Shared { uint64_t id, base, bytes; };
+  std::vector<Shared> shared;
+  uint64_t next_share = 1;
+};
+
+namespace {
+std::mutex g_servers_mu;
+std::map<int, Server*> g_servers;   // in-process servers live until process exit
+
+Server* local_server(int device, std::string* err, int* rc) {
+  std::lock_guard<std::mutex> g(g_servers_mu);
+  auto it = g_servers.find(device);
+  if (it != g_servers.end()) return it->second;
+  Server* s = new Server(device);
+  *rc = s->init(err);
+  if (*rc != SLATE_OK) {
+    delete s;
+    return nullptr;
+  }
+  g_servers[device] = s;
+  return s;
+}
+
+slate_status fail(slate_session* s, slate_status rc, const std::string& msg) {
+  if (s) s->last_error = msg;
+  return rc;
+}
+}  // namespace
+
+extern "C" {
+
+const char* slate_status_string(slate_status st) {
+  switch (st) {
+    case SLATE_OK: return "SLATE_OK";
+    case SLATE_DONE: return "SLATE_DONE";
+    case SLATE_EINVAL: return "SLATE_EINVAL";
+    case SLATE_ENOMEM: return "SLATE_ENOMEM";
+    case SLATE_ECUDA: return "SLATE_ECUDA";
+    case SLATE_EIPC: return "SLATE_EIPC";
+    case SLATE_ETIMEDOUT: return "SLATE_ETIMEDOUT";
+    case SLATE_ENOTFOUND: return "SLATE_ENOTFOUND";
+    case SLATE_ESTATE: return "SLATE_ESTATE";
+    case SLATE_EUNSUPPORTED: return "SLATE_EUNSUPPORTED";
+    default: return "SLATE_UNKNOWN";
+  }
+}
+
+const char* slate_last_error(slate_session* s) { return s ? s->last_error.c_str() : "no session"; }
+
+slate_status slate_attach(const char* endpoint, int device, slate_session** out) {
+  if (!out) return SLATE_EINVAL;
+  *out = nullptr;
+  auto s = std::make_unique<slate_session>();
+  std::string err;
+  int rc = SLATE_OK;
+  if (endpoint == nullptr) {
+    if (device < 0) return SLATE_EINVAL;
+    s->srv = local_server(device, &err, &rc);
+    if (!s->srv) return rc;
+    s->queue = s->srv->open_queue();
+    if (!s->queue) return SLATE_ENOMEM;
+  } else {
+    s->remote = std::make_unique<slate::RemoteClient>();
+    rc = s->remote->connect(endpoint, &err);
+    if (rc != SLATE_OK) return rc;
+  }
+  *out = s.release();
+  return SLATE_OK;
+}
+
+slate_status slate_detach(slate_session* s) {
+  if (!s) return SLATE_EINVAL;
+  std::string err;
+  int rc = SLATE_OK;
+  {
+    std::lock_guard<std::mutex> g(s->mu);
+    if (s->srv) rc = s->srv->close_queue(s->queue, 60000000, &err);
+    else if (s->remote) rc = s->remote->detach(&err);
+  }
+  delete s;
+  return rc;
+}
+
+slate_status slate_get_info(slate_session* s, slate_info* out) {
+  if (!s || !out) return SLATE_EINVAL;
+  std::lock_guard<std::mutex> g(s->mu);
+  if (s->srv) {
+    *out = s->srv->info();
+    return SLATE_OK;
+  }
+  std::string err;
+  const int rc = s->remote->info(out, &err);
+  return rc == SLATE_OK ? rc : fail(s, rc, err);
+}
+
+slate_status slate_share_buffer(slate_session* s, uint64_t dev_ptr, size_t bytes, uint64_t* handle) {
+  if (!s || !handle || !dev_ptr || !bytes) return fail(s, SLATE_EINVAL, "null or empty buffer");
+  std::lock_guard<std::mutex> g(s->mu);
+  cudaPointerAttributes attr;
+  if (cudaPointerGetAttributes(&attr, reinterpret_cast<void*>(dev_ptr)) != cudaSuccess ||
+      attr.type != cudaMemoryTypeDevice) {
+    cudaGetLastError();
+    return fail(s, SLATE_EINVAL, "not device memory");
+  }
+  if (s->remote) {
+    std::string err;
+    const int rc = s->remote->share(dev_ptr, bytes, handle, &err);
+    return rc == SLATE_OK ? rc : fail(s, rc, err);
+  }
+  *handle = s->next_share++;
+  s->shared.push_back({*handle, dev_ptr, bytes});
+  return SLATE_OK;
+}
+
+slate_status slate_unshare_buffer(slate_session* s, uint64_t handle) {
+  if (!s) return SLATE_EINVAL;
+  std::lock_guard<std::mutex> g(s->mu);
+  if (s->remote) {
+    std::string err;
+    const int rc = s->remote->unshare(handle, &err);
+    return rc == SLATE_OK ? rc : fail(s, rc, err);
+  }
+  for (size_t i = 0; i < s->shared.size(); ++i)
+    if (s->shared[i].id == handle) {
+      s->shared.erase(s->shared.begin() + long(i));
+      return SLATE_OK;
+    }
+  return fail(s, SLATE_ENOTFOUND, "unknown buffer handle");
+}
+
+slate_status slate_register_kernel(slate_session* s, const slate_kernel_desc* d, slate_kernel* out) {
+  if (!s || !d || !out) return fail(s, SLATE_EINVAL, "null argument");
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  const int rc = s->srv ? s->srv->register_kernel(d, out, &err) : s->remote->register_kernel(d, out, &err);
+  return rc == SLATE_OK ? rc : fail(s, rc, err);
+}
+
+slate_status slate_launch(slate_session* s, slate_kernel k, const slate_launch_desc* d, slate_launch_id* out) {
+  if (!s || !d || !out) return fail(s, SLATE_EINVAL, "null argument");
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  const int rc = s->srv ? s->srv->launch(s->queue, k, d, out, &err) : s->remote->launch(k, d, out, &err);
+  return rc == SLATE_OK ? rc : fail(s, rc, err);
+}
+
+slate_status slate_resize(slate_session* s, slate_launch_id l, uint32_t lo, uint32_t hi) {
+  if (!s) return SLATE_EINVAL;
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  const int rc = s->srv ? s->srv->resize(s->queue, l, lo, hi, &err) : s->remote->resize(l, lo, hi, &err);
+  return rc >= SLATE_OK ? rc : fail(s, rc, err);
+}
+
+slate_status slate_sync(slate_session* s, slate_launch_id l, int64_t timeout_us) {
+  if (!s) return SLATE_EINVAL;
+  std::string err;
+  // not under the session mutex: other threads may keep launching on the session
+  const int rc = s->srv ? s->srv->sync(s->queue, l, timeout_us, &err) : s->remote->sync(l, timeout_us, &err);
+  if (rc != SLATE_OK) {
+    std::lock_guard<std::mutex> g(s->mu);
+    return fail(s, rc, err);
+  }
+  return rc;
+}
+
+slate_status slate_profile(slate_session* s, slate_kernel k, const slate_launch_desc* d, uint32_t flags,
+                           slate_profile_t* out) {
+  if (!s || !d || !out) return fail(s, SLATE_EINVAL, "null argument");
+  std::string err;
+  const int rc = s->srv ? s->srv->profile(k, d, flags, out, &err) : s->remote->profile(k, d, flags, out, &err);
+  if (rc != SLATE_OK) {
+    std::lock_guard<std::mutex> g(s->mu);
+    return fail(s, rc, err);
+  }
+  return rc;
+}
+
+slate_status slate_query(slate_session* s, slate_launch_id l, slate_launch_info* out) {
+  if (!s || !out) return fail(s, SLATE_EINVAL, "null argument");
+  std::string err;
+  const int rc = s->srv ? s->srv->query(l, out, &err) : s->remote->query(l, out, &err);
+  if (rc != SLATE_OK) {
+    std::lock_guard<std::mutex> g(s->mu);
+    return fail(s, rc, err);
+  }
+  return rc;
+}
+
+}  // extern "C"

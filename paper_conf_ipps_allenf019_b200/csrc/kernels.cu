@@ -1,0 +1,80 @@
+// kernels.cu -- instantiates the worker and standalone kernels for every tenant
+// kind and exposes a small host-side dispatch table to the runtime.
+#include <cstring>
+#include "kernels.h"
+#include "slate_device.cuh"
+#include "tenants.cuh"
+#include "gemm_tc.cuh"
+
+namespace slate {
+
+__global__ void calibrate_kernel(uint32_t* out, uint32_t spin_ns) {
+  if (threadIdx.x == 0) out[blockIdx.x] = smid();
+  const uint64_t t0 = globaltimer();
+  while (globaltimer() - t0 < spin_ns) {
+  }
+}
+
+namespace {
+
+template <class Tn>
+cudaError_t launch_worker_t(const WorkerCommon& w, const void* args, uint32_t grid, cudaStream_t st) {
+  WorkerParams<typename Tn::Args> p;
+  std::memcpy(&p.args, args, sizeof(typename Tn::Args));
+  p.gx = w.gx; p.gy = w.gy; p.gz = w.gz; p.B = w.B; p.iters = w.iters; p.occ = w.occ;
+  p.bound_lo = w.bound_lo; p.bound_hi = w.bound_hi; p.n_ranks = w.n_ranks;
+  p.standby_timeout_ns = w.standby_timeout_ns;
+  p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
+  void* kargs[] = {&p};
+  return cudaLaunchKernel(reinterpret_cast<const void*>(&slate_worker<Tn>), dim3(grid), dim3(Tn::kThreads), kargs,
+                          Tn::kSmem, st);
+}
+
+template <class Tn>
+cudaError_t launch_standalone_t(const void* args, dim3 grid, cudaStream_t st) {
+  typename Tn::Args a;
+  std::memcpy(&a, args, sizeof(a));
+  void* kargs[] = {&a};
+  return cudaLaunchKernel(reinterpret_cast<const void*>(&standalone<Tn>), grid, dim3(Tn::kThreads), kargs, Tn::kSmem,
+                          st);
+}
+
+template <class Tn>
+KindOps make_ops(uint32_t default_iters) {
+  KindOps o;
+  o.worker_fn = reinterpret_cast<const void*>(&slate_worker<Tn>);
+  o.standalone_fn = reinterpret_cast<const void*>(&standalone<Tn>);
+  o.threads = Tn::kThreads;
+  o.smem = Tn::kSmem;
+  o.args_size = sizeof(typename Tn::Args);
+  o.default_iters = default_iters;
+  o.launch_worker = &launch_worker_t<Tn>;
+  o.launch_standalone = &launch_standalone_t<Tn>;
+  return o;
+}
+
+}  // namespace
+
+const KindOps* kind_ops(uint32_t kind) {
+  static KindOps table[SLATE_KIND_MAX_];
+  static bool init = false;
+  if (!init) {
+    table[SLATE_KIND_TRIAD] = make_ops<Triad>(0);
+    table[SLATE_KIND_COPY] = make_ops<Copy>(0);
+    table[SLATE_KIND_SGEMM_NAIVE] = make_ops<SgemmNaive>(0);
+    table[SLATE_KIND_SPMV_CSR] = make_ops<SpmvCsr>(0);
+    table[SLATE_KIND_BLACKSCHOLES] = make_ops<BlackScholes>(0);
+    table[SLATE_KIND_STENCIL2D] = make_ops<Stencil2D>(0);
+    table[SLATE_KIND_GEMM_BF16] = gemm_tc_ops();
+    init = true;
+  }
+  if (kind == 0 || kind >= SLATE_KIND_MAX_) return nullptr;
+  return table[kind].worker_fn ? &table[kind] : nullptr;
+}
+
+cudaError_t launch_calibrate(uint32_t* out, uint32_t blocks, uint32_t spin_ns, cudaStream_t st) {
+  calibrate_kernel<<<blocks, 64, 0, st>>>(out, spin_ns);
+  return cudaGetLastError();
+}
+
+}  // namespace slate

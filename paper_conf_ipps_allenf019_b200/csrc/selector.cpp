@@ -1,0 +1,96 @@
+// selector.cpp -- workload classification, the Tab I policy, the selection
+// algorithm and the SM split (§III-B; readings Q8-Q10, Q13 in
+// DESIGN.md).  Pure host functions, exported through the C ABI so they can be
+// checked against the oracle without a GPU.
+#include <cmath>
+#include <cstdint>
+#include <limits>
+#include <vector>
+
+#include "../../include/slate.h"
+
+namespace {
+
+// Tab I exactly as printed; row = active kernel, column = candidate;
+// order L_C, M_C, H_C, M_M, H_M; 1 = corun, 0 = solo.
+const int kLiteral[5][5] = {
+    {1, 1, 0, 1, 1},
+    {1, 1, 0, 0, 1},
+    {0, 0, 0, 0, 1},
+    {1, 0, 1, 0, 0},
+    {1, 1, 0, 0, 0},
+};
+
+int level(double frac, double lo, double hi) { return frac < lo ? 0 : (frac < hi ? 1 : 2); }
+
+// solo time on s SMs, linear in throughput between samples, 0 throughput at 0 SMs
+double interp(const uint32_t* sms, const double* ms, uint32_t n, double s) {
+  if (n == 0) return std::numeric_limits<double>::infinity();
+  if (s >= sms[n - 1]) return ms[n - 1];
+  double s0 = 0, r0 = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    const double s1 = sms[i], r1 = 1.0 / ms[i];
+    if (s <= s1) {
+      const double r = r0 + (r1 - r0) * (s - s0) / (s1 - s0);
+      return r <= 0 ? std::numeric_limits<double>::infinity() : 1.0 / r;
+    }
+    s0 = s1;
+    r0 = r1;
+  }
+  return ms[n - 1];
+}
+
+}  // namespace
+
+extern "C" {
+
+uint32_t slate_classify(double hbm_frac, double fp32_frac, double tc_frac, uint32_t* c_level, uint32_t* m_level) {
+  // Q9: memory L < 25% <= M < 85% <= H; compute (max of FP32, tensor) L < 1% <= M < 10% <= H
+  const int m = level(hbm_frac, 0.25, 0.85);
+  const int c = level(fp32_frac > tc_frac ? fp32_frac : tc_frac, 0.01, 0.10);
+  if (c_level) *c_level = uint32_t(c);
+  if (m_level) *m_level = uint32_t(m);
+  // memory intensity has priority: H_M, M_M, else L_C/M_C/H_C by compute
+  if (m == 2) return 4;
+  if (m == 1) return 3;
+  return uint32_t(c);
+}
+
+int slate_policy(uint32_t a, uint32_t b, int literal) {
+  if (a > 4 || b > 4) return 0;
+  if (literal) return kLiteral[a][b];
+  // Q8: symmetric table, the upper triangle (holding the H_C row) authoritative
+  return a <= b ? kLiteral[a][b] : kLiteral[b][a];
+}
+
+int slate_select(uint32_t active, const uint32_t* cats, const uint32_t* bypassed, uint32_t n, uint32_t max_bypass,
+                 int literal) {
+  // test J_{k+1} first, then the rest of the queue; -1 = run J_k solo
+  for (uint32_t i = 0; i < n; ++i) {
+    if (slate_policy(active, cats[i], literal)) return int(i);
+    if (bypassed && bypassed[i] >= max_bypass) return -1;   // Q13: no look-ahead past a starving kernel
+  }
+  return -1;
+}
+
+uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, const uint32_t* sms_b,
+                            const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t step, double* makespan_ms) {
+  if (step == 0) step = 1;
+  double best_t = std::numeric_limits<double>::infinity();
+  uint32_t best_s = n_sms / 2;
+  const double ta_full = interp(sms_a, ms_a, n_a, n_sms), tb_full = interp(sms_b, ms_b, n_b, n_sms);
+  for (uint32_t s = step; s + step <= n_sms; s += step) {
+    const double ta = interp(sms_a, ms_a, n_a, double(n_sms - s));
+    const double tb = interp(sms_b, ms_b, n_b, double(s));
+    // fluid model: the first to finish hands its SMs to the other
+    const double t = tb <= ta ? tb + (1.0 - tb / ta) * ta_full : ta + (1.0 - ta / tb) * tb_full;
+    if (t < best_t - 1e-12) {
+      best_t = t;
+      best_s = s;
+    }
+  }
+  if (makespan_ms) *makespan_ms = best_t;
+  return best_s;
+}
+
+}  // extern "C"

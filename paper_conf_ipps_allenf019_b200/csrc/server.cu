@@ -1,0 +1,983 @@
+// server.cu -- the single-context Slate server (see server.h).
+//
+// Paper map: context funnelling and sessions (§IV-A), the profiler
+// and profile table, the scheduler triggered by arrival and
+// completion of kernels, selection (Tab I), dynamic resizing
+// (P:L123-127).  B200 design in DESIGN.md §Runtime.
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <sstream>
+
+#include <cuda.h>
+#include "server.h"
+
+namespace slate {
+
+typedef CUresult (*WriteValue64Fn)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+
+#define CK(call)                                                                   \
+  do {                                                                             \
+    cudaError_t e_ = (call);                                                       \
+    if (e_ != cudaSuccess) {                                                       \
+      if (err) *err = std::string(#call) + ": " + cudaGetErrorString(e_);          \
+      return SLATE_ECUDA;                                                          \
+    }                                                                              \
+  } while (0)
+
+static double env_double(const char* name, double dflt) {
+  const char* v = std::getenv(name);
+  return v && *v ? std::atof(v) : dflt;
+}
+
+static uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+Server::Server(int device) : device_(device) {}
+
+Server::~Server() {
+  {
+    std::lock_guard<std::mutex> g(mu_);
+    stop_ = true;
+  }
+  cv_.notify_all();
+  if (poller_.joinable()) poller_.join();
+}
+
+double Server::now_us() const {
+  return std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+int Server::init(std::string* err) {
+  CK(cudaSetDevice(device_));
+  CK(cudaFree(nullptr));
+  cudaDeviceProp prop;
+  CK(cudaGetDeviceProperties(&prop, device_));
+  if (prop.major < 10) {
+    if (err) *err = "libslate is built for sm_100a (B200); device is sm_" + std::to_string(prop.major * 10 + prop.minor);
+    return SLATE_ECUDA;
+  }
+  cudaDriverEntryPointQueryResult q;
+  CK(cudaGetDriverEntryPoint("cuStreamWriteValue64", &write_value64_, cudaEnableDefault, &q));
+  if (!write_value64_) {
+    if (err) *err = "cuStreamWriteValue64 not available";
+    return SLATE_ECUDA;
+  }
+  int lo_prio, hi_prio;
+  CK(cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio));
+  CK(cudaStreamCreateWithPriority(&ctrl_stream_, cudaStreamNonBlocking, hi_prio));
+  CK(cudaStreamCreateWithPriority(&copy_stream_, cudaStreamNonBlocking, hi_prio));
+  CK(cudaEventCreate(&epoch_ev_));
+  CK(cudaEventRecord(epoch_ev_, copy_stream_));
+
+  // ---- SM calibration (K13): %smid is a virtual id on sm_100a; rank = order in the sorted set
+  {
+    const uint32_t blocks = 32u * uint32_t(prop.multiProcessorCount);
+    uint32_t* d_ids = nullptr;
+    CK(cudaMalloc(&d_ids, blocks * 4));
+    if (launch_calibrate(d_ids, blocks, 20000, copy_stream_) != cudaSuccess) {
+      if (err) *err = "calibration launch failed";
+      return SLATE_ECUDA;
+    }
+    std::vector<uint32_t> ids(blocks);
+    CK(cudaMemcpyAsync(ids.data(), d_ids, blocks * 4, cudaMemcpyDeviceToHost, copy_stream_));
+    CK(cudaStreamSynchronize(copy_stream_));
+    CK(cudaFree(d_ids));
+    std::sort(ids.begin(), ids.end());
+    ids.erase(std::unique(ids.begin(), ids.end()), ids.end());
+    if (ids.empty() || ids.back() >= 1024 || ids.size() > size_t(kMaxRanks)) {
+      if (err) *err = "SM calibration out of bounds";
+      return SLATE_ECUDA;
+    }
+    n_sms_ = int(ids.size());
+    max_smid_ = ids.back();
+    std::vector<uint16_t> lut(1024, uint16_t(n_sms_ - 1));   // unseen ids: clamp (never expected)
+    for (size_t r = 0; r < ids.size(); ++r) lut[ids[r]] = uint16_t(r);
+    CK(cudaMalloc(&d_rank_of_, 1024 * sizeof(uint16_t)));
+    CK(cudaMemcpy(d_rank_of_, lut.data(), 1024 * sizeof(uint16_t), cudaMemcpyHostToDevice));
+  }
+  // ---- pools
+  CK(cudaMalloc(&d_tc_, sizeof(TaskCtl) * kSlots));
+  CK(cudaMemset(d_tc_, 0, sizeof(TaskCtl) * kSlots));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&h_mirror_), sizeof(HostMirror) * kSlots, cudaHostAllocMapped));
+  std::memset(reinterpret_cast<void*>(h_mirror_), 0, sizeof(HostMirror) * kSlots);
+  CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&d_mirror_), h_mirror_, 0));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&h_snap_), kTaskCtlHeader * kSlots, cudaHostAllocDefault));
+  CK(cudaHostAlloc(&h_zero_, sizeof(TaskCtl), cudaHostAllocDefault));
+  std::memset(h_zero_, 0, sizeof(TaskCtl));
+  for (int i = kSlots - 1; i >= 0; --i) free_slots_.push_back(i);
+  slot_zeroed_.assign(kSlots, nullptr);
+  CK(cudaMalloc(&d_ctrl_pool_, 128 * kQueues));
+  CK(cudaMemset(d_ctrl_pool_, 0, 128 * kQueues));
+  for (int i = kQueues - 1; i >= 0; --i) free_ctrl_.push_back(i);
+
+  peak_hbm_ = env_double("SLATE_PEAK_HBM_GBPS", 6650.0);
+  peak_fp32_ = env_double("SLATE_PEAK_FP32_GFLOPS", 2.0 * 128 * prop.multiProcessorCount * (prop.clockRate / 1e6));
+  peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
+  standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
+  poller_ = std::thread([this] { poller_main(); });
+  return SLATE_OK;
+}
+
+slate_info Server::info() const {
+  slate_info i{};
+  i.abi_version = SLATE_ABI_VERSION;
+  i.num_sms = uint32_t(n_sms_);
+  i.max_smid = max_smid_;
+  i.device = uint32_t(device_);
+  i.peak_hbm_gbps = peak_hbm_;
+  i.peak_fp32_gflops = peak_fp32_;
+  i.peak_tc_tflops = peak_tc_;
+  return i;
+}
+
+// ------------------------------------------------------------------ queues
+uint32_t Server::open_queue() {
+  std::lock_guard<std::mutex> g(mu_);
+  if (free_ctrl_.empty()) return 0;
+  auto Q = std::make_unique<Queue>();
+  Q->id = next_queue_id_++;
+  const int slot = free_ctrl_.back();
+  free_ctrl_.pop_back();
+  Q->d_ctrl = d_ctrl_pool_ + slot * 16;
+  Q->lo = 0;
+  Q->hi = uint32_t(n_sms_ - 1);
+  cudaStreamCreateWithFlags(&Q->stream, cudaStreamNonBlocking);
+  cudaStreamCreateWithFlags(&Q->aux, cudaStreamNonBlocking);
+  const uint32_t id = Q->id;
+  queues_[id] = std::move(Q);
+  return id;
+}
+
+int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
+  const int rc = sync(q, 0, timeout_us, err);
+  std::lock_guard<std::mutex> g(mu_);
+  auto it = queues_.find(q);
+  if (it == queues_.end()) return SLATE_ENOTFOUND;
+  Queue& Q = *it->second;
+  Q.closed = true;
+  if (rc == SLATE_OK) {
+    cudaStreamSynchronize(Q.stream);
+    cudaStreamSynchronize(Q.aux);
+    const int slot = int((Q.d_ctrl - d_ctrl_pool_) / 16);
+    free_ctrl_.push_back(slot);
+    cudaStreamDestroy(Q.stream);
+    cudaStreamDestroy(Q.aux);
+    queues_.erase(it);
+  }
+  return rc;
+}
+
+// ------------------------------------------------------------------ kernels
+int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err) {
+  if (!d || !out || d->abi_version != SLATE_ABI_VERSION) {
+    if (err) *err = "bad kernel descriptor";
+    return SLATE_EINVAL;
+  }
+  if (d->kind == 0 || d->kind >= SLATE_KIND_MAX_ || (d->flags & ~SLATE_KFLAG_COVERAGE)) {
+    if (err) *err = "bad kind or flags";
+    return SLATE_EINVAL;
+  }
+  const KindOps* ops = kind_ops(d->kind);
+  if (!ops) {
+    if (err) *err = "kind not built into this library";
+    return SLATE_EUNSUPPORTED;
+  }
+  std::lock_guard<std::mutex> g(mu_);
+  const uint32_t iters = d->iters ? d->iters : ops->default_iters;   // 0 = auto per launch
+  for (auto& kv : kernels_) {
+    const KernelEntry& k = *kv.second;
+    if (k.desc.kind == d->kind && k.desc.iters == iters && k.desc.flags == d->flags) {
+      *out = k.id;
+      return SLATE_OK;
+    }
+  }
+  auto k = std::make_unique<KernelEntry>();
+  k->id = next_kernel_id_++;
+  k->desc = *d;
+  k->desc.iters = iters;
+  k->ops = ops;
+  if (ops->smem > 48 * 1024) {
+    CK(cudaFuncSetAttribute(ops->worker_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem));
+    CK(cudaFuncSetAttribute(ops->standalone_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem));
+  }
+  int occ = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ops->worker_fn, ops->threads, ops->smem));
+  if (occ < 1) {
+    if (err) *err = "worker does not fit on an SM";
+    return SLATE_ECUDA;
+  }
+  k->occ = occ;
+  *out = k->id;
+  kernels_[k->id] = std::move(k);
+  return SLATE_OK;
+}
+
+bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const {
+  auto fail = [&](const char* m) {
+    if (err) *err = m;
+    return false;
+  };
+  if (!d || !d->args || d->args_size != k.ops->args_size) return fail("args missing or args_size mismatch");
+  uint64_t g[3] = {0, 1, 1};
+  auto al = [](uint64_t p) { return (p & 15) == 0; };
+  switch (k.desc.kind) {
+    case SLATE_KIND_TRIAD: {
+      auto a = static_cast<const slate_args_triad*>(d->args);
+      if (!al(a->a) || !al(a->b) || !al(a->c)) return fail("triad arrays must be 16-byte aligned");
+      g[0] = cdiv(a->n, 1024);
+      break;
+    }
+    case SLATE_KIND_COPY: {
+      auto a = static_cast<const slate_args_copy*>(d->args);
+      if (!al(a->a) || !al(a->b)) return fail("copy arrays must be 16-byte aligned");
+      g[0] = cdiv(a->n, 4096);
+      break;
+    }
+    case SLATE_KIND_SGEMM_NAIVE: {
+      auto a = static_cast<const slate_args_sgemm*>(d->args);
+      g[0] = cdiv(a->n, 16);
+      g[1] = cdiv(a->m, 16);
+      if (a->k == 0) return fail("k == 0");
+      break;
+    }
+    case SLATE_KIND_SPMV_CSR: {
+      auto a = static_cast<const slate_args_spmv*>(d->args);
+      g[0] = cdiv(a->n_rows, 32);
+      break;
+    }
+    case SLATE_KIND_BLACKSCHOLES: {
+      auto a = static_cast<const slate_args_bs*>(d->args);
+      if (!al(a->S) || !al(a->X) || !al(a->T) || !al(a->call) || !al(a->put)) return fail("bs arrays must be 16-byte aligned");
+      if (a->n_scen == 0) return fail("n_scen == 0");
+      g[0] = cdiv(a->n, 1024);
+      break;
+    }
+    case SLATE_KIND_STENCIL2D: {
+      auto a = static_cast<const slate_args_stencil*>(d->args);
+      g[0] = cdiv(a->w, 32);
+      g[1] = cdiv(a->h, 8);
+      break;
+    }
+    case SLATE_KIND_GEMM_BF16: {
+      auto a = static_cast<const slate_args_gemm*>(d->args);
+      if (a->m % 128 || a->n % 128 || a->k % 64 || a->k == 0) return fail("gemm_bf16 needs m, n % 128 == 0 and k % 64 == 0");
+      if (!al(a->A) || !al(a->B) || !al(a->C)) return fail("gemm arrays must be 16-byte aligned");
+      g[0] = a->n / 128;
+      g[1] = a->m / 128;
+      break;
+    }
+    default:
+      return fail("unknown kind");
+  }
+  if (d->grid[0] != g[0] || d->grid[1] != g[1] || d->grid[2] != g[2]) return fail("grid does not match the kind's args");
+  const uint64_t total = g[0] * g[1] * g[2];
+  if (total == 0) return fail("empty grid");
+  if (total >= (1ull << 31)) return fail("grid too large (B >= 2^31)");
+  *B = uint32_t(total);
+  return true;
+}
+
+// algorithmic work per launch: bytes moved, fp32 flops, tensor-core flops
+void Server::work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const {
+  *bytes = *fp32 = *tc = 0;
+  switch (k.desc.kind) {
+    case SLATE_KIND_TRIAD: {
+      auto a = static_cast<const slate_args_triad*>(d->args);
+      *bytes = 12.0 * a->n;
+      *fp32 = 2.0 * a->n;
+      break;
+    }
+    case SLATE_KIND_COPY: {
+      auto a = static_cast<const slate_args_copy*>(d->args);
+      *bytes = 8.0 * a->n;
+      break;
+    }
+    case SLATE_KIND_SGEMM_NAIVE: {
+      auto a = static_cast<const slate_args_sgemm*>(d->args);
+      *bytes = 4.0 * (double(a->m) * a->k + double(a->k) * a->n + double(a->m) * a->n);
+      *fp32 = 2.0 * a->m * double(a->n) * a->k;
+      break;
+    }
+    case SLATE_KIND_SPMV_CSR: {
+      auto a = static_cast<const slate_args_spmv*>(d->args);
+      int nnz = 0;
+      cudaMemcpy(&nnz, reinterpret_cast<const int*>(a->rowptr) + a->n_rows, 4, cudaMemcpyDeviceToHost);
+      *bytes = 8.0 * nnz + 4.0 * (a->n_rows + 1) + 4.0 * a->n_rows + 4.0 * a->n_cols;
+      *fp32 = 2.0 * nnz;
+      break;
+    }
+    case SLATE_KIND_BLACKSCHOLES: {
+      auto a = static_cast<const slate_args_bs*>(d->args);
+      *bytes = 20.0 * a->n + 4.0 * a->n_scen;
+      *fp32 = 36.0 * a->n * a->n_scen;   // 36 flops per option-scenario
+      break;
+    }
+    case SLATE_KIND_STENCIL2D: {
+      auto a = static_cast<const slate_args_stencil*>(d->args);
+      *bytes = 8.0 * a->h * double(a->w);
+      *fp32 = 4.0 * a->h * double(a->w);
+      break;
+    }
+    case SLATE_KIND_GEMM_BF16: {
+      auto a = static_cast<const slate_args_gemm*>(d->args);
+      *bytes = 2.0 * (double(a->m) * a->k + double(a->n) * a->k) + 4.0 * double(a->m) * a->n;
+      *tc = 2.0 * a->m * double(a->n) * a->k;
+      break;
+    }
+  }
+}
+
+int Server::alloc_slot() {
+  if (free_slots_.empty()) return -1;
+  const int s = free_slots_.back();
+  free_slots_.pop_back();
+  return s;
+}
+
+// a freed control block is zeroed by DMA on the copy stream right away, so the
+// next launch that takes the slot only waits on an (already complete) event
+void Server::free_slot(int slot) {
+  cudaMemcpyAsync(d_tc_ + slot, h_zero_, sizeof(TaskCtl), cudaMemcpyHostToDevice, copy_stream_);
+  if (!slot_zeroed_[slot]) cudaEventCreateWithFlags(&slot_zeroed_[slot], cudaEventDisableTiming);
+  cudaEventRecord(slot_zeroed_[slot], copy_stream_);
+  free_slots_.push_back(slot);
+}
+
+// reading Q11: the paper's default task of 10 blocks, reduced so every
+// worker gets at least ~4 tasks (a fixed 10 mis-fits small grids)
+uint32_t Server::auto_iters(uint32_t B, int occ) const {
+  const uint64_t workers = uint64_t(occ) * uint64_t(n_sms_);
+  const uint64_t it = B / (4 * workers);
+  return uint32_t(it < 1 ? 1 : (it > 10 ? 10 : it));
+}
+
+// ------------------------------------------------------------------ control word
+int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* err) {
+  Q.epoch += 1;
+  Q.lo = lo;
+  Q.hi = hi;
+  const uint64_t v = pack_ctrl(Q.epoch, lo, hi);
+  // a stream memory write needs no SM: it lands even while persistent workers fill every SM
+  const CUresult r = reinterpret_cast<WriteValue64Fn>(write_value64_)(
+      reinterpret_cast<CUstream>(ctrl_stream_), reinterpret_cast<CUdeviceptr>(Q.d_ctrl), v, 0);
+  if (r != CUDA_SUCCESS) {
+    if (err) *err = "cuStreamWriteValue64 failed: " + std::to_string(int(r));
+    return SLATE_ECUDA;
+  }
+  // later launches of this queue start after the write
+  cudaEvent_t ev;
+  CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  CK(cudaEventRecord(ev, ctrl_stream_));
+  CK(cudaStreamWaitEvent(Q.stream, ev, 0));
+  CK(cudaStreamWaitEvent(Q.aux, ev, 0));
+  cudaEventDestroy(ev);
+  return SLATE_OK;
+}
+
+// ------------------------------------------------------------------ issue
+int Server::issue(Launch& L, Queue& Q, std::string* err) {
+  const KindOps* ops = L.k->ops;
+  if (Q.last_topup_end) {   // stream semantics: the predecessor's top-up workers must finish first
+    CK(cudaStreamWaitEvent(Q.stream, Q.last_topup_end, 0));
+  }
+  CK(cudaEventCreate(&L.ev_start));
+  cudaEvent_t ev_end;
+  CK(cudaEventCreate(&ev_end));
+  const auto& g = L.desc.grid;
+  if (L.desc.mode == SLATE_MODE_STANDALONE) {
+    CK(cudaEventRecord(L.ev_start, Q.stream));
+    CK(ops->launch_standalone(L.args.data(), dim3(g[0], g[1], g[2]), Q.stream));
+    CK(cudaEventRecord(ev_end, Q.stream));
+    L.ev_end.push_back(ev_end);
+    L.ev_done.push_back(ev_end);
+  } else {
+    const int slot = alloc_slot();
+    if (slot < 0) {
+      if (err) *err = "control-block pool exhausted";
+      return SLATE_ENOMEM;
+    }
+    L.slot = slot;
+    std::memset(reinterpret_cast<void*>(h_mirror_ + slot), 0, sizeof(HostMirror));
+    // the control block was zeroed by DMA when it was freed (no SM needed)
+    if (slot_zeroed_[slot]) CK(cudaStreamWaitEvent(Q.stream, slot_zeroed_[slot], 0));
+    CK(cudaEventRecord(L.ev_start, Q.stream));
+    WorkerCommon w{};
+    w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = L.B; w.iters = L.iters; w.occ = uint32_t(L.k->occ);
+    w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
+    w.standby_timeout_ns = standby_timeout_ns_;
+    w.ctrl = Q.d_ctrl; w.tc = d_tc_ + slot; w.mirror = d_mirror_ + slot;
+    w.cov = reinterpret_cast<uint32_t*>(L.desc.coverage);
+    w.rank_of = d_rank_of_;
+    CK(ops->launch_worker(w, L.args.data(), uint32_t(L.k->occ) * uint32_t(n_sms_), Q.stream));
+    CK(cudaEventRecord(ev_end, Q.stream));
+    L.ev_end.push_back(ev_end);
+    cudaEvent_t ev_snap;
+    CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
+    CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+    CK(cudaMemcpyAsync(h_snap_ + size_t(slot) * kTaskCtlHeader, d_tc_ + slot, kTaskCtlHeader, cudaMemcpyDeviceToHost,
+                       copy_stream_));
+    CK(cudaEventRecord(ev_snap, copy_stream_));
+    L.ev_done.push_back(ev_snap);
+  }
+  L.state = 1;
+  Q.issued.push_back(L.id);
+  cv_.notify_all();
+  return SLATE_OK;
+}
+
+// grow: workers for the ranks newly in range of the queue's running launch.
+// Only the LAST issued launch of the queue gets a top-up (a launch already
+// queued behind it on the stream picks up the new range by itself); later
+// launches wait for the top-up's end (stream semantics).
+int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
+  if (Q.issued.size() != 1 || !Q.pending.empty()) return SLATE_OK;
+  Launch& R = *launches_[Q.issued.front()];
+  if (R.state != 1 || R.slot < 0 || R.desc.mode == SLATE_MODE_STANDALONE) return SLATE_OK;
+  if (h_mirror_[R.slot].complete) return SLATE_OK;
+  const auto& g = R.desc.grid;
+  CK(cudaStreamWaitEvent(Q.aux, R.ev_start, 0));
+  WorkerCommon w{};
+  w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = R.B; w.iters = R.iters; w.occ = uint32_t(R.k->occ);
+  w.bound_lo = Q.lo; w.bound_hi = Q.hi; w.n_ranks = uint32_t(n_sms_);
+  w.standby_timeout_ns = standby_timeout_ns_;
+  w.ctrl = Q.d_ctrl; w.tc = d_tc_ + R.slot; w.mirror = d_mirror_ + R.slot;
+  w.cov = reinterpret_cast<uint32_t*>(R.desc.coverage);
+  w.rank_of = d_rank_of_;
+  CK(R.k->ops->launch_worker(w, R.args.data(), uint32_t(R.k->occ) * uint32_t(n_sms_), Q.aux));
+  cudaEvent_t ev_end, ev_snap;
+  CK(cudaEventCreate(&ev_end));
+  CK(cudaEventRecord(ev_end, Q.aux));
+  R.ev_end.push_back(ev_end);
+  CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
+  CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+  CK(cudaMemcpyAsync(h_snap_ + size_t(R.slot) * kTaskCtlHeader, d_tc_ + R.slot, kTaskCtlHeader,
+                     cudaMemcpyDeviceToHost, copy_stream_));
+  CK(cudaEventRecord(ev_snap, copy_stream_));
+  R.ev_done.push_back(ev_snap);
+  Q.last_topup_end = ev_end;
+  R.n_topups += 1;
+  return SLATE_OK;
+}
+
+// ------------------------------------------------------------------ launch
+int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_t* out, std::string* err) {
+  std::unique_lock<std::mutex> g(mu_);
+  auto qi = queues_.find(q);
+  if (qi == queues_.end()) return SLATE_ENOTFOUND;
+  auto ki = kernels_.find(kid);
+  if (ki == kernels_.end()) {
+    if (err) *err = "unknown kernel";
+    return SLATE_ENOTFOUND;
+  }
+  const KernelEntry& k = *ki->second;
+  uint32_t B = 0;
+  if (!validate(k, d, &B, err)) return SLATE_EINVAL;
+  if (d->placement > SLATE_PLACE_CORUN || d->mode > SLATE_MODE_STANDALONE) {
+    if (err) *err = "bad placement or mode";
+    return SLATE_EINVAL;
+  }
+  if (d->placement == SLATE_PLACE_CORUN && (d->sm_lo > d->sm_hi || d->sm_hi >= uint32_t(n_sms_))) {
+    if (err) *err = "bad SM range";
+    return SLATE_EINVAL;
+  }
+  if (d->coverage && !(k.desc.flags & SLATE_KFLAG_COVERAGE)) {
+    if (err) *err = "coverage log given but the kernel was not registered with SLATE_KFLAG_COVERAGE";
+    return SLATE_EINVAL;
+  }
+  auto L = std::make_unique<Launch>();
+  L->id = next_launch_id_++;
+  L->queue = q;
+  L->k = &k;
+  L->desc = *d;
+  L->args.assign(static_cast<const unsigned char*>(d->args), static_cast<const unsigned char*>(d->args) + d->args_size);
+  L->desc.args = nullptr;
+  L->B = B;
+  L->iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ);
+  Launch& LL = *L;
+  launches_[L->id] = std::move(L);
+  *out = LL.id;
+  Queue& Q = *qi->second;
+  int rc = SLATE_OK;
+  if (d->mode == SLATE_MODE_STANDALONE) {
+    rc = issue(LL, Q, err);
+  } else if (d->placement == SLATE_PLACE_CORUN) {
+    const uint32_t old_lo = Q.lo, old_hi = Q.hi;
+    if (!Q.active) {
+      Q.active = true;
+      active_.push_back(Q.id);
+      rc = write_ctrl(Q, d->sm_lo, d->sm_hi, false, err);
+    } else if (Q.lo != d->sm_lo || Q.hi != d->sm_hi) {
+      rc = write_ctrl(Q, d->sm_lo, d->sm_hi, true, err);
+      if (rc == SLATE_OK && (d->sm_lo < old_lo || d->sm_hi > old_hi)) rc = grow_running(Q, old_lo, old_hi, err);
+    }
+    Q.explicit_range = true;
+    if (rc == SLATE_OK) rc = issue(LL, Q, err);
+  } else if (Q.active) {
+    rc = issue(LL, Q, err);
+  } else {
+    Q.pending.push_back(LL.id);
+    if (std::find(waiting_.begin(), waiting_.end(), Q.id) == waiting_.end()) waiting_.push_back(Q.id);
+    schedule();
+  }
+  return rc;
+}
+
+// ------------------------------------------------------------------ scheduler
+std::string Server::profile_key(const KernelEntry& k, const slate_launch_desc* d) const {
+  std::ostringstream s;
+  s << k.desc.kind << ':' << k.desc.iters << ':';
+  const void* a = d->args;
+  switch (k.desc.kind) {
+    case SLATE_KIND_TRIAD: s << static_cast<const slate_args_triad*>(a)->n; break;
+    case SLATE_KIND_COPY: s << static_cast<const slate_args_copy*>(a)->n; break;
+    case SLATE_KIND_SGEMM_NAIVE: { auto x = static_cast<const slate_args_sgemm*>(a); s << x->m << 'x' << x->n << 'x' << x->k; break; }
+    case SLATE_KIND_SPMV_CSR: { auto x = static_cast<const slate_args_spmv*>(a); s << x->n_rows << 'x' << x->n_cols; break; }
+    case SLATE_KIND_BLACKSCHOLES: { auto x = static_cast<const slate_args_bs*>(a); s << x->n << 'p' << x->n_scen; break; }
+    case SLATE_KIND_STENCIL2D: { auto x = static_cast<const slate_args_stencil*>(a); s << x->h << 'x' << x->w; break; }
+    case SLATE_KIND_GEMM_BF16: { auto x = static_cast<const slate_args_gemm*>(a); s << x->m << 'x' << x->n << 'x' << x->k; break; }
+  }
+  return s.str();
+}
+
+int Server::category_of(const Launch& L) const {
+  slate_launch_desc d = L.desc;
+  d.args = L.args.data();
+  auto it = profiles_.find(profile_key(*L.k, &d));
+  return it == profiles_.end() ? -1 : int(it->second.p.category);
+}
+
+static const slate_profile_t* find_profile(const std::map<std::string, ProfileEntry>& t, const std::string& key) {
+  auto it = t.find(key);
+  return it == t.end() ? nullptr : &it->second.p;
+}
+
+void Server::schedule() {
+  std::string err;
+  while (!waiting_.empty() && !profiling_) {
+    if (active_.empty()) {
+      const uint32_t qid = waiting_.front();
+      waiting_.pop_front();
+      bypassed_.erase(qid);
+      Queue& Q = *queues_[qid];
+      Q.active = true;
+      Q.explicit_range = false;
+      active_.push_back(qid);
+      write_ctrl(Q, 0, uint32_t(n_sms_ - 1), false, &err);
+      while (!Q.pending.empty()) {
+        Launch& L = *launches_[Q.pending.front()];
+        Q.pending.pop_front();
+        issue(L, Q, &err);
+      }
+      continue;
+    }
+    if (active_.size() >= 2) break;
+    Queue& A = *queues_[active_[0]];
+    if (A.explicit_range) break;
+    // the active kernel: the last launch issued on A (or pending on it)
+    const Launch* LA = nullptr;
+    if (!A.issued.empty()) LA = launches_[A.issued.back()].get();
+    if (!LA || LA->desc.placement == SLATE_PLACE_SOLO) break;
+    const int catA = category_of(*LA);
+    if (catA < 0) break;
+    std::vector<uint32_t> cats, byp;
+    std::vector<uint32_t> qids;
+    for (uint32_t qid : waiting_) {
+      const Queue& W = *queues_[qid];
+      const Launch& H = *launches_[W.pending.front()];
+      const int c = (H.desc.placement == SLATE_PLACE_SOLO) ? -1 : category_of(H);
+      cats.push_back(c < 0 ? 99u : uint32_t(c));   // unknown profile or SOLO: never complementary
+      byp.push_back(bypassed_[qid]);
+      qids.push_back(qid);
+    }
+    const int idx = slate_select(uint32_t(catA), cats.data(), byp.data(), uint32_t(cats.size()), 4, 0);
+    if (idx < 0) break;
+    for (int i = 0; i < idx; ++i) bypassed_[qids[i]] += 1;
+    Queue& Bq = *queues_[qids[idx]];
+    const Launch& HB = *launches_[Bq.pending.front()];
+    // split from the profile curves (reading Q10), else half
+    uint32_t s = uint32_t(n_sms_ / 2);
+    {
+      slate_launch_desc da = LA->desc, db = HB.desc;
+      da.args = LA->args.data();
+      db.args = HB.args.data();
+      const slate_profile_t* pa = find_profile(profiles_, profile_key(*LA->k, &da));
+      const slate_profile_t* pb = find_profile(profiles_, profile_key(*HB.k, &db));
+      if (pa && pb && pa->n_curve >= 2 && pb->n_curve >= 2) {
+        std::vector<uint32_t> sa, sb;
+        std::vector<double> ta, tb;
+        for (int i = int(pa->n_curve) - 1; i >= 0; --i) { sa.push_back(pa->curve_sms[i]); ta.push_back(pa->curve_ms[i]); }
+        for (int i = int(pb->n_curve) - 1; i >= 0; --i) { sb.push_back(pb->curve_sms[i]); tb.push_back(pb->curve_ms[i]); }
+        // curves are stored in descending SM order; interp wants ascending
+        s = slate_choose_split(sa.data(), ta.data(), uint32_t(sa.size()), sb.data(), tb.data(), uint32_t(sb.size()),
+                               uint32_t(n_sms_), 2, nullptr);
+      }
+    }
+    const uint32_t old_lo = A.lo, old_hi = A.hi;
+    const double t0 = now_us();
+    write_ctrl(A, 0, uint32_t(n_sms_) - s - 1, true, &err);   // shrink the running kernel
+    if (!A.issued.empty()) {
+      Launch& R = *launches_[A.issued.front()];
+      if (R.resize_us.size() < 16) {
+        R.pending_resize.push_back({A.epoch, 1, t0, int(R.resize_us.size())});
+        R.resize_us.push_back(-1);
+      }
+      R.n_resizes += 1;
+    }
+    (void)old_lo;
+    (void)old_hi;
+    waiting_.erase(std::find(waiting_.begin(), waiting_.end(), Bq.id));
+    bypassed_.erase(Bq.id);
+    Bq.active = true;
+    Bq.explicit_range = false;
+    active_.push_back(Bq.id);
+    write_ctrl(Bq, uint32_t(n_sms_) - s, uint32_t(n_sms_ - 1), false, &err);
+    while (!Bq.pending.empty()) {
+      Launch& L = *launches_[Bq.pending.front()];
+      Bq.pending.pop_front();
+      issue(L, Bq, &err);
+    }
+    break;   // at most two co-runners (reading Q13)
+  }
+}
+
+// the queue has nothing left: its SMs go to the co-runner
+void Server::release(Queue& Q) {
+  std::string err;
+  Q.active = false;
+  Q.explicit_range = false;
+  active_.erase(std::remove(active_.begin(), active_.end(), Q.id), active_.end());
+  if (active_.size() == 1) {
+    Queue& A = *queues_[active_[0]];
+    if (!A.explicit_range && (A.lo != 0 || A.hi != uint32_t(n_sms_ - 1))) {
+      const uint32_t old_lo = A.lo, old_hi = A.hi;
+      const double t0 = now_us();
+      write_ctrl(A, 0, uint32_t(n_sms_ - 1), true, &err);
+      if (!A.issued.empty()) {
+        Launch& R = *launches_[A.issued.front()];
+        if (R.resize_us.size() < 16) {
+          R.pending_resize.push_back({A.epoch, 2, t0, int(R.resize_us.size())});
+          R.resize_us.push_back(-1);
+        }
+        R.n_resizes += 1;
+      }
+      grow_running(A, old_lo, old_hi, &err);
+    }
+  }
+  schedule();
+}
+
+int Server::resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string* err) {
+  if (lo > hi || hi >= uint32_t(n_sms_)) {
+    if (err) *err = "bad SM range";
+    return SLATE_EINVAL;
+  }
+  std::lock_guard<std::mutex> g(mu_);
+  auto li = launches_.find(l);
+  if (li == launches_.end() || li->second->queue != q) return SLATE_ENOTFOUND;
+  Queue& Q = *queues_[q];
+  Launch& L = *li->second;
+  const uint32_t old_lo = Q.lo, old_hi = Q.hi;
+  const bool shrink = lo > old_lo || hi < old_hi;
+  const bool grow = lo < old_lo || hi > old_hi;
+  const double t0 = now_us();
+  int rc = write_ctrl(Q, lo, hi, true, err);
+  if (rc != SLATE_OK) return rc;
+  if (!Q.active) {
+    Q.active = true;
+    active_.push_back(Q.id);
+  }
+  Q.explicit_range = true;
+  if (L.state == 2) return SLATE_DONE;
+  // measure on the queue's running launch
+  if (!Q.issued.empty()) {
+    Launch& R = *launches_[Q.issued.front()];
+    R.n_resizes += 1;
+    if (R.resize_us.size() < 16 && (shrink || grow)) {
+      R.pending_resize.push_back({Q.epoch, shrink ? 1 : 2, t0, int(R.resize_us.size())});
+      R.resize_us.push_back(-1);
+    }
+  }
+  if (grow) rc = grow_running(Q, old_lo, old_hi, err);
+  return rc;
+}
+
+// ------------------------------------------------------------------ poller
+bool Server::launch_done_events(Launch& L) {
+  for (cudaEvent_t e : L.ev_done) {
+    const cudaError_t r = cudaEventQuery(e);
+    if (r == cudaErrorNotReady) return false;
+    if (r != cudaSuccess) {   // sticky kernel error: the launch is over
+      L.error = int(r);
+      return true;
+    }
+  }
+  return true;
+}
+
+void Server::poll_once() {
+  const double t = now_us();
+  std::vector<uint32_t> idle;
+  for (auto& kv : queues_) {
+    Queue& Q = *kv.second;
+    bool first = true;
+    while (!Q.issued.empty()) {
+      Launch& L = *launches_[Q.issued.front()];
+      if (first && L.slot >= 0) {
+        const HostMirror& m = h_mirror_[L.slot];
+        for (auto it = L.pending_resize.begin(); it != L.pending_resize.end();) {
+          const bool seen = it->kind == 1 ? (m.shrink_epoch >= it->epoch) : (m.join_epoch >= it->epoch);
+          if (seen) {
+            L.resize_us[it->idx] = t - it->t0_us;
+            it = L.pending_resize.erase(it);
+          } else {
+            ++it;
+          }
+        }
+      }
+      first = false;
+      if (!launch_done_events(L)) break;
+      if (L.slot >= 0) {
+        std::memcpy(L.snapshot, h_snap_ + size_t(L.slot) * kTaskCtlHeader, kTaskCtlHeader);
+        L.has_snapshot = true;
+        free_slot(L.slot);
+        L.slot = -1;
+      }
+      L.pending_resize.clear();
+      L.state = 2;
+      Q.issued.pop_front();
+      if (Q.last_topup_end && Q.issued.empty()) Q.last_topup_end = nullptr;
+      cv_.notify_all();
+    }
+    if (Q.active && Q.issued.empty() && Q.pending.empty()) idle.push_back(Q.id);
+  }
+  for (uint32_t q : idle) release(*queues_[q]);
+}
+
+void Server::poller_main() {
+  cudaSetDevice(device_);
+  std::unique_lock<std::mutex> g(mu_);
+  while (!stop_) {
+    bool busy = false;
+    for (auto& kv : queues_)
+      if (!kv.second->issued.empty()) busy = true;
+    if (!busy) {
+      cv_.wait_for(g, std::chrono::milliseconds(2));
+      continue;
+    }
+    poll_once();
+    g.unlock();
+    std::this_thread::yield();
+    g.lock();
+  }
+}
+
+// ------------------------------------------------------------------ sync / query
+int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
+  std::unique_lock<std::mutex> g(mu_);
+  const auto deadline = std::chrono::steady_clock::now() + std::chrono::microseconds(timeout_us < 0 ? 0 : timeout_us);
+  auto done = [&]() -> bool {
+    if (l) {
+      auto it = launches_.find(l);
+      return it == launches_.end() || it->second->state == 2;
+    }
+    auto qi = queues_.find(q);
+    return qi == queues_.end() || (qi->second->issued.empty() && qi->second->pending.empty());
+  };
+  if (l && launches_.find(l) == launches_.end()) return SLATE_ENOTFOUND;
+  while (!done()) {
+    if (timeout_us < 0) {
+      cv_.wait_for(g, std::chrono::milliseconds(5));
+    } else {
+      if (std::chrono::steady_clock::now() >= deadline) {
+        if (err) *err = "slate_sync timed out";
+        return SLATE_ETIMEDOUT;
+      }
+      cv_.wait_until(g, std::min(deadline, std::chrono::steady_clock::now() + std::chrono::milliseconds(5)));
+    }
+  }
+  for (auto& kv : launches_) {
+    const Launch& L = *kv.second;
+    if ((l ? L.id == l : L.queue == q) && L.error) {
+      if (err) *err = std::string("CUDA error: ") + cudaGetErrorString(cudaError_t(L.error));
+      return SLATE_ECUDA;
+    }
+  }
+  return SLATE_OK;
+}
+
+int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
+  std::unique_lock<std::mutex> g(mu_);
+  auto it = launches_.find(l);
+  if (it == launches_.end()) return SLATE_ENOTFOUND;
+  Launch& L = *it->second;
+  std::memset(out, 0, sizeof(*out));
+  out->state = uint32_t(L.state);
+  out->total_blocks = L.B;
+  out->iters = L.iters;
+  Queue* Q = queues_.count(L.queue) ? queues_[L.queue].get() : nullptr;
+  if (Q) {
+    out->sm_lo = Q->lo;
+    out->sm_hi = Q->hi;
+    out->epoch = Q->epoch;
+  }
+  out->n_resizes = L.n_resizes;
+  out->n_topups = L.n_topups;
+  for (int i = 0; i < 16; ++i) out->resize_us[i] = i < int(L.resize_us.size()) ? L.resize_us[i] : -1.0;
+  TaskCtl tc;
+  std::memset(&tc, 0, sizeof(tc));
+  if (L.desc.mode == SLATE_MODE_STANDALONE) {
+    if (L.state == 2) { out->blocks_done = L.B; }
+  } else if (L.has_snapshot) {
+    std::memcpy(&tc, L.snapshot, kTaskCtlHeader);
+  } else if (L.slot >= 0) {
+    CK(cudaMemcpyAsync(&tc, d_tc_ + L.slot, kTaskCtlHeader, cudaMemcpyDeviceToHost, copy_stream_));
+    CK(cudaStreamSynchronize(copy_stream_));
+  }
+  if (L.desc.mode != SLATE_MODE_STANDALONE) {
+    out->blocks_done = uint32_t(tc.done);
+    out->tasks_done = uint32_t(tc.done >> 32);
+    out->next_raw = tc.next;
+    const uint64_t clamp = cdiv(L.B, L.iters) * L.iters;
+    out->next_clamped = uint32_t(std::min<uint64_t>(tc.next, clamp));
+    out->live_workers = tc.live;
+    out->workers_started = tc.started;
+    out->t_first_ns = tc.t_first;
+    out->t_last_ns = tc.t_last;
+    out->shrink_epoch = tc.shrink_epoch;
+    out->join_epoch = tc.join_epoch;
+  }
+  if (L.state == 2) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, epoch_ev_, L.ev_start) == cudaSuccess) out->start_ms = ms;
+    double end = 0;
+    for (cudaEvent_t e : L.ev_end)
+      if (cudaEventElapsedTime(&ms, epoch_ev_, e) == cudaSuccess) end = std::max(end, double(ms));
+    out->end_ms = end;
+    if (L.desc.coverage) {
+      std::vector<uint32_t> cov(L.B);
+      CK(cudaMemcpyAsync(cov.data(), reinterpret_cast<void*>(L.desc.coverage), size_t(L.B) * 4, cudaMemcpyDeviceToHost,
+                         copy_stream_));
+      CK(cudaStreamSynchronize(copy_stream_));
+      out->coverage_ok = std::all_of(cov.begin(), cov.end(), [](uint32_t v) { return v == 1; }) ? 1 : 0;
+    }
+  }
+  return SLATE_OK;
+}
+
+// ------------------------------------------------------------------ profile
+int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t lo, uint32_t hi, int reps, double* ms,
+                      std::string* err) {
+  // a private queue: its own stream and resize word; one control block slot
+  int slot;
+  uint64_t* ctrl;
+  {
+    std::lock_guard<std::mutex> g(mu_);
+    slot = alloc_slot();
+    if (slot < 0 || free_ctrl_.empty()) {
+      if (slot >= 0) free_slots_.push_back(slot);
+      if (err) *err = "pool exhausted";
+      return SLATE_ENOMEM;
+    }
+    ctrl = d_ctrl_pool_ + free_ctrl_.back() * 16;
+    free_ctrl_.pop_back();
+  }
+  cudaStream_t st;
+  CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+  const uint64_t cv = pack_ctrl(1, lo, hi);
+  CK(cudaMemcpyAsync(ctrl, &cv, 8, cudaMemcpyHostToDevice, st));
+  uint32_t B = 0;
+  validate(k, d, &B, nullptr);
+  WorkerCommon w{};
+  w.gx = d->grid[0]; w.gy = d->grid[1]; w.gz = d->grid[2]; w.B = B; w.occ = uint32_t(k.occ);
+  w.iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ);
+  w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
+  w.standby_timeout_ns = standby_timeout_ns_;
+  w.ctrl = ctrl; w.tc = d_tc_ + slot; w.mirror = nullptr; w.cov = nullptr; w.rank_of = d_rank_of_;
+  cudaEvent_t e0, e1;
+  CK(cudaEventCreate(&e0));
+  CK(cudaEventCreate(&e1));
+  std::vector<double> times;
+  for (int r = 0; r < reps + 1; ++r) {
+    CK(cudaMemcpyAsync(d_tc_ + slot, h_zero_, sizeof(TaskCtl), cudaMemcpyHostToDevice, st));
+    CK(cudaEventRecord(e0, st));
+    CK(k.ops->launch_worker(w, d->args, uint32_t(k.occ) * uint32_t(n_sms_), st));
+    CK(cudaEventRecord(e1, st));
+    CK(cudaEventSynchronize(e1));
+    float t;
+    CK(cudaEventElapsedTime(&t, e0, e1));
+    if (r > 0) times.push_back(t);   // the first run warms up
+  }
+  std::sort(times.begin(), times.end());
+  *ms = times[times.size() / 2];
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaStreamDestroy(st);
+  std::lock_guard<std::mutex> g(mu_);
+  free_slot(slot);
+  free_ctrl_.push_back(int((ctrl - d_ctrl_pool_) / 16));
+  return SLATE_OK;
+}
+
+int Server::profile(uint64_t kid, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err) {
+  const KernelEntry* kp;
+  std::string key;
+  {
+    std::unique_lock<std::mutex> g(mu_);
+    auto ki = kernels_.find(kid);
+    if (ki == kernels_.end()) return SLATE_ENOTFOUND;
+    kp = ki->second.get();
+    uint32_t B;
+    if (!validate(*kp, d, &B, err)) return SLATE_EINVAL;
+    key = profile_key(*kp, d);
+    auto pi = profiles_.find(key);
+    if (pi != profiles_.end() && !(flags & SLATE_PROF_FORCE) &&
+        (!(flags & SLATE_PROF_CURVE) || pi->second.p.n_curve > 1)) {
+      *out = pi->second.p;
+      return SLATE_OK;
+    }
+    // the profile needs the GPU to itself (P:L153 profiles are solo runs)
+    cv_.wait(g, [&] { return active_.empty() && waiting_.empty() && !profiling_; });
+    profiling_ = true;
+  }
+  slate_profile_t p{};
+  double bytes, fp32, tc;
+  work(*kp, d, &bytes, &fp32, &tc);
+  p.bytes = bytes;
+  p.flops = fp32 + tc;
+  std::vector<uint32_t> pts = {uint32_t(n_sms_)};
+  if (flags & SLATE_PROF_CURVE) {
+    for (double f : {0.75, 0.5, 1.0 / 3.0, 0.25, 0.125}) pts.push_back(std::max<uint32_t>(1, uint32_t(std::lround(n_sms_ * f))));
+  }
+  int rc = SLATE_OK;
+  for (size_t i = 0; i < pts.size() && rc == SLATE_OK; ++i) {
+    double ms = 0;
+    rc = run_timed(*kp, d, 0, pts[i] - 1, 3, &ms, err);
+    p.curve_sms[i] = pts[i];
+    p.curve_ms[i] = ms;
+    p.n_curve = uint32_t(i + 1);
+  }
+  if (rc == SLATE_OK) {
+    p.solo_ms = p.curve_ms[0];
+    const double s = p.solo_ms * 1e-3;
+    p.hbm_gbps = bytes / s / 1e9;
+    p.fp32_gflops = fp32 / s / 1e9;
+    p.tc_tflops = tc / s / 1e12;
+    p.hbm_frac = p.hbm_gbps / peak_hbm_;
+    p.fp32_frac = p.fp32_gflops / peak_fp32_;
+    p.tc_frac = p.tc_tflops / peak_tc_;
+    p.category = slate_classify(p.hbm_frac, p.fp32_frac, p.tc_frac, &p.c_level, &p.m_level);
+  }
+  std::lock_guard<std::mutex> g(mu_);
+  profiling_ = false;
+  if (rc == SLATE_OK) {
+    profiles_[key].p = p;
+    *out = p;
+  }
+  cv_.notify_all();
+  schedule();
+  return rc;
+}
+
+}  // namespace slate

@@ -1,0 +1,151 @@
+// server.h -- the single-context Slate server (§IV-A): kernel
+// registry, per-session queues with SM ranges, the workload-aware scheduler
+// (Tab I selector + split), the resize controller, the completion poller and
+// the kernel profile table.  Used in-process by libslate and by the `slated`
+// daemon; no torch types, no Python.
+#pragma once
+#include <condition_variable>
+#include <cstdint>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include <cuda_runtime.h>
+#include "kernels.h"
+
+namespace slate {
+
+struct KernelEntry {
+  uint64_t id;
+  slate_kernel_desc desc;
+  const KindOps* ops;
+  int occ;                      // resident worker CTAs per SM
+};
+
+struct Launch {
+  uint64_t id;
+  uint32_t queue;
+  const KernelEntry* k;
+  slate_launch_desc desc;       // args pointer rewritten to `args`
+  std::vector<unsigned char> args;
+  uint32_t B = 0, iters = 1;
+  int state = 0;                // 0 queued, 1 issued, 2 complete
+  int slot = -1;                // TaskCtl / mirror slot
+  cudaEvent_t ev_start = nullptr;
+  std::vector<cudaEvent_t> ev_end;    // kernel ends (main + top-ups), for timing
+  std::vector<cudaEvent_t> ev_done;   // all must complete (main + top-ups, after snapshots)
+  int error = 0;                      // cudaError_t seen on completion
+  bool mirror_complete_seen = false;
+  uint32_t n_resizes = 0, n_topups = 0;
+  std::vector<double> resize_us;
+  // pending resize measurements: epoch, kind (1 shrink, 2 grow), host t0
+  struct PendingResize { uint32_t epoch; int kind; double t0_us; int idx; };
+  std::vector<PendingResize> pending_resize;
+  unsigned char snapshot[kTaskCtlHeader];   // final TaskCtl header copy
+  bool has_snapshot = false;
+};
+
+struct Queue {
+  uint32_t id;
+  cudaStream_t stream = nullptr;
+  cudaStream_t aux = nullptr;   // top-up launches
+  uint64_t* d_ctrl = nullptr;   // the resize word {epoch, lo, hi}
+  uint32_t epoch = 0, lo = 0, hi = 0;
+  bool active = false;          // holds an SM range
+  bool explicit_range = false;  // set by a CORUN placement
+  std::deque<uint64_t> pending; // launches waiting for SMs (AUTO/SOLO)
+  std::deque<uint64_t> issued;  // issued, not complete (stream order)
+  cudaEvent_t last_topup_end = nullptr;  // successors must wait for it
+  bool closed = false;
+};
+
+struct ProfileEntry {
+  slate_profile_t p;
+};
+
+class Server {
+ public:
+  explicit Server(int device);
+  ~Server();
+  int init(std::string* err);
+
+  int num_sms() const { return n_sms_; }
+  slate_info info() const;
+
+  uint32_t open_queue();
+  int close_queue(uint32_t q, int64_t timeout_us, std::string* err);
+
+  int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
+  int launch(uint32_t q, uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err);
+  int resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
+  int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);
+  int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
+  int query(uint64_t l, slate_launch_info* out, std::string* err);
+
+ private:
+  // all private helpers are called with mu_ held
+  int issue(Launch& L, Queue& Q, std::string* err);
+  int write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool immediate, std::string* err);
+  int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
+  void schedule();
+  void release(Queue& Q);
+  void poll_once();
+  void poller_main();
+  int category_of(const Launch& L) const;
+  std::string profile_key(const KernelEntry& k, const slate_launch_desc* d) const;
+  int run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t lo, uint32_t hi, int reps, double* ms,
+                std::string* err);
+  double now_us() const;
+  bool launch_done_events(Launch& L);
+  int alloc_slot();
+  void free_slot(int slot);
+  uint32_t auto_iters(uint32_t B, int occ) const;
+  bool validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const;
+  void work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const;
+
+  int device_;
+  int n_sms_ = 0;
+  uint32_t max_smid_ = 0;
+  uint16_t* d_rank_of_ = nullptr;
+  cudaStream_t ctrl_stream_ = nullptr;
+  cudaStream_t copy_stream_ = nullptr;
+  cudaEvent_t epoch_ev_ = nullptr;
+  void* write_value64_ = nullptr;   // cuStreamWriteValue64 (driver entry point)
+
+  // pools
+  static constexpr int kSlots = 512;
+  TaskCtl* d_tc_ = nullptr;
+  HostMirror* h_mirror_ = nullptr;
+  HostMirror* d_mirror_ = nullptr;
+  unsigned char* h_snap_ = nullptr;   // pinned, kSlots * kTaskCtlHeader
+  void* h_zero_ = nullptr;            // pinned zeros (TaskCtl reset by DMA, no SM)
+  std::vector<int> free_slots_;
+  std::vector<cudaEvent_t> slot_zeroed_;   // DMA zeroing of a freed slot, off the critical path
+  static constexpr int kQueues = 64;
+  uint64_t* d_ctrl_pool_ = nullptr;
+  std::vector<int> free_ctrl_;
+
+  double peak_hbm_ = 6650.0, peak_fp32_ = 74400.0, peak_tc_ = 1590.0;
+  uint32_t standby_timeout_ns_ = 200000;
+
+  mutable std::mutex mu_;
+  std::condition_variable cv_;       // state changes (completion, activation)
+  std::map<uint64_t, std::unique_ptr<KernelEntry>> kernels_;
+  std::map<uint32_t, std::unique_ptr<Queue>> queues_;
+  std::map<uint64_t, std::unique_ptr<Launch>> launches_;
+  std::deque<uint32_t> waiting_;     // queues waiting for SMs, FIFO
+  std::map<uint32_t, uint32_t> bypassed_;
+  std::vector<uint32_t> active_;     // queues holding SMs
+  std::map<std::string, ProfileEntry> profiles_;
+  uint64_t next_kernel_id_ = 1, next_launch_id_ = 1;
+  uint32_t next_queue_id_ = 1;
+  bool profiling_ = false;
+  bool stop_ = false;
+  std::thread poller_;
+};
+
+}  // namespace slate

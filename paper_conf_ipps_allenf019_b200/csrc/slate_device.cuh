@@ -1,0 +1,281 @@
+// slate_device.cuh -- the transformed kernel K*(B*,T) for sm_100a.
+//
+// Paper: Listing 1 (SM binding), Listing 2 (task queue + decode,
+// P:L195-231), §III-C (dynamic resizing).
+// Design: persistent worker CTAs read %smid -> dense
+// rank (reading Q5), check it
+// against the queue's resize word {epoch, lo, hi} (one acquire load), pull
+// SLATE_ITERS consecutive original blocks from the task counter with ONE
+// atomic issued by lane 0 and broadcast by __shfl_sync, decode the task start
+// once (one div + one mod per task) and walk the blocks with x++ and
+// x->y->z rollover, run the tenant body, and re-check the resize word at every
+// task boundary.  Shrink = workers outside the new range
+// retire; grow = waiting CTAs join / a top-up launch adds workers on the new
+// ranks; progress lives only in the counter.  No relaunch (north star).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "kernels.h"
+
+namespace slate {
+
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t r;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(r));
+  return r;
+}
+__device__ __forceinline__ uint64_t ld_acquire_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+template <class Args>
+struct WorkerParams {
+  Args args;
+  uint32_t gx, gy, gz;            // original grid (gridDim of K)
+  uint32_t B;                     // slateMax = gx*gy*gz
+  uint32_t iters;                 // SLATE_ITERS
+  uint32_t occ;                   // resident CTAs per SM of this worker
+  uint32_t bound_lo, bound_hi;    // launch bound (top-up launches), else [0, N-1]
+  uint32_t n_ranks;
+  uint32_t standby_timeout_ns;
+  const uint64_t* ctrl;           // the queue's resize word
+  TaskCtl* tc;
+  HostMirror* mirror;             // device alias of the pinned mirror (may be null)
+  uint32_t* cov;                  // coverage log u32[B] or null
+  const uint16_t* rank_of;        // %smid -> rank
+};
+
+// ------------------------------------------------------------------ decode (Lst2 (4))
+struct BlockWalk {
+  uint32_t x, y, z;
+  __device__ __forceinline__ void start(uint32_t g, uint32_t gx, uint32_t gy) {
+    // one division and one modulo per task; z for 3-D grids (Q18)
+    const uint32_t yz = g / gx;
+    x = g - yz * gx;
+    y = yz % gy;
+    z = yz / gy;
+  }
+  __device__ __forceinline__ void advance(uint32_t gx, uint32_t gy) {
+    // ++blockID.x with rollover, extended y -> z
+    if (++x == gx) {
+      x = 0;
+      if (++y == gy) { y = 0; ++z; }
+    }
+  }
+};
+
+// ------------------------------------------------------------------ bookkeeping
+template <class P>
+__device__ __forceinline__ bool in_range(const P& p, uint32_t rank, uint64_t c) {
+  return rank >= ctrl_lo(c) && rank <= ctrl_hi(c) && rank >= p.bound_lo && rank <= p.bound_hi;
+}
+
+// Lst1 prologue, by ONE thread for its CTA: returns true if the CTA works.
+// An out-of-range CTA waits (standby) while the tenant is under-staffed, so a
+// launch cannot burn its grid on SMs it does not own; it leaves once the
+// tenant has occ*|range| workers or the queue is drained, and after a timeout
+// with zero live workers it runs anyway (liveness).
+template <class P>
+__device__ bool prologue(const P& p, uint32_t rank, uint32_t units) {
+  TaskCtl* tc = p.tc;
+  const uint64_t t0 = globaltimer();
+  uint32_t backoff = 256;
+  for (;;) {
+    const uint64_t c = ld_acquire_u64(p.ctrl);
+    if (ld_relaxed_u32(&tc->next) >= p.B) return false;                 // exit (2)
+    bool join = in_range(p, rank, c);
+    if (!join) {
+      const uint32_t live = ld_relaxed_u32(&tc->live);
+      const uint32_t target = p.occ * (ctrl_hi(c) - ctrl_lo(c) + 1) * units;
+      if (live >= target) return false;                                  // exit (1)
+      if (live == 0 && globaltimer() - t0 > p.standby_timeout_ns) join = true;
+    }
+    if (join) {
+      atomicAdd(&tc->live, units);
+      atomicAdd(&tc->live_rank[rank], units);
+      atomicAdd(&tc->started, units);
+      const uint32_t e = ctrl_epoch(c);
+      if (e > 0 && atomicMax(&tc->join_epoch, e) < e && p.mirror) {      // grow observed
+        p.mirror->join_ns = globaltimer();
+        __threadfence_system();
+        p.mirror->join_epoch = e;
+      }
+      return true;
+    }
+    __nanosleep(backoff);
+    if (backoff < 4096) backoff <<= 1;
+  }
+}
+
+// Whole warp: after the epoch changed, signal the host when no worker is live
+// on a rank outside the new range (end of a shrink).  Called by retiring
+// workers and by the first boundary of each worker after an epoch change.
+template <class P>
+__device__ void check_shrink_done(const P& p, uint64_t c, uint32_t lane) {
+  TaskCtl* tc = p.tc;
+  __syncwarp();      // lane 0's live_rank decrement happens-before the other lanes' scan
+  __threadfence();   // fence.sc: order our live_rank decrement before the scan
+  bool busy = false;
+  for (uint32_t r = lane; r < p.n_ranks; r += 32)
+    if ((r < ctrl_lo(c) || r > ctrl_hi(c)) && ld_relaxed_u32(&tc->live_rank[r]) != 0) busy = true;
+  busy = __any_sync(0xffffffffu, busy);
+  const uint32_t e = ctrl_epoch(c);
+  if (!busy && lane == 0 && atomicMax(&tc->shrink_epoch, e) < e && p.mirror) {
+    p.mirror->shrink_ns = globaltimer();
+    __threadfence_system();
+    p.mirror->shrink_epoch = e;
+  }
+}
+
+// Retire unless this is the last live worker and tasks remain (liveness rule).
+__device__ __forceinline__ bool try_retire(TaskCtl* tc, uint32_t units, uint32_t B) {
+  uint32_t v = ld_relaxed_u32(&tc->live);
+  while (v > units) {
+    const uint32_t w = atomicCAS(&tc->live, v, v - units);
+    if (w == v) return true;
+    v = w;
+  }
+  (void)B;
+  return false;   // the last live worker stays (its next fetch exits if the queue is drained)
+}
+
+template <class P>
+__device__ __forceinline__ void task_done(const P& p, uint32_t g, uint32_t n) {
+  TaskCtl* tc = p.tc;
+  const unsigned long long old = atomicAdd(&tc->done, (1ull << 32) | n);
+  if (uint32_t(old) + n == p.B) {                                       // last block of the launch
+    const uint64_t t = globaltimer();
+    tc->t_last = t;
+    if (p.mirror) {
+      p.mirror->t_last = t;
+      __threadfence_system();
+      p.mirror->complete = 1;
+    }
+  }
+}
+
+// Fetch decision for one worker, made by ONE lane.  Returns the task start g,
+// or 0xffffffff to leave (retired, or the queue is drained).
+//   first: true at the worker's first boundary (prologue already checked ctrl)
+template <class P>
+__device__ __forceinline__ uint32_t boundary_fetch(const P& p, uint32_t rank, uint32_t units,
+                                                   uint64_t& c, bool& retired, bool& epoch_changed) {
+  TaskCtl* tc = p.tc;
+  const uint64_t c2 = ld_acquire_u64(p.ctrl);
+  epoch_changed = ctrl_epoch(c2) != ctrl_epoch(c);
+  c = c2;
+  retired = false;
+  if (!in_range(p, rank, c2) && try_retire(tc, units, p.B)) {
+    retired = true;
+    return 0xffffffffu;
+  }
+  const uint32_t g = atomicAdd(&tc->next, p.iters);                     // Lst2 (2)
+  if (g >= p.B) {                                                       // Q3: nothing to run
+    atomicSub(&tc->live, units);
+    return 0xffffffffu;
+  }
+  if (g == 0) tc->t_first = globaltimer();
+  return g;
+}
+
+// ------------------------------------------------------------------ the worker
+// Tn (tenant) provides: using Args; kThreads; kSmem;
+//   __device__ static void cta_block(const Args&, uint32_t x, uint32_t y, uint32_t z, char* smem)
+// executed by all kThreads threads of the CTA (may use __syncthreads).
+//
+// Per task (Lst2): lane 0 of warp 0 loads the resize word (acquire), retires
+// the CTA if its rank left the range (unless it is the last live worker), else
+// fetches `iters` blocks with ONE atomicAdd on the task counter; the values go
+// to warp 0 by __shfl_sync and to the other warps through shared memory and
+// the barrier (reading Q19).
+template <class Tn>
+__device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args>& p) {
+  extern __shared__ __align__(128) char dyn_smem[];
+  __shared__ uint32_t s_go;
+  __shared__ uint32_t s_g;
+  __shared__ uint32_t s_retired;
+  __shared__ uint32_t s_rank;
+  const uint32_t lane = threadIdx.x & 31;
+
+  // ---- Lst1: the block leader binds the CTA to its SM
+  if (threadIdx.x == 0) {
+    const uint32_t r = p.rank_of[smid()];
+    s_rank = r;
+    s_go = prologue(p, r, 1u) ? 1u : 0u;
+  }
+  __syncthreads();
+  if (!s_go) return;
+  const uint32_t rank = s_rank;
+  uint64_t c = ld_acquire_u64(p.ctrl);
+
+  for (;;) {
+    if (threadIdx.x < 32) {
+      uint32_t g = 0, ret = 0, chg = 0;
+      if (lane == 0) {
+        bool retired, changed;
+        g = boundary_fetch(p, rank, 1u, c, retired, changed);   // Lst2 (2)
+        ret = retired;
+        chg = changed;
+      }
+      g = __shfl_sync(0xffffffffu, g, 0);
+      chg = __shfl_sync(0xffffffffu, chg, 0);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if (lane == 0) {
+        s_g = g;
+        s_retired = ret;
+      }
+      if (chg && g != 0xffffffffu) check_shrink_done(p, c, lane);
+    }
+    __syncthreads();
+    const uint32_t g = s_g;
+    if (g == 0xffffffffu) {   // Lst2 (1): retreat or queue exhausted
+      if (threadIdx.x < 32) {
+        if (lane == 0) atomicSub(&p.tc->live_rank[rank], 1u);
+        if (s_retired) check_shrink_done(p, c, lane);
+      }
+      return;
+    }
+    const uint32_t n = min(p.iters, p.B - g);   // clamp the last task
+    BlockWalk w;
+    w.start(g, p.gx, p.gy);
+    for (uint32_t i = 0; i < n; ++i) {           // Lst2 (3): the task's blocks, in order
+      Tn::cta_block(p.args, w.x, w.y, w.z, dyn_smem);   // Lst2 (5): the user code
+      if (p.cov && threadIdx.x == 0) atomicAdd(&p.cov[g + i], 1u);
+      w.advance(p.gx, p.gy);                     // Lst2 (4)
+    }
+    __syncthreads();   // every thread is done with the task (and with s_g)
+    if (threadIdx.x == 0) task_done(p, g, n);
+  }
+}
+
+template <class Tn>
+__global__ void __launch_bounds__(Tn::kThreads) slate_worker(const __grid_constant__ WorkerParams<typename Tn::Args> p) {
+  worker_body<Tn>(p);
+}
+
+// The original kernel K(B,T) on the hardware block scheduler: the same body
+// code, blockIdx from hardware.  Used for the bit-exact comparison (north
+// star) and as the "vanilla CUDA" schedule.
+template <class Tn>
+__global__ void __launch_bounds__(Tn::kThreads) standalone(const __grid_constant__ typename Tn::Args a) {
+  extern __shared__ __align__(128) char dyn_smem[];
+  Tn::cta_block(a, blockIdx.x, blockIdx.y, blockIdx.z, dyn_smem);
+}
+
+// SM-id calibration probe (K13): every CTA records its %smid.
+__global__ void calibrate_kernel(uint32_t* out, uint32_t spin_ns);
+
+}  // namespace slate

@@ -1,0 +1,97 @@
+"""GPU parity of the slate path (-m gpu): every tenant through the C ABI,
+  * slate worker output == the same tenant's standalone launch, bit for bit;
+  * output == oracle (exact on integer inputs, Q17 tolerance on floats);
+  * coverage log all ones and counters == oracle.expected_counters
+    (blocks_done, tasks_done, next_clamped), for iters in {1, 10}, on the full
+    GPU and on a sub-range of SMs.
+Sizes span several tiles and a ragged tail."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import tenants as OT
+from paper_conf_ipps_allenf019_b200 import slate as S
+
+from gpu_helpers import (make_bs, make_copy, make_gemm, make_sgemm, make_spmv, make_stencil, make_triad)
+
+pytestmark = pytest.mark.gpu
+
+CASES = {
+    "triad_float": lambda: make_triad(1024 * 37 + 517, 101),
+    "triad_int": lambda: make_triad(1024 * 50 + 4, 102, "int"),
+    "copy": lambda: make_copy(4096 * 21 + 999, 103),
+    "sgemm_float": lambda: make_sgemm(200, 232, 96, 104),
+    "sgemm_int": lambda: make_sgemm(256, 256, 256, 105, "int"),
+    "spmv_float": lambda: make_spmv(32 * 300 + 7, 106, band=512),
+    "spmv_int": lambda: make_spmv(32 * 128, 107, "int", band=64),
+    "bs": lambda: make_bs(1024 * 12 + 4 * 33 + 2, 108, n_scen=5),
+    "stencil_float": lambda: make_stencil(8 * 37 + 3, 32 * 9 + 5, 109),
+    "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
+}
+
+
+@pytest.fixture(scope="module")
+def sess():
+    s = S.Session(None, 0)
+    yield s
+    s.close()
+
+
+def _run(sess, t, kernel, **kw):
+    t.zero_outputs()
+    cov = torch.zeros(int(np.prod(t.grid)), dtype=torch.int32, device="cuda:0")
+    torch.cuda.synchronize()   # the server's streams do not wait for torch's stream
+    lid = sess.launch(kernel, t.args, t.grid, coverage=cov if kw.pop("cov", True) else None, **kw)
+    sess.sync(lid)
+    torch.cuda.synchronize()
+    return lid, t.snapshot(), cov
+
+
+@pytest.mark.parametrize("name", sorted(CASES))
+def test_tenant_parity(sess, name):
+    t = CASES[name]()
+    k_std = sess.register_kernel(t.kind)
+    lid, ref_outs, _ = _run(sess, t, k_std, mode=S.MODE_STANDALONE, cov=False)
+    ok, err = t.check(ref_outs)
+    assert ok, "standalone vs oracle: %s (worst %.3g of tolerance)" % (name, err)
+    B = int(np.prod(t.grid))
+    n = sess.info()["num_sms"]
+    for iters in (1, 10):
+        k = sess.register_kernel(t.kind, iters=iters, flags=S.KFLAG_COVERAGE)
+        for sm in [(0, n - 1), (3, 3 + n // 3)]:
+            lid, outs, cov = _run(sess, t, k, placement=S.PLACE_CORUN, sm=sm)
+            for a, b in zip(outs, ref_outs):
+                assert torch.equal(a, b), "slate vs standalone not bit-exact: %s iters=%d sm=%s" % (name, iters, sm)
+            q = sess.query(lid)
+            ex = OT.expected_counters(B, iters)
+            assert q["state"] == 2 and q["coverage_ok"] == 1
+            assert np.array_equal(cov.cpu().numpy(), ex["coverage"].astype(np.int32))
+            assert (q["blocks_done"], q["tasks_done"], q["next_clamped"]) == \
+                (ex["blocks_done"], ex["tasks_done"], ex["next_clamped"]), (name, iters, q)
+            assert q["live_workers"] == 0
+
+
+def test_empty_and_single_block(sess):
+    t = make_triad(3, 111)          # one block, 3 elements (ragged inside a float4)
+    k = sess.register_kernel(t.kind, iters=10, flags=S.KFLAG_COVERAGE)
+    lid, outs, cov = _run(sess, t, k, placement=S.PLACE_CORUN, sm=(0, 0))
+    assert t.check(outs)[0]
+    assert sess.query(lid)["tasks_done"] == 1
+    with pytest.raises(S.SlateError):
+        args, grid = S.triad_args(torch.zeros(0, device="cuda:0"), torch.zeros(0, device="cuda:0"),
+                                  torch.zeros(0, device="cuda:0"), 1.0)
+        sess.launch(k, args, grid)
+    with pytest.raises(S.SlateError):          # grid inconsistent with args
+        sess.launch(k, t.args, (2, 1, 1))
+    with pytest.raises(S.SlateError):          # bad SM range
+        sess.launch(k, t.args, t.grid, placement=S.PLACE_CORUN, sm=(5, 4))
+
+
+def test_auto_solo_path(sess):
+    t = make_stencil(8 * 64, 32 * 64, 112)
+    k = sess.register_kernel(t.kind)
+    lid = sess.launch(k, t.args, t.grid, placement=S.PLACE_AUTO)
+    sess.sync(lid)
+    assert t.check(t.snapshot())[0]
+    q = sess.query(lid)
+    assert q["blocks_done"] == q["total_blocks"] and q["end_ms"] >= q["start_ms"] > 0

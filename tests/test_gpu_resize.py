@@ -1,0 +1,106 @@
+"""GPU tests of dynamic resizing (-m gpu): random resize storms from the host
+while a launch runs must keep every original block executed exactly once
+(coverage log all ones, exact counters) and the output bit-identical to the
+standalone launch (P:L127 progress carried in slateIdx; P:L243-245 exit
+conditions); shrink and grow latencies are observed."""
+import random
+import time
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import tenants as OT
+from paper_conf_ipps_allenf019_b200 import slate as S
+
+from gpu_helpers import make_bs, make_copy, make_stencil, make_triad, within
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sess():
+    s = S.Session(None, 0)
+    yield s
+    s.close()
+
+
+def _storm(sess, t, iters, n_resizes, seed, gap_us):
+    n = sess.info()["num_sms"]
+    k_std = sess.register_kernel(t.kind)
+    t.zero_outputs()
+    torch.cuda.synchronize()
+    sess.sync(sess.launch(k_std, t.args, t.grid, mode=S.MODE_STANDALONE))
+    ref = t.snapshot()
+    k = sess.register_kernel(t.kind, iters=iters, flags=S.KFLAG_COVERAGE)
+    t.zero_outputs()
+    B = int(np.prod(t.grid))
+    cov = torch.zeros(B, dtype=torch.int32, device="cuda:0")
+    torch.cuda.synchronize()   # the server's streams do not wait for torch's stream
+    rng = random.Random(seed)
+    lid = sess.launch(k, t.args, t.grid, placement=S.PLACE_CORUN, sm=(0, n - 1), coverage=cov)
+    done = 0
+    for _ in range(n_resizes):
+        lo = rng.randrange(0, n)
+        hi = rng.randrange(lo, n)
+        st = sess.resize(lid, lo, hi)
+        done += 1
+        if st == S.DONE:
+            break
+        t0 = time.perf_counter()
+        while (time.perf_counter() - t0) * 1e6 < gap_us:
+            pass
+    sess.sync(lid)
+    torch.cuda.synchronize()
+    q = sess.query(lid)
+    ex = OT.expected_counters(B, iters)
+    assert q["coverage_ok"] == 1 and np.array_equal(cov.cpu().numpy(), ex["coverage"].astype(np.int32))
+    assert (q["blocks_done"], q["tasks_done"], q["next_clamped"]) == \
+        (ex["blocks_done"], ex["tasks_done"], ex["next_clamped"])
+    for a, b in zip(t.snapshot(), ref):
+        assert torch.equal(a, b)
+    return q, done
+
+
+def test_resize_storm_bs(sess):
+    t = make_bs(1 << 21, 201, n_scen=64)
+    q, done = _storm(sess, t, 1, 30, 1, 100)
+    assert done >= 5 and q["n_resizes"] >= 5
+    # the launch really ran on sub-ranges: a sampled block matches the oracle
+    S_, X_, T_ = (x.cpu().numpy() for x in t._keep[:3])
+    sig = t._keep[3].cpu().numpy()
+    blocks = [0, 777, int(np.prod(t.grid)) - 1]
+    c_ref, p_ref = OT.blackscholes(S_, X_, T_, 0.02, sig, blocks=blocks)
+    out = t.snapshot()[0].cpu().numpy()
+    idx = np.concatenate([np.arange(b * 1024, min((b + 1) * 1024, len(S_))) for b in blocks])
+    assert within(out[idx], c_ref[idx], S_[idx].astype(np.float64))[0]
+
+
+def test_resize_storm_cta_tenant(sess):
+    t = make_stencil(8192, 8192, 202)
+    q, done = _storm(sess, t, 10, 30, 2, 20)
+    assert done >= 3
+
+
+def test_resize_storm_iters1_copy(sess):
+    t = make_copy(1 << 29, 203)
+    q, done = _storm(sess, t, 1, 40, 3, 10)
+    assert done >= 10
+    assert len(q["resize_us"]) >= 3, q
+
+
+def test_shrink_then_grow_latency(sess):
+    n = sess.info()["num_sms"]
+    t = make_triad(1 << 28, 204)
+    k = sess.register_kernel(t.kind, iters=1)
+    lid = sess.launch(k, t.args, t.grid, placement=S.PLACE_CORUN, sm=(0, n - 1))
+    time.sleep(0.0002)
+    sess.resize(lid, 0, n // 2 - 1)      # shrink: workers on the upper half retire
+    time.sleep(0.0002)
+    sess.resize(lid, 0, n - 1)           # grow: a top-up launch adds workers
+    sess.sync(lid)
+    q = sess.query(lid)
+    assert q["blocks_done"] == q["total_blocks"]
+    assert q["n_topups"] >= 1
+    lat = q["resize_us"]
+    assert len(lat) == 2 and all(0 < v < 5000 for v in lat), lat

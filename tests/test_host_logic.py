@@ -1,0 +1,84 @@
+"""CPU-only checks of the C-ABI library: it loads without a GPU, exports every
+symbol include/slate.h declares, refuses to run without a GPU (no CPU
+fallback), and its host-side selector logic agrees with the oracle."""
+import itertools
+import os
+import random
+import re
+
+import pytest
+
+from oracle import selector as OS
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def S():
+    from paper_conf_ipps_allenf019_b200 import build
+    build.build()
+    from paper_conf_ipps_allenf019_b200 import slate
+    return slate
+
+
+def _declared():
+    txt = open(os.path.join(ROOT, "include", "slate.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(slate_[a-z_0-9]+)\s*\(", txt)))
+
+
+def test_exports_every_declared_symbol(S):
+    import ctypes
+    lib = ctypes.CDLL(S.LIB_PATH)
+    names = _declared()
+    assert len(names) >= 17
+    for n in names:
+        assert hasattr(lib, n), n
+    assert sorted(S.EXPORTED) == names
+
+
+def test_no_cpu_fallback(S):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(S.SlateError) as e:
+        S.Session(None, 0)
+    assert e.value.status == S.ECUDA
+    assert S.status_string(S.ECUDA) == "SLATE_ECUDA"
+
+
+def test_policy_matches_oracle(S):
+    for a, b in itertools.product(OS.CATEGORIES, repeat=2):
+        for lit in (False, True):
+            assert S.policy(a, b, lit) == OS.policy(a, b, lit)
+
+
+def test_classify_matches_oracle(S):
+    fr = [0.0, 0.005, 0.0099, 0.01, 0.05, 0.0999, 0.1, 0.2, 0.2499, 0.25, 0.5, 0.8499, 0.85, 1.0, 1.2]
+    for m, f, t in itertools.product(fr, fr, [0.0, 0.02, 0.5]):
+        c, mm, cat = OS.classify(m, f, t, 1.0, 1.0, 1.0)
+        assert S.classify(m, f, t) == (c, mm, cat)
+
+
+def test_select_matches_oracle(S):
+    rng = random.Random(5)
+    for _ in range(2000):
+        active = rng.choice(OS.CATEGORIES)
+        q = [rng.choice(OS.CATEGORIES) for _ in range(rng.randrange(0, 6))]
+        byp = [rng.randrange(0, 6) for _ in q]
+        assert S.select(active, q) == OS.select(active, q)
+        assert S.select(active, q, bypassed=byp) == OS.select(active, q, bypassed=byp)
+
+
+def test_choose_split_matches_oracle(S):
+    rng = random.Random(7)
+    pts = [148, 111, 74, 49, 37, 18]
+    for _ in range(200):
+        knee_a, knee_b = rng.uniform(10, 148), rng.uniform(10, 148)
+        ta, tb = rng.uniform(0.2, 5), rng.uniform(0.2, 5)
+        ca = {s: ta * max(1.0, knee_a / s) for s in pts}
+        cb = {s: tb * max(1.0, knee_b / s) for s in pts}
+        s1, t1 = S.choose_split(ca, cb, 148)
+        s2, t2 = OS.choose_split(ca, cb, 148)
+        assert abs(t1 - t2) <= 1e-9 * t2
+        assert s1 == s2 or abs(OS.corun_makespan(ca, cb, 148, s1) - t2) <= 1e-9 * t2
