@@ -143,12 +143,6 @@ def spmv_csr(rowptr, col, val, xvec, blocks=None):
 
 
 # ---------------------------------------------------------------- Black-Scholes
-def bs_sigmas(p_count, sigma0=0.30, dsigma=0.01):
-    """Volatility scenarios sigma_p = sigma0 + p*dsigma, p = 0..P-1 (reading Q16).
-    Computed in float32 -- the same float32 values the kernel is given."""
-    return (np.float32(sigma0) + np.float32(dsigma) * np.arange(p_count, dtype=np.float32)).astype(np.float32)
-
-
 def phi(x):
     """Standard normal CDF, Phi(x) = erfc(-x / sqrt(2)) / 2, in double."""
     return 0.5 * erfc(-x / math.sqrt(2.0))

@@ -35,8 +35,8 @@ cudaError_t launch_standalone_t(const void* args, dim3 grid, cudaStream_t st) {
   typename Tn::Args a;
   std::memcpy(&a, args, sizeof(a));
   void* kargs[] = {&a};
-  return cudaLaunchKernel(reinterpret_cast<const void*>(&standalone<Tn>), grid, dim3(Tn::kThreads), kargs, Tn::kSmem,
-                          st);
+  return cudaLaunchKernel(reinterpret_cast<const void*>(&standalone<Tn>), grid, dim3(Tn::kThreads), kargs,
+                          Tn::kSmemStandalone, st);
 }
 
 template <class Tn>
@@ -46,6 +46,7 @@ KindOps make_ops(uint32_t default_iters) {
   o.standalone_fn = reinterpret_cast<const void*>(&standalone<Tn>);
   o.threads = Tn::kThreads;
   o.smem = Tn::kSmem;
+  o.smem_standalone = Tn::kSmemStandalone;
   o.args_size = sizeof(typename Tn::Args);
   o.default_iters = default_iters;
   o.launch_worker = &launch_worker_t<Tn>;

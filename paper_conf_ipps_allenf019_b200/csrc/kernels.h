@@ -62,7 +62,8 @@ struct KindOps {
   const void* worker_fn = nullptr;
   const void* standalone_fn = nullptr;
   int threads = 0;
-  int smem = 0;
+  int smem = 0;              // dynamic smem of the worker
+  int smem_standalone = 0;   // dynamic smem of the standalone kernel
   size_t args_size = 0;
   uint32_t default_iters = 0;   // 0: auto (reading Q11)
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;

@@ -198,10 +198,10 @@ int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::stri
   k->desc = *d;
   k->desc.iters = iters;
   k->ops = ops;
-  if (ops->smem > 48 * 1024) {
+  if (ops->smem > 48 * 1024)
     CK(cudaFuncSetAttribute(ops->worker_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem));
-    CK(cudaFuncSetAttribute(ops->standalone_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem));
-  }
+  if (ops->smem_standalone > 48 * 1024)
+    CK(cudaFuncSetAttribute(ops->standalone_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem_standalone));
   int occ = 0;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ops->worker_fn, ops->threads, ops->smem));
   if (occ < 1) {
@@ -244,6 +244,7 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     }
     case SLATE_KIND_SPMV_CSR: {
       auto a = static_cast<const slate_args_spmv*>(d->args);
+      if (!al(a->col) || !al(a->val)) return fail("spmv col/val must be 16-byte aligned");
       g[0] = cdiv(a->n_rows, 32);
       break;
     }
@@ -377,7 +378,35 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
 }
 
 // ------------------------------------------------------------------ issue
+// Launches of a queue reach its stream in submission order; one that finds no
+// free control block waits in Q.deferred (and so do all later ones) until the
+// poller frees blocks.
 int Server::issue(Launch& L, Queue& Q, std::string* err) {
+  const bool needs_slot = L.desc.mode != SLATE_MODE_STANDALONE;
+  if (!Q.deferred.empty() || (needs_slot && free_slots_.empty())) {
+    Q.deferred.push_back(L.id);
+    return SLATE_OK;
+  }
+  return issue_now(L, Q, err);
+}
+
+void Server::fail_launch(Launch& L, int code) {
+  L.error = code;
+  L.state = 2;
+  cv_.notify_all();
+}
+
+void Server::drain_deferred(Queue& Q) {
+  std::string err;
+  while (!Q.deferred.empty()) {
+    Launch& L = *launches_[Q.deferred.front()];
+    if (L.desc.mode != SLATE_MODE_STANDALONE && free_slots_.empty()) break;
+    Q.deferred.pop_front();
+    if (issue_now(L, Q, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
+  }
+}
+
+int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
   const KindOps* ops = L.k->ops;
   if (Q.last_topup_end) {   // stream semantics: the predecessor's top-up workers must finish first
     CK(cudaStreamWaitEvent(Q.stream, Q.last_topup_end, 0));
@@ -432,7 +461,7 @@ int Server::issue(Launch& L, Queue& Q, std::string* err) {
 // queued behind it on the stream picks up the new range by itself); later
 // launches wait for the top-up's end (stream semantics).
 int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
-  if (Q.issued.size() != 1 || !Q.pending.empty()) return SLATE_OK;
+  if (Q.issued.size() != 1 || !Q.pending.empty() || !Q.deferred.empty()) return SLATE_OK;
   Launch& R = *launches_[Q.issued.front()];
   if (R.state != 1 || R.slot < 0 || R.desc.mode == SLATE_MODE_STANDALONE) return SLATE_OK;
   if (h_mirror_[R.slot].complete) return SLATE_OK;
@@ -508,6 +537,26 @@ int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_
       Q.active = true;
       active_.push_back(Q.id);
       rc = write_ctrl(Q, d->sm_lo, d->sm_hi, false, err);
+      // co-runners yield the requested SMs (shrink on arrival)
+      for (uint32_t other : active_) {
+        if (other == Q.id) continue;
+        Queue& A = *queues_[other];
+        if (A.hi < d->sm_lo || A.lo > d->sm_hi) continue;
+        const uint32_t left = d->sm_lo > A.lo ? d->sm_lo - A.lo : 0;     // [A.lo, sm_lo - 1]
+        const uint32_t right = A.hi > d->sm_hi ? A.hi - d->sm_hi : 0;    // [sm_hi + 1, A.hi]
+        if (!left && !right) continue;                                     // nothing left to keep: overlap
+        const uint32_t nlo = left >= right ? A.lo : d->sm_hi + 1;
+        const uint32_t nhi = left >= right ? d->sm_lo - 1 : A.hi;
+        const double t0 = now_us();
+        if (write_ctrl(A, nlo, nhi, true, err) == SLATE_OK && !A.issued.empty()) {
+          Launch& R = *launches_[A.issued.front()];
+          R.n_resizes += 1;
+          if (R.resize_us.size() < 16) {
+            R.pending_resize.push_back({A.epoch, 1, t0, int(R.resize_us.size())});
+            R.resize_us.push_back(-1);
+          }
+        }
+      }
     } else if (Q.lo != d->sm_lo || Q.hi != d->sm_hi) {
       rc = write_ctrl(Q, d->sm_lo, d->sm_hi, true, err);
       if (rc == SLATE_OK && (d->sm_lo < old_lo || d->sm_hi > old_hi)) rc = grow_running(Q, old_lo, old_hi, err);
@@ -521,6 +570,7 @@ int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_
     if (std::find(waiting_.begin(), waiting_.end(), Q.id) == waiting_.end()) waiting_.push_back(Q.id);
     schedule();
   }
+  if (rc != SLATE_OK) fail_launch(LL, int(cudaErrorLaunchFailure));
   return rc;
 }
 
@@ -568,7 +618,7 @@ void Server::schedule() {
       while (!Q.pending.empty()) {
         Launch& L = *launches_[Q.pending.front()];
         Q.pending.pop_front();
-        issue(L, Q, &err);
+        if (issue(L, Q, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
       }
       continue;
     }
@@ -636,7 +686,7 @@ void Server::schedule() {
     while (!Bq.pending.empty()) {
       Launch& L = *launches_[Bq.pending.front()];
       Bq.pending.pop_front();
-      issue(L, Bq, &err);
+      if (issue(L, Bq, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
     }
     break;   // at most two co-runners (reading Q13)
   }
@@ -649,8 +699,9 @@ void Server::release(Queue& Q) {
   Q.explicit_range = false;
   active_.erase(std::remove(active_.begin(), active_.end(), Q.id), active_.end());
   if (active_.size() == 1) {
+    // the survivor claims the released SMs, explicit placement or not
     Queue& A = *queues_[active_[0]];
-    if (!A.explicit_range && (A.lo != 0 || A.hi != uint32_t(n_sms_ - 1))) {
+    if (A.lo != 0 || A.hi != uint32_t(n_sms_ - 1)) {
       const uint32_t old_lo = A.lo, old_hi = A.hi;
       const double t0 = now_us();
       write_ctrl(A, 0, uint32_t(n_sms_ - 1), true, &err);
@@ -750,7 +801,8 @@ void Server::poll_once() {
       if (Q.last_topup_end && Q.issued.empty()) Q.last_topup_end = nullptr;
       cv_.notify_all();
     }
-    if (Q.active && Q.issued.empty() && Q.pending.empty()) idle.push_back(Q.id);
+    drain_deferred(Q);
+    if (Q.active && Q.issued.empty() && Q.pending.empty() && Q.deferred.empty()) idle.push_back(Q.id);
   }
   for (uint32_t q : idle) release(*queues_[q]);
 }
@@ -761,7 +813,7 @@ void Server::poller_main() {
   while (!stop_) {
     bool busy = false;
     for (auto& kv : queues_)
-      if (!kv.second->issued.empty()) busy = true;
+      if (!kv.second->issued.empty() || !kv.second->deferred.empty()) busy = true;
     if (!busy) {
       cv_.wait_for(g, std::chrono::milliseconds(2));
       continue;
@@ -783,7 +835,8 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
       return it == launches_.end() || it->second->state == 2;
     }
     auto qi = queues_.find(q);
-    return qi == queues_.end() || (qi->second->issued.empty() && qi->second->pending.empty());
+    return qi == queues_.end() ||
+           (qi->second->issued.empty() && qi->second->pending.empty() && qi->second->deferred.empty());
   };
   if (l && launches_.find(l) == launches_.end()) return SLATE_ENOTFOUND;
   while (!done()) {

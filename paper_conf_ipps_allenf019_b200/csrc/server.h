@@ -58,6 +58,7 @@ struct Queue {
   bool active = false;          // holds an SM range
   bool explicit_range = false;  // set by a CORUN placement
   std::deque<uint64_t> pending; // launches waiting for SMs (AUTO/SOLO)
+  std::deque<uint64_t> deferred;  // granted SMs but waiting for a control block (stream order)
   std::deque<uint64_t> issued;  // issued, not complete (stream order)
   cudaEvent_t last_topup_end = nullptr;  // successors must wait for it
   bool closed = false;
@@ -89,6 +90,9 @@ class Server {
  private:
   // all private helpers are called with mu_ held
   int issue(Launch& L, Queue& Q, std::string* err);
+  int issue_now(Launch& L, Queue& Q, std::string* err);
+  void drain_deferred(Queue& Q);
+  void fail_launch(Launch& L, int code);
   int write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool immediate, std::string* err);
   int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
   void schedule();
@@ -117,7 +121,7 @@ class Server {
   void* write_value64_ = nullptr;   // cuStreamWriteValue64 (driver entry point)
 
   // pools
-  static constexpr int kSlots = 512;
+  static constexpr int kSlots = 4096;
   TaskCtl* d_tc_ = nullptr;
   HostMirror* h_mirror_ = nullptr;
   HostMirror* d_mirror_ = nullptr;

@@ -205,7 +205,7 @@ template <class Tn>
 __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args>& p) {
   extern __shared__ __align__(128) char dyn_smem[];
   __shared__ uint32_t s_go;
-  __shared__ uint32_t s_g;
+  __shared__ uint32_t s_g[2];
   __shared__ uint32_t s_retired;
   __shared__ uint32_t s_rank;
   const uint32_t lane = threadIdx.x & 31;
@@ -214,19 +214,27 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
   if (threadIdx.x == 0) {
     const uint32_t r = p.rank_of[smid()];
     s_rank = r;
+    s_retired = 0;
     s_go = prologue(p, r, 1u) ? 1u : 0u;
   }
   __syncthreads();
   if (!s_go) return;
   const uint32_t rank = s_rank;
   uint64_t c = ld_acquire_u64(p.ctrl);
+  if constexpr (Tn::kHasInit) {
+    Tn::cta_init(dyn_smem);
+    __syncthreads();
+  }
 
-  for (;;) {
+  // Lst2 (2): one lane fetches (after checking the resize word), warp 0 gets the
+  // value by __shfl_sync, the other warps through shared memory (reading Q19).
+  // Ends with a barrier; every thread returns the same task start.
+  auto fetch = [&](int slot) -> uint32_t {
     if (threadIdx.x < 32) {
       uint32_t g = 0, ret = 0, chg = 0;
       if (lane == 0) {
         bool retired, changed;
-        g = boundary_fetch(p, rank, 1u, c, retired, changed);   // Lst2 (2)
+        g = boundary_fetch(p, rank, 1u, c, retired, changed);
         ret = retired;
         chg = changed;
       }
@@ -234,30 +242,48 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
       chg = __shfl_sync(0xffffffffu, chg, 0);
       c = __shfl_sync(0xffffffffu, c, 0);
       if (lane == 0) {
-        s_g = g;
-        s_retired = ret;
+        s_g[slot] = g;
+        if (ret) s_retired = 1;
       }
       if (chg && g != 0xffffffffu) check_shrink_done(p, c, lane);
     }
     __syncthreads();
-    const uint32_t g = s_g;
-    if (g == 0xffffffffu) {   // Lst2 (1): retreat or queue exhausted
-      if (threadIdx.x < 32) {
-        if (lane == 0) atomicSub(&p.tc->live_rank[rank], 1u);
-        if (s_retired) check_shrink_done(p, c, lane);
+    return s_g[slot];
+  };
+
+  uint32_t g = fetch(0);
+  int slot = 0;
+  while (g != 0xffffffffu) {                      // Lst2 (1): until retreat or an empty queue
+    const uint32_t n = min(p.iters, p.B - g);     // clamp the last task
+    if constexpr (Tn::kLookahead) {
+      // the next task is fetched (resize word checked) before this one runs,
+      // so the tenant can stream its data in while this task computes
+      const uint32_t g2 = fetch(slot ^ 1);
+      const uint32_t n2 = g2 == 0xffffffffu ? 0u : min(p.iters, p.B - g2);
+      Tn::cta_task2(p.args, g, n, g2, n2, dyn_smem);
+      if (p.cov && threadIdx.x == 0)
+        for (uint32_t i = 0; i < n; ++i) atomicAdd(&p.cov[g + i], 1u);
+      __syncthreads();
+      if (threadIdx.x == 0) task_done(p, g, n);
+      g = g2;
+      slot ^= 1;
+    } else {
+      BlockWalk w;
+      w.start(g, p.gx, p.gy);
+      for (uint32_t i = 0; i < n; ++i) {          // Lst2 (3): the task's blocks, in order
+        Tn::cta_block(p.args, w.x, w.y, w.z, dyn_smem);   // Lst2 (5): the user code
+        if (p.cov && threadIdx.x == 0) atomicAdd(&p.cov[g + i], 1u);
+        w.advance(p.gx, p.gy);                    // Lst2 (4)
       }
-      return;
+      __syncthreads();   // every thread is done with the task
+      if (threadIdx.x == 0) task_done(p, g, n);
+      g = fetch(0);
     }
-    const uint32_t n = min(p.iters, p.B - g);   // clamp the last task
-    BlockWalk w;
-    w.start(g, p.gx, p.gy);
-    for (uint32_t i = 0; i < n; ++i) {           // Lst2 (3): the task's blocks, in order
-      Tn::cta_block(p.args, w.x, w.y, w.z, dyn_smem);   // Lst2 (5): the user code
-      if (p.cov && threadIdx.x == 0) atomicAdd(&p.cov[g + i], 1u);
-      w.advance(p.gx, p.gy);                     // Lst2 (4)
-    }
-    __syncthreads();   // every thread is done with the task (and with s_g)
-    if (threadIdx.x == 0) task_done(p, g, n);
+  }
+  if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
+  if (threadIdx.x < 32) {
+    if (lane == 0) atomicSub(&p.tc->live_rank[rank], 1u);
+    if (s_retired) check_shrink_done(p, c, lane);
   }
 }
 
@@ -272,7 +298,12 @@ __global__ void __launch_bounds__(Tn::kThreads) slate_worker(const __grid_consta
 template <class Tn>
 __global__ void __launch_bounds__(Tn::kThreads) standalone(const __grid_constant__ typename Tn::Args a) {
   extern __shared__ __align__(128) char dyn_smem[];
+  if constexpr (Tn::kHasInit) {
+    Tn::cta_init(dyn_smem);
+    __syncthreads();
+  }
   Tn::cta_block(a, blockIdx.x, blockIdx.y, blockIdx.z, dyn_smem);
+  if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
 }
 
 // SM-id calibration probe (K13): every CTA records its %smid.

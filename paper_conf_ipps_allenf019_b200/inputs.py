@@ -82,6 +82,12 @@ def bs_inputs(n, seed):
     return S, X, T, np.float32(0.02)
 
 
+def bs_sigmas(p_count, sigma0=0.30, dsigma=0.01):
+    """Volatility scenarios sigma_p = sigma0 + p*dsigma, p = 0..P-1 (reading Q16),
+    as float32: the values both the kernel and the oracle are given."""
+    return (np.float32(sigma0) + np.float32(dsigma) * np.arange(p_count, dtype=np.float32)).astype(np.float32)
+
+
 def stencil_inputs(h, w, seed, mode="float"):
     """HxW fp32 field: U[0,1) (float) or a random integer linear field
     f = a*i + b*j + c with small integer a, b, c (int)."""

@@ -100,7 +100,7 @@ def make_spmv(n_rows, seed, mode="float", band=4096):
 
 def make_bs(n, seed, n_scen=4):
     Sx, X, T, r = I.bs_inputs(n, seed)
-    sig = OT.bs_sigmas(n_scen)
+    sig = I.bs_sigmas(n_scen)
     S_d, X_d, T_d, sig_d = dev(Sx), dev(X), dev(T), dev(sig)
     call_d, put_d = torch.zeros(n, device=DEV), torch.zeros(n, device=DEV)
     args, grid = S.bs_args(S_d, X_d, T_d, call_d, put_d, sig_d, r)
