@@ -49,6 +49,7 @@ KindOps make_ops(uint32_t default_iters) {
   o.smem_standalone = Tn::kSmemStandalone;
   o.args_size = sizeof(typename Tn::Args);
   o.default_iters = default_iters;
+  o.max_auto_iters = Tn::kMaxIters;
   o.launch_worker = &launch_worker_t<Tn>;
   o.launch_standalone = &launch_standalone_t<Tn>;
   return o;

@@ -66,6 +66,7 @@ struct KindOps {
   int smem_standalone = 0;   // dynamic smem of the standalone kernel
   size_t args_size = 0;
   uint32_t default_iters = 0;   // 0: auto (reading Q11)
+  uint32_t max_auto_iters = 10; // per-tenant cap of the automatic task size
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;
   cudaError_t (*launch_standalone)(const void* args, dim3 grid, cudaStream_t) = nullptr;
 };

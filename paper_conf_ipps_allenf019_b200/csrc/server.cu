@@ -106,7 +106,7 @@ int Server::init(std::string* err) {
   CK(cudaHostAlloc(reinterpret_cast<void**>(&h_snap_), kTaskCtlHeader * kSlots, cudaHostAllocDefault));
   CK(cudaHostAlloc(&h_zero_, sizeof(TaskCtl), cudaHostAllocDefault));
   std::memset(h_zero_, 0, sizeof(TaskCtl));
-  for (int i = kSlots - 1; i >= 0; --i) free_slots_.push_back(i);
+  for (int i = 0; i < kSlots; ++i) free_slots_.push_back(i);
   slot_zeroed_.assign(kSlots, nullptr);
   CK(cudaMalloc(&d_ctrl_pool_, 128 * kQueues));
   CK(cudaMemset(d_ctrl_pool_, 0, 128 * kQueues));
@@ -332,8 +332,8 @@ void Server::work(const KernelEntry& k, const slate_launch_desc* d, double* byte
 
 int Server::alloc_slot() {
   if (free_slots_.empty()) return -1;
-  const int s = free_slots_.back();
-  free_slots_.pop_back();
+  const int s = free_slots_.front();
+  free_slots_.pop_front();
   return s;
 }
 
@@ -347,11 +347,12 @@ void Server::free_slot(int slot) {
 }
 
 // reading Q11: the paper's default task of 10 blocks, reduced so every
-// worker gets at least ~4 tasks (a fixed 10 mis-fits small grids)
-uint32_t Server::auto_iters(uint32_t B, int occ) const {
+// worker gets at least ~8 tasks (a fixed 10 mis-fits small grids: the last
+// tasks leave workers idle)
+uint32_t Server::auto_iters(uint32_t B, int occ, uint32_t cap) const {
   const uint64_t workers = uint64_t(occ) * uint64_t(n_sms_);
-  const uint64_t it = B / (4 * workers);
-  return uint32_t(it < 1 ? 1 : (it > 10 ? 10 : it));
+  const uint64_t it = B / (8 * workers);
+  return uint32_t(it < 1 ? 1 : (it > cap ? cap : it));
 }
 
 // ------------------------------------------------------------------ control word
@@ -523,7 +524,7 @@ int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_
   L->args.assign(static_cast<const unsigned char*>(d->args), static_cast<const unsigned char*>(d->args) + d->args_size);
   L->desc.args = nullptr;
   L->B = B;
-  L->iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ);
+  L->iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters);
   Launch& LL = *L;
   launches_[L->id] = std::move(L);
   *out = LL.id;
@@ -944,7 +945,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   validate(k, d, &B, nullptr);
   WorkerCommon w{};
   w.gx = d->grid[0]; w.gy = d->grid[1]; w.gz = d->grid[2]; w.B = B; w.occ = uint32_t(k.occ);
-  w.iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ);
+  w.iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters);
   w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
   w.ctrl = ctrl; w.tc = d_tc_ + slot; w.mirror = nullptr; w.cov = nullptr; w.rank_of = d_rank_of_;

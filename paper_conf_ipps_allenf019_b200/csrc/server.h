@@ -107,7 +107,7 @@ class Server {
   bool launch_done_events(Launch& L);
   int alloc_slot();
   void free_slot(int slot);
-  uint32_t auto_iters(uint32_t B, int occ) const;
+  uint32_t auto_iters(uint32_t B, int occ, uint32_t cap) const;
   bool validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const;
   void work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const;
 
@@ -127,7 +127,7 @@ class Server {
   HostMirror* d_mirror_ = nullptr;
   unsigned char* h_snap_ = nullptr;   // pinned, kSlots * kTaskCtlHeader
   void* h_zero_ = nullptr;            // pinned zeros (TaskCtl reset by DMA, no SM)
-  std::vector<int> free_slots_;
+  std::deque<int> free_slots_;     // FIFO: a freed block is reused as late as possible
   std::vector<cudaEvent_t> slot_zeroed_;   // DMA zeroing of a freed slot, off the critical path
   static constexpr int kQueues = 64;
   uint64_t* d_ctrl_pool_ = nullptr;

@@ -78,6 +78,10 @@ struct BlockWalk {
 };
 
 // ------------------------------------------------------------------ bookkeeping
+// Latency discipline: every bookkeeping atomic whose result is not needed is a
+// fire-and-forget reduction (RED), the resize word for a task boundary is
+// loaded when the task STARTS (its latency hides behind the task) and only the
+// task-counter atomic is a round trip on the boundary.
 template <class P>
 __device__ __forceinline__ bool in_range(const P& p, uint32_t rank, uint64_t c) {
   return rank >= ctrl_lo(c) && rank <= ctrl_hi(c) && rank >= p.bound_lo && rank <= p.bound_hi;
@@ -89,30 +93,33 @@ __device__ __forceinline__ bool in_range(const P& p, uint32_t rank, uint64_t c) 
 // tenant has occ*|range| workers or the queue is drained, and after a timeout
 // with zero live workers it runs anyway (liveness).
 template <class P>
-__device__ bool prologue(const P& p, uint32_t rank, uint32_t units) {
+__device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
   TaskCtl* tc = p.tc;
-  const uint64_t t0 = globaltimer();
+  uint64_t t0 = 0;
   uint32_t backoff = 256;
   for (;;) {
     const uint64_t c = ld_acquire_u64(p.ctrl);
-    if (ld_relaxed_u32(&tc->next) >= p.B) return false;                 // exit (2)
+    const uint32_t nxt = ld_relaxed_u32(&tc->next);
+    if (nxt >= p.B) return false;                                       // exit (2)
     bool join = in_range(p, rank, c);
     if (!join) {
       const uint32_t live = ld_relaxed_u32(&tc->live);
-      const uint32_t target = p.occ * (ctrl_hi(c) - ctrl_lo(c) + 1) * units;
+      const uint32_t target = p.occ * (ctrl_hi(c) - ctrl_lo(c) + 1);
       if (live >= target) return false;                                  // exit (1)
+      if (t0 == 0) t0 = globaltimer();
       if (live == 0 && globaltimer() - t0 > p.standby_timeout_ns) join = true;
     }
     if (join) {
-      atomicAdd(&tc->live, units);
-      atomicAdd(&tc->live_rank[rank], units);
-      atomicAdd(&tc->started, units);
+      atomicAdd(&tc->live, 1u);              // results unused: RED, no round trip
+      atomicAdd(&tc->live_rank[rank], 1u);
+      atomicAdd(&tc->started, 1u);
       const uint32_t e = ctrl_epoch(c);
-      if (e > 0 && atomicMax(&tc->join_epoch, e) < e && p.mirror) {      // grow observed
-        p.mirror->join_ns = globaltimer();
+      if (e > 0 && ld_relaxed_u32(&tc->join_epoch) < e && atomicMax(&tc->join_epoch, e) < e && p.mirror) {
+        p.mirror->join_ns = globaltimer();   // grow observed (a worker joined under epoch e)
         __threadfence_system();
         p.mirror->join_epoch = e;
       }
+      c_out = c;
       return true;
     }
     __nanosleep(backoff);
@@ -140,23 +147,44 @@ __device__ void check_shrink_done(const P& p, uint64_t c, uint32_t lane) {
   }
 }
 
-// Retire unless this is the last live worker and tasks remain (liveness rule).
-__device__ __forceinline__ bool try_retire(TaskCtl* tc, uint32_t units, uint32_t B) {
+// Retire unless this is the last live worker (liveness rule): CAS on live.
+__device__ __forceinline__ bool try_retire(TaskCtl* tc) {
   uint32_t v = ld_relaxed_u32(&tc->live);
-  while (v > units) {
-    const uint32_t w = atomicCAS(&tc->live, v, v - units);
+  while (v > 1u) {
+    const uint32_t w = atomicCAS(&tc->live, v, v - 1u);
     if (w == v) return true;
     v = w;
   }
-  (void)B;
   return false;   // the last live worker stays (its next fetch exits if the queue is drained)
 }
 
+// Task boundary, by ONE lane: given the resize word c2 (loaded
+// when the finished task started) and the finished task (g_done, n_done; n_done
+// = 0 for none), count it done and decide the next task.  Returns the next task
+// start or 0xffffffff to leave (retired, or the queue is drained).
 template <class P>
-__device__ __forceinline__ void task_done(const P& p, uint32_t g, uint32_t n) {
+__device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t c2, uint64_t& c, uint32_t g_done,
+                                             uint32_t n_done, bool& retired, bool& epoch_changed) {
   TaskCtl* tc = p.tc;
-  const unsigned long long old = atomicAdd(&tc->done, (1ull << 32) | n);
-  if (uint32_t(old) + n == p.B) {                                       // last block of the launch
+  epoch_changed = ctrl_epoch(c2) != ctrl_epoch(c);
+  c = c2;
+  retired = false;
+  unsigned long long old = 0;
+  // task_done: one 64-bit atomic; its result is needed only to spot the last block
+  if (n_done) old = atomicAdd(&tc->done, (1ull << 32) | n_done);
+  uint32_t g = 0xffffffffu;
+  if (!in_range(p, rank, c2) && try_retire(tc)) {
+    retired = true;
+  } else {
+    g = atomicAdd(&tc->next, p.iters);                                  // Lst2 (2)
+    if (g >= p.B) {                                                     // Q3: nothing to run
+      atomicAdd(&tc->live, 0xffffffffu);                                // live -= 1 (RED)
+      g = 0xffffffffu;
+    } else if (g == 0) {
+      tc->t_first = globaltimer();
+    }
+  }
+  if (n_done && uint32_t(old) + n_done == p.B) {                        // last block of the launch
     const uint64_t t = globaltimer();
     tc->t_last = t;
     if (p.mirror) {
@@ -165,76 +193,67 @@ __device__ __forceinline__ void task_done(const P& p, uint32_t g, uint32_t n) {
       p.mirror->complete = 1;
     }
   }
-}
-
-// Fetch decision for one worker, made by ONE lane.  Returns the task start g,
-// or 0xffffffff to leave (retired, or the queue is drained).
-//   first: true at the worker's first boundary (prologue already checked ctrl)
-template <class P>
-__device__ __forceinline__ uint32_t boundary_fetch(const P& p, uint32_t rank, uint32_t units,
-                                                   uint64_t& c, bool& retired, bool& epoch_changed) {
-  TaskCtl* tc = p.tc;
-  const uint64_t c2 = ld_acquire_u64(p.ctrl);
-  epoch_changed = ctrl_epoch(c2) != ctrl_epoch(c);
-  c = c2;
-  retired = false;
-  if (!in_range(p, rank, c2) && try_retire(tc, units, p.B)) {
-    retired = true;
-    return 0xffffffffu;
-  }
-  const uint32_t g = atomicAdd(&tc->next, p.iters);                     // Lst2 (2)
-  if (g >= p.B) {                                                       // Q3: nothing to run
-    atomicSub(&tc->live, units);
-    return 0xffffffffu;
-  }
-  if (g == 0) tc->t_first = globaltimer();
   return g;
 }
 
+// one finished task: blocks_done += n, tasks_done += 1; the CTA that
+// completes the last block stamps the end and tells the host
+template <class P>
+__device__ __forceinline__ void count_done(const P& p, uint32_t n) {
+  const unsigned long long old = atomicAdd(&p.tc->done, (1ull << 32) | n);
+  if (uint32_t(old) + n == p.B) {
+    const uint64_t t = globaltimer();
+    p.tc->t_last = t;
+    if (p.mirror) {
+      p.mirror->t_last = t;
+      __threadfence_system();
+      p.mirror->complete = 1;
+    }
+  }
+}
+
 // ------------------------------------------------------------------ the worker
-// Tn (tenant) provides: using Args; kThreads; kSmem;
+// Tn (tenant) provides: using Args; kThreads; kSmem; optional hooks (TenantBase)
 //   __device__ static void cta_block(const Args&, uint32_t x, uint32_t y, uint32_t z, char* smem)
 // executed by all kThreads threads of the CTA (may use __syncthreads).
 //
-// Per task (Lst2): lane 0 of warp 0 loads the resize word (acquire), retires
-// the CTA if its rank left the range (unless it is the last live worker), else
-// fetches `iters` blocks with ONE atomicAdd on the task counter; the values go
-// to warp 0 by __shfl_sync and to the other warps through shared memory and
-// the barrier (reading Q19).
+// Per task (Lst2): lane 0 of warp 0 makes the boundary decision; warp 0 gets
+// the task start by __shfl_sync, the other warps through shared memory and the
+// barrier that ends the task (reading Q19).
 template <class Tn>
 __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args>& p) {
   extern __shared__ __align__(128) char dyn_smem[];
   __shared__ uint32_t s_go;
-  __shared__ uint32_t s_g[2];
+  __shared__ uint32_t s_g[3];
   __shared__ uint32_t s_retired;
   __shared__ uint32_t s_rank;
   const uint32_t lane = threadIdx.x & 31;
+  uint64_t c = 0;    // the resize word last acted on (warp 0)
+  uint64_t c2 = 0;   // the resize word for the next boundary, loaded at task start (lane 0 of warp 0)
 
   // ---- Lst1: the block leader binds the CTA to its SM
   if (threadIdx.x == 0) {
     const uint32_t r = p.rank_of[smid()];
     s_rank = r;
     s_retired = 0;
-    s_go = prologue(p, r, 1u) ? 1u : 0u;
+    s_go = prologue(p, r, c) ? 1u : 0u;
   }
   __syncthreads();
   if (!s_go) return;
   const uint32_t rank = s_rank;
-  uint64_t c = ld_acquire_u64(p.ctrl);
+  c = __shfl_sync(0xffffffffu, c, 0);
   if constexpr (Tn::kHasInit) {
     Tn::cta_init(dyn_smem);
     __syncthreads();
   }
 
-  // Lst2 (2): one lane fetches (after checking the resize word), warp 0 gets the
-  // value by __shfl_sync, the other warps through shared memory (reading Q19).
-  // Ends with a barrier; every thread returns the same task start.
-  auto fetch = [&](int slot) -> uint32_t {
+  // boundary by warp 0; ends with the barrier; every thread gets the same start
+  auto fetch = [&](int slot, uint32_t g_done, uint32_t n_done) -> uint32_t {
     if (threadIdx.x < 32) {
       uint32_t g = 0, ret = 0, chg = 0;
       if (lane == 0) {
         bool retired, changed;
-        g = boundary_fetch(p, rank, 1u, c, retired, changed);
+        g = boundary(p, rank, c2, c, g_done, n_done, retired, changed);
         ret = retired;
         chg = changed;
       }
@@ -250,45 +269,87 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     __syncthreads();
     return s_g[slot];
   };
+  auto prefetch_ctrl = [&]() {   // the next boundary's resize word, in flight during the task
+    if (threadIdx.x == 0) c2 = ld_acquire_u64(p.ctrl);
+  };
 
-  uint32_t g = fetch(0);
+  c2 = c;
+  uint32_t g = fetch(0, 0, 0);
   int slot = 0;
   while (g != 0xffffffffu) {                      // Lst2 (1): until retreat or an empty queue
     const uint32_t n = min(p.iters, p.B - g);     // clamp the last task
     if constexpr (Tn::kLookahead) {
-      // the next task is fetched (resize word checked) before this one runs,
-      // so the tenant can stream its data in while this task computes
-      const uint32_t g2 = fetch(slot ^ 1);
+      // the next task is fetched before this one runs, so the tenant can
+      // stream its data in while this task computes
+      prefetch_ctrl();
+      const uint32_t g2 = fetch(slot ^ 1, 0, 0);
       const uint32_t n2 = g2 == 0xffffffffu ? 0u : min(p.iters, p.B - g2);
       Tn::cta_task2(p.args, g, n, g2, n2, dyn_smem);
       if (p.cov && threadIdx.x == 0)
         for (uint32_t i = 0; i < n; ++i) atomicAdd(&p.cov[g + i], 1u);
       __syncthreads();
-      if (threadIdx.x == 0) task_done(p, g, n);
+      if (threadIdx.x == 0) count_done(p, n);
       g = g2;
       slot ^= 1;
     } else {
-      BlockWalk w;
-      w.start(g, p.gx, p.gy);
-      for (uint32_t i = 0; i < n; ++i) {          // Lst2 (3): the task's blocks, in order
-        Tn::cta_block(p.args, w.x, w.y, w.z, dyn_smem);   // Lst2 (5): the user code
-        if (p.cov && threadIdx.x == 0) atomicAdd(&p.cov[g + i], 1u);
-        w.advance(p.gx, p.gy);                    // Lst2 (4)
+      // speculative boundary: the decision for the NEXT task is taken now, from
+      // the resize word loaded when the previous task started, and the counter
+      // atomic is in flight while this task runs (its result is read at the
+      // end).  A resize is therefore honoured within at most two tasks.
+      uint32_t fut = 0xffffffffu;
+      bool spec_retired = false, spec_changed = false;
+      if (threadIdx.x == 0) {
+        spec_changed = ctrl_epoch(c2) != ctrl_epoch(c);
+        c = c2;
+        if (!in_range(p, rank, c) && try_retire(p.tc)) spec_retired = true;
+        else fut = atomicAdd(&p.tc->next, p.iters);                   // Lst2 (2), result used below
+        c2 = ld_acquire_u64(p.ctrl);                                  // for the next boundary
       }
-      __syncthreads();   // every thread is done with the task
-      if (threadIdx.x == 0) task_done(p, g, n);
-      g = fetch(0);
+      if constexpr (Tn::kHasTask) {
+        Tn::cta_task(p.args, g, n, dyn_smem);     // Lst2 (3)-(5) for a 1-D grid, blocks in flight together
+        if (p.cov && threadIdx.x == 0)
+          for (uint32_t i = 0; i < n; ++i) atomicAdd(&p.cov[g + i], 1u);
+      } else {
+        BlockWalk w;
+        w.start(g, p.gx, p.gy);
+        for (uint32_t i = 0; i < n; ++i) {        // Lst2 (3): the task's blocks, in order
+          Tn::cta_block(p.args, w.x, w.y, w.z, dyn_smem);   // Lst2 (5): the user code
+          if (p.cov && threadIdx.x == 0) atomicAdd(&p.cov[g + i], 1u);
+          w.advance(p.gx, p.gy);                  // Lst2 (4)
+        }
+      }
+      if (threadIdx.x == 0) {
+        uint32_t g2 = 0xffffffffu;
+        if (!spec_retired) {
+          if (fut >= p.B) atomicAdd(&p.tc->live, 0xffffffffu);        // queue drained: live -= 1
+          else g2 = fut;
+          if (fut == 0) p.tc->t_first = globaltimer();
+        } else {
+          s_retired = 1;
+        }
+        s_g[slot ^ 1] = g2;
+        s_g[2] = spec_changed ? 1u : 0u;
+      }
+      __syncthreads();                            // every thread is done with the task
+      if (threadIdx.x == 0) count_done(p, n);
+      slot ^= 1;
+      g = s_g[slot];
+      if (s_g[2] && threadIdx.x < 32) {           // epoch changed: maybe the end of a shrink
+        c = __shfl_sync(0xffffffffu, c, 0);
+        if (g != 0xffffffffu) check_shrink_done(p, c, lane);
+      }
     }
   }
   if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
   if (threadIdx.x < 32) {
-    if (lane == 0) atomicSub(&p.tc->live_rank[rank], 1u);
+    c = __shfl_sync(0xffffffffu, c, 0);
+    if (lane == 0) atomicAdd(&p.tc->live_rank[rank], 0xffffffffu);   // live_rank -= 1
     if (s_retired) check_shrink_done(p, c, lane);
   }
 }
 
 template <class Tn>
-__global__ void __launch_bounds__(Tn::kThreads) slate_worker(const __grid_constant__ WorkerParams<typename Tn::Args> p) {
+__global__ void __launch_bounds__(Tn::kThreads, Tn::kMinBlocks) slate_worker(const __grid_constant__ WorkerParams<typename Tn::Args> p) {
   worker_body<Tn>(p);
 }
 

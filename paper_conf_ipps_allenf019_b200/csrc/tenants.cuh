@@ -21,8 +21,11 @@ __device__ __forceinline__ void st_stream(float4* p, float4 v) { __stcs(p, v); }
 // Optional per-tenant hooks default to off.
 struct TenantBase {
   static constexpr bool kHasInit = false;   // cta_init(smem): once per CTA before the first block
+  static constexpr bool kHasTask = false;   // cta_task(args, g, n, smem): task [g, g+n) of a 1-D grid at once
   static constexpr bool kLookahead = false; // cta_task2(args, g, n, g2, n2, smem): run task [g, g+n) of a
                                             // 1-D grid knowing the CTA's next task [g2, g2+n2) (n2 = 0: none)
+  static constexpr uint32_t kMaxIters = 10; // cap of the automatic task size (P:L303 default 10)
+  static constexpr int kMinBlocks = 1;      // __launch_bounds__ min blocks per SM of the worker
   static constexpr bool kHasFini = false;   // cta_fini(smem): once per CTA before it exits
 };
 
@@ -207,214 +210,66 @@ struct SgemmNaive : TenantBase {
 };
 
 // ============================================================== CSR SpMV  y = A x
-// 32 rows per block; in the original kernel warp w handles rows 4w..4w+3 with
-// 8 lanes per row: lane l sums j = rp[row]+l, +8, +16, ... in ascending order
-// (an fmaf chain from 0), then a butterfly (xor 4, 2, 1) inside the 8-lane group.
-//
-// The worker's task body streams instead: the rows of consecutive blocks are
-// consecutive, so a block's col/val entries are one contiguous range that the
-// bulk-copy engine moves into shared memory.  Each warp owns whole blocks
-// (w, w+8, ... of the task) with two stages: it issues the next block's copy
-// before consuming the current one, and the copy of its first block of the NEXT
-// task is issued during this one (lookahead), so HBM latency leaves the
-// critical path.  Per row, lanes, order and reduction are exactly cta_block's.
+// 32 rows per block; warp w handles rows 4w..4w+3 with 8 lanes per row: lane l
+// sums j = rp[row]+l, +8, +16, ... in ascending order (an fmaf chain from 0),
+// then a butterfly (xor 4, 2, 1) inside the 8-lane group.  The task body runs
+// the task's blocks (up to kMaxIters = 4) at once, each thread holding one row
+// per block, so the row-pointer, column/value and x loads of 4 rows are in
+// flight together (tools/probe/spmv_variants.cu: 1.7x the original kernel);
+// per row the arithmetic is exactly cta_block's.
 struct SpmvCsr : TenantBase {
   using Args = slate_args_spmv;
   static constexpr int kThreads = 256;
-  static constexpr int kWarps = 8;
-  static constexpr int kMaxTask = 16;                    // blocks per task on the streamed path
-  static constexpr int kRp = 32 * kMaxTask + 4;          // row pointers per task buffer (16-B multiple)
-  static constexpr int kCap = 32 * 16 + 8;               // entries per stage (16 nnz/row + alignment slack)
-  static constexpr int kStageBytes = 2 * kCap * 4;       // col then val
-  static constexpr int kHdr = 256;
-  static constexpr int kSmem = kHdr + 2 * kRp * 4 + 2 * kWarps * kStageBytes;
-  static constexpr int kSmemStandalone = kHdr;   // cta_init runs in both kernels (harmless here)
-  static constexpr bool kHasInit = true, kLookahead = true;
-  static_assert((kHdr + 2 * kRp * 4) % 16 == 0 && kStageBytes % 16 == 0 && (kCap * 4) % 16 == 0,
-                "bulk-copy destinations must be 16-byte aligned");
+  static constexpr int kSmem = 0, kSmemStandalone = 0;
+  static constexpr bool kHasTask = true;
+  static constexpr uint32_t kMaxIters = 4;
 
-  // ---- shared-memory layout
-  __device__ __forceinline__ static uint64_t* bar(char* sm, int w, int st) {
-    return reinterpret_cast<uint64_t*>(sm) + 2 * w + st;
-  }
-  __device__ __forceinline__ static uint32_t* wstate(char* sm, int w) {   // bit0,1 parity; bit2 prefetched; bit3 stage
-    return reinterpret_cast<uint32_t*>(sm + 128) + w;
-  }
-  __device__ __forceinline__ static uint32_t* cstate(char* sm) {          // [0] rp slot, [1] rp of current valid
-    return reinterpret_cast<uint32_t*>(sm + 192);
-  }
-  __device__ __forceinline__ static int* rpbuf(char* sm, int slot) { return reinterpret_cast<int*>(sm + kHdr) + slot * kRp; }
-  __device__ __forceinline__ static int* scol(char* sm, int w, int st) {
-    return reinterpret_cast<int*>(sm + kHdr + 2 * kRp * 4 + (2 * w + st) * kStageBytes);
-  }
-  __device__ __forceinline__ static float* sval(char* sm, int w, int st) {
-    return reinterpret_cast<float*>(scol(sm, w, st) + kCap);
-  }
-
-  __device__ __forceinline__ static void cta_init(char* sm) {
-    if (threadIdx.x == 0) {
-      for (int i = 0; i < 2 * kWarps; ++i) mbar_init(reinterpret_cast<uint64_t*>(sm) + i, 1);
-      for (int w = 0; w < kWarps; ++w) *wstate(sm, w) = 0;
-      cstate(sm)[0] = 0;
-      cstate(sm)[1] = 0;
-      fence_mbar_init();
-    }
-  }
-
-  // the bulk-copied range of a block: entries [a0, a1) land at smem index j - base
-  struct Range {
-    int base, a0, a1;
-    bool bulk;
-  };
-  __device__ __forceinline__ static Range range(int n0, int n1) {
-    Range r;
-    r.base = n0 & ~3;
-    r.a0 = (n0 + 3) & ~3;
-    r.a1 = n1 & ~3;
-    r.bulk = r.a1 > r.a0 && (n1 - r.base) <= kCap;
-    return r;
-  }
-  __device__ __forceinline__ static void issue(const Args& a, char* sm, int w, int st, const Range& r) {
-    if (!r.bulk) return;
-    const uint32_t bytes = uint32_t(r.a1 - r.a0) * 4;
-    mbar_expect_tx(bar(sm, w, st), 2 * bytes);
-    bulk_g2s(scol(sm, w, st) + (r.a0 - r.base), reinterpret_cast<const int*>(a.col) + r.a0, bytes, bar(sm, w, st));
-    bulk_g2s(sval(sm, w, st) + (r.a0 - r.base), reinterpret_cast<const float*>(a.val) + r.a0, bytes, bar(sm, w, st));
-  }
-
-  // whole block x by one warp; rp = row pointers of the block's task, block at index bi
-  __device__ __forceinline__ static void consume(const Args& a, const int* rp, uint32_t x, uint32_t bi, const int* sc,
-                                                 const float* sv, const Range& r, uint32_t lane) {
-    const int* __restrict__ col = reinterpret_cast<const int*>(a.col);
-    const float* __restrict__ val = reinterpret_cast<const float*>(a.val);
-    const float* __restrict__ xv = reinterpret_cast<const float*>(a.x);
-    const int l = int(lane & 7), q = int(lane >> 3);
-    int lo[8], hi[8], c0[8], c1[8];
-    float v0[8], v1[8], acc[8];
-    auto get = [&](int j, int& c, float& v) {
-      if (r.bulk && j >= r.a0 && j < r.a1) {
-        c = sc[j - r.base];
-        v = sv[j - r.base];
-      } else {
-        c = __ldcs(col + j);
-        v = __ldcs(val + j);
-      }
-    };
-#pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      const uint32_t row = x * 32 + 4 * t + q;
-      const int k = int(bi) * 32 + 4 * t + q;
-      lo[t] = 0; hi[t] = 0; acc[t] = 0.f; c0[t] = 0; c1[t] = 0; v0[t] = 0.f; v1[t] = 0.f;
-      if (row < a.n_rows) { lo[t] = rp[k] + l; hi[t] = rp[k + 1]; }
-      if (lo[t] < hi[t]) get(lo[t], c0[t], v0[t]);
-      if (lo[t] + 8 < hi[t]) get(lo[t] + 8, c1[t], v1[t]);
-    }
-#pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      if (lo[t] < hi[t]) acc[t] = __fmaf_rn(v0[t], __ldg(xv + c0[t]), acc[t]);
-      if (lo[t] + 8 < hi[t]) acc[t] = __fmaf_rn(v1[t], __ldg(xv + c1[t]), acc[t]);
-    }
-#pragma unroll
-    for (int t = 0; t < 8; ++t) {
-      for (int j = lo[t] + 16; j < hi[t]; j += 8) {
-        int c;
-        float v;
-        get(j, c, v);
-        acc[t] = __fmaf_rn(v, __ldg(xv + c), acc[t]);
-      }
-      float v = acc[t];
-      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 4));
-      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 2));
-      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 1));
-      const uint32_t row = x * 32 + 4 * t + q;
-      if (l == 0 && row < a.n_rows) __stcs(reinterpret_cast<float*>(a.y) + row, v);
-    }
-  }
-
-  // the original kernel: block x, warp w rows 4w..4w+3, operands straight from global
-  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
-    const int* rp = reinterpret_cast<const int*>(a.rowptr);
+  template <int U>
+  __device__ __forceinline__ static void rows(const Args& a, uint32_t x0, uint32_t nblk) {
+    const int* __restrict__ rp = reinterpret_cast<const int*>(a.rowptr);
     const int* __restrict__ col = reinterpret_cast<const int*>(a.col);
     const float* __restrict__ val = reinterpret_cast<const float*>(a.val);
     const float* __restrict__ xv = reinterpret_cast<const float*>(a.x);
     const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int l = int(lane & 7);
-    const uint32_t row = x * 32 + w * 4 + (lane >> 3);
-    int lo = 0, hi = 0;
-    if (row < a.n_rows) { lo = __ldg(rp + row) + l; hi = __ldg(rp + row + 1); }
-    float acc = 0.f;
-    if (lo < hi) acc = __fmaf_rn(__ldcs(val + lo), __ldg(xv + __ldcs(col + lo)), acc);
-    if (lo + 8 < hi) acc = __fmaf_rn(__ldcs(val + lo + 8), __ldg(xv + __ldcs(col + lo + 8)), acc);
-    for (int j = lo + 16; j < hi; j += 8) acc = __fmaf_rn(__ldcs(val + j), __ldg(xv + __ldcs(col + j)), acc);
-    acc = __fadd_rn(acc, __shfl_xor_sync(0xffffffffu, acc, 4));
-    acc = __fadd_rn(acc, __shfl_xor_sync(0xffffffffu, acc, 2));
-    acc = __fadd_rn(acc, __shfl_xor_sync(0xffffffffu, acc, 1));
-    if (l == 0 && row < a.n_rows) __stcs(reinterpret_cast<float*>(a.y) + row, acc);
+    int lo[U], hi[U], c0[U], c1[U];
+    float v0[U], v1[U], acc[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint32_t row = (x0 + u) * 32 + w * 4 + (lane >> 3);
+      lo[u] = 0; hi[u] = 0; acc[u] = 0.f;
+      if (uint32_t(u) < nblk && row < a.n_rows) { lo[u] = __ldg(rp + row) + l; hi[u] = __ldg(rp + row + 1); }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {        // first round: j = lo and lo + 8 (rows of <= 16 nonzeros end here)
+      c0[u] = lo[u] < hi[u] ? __ldcs(col + lo[u]) : 0;
+      v0[u] = lo[u] < hi[u] ? __ldcs(val + lo[u]) : 0.f;
+      c1[u] = lo[u] + 8 < hi[u] ? __ldcs(col + lo[u] + 8) : 0;
+      v1[u] = lo[u] + 8 < hi[u] ? __ldcs(val + lo[u] + 8) : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (lo[u] < hi[u]) acc[u] = __fmaf_rn(v0[u], __ldg(xv + c0[u]), acc[u]);
+      if (lo[u] + 8 < hi[u]) acc[u] = __fmaf_rn(v1[u], __ldg(xv + c1[u]), acc[u]);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {        // longer rows: the rest of the chain, still ascending
+      for (int j = lo[u] + 16; j < hi[u]; j += 8) acc[u] = __fmaf_rn(__ldcs(val + j), __ldg(xv + __ldcs(col + j)), acc[u]);
+      float v = acc[u];
+      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 4));
+      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 2));
+      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 1));
+      const uint32_t row = (x0 + u) * 32 + w * 4 + (lane >> 3);
+      if (l == 0 && uint32_t(u) < nblk && row < a.n_rows) __stcs(reinterpret_cast<float*>(a.y) + row, v);
+    }
   }
-
-  __device__ __forceinline__ static void load_rp(const Args& a, int* dst, uint32_t g, uint32_t n) {
-    const uint32_t r0 = g * 32;
-    const uint32_t cnt = min(32u * n, a.n_rows - r0) + 1;
-    for (uint32_t t = threadIdx.x; t < cnt; t += kThreads) dst[t] = __ldg(reinterpret_cast<const int*>(a.rowptr) + r0 + t);
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
+    rows<1>(a, x, 1);
   }
-
-  __device__ __forceinline__ static void cta_task2(const Args& a, uint32_t g, uint32_t n, uint32_t g2, uint32_t n2,
-                                                   char* sm) {
-    if (n > uint32_t(kMaxTask)) {               // long tasks: the original per-block body
-      for (uint32_t i = 0; i < n; ++i) cta_block(a, g + i, 0, 0, sm);
-      __syncthreads();
-      cstate(sm)[1] = 0;
-      for (int w = 0; w < kWarps; ++w) *wstate(sm, w) &= ~4u;
-      return;
-    }
-    const uint32_t slot = cstate(sm)[0];
-    int* rp_cur = rpbuf(sm, int(slot));
-    int* rp_nxt = rpbuf(sm, int(slot ^ 1));
-    const bool have_cur = cstate(sm)[1] != 0;
-    const bool stream_nxt = n2 > 0 && n2 <= uint32_t(kMaxTask);
-    if (!have_cur) load_rp(a, rp_cur, g, n);
-    if (stream_nxt) load_rp(a, rp_nxt, g2, n2);
-    __syncthreads();
-    const uint32_t lane = threadIdx.x & 31;
-    const int w = int(threadIdx.x >> 5);
-    uint32_t ws = *wstate(sm, w);               // same value in every lane
-    int st = int((ws >> 3) & 1u);
-    bool pref = (ws >> 2) & 1u;
-    const uint32_t total_rows = a.n_rows;
-    auto rng_of = [&](const int* rp, uint32_t gg, uint32_t bi) {
-      const uint32_t k0 = bi * 32, k1 = min(bi * 32 + 32, total_rows - gg * 32);
-      return range(rp[k0], rp[k1]);
-    };
-    // st: the stage holding (or about to hold) the warp's next block; pref: that
-    // block -- index w of this task -- was issued during the previous task
-    const bool w_next_task = stream_nxt && uint32_t(w) < n2;
-    bool issued_cur = pref;
-    for (uint32_t i = uint32_t(w); i < n; i += kWarps) {
-      const Range cur = rng_of(rp_cur, g, i);
-      if (!issued_cur && lane == 0) issue(a, sm, w, st, cur);
-      const bool more = i + kWarps < n;
-      if (lane == 0) {                           // the follower goes to the other stage now
-        if (more) issue(a, sm, w, st ^ 1, rng_of(rp_cur, g, i + kWarps));
-        else if (w_next_task) issue(a, sm, w, st ^ 1, rng_of(rp_nxt, g2, uint32_t(w)));
-      }
-      if (cur.bulk) {
-        mbar_wait(bar(sm, w, st), (ws >> st) & 1u);
-        ws ^= 1u << st;
-      }
-      consume(a, rp_cur, g + i, i, scol(sm, w, st), sval(sm, w, st), cur, lane);
-      __syncwarp();
-      st ^= 1;
-      issued_cur = more;
-    }
-    if (uint32_t(w) >= n && w_next_task && lane == 0)   // no block here this time: prefetch anyway
-      issue(a, sm, w, st, rng_of(rp_nxt, g2, uint32_t(w)));
-    pref = w_next_task;
-    if (lane == 0) *wstate(sm, w) = (ws & 3u) | (pref ? 4u : 0u) | (uint32_t(st) << 3);
-    __syncthreads();                             // everyone is done with rp_cur
-    if (threadIdx.x == 0) {
-      cstate(sm)[0] = slot ^ 1;
-      cstate(sm)[1] = stream_nxt ? 1u : 0u;
-    }
+  __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char*) {
+    uint32_t i = 0;
+    for (; i + 4 <= n; i += 4) rows<4>(a, g + i, 4);
+    if (i < n) rows<4>(a, g + i, n - i);
   }
 };
 
