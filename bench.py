@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="slate", choices=["slate", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-c3", action="store_true", help="skip the C3 (GEMM + copy) companion measurement")
     ap.add_argument("--cpu-sample-s", type=float, default=12.0, help="target seconds of oracle work for cpu_baseline")
     return ap.parse_args()
 
@@ -172,53 +173,78 @@ class Clocks:
 
 
 # ------------------------------------------------------------------ the GPU workload
-class Pair:
-    def __init__(self, S, dev):
-        import torch
-        from paper_conf_ipps_allenf019_b200 import inputs as I
-        self.S, self.torch = S, torch
-        rp, col, val, x = I.spmv_inputs(N_ROWS, I.seed_for(2, 0))
-        S_, X_, T_, r = I.bs_inputs(N_OPT, I.seed_for(2, 1))
-        sig = I.bs_sigmas(P_SCEN)
-        self.host = {"rp": rp, "col": col, "val": val, "x": x, "S": S_, "X": X_, "T": T_, "sig": sig}
-        self.pinned = {k: torch.from_numpy(v).pin_memory() for k, v in self.host.items()}
-        self.d = {k: v.to(dev) for k, v in self.pinned.items()}
-        self.d["y"] = torch.zeros(N_ROWS, device=dev)
-        self.d["call"] = torch.zeros(N_OPT, device=dev)
-        self.d["put"] = torch.zeros(N_OPT, device=dev)
-        self.out_pinned = {k: torch.empty(self.d[k].numel(), dtype=torch.float32).pin_memory()
-                           for k in ("y", "call", "put")}
-        self.nnz = int(rp[-1])
-        self.r = float(r)
-        self.flush_buf = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MB > L2
-        torch.cuda.synchronize()
-        d = self.d
-        self.spmv_args, self.spmv_grid = S.spmv_args(d["rp"], d["col"], d["val"], d["x"], d["y"])
-        self.bs_args, self.bs_grid = S.bs_args(d["S"], d["X"], d["T"], d["call"], d["put"], d["sig"], self.r)
-        self.h2d_bytes = sum(v.numel() * v.element_size() for v in self.pinned.values())
-        self.d2h_bytes = sum(v.numel() * v.element_size() for v in self.out_pinned.values())
-        # algorithmic work per launch
-        self.spmv_bytes = 8.0 * self.nnz + 4.0 * (N_ROWS + 1) + 4.0 * N_ROWS + 4.0 * N_ROWS
-        self.bs_bytes = 20.0 * N_OPT + 4.0 * P_SCEN
-        self.bs_flops = float(FP32_FLOPS_PER_OPTION_SCENARIO) * N_OPT * P_SCEN
+class Job:
+    """One tenant job: `reps` back-to-back launches of one kernel."""
 
-    def flush_l2(self):
-        self.flush_buf.fill_(1.0)
-        self.torch.cuda.synchronize()
-
-    def copy_in(self):
-        for k, v in self.pinned.items():
-            self.d[k].copy_(v, non_blocking=True)
-        self.torch.cuda.synchronize()
-
-    def copy_out(self):
-        for k, v in self.out_pinned.items():
-            v.copy_(self.d[k], non_blocking=True)
-        self.torch.cuda.synchronize()
+    def __init__(self, name, kind, args, grid, reps, bytes_, fp32, tc):
+        self.name, self.kind, self.args, self.grid, self.reps = name, kind, args, grid, reps
+        self.bytes, self.fp32, self.tc = bytes_, fp32, tc      # algorithmic work per launch
 
 
-def submit(sess, kernel, args, grid, reps, **kw):
-    return [sess.launch(kernel, args, grid, **kw) for _ in range(reps)]
+class Workload:
+    """A pair of jobs A (submitted first) and B (arrives `arrival_ms` later)."""
+
+    def __init__(self, name, a, b, keep, arrival_frac=0.0):
+        self.name, self.a, self.b, self._keep, self.arrival_frac = name, a, b, keep, arrival_frac
+        self.arrival_ms = 0.0
+
+
+def make_c2(S, dev):
+    import torch
+    from paper_conf_ipps_allenf019_b200 import inputs as I
+    rp, col, val, x = I.spmv_inputs(N_ROWS, I.seed_for(2, 0))
+    S_, X_, T_, r = I.bs_inputs(N_OPT, I.seed_for(2, 1))
+    sig = I.bs_sigmas(P_SCEN)
+    host = {"rp": rp, "col": col, "val": val, "x": x, "S": S_, "X": X_, "T": T_, "sig": sig}
+    pinned = {k: torch.from_numpy(v).pin_memory() for k, v in host.items()}
+    d = {k: v.to(dev) for k, v in pinned.items()}
+    d["y"] = torch.zeros(N_ROWS, device=dev)
+    d["call"] = torch.zeros(N_OPT, device=dev)
+    d["put"] = torch.zeros(N_OPT, device=dev)
+    torch.cuda.synchronize()
+    nnz = int(rp[-1])
+    spmv_args, spmv_grid = S.spmv_args(d["rp"], d["col"], d["val"], d["x"], d["y"])
+    bs_args, bs_grid = S.bs_args(d["S"], d["X"], d["T"], d["call"], d["put"], d["sig"], float(r))
+    bs = Job("blackscholes", S.KIND_BLACKSCHOLES, bs_args, bs_grid, R_BS, 20.0 * N_OPT + 4.0 * P_SCEN,
+             float(FP32_FLOPS_PER_OPTION_SCENARIO) * N_OPT * P_SCEN, 0.0)
+    sp = Job("spmv", S.KIND_SPMV_CSR, spmv_args, spmv_grid, R_SPMV,
+             8.0 * nnz + 4.0 * (N_ROWS + 1) + 4.0 * N_ROWS + 4.0 * N_ROWS, 2.0 * nnz, 0.0)
+    w = Workload("C2", bs, sp, d)
+    w.pinned = pinned
+    w.out_names = ("y", "call", "put")
+    w.out_pinned = {k: torch.empty(d[k].numel(), dtype=torch.float32).pin_memory() for k in w.out_names}
+    w.h2d_bytes = sum(v.numel() * v.element_size() for v in pinned.values())
+    w.d2h_bytes = sum(v.numel() * v.element_size() for v in w.out_pinned.values())
+    return w
+
+
+C3 = {"workload": "C3: tensor-core bf16 GEMM 8192^3 (tcgen05) co-run with STREAM copy 2^30 fp32 (4 GiB), copy "
+                  "arriving at 25% of the GEMM job (dynamic resize mid-run)",
+      "gemm_launches_per_job": int(os.environ.get("SLATE_C3_REPS", "1")),
+      "copy_launches_per_job": int(os.environ.get("SLATE_C3_REPS", "1"))}
+
+
+def make_c3(S, dev):
+    import torch
+    g = torch.Generator(device=dev)
+    g.manual_seed(20190520 + 300)
+    m = n = k = 8192
+    A = (torch.rand(m, k, device=dev, generator=g) * 2 - 1).to(torch.bfloat16)
+    B = (torch.rand(n, k, device=dev, generator=g) * 2 - 1).to(torch.bfloat16)
+    C = torch.zeros(m, n, device=dev)
+    cb = torch.rand(1 << 30, device=dev, generator=g)
+    ca = torch.empty(1 << 30, device=dev)
+    torch.cuda.synchronize()
+    gargs, ggrid = S.gemm_args(A.view(torch.int16), B.view(torch.int16), C)
+    cargs, cgrid = S.copy_args(ca, cb)
+    ge = Job("gemm_bf16", S.KIND_GEMM_BF16, gargs, ggrid, C3["gemm_launches_per_job"],
+             2.0 * (m * k + n * k) + 4.0 * m * n, 0.0, 2.0 * m * n * k)
+    cp = Job("copy", S.KIND_COPY, cargs, cgrid, C3["copy_launches_per_job"], 8.0 * (1 << 30), 0.0, 0.0)
+    return Workload("C3", ge, cp, (A, B, C, ca, cb), arrival_frac=0.25)
+
+
+def submit(sess, kernel, job, **kw):
+    return [sess.launch(kernel, job.args, job.grid, **kw) for _ in range(job.reps)]
 
 
 def collect(sess, ids):
@@ -234,31 +260,40 @@ def span(qs):
     return min(q["start_ms"] for q in qs), max(q["end_ms"] for q in qs)
 
 
-def run_schedule(name, pair, sA, sB, kA, kB):
-    """One pair-job under a schedule; A = Black-Scholes job, B = SpMV job.
-    Returns (makespan_ms, turnaround_A_ms, turnaround_B_ms, queries_A, queries_B)."""
-    S = pair.S
+def spin_ms(ms):
+    t0 = time.perf_counter()
+    while (time.perf_counter() - t0) * 1e3 < ms:
+        pass
+
+
+def run_schedule(name, w, sA, sB, kA, kB, S):
+    """One pair-job under a schedule.  Returns (makespan, turnaround_A, turnaround_B, qa, qb) in ms,
+    turnarounds measured from the first launch's start (B's arrival delay included)."""
+    a, b = w.a, w.b
     if name == "seq_cuda":          # vanilla CUDA: the two jobs back to back, original kernels
-        a = submit(sA, kA, pair.bs_args, pair.bs_grid, R_BS, mode=S.MODE_STANDALONE)
-        b = submit(sA, kB, pair.spmv_args, pair.spmv_grid, R_SPMV, mode=S.MODE_STANDALONE)
-        qa, qb = collect(sA, a), collect(sA, b)
+        ia = submit(sA, kA, a, mode=S.MODE_STANDALONE)
+        ib = submit(sA, kB, b, mode=S.MODE_STANDALONE)
+        qa, qb = collect(sA, ia), collect(sA, ib)
     elif name == "seq_slate":       # Slate workers on all SMs, back to back
-        a = submit(sA, kA, pair.bs_args, pair.bs_grid, R_BS, placement=S.PLACE_SOLO)
-        b = submit(sA, kB, pair.spmv_args, pair.spmv_grid, R_SPMV, placement=S.PLACE_SOLO)
-        qa, qb = collect(sA, a), collect(sA, b)
+        ia = submit(sA, kA, a, placement=S.PLACE_SOLO)
+        ib = submit(sA, kB, b, placement=S.PLACE_SOLO)
+        qa, qb = collect(sA, ia), collect(sA, ib)
     elif name == "streams":         # plain concurrent streams: hardware leftover policy
-        a = submit(sA, kA, pair.bs_args, pair.bs_grid, R_BS, mode=S.MODE_STANDALONE)
-        b = submit(sB, kB, pair.spmv_args, pair.spmv_grid, R_SPMV, mode=S.MODE_STANDALONE)
-        qa, qb = collect(sA, a), collect(sB, b)
+        ia = submit(sA, kA, a, mode=S.MODE_STANDALONE)
+        spin_ms(w.arrival_ms)
+        ib = submit(sB, kB, b, mode=S.MODE_STANDALONE)
+        qa, qb = collect(sA, ia), collect(sB, ib)
     elif name == "slate":           # Slate AUTO: selector + split + shrink on arrival + grow on completion
-        a = submit(sA, kA, pair.bs_args, pair.bs_grid, R_BS, placement=S.PLACE_AUTO)
-        b = submit(sB, kB, pair.spmv_args, pair.spmv_grid, R_SPMV, placement=S.PLACE_AUTO)
-        qa, qb = collect(sA, a), collect(sB, b)
-    elif name == "slate_forced":    # diagnostic: co-run regardless of Tab I, split from the T(s) curves;
-        n, s_b = pair.n_sms, pair.split   # the server shrinks A on B's arrival and grows the survivor
-        a = submit(sA, kA, pair.bs_args, pair.bs_grid, R_BS, placement=S.PLACE_AUTO)
-        b = submit(sB, kB, pair.spmv_args, pair.spmv_grid, R_SPMV, placement=S.PLACE_CORUN, sm=(n - s_b, n - 1))
-        qa, qb = collect(sA, a), collect(sB, b)
+        ia = submit(sA, kA, a, placement=S.PLACE_AUTO)
+        spin_ms(w.arrival_ms)
+        ib = submit(sB, kB, b, placement=S.PLACE_AUTO)
+        qa, qb = collect(sA, ia), collect(sB, ib)
+    elif name == "slate_forced":    # co-run regardless of Tab I, split from the T(s) curves
+        n, s_b = w.n_sms, w.split
+        ia = submit(sA, kA, a, placement=S.PLACE_AUTO)
+        spin_ms(w.arrival_ms)
+        ib = submit(sB, kB, b, placement=S.PLACE_CORUN, sm=(n - s_b, n - 1))
+        qa, qb = collect(sA, ia), collect(sB, ib)
     else:
         raise ValueError(name)
     a0, a1 = span(qa)
@@ -273,13 +308,120 @@ def stp_antt(solo, turn):
     return stp, antt
 
 
-def median_schedule(name, pair, sA, sB, kA, kB, reps):
+def flush_l2(buf):
+    buf.fill_(1.0)
+    import torch
+    torch.cuda.synchronize()
+
+
+def median_schedule(name, w, sA, sB, kA, kB, S, flush, reps):
     rs = []
     for _ in range(reps):
-        pair.flush_l2()
-        rs.append(run_schedule(name, pair, sA, sB, kA, kB))
+        flush_l2(flush)
+        rs.append(run_schedule(name, w, sA, sB, kA, kB, S))
     rs.sort(key=lambda r: r[0])
     return rs[len(rs) // 2]
+
+
+def prof_view(p):
+    return {"solo_ms": round(p["solo_ms"], 4), "hbm_gbps": round(p["hbm_gbps"], 1),
+            "fp32_gflops": round(p["fp32_gflops"], 1), "tc_tflops": round(p["tc_tflops"], 1),
+            "category": p["category_name"],
+            "curve": {str(s): round(t, 4) for s, t in zip(p["curve_sms"], p["curve_ms"])}}
+
+
+def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
+    """Profiles, baselines and (if `timed` is None) `steps` timed Slate co-run steps.
+    Returns a dict of results; `timed(callback)` lets the caller bracket the timed loop."""
+    info = sA.info()
+    kA, kB = sA.register_kernel(w.a.kind), sA.register_kernel(w.b.kind)
+    pa = sA.profile(kA, w.a.args, w.a.grid, S.PROF_CURVE)
+    pb = sA.profile(kB, w.b.args, w.b.grid, S.PROF_CURVE)
+    w.n_sms = info["num_sms"]
+    w.split, _ = S.choose_split(dict(zip(pa["curve_sms"], pa["curve_ms"])), dict(zip(pb["curve_sms"], pb["curve_ms"])),
+                                w.n_sms)
+    w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
+    base = {}
+    for name in ("seq_cuda", "seq_slate", "streams", "slate_forced"):
+        run_schedule(name, w, sA, sB, kA, kB, S)
+        base[name] = median_schedule(name, w, sA, sB, kA, kB, S, flush, 3)
+    solo_a = base["seq_cuda"][1]
+    solo_b = base["seq_cuda"][0] - base["seq_cuda"][1]
+    t_seq = base["seq_cuda"][0]
+    for _ in range(max(3, warmup)):
+        flush_l2(flush)
+        run_schedule("slate", w, sA, sB, kA, kB, S)
+
+    def loop():
+        out = []
+        for _ in range(steps):
+            flush_l2(flush)
+            out.append(run_schedule("slate", w, sA, sB, kA, kB, S))
+        return out
+
+    steps_out = timed(loop) if timed else loop()
+    med = sorted(steps_out, key=lambda r: r[0])[len(steps_out) // 2]
+
+    def summary(r):
+        mk, ta, tb = r[0], r[1], r[2]
+        # B's turnaround counts from its arrival
+        stp, antt = stp_antt([solo_a, solo_b], [ta, max(tb - w.arrival_ms, 1e-9)])
+        la = [q["end_ms"] - q["start_ms"] for q in r[3]]
+        lb = [q["end_ms"] - q["start_ms"] for q in r[4]]
+        return {"makespan_ms": round(mk, 3), "turnaround_%s_ms" % w.a.name: round(ta, 3),
+                "turnaround_%s_ms" % w.b.name: round(tb, 3), "gain_vs_seq_cuda": round(t_seq / mk, 4),
+                "stp": round(stp, 4), "antt": round(antt, 4),
+                "launch_ms_%s" % w.a.name: [round(x, 3) for x in la] if len(la) <= 8 else round(sum(la) / len(la), 4),
+                "launch_ms_%s" % w.b.name: [round(x, 3) for x in lb] if len(lb) <= 8 else round(sum(lb) / len(lb), 4)}
+
+    sched = {k: summary(v) for k, v in base.items()}
+    sched["slate_corun"] = summary(med)
+    qa, qb = med[3], med[4]
+    resize = [v for q in qa + qb for v in q["resize_us"]]
+    mk = med[0]
+    peak_hbm = float(peaks.get("hbm_gbs", 6650.0))
+    peak_fp32 = info["peak_fp32_gflops"] / 1e3
+    peak_tc = float(peaks.get("bf16_tflops_sustained", 1376.7))
+    jb = w.a.reps * w.a.bytes + w.b.reps * w.b.bytes
+    jf = w.a.reps * w.a.fp32 + w.b.reps * w.b.fp32
+    jt = w.a.reps * w.a.tc + w.b.reps * w.b.tc
+    util = {"U_HBM": round(jb / (mk * 1e-3) / 1e9 / peak_hbm, 4),
+            "U_FP32": round(jf / (mk * 1e-3) / 1e12 / peak_fp32, 4),
+            "U_TC": round(jt / (mk * 1e-3) / 1e12 / peak_tc, 4),
+            "hbm_gbps": round(jb / (mk * 1e-3) / 1e9, 1)}
+    util["U_sum"] = round(util["U_HBM"] + util["U_FP32"] + util["U_TC"], 4)
+    # roofline of the kernel with the largest summed launch time in the co-run
+    durs = {w.a.name: [q["end_ms"] - q["start_ms"] for q in qa], w.b.name: [q["end_ms"] - q["start_ms"] for q in qb]}
+    job = {w.a.name: w.a, w.b.name: w.b}
+    top = max(durs, key=lambda k: sum(durs[k]))
+    j, avg = job[top], sum(durs[top]) / len(durs[top])
+    kname = {"blackscholes": "BlackScholes", "spmv": "SpmvCsr", "gemm_bf16": "GemmBf16", "copy": "Copy"}[top]
+    if j.tc:
+        ach = j.tc / (avg * 1e-3) / 1e12
+        roof = {"kernel": "slate_worker<%s>" % kname, "bound": "tensor", "achieved": round(ach, 2), "peak": peak_tc,
+                "unit": "TFLOP/s", "frac": round(ach / peak_tc, 4), "peak_source": "MEASURED_PEAKS.json bf16_tflops_sustained"}
+    elif j.fp32 and j.fp32 / j.bytes > 1.0:
+        ach = j.fp32 / (avg * 1e-3) / 1e12
+        roof = {"kernel": "slate_worker<%s>" % kname, "bound": "alu", "achieved": round(ach, 3),
+                "peak": round(peak_fp32, 2), "unit": "TFLOP/s", "frac": round(ach / peak_fp32, 4),
+                "peak_source": "FP32 = 148 SMs x 128 lanes x 2 flop x 1.965 GHz (DESIGN.md §5)"}
+    else:
+        ach = j.bytes / (avg * 1e-3) / 1e9
+        roof = {"kernel": "slate_worker<%s>" % kname, "bound": "hbm", "achieved": round(ach, 1), "peak": peak_hbm,
+                "unit": "GB/s", "frac": round(ach / peak_hbm, 4), "peak_source": "MEASURED_PEAKS.json hbm_gbs"}
+    roof["avg_launch_ms"] = round(avg, 5)
+    roof["traffic"] = None
+    ncu_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(ncu_path):
+        roof["traffic"] = json.load(open(ncu_path)).get(roof["kernel"])
+    return {"steps": steps_out, "med": med, "t_seq": t_seq, "schedules": sched,
+            "gain_vs_sequential": round(t_seq / mk, 4), "gain_vs_slate_sequential": round(base["seq_slate"][0] / mk, 4),
+            "resize_us": {"n": len(resize), "p50": round(statistics.median(resize), 2) if resize else None,
+                          "p99": round(float(np.percentile(resize, 99)), 2) if resize else None,
+                          "max": round(max(resize), 2) if resize else None,
+                          "topups": sum(q["n_topups"] for q in qa + qb)},
+            "split_sms_b": w.split, "arrival_ms": round(w.arrival_ms, 3),
+            "utilisation": util, "profiles": {w.a.name: prof_view(pa), w.b.name: prof_view(pb)}, "roofline": roof}
 
 
 def run_slate(args, world, rank, local):
@@ -293,133 +435,80 @@ def run_slate(args, world, rank, local):
         peaks = json.load(open(pk_path))
         os.environ.setdefault("SLATE_PEAK_HBM_GBPS", str(peaks.get("hbm_gbs", 6650.0)))
         os.environ.setdefault("SLATE_PEAK_TC_TFLOPS", str(peaks.get("bf16_tflops", 1590.0)))
-    peak_hbm = float(peaks.get("hbm_gbs", 6650.0))
     sA, sB = S.Session(None, local), S.Session(None, local)
-    info = sA.info()
-    peak_fp32 = info["peak_fp32_gflops"] / 1e3   # TFLOP/s, from 148 SMs x 128 lanes x 2 x clock
-    pair = Pair(S, dev)
-    kA, kB = sA.register_kernel(S.KIND_BLACKSCHOLES), sA.register_kernel(S.KIND_SPMV_CSR)
-    # the profile table: solo T(s) curves that feed the selector and the split
-    prof_bs = sA.profile(kA, pair.bs_args, pair.bs_grid, S.PROF_CURVE)
-    prof_sp = sA.profile(kB, pair.spmv_args, pair.spmv_grid, S.PROF_CURVE)
-    pair.n_sms = info["num_sms"]
-    pair.split, _ = S.choose_split(dict(zip(prof_bs["curve_sms"], prof_bs["curve_ms"])),
-                                   dict(zip(prof_sp["curve_sms"], prof_sp["curve_ms"])), pair.n_sms)
+    flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MB > L2
 
-    # ---- baselines (each the median of 3 runs after one warm-up)
-    base = {}
-    for name in ("seq_cuda", "seq_slate", "streams", "slate_forced"):
-        run_schedule(name, pair, sA, sB, kA, kB)
-        base[name] = median_schedule(name, pair, sA, sB, kA, kB, 3)
-    # solo job times: each job alone on the GPU with the original kernels (the T_k of P:L99)
-    solo_a = base["seq_cuda"][1]
-    solo_b = base["seq_cuda"][0] - base["seq_cuda"][1]
-    t_seq = base["seq_cuda"][0]
+    # ---- C2, the headline (BASELINE configs[1]); its timed loop is the bench's timed region
+    w2 = make_c2(S, dev)
+    clocks = {}
 
-    # ---- the timed hot path: Slate co-run steps
-    for _ in range(max(3, args.warmup)):
-        pair.flush_l2()
-        run_schedule("slate", pair, sA, sB, kA, kB)
-    clocks = Clocks(local)
-    steps = []
-    barrier(world)
-    torch.cuda.synchronize()
-    for _ in range(args.steps):
-        pair.flush_l2()
-        steps.append(run_schedule("slate", pair, sA, sB, kA, kB))
-    torch.cuda.synchronize()
-    barrier(world)
-    clk = clocks.stop()
-    total_ms = sum(s[0] for s in steps)
+    def timed(loop):
+        clocks["c"] = Clocks(local)
+        barrier(world)
+        torch.cuda.synchronize()
+        out = loop()
+        torch.cuda.synchronize()
+        barrier(world)
+        clocks["r"] = clocks["c"].stop()
+        return out
+
+    r2 = evaluate(w2, S, sA, sB, flush, args.steps, args.warmup, peaks, timed)
+    total_ms = sum(s[0] for s in r2["steps"])
     total_ms_max = allmax(world, total_ms)
     value = world * args.steps / (total_ms_max / 1e3)
-    med = sorted(steps, key=lambda s: s[0])[len(steps) // 2]
-    makespan = med[0]
+    n_launch = sum(len(s[3]) + len(s[4]) + sum(q["n_topups"] for q in s[3] + s[4]) for s in r2["steps"])
 
     # ---- e2e: host buffers in, the same co-run through the public API, results out
+    kA, kB = sA.register_kernel(w2.a.kind), sA.register_kernel(w2.b.kind)
     e2e_times = []
     for i in range(args.steps + 1):
-        pair.flush_l2()
+        flush_l2(flush)
         t0 = time.perf_counter()
-        pair.copy_in()
-        run_schedule("slate", pair, sA, sB, kA, kB)
-        pair.copy_out()
+        for k, v in w2.pinned.items():
+            w2._keep[k].copy_(v, non_blocking=True)
+        torch.cuda.synchronize()
+        run_schedule("slate", w2, sA, sB, kA, kB, S)
+        for k in w2.out_names:
+            w2.out_pinned[k].copy_(w2._keep[k], non_blocking=True)
+        torch.cuda.synchronize()
         if i:
             e2e_times.append(time.perf_counter() - t0)
     e2e_s = allmax(world, statistics.median(e2e_times))
+    h2d_bytes, d2h_bytes = w2.h2d_bytes, w2.d2h_bytes
+    del w2
 
-    # ---- metrics
-    def sched_summary(r):
-        mk, ta, tb = r[0], r[1], r[2]
-        stp, antt = stp_antt([solo_a, solo_b], [ta, tb])
-        return {"makespan_ms": round(mk, 3), "turnaround_bs_ms": round(ta, 3), "turnaround_spmv_ms": round(tb, 3),
-                "gain_vs_seq_cuda": round(t_seq / mk, 4), "stp": round(stp, 4), "antt": round(antt, 4)}
-
-    schedules = {k: sched_summary(v) for k, v in base.items()}
-    schedules["slate_corun"] = sched_summary(med)
-    qa, qb = med[3], med[4]
-    # per-kernel durations in the co-run (CUDA events on the launching streams)
-    dur_bs = [q["end_ms"] - q["start_ms"] for q in qa]
-    dur_sp = [q["end_ms"] - q["start_ms"] for q in qb]
-    resize = [v for q in qa + qb for v in q["resize_us"]]
-    topups = sum(q["n_topups"] for q in qa + qb)
-    sum_bs, sum_sp = sum(dur_bs), sum(dur_sp)
-    if sum_bs >= sum_sp:
-        avg = sum_bs / len(dur_bs)
-        ach = pair.bs_flops / (avg * 1e-3) / 1e12
-        roof = {"kernel": "slate_worker<BlackScholes>", "bound": "alu", "achieved": round(ach, 3),
-                "peak": round(peak_fp32, 2), "unit": "TFLOP/s", "frac": round(ach / peak_fp32, 4),
-                "traffic": None, "avg_launch_ms": round(avg, 5),
-                "peak_source": "FP32 = 148 SMs x 128 lanes x 2 flop x 1.965 GHz (DESIGN.md §Roofline)"}
-    else:
-        avg = sum_sp / len(dur_sp)
-        ach = pair.spmv_bytes / (avg * 1e-3) / 1e9
-        roof = {"kernel": "slate_worker<SpmvCsr>", "bound": "hbm", "achieved": round(ach, 1), "peak": peak_hbm,
-                "unit": "GB/s", "frac": round(ach / peak_hbm, 4), "traffic": None, "avg_launch_ms": round(avg, 5),
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6650 GB/s"}
-    ncu_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(ncu_path):
-        tr = json.load(open(ncu_path)).get(roof["kernel"])
-        if tr:
-            roof["traffic"] = tr
-    job_bytes = R_BS * pair.bs_bytes + R_SPMV * pair.spmv_bytes
-    job_flops = R_BS * pair.bs_flops
-    util = {"U_HBM": round(job_bytes / (makespan * 1e-3) / 1e9 / peak_hbm, 4),
-            "U_FP32": round(job_flops / (makespan * 1e-3) / 1e12 / peak_fp32, 4),
-            "hbm_gbps": round(job_bytes / (makespan * 1e-3) / 1e9, 1),
-            "fp32_tflops": round(job_flops / (makespan * 1e-3) / 1e12, 3)}
-    util["U_HBM_plus_U_FP32"] = round(util["U_HBM"] + util["U_FP32"], 4)
+    # ---- C3 (configs[2]): the tensor-core + HBM pair with a resize mid-run
+    c3 = None
+    if not args.no_c3:
+        w3 = make_c3(S, dev)
+        r3 = evaluate(w3, S, sA, sB, flush, max(3, args.steps // 2), args.warmup, peaks)
+        c3 = {k: r3[k] for k in ("gain_vs_sequential", "gain_vs_slate_sequential", "schedules", "resize_us",
+                                 "split_sms_b", "arrival_ms", "utilisation", "profiles", "roofline")}
+        c3["config"] = C3
+        c3["stp"] = r3["schedules"]["slate_corun"]["stp"]
+        c3["antt"] = r3["schedules"]["slate_corun"]["antt"]
+        del w3
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         pair_s, sample = oracle_pair_seconds(args.cpu_sample_s)
         cpu = {"value": 1.0 / pair_s, "unit": "pair-jobs/s", "cores": 1, "kind": "oracle", "sample": sample}
 
-    def prof_view(p):
-        return {"solo_ms": round(p["solo_ms"], 4), "hbm_gbps": round(p["hbm_gbps"], 1),
-                "fp32_gflops": round(p["fp32_gflops"], 1), "category": p["category_name"],
-                "curve": {str(s): round(t, 4) for s, t in zip(p["curve_sms"], p["curve_ms"])}}
-
-    n_launch = sum(len(s[3]) + len(s[4]) for s in steps) + sum(q["n_topups"] for s in steps for q in s[3] + s[4])
     line = {
         "metric": METRIC, "value": round(value, 4), "unit": "pair-jobs/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(total_ms_max / args.steps, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic", "config": CONFIG,
-        "gain_vs_sequential": round(t_seq / makespan, 4),
-        "gain_vs_slate_sequential": round(base["seq_slate"][0] / makespan, 4),
-        "stp": schedules["slate_corun"]["stp"], "antt": schedules["slate_corun"]["antt"],
-        "schedules": schedules, "forced_split_sms_spmv": pair.split,
-        "resize_us": {"n": len(resize), "p50": round(statistics.median(resize), 2) if resize else None,
-                      "p99": round(float(np.percentile(resize, 99)), 2) if resize else None,
-                      "max": round(max(resize), 2) if resize else None, "topups": topups},
-        "corun_utilisation": util,
-        "profiles": {"blackscholes": prof_view(prof_bs), "spmv": prof_view(prof_sp)},
-        "roofline": roof,
-        "clocks": clk,
-        "e2e": {"value": round(world / e2e_s, 4), "unit": "pair-jobs/s", "h2d_bytes_per_step": pair.h2d_bytes,
-                "d2h_bytes_per_step": pair.d2h_bytes},
+        "gain_vs_sequential": r2["gain_vs_sequential"], "gain_vs_slate_sequential": r2["gain_vs_slate_sequential"],
+        "stp": r2["schedules"]["slate_corun"]["stp"], "antt": r2["schedules"]["slate_corun"]["antt"],
+        "schedules": r2["schedules"], "forced_split_sms_spmv": r2["split_sms_b"], "resize_us": r2["resize_us"],
+        "corun_utilisation": r2["utilisation"], "profiles": r2["profiles"], "roofline": r2["roofline"],
+        "clocks": clocks.get("r"),
+        "e2e": {"value": round(world / e2e_s, 4), "unit": "pair-jobs/s", "h2d_bytes_per_step": h2d_bytes,
+                "d2h_bytes_per_step": d2h_bytes},
         "gpu_launches": n_launch,
     }
+    if c3:
+        line["c3"] = c3
     if cpu:
         line["cpu_baseline"] = cpu
     if rank == 0:

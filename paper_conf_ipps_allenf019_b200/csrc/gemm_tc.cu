@@ -62,11 +62,14 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
+// operand panels are re-read by neighbouring tiles: keep them in L2 (evict-last)
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
   asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-          s_u32(dst)),
-      "l"(map), "r"(x), "r"(y), "r"(s_u32(bar))
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, "
+      "%3}], [%4], %5;" ::"r"(s_u32(dst)),
+      "l"(map), "r"(x), "r"(y), "r"(s_u32(bar)), "l"(pol)
       : "memory");
 }
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap* m) {
@@ -108,6 +111,20 @@ __device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
 }
 // instruction descriptor: D fp32, A bf16, B bf16, both K-major, N = 128, M = 128
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(BN >> 3) << 17) | (uint32_t(BM >> 4) << 24);
+
+// Original block b -> output tile (m, n): grouped rasterisation, kGroupM tile
+// rows per group swept column by column, so the ~148 tiles in flight share a
+// few A row panels and B column panels in L2 (a property of the tenant kernel:
+// standalone and slate use the same map; every tile is computed exactly once).
+constexpr uint32_t kGroupM = 8;
+__device__ __forceinline__ void tile_of(uint32_t b, uint32_t gx, uint32_t gy, uint32_t& m0, uint32_t& n0) {
+  const uint32_t per_group = kGroupM * gx;
+  const uint32_t first_m = (b / per_group) * kGroupM;
+  const uint32_t rows = min(gy - first_m, kGroupM);
+  const uint32_t r = b % per_group;
+  m0 = (first_m + r % rows) * BM;
+  n0 = (r / rows) * BN;
+}
 
 struct Smem {
   uint64_t full[kStages], empty[kStages];
@@ -198,21 +215,34 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
         } else {
           g = t == 0 ? blockIdx.y * gridDim.x + blockIdx.x : 0xffffffffu;
         }
-        const uint32_t j = t & 1, u = t >> 1;
-        mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
-        S.tileq[j] = g;
-        mbar_arrive(&S.tq_full[j]);
-        ++t;
-        if (g == 0xffffffffu) break;
-        const uint32_t m0 = (g / p.gx) * BM, n0 = (g % p.gx) * BN;
-        for (uint32_t kb = 0; kb < num_kb; ++kb, ++it) {
-          const uint32_t s = it % kStages, r = it / kStages;
-          mbar_wait(&S.empty[s], (r & 1) ^ 1);
-          char* sa = ring + s * kStageBytes;
-          char* sb = sa + BM * BK * 2;
-          mbar_expect_tx(&S.full[s], kStageBytes);
-          tma_load_2d(sa, &p.tma_a, int(kb * BK), int(m0), &S.full[s]);
-          tma_load_2d(sb, &p.tma_b, int(kb * BK), int(n0), &S.full[s]);
+        if (g == 0xffffffffu) {                          // sentinel: the other roles stop
+          const uint32_t j = t & 1, u = t >> 1;
+          mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
+          S.tileq[j] = g;
+          mbar_arrive(&S.tq_full[j]);
+          break;
+        }
+        // a task = n consecutive tiles (SLATE_ITERS), handed out one by one;
+        // bit 31 marks the last tile of the task (tasks_done counts tasks)
+        const uint32_t n = kSlate ? min(p.iters, p.B - g) : 1u;
+        for (uint32_t i = 0; i < n; ++i) {
+          const uint32_t tile = g + i;
+          const uint32_t j = t & 1, u = t >> 1;
+          mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
+          S.tileq[j] = tile | (i + 1 == n ? 0x80000000u : 0u);
+          mbar_arrive(&S.tq_full[j]);
+          ++t;
+          uint32_t m0, n0;
+          tile_of(tile, p.gx, p.gy, m0, n0);
+          for (uint32_t kb = 0; kb < num_kb; ++kb, ++it) {
+            const uint32_t s = it % kStages, r = it / kStages;
+            mbar_wait(&S.empty[s], (r & 1) ^ 1);
+            char* sa = ring + s * kStageBytes;
+            char* sb = sa + BM * BK * 2;
+            mbar_expect_tx(&S.full[s], kStageBytes);
+            tma_load_2d(sa, &p.tma_a, int(kb * BK), int(m0), &S.full[s]);
+            tma_load_2d(sb, &p.tma_b, int(kb * BK), int(n0), &S.full[s]);
+          }
         }
       }
     }
@@ -252,14 +282,17 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
     for (;;) {
       const uint32_t j = t & 1, u = t >> 1;
       mbar_wait(&S.tq_full[j], u & 1);
-      const uint32_t g = S.tileq[j];
+      const uint32_t entry = S.tileq[j];
       __syncwarp();
       if (lane == 0) mbar_arrive(&S.tq_empty[j]);
-      if (g == 0xffffffffu) break;
+      if (entry == 0xffffffffu) break;
+      const uint32_t g = entry & 0x7fffffffu;
+      const bool last_of_task = (entry >> 31) != 0;
       const uint32_t b = t & 1, v = t >> 1;
       mbar_wait(&S.tmem_full[b], v & 1);
       tc_fence_after();
-      const uint32_t m0 = (g / p.gx) * BM, n0 = (g % p.gx) * BN;
+      uint32_t m0, n0;
+      tile_of(g, p.gx, p.gy, m0, n0);
       const uint32_t row = m0 + ew * 32 + lane;
       float* crow = reinterpret_cast<float*>(p.args.C) + uint64_t(row) * p.args.n + n0;
 #pragma unroll 1
@@ -278,7 +311,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
         mbar_arrive(&S.tmem_empty[b]);
         if constexpr (kSlate) {
           if (p.cov) atomicAdd(&p.cov[g], 1u);
-          count_done(p, 1u);
+          count_done(p, 1u, last_of_task ? 1u : 0u);
         }
       }
       ++t;

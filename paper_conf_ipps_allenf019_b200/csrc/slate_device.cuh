@@ -199,8 +199,8 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
 // one finished task: blocks_done += n, tasks_done += 1; the CTA that
 // completes the last block stamps the end and tells the host
 template <class P>
-__device__ __forceinline__ void count_done(const P& p, uint32_t n) {
-  const unsigned long long old = atomicAdd(&p.tc->done, (1ull << 32) | n);
+__device__ __forceinline__ void count_done(const P& p, uint32_t n, uint32_t tasks = 1) {
+  const unsigned long long old = atomicAdd(&p.tc->done, (uint64_t(tasks) << 32) | n);
   if (uint32_t(old) + n == p.B) {
     const uint64_t t = globaltimer();
     p.tc->t_last = t;

@@ -27,6 +27,8 @@ CASES = {
     "bs": lambda: make_bs(1024 * 12 + 4 * 33 + 2, 108, n_scen=5),
     "stencil_float": lambda: make_stencil(8 * 37 + 3, 32 * 9 + 5, 109),
     "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
+    "gemm_int": lambda: make_gemm(256, 384, 512, 113, "int"),
+    "gemm_float": lambda: make_gemm(384, 256, 1024, 114),
 }
 
 
@@ -95,3 +97,24 @@ def test_auto_solo_path(sess):
     assert t.check(t.snapshot())[0]
     q = sess.query(lid)
     assert q["blocks_done"] == q["total_blocks"] and q["end_ms"] >= q["start_ms"] > 0
+
+
+def test_gemm_full_size_sampled(sess):
+    """bf16 GEMM 8192^3 (BASELINE config 3) in the bench's launch configuration:
+    slate == standalone bit for bit, exact counters, and 24 sampled 128x128
+    tiles against the fp64 oracle; integer inputs in [-2, 2] keep every partial
+    sum below 2^24, so those tiles must match exactly."""
+    import random
+    for mode in ("int", "float"):
+        t = make_gemm(8192, 8192, 8192, 115, mode)
+        k_std = sess.register_kernel(t.kind)
+        _, ref, _ = _run(sess, t, k_std, mode=S.MODE_STANDALONE, cov=False)
+        k = sess.register_kernel(t.kind, flags=S.KFLAG_COVERAGE)
+        lid, outs, cov = _run(sess, t, k, placement=S.PLACE_AUTO)
+        assert torch.equal(outs[0], ref[0])
+        q = sess.query(lid)
+        assert q["coverage_ok"] == 1 and q["blocks_done"] == 4096 and q["tasks_done"] == 4096
+        rng = random.Random(116)
+        tiles = [(0, 0), (63, 63)] + [(rng.randrange(64), rng.randrange(64)) for _ in range(22)]
+        ok, err = t.check(outs, rows=tiles)
+        assert ok, (mode, err)

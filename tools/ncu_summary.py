@@ -32,9 +32,9 @@ KEYS = {
     "lts__t_sectors_op_atom.sum": "l2_atom_sectors",
     "smsp__inst_executed.sum": "inst_executed",
 }
-UNIT = {"dram_read": {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9},
-        "dram_write": {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9},
-        "duration_us": {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3}}
+B = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9}
+UNIT = {"dram_read": B, "dram_write": B,
+        "duration_us": {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "ns": 1e-3, "us": 1.0, "ms": 1e3}}
 
 
 def main(rep, out):
