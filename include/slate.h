@@ -267,6 +267,17 @@ typedef struct {
 /* Counters and timing of a launch (copied out).  Errors: ENOTFOUND. */
 slate_status slate_query(slate_session* s, slate_launch_id l, slate_launch_info* out);
 
+/* ------------------------------------------------------------------ server */
+/* Run a Slate server for CUDA device `device` on the calling thread (the body
+ * of the `slated` daemon): creates the single CUDA context every client's
+ * kernels run in, publishes the POSIX shared-memory endpoint (e.g.
+ * "/slate-gpu0"; replaced if stale), gives every attaching client session its
+ * own server thread and queue, and returns after SIGINT/SIGTERM, when
+ * it unlinks the endpoint.  flags: reserved, 0.
+ * Errors: EINVAL (endpoint must start with '/'), ECUDA (no usable device),
+ * EIPC (shared memory could not be created). */
+slate_status slate_serve(const char* endpoint, int device, uint32_t flags);
+
 /* ------------------------------------------------------------------ strings */
 const char* slate_status_string(slate_status st);     /* static string */
 const char* slate_last_error(slate_session* s);       /* session-owned, valid until the next call */

@@ -73,8 +73,8 @@ def build(force=False, verbose=False):
             raise RuntimeError("link failed:\n%s\n%s%s" % (" ".join(cmd), r.stdout, r.stderr))
     daemon_src = os.path.join(CSRC, "slated.cpp")
     if os.path.exists(daemon_src) and (force or _stale(DAEMON, [daemon_src, LIB] + hdrs)):
-        cmd = [NVCC] + ARCH + FLAGS + [daemon_src, "-o", DAEMON, "-L", PKG, "-lslate",
-                                       "-Xlinker", "-rpath=$ORIGIN/..", "-lpthread", "-lrt"]
+        cmd = ["g++", "-O2", "-std=c++17", "-I", os.path.join(ROOT, "include"), daemon_src, "-o", DAEMON,
+               "-L", PKG, "-lslate", "-Wl,-rpath,$ORIGIN/..", "-lpthread", "-lrt"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError("daemon build failed:\n%s\n%s%s" % (" ".join(cmd), r.stdout, r.stderr))

@@ -8,6 +8,7 @@
 #include <string>
 #include <vector>
 
+#include "capi_internal.h"
 #include "ipc.h"
 #include "server.h"
 
@@ -24,11 +25,11 @@ struct slate_session {
   uint64_t next_share = 1;
 };
 
-namespace {
-std::mutex g_servers_mu;
-std::map<int, Server*> g_servers;   // in-process servers live until process exit
+namespace slate {
+static std::mutex g_servers_mu;
+static std::map<int, Server*> g_servers;   // in-process servers live until process exit
 
-Server* local_server(int device, std::string* err, int* rc) {
+Server* get_local_server(int device, std::string* err, int* rc) {
   std::lock_guard<std::mutex> g(g_servers_mu);
   auto it = g_servers.find(device);
   if (it != g_servers.end()) return it->second;
@@ -41,7 +42,9 @@ Server* local_server(int device, std::string* err, int* rc) {
   g_servers[device] = s;
   return s;
 }
+}  // namespace slate
 
+namespace {
 slate_status fail(slate_session* s, slate_status rc, const std::string& msg) {
   if (s) s->last_error = msg;
   return rc;
@@ -76,7 +79,7 @@ slate_status slate_attach(const char* endpoint, int device, slate_session** out)
   int rc = SLATE_OK;
   if (endpoint == nullptr) {
     if (device < 0) return SLATE_EINVAL;
-    s->srv = local_server(device, &err, &rc);
+    s->srv = slate::get_local_server(device, &err, &rc);
     if (!s->srv) return rc;
     s->queue = s->srv->open_queue();
     if (!s->queue) return SLATE_ENOMEM;

@@ -1,0 +1,297 @@
+// serve.cu -- the `slated` server loop (slate_serve): one CUDA context per GPU
+// for every client process (P:L135 context funnelling), one CPU thread per
+// session, commands over the shared-memory slots of ipc.h, device
+// buffers imported once per allocation through CUDA IPC and every pointer
+// argument rewritten to the server's mapping.
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <thread>
+#include <vector>
+
+#include <fcntl.h>
+#include <signal.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include "capi_internal.h"
+#include "ipc.h"
+#include "server.h"
+
+namespace slate {
+namespace {
+
+volatile sig_atomic_t g_stop = 0;
+const bool g_debug = std::getenv("SLATE_DEBUG") != nullptr;
+#define DBG(...) do { if (g_debug) { std::fprintf(stderr, __VA_ARGS__); std::fflush(stderr); } } while (0)
+void on_signal(int) { g_stop = 1; }
+
+// server-wide cache of opened IPC allocations (a handle can be opened once per context)
+struct Opened {
+  void* ptr;
+  int refs;
+};
+std::mutex g_ipc_mu;
+std::map<std::string, Opened> g_ipc;
+
+struct Import {
+  uint64_t id, client_base, size;
+  char* server_base;
+  std::string key;
+};
+
+class Session {
+ public:
+  Session(Server* srv, Slot* slot, int device) : srv_(srv), slot_(slot), device_(device) {}
+  void run();
+
+ private:
+  int handle(const Request& rq, Response& rs);
+  bool translate(uint64_t& p, std::string* err) const;
+  void release_imports();
+  Server* srv_;
+  Slot* slot_;
+  int device_;
+  uint32_t queue_ = 0;
+  std::vector<Import> imports_;
+  uint64_t next_import_ = 1;
+};
+
+bool Session::translate(uint64_t& p, std::string* err) const {
+  if (p == 0) return true;
+  for (const Import& im : imports_)
+    if (p >= im.client_base && p < im.client_base + im.size) {
+      p = reinterpret_cast<uint64_t>(im.server_base) + (p - im.client_base);
+      return true;
+    }
+  if (err) *err = "device pointer outside every shared buffer (slate_share_buffer it first)";
+  return false;
+}
+
+void Session::release_imports() {
+  std::lock_guard<std::mutex> g(g_ipc_mu);
+  for (const Import& im : imports_) {
+    auto it = g_ipc.find(im.key);
+    if (it != g_ipc.end() && --it->second.refs == 0) {
+      cudaIpcCloseMemHandle(it->second.ptr);
+      g_ipc.erase(it);
+    }
+  }
+  imports_.clear();
+}
+
+int Session::handle(const Request& rq, Response& rs) {
+  std::string err;
+  int rc = SLATE_OK;
+  DBG("slated[q%u]: cmd %u id %llu\n", queue_, rq.cmd, (unsigned long long)rq.id);
+  switch (rq.cmd) {
+    case CMD_INFO:
+      rs.info = srv_->info();
+      rs.info.server_pid = uint64_t(getpid());
+      break;
+    case CMD_SHARE: {
+      std::string key(reinterpret_cast<const char*>(&rq.handle), sizeof(rq.handle));
+      void* ptr = nullptr;
+      {
+        std::lock_guard<std::mutex> g(g_ipc_mu);
+        auto it = g_ipc.find(key);
+        if (it != g_ipc.end()) {
+          it->second.refs += 1;
+          ptr = it->second.ptr;
+        } else {
+          const cudaError_t e = cudaIpcOpenMemHandle(&ptr, rq.handle, cudaIpcMemLazyEnablePeerAccess);
+          if (e != cudaSuccess) {
+            cudaGetLastError();
+            err = std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e);
+            rc = SLATE_EIPC;
+            break;
+          }
+          g_ipc[key] = {ptr, 1};
+        }
+      }
+      imports_.push_back({next_import_, rq.alloc_base, rq.alloc_size, static_cast<char*>(ptr), key});
+      rs.out = next_import_++;
+      break;
+    }
+    case CMD_UNSHARE: {
+      rc = SLATE_ENOTFOUND;
+      for (size_t i = 0; i < imports_.size(); ++i)
+        if (imports_[i].id == rq.id) {
+          std::lock_guard<std::mutex> g(g_ipc_mu);
+          auto it = g_ipc.find(imports_[i].key);
+          if (it != g_ipc.end() && --it->second.refs == 0) {
+            cudaIpcCloseMemHandle(it->second.ptr);
+            g_ipc.erase(it);
+          }
+          imports_.erase(imports_.begin() + long(i));
+          rc = SLATE_OK;
+          break;
+        }
+      break;
+    }
+    case CMD_REGISTER:
+      rc = srv_->register_kernel(&rq.kdesc, &rs.out, &err);
+      break;
+    case CMD_LAUNCH:
+    case CMD_PROFILE: {
+      // rewrite every pointer argument into the server's address space
+      unsigned char args[kMaxArgs];
+      std::memcpy(args, rq.args, sizeof(args));
+      slate_launch_desc d = rq.ldesc;
+      d.args = args;
+      uint32_t kind = 0;
+      if (!srv_->kernel_kind(rq.id, &kind)) {
+        rc = SLATE_ENOTFOUND;
+        err = "unknown kernel";
+        break;
+      }
+      const size_t* offs;
+      const int nf = pointer_fields(kind, &offs);
+      bool ok = d.args_size <= sizeof(args);
+      for (int i = 0; ok && i < nf; ++i) {
+        uint64_t p;
+        std::memcpy(&p, args + offs[i], 8);
+        ok = translate(p, &err);
+        std::memcpy(args + offs[i], &p, 8);
+      }
+      if (ok) ok = translate(d.coverage, &err);
+      if (!ok) {
+        rc = SLATE_EINVAL;
+        break;
+      }
+      if (rq.cmd == CMD_LAUNCH) rc = srv_->launch(queue_, rq.id, &d, &rs.out, &err);
+      else rc = srv_->profile(rq.id, &d, rq.flags, &rs.prof, &err);
+      break;
+    }
+    case CMD_RESIZE:
+      rc = srv_->resize(queue_, rq.id, rq.lo, rq.hi, &err);
+      break;
+    case CMD_SYNC:
+      rc = srv_->sync(queue_, rq.id, rq.timeout_us, &err);
+      break;
+    case CMD_QUERY:
+      rc = srv_->query(rq.id, &rs.linfo, &err);
+      break;
+    default:
+      rc = SLATE_EINVAL;
+      err = "unknown command";
+  }
+  rs.status = rc;
+  DBG("slated[q%u]: cmd %u -> %d %s\n", queue_, rq.cmd, rc, err.c_str());
+  std::strncpy(rs.err, err.c_str(), sizeof(rs.err) - 1);
+  rs.err[sizeof(rs.err) - 1] = 0;
+  return rc;
+}
+
+void Session::run() {
+  cudaSetDevice(device_);
+  queue_ = srv_->open_queue();
+  DBG("slated: session for pid %llu -> queue %u\n", (unsigned long long)slot_->client_pid, queue_);
+  uint64_t last = slot_->req_seq.load();
+  slot_->resp_seq.store(last);
+  slot_->state.store(queue_ ? SLOT_ACTIVE : SLOT_CLOSING, std::memory_order_release);
+  auto idle_since = std::chrono::steady_clock::now();
+  auto last_check = idle_since;
+  bool detached = false;
+  while (!g_stop && queue_) {
+    const uint64_t seq = slot_->req_seq.load(std::memory_order_acquire);
+    if (seq != last) {
+      Request rq;
+      std::memcpy(&rq, &slot_->req, sizeof(Request));
+      Response rs;
+      std::memset(&rs, 0, sizeof(rs));
+      if (rq.cmd == CMD_DETACH) {
+        std::string err;
+        rs.status = srv_->close_queue(queue_, 60000000, &err);
+        release_imports();
+        detached = true;
+      } else {
+        handle(rq, rs);
+      }
+      std::memcpy(&slot_->resp, &rs, sizeof(Response));
+      last = seq;
+      slot_->resp_seq.store(seq, std::memory_order_release);
+      idle_since = std::chrono::steady_clock::now();
+      if (detached) break;
+      continue;
+    }
+    const auto now = std::chrono::steady_clock::now();
+    if (now - last_check > std::chrono::milliseconds(100)) {   // client gone: clean up its session
+      last_check = now;
+      if (kill(pid_t(slot_->client_pid), 0) != 0) break;
+    }
+    if (now - idle_since < std::chrono::microseconds(200)) std::this_thread::yield();
+    else std::this_thread::sleep_for(std::chrono::microseconds(20));
+  }
+  if (!detached && queue_) {
+    std::string err;
+    srv_->close_queue(queue_, 60000000, &err);
+    release_imports();
+  }
+  if (detached) {   // the client is reading its DETACH response: wait for its ack (or its exit)
+    const auto t0 = std::chrono::steady_clock::now();
+    while (!slot_->ack.load(std::memory_order_acquire) && kill(pid_t(slot_->client_pid), 0) == 0 &&
+           std::chrono::steady_clock::now() - t0 < std::chrono::seconds(5))
+      std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
+  DBG("slated: session of pid %llu closed (queue %u)\n", (unsigned long long)slot_->client_pid, queue_);
+  // sequence numbers are never reset: the next client starts from the current value
+  slot_->client_pid = 0;
+  slot_->state.store(SLOT_FREE, std::memory_order_release);
+}
+
+}  // namespace
+}  // namespace slate
+
+extern "C" slate_status slate_serve(const char* endpoint, int device, uint32_t flags) {
+  using namespace slate;
+  (void)flags;
+  if (!endpoint || endpoint[0] != '/') return SLATE_EINVAL;
+  std::string err;
+  int rc = SLATE_OK;
+  Server* srv = get_local_server(device, &err, &rc);
+  if (!srv) {
+    fprintf(stderr, "slated: %s\n", err.c_str());
+    return rc;
+  }
+  shm_unlink(endpoint);
+  const int fd = shm_open(endpoint, O_CREAT | O_RDWR | O_EXCL, 0666);
+  if (fd < 0 || ftruncate(fd, sizeof(ShmLayout)) != 0) return SLATE_EIPC;
+  void* p = mmap(nullptr, sizeof(ShmLayout), PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  if (p == MAP_FAILED) return SLATE_EIPC;
+  std::memset(p, 0, sizeof(ShmLayout));
+  ShmLayout* shm = new (p) ShmLayout();
+  shm->hdr.magic = kShmMagic;
+  shm->hdr.version = kShmVersion;
+  shm->hdr.nslots = kSlots;
+  shm->hdr.server_pid = uint64_t(getpid());
+  shm->hdr.info = srv->info();
+  shm->hdr.info.server_pid = uint64_t(getpid());
+  signal(SIGINT, on_signal);
+  signal(SIGTERM, on_signal);
+  shm->hdr.alive.store(1, std::memory_order_release);
+  fprintf(stderr, "slated: serving %s on device %d (%u SMs)\n", endpoint, device, srv->info().num_sms);
+  std::vector<std::thread> threads;
+  while (!g_stop) {
+    for (int i = 0; i < kSlots; ++i) {
+      Slot& s = shm->slots[i];
+      if (s.state.load(std::memory_order_acquire) == SLOT_CLAIMED && s.client_pid) {
+        s.state.store(SLOT_CLOSING);   // owned by the watcher until the session thread opens it
+        DBG("slated: slot %d claimed by pid %llu\n", i, (unsigned long long)s.client_pid);
+        threads.emplace_back([srv, &s, device] { Session(srv, &s, device).run(); });
+      }
+    }
+    std::this_thread::sleep_for(std::chrono::microseconds(200));
+  }
+  shm->hdr.alive.store(0);
+  for (auto& t : threads) t.join();
+  munmap(p, sizeof(ShmLayout));
+  close(fd);
+  shm_unlink(endpoint);
+  return SLATE_OK;
+}

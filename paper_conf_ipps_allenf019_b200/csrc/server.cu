@@ -170,6 +170,14 @@ int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
 }
 
 // ------------------------------------------------------------------ kernels
+bool Server::kernel_kind(uint64_t k, uint32_t* kind) const {
+  std::lock_guard<std::mutex> g(mu_);
+  auto it = kernels_.find(k);
+  if (it == kernels_.end()) return false;
+  *kind = it->second->desc.kind;
+  return true;
+}
+
 int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err) {
   if (!d || !out || d->abi_version != SLATE_ABI_VERSION) {
     if (err) *err = "bad kernel descriptor";

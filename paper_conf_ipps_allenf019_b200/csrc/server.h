@@ -86,6 +86,7 @@ class Server {
   int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);
+  bool kernel_kind(uint64_t k, uint32_t* kind) const;
 
  private:
   // all private helpers are called with mu_ held

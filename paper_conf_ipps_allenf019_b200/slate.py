@@ -129,6 +129,7 @@ for _name, _args in [
     ("slate_sync", [ctypes.c_void_p, c_u64, c_i64]),
     ("slate_profile", [ctypes.c_void_p, c_u64, _P(LaunchDesc), c_u32, _P(Profile)]),
     ("slate_query", [ctypes.c_void_p, c_u64, _P(LaunchInfo)]),
+    ("slate_serve", [ctypes.c_char_p, ctypes.c_int, c_u32]),
 ]:
     getattr(_lib, _name).restype = c_i32
     getattr(_lib, _name).argtypes = _args
@@ -144,7 +145,8 @@ _lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c
 EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffer", "slate_unshare_buffer",
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
-            "slate_choose_split"]
+            "slate_choose_split", "slate_serve"]
+DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
 def status_string(st):
@@ -198,6 +200,9 @@ class Session:
         nb = nbytes if nbytes is not None else t.numel() * t.element_size()
         self._check(_lib.slate_share_buffer(self._h, _ptr(t), nb, ctypes.byref(h)), "slate_share_buffer")
         return h.value
+
+    def share_tensors(self, *tensors):
+        return [self.share_buffer(t) for t in tensors]
 
     def unshare_buffer(self, handle):
         self._check(_lib.slate_unshare_buffer(self._h, handle), "slate_unshare_buffer")
