@@ -65,7 +65,8 @@ def dist_init(args):
     if world > 1:
         import torch.distributed as dist
         import torch
-        torch.cuda.set_device(local)
+        if torch.cuda.is_available():
+            torch.cuda.set_device(local)
         dist.init_process_group("nccl" if torch.cuda.is_available() else "gloo")
     return world, rank, local
 
@@ -77,13 +78,20 @@ def barrier(world):
 
 
 def allmax(world, x):
+    """Max over ranks (the timed region is the slowest rank's, contract)."""
     if world == 1:
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([float(x)], device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([float(x)], device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def aggregate(world, steps, total_ms_per_rank_max):
+    """Whole-job throughput: pair-jobs of every rank / the slowest rank's device time."""
+    return world * steps / (total_ms_per_rank_max / 1e3)
 
 
 # ------------------------------------------------------------------ CPU oracle (reference / cpu_baseline)
@@ -455,7 +463,7 @@ def run_slate(args, world, rank, local):
     r2 = evaluate(w2, S, sA, sB, flush, args.steps, args.warmup, peaks, timed)
     total_ms = sum(s[0] for s in r2["steps"])
     total_ms_max = allmax(world, total_ms)
-    value = world * args.steps / (total_ms_max / 1e3)
+    value = aggregate(world, args.steps, total_ms_max)
     n_launch = sum(len(s[3]) + len(s[4]) + sum(q["n_topups"] for q in s[3] + s[4]) for s in r2["steps"])
 
     # ---- e2e: host buffers in, the same co-run through the public API, results out

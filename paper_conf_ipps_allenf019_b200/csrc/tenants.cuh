@@ -75,6 +75,7 @@ __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_
 struct Triad : TenantBase {
   using Args = slate_args_triad;
   static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 8;       // 32 registers, no spill: 64 warps/SM for HBM latency
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
@@ -203,6 +204,7 @@ __device__ __forceinline__ uint32_t* Copy::state(char* smem) { return reinterpre
 struct SgemmNaive : TenantBase {
   using Args = slate_args_sgemm;
   static constexpr int kThreads = 256;        // 16 x 16
+  static constexpr int kMinBlocks = 8;       // 32 registers, no spill (the worker logic alone pushed it to 64)
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t y, uint32_t, char*) {
@@ -228,6 +230,7 @@ struct SgemmNaive : TenantBase {
 struct SpmvCsr : TenantBase {
   using Args = slate_args_spmv;
   static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 6;       // 40 registers (8-B spill): latency-bound, occupancy is throughput
   static constexpr int kSmem = 0, kSmemStandalone = 0;
   static constexpr bool kHasTask = true;
   static constexpr uint32_t kMaxIters = 4;
@@ -352,6 +355,7 @@ struct BlackScholes : TenantBase {
 struct Stencil2D : TenantBase {
   using Args = slate_args_stencil;
   static constexpr int kThreads = 256;        // 32 x 8
+  static constexpr int kMinBlocks = 8;       // 32 registers, no spill
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t bx, uint32_t by, uint32_t, char*) {
