@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--impl", default="slate", choices=["slate", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-c3", action="store_true", help="skip the C3 (GEMM + copy) companion measurement")
+    ap.add_argument("--no-c4", action="store_true", help="skip the C4 (4 client processes via slated) measurement")
     ap.add_argument("--cpu-sample-s", type=float, default=12.0, help="target seconds of oracle work for cpu_baseline")
     return ap.parse_args()
 
@@ -497,6 +498,19 @@ def run_slate(args, world, rank, local):
         c3["antt"] = r3["schedules"]["slate_corun"]["antt"]
         del w3
 
+    # ---- C4 (configs[3]): four client processes through the slated daemon (rank 0 only)
+    c4 = None
+    if rank == 0 and not args.no_c4:
+        try:
+            sys.path.insert(0, os.path.join(ROOT, "tools"))
+            import c4_bench
+            sA.close()
+            sB.close()
+            sA = sB = None
+            c4 = c4_bench.run(max(3, args.steps // 2))
+        except Exception as e:   # reported, never fatal for the headline
+            c4 = {"error": str(e)[:300]}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         pair_s, sample = oracle_pair_seconds(args.cpu_sample_s)
@@ -517,12 +531,15 @@ def run_slate(args, world, rank, local):
     }
     if c3:
         line["c3"] = c3
+    if c4:
+        line["c4"] = c4
     if cpu:
         line["cpu_baseline"] = cpu
     if rank == 0:
         print(json.dumps(line), flush=True)
-    sA.close()
-    sB.close()
+    if sA:
+        sA.close()
+        sB.close()
 
 
 def main():

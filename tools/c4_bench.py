@@ -1,0 +1,178 @@
+"""C4 (BASELINE configs[3]): a 4-tenant mix -- triad, SpMV, 2-D stencil, bf16 GEMM --
+from four separate client processes through one `slated` server (shared-memory
+command slots, buffers by CUDA IPC), AUTO placement: the selector pairs the
+GEMM (H_C) with a memory tenant at a time and runs memory tenants solo with
+each other (Tab I).  Compared with the same four jobs run back to back with
+the original kernels by one client.  Device times come from the server's
+CUDA events (slate_query start/end, one clock for every client).
+
+    python tools/c4_bench.py [--steps K]     (prints one JSON line)
+"""
+import argparse
+import json
+import os
+import signal
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+JOBS = {   # kind -> launches per job (each job ~ 8-18 ms solo)
+    "triad": 64, "spmv": 256, "stencil": 64, "gemm": 96,
+}
+
+
+def build(kind, S, dev):
+    import torch
+    from paper_conf_ipps_allenf019_b200 import inputs as I
+    g = torch.Generator(device=dev)
+    g.manual_seed(20190520 + 400 + len(kind))
+    if kind == "triad":
+        n = 1 << 26
+        a, b, c = torch.zeros(n, device=dev), torch.rand(n, device=dev, generator=g), torch.rand(n, device=dev, generator=g)
+        keep = (a, b, c)
+        args, grid = S.triad_args(a, b, c, 3.0)
+        k = S.KIND_TRIAD
+    elif kind == "spmv":
+        rp, col, val, x = (torch.from_numpy(v).to(dev) for v in I.spmv_inputs(1 << 20, I.seed_for(4, 1)))
+        y = torch.zeros(1 << 20, device=dev)
+        keep = (rp, col, val, x, y)
+        args, grid = S.spmv_args(rp, col, val, x, y)
+        k = S.KIND_SPMV_CSR
+    elif kind == "stencil":
+        f = torch.rand(8192, 8192, device=dev, generator=g)
+        o = torch.zeros_like(f)
+        keep = (f, o)
+        args, grid = S.stencil_args(f, o)
+        k = S.KIND_STENCIL2D
+    else:
+        A = (torch.rand(4096, 4096, device=dev, generator=g) * 2 - 1).to(torch.bfloat16)
+        B = (torch.rand(4096, 4096, device=dev, generator=g) * 2 - 1).to(torch.bfloat16)
+        C = torch.zeros(4096, 4096, device=dev)
+        keep = (A, B, C)
+        args, grid = S.gemm_args(A.view(torch.int16), B.view(torch.int16), C)
+        k = S.KIND_GEMM_BF16
+    torch.cuda.synchronize()
+    return k, args, grid, keep
+
+
+def client(endpoint, kind, steps, go_path):
+    """One tenant process: profile, then `steps` jobs, each released by the parent."""
+    from paper_conf_ipps_allenf019_b200 import slate as S
+    s = S.Session(endpoint)
+    k, args, grid, keep = build(kind, S, "cuda:0")
+    for t in keep:
+        s.share_buffer(t)
+    kid = s.register_kernel(k)
+    s.profile(kid, args, grid, S.PROF_CURVE)
+    print("READY", flush=True)
+    out = []
+    for step in range(steps):
+        while not os.path.exists("%s.%d" % (go_path, step)):
+            time.sleep(0.0005)
+        ids = [s.launch(kid, args, grid, placement=S.PLACE_AUTO) for _ in range(JOBS[kind])]
+        s.sync(0)
+        qs = [s.query(i) for i in ids]
+        out.append([min(q["start_ms"] for q in qs), max(q["end_ms"] for q in qs),
+                    sum(len(q["resize_us"]) for q in qs), [v for q in qs for v in q["resize_us"]]])
+    print("RESULT " + json.dumps(out), flush=True)
+    s.close()
+
+
+def sequential(endpoint):
+    """The four jobs back to back with the original kernels, one client (vanilla CUDA)."""
+    from paper_conf_ipps_allenf019_b200 import slate as S
+    s = S.Session(endpoint)
+    built = {k: build(k, S, "cuda:0") for k in JOBS}
+    for k, (_, _, _, keep) in built.items():
+        for t in keep:
+            s.share_buffer(t)
+    kids = {k: s.register_kernel(v[0]) for k, v in built.items()}
+    times = []
+    for rep in range(4):
+        ids = []
+        per = {}
+        for k, (_, args, grid, _) in built.items():
+            li = [s.launch(kids[k], args, grid, mode=S.MODE_STANDALONE) for _ in range(JOBS[k])]
+            ids += li
+            per[k] = li
+        s.sync(0)
+        qs = {i: s.query(i) for i in ids}
+        t0 = min(q["start_ms"] for q in qs.values())
+        t1 = max(q["end_ms"] for q in qs.values())
+        solo = {k: max(qs[i]["end_ms"] for i in li) - min(qs[i]["start_ms"] for i in li) for k, li in per.items()}
+        if rep:
+            times.append((t1 - t0, solo))
+    s.close()
+    times.sort(key=lambda x: x[0])
+    return times[len(times) // 2]
+
+
+def run(steps):
+    """Run the C4 measurement (daemon + 4 client processes); returns the result dict."""
+    from paper_conf_ipps_allenf019_b200 import slate as S
+    cmd = [sys.executable, __file__, "--steps", str(steps)]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=900)
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    if not lines:
+        raise RuntimeError("c4 failed: " + out.stderr[-500:])
+    return json.loads(lines[-1])
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--client", nargs=3)
+    a = ap.parse_args()
+    if a.client:
+        client(a.client[0], a.client[1], a.steps, a.client[2])
+        return
+    from paper_conf_ipps_allenf019_b200 import slate as S
+    ep = "/slate-c4-%d" % os.getpid()
+    go = "/tmp/slate_c4_go_%d" % os.getpid()
+    d = subprocess.Popen([S.DAEMON, "--endpoint", ep], stderr=subprocess.DEVNULL)
+    for _ in range(300):
+        try:
+            S.Session(ep).close()
+            break
+        except S.SlateError:
+            time.sleep(0.2)
+    seq_ms, solo = sequential(ep)
+    ps = {k: subprocess.Popen([sys.executable, __file__, "--steps", str(a.steps), "--client", ep, k, go],
+                              stdout=subprocess.PIPE, text=True) for k in JOBS}
+    for p in ps.values():
+        assert "READY" in p.stdout.readline()
+    for step in range(a.steps):
+        open("%s.%d" % (go, step), "w").close()
+        time.sleep(0.3)
+    res = {}
+    for k, p in ps.items():
+        out, _ = p.communicate(timeout=600)
+        res[k] = json.loads([l for l in out.splitlines() if l.startswith("RESULT ")][0][7:])
+    d.send_signal(signal.SIGTERM)
+    d.wait(timeout=30)
+    for step in range(a.steps):
+        os.unlink("%s.%d" % (go, step))
+    spans, stps, resize = [], [], []
+    for step in range(a.steps):
+        t0 = min(res[k][step][0] for k in JOBS)
+        t1 = max(res[k][step][1] for k in JOBS)
+        spans.append(t1 - t0)
+        # turnaround of each job from the step's release (all four arrive together)
+        stps.append(sum(solo[k] / (res[k][step][1] - t0) for k in JOBS))
+        resize += [v for k in JOBS for v in res[k][step][3]]
+    spans_sorted = sorted(spans)
+    mk = spans_sorted[len(spans) // 2]
+    print(json.dumps({"config": "C4: triad 2^26, SpMV 2^20, stencil 8192^2, bf16 GEMM 4096^3 from 4 client processes "
+                                "via slated (AUTO)",
+                      "jobs": JOBS, "seq_cuda_ms": round(seq_ms, 3), "solo_ms": {k: round(v, 3) for k, v in solo.items()},
+                      "corun_makespan_ms": round(mk, 3), "gain_vs_sequential": round(seq_ms / mk, 4),
+                      "stp_median": round(sorted(stps)[len(stps) // 2], 4), "makespans_ms": [round(x, 3) for x in spans],
+                      "resize_us": {"n": len(resize), "p50": round(sorted(resize)[len(resize) // 2], 2) if resize else None,
+                                    "max": round(max(resize), 2) if resize else None}}))
+
+
+if __name__ == "__main__":
+    main()
