@@ -142,8 +142,8 @@ typedef struct {
   uint32_t abi_version;    /* SLATE_ABI_VERSION */
   uint32_t kind;           /* slate_kind */
   uint32_t iters;          /* SLATE_ITERS, blocks per task; 0 -> auto per launch (reading
-                              Q11): min(cap, max(1, B / (8 * occ * N))), cap = 10 except
-                              SPMV_CSR 4; GEMM_BF16 -> 1 */
+                              Q11): min(cap, max(1, B / (t * occ * N))), cap = 10, t = 8;
+                              SPMV_CSR cap 8, t = 4; GEMM_BF16 -> 1 */
   uint32_t flags;          /* SLATE_KFLAG_* */
 } slate_kernel_desc;
 

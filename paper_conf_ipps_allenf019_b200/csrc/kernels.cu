@@ -50,6 +50,7 @@ KindOps make_ops(uint32_t default_iters) {
   o.args_size = sizeof(typename Tn::Args);
   o.default_iters = default_iters;
   o.max_auto_iters = Tn::kMaxIters;
+  o.tasks_per_worker = Tn::kTasksPerWorker;
   o.launch_worker = &launch_worker_t<Tn>;
   o.launch_standalone = &launch_standalone_t<Tn>;
   return o;

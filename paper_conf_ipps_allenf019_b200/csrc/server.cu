@@ -357,9 +357,9 @@ void Server::free_slot(int slot) {
 // reading Q11: the paper's default task of 10 blocks, reduced so every
 // worker gets at least ~8 tasks (a fixed 10 mis-fits small grids: the last
 // tasks leave workers idle)
-uint32_t Server::auto_iters(uint32_t B, int occ, uint32_t cap) const {
+uint32_t Server::auto_iters(uint32_t B, int occ, uint32_t cap, uint32_t per_worker) const {
   const uint64_t workers = uint64_t(occ) * uint64_t(n_sms_);
-  const uint64_t it = B / (8 * workers);
+  const uint64_t it = B / (uint64_t(per_worker ? per_worker : 8) * workers);
   return uint32_t(it < 1 ? 1 : (it > cap ? cap : it));
 }
 
@@ -438,8 +438,10 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     }
     L.slot = slot;
     std::memset(reinterpret_cast<void*>(h_mirror_ + slot), 0, sizeof(HostMirror));
-    // the control block was zeroed by DMA when it was freed (no SM needed)
-    if (slot_zeroed_[slot]) CK(cudaStreamWaitEvent(Q.stream, slot_zeroed_[slot], 0));
+    // the control block was zeroed by DMA when it was freed (no SM needed); only
+    // wait (a cross-stream dependency) if that copy has not finished yet
+    if (slot_zeroed_[slot] && cudaEventQuery(slot_zeroed_[slot]) != cudaSuccess)
+      CK(cudaStreamWaitEvent(Q.stream, slot_zeroed_[slot], 0));
     CK(cudaEventRecord(L.ev_start, Q.stream));
     WorkerCommon w{};
     w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = L.B; w.iters = L.iters; w.occ = uint32_t(L.k->occ);
@@ -532,7 +534,7 @@ int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_
   L->args.assign(static_cast<const unsigned char*>(d->args), static_cast<const unsigned char*>(d->args) + d->args_size);
   L->desc.args = nullptr;
   L->B = B;
-  L->iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters);
+  L->iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters, k.ops->tasks_per_worker);
   Launch& LL = *L;
   launches_[L->id] = std::move(L);
   *out = LL.id;
@@ -953,7 +955,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   validate(k, d, &B, nullptr);
   WorkerCommon w{};
   w.gx = d->grid[0]; w.gy = d->grid[1]; w.gz = d->grid[2]; w.B = B; w.occ = uint32_t(k.occ);
-  w.iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters);
+  w.iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters, k.ops->tasks_per_worker);
   w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
   w.ctrl = ctrl; w.tc = d_tc_ + slot; w.mirror = nullptr; w.cov = nullptr; w.rank_of = d_rank_of_;

@@ -108,7 +108,7 @@ class Server {
   bool launch_done_events(Launch& L);
   int alloc_slot();
   void free_slot(int slot);
-  uint32_t auto_iters(uint32_t B, int occ, uint32_t cap) const;
+  uint32_t auto_iters(uint32_t B, int occ, uint32_t cap, uint32_t per_worker) const;
   bool validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const;
   void work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const;
 

@@ -276,6 +276,9 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
   c2 = c;
   uint32_t g = fetch(0, 0, 0);
   int slot = 0;
+  // finished work is counted once per CTA at exit (one atomic per worker, not
+  // per task); the CTA whose count completes B stamps the end of the launch
+  uint32_t my_blocks = 0, my_tasks = 0;
   while (g != 0xffffffffu) {                      // Lst2 (1): until retreat or an empty queue
     const uint32_t n = min(p.iters, p.B - g);     // clamp the last task
     if constexpr (Tn::kLookahead) {
@@ -288,9 +291,32 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
       if (p.cov && threadIdx.x == 0)
         for (uint32_t i = 0; i < n; ++i) atomicAdd(&p.cov[g + i], 1u);
       __syncthreads();
-      if (threadIdx.x == 0) count_done(p, n);
+      my_blocks += n;
+      my_tasks += 1;
       g = g2;
       slot ^= 1;
+    } else if constexpr (!Tn::kSpeculative) {
+      // the boundary's resize word is in flight during the task; the counter
+      // atomic is one round trip at the boundary (fewer live registers than
+      // the speculative form below)
+      prefetch_ctrl();
+      if constexpr (Tn::kHasTask) {
+        Tn::cta_task(p.args, g, n, dyn_smem);
+        if (p.cov && threadIdx.x == 0)
+          for (uint32_t i = 0; i < n; ++i) atomicAdd(&p.cov[g + i], 1u);
+      } else {
+        BlockWalk w;
+        w.start(g, p.gx, p.gy);
+        for (uint32_t i = 0; i < n; ++i) {
+          Tn::cta_block(p.args, w.x, w.y, w.z, dyn_smem);
+          if (p.cov && threadIdx.x == 0) atomicAdd(&p.cov[g + i], 1u);
+          w.advance(p.gx, p.gy);
+        }
+      }
+      __syncthreads();
+      my_blocks += n;
+      my_tasks += 1;
+      g = fetch(slot ^= 1, 0, 0);
     } else {
       // speculative boundary: the decision for the NEXT task is taken now, from
       // the resize word loaded when the previous task started, and the counter
@@ -331,7 +357,8 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
         s_g[2] = spec_changed ? 1u : 0u;
       }
       __syncthreads();                            // every thread is done with the task
-      if (threadIdx.x == 0) count_done(p, n);
+      my_blocks += n;
+      my_tasks += 1;
       slot ^= 1;
       g = s_g[slot];
       if (s_g[2] && threadIdx.x < 32) {           // epoch changed: maybe the end of a shrink
@@ -341,6 +368,7 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     }
   }
   if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
+  if (threadIdx.x == 0 && my_blocks) count_done(p, my_blocks, my_tasks);
   if (threadIdx.x < 32) {
     c = __shfl_sync(0xffffffffu, c, 0);
     if (lane == 0) atomicAdd(&p.tc->live_rank[rank], 0xffffffffu);   // live_rank -= 1

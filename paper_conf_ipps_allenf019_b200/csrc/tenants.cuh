@@ -26,6 +26,8 @@ struct TenantBase {
                                             // 1-D grid knowing the CTA's next task [g2, g2+n2) (n2 = 0: none)
   static constexpr uint32_t kMaxIters = 10; // cap of the automatic task size (P:L303 default 10)
   static constexpr int kMinBlocks = 1;      // __launch_bounds__ min blocks per SM of the worker
+  static constexpr bool kSpeculative = false; // fetch the next task while this one runs (+registers)
+  static constexpr uint32_t kTasksPerWorker = 8; // auto task size aims at >= this many tasks per worker
   static constexpr bool kHasFini = false;   // cta_fini(smem): once per CTA before it exits
 };
 
@@ -223,17 +225,19 @@ struct SgemmNaive : TenantBase {
 // 32 rows per block; warp w handles rows 4w..4w+3 with 8 lanes per row: lane l
 // sums j = rp[row]+l, +8, +16, ... in ascending order (an fmaf chain from 0),
 // then a butterfly (xor 4, 2, 1) inside the 8-lane group.  The task body runs
-// the task's blocks (up to kMaxIters = 4) at once, each thread holding one row
+// the task's blocks (up to kMaxIters = kU) at once, each thread holding one row
 // per block, so the row-pointer, column/value and x loads of 4 rows are in
 // flight together (tools/probe/spmv_variants.cu: 1.7x the original kernel);
 // per row the arithmetic is exactly cta_block's.
-struct SpmvCsr : TenantBase {
+template <int kU, int kMB>
+struct SpmvCsrT : TenantBase {
   using Args = slate_args_spmv;
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 6;       // 40 registers (8-B spill): latency-bound, occupancy is throughput
+  static constexpr int kMinBlocks = kMB;     // latency-bound: occupancy is throughput
   static constexpr int kSmem = 0, kSmemStandalone = 0;
   static constexpr bool kHasTask = true;
-  static constexpr uint32_t kMaxIters = 4;
+  static constexpr uint32_t kMaxIters = kU;
+  static constexpr uint32_t kTasksPerWorker = 4;   // full kU-block tasks (the body holds kU rows per thread)
 
   template <int U>
   __device__ __forceinline__ static void rows(const Args& a, uint32_t x0, uint32_t nblk) {
@@ -279,10 +283,13 @@ struct SpmvCsr : TenantBase {
   }
   __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char*) {
     uint32_t i = 0;
-    for (; i + 4 <= n; i += 4) rows<4>(a, g + i, 4);
-    if (i < n) rows<4>(a, g + i, n - i);
+    for (; i + kU <= n; i += kU) rows<kU>(a, g + i, kU);
+    if (i < n) rows<kU>(a, g + i, n - i);
   }
 };
+// the configuration in use: 8 blocks' rows in flight per thread, 4 CTAs/SM
+// (tools/probe/worker_overhead.cu: fastest of U in {1..8} x occupancy {4, 6, 8})
+using SpmvCsr = SpmvCsrT<8, 4>;
 
 // ============================================================== Black-Scholes
 // European call/put as in the CUDA SDK BlackScholes sample: the normal CDF by
@@ -292,6 +299,7 @@ struct SpmvCsr : TenantBase {
 struct BlackScholes : TenantBase {
   using Args = slate_args_bs;
   static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 6;       // 40 registers, no spill (non-speculative boundary)
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
   __device__ __forceinline__ static float cnd(float d) {

@@ -97,7 +97,15 @@ int main() {
     p.args = a; p.gx = nblk; p.gy = 1; p.gz = 1; p.B = nblk; p.iters = it; p.occ = occ; p.bound_lo = 0; p.bound_hi = 147;
     p.n_ranks = 148; p.standby_timeout_ns = 200000; p.ctrl = ctrl; p.tc = tc; p.mirror = nullptr; p.cov = nullptr; p.rank_of = lut;
     timeit("slate_worker<SpmvCsr> (the real one)", [&] { slate_worker<SpmvCsr><<<148 * occ, 256>>>(p); });
-    timeit("slate_worker<SpmvCsr> grid 148*8", [&] { slate_worker<SpmvCsr><<<148 * 8, 256>>>(p); });
+    auto variant = [&](const char* name, auto kern, int it2) {
+      int o; cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, 256, 0);
+      WorkerParams<slate_args_spmv> q = p; q.occ = o; q.iters = it2;
+      char buf[96]; snprintf(buf, sizeof buf, "%s occ %d", name, o);
+      timeit(buf, [&] { kern<<<148 * o, 256>>>(q); });
+    };
+    variant("U8 mb4 (SpmvCsr now)", slate_worker<SpmvCsrT<8, 4>>, 8);
+    variant("U4 mb6", slate_worker<SpmvCsrT<4, 6>>, 4);
+    variant("U3 mb8", slate_worker<SpmvCsrT<3, 8>>, 3);
   }
   return 0;
 }
