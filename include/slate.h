@@ -282,6 +282,12 @@ slate_status slate_serve(const char* endpoint, int device, uint32_t flags);
 const char* slate_status_string(slate_status st);     /* static string */
 const char* slate_last_error(slate_session* s);       /* session-owned, valid until the next call */
 
+/* The block geometry of a kind (what one original block of K(B,T) owns):
+ * elements per block for 1-D kinds (tile_m = 1), else the output tile rows x
+ * columns (sgemm 16 x 16, stencil 8 x 32, gemm 128 x tile_n of this build).
+ * Returns SLATE_EINVAL for an unknown kind.  No GPU needed. */
+slate_status slate_kind_geometry(uint32_t kind, uint32_t* tile_m, uint32_t* tile_n);
+
 /* ------------------------------------------------------------------ host logic
  * The selector's pure functions, exported so they can be checked without a GPU.
  * Categories: 0 L_C, 1 M_C, 2 H_C, 3 M_M, 4 H_M. */

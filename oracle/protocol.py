@@ -56,6 +56,8 @@ class Config:
     hi: int
     resizes: list = field(default_factory=list)   # [(lo, hi), ...] applied in order at random times
     grid: int = 0             # CTAs per launch; default occ * ranks (one full wave)
+    abort: bool = False       # long-task tenants: a retiring worker may abandon its task
+                              # mid-way and return it (Q28)
 
 
 def _in(rank, lo, hi):
@@ -71,6 +73,7 @@ class Model:
         self.epoch = 0
         self.lo, self.hi = cfg.lo, cfg.hi  # the resize word {epoch, lo, hi}
         self.live = 0                      # live worker CTAs of the tenant
+        self.returned = []                 # abandoned task starts, FIFO (Q28)
         self.cov = [0] * cfg.blocks        # executions per original block
         self.blocks_done = 0
         self.tasks_done = 0
@@ -95,7 +98,7 @@ class Model:
             self.live -= 1
 
     def key(self):
-        return (self.next, self.epoch, self.lo, self.hi, self.live, tuple(self.cov), self.blocks_done,
+        return (self.next, self.epoch, self.lo, self.hi, self.live, tuple(self.returned), tuple(self.cov), self.blocks_done,
                 self.tasks_done, tuple(sorted(self.task_starts)), self.resize_i,
                 tuple(tuple(c) for c in self.ctas), tuple(self.resident))
 
@@ -110,6 +113,10 @@ class Model:
                         acts.append(("place", i, r))
             elif st in (PROLOGUE, FETCH, EXEC, CHECK):
                 acts.append(("step", i))
+                # Q28: a worker outside the range may abandon its running task and
+                # retire, unless it is the last live worker (one atomic on {live, returned})
+                if st == EXEC and self.cfg.abort and not self.in_range(c) and self.live > 1:
+                    acts.append(("abort", i))
             elif st == STANDBY:
                 acts.append(("step", i))
                 if self.live == 0 and self.next < self.cfg.blocks:
@@ -141,13 +148,17 @@ class Model:
         i = act[1]
         c = self.ctas[i]
         st = c[0]
+        if act[0] == "abort":              # return the task, retire (live -1, returned +1 at once)
+            self.returned.append(c[4])
+            self.exit(c, True)
+            return
         if act[0] == "timeout":            # standby with no live worker: run anyway (liveness)
             self.live += 1
             c[0], c[7] = FETCH, True
             return
         if st in (PROLOGUE, STANDBY):
             # Lst1: leader reads the SM id and the bound; here also the queue state
-            if self.next >= cfg.blocks:
+            if self.next >= cfg.blocks and not self.returned:
                 self.exit(c, False)        # exit (2): nothing left to do
             elif self.in_range(c):
                 self.live += 1
@@ -157,11 +168,15 @@ class Model:
             else:
                 c[0] = STANDBY             # wait: the tenant is under-staffed
         elif st == FETCH:
+            if self.returned:              # Q28: returned tasks first
+                g = self.returned.pop(0)
+                c[0], c[4], c[5] = EXEC, g, min(cfg.iters, cfg.blocks - g)
+                return
             # Lst2 (2): globIdx = atomicAdd(&slateIdx, SLATE_ITERS)
             g = self.next
             self.next += cfg.iters
             if g >= cfg.blocks:            # Q3: never run a task that starts past the end
-                self.exit(c, True)         # exit (2)
+                self.exit(c, True)         # exit (2): the returned list was empty in the same atomic step
             else:
                 c[0], c[4], c[5] = EXEC, g, min(cfg.iters, cfg.blocks - g)
                 self.task_starts.append(g)
@@ -175,7 +190,7 @@ class Model:
         elif st == CHECK:
             # Lst2 (1) loop condition: retreat is examined only between tasks
             c[6] = self.epoch
-            if self.in_range(c) or (self.live == 1 and self.next < cfg.blocks):
+            if self.in_range(c) or (self.live == 1 and (self.next < cfg.blocks or self.returned)):
                 c[0] = FETCH               # stay (the last live worker never retires)
             else:
                 self.exit(c, True)         # exit (3): retreated
@@ -197,6 +212,8 @@ class Model:
             raise ProtocolViolation("next_clamped")
         if self.live != 0:
             raise ProtocolViolation("live workers at the end")
+        if self.returned:
+            raise ProtocolViolation("returned tasks never executed")
 
     def check_step(self):
         if any(v > 1 for v in self.cov):

@@ -71,6 +71,25 @@ const char* slate_status_string(slate_status st) {
 
 const char* slate_last_error(slate_session* s) { return s ? s->last_error.c_str() : "no session"; }
 
+slate_status slate_kind_geometry(uint32_t kind, uint32_t* tile_m, uint32_t* tile_n) {
+  if (!tile_m || !tile_n) return SLATE_EINVAL;
+  switch (kind) {
+    case SLATE_KIND_TRIAD: *tile_m = 1; *tile_n = 1024; return SLATE_OK;
+    case SLATE_KIND_COPY: *tile_m = 1; *tile_n = 4096; return SLATE_OK;
+    case SLATE_KIND_SGEMM_NAIVE: *tile_m = 16; *tile_n = 16; return SLATE_OK;
+    case SLATE_KIND_SPMV_CSR: *tile_m = 1; *tile_n = 32; return SLATE_OK;
+    case SLATE_KIND_BLACKSCHOLES: *tile_m = 1; *tile_n = 1024; return SLATE_OK;
+    case SLATE_KIND_STENCIL2D: *tile_m = 8; *tile_n = 32; return SLATE_OK;
+    case SLATE_KIND_GEMM_BF16: {
+      const slate::KindOps* o = slate::kind_ops(kind);
+      *tile_m = 128;
+      *tile_n = o && o->tile_n ? o->tile_n : 128;
+      return SLATE_OK;
+    }
+    default: return SLATE_EINVAL;
+  }
+}
+
 slate_status slate_attach(const char* endpoint, int device, slate_session** out) {
   if (!out) return SLATE_EINVAL;
   *out = nullptr;

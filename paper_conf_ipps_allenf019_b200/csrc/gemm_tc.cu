@@ -23,11 +23,14 @@
 namespace slate {
 namespace gemm {
 
-constexpr int BM = 128, BN = 128, BK = 64;        // tile and K slice
-constexpr int kStages = 6;
+#ifndef SLATE_GEMM_BN
+#define SLATE_GEMM_BN 256
+#endif
+constexpr int BM = 128, BN = SLATE_GEMM_BN, BK = 64;   // tile and K slice
+constexpr int kStageBytes = (BM + BN) * BK * 2;        // 32 KiB (BN 128) / 48 KiB (BN 256)
+constexpr int kStages = (6 * 32768) / kStageBytes;     // ~192 KiB ring
 constexpr int kThreads = 256;
-constexpr int kStageBytes = (BM + BN) * BK * 2;   // 32 KiB
-constexpr int kTmemCols = 256;                    // two 128-column fp32 accumulators
+constexpr int kTmemCols = 2 * BN;                      // two fp32 accumulators of BN columns
 constexpr int kSmemBytes = 1024 /*align slack*/ + kStages * kStageBytes + 256 /*barriers*/;
 
 struct Params {
@@ -130,10 +133,25 @@ struct Smem {
   uint64_t full[kStages], empty[kStages];
   uint64_t tmem_full[2], tmem_empty[2];
   uint64_t tq_full[2], tq_empty[2];
+  uint64_t drain;
   uint32_t tileq[2];
+  volatile uint32_t kb_limit[2];   // k-slices the producer issues for the tile in queue slot j
+  volatile uint32_t aborted[2];    // the tile in accumulator b was abandoned (Q28): no store
   uint32_t tmem_base;
   uint32_t go, rank, retired;
 };
+
+__device__ __forceinline__ bool mbar_try(uint64_t* b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(s_u32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
 
 // ------------------------------------------------------------------ the kernel
 template <bool kSlate>
@@ -166,7 +184,9 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       mbar_init(&S.tmem_empty[i], 1);
       mbar_init(&S.tq_full[i], 1);
       mbar_init(&S.tq_empty[i], 1 + 4);   // MMA thread + one lane of each epilogue warp
+      S.aborted[i] = 0;
     }
+    mbar_init(&S.drain, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0 && lane == 0) {
@@ -189,52 +209,61 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
     // ===================== producer + slate task decisions =====================
     if (lane == 0) {
       uint32_t t = 0, it = 0;   // tiles handed out, k-slices issued
-      uint64_t c2 = 0;
-      bool first = true;
-      for (;;) {
-        uint32_t g;
+      bool stop = false;
+      while (!stop) {
+        uint32_t g = 0xffffffffu, n = 1;
         if constexpr (kSlate) {
-          // task boundary: resize word, then the counter
-          c2 = ld_acquire_u64(p.ctrl);
-          const bool chg = !first && ctrl_epoch(c2) != ctrl_epoch(c);
-          (void)chg;
-          c = c2;
-          first = false;
-          g = 0xffffffffu;
+          // task boundary: resize word, returned tasks, then the counter
+          c = ld_acquire_u64(p.ctrl);
           if (!in_range(p, S.rank, c) && try_retire(p.tc)) {
             S.retired = 1;
           } else {
-            const uint32_t f = atomicAdd(&p.tc->next, p.iters);           // Lst2 (2), iters = 1
-            if (f < p.B) {
-              g = f;
-              if (f == 0) p.tc->t_first = globaltimer();
-            } else {
-              atomicAdd(&p.tc->live, 0xffffffffu);
+            bool leave;
+            g = take_returned(p.tc, false, leave);            // an abandoned tile first (Q28)
+            if (g == 0xffffffffu) {
+              const uint32_t f = atomicAdd(&p.tc->next, p.iters);   // Lst2 (2)
+              if (f < p.B) {
+                g = f;
+                n = min(p.iters, p.B - f);
+                if (f == 0) p.tc->t_first = globaltimer();
+              } else {
+                g = take_returned(p.tc, true, leave);          // drained: leave unless one was returned
+              }
             }
           }
         } else {
           g = t == 0 ? blockIdx.y * gridDim.x + blockIdx.x : 0xffffffffu;
         }
-        if (g == 0xffffffffu) {                          // sentinel: the other roles stop
-          const uint32_t j = t & 1, u = t >> 1;
-          mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
-          S.tileq[j] = g;
-          mbar_arrive(&S.tq_full[j]);
-          break;
-        }
+        if (g == 0xffffffffu) break;
         // a task = n consecutive tiles (SLATE_ITERS), handed out one by one;
         // bit 31 marks the last tile of the task (tasks_done counts tasks)
-        const uint32_t n = kSlate ? min(p.iters, p.B - g) : 1u;
-        for (uint32_t i = 0; i < n; ++i) {
+        for (uint32_t i = 0; i < n && !stop; ++i) {
           const uint32_t tile = g + i;
           const uint32_t j = t & 1, u = t >> 1;
           mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
+          S.kb_limit[j] = num_kb;
           S.tileq[j] = tile | (i + 1 == n ? 0x80000000u : 0u);
           mbar_arrive(&S.tq_full[j]);
           ++t;
           uint32_t m0, n0;
           tile_of(tile, p.gx, p.gy, m0, n0);
           for (uint32_t kb = 0; kb < num_kb; ++kb, ++it) {
+            if constexpr (kSlate) {
+              // Q28: a worker that left the range abandons its tile mid-way (if it
+              // is not the last live worker) and gives the tile back; nothing of it
+              // is stored.  Checked every 16 K slices (~4-8 us).
+              if ((kb & 15) == 15 && n == 1) {
+                const uint64_t c2 = ld_acquire_u64(p.ctrl);
+                if (!in_range(p, S.rank, c2) && try_retire(p.tc, true)) {
+                  give_back_task(p.tc, tile);
+                  c = c2;
+                  S.retired = 1;
+                  S.kb_limit[j] = kb;            // the MMA consumes the kb slices issued, then aborts
+                  stop = true;
+                  break;
+                }
+              }
+            }
             const uint32_t s = it % kStages, r = it / kStages;
             mbar_wait(&S.empty[s], (r & 1) ^ 1);
             char* sa = ring + s * kStageBytes;
@@ -245,6 +274,11 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
           }
         }
       }
+      // sentinel: the other roles stop after the tiles already handed out
+      const uint32_t j = t & 1, u = t >> 1;
+      mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
+      S.tileq[j] = 0xffffffffu;
+      mbar_arrive(&S.tq_full[j]);
     }
   } else if (warp == 1) {
     // ===================== MMA issuer (one thread) =====================
@@ -254,15 +288,21 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
         const uint32_t j = t & 1, u = t >> 1;
         mbar_wait(&S.tq_full[j], u & 1);
         const uint32_t g = S.tileq[j];
-        mbar_arrive(&S.tq_empty[j]);
-        if (g == 0xffffffffu) break;
+        if (g == 0xffffffffu) {
+          mbar_arrive(&S.tq_empty[j]);
+          break;
+        }
         const uint32_t b = t & 1, v = t >> 1;
         mbar_wait(&S.tmem_empty[b], (v & 1) ^ 1);     // the epilogue has drained this accumulator
         tc_fence_after();
         const uint32_t d = tmem + b * BN;
+        bool abandoned = false;
         for (uint32_t kb = 0; kb < num_kb; ++kb, ++it) {
           const uint32_t s = it % kStages, r = it / kStages;
-          mbar_wait(&S.full[s], r & 1);
+          while (!mbar_try(&S.full[s], r & 1)) {
+            if (kb >= S.kb_limit[j]) { abandoned = true; break; }   // Q28: no more slices will come
+          }
+          if (abandoned) break;
           tc_fence_after();
           const uint32_t sa = s_u32(ring + s * kStageBytes);
           const uint32_t sb = sa + BM * BK * 2;
@@ -271,7 +311,15 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
             tc_mma(d, sw128_desc(sa + kk * 32), sw128_desc(sb + kk * 32), kIdesc, (kb | kk) != 0);
           tc_commit(&S.empty[s]);                      // frees the stage when these MMAs complete
         }
-        tc_commit(&S.tmem_full[b]);                    // accumulator ready
+        mbar_arrive(&S.tq_empty[j]);
+        if (abandoned) {
+          tc_commit(&S.drain);                          // the issued MMAs finish before TMEM is let go
+          mbar_wait(&S.drain, 0);
+          S.aborted[b] = 1;
+          mbar_arrive(&S.tmem_full[b]);                 // wake the epilogue: nothing to store
+        } else {
+          tc_commit(&S.tmem_full[b]);                   // accumulator ready
+        }
         ++t;
       }
     }
@@ -291,6 +339,15 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       const uint32_t b = t & 1, v = t >> 1;
       mbar_wait(&S.tmem_full[b], v & 1);
       tc_fence_after();
+      if (S.aborted[b]) {                               // abandoned tile (Q28): nothing stored or counted
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (ew == 0 && lane == 0) {
+          S.aborted[b] = 0;
+          mbar_arrive(&S.tmem_empty[b]);
+        }
+        ++t;
+        continue;
+      }
       uint32_t m0, n0;
       tile_of(g, p.gx, p.gy, m0, n0);
       const uint32_t row = m0 + ew * 32 + lane;
@@ -346,13 +403,13 @@ static EncodeTiledFn encode_fn() {
   return fn;
 }
 
-// a rows x k bf16 K-major matrix, boxes of 128 rows x 64 columns, 128-B swizzle
-static bool make_map(CUtensorMap* m, const void* base, uint32_t rows, uint32_t k) {
+// a rows x k bf16 K-major matrix, boxes of box_rows rows x 64 columns, 128-B swizzle
+static bool make_map(CUtensorMap* m, const void* base, uint32_t rows, uint32_t k, uint32_t box_rows) {
   EncodeTiledFn enc = encode_fn();
   if (!enc) return false;
   const cuuint64_t dims[2] = {k, rows};
   const cuuint64_t strides[1] = {cuuint64_t(k) * 2};
-  const cuuint32_t box[2] = {BK, BM};
+  const cuuint32_t box[2] = {BK, box_rows};
   const cuuint32_t estr[2] = {1, 1};
   return enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -362,8 +419,8 @@ static bool make_map(CUtensorMap* m, const void* base, uint32_t rows, uint32_t k
 static cudaError_t fill(Params& p, const void* args) {
   std::memset(&p, 0, sizeof(p));
   std::memcpy(&p.args, args, sizeof(p.args));
-  if (!make_map(&p.tma_a, reinterpret_cast<const void*>(p.args.A), p.args.m, p.args.k) ||
-      !make_map(&p.tma_b, reinterpret_cast<const void*>(p.args.B), p.args.n, p.args.k))
+  if (!make_map(&p.tma_a, reinterpret_cast<const void*>(p.args.A), p.args.m, p.args.k, BM) ||
+      !make_map(&p.tma_b, reinterpret_cast<const void*>(p.args.B), p.args.n, p.args.k, BN))
     return cudaErrorInvalidValue;
   return cudaSuccess;
 }
@@ -403,6 +460,7 @@ KindOps gemm_tc_ops() {
   o.args_size = sizeof(slate_args_gemm);
   o.default_iters = 1;   // one tile per task: resize latency ~ one tile (SURVEY §7 hard part 3)
   o.max_auto_iters = 1;
+  o.tile_n = gemm::BN;
   o.launch_worker = &gemm::launch_worker;
   o.launch_standalone = &gemm::launch_standalone;
   return o;

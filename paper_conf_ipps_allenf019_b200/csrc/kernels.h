@@ -1,6 +1,7 @@
 // kernels.h -- host/device shared layout of the slate control structures and
 // the host-side dispatch table over tenant kinds.  No torch types anywhere.
 #pragma once
+#include <cstddef>
 #include <cstdint>
 #include <cuda_runtime.h>
 #include "../../include/slate.h"
@@ -23,16 +24,22 @@ __host__ __device__ __forceinline__ uint32_t ctrl_hi(uint64_t c) { return uint32
 struct alignas(128) TaskCtl {
   uint32_t next;                  // slateIdx: next original block to hand out
   uint32_t pad0[31];
-  unsigned long long done;        // (tasks_done << 32) | blocks_done, one atomic per task
-  uint32_t live;                  // live worker CTAs
+  unsigned long long done;        // (tasks_done << 32) | blocks_done
+  unsigned long long live_pending;// (returned tasks << 32) | live worker CTAs: one word, so that
+                                  // abandoning a task and retiring is one atomic step (Q28)
   uint32_t started;               // workers that joined
+  uint32_t pad_s;
   unsigned long long t_first;     // %globaltimer at the start of the task at block 0
   unsigned long long t_last;      // %globaltimer when blocks_done reached B
   uint32_t shrink_epoch;          // last epoch whose shrink was observed complete
   uint32_t join_epoch;            // last epoch in which a worker joined (grow)
-  uint32_t pad1[22];
+  uint32_t pad1[20];
   uint32_t live_rank[kMaxRanks];  // live workers per SM rank
+  uint32_t ret_head, ret_tail;    // ring of abandoned task starts (+1; 0 = slot empty)
+  uint32_t pad2[30];
+  uint32_t ret[kMaxRanks];
 };
+static_assert(offsetof(TaskCtl, live_rank) == 256, "TaskCtl header must stay 256 B (the query snapshot)");
 constexpr size_t kTaskCtlHeader = 256;   // the part snapshotted to the host at the end
 
 // Per launch, in mapped pinned host memory: what the host poller watches.
@@ -68,6 +75,7 @@ struct KindOps {
   uint32_t default_iters = 0;   // 0: auto (reading Q11)
   uint32_t max_auto_iters = 10; // per-tenant cap of the automatic task size
   uint32_t tasks_per_worker = 8; // the automatic task size aims at >= this many tasks per worker
+  uint32_t tile_n = 0;           // GEMM: output columns per original block
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;
   cudaError_t (*launch_standalone)(const void* args, dim3 grid, cudaStream_t) = nullptr;
 };

@@ -271,9 +271,10 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     }
     case SLATE_KIND_GEMM_BF16: {
       auto a = static_cast<const slate_args_gemm*>(d->args);
-      if (a->m % 128 || a->n % 128 || a->k % 64 || a->k == 0) return fail("gemm_bf16 needs m, n % 128 == 0 and k % 64 == 0");
+      const uint32_t tn = k.ops->tile_n ? k.ops->tile_n : 128;
+      if (a->m % 128 || a->n % tn || a->k % 64 || a->k == 0) return fail("gemm_bf16 needs m % 128, n % tile_n, k % 64 == 0");
       if (!al(a->A) || !al(a->B) || !al(a->C)) return fail("gemm arrays must be 16-byte aligned");
-      g[0] = a->n / 128;
+      g[0] = a->n / tn;
       g[1] = a->m / 128;
       break;
     }
@@ -905,7 +906,7 @@ int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
     out->next_raw = tc.next;
     const uint64_t clamp = cdiv(L.B, L.iters) * L.iters;
     out->next_clamped = uint32_t(std::min<uint64_t>(tc.next, clamp));
-    out->live_workers = tc.live;
+    out->live_workers = uint32_t(tc.live_pending);
     out->workers_started = tc.started;
     out->t_first_ns = tc.t_first;
     out->t_last_ns = tc.t_last;

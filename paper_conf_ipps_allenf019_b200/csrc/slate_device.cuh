@@ -35,6 +35,11 @@ __device__ __forceinline__ uint64_t ld_acquire_u64(const uint64_t* p) {
   asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const unsigned long long* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -103,14 +108,14 @@ __device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
     if (nxt >= p.B) return false;                                       // exit (2)
     bool join = in_range(p, rank, c);
     if (!join) {
-      const uint32_t live = ld_relaxed_u32(&tc->live);
+      const uint32_t live = uint32_t(ld_relaxed_u64(&tc->live_pending));
       const uint32_t target = p.occ * (ctrl_hi(c) - ctrl_lo(c) + 1);
       if (live >= target) return false;                                  // exit (1)
       if (t0 == 0) t0 = globaltimer();
       if (live == 0 && globaltimer() - t0 > p.standby_timeout_ns) join = true;
     }
     if (join) {
-      atomicAdd(&tc->live, 1u);              // results unused: RED, no round trip
+      atomicAdd(&tc->live_pending, 1ull);    // results unused: RED, no round trip
       atomicAdd(&tc->live_rank[rank], 1u);
       atomicAdd(&tc->started, 1u);
       const uint32_t e = ctrl_epoch(c);
@@ -148,14 +153,52 @@ __device__ void check_shrink_done(const P& p, uint64_t c, uint32_t lane) {
 }
 
 // Retire unless this is the last live worker (liveness rule): CAS on live.
-__device__ __forceinline__ bool try_retire(TaskCtl* tc) {
-  uint32_t v = ld_relaxed_u32(&tc->live);
-  while (v > 1u) {
-    const uint32_t w = atomicCAS(&tc->live, v, v - 1u);
+// With `give_back`, the same atomic step also counts one returned task (Q28).
+__device__ __forceinline__ bool try_retire(TaskCtl* tc, bool give_back = false) {
+  unsigned long long v = ld_relaxed_u64(&tc->live_pending);
+  const unsigned long long delta = give_back ? (1ull << 32) - 1ull : ~0ull;   // live -1 (, returned +1)
+  while (uint32_t(v) > 1u) {
+    const unsigned long long w = atomicCAS(&tc->live_pending, v, v + delta);
     if (w == v) return true;
     v = w;
   }
   return false;   // the last live worker stays (its next fetch exits if the queue is drained)
+}
+
+// Q28 returned-task ring (long-task tenants only).  A retiring worker that
+// abandons its task first wins try_retire(give_back) and then publishes the
+// task start; a fetcher first claims a returned task in the same word and then
+// takes the next ring slot, waiting for its publication.
+__device__ __forceinline__ void give_back_task(TaskCtl* tc, uint32_t g) {
+  const uint32_t t = atomicAdd(&tc->ret_tail, 1u) % kMaxRanks;
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(&tc->ret[t]), "r"(g + 1u) : "memory");
+}
+// one lane: a returned task if any (0xffffffff if none), or, when the queue is
+// drained and none is returned, leave (live -= 1) -- atomically with respect to
+// returns, so a returned task can never be orphaned.
+__device__ __forceinline__ uint32_t take_returned(TaskCtl* tc, bool drained, bool& leave) {
+  leave = false;
+  unsigned long long v = ld_relaxed_u64(&tc->live_pending);
+  for (;;) {
+    if ((v >> 32) != 0) {
+      const unsigned long long w = atomicCAS(&tc->live_pending, v, v - (1ull << 32));
+      if (w != v) { v = w; continue; }
+      const uint32_t h = atomicAdd(&tc->ret_head, 1u) % kMaxRanks;
+      uint32_t g1;
+      do {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(g1) : "l"(&tc->ret[h]) : "memory");
+      } while (g1 == 0);
+      tc->ret[h] = 0;
+      return g1 - 1u;
+    }
+    if (!drained) return 0xffffffffu;
+    const unsigned long long w = atomicCAS(&tc->live_pending, v, v - 1ull);
+    if (w == v) {
+      leave = true;
+      return 0xffffffffu;
+    }
+    v = w;
+  }
 }
 
 // Task boundary, by ONE lane: given the resize word c2 (loaded
@@ -178,7 +221,7 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
   } else {
     g = atomicAdd(&tc->next, p.iters);                                  // Lst2 (2)
     if (g >= p.B) {                                                     // Q3: nothing to run
-      atomicAdd(&tc->live, 0xffffffffu);                                // live -= 1 (RED)
+      atomicAdd(&tc->live_pending, ~0ull);                               // live -= 1 (RED)
       g = 0xffffffffu;
     } else if (g == 0) {
       tc->t_first = globaltimer();
@@ -347,7 +390,7 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
       if (threadIdx.x == 0) {
         uint32_t g2 = 0xffffffffu;
         if (!spec_retired) {
-          if (fut >= p.B) atomicAdd(&p.tc->live, 0xffffffffu);        // queue drained: live -= 1
+          if (fut >= p.B) atomicAdd(&p.tc->live_pending, ~0ull);      // queue drained: live -= 1
           else g2 = fut;
           if (fut == 0) p.tc->t_first = globaltimer();
         } else {

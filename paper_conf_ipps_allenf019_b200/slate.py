@@ -130,6 +130,7 @@ for _name, _args in [
     ("slate_profile", [ctypes.c_void_p, c_u64, _P(LaunchDesc), c_u32, _P(Profile)]),
     ("slate_query", [ctypes.c_void_p, c_u64, _P(LaunchInfo)]),
     ("slate_serve", [ctypes.c_char_p, ctypes.c_int, c_u32]),
+    ("slate_kind_geometry", [c_u32, _P(c_u32), _P(c_u32)]),
 ]:
     getattr(_lib, _name).restype = c_i32
     getattr(_lib, _name).argtypes = _args
@@ -145,7 +146,7 @@ _lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c
 EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffer", "slate_unshare_buffer",
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
-            "slate_choose_split", "slate_serve"]
+            "slate_choose_split", "slate_serve", "slate_kind_geometry"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -317,7 +318,18 @@ def stencil_args(inp, out):
     return ArgsStencil(_ptr(inp), _ptr(out), h, w), (cdiv(w, 32), cdiv(h, 8), 1)
 
 
+def kind_geometry(kind):
+    tm, tn = c_u32(), c_u32()
+    st = _lib.slate_kind_geometry(kind, ctypes.byref(tm), ctypes.byref(tn))
+    if st != OK:
+        raise SlateError(st, "slate_kind_geometry(%d)" % kind)
+    return tm.value, tn.value
+
+
+GEMM_TILE_M, GEMM_TILE_N = kind_geometry(KIND_GEMM_BF16)
+
+
 def gemm_args(A, B, C):
     m, k = A.shape
     n, _ = B.shape
-    return ArgsGemm(_ptr(A), _ptr(B), _ptr(C), m, n, k, 0), (n // 128, m // 128, 1)
+    return ArgsGemm(_ptr(A), _ptr(B), _ptr(C), m, n, k, 0), (n // GEMM_TILE_N, m // GEMM_TILE_M, 1)

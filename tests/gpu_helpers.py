@@ -143,7 +143,7 @@ def make_gemm(m, n, k, seed, mode="float"):
             if mode == "int":
                 return np.array_equal(C, ref), 0.0
             return within(C, ref, np.abs(OT.bf16_to_f64(A)) @ np.abs(OT.bf16_to_f64(B)).T)
-        # sampled tiles (x, y) at full size
+        # sampled 128 x 128 tiles (x, y) at full size (the oracle's tiling, independent of the kernel's)
         worst, ok = 0.0, True
         for (x, y) in rows:
             ref = OT.gemm_bf16_tile(A, B, x, y)

@@ -27,7 +27,7 @@ CASES = {
     "bs": lambda: make_bs(1024 * 12 + 4 * 33 + 2, 108, n_scen=5),
     "stencil_float": lambda: make_stencil(8 * 37 + 3, 32 * 9 + 5, 109),
     "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
-    "gemm_int": lambda: make_gemm(256, 384, 512, 113, "int"),
+    "gemm_int": lambda: make_gemm(256, 512, 512, 113, "int"),
     "gemm_float": lambda: make_gemm(384, 256, 1024, 114),
 }
 
@@ -113,7 +113,8 @@ def test_gemm_full_size_sampled(sess):
         lid, outs, cov = _run(sess, t, k, placement=S.PLACE_AUTO)
         assert torch.equal(outs[0], ref[0])
         q = sess.query(lid)
-        assert q["coverage_ok"] == 1 and q["blocks_done"] == 4096 and q["tasks_done"] == 4096
+        B = int(np.prod(t.grid))
+        assert q["coverage_ok"] == 1 and q["blocks_done"] == B and q["tasks_done"] == B
         rng = random.Random(116)
         tiles = [(0, 0), (63, 63)] + [(rng.randrange(64), rng.randrange(64)) for _ in range(22)]
         ok, err = t.check(outs, rows=tiles)

@@ -13,7 +13,7 @@ import torch
 from oracle import tenants as OT
 from paper_conf_ipps_allenf019_b200 import slate as S
 
-from gpu_helpers import make_bs, make_copy, make_stencil, make_triad, within
+from gpu_helpers import make_bs, make_copy, make_gemm, make_stencil, make_triad, within
 
 pytestmark = pytest.mark.gpu
 
@@ -104,3 +104,33 @@ def test_shrink_then_grow_latency(sess):
     assert q["n_topups"] >= 1
     lat = q["resize_us"]
     assert len(lat) == 2 and all(0 < v < 5000 for v in lat), lat
+
+
+def test_resize_storm_gemm_abandons_tiles(sess):
+    """tcgen05 GEMM under a resize storm: workers leaving the range abandon their
+    tile mid-K and give it back (Q28); every tile is still stored exactly once,
+    bit-identical to the standalone launch (integer inputs: exact vs the oracle
+    on sampled tiles)."""
+    t = make_gemm(4096, 4096, 8192, 205, "int")
+    q, done = _storm(sess, t, 1, 40, 4, 30)
+    assert done >= 5
+    ok, err = t.check(t.snapshot(), rows=[(0, 0), (15, 31), (7, 3)])
+    assert ok
+
+
+def test_gemm_shrink_latency(sess):
+    n = sess.info()["num_sms"]
+    t = make_gemm(8192, 8192, 8192, 206)
+    k = sess.register_kernel(t.kind)
+    lats = []
+    for _ in range(3):
+        lid = sess.launch(k, t.args, t.grid, placement=S.PLACE_CORUN, sm=(0, n - 1))
+        time.sleep(0.0003)
+        sess.resize(lid, 0, n // 2 - 1)
+        time.sleep(0.0002)
+        sess.resize(lid, 0, n - 1)
+        sess.sync(lid)
+        q = sess.query(lid)
+        assert q["blocks_done"] == q["total_blocks"]
+        lats += q["resize_us"]
+    assert lats and max(lats) < 200, lats

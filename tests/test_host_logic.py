@@ -82,3 +82,12 @@ def test_choose_split_matches_oracle(S):
         s2, t2 = OS.choose_split(ca, cb, 148)
         assert abs(t1 - t2) <= 1e-9 * t2
         assert s1 == s2 or abs(OS.corun_makespan(ca, cb, 148, s1) - t2) <= 1e-9 * t2
+
+
+def test_kind_geometry(S):
+    assert S.kind_geometry(S.KIND_TRIAD) == (1, 1024)
+    assert S.kind_geometry(S.KIND_SGEMM_NAIVE) == (16, 16)
+    tm, tn = S.kind_geometry(S.KIND_GEMM_BF16)
+    assert tm == 128 and tn in (128, 256)
+    with pytest.raises(S.SlateError):
+        S.kind_geometry(99)

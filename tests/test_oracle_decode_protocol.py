@@ -59,6 +59,8 @@ def test_task_partition_is_exact():
     P.Config(blocks=5, iters=2, ranks=2, occ=1, lo=0, hi=0, resizes=[(1, 1)]),
     P.Config(blocks=3, iters=3, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1), (0, 0)]),
     P.Config(blocks=4, iters=1, ranks=1, occ=2, lo=0, hi=0, resizes=[]),
+    P.Config(blocks=3, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1), (0, 1)], abort=True),
+    P.Config(blocks=4, iters=2, ranks=2, occ=1, lo=0, hi=1, resizes=[(0, 0)], abort=True),
 ])
 def test_protocol_exhaustive(cfg):
     n = P.explore(cfg)
@@ -70,6 +72,7 @@ def test_protocol_random_seeds():
         P.Config(blocks=1000, iters=3, ranks=8, occ=2, lo=0, hi=7, resizes=[(0, 3), (5, 7), (0, 7)]),
         P.Config(blocks=997, iters=10, ranks=6, occ=3, lo=2, hi=3, resizes=[(0, 5), (4, 4), (1, 2)]),
         P.Config(blocks=50, iters=1, ranks=4, occ=1, lo=0, hi=3, resizes=[(3, 3)] * 3 + [(0, 0)]),
+        P.Config(blocks=300, iters=1, ranks=6, occ=1, lo=0, hi=5, resizes=[(0, 2), (3, 5), (1, 1), (0, 5)], abort=True),
     ]
     for cfg in cfgs:
         for seed in range(40):
@@ -108,3 +111,39 @@ def test_protocol_detects_a_broken_rule():
             failed = True
             break
     assert failed
+
+
+def test_protocol_abort_needs_the_combined_word():
+    """Q28: if abandoning a task and retiring were two steps (a worker may retire
+    while the last other worker exits on an empty return list), a returned task
+    could be orphaned: the mutation must fail."""
+    class Split(P.Model):
+        def actions(self):
+            acts = super().actions()
+            for i, c in enumerate(self.ctas):   # abort allowed even as the last live worker
+                if c[0] == P.EXEC and self.cfg.abort and not self.in_range(c) and self.live == 1:
+                    acts.append(("abort", i))
+            return acts
+
+    cfg = P.Config(blocks=2, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1)], grid=1, abort=True)
+    m = Split(cfg)
+    with pytest.raises(P.ProtocolViolation):
+        # explore every interleaving of the broken model
+        import copy
+        stack, seen = [m], set()
+        while stack:
+            x = stack.pop()
+            k = x.key()
+            if k in seen:
+                continue
+            seen.add(k)
+            if x.done():
+                x.check_final()
+                continue
+            acts = x.actions()
+            if not acts:
+                raise P.ProtocolViolation("deadlock")
+            for a in acts:
+                y = copy.deepcopy(x)
+                y.apply(a)
+                stack.append(y)
