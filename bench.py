@@ -347,8 +347,12 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     pa = sA.profile(kA, w.a.args, w.a.grid, S.PROF_CURVE)
     pb = sA.profile(kB, w.b.args, w.b.grid, S.PROF_CURVE)
     w.n_sms = info["num_sms"]
-    w.split, _ = S.choose_split(dict(zip(pa["curve_sms"], pa["curve_ms"])), dict(zip(pb["curve_sms"], pb["curve_ms"])),
-                                w.n_sms)
+    # the split the server's AUTO placement takes (reading Q10 + the Q29 saturation cap)
+    ca, cb = dict(zip(pa["curve_sms"], pa["curve_ms"])), dict(zip(pb["curve_sms"], pb["curve_ms"]))
+    mem_a, mem_b = pa["category_name"].endswith("_M"), pb["category_name"].endswith("_M")
+    lo_b = w.n_sms - S.saturation_sms(ca, w.n_sms) if mem_a and not mem_b else 0
+    hi_b = S.saturation_sms(cb, w.n_sms) if mem_b and not mem_a else 0
+    w.split, _ = S.choose_split(ca, cb, w.n_sms, 2, lo_b, hi_b)
     w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
     base = {}
     for name in ("seq_cuda", "seq_slate", "streams", "slate_forced"):

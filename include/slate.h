@@ -304,11 +304,22 @@ int slate_select(uint32_t cat_active, const uint32_t* queue_cats, const uint32_t
                  uint32_t max_bypass, int literal);
 /* SM split for a co-run (reading Q10): SMs for candidate B (A keeps n - s),
  * minimising the fluid-model makespan with grow-on-completion, given solo
- * time curves (sms ascending, ms).  Returns s (multiple of step) and the
- * predicted makespan in *makespan_ms (may be NULL). */
+ * time curves (sms ascending, ms).  s ranges over the multiples of step in
+ * [step, n_sms - step], further limited to [lo_b, hi_b] where those are
+ * non-zero (reading Q29; if that leaves nothing, the bound nearest the range
+ * is used).  Returns s and the predicted makespan in *makespan_ms (may be
+ * NULL). */
 uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t n_a,
                             const uint32_t* sms_b, const double* ms_b, uint32_t n_b,
-                            uint32_t n_sms, uint32_t step, double* makespan_ms);
+                            uint32_t n_sms, uint32_t step, uint32_t lo_b, uint32_t hi_b,
+                            double* makespan_ms);
+/* Reading Q29 (bandwidth saturation cap): the fewest SMs (1..n_sms) on which
+ * a solo curve (sms ascending, ms) comes within frac (0 < frac <= 1) of its
+ * full-chip rate: interp(s) <= interp(n_sms) / frac.  The scheduler caps a
+ * memory-bound co-runner at saturation_sms(curve, 0.9): past that point it
+ * gains little bandwidth but saturates HBM, which stalls the compute-bound
+ * partner's operand loads (measured). */
+uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n, uint32_t n_sms, double frac);
 
 #ifdef __cplusplus
 }

@@ -75,6 +75,26 @@ const KindOps* kind_ops(uint32_t kind) {
   return table[kind].worker_fn ? &table[kind] : nullptr;
 }
 
+// host <-> device clock offset: the host raises flag[i] (mapped memory) at a
+// known host time; the kernel stamps %globaltimer the moment it sees it.
+__global__ void clock_probe_kernel(volatile uint32_t* flag, volatile unsigned long long* stamp, int rounds) {
+  if (threadIdx.x || blockIdx.x) return;
+  for (int i = 0; i < rounds; ++i) {
+    flag[2 * i + 1] = 1;                       // ready for round i
+    __threadfence_system();
+    while (flag[2 * i] == 0) {
+    }
+    stamp[i] = globaltimer();
+    __threadfence_system();
+  }
+}
+
+cudaError_t launch_clock_probe(volatile uint32_t* flag, volatile unsigned long long* stamp, int rounds,
+                               cudaStream_t st) {
+  clock_probe_kernel<<<1, 32, 0, st>>>(flag, stamp, rounds);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_calibrate(uint32_t* out, uint32_t blocks, uint32_t spin_ns, cudaStream_t st) {
   calibrate_kernel<<<blocks, 64, 0, st>>>(out, spin_ns);
   return cudaGetLastError();

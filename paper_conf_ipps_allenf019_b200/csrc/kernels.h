@@ -82,5 +82,7 @@ struct KindOps {
 
 const KindOps* kind_ops(uint32_t kind);   // nullptr if the kind is not built
 cudaError_t launch_calibrate(uint32_t* out, uint32_t blocks, uint32_t spin_ns, cudaStream_t st);
+cudaError_t launch_clock_probe(volatile uint32_t* flag, volatile unsigned long long* stamp, int rounds,
+                               cudaStream_t st);
 
 }  // namespace slate

@@ -73,13 +73,26 @@ int slate_select(uint32_t active, const uint32_t* cats, const uint32_t* bypassed
   return -1;
 }
 
+uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n, uint32_t n_sms, double frac) {
+  const double t_full = interp(sms, ms, n, double(n_sms));
+  for (uint32_t s = 1; s <= n_sms; ++s)
+    if (interp(sms, ms, n, double(s)) <= t_full / frac) return s;
+  return n_sms;
+}
+
 uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, const uint32_t* sms_b,
-                            const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t step, double* makespan_ms) {
+                            const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
+                            uint32_t hi_b, double* makespan_ms) {
   if (step == 0) step = 1;
   double best_t = std::numeric_limits<double>::infinity();
   uint32_t best_s = n_sms / 2;
   const double ta_full = interp(sms_a, ms_a, n_a, n_sms), tb_full = interp(sms_b, ms_b, n_b, n_sms);
-  for (uint32_t s = step; s + step <= n_sms; s += step) {
+  std::vector<uint32_t> cands;
+  for (uint32_t s = step; s + step <= n_sms; s += step)
+    if ((!lo_b || s >= lo_b) && (!hi_b || s <= hi_b)) cands.push_back(s);
+  if (cands.empty())   // the bounds exclude every candidate: the bound nearest the range
+    cands.push_back(std::min(std::max(step, lo_b ? lo_b : step), n_sms - step));
+  for (uint32_t s : cands) {
     const double ta = interp(sms_a, ms_a, n_a, double(n_sms - s));
     const double tb = interp(sms_b, ms_b, n_b, double(s));
     // fluid model: the first to finish hands its SMs to the other

@@ -43,6 +43,8 @@ Server::~Server() {
   }
   cv_.notify_all();
   if (poller_.joinable()) poller_.join();
+  clk_stop_.store(true);
+  if (clock_.joinable()) clock_.join();
 }
 
 double Server::now_us() const {
@@ -112,12 +114,108 @@ int Server::init(std::string* err) {
   CK(cudaMemset(d_ctrl_pool_, 0, 128 * kQueues));
   for (int i = kQueues - 1; i >= 0; --i) free_ctrl_.push_back(i);
 
+  {
+    CK(cudaHostAlloc((void**)&clk_flag_, 64 * sizeof(uint32_t), cudaHostAllocMapped));
+    CK(cudaHostAlloc((void**)&clk_stamp_, 32 * sizeof(unsigned long long), cudaHostAllocMapped));
+    CK(cudaHostGetDevicePointer((void**)&clk_dflag_, (void*)clk_flag_, 0));
+    CK(cudaHostGetDevicePointer((void**)&clk_dstamp_, (void*)clk_stamp_, 0));
+    int lo_prio, hi_prio;
+    CK(cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio));
+    CK(cudaStreamCreateWithPriority(&clk_stream_, cudaStreamNonBlocking, lo_prio));
+    clock_ = std::thread([this] { clock_main(); });   // resize latencies use host observation until anchored
+  }
   peak_hbm_ = env_double("SLATE_PEAK_HBM_GBPS", 6650.0);
   peak_fp32_ = env_double("SLATE_PEAK_FP32_GFLOPS", 2.0 * 128 * prop.multiProcessorCount * (prop.clockRate / 1e6));
   peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
   standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
+  saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.9);   // reading Q29 (1.0: no cap)
   poller_ = std::thread([this] { poller_main(); });
   return SLATE_OK;
+}
+
+// host <-> device clock: a mapped-memory ping-pong gives one
+// anchor -- the smallest (device stamp - host raise time) over 32 rounds, i.e.
+// the offset plus the one-way host->device latency (< 1 us).  %globaltimer
+// drifts against the host's steady clock at a constant rate (measured ~ -33 ppm,
+// tools/probe/clock_drift.cu), so a background thread keeps re-anchoring and the
+// mapping is a least-squares line through the recent anchors.  Resize latencies
+// are device completion stamps minus the host's resize call mapped through it.
+int Server::clock_anchor(double* th_out, double* off_out) {
+  const int rounds = 32;
+  for (int i = 0; i < 2 * rounds; ++i) clk_flag_[i] = 0;
+  for (int i = 0; i < rounds; ++i) clk_stamp_[i] = 0;
+  if (launch_clock_probe(clk_dflag_, clk_dstamp_, rounds, clk_stream_) != cudaSuccess) return SLATE_ECUDA;
+  double best = 1e300, th_best = 0;
+  bool released = false;
+  for (int i = 0; i < rounds; ++i) {
+    // the probe may wait behind persistent workers for a free CTA slot
+    uint32_t spins = 0;
+    while (clk_flag_[2 * i + 1] == 0) {
+      if (clk_stop_.load()) {   // let a started probe run to its end
+        for (int j = 0; j < rounds; ++j) clk_flag_[2 * j] = 1;
+        released = true;
+        break;
+      }
+      if (++spins > 1000) std::this_thread::sleep_for(std::chrono::microseconds(20));
+    }
+    if (released) break;
+    const double th = now_us();
+    clk_flag_[2 * i] = 1;
+    while (clk_stamp_[i] == 0) {
+    }
+    if (!clk_base_ns_) clk_base_ns_ = clk_stamp_[i];
+    const double off = double(int64_t(clk_stamp_[i] - clk_base_ns_)) * 1e-3 - th;
+    if (off < best) {
+      best = off;
+      th_best = th;
+    }
+  }
+  if (cudaStreamSynchronize(clk_stream_) != cudaSuccess || released) return SLATE_ECUDA;
+  *th_out = th_best;
+  *off_out = best;
+  return SLATE_OK;
+}
+
+bool Server::host_to_dev_us(double t, double* out) const {
+  std::lock_guard<std::mutex> g(clk_mu_);
+  if (clk_anchors_.empty()) return false;
+  *out = t + clk_a_ + clk_b_ * (t - clk_tref_);
+  return true;
+}
+
+void Server::clock_main() {
+  cudaSetDevice(device_);
+  int n = 0;
+  while (!clk_stop_.load()) {
+    double th, off;
+    if (clock_anchor(&th, &off) == SLATE_OK) {
+      std::lock_guard<std::mutex> g(clk_mu_);
+      clk_anchors_.emplace_back(th, off);
+      if (clk_anchors_.size() > 24) clk_anchors_.pop_front();
+      double mt = 0, mo = 0;
+      for (auto& a : clk_anchors_) {
+        mt += a.first;
+        mo += a.second;
+      }
+      mt /= clk_anchors_.size();
+      mo /= clk_anchors_.size();
+      double sxx = 0, sxy = 0;
+      for (auto& a : clk_anchors_) {
+        sxx += (a.first - mt) * (a.first - mt);
+        sxy += (a.first - mt) * (a.second - mo);
+      }
+      clk_tref_ = mt;
+      clk_a_ = mo;
+      clk_b_ = sxx > 0 ? sxy / sxx : 0.0;
+      if (std::getenv("SLATE_DEBUG"))
+        fprintf(stderr, "[slate] clock anchor %d: off %.3f us, drift %.2f ppm\n", n, off, clk_b_ * 1e6);
+    }
+    ++n;
+    // dense anchors first (the drift rate), then a slow refresh
+    const int wait_ms = n < 8 ? 50 : 250;
+    for (int i = 0; i < wait_ms && !clk_stop_.load(); i += 10)
+      std::this_thread::sleep_for(std::chrono::milliseconds(10));
+  }
 }
 
 slate_info Server::info() const {
@@ -671,9 +769,18 @@ void Server::schedule() {
         std::vector<double> ta, tb;
         for (int i = int(pa->n_curve) - 1; i >= 0; --i) { sa.push_back(pa->curve_sms[i]); ta.push_back(pa->curve_ms[i]); }
         for (int i = int(pb->n_curve) - 1; i >= 0; --i) { sb.push_back(pb->curve_sms[i]); tb.push_back(pb->curve_ms[i]); }
-        // curves are stored in descending SM order; interp wants ascending
+        // curves are stored in descending SM order; interp wants ascending.
+        // Reading Q29: a memory-bound tenant paired with a compute-bound one gets
+        // no more SMs than it needs for 90% of its full-chip bandwidth.
+        const bool memA = catA >= 3, memB = category_of(HB) >= 3;
+        uint32_t lo_b = 0, hi_b = 0;
+        if (memB && !memA)
+          hi_b = slate_saturation_sms(sb.data(), tb.data(), uint32_t(sb.size()), uint32_t(n_sms_), saturation_frac_);
+        if (memA && !memB)
+          lo_b = uint32_t(n_sms_) -
+                 slate_saturation_sms(sa.data(), ta.data(), uint32_t(sa.size()), uint32_t(n_sms_), saturation_frac_);
         s = slate_choose_split(sa.data(), ta.data(), uint32_t(sa.size()), sb.data(), tb.data(), uint32_t(sb.size()),
-                               uint32_t(n_sms_), 2, nullptr);
+                               uint32_t(n_sms_), 2, lo_b, hi_b, nullptr);
       }
     }
     const uint32_t old_lo = A.lo, old_hi = A.hi;
@@ -792,7 +899,19 @@ void Server::poll_once() {
         for (auto it = L.pending_resize.begin(); it != L.pending_resize.end();) {
           const bool seen = it->kind == 1 ? (m.shrink_epoch >= it->epoch) : (m.join_epoch >= it->epoch);
           if (seen) {
-            L.resize_us[it->idx] = t - it->t0_us;
+            // completion time on the device clock (the last retire / the first join),
+            // start time = the host's resize call mapped onto the device clock
+            const unsigned long long done_ns = it->kind == 1 ? m.shrink_ns : m.join_ns;
+            double t0_dev;
+            if (clk_base_ns_ && host_to_dev_us(it->t0_us, &t0_dev)) {
+              const double dev_done_us = double(int64_t(done_ns - clk_base_ns_)) * 1e-3;
+              L.resize_us[it->idx] = std::max(0.0, dev_done_us - t0_dev);
+            } else {
+              L.resize_us[it->idx] = t - it->t0_us;
+            }
+            if (std::getenv("SLATE_DEBUG"))
+              fprintf(stderr, "[slate] resize kind %d epoch %u: %.3f us on the device clock, %.3f us host-observed\n",
+                      it->kind, it->epoch, L.resize_us[it->idx], t - it->t0_us);
             it = L.pending_resize.erase(it);
           } else {
             ++it;

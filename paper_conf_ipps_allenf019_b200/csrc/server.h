@@ -4,6 +4,7 @@
 // the kernel profile table.  Used in-process by libslate and by the `slated`
 // daemon; no torch types, no Python.
 #pragma once
+#include <atomic>
 #include <condition_variable>
 #include <cstdint>
 #include <deque>
@@ -105,6 +106,21 @@ class Server {
   int run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t lo, uint32_t hi, int reps, double* ms,
                 std::string* err);
   double now_us() const;
+  // host steady clock <-> device %globaltimer (they drift apart ~30 ppm, linearly)
+  int clock_anchor(double* th, double* off);
+  void clock_main();
+  bool host_to_dev_us(double t_host_us, double* t_dev_us) const;   // t_dev relative to clk_base_ns_
+  volatile uint32_t* clk_flag_ = nullptr;
+  volatile unsigned long long* clk_stamp_ = nullptr;
+  uint32_t* clk_dflag_ = nullptr;
+  unsigned long long* clk_dstamp_ = nullptr;
+  cudaStream_t clk_stream_ = nullptr;
+  unsigned long long clk_base_ns_ = 0;
+  mutable std::mutex clk_mu_;
+  std::deque<std::pair<double, double>> clk_anchors_;   // (host us, device - host us)
+  double clk_a_ = 0, clk_b_ = 0, clk_tref_ = 0;
+  std::atomic<bool> clk_stop_{false};
+  std::thread clock_;
   bool launch_done_events(Launch& L);
   int alloc_slot();
   void free_slot(int slot);
@@ -136,6 +152,7 @@ class Server {
 
   double peak_hbm_ = 6650.0, peak_fp32_ = 74400.0, peak_tc_ = 1590.0;
   uint32_t standby_timeout_ns_ = 200000;
+  double saturation_frac_ = 0.9;
 
   mutable std::mutex mu_;
   std::condition_variable cv_;       // state changes (completion, activation)

@@ -141,12 +141,15 @@ _lib.slate_policy.argtypes = [c_u32, c_u32, ctypes.c_int]
 _lib.slate_select.restype = ctypes.c_int
 _lib.slate_select.argtypes = [c_u32, _P(c_u32), _P(c_u32), c_u32, c_u32, ctypes.c_int]
 _lib.slate_choose_split.restype = c_u32
-_lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c_f64), c_u32, c_u32, c_u32, _P(c_f64)]
+_lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c_f64), c_u32, c_u32, c_u32, c_u32,
+                                    c_u32, _P(c_f64)]
+_lib.slate_saturation_sms.restype = c_u32
+_lib.slate_saturation_sms.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_u32, c_f64]
 
 EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffer", "slate_unshare_buffer",
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
-            "slate_choose_split", "slate_serve", "slate_kind_geometry"]
+            "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -270,15 +273,22 @@ def select(active, queue, bypassed=None, max_bypass=4, literal=False):
     return None if r < 0 else r
 
 
-def choose_split(curve_a, curve_b, n_sms, step=2):
-    ka, kb = sorted(curve_a), sorted(curve_b)
-    sa = (c_u32 * len(ka))(*ka)
-    ta = (c_f64 * len(ka))(*[curve_a[k] for k in ka])
-    sb = (c_u32 * len(kb))(*kb)
-    tb = (c_f64 * len(kb))(*[curve_b[k] for k in kb])
+def _curve(c):
+    k = sorted(c)
+    return (c_u32 * len(k))(*k), (c_f64 * len(k))(*[c[x] for x in k]), len(k)
+
+
+def choose_split(curve_a, curve_b, n_sms, step=2, lo_b=0, hi_b=0):
+    sa, ta, na = _curve(curve_a)
+    sb, tb, nb = _curve(curve_b)
     t = c_f64()
-    s = _lib.slate_choose_split(sa, ta, len(ka), sb, tb, len(kb), n_sms, step, ctypes.byref(t))
+    s = _lib.slate_choose_split(sa, ta, na, sb, tb, nb, n_sms, step, lo_b, hi_b, ctypes.byref(t))
     return s, t.value
+
+
+def saturation_sms(curve, n_sms, frac=0.9):
+    sc, tc, nc = _curve(curve)
+    return _lib.slate_saturation_sms(sc, tc, nc, n_sms, frac)
 
 
 # ------------------------------------------------------------------ per-kind marshalling

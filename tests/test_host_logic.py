@@ -84,6 +84,24 @@ def test_choose_split_matches_oracle(S):
         assert s1 == s2 or abs(OS.corun_makespan(ca, cb, 148, s1) - t2) <= 1e-9 * t2
 
 
+def test_choose_split_bounds_and_saturation_match_oracle(S):
+    rng = random.Random(11)
+    pts = [148, 111, 74, 49, 37, 18]
+    for _ in range(200):
+        knee_a, knee_b = rng.uniform(10, 148), rng.uniform(10, 148)
+        ca = {s: rng.uniform(0.2, 5) * max(1.0, knee_a / s) for s in pts}
+        cb = {s: rng.uniform(0.2, 5) * max(1.0, knee_b / s) for s in pts}
+        for c in (ca, cb):
+            frac = rng.choice([0.5, 0.8, 0.9, 1.0])
+            assert S.saturation_sms(c, 148, frac) == OS.saturation_sms(c, 148, frac)
+        lo = rng.choice([0, 0, rng.randrange(1, 148)])
+        hi = rng.choice([0, 0, rng.randrange(1, 148)])
+        s1, t1 = S.choose_split(ca, cb, 148, 2, lo, hi)
+        s2, t2 = OS.choose_split(ca, cb, 148, 2, lo, hi)
+        assert abs(t1 - t2) <= 1e-9 * t2
+        assert s1 == s2 or abs(OS.corun_makespan(ca, cb, 148, s1) - t2) <= 1e-9 * t2
+
+
 def test_kind_geometry(S):
     assert S.kind_geometry(S.KIND_TRIAD) == (1, 1024)
     assert S.kind_geometry(S.KIND_SGEMM_NAIVE) == (16, 16)

@@ -95,6 +95,28 @@ def test_split_fluid_model():
     assert S.interp_time(curve_a, 148) == 1.0 and S.interp_time(curve_a, 200) == 1.0
 
 
+def test_saturation_cap_reading_q29():
+    # throughput linear between (37, 1/2T) and (74, 1/T): rate(s) = s / (74 T) there,
+    # so rate >= 0.9 / T first holds at s = ceil(0.9 * 74) = 67
+    curve = {148: 1.0, 74: 1.0, 37: 2.0}
+    assert S.saturation_sms(curve, 148, 0.9) == 67
+    assert S.saturation_sms(curve, 148, 1.0) == 74
+    # a linearly scaling kernel needs 90% of the chip for 90% of its rate
+    lin = {k: 148.0 / k for k in (37, 74, 148)}
+    assert S.saturation_sms(lin, 148, 0.9) == 134          # ceil(0.9 * 148)
+    # bounds restrict the split; an empty window falls back to the nearest bound
+    curve_a = {s: 148.0 / s for s in (18, 37, 74, 111, 148)}
+    curve_b = {s: max(1.0, 74.0 / s) for s in (18, 37, 74, 111, 148)}
+    s_free, _ = S.choose_split(curve_a, curve_b, 148)
+    s_cap, t_cap = S.choose_split(curve_a, curve_b, 148, hi_b=40)
+    assert s_free > 40 and s_cap == 40
+    assert abs(t_cap - S.corun_makespan(curve_a, curve_b, 148, 40)) < 1e-12
+    s_lo, _ = S.choose_split(curve_a, curve_b, 148, lo_b=100)
+    assert s_lo >= 100 and s_lo % 2 == 0
+    assert S.choose_split(curve_a, curve_b, 148, lo_b=147)[0] == 146
+    assert S.choose_split(curve_a, curve_b, 148, hi_b=1)[0] == 2
+
+
 def test_metrics_closed_forms():
     # P10: perfect overlap of equal jobs, no slowdown -> G = 2, STP = 2, ANTT = 1
     assert M.gain([1, 1], [1, 1]) == 2.0

@@ -1,5 +1,6 @@
 """Diagnostic: C3 pair-job makespan under forced splits (copy on the top s SMs)."""
 import json
+import os
 import sys
 
 import torch
@@ -18,7 +19,8 @@ w.n_sms = 148
 w.arrival_ms = 0.25 * pa["solo_ms"] * w.a.reps
 seq = bench.median_schedule("seq_cuda", w, sA, sB, kA, kB, S, flush, 3)[0]
 out = {"seq_cuda_ms": seq}
-for s_b in (24, 32, 40, 48, 56, 64, 74):
+print("seq_cuda_ms", round(seq, 3), "gemm solo", round(pa["solo_ms"], 3), flush=True)
+for s_b in [int(x) for x in os.environ.get("SLATE_SWEEP_SPLITS", "24,32,40,48,56,64,72,80").split(",")]:
     w.split = s_b
     bench.run_schedule("slate_forced", w, sA, sB, kA, kB, S)
     r = bench.median_schedule("slate_forced", w, sA, sB, kA, kB, S, flush, 3)
@@ -28,4 +30,4 @@ for s_b in (24, 32, 40, 48, 56, 64, 74):
                 "resize_us": [v for q in r[3] + r[4] for v in q["resize_us"]],
                 "topups": sum(q["n_topups"] for q in r[3] + r[4])}
     print(s_b, out[s_b], flush=True)
-json.dump(out, open("gpurun_out/c3_sweep.json", "w"), indent=1)
+json.dump(out, open(os.environ.get("SLATE_SWEEP_OUT", "gpurun_out/c3_sweep.json"), "w"), indent=1)
