@@ -350,8 +350,10 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     # the split the server's AUTO placement takes (reading Q10 + the Q29 saturation cap)
     ca, cb = dict(zip(pa["curve_sms"], pa["curve_ms"])), dict(zip(pb["curve_sms"], pb["curve_ms"]))
     mem_a, mem_b = pa["category_name"].endswith("_M"), pb["category_name"].endswith("_M")
-    lo_b = w.n_sms - S.saturation_sms(ca, w.n_sms) if mem_a and not mem_b else 0
-    hi_b = S.saturation_sms(cb, w.n_sms) if mem_b and not mem_a else 0
+    frac = float(os.environ.get("SLATE_SATURATION_FRAC", "0.95"))
+    cap = frac < 1.0
+    lo_b = w.n_sms - S.saturation_sms(ca, w.n_sms, frac) if cap and mem_a and not mem_b else 0
+    hi_b = S.saturation_sms(cb, w.n_sms, frac) if cap and mem_b and not mem_a else 0
     w.split, _ = S.choose_split(ca, cb, w.n_sms, 2, lo_b, hi_b)
     w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
     base = {}

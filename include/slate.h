@@ -316,9 +316,10 @@ uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t 
 /* Reading Q29 (bandwidth saturation cap): the fewest SMs (1..n_sms) on which
  * a solo curve (sms ascending, ms) comes within frac (0 < frac <= 1) of its
  * full-chip rate: interp(s) <= interp(n_sms) / frac.  The scheduler caps a
- * memory-bound co-runner at saturation_sms(curve, 0.9): past that point it
- * gains little bandwidth but saturates HBM, which stalls the compute-bound
- * partner's operand loads (measured). */
+ * memory-bound co-runner at saturation_sms(curve, f), f = SLATE_SATURATION_FRAC
+ * in the server's environment (default 0.95, 1.0 = no cap): past that point it
+ * gains little bandwidth but raises the HBM latency its compute-bound partner
+ * sees. */
 uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n, uint32_t n_sms, double frac);
 
 #ifdef __cplusplus

@@ -82,7 +82,7 @@ slate_status slate_kind_geometry(uint32_t kind, uint32_t* tile_m, uint32_t* tile
     case SLATE_KIND_STENCIL2D: *tile_m = 8; *tile_n = 32; return SLATE_OK;
     case SLATE_KIND_GEMM_BF16: {
       const slate::KindOps* o = slate::kind_ops(kind);
-      *tile_m = 128;
+      *tile_m = o && o->tile_m ? o->tile_m : 128;
       *tile_n = o && o->tile_n ? o->tile_n : 128;
       return SLATE_OK;
     }

@@ -128,7 +128,7 @@ int Server::init(std::string* err) {
   peak_fp32_ = env_double("SLATE_PEAK_FP32_GFLOPS", 2.0 * 128 * prop.multiProcessorCount * (prop.clockRate / 1e6));
   peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
   standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
-  saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.9);   // reading Q29 (1.0: no cap)
+  saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.95);   // reading Q29 (1.0: no cap)
   poller_ = std::thread([this] { poller_main(); });
   return SLATE_OK;
 }
@@ -369,11 +369,12 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     }
     case SLATE_KIND_GEMM_BF16: {
       auto a = static_cast<const slate_args_gemm*>(d->args);
-      const uint32_t tn = k.ops->tile_n ? k.ops->tile_n : 128;
-      if (a->m % 128 || a->n % tn || a->k % 64 || a->k == 0) return fail("gemm_bf16 needs m % 128, n % tile_n, k % 64 == 0");
+      const uint32_t tn = k.ops->tile_n ? k.ops->tile_n : 128, tm = k.ops->tile_m ? k.ops->tile_m : 128;
+      if (a->m % tm || a->n % tn || a->k % 64 || a->k == 0)
+        return fail("gemm_bf16 needs m % tile_m, n % tile_n, k % 64 == 0 (slate_kind_geometry)");
       if (!al(a->A) || !al(a->B) || !al(a->C)) return fail("gemm arrays must be 16-byte aligned");
       g[0] = a->n / tn;
-      g[1] = a->m / 128;
+      g[1] = a->m / tm;
       break;
     }
     default:
@@ -771,12 +772,13 @@ void Server::schedule() {
         for (int i = int(pb->n_curve) - 1; i >= 0; --i) { sb.push_back(pb->curve_sms[i]); tb.push_back(pb->curve_ms[i]); }
         // curves are stored in descending SM order; interp wants ascending.
         // Reading Q29: a memory-bound tenant paired with a compute-bound one gets
-        // no more SMs than it needs for 90% of its full-chip bandwidth.
+        // no more SMs than it needs for 95% of its full-chip bandwidth
+        // (SLATE_SATURATION_FRAC; 1.0 turns the cap off).
         const bool memA = catA >= 3, memB = category_of(HB) >= 3;
         uint32_t lo_b = 0, hi_b = 0;
-        if (memB && !memA)
+        if (saturation_frac_ < 1.0 && memB && !memA)
           hi_b = slate_saturation_sms(sb.data(), tb.data(), uint32_t(sb.size()), uint32_t(n_sms_), saturation_frac_);
-        if (memA && !memB)
+        if (saturation_frac_ < 1.0 && memA && !memB)
           lo_b = uint32_t(n_sms_) -
                  slate_saturation_sms(sa.data(), ta.data(), uint32_t(sa.size()), uint32_t(n_sms_), saturation_frac_);
         s = slate_choose_split(sa.data(), ta.data(), uint32_t(sa.size()), sb.data(), tb.data(), uint32_t(sb.size()),

@@ -152,7 +152,7 @@ class Server {
 
   double peak_hbm_ = 6650.0, peak_fp32_ = 74400.0, peak_tc_ = 1590.0;
   uint32_t standby_timeout_ns_ = 200000;
-  double saturation_frac_ = 0.9;
+  double saturation_frac_ = 0.95;
 
   mutable std::mutex mu_;
   std::condition_variable cv_;       // state changes (completion, activation)

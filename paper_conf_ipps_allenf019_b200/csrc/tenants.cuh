@@ -107,10 +107,16 @@ struct Triad : TenantBase {
 struct Copy : TenantBase {
   using Args = slate_args_copy;
   static constexpr int kThreads = 128;
-  static constexpr int kStages = 4;
+#ifndef SLATE_COPY_STAGES
+#define SLATE_COPY_STAGES 4
+#endif
+#ifndef SLATE_COPY_SMEM_PAD
+#define SLATE_COPY_SMEM_PAD 0
+#endif
+  static constexpr int kStages = SLATE_COPY_STAGES;
   static constexpr int kBlockBytes = 16384;
   static constexpr int kHdr = 128;                       // barriers + parity word
-  static constexpr int kSmem = kHdr + kStages * kBlockBytes;
+  static constexpr int kSmem = kHdr + kStages * kBlockBytes + SLATE_COPY_SMEM_PAD;
   static constexpr int kSmemStandalone = kHdr + kBlockBytes;
   static constexpr bool kHasInit = true, kLookahead = true, kHasFini = true;
 

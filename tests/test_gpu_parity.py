@@ -28,7 +28,7 @@ CASES = {
     "stencil_float": lambda: make_stencil(8 * 37 + 3, 32 * 9 + 5, 109),
     "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
     "gemm_int": lambda: make_gemm(256, 512, 512, 113, "int"),
-    "gemm_float": lambda: make_gemm(384, 256, 1024, 114),
+    "gemm_float": lambda: make_gemm(768, 512, 1024, 114),
 }
 
 

@@ -106,6 +106,6 @@ def test_kind_geometry(S):
     assert S.kind_geometry(S.KIND_TRIAD) == (1, 1024)
     assert S.kind_geometry(S.KIND_SGEMM_NAIVE) == (16, 16)
     tm, tn = S.kind_geometry(S.KIND_GEMM_BF16)
-    assert tm == 128 and tn in (128, 256)
+    assert (tm, tn) == (256, 256)          # one CTA-pair tile per original block
     with pytest.raises(S.SlateError):
         S.kind_geometry(99)

@@ -11,7 +11,7 @@ from gpu_helpers import make_gemm  # noqa: E402
 from paper_conf_ipps_allenf019_b200 import slate as S  # noqa: E402
 
 s = S.Session(None, 0)
-for (m, n, k, mode) in [(128, 128, 64, "int"), (256, 384, 512, "int"), (384, 256, 1024, "float")]:
+for (m, n, k, mode) in [(256, 256, 64, "int"), (256, 512, 512, "int"), (512, 256, 1024, "float"), (768, 512, 2048, "float")]:
     t = make_gemm(m, n, k, 7, mode)
     ks = s.register_kernel(S.KIND_GEMM_BF16)
     s.sync(s.launch(ks, t.args, t.grid, mode=S.MODE_STANDALONE), timeout_us=10_000_000)
