@@ -42,18 +42,26 @@ constexpr int kTileM = 2 * BM;
 constexpr int kHalfBytes = BM * BK * 2;                 // 16 KiB: one operand half of one slice
 constexpr int kStageBytes = 2 * kHalfBytes;             // A half + B half per CTA
 constexpr int kPairStageBytes = 2 * kStageBytes;        // what the leader's full barrier expects
+#ifndef SLATE_GEMM_TMA_STORE
+#define SLATE_GEMM_TMA_STORE 1
+#endif
 #ifndef SLATE_GEMM_STAGES
-#define SLATE_GEMM_STAGES 7
+#define SLATE_GEMM_STAGES (SLATE_GEMM_TMA_STORE ? 6 : 7)
 #endif
 constexpr int kStages = SLATE_GEMM_STAGES;
 constexpr int kThreads = 256;
 constexpr int kTmemCols = 2 * BN;                       // two fp32 accumulators of BN columns
-constexpr int kSmemBytes = 1024 /*align slack*/ + kStages * kStageBytes + 512 /*barriers*/;
+// epilogue staging for the TMA store of C: per epilogue warp two 32 x 32 fp32
+// boxes (4 KiB each, SWIZZLE_128B), so a box is written while the previous one drains
+constexpr int kBoxBytes = 32 * 32 * 4;
+constexpr int kStagingBytes = SLATE_GEMM_TMA_STORE ? 4 * 2 * kBoxBytes : 0;
+constexpr int kSmemBytes = 1024 /*align slack*/ + kStages * kStageBytes + kStagingBytes + 512 /*barriers*/;
 static_assert(kSmemBytes <= 232448, "shared memory budget");
 
 struct Params {
   CUtensorMap tma_a;     // 64-B aligned members first
   CUtensorMap tma_b;
+  CUtensorMap tma_c;     // fp32 C, boxes of 32 x 32, SWIZZLE_128B (epilogue TMA store)
   slate_args_gemm args;
   uint32_t gx, gy, B, iters, occ, bound_lo, bound_hi, n_ranks, standby_timeout_ns;
   const uint64_t* ctrl;
@@ -270,7 +278,8 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
   // 1024-B aligned ring (SWIZZLE_128B atoms), barriers after it; identical
   // offsets in both CTAs (the pair's MMA reads the peer at the leader's offsets)
   char* ring = reinterpret_cast<char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  Smem& S = *reinterpret_cast<Smem*>(ring + kStages * kStageBytes);
+  char* staging = ring + kStages * kStageBytes;
+  Smem& S = *reinterpret_cast<Smem*>(staging + kStagingBytes);
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t crank = cta_rank();
   const bool leader = crank == 0;
@@ -314,6 +323,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&p.tma_a);
     prefetch_tmap(&p.tma_b);
+    if (SLATE_GEMM_TMA_STORE) prefetch_tmap(&p.tma_c);
   }
   if (warp == 2) {   // TMEM of both SMs, allocated by warp 2 of each CTA
     asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(s_u32(&S.tmem_base)),
@@ -515,6 +525,55 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       }
       uint32_t m0, n0;
       tile_of(g, p.gx, p.gy, m0, n0);
+#if SLATE_GEMM_TMA_STORE
+      // TMEM -> registers -> swizzled staging box -> TMA store (coalesced by the
+      // bulk engine; the LSU only writes shared memory)
+      const uint32_t y0 = m0 + crank * BM + ew * 32;
+#pragma unroll 1
+      for (uint32_t cb = 0; cb < BN / 32; ++cb) {
+        uint32_t r[32];
+        tmem_ld32(tmem + ((ew * 32) << 16) + b * BN + cb * 32, r);
+        char* box = staging + (ew * 2 + (cb & 1)) * kBoxBytes;
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");   // box drained
+        __syncwarp();
+#pragma unroll
+        for (int q = 0; q < 8; ++q)   // row `lane`, 16-B chunk q at chunk position q ^ (row % 8)
+          *reinterpret_cast<uint4*>(box + lane * 128 + ((q ^ (lane & 7)) << 4)) =
+              make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) {
+          uint64_t pol;
+          asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+          asm volatile(
+              "cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
+                  &p.tma_c),
+              "r"(int(n0 + cb * 32)), "r"(int(y0)), "r"(s_u32(box)), "l"(pol)
+              : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+      tc_fence_before();
+      asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps of this CTA read TMEM
+      if (ew == 0 && lane == 0) mbar_arrive_remote(tmem_empty0 + b * 8);
+      if constexpr (kSlate) {
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // this warp's C is written
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (ew == 0 && lane == 0) {
+          // the second CTA of the pair to finish counts the tile
+          __threadfence();
+          uint32_t old;
+          asm volatile("atom.acq_rel.cluster.shared::cluster.add.u32 %0, [%1], 1;"
+                       : "=r"(old)
+                       : "r"(done_cnt0 + b * 4)
+                       : "memory");
+          if (old & 1u) {
+            if (p.cov) atomicAdd(&p.cov[g], 1u);
+            count_done(p, 1u, last_of_task ? 1u : 0u);
+          }
+        }
+      }
+#else
       const uint32_t row = m0 + crank * BM + ew * 32 + lane;
       float* crow = reinterpret_cast<float*>(p.args.C) + uint64_t(row) * p.args.n + n0;
 #pragma unroll 1
@@ -546,8 +605,10 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
           }
         }
       }
+#endif
       ++t;
     }
+    if (SLATE_GEMM_TMA_STORE && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
   __syncthreads();
   cluster_sync();   // no CTA of the pair leaves while the other may still address it
@@ -595,11 +656,25 @@ static bool make_map(CUtensorMap* m, const void* base, uint32_t rows, uint32_t k
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// C: m x n fp32 row-major, boxes of 32 x 32, 128-B swizzle (the epilogue's staging layout)
+static bool make_map_c(CUtensorMap* m, void* base, uint32_t rows, uint32_t n) {
+  EncodeTiledFn enc = encode_fn();
+  if (!enc) return false;
+  const cuuint64_t dims[2] = {n, rows};
+  const cuuint64_t strides[1] = {cuuint64_t(n) * 4};
+  const cuuint32_t box[2] = {32, 32};
+  const cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+             CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) ==
+         CUDA_SUCCESS;
+}
+
 static cudaError_t fill(Params& p, const void* args) {
   std::memset(&p, 0, sizeof(p));
   std::memcpy(&p.args, args, sizeof(p.args));
   if (!make_map(&p.tma_a, reinterpret_cast<const void*>(p.args.A), p.args.m, p.args.k) ||
-      !make_map(&p.tma_b, reinterpret_cast<const void*>(p.args.B), p.args.n, p.args.k))
+      !make_map(&p.tma_b, reinterpret_cast<const void*>(p.args.B), p.args.n, p.args.k) ||
+      !make_map_c(&p.tma_c, reinterpret_cast<void*>(p.args.C), p.args.m, p.args.n))
     return cudaErrorInvalidValue;
   return cudaSuccess;
 }
