@@ -122,7 +122,8 @@ int Server::init(std::string* err) {
     int lo_prio, hi_prio;
     CK(cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio));
     CK(cudaStreamCreateWithPriority(&clk_stream_, cudaStreamNonBlocking, lo_prio));
-    clock_ = std::thread([this] { clock_main(); });   // resize latencies use host observation until anchored
+    // resize latencies use host observation until anchored (and for good with SLATE_CLOCK_SYNC=0)
+    if (env_double("SLATE_CLOCK_SYNC", 1.0) != 0.0) clock_ = std::thread([this] { clock_main(); });
   }
   peak_hbm_ = env_double("SLATE_PEAK_HBM_GBPS", 6650.0);
   peak_fp32_ = env_double("SLATE_PEAK_FP32_GFLOPS", 2.0 * 128 * prop.multiProcessorCount * (prop.clockRate / 1e6));
@@ -146,23 +147,22 @@ int Server::clock_anchor(double* th_out, double* off_out) {
   for (int i = 0; i < rounds; ++i) clk_stamp_[i] = 0;
   if (launch_clock_probe(clk_dflag_, clk_dstamp_, rounds, clk_stream_) != cudaSuccess) return SLATE_ECUDA;
   double best = 1e300, th_best = 0;
-  bool released = false;
-  for (int i = 0; i < rounds; ++i) {
+  bool ok = true;
+  for (int i = 0; i < rounds && ok; ++i) {
     // the probe may wait behind persistent workers for a free CTA slot
+    const double t_wait = now_us();
     uint32_t spins = 0;
-    while (clk_flag_[2 * i + 1] == 0) {
-      if (clk_stop_.load()) {   // let a started probe run to its end
-        for (int j = 0; j < rounds; ++j) clk_flag_[2 * j] = 1;
-        released = true;
-        break;
-      }
+    while (clk_flag_[2 * i + 1] == 0 && clk_stamp_[i] == 0) {
+      if (clk_stop_.load() || now_us() - t_wait > 200e3) { ok = false; break; }
       if (++spins > 1000) std::this_thread::sleep_for(std::chrono::microseconds(20));
     }
-    if (released) break;
+    if (!ok) break;
     const double th = now_us();
     clk_flag_[2 * i] = 1;
     while (clk_stamp_[i] == 0) {
+      if (now_us() - th > 50e3) { ok = false; break; }
     }
+    if (!ok || clk_stamp_[i] == 1ull) { ok = false; break; }   // the probe timed out
     if (!clk_base_ns_) clk_base_ns_ = clk_stamp_[i];
     const double off = double(int64_t(clk_stamp_[i] - clk_base_ns_)) * 1e-3 - th;
     if (off < best) {
@@ -170,7 +170,9 @@ int Server::clock_anchor(double* th_out, double* off_out) {
       th_best = th;
     }
   }
-  if (cudaStreamSynchronize(clk_stream_) != cudaSuccess || released) return SLATE_ECUDA;
+  if (!ok)
+    for (int j = 0; j < 2 * rounds; ++j) clk_flag_[j] = 1;   // let the probe finish
+  if (cudaStreamSynchronize(clk_stream_) != cudaSuccess || !ok) return SLATE_ECUDA;
   *th_out = th_best;
   *off_out = best;
   return SLATE_OK;
@@ -185,10 +187,12 @@ bool Server::host_to_dev_us(double t, double* out) const {
 
 void Server::clock_main() {
   cudaSetDevice(device_);
-  int n = 0;
+  int n = 0, fails = 0;
   while (!clk_stop_.load()) {
     double th, off;
-    if (clock_anchor(&th, &off) == SLATE_OK) {
+    if (clock_anchor(&th, &off) != SLATE_OK) {
+      if (++fails > 8) return;   // e.g. under a kernel-replaying profiler: keep host-observed latencies
+    } else {
       std::lock_guard<std::mutex> g(clk_mu_);
       clk_anchors_.emplace_back(th, off);
       if (clk_anchors_.size() > 24) clk_anchors_.pop_front();
