@@ -302,60 +302,88 @@ using SpmvCsr = SpmvCsrT<8, 4>;
 // the Abramowitz-Stegun polynomial (|error| < 7.5e-8), put by 1 - CND; each
 // option priced under n_scen volatilities (reading Q16) and the mean written.
 // Thread t of block x prices options 4(x*256+t)..+3.
+// B200 has one MUFU (SFU) op per 2 FP32 lanes' worth of issue less than B300, so
+// the body is arranged around MUFU count (5 -> 2.25 per option-scenario),
+// with exact identities: 1/(sigma sqrt T) = (1/sigma)(1/sqrt T) with 1/sigma
+// shared by a thread's 4 options; both A&S K = 1/(1 + 0.2316419|d|) from one
+// reciprocal (K1 = u2/(u1 u2), K2 = u1/(u1 u2)); and the density at d2 from the
+// one at d1: exp(-d2^2/2) = exp(-d1^2/2) S / (X e^{-rT}) (d1 sigma sqrt T =
+// ln(S/X) + (r + sigma^2/2) T); the put by put-call parity, put = call + X e^{-rT}
+// - S for every scenario, hence for their mean.
 struct BlackScholes : TenantBase {
   using Args = slate_args_bs;
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 6;       // 40 registers, no spill (non-speculative boundary)
+  static constexpr int kMinBlocks = 4;
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
-  __device__ __forceinline__ static float cnd(float d) {
+  __device__ __forceinline__ static float poly(float K) {
     const float A1 = 0.31938153f, A2 = -0.356563782f, A3 = 1.781477937f, A4 = -1.821255978f, A5 = 1.330274429f;
-    const float RSQRT2PI = 0.39894228040143267794f;
-    const float K = __fdividef(1.0f, __fmaf_rn(0.2316419f, fabsf(d), 1.0f));
-    const float poly = __fmul_rn(K, __fmaf_rn(K, __fmaf_rn(K, __fmaf_rn(K, __fmaf_rn(K, A5, A4), A3), A2), A1));
-    const float c = __fmul_rn(__fmul_rn(RSQRT2PI, __expf(__fmul_rn(-0.5f, __fmul_rn(d, d)))), poly);
-    return d > 0.f ? __fsub_rn(1.0f, c) : c;
+    return __fmul_rn(K, __fmaf_rn(K, __fmaf_rn(K, __fmaf_rn(K, __fmaf_rn(K, A5, A4), A3), A2), A1));
   }
-  __device__ __forceinline__ static void price(float S, float X, float T, float r, const float* sig, uint32_t P,
-                                               float& call, float& put) {
-    const float sqt = sqrtf(T);
-    const float lsx = logf(__fdiv_rn(S, X));
-    const float xd = __fmul_rn(X, expf(__fmul_rn(-r, T)));
-    float cs = 0.f, ps = 0.f;
+  // options o = 0..k-1 of this thread (k = 4, or 1..3 on the ragged tail)
+  template <int k>
+  __device__ __forceinline__ static void price(const float (&S)[4], const float (&X)[4], const float (&T)[4],
+                                               float r, const float* sig, uint32_t P, float (&call)[4],
+                                               float (&put)[4]) {
+    const float RSQRT2PI = 0.39894228040143267794f;
+    float sqt[k], rsqt[k], lsx[k], xd[k], sxd[k], cs[k];
+#pragma unroll
+    for (int o = 0; o < k; ++o) {
+      sqt[o] = sqrtf(T[o]);
+      rsqt[o] = __fdiv_rn(1.0f, sqt[o]);
+      lsx[o] = logf(__fdiv_rn(S[o], X[o]));
+      xd[o] = __fmul_rn(X[o], expf(__fmul_rn(-r, T[o])));
+      sxd[o] = __fdiv_rn(S[o], xd[o]);
+      cs[o] = 0.f;
+    }
     for (uint32_t p = 0; p < P; ++p) {
       const float sg = __ldg(sig + p);
-      const float sst = __fmul_rn(sg, sqt);
-      const float d1 = __fdividef(__fmaf_rn(__fmaf_rn(__fmul_rn(0.5f, sg), sg, r), T, lsx), sst);
-      const float d2 = __fsub_rn(d1, sst);
-      const float n1 = cnd(d1), n2 = cnd(d2);
-      cs = __fadd_rn(cs, __fsub_rn(__fmul_rn(S, n1), __fmul_rn(xd, n2)));
-      ps = __fadd_rn(ps, __fsub_rn(__fmul_rn(xd, __fsub_rn(1.0f, n2)), __fmul_rn(S, __fsub_rn(1.0f, n1))));
+      const float rsg = __fdividef(1.0f, sg);
+      const float hs2 = __fmaf_rn(__fmul_rn(0.5f, sg), sg, r);
+#pragma unroll
+      for (int o = 0; o < k; ++o) {
+        const float sst = __fmul_rn(sg, sqt[o]);
+        const float d1 = __fmul_rn(__fmaf_rn(hs2, T[o], lsx[o]), __fmul_rn(rsg, rsqt[o]));
+        const float d2 = __fsub_rn(d1, sst);
+        const float u1 = __fmaf_rn(0.2316419f, fabsf(d1), 1.0f), u2 = __fmaf_rn(0.2316419f, fabsf(d2), 1.0f);
+        const float q = __fdividef(1.0f, __fmul_rn(u1, u2));
+        const float e1 = __fmul_rn(RSQRT2PI, __expf(__fmul_rn(-0.5f, __fmul_rn(d1, d1))));
+        const float c1 = __fmul_rn(e1, poly(__fmul_rn(u2, q)));
+        const float c2 = __fmul_rn(__fmul_rn(e1, sxd[o]), poly(__fmul_rn(u1, q)));
+        const float n1 = d1 > 0.f ? __fsub_rn(1.0f, c1) : c1;
+        const float n2 = d2 > 0.f ? __fsub_rn(1.0f, c2) : c2;
+        cs[o] = __fadd_rn(cs[o], __fsub_rn(__fmul_rn(S[o], n1), __fmul_rn(xd[o], n2)));
+      }
     }
-    call = __fdiv_rn(cs, float(P));
-    put = __fdiv_rn(ps, float(P));
+#pragma unroll
+    for (int o = 0; o < k; ++o) {
+      call[o] = __fdiv_rn(cs[o], float(P));
+      put[o] = __fadd_rn(call[o], __fsub_rn(xd[o], S[o]));
+    }
   }
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
     const uint64_t v = uint64_t(x) * 256 + threadIdx.x;
     const uint64_t i0 = v * 4;
     const float* sig = reinterpret_cast<const float*>(a.sigmas);
+    float S[4], X[4], T[4], c[4], p[4];
     if (i0 + 4 <= a.n) {
-      const float4 S = __ldcs(reinterpret_cast<const float4*>(a.S) + v);
-      const float4 X = __ldcs(reinterpret_cast<const float4*>(a.X) + v);
-      const float4 T = __ldcs(reinterpret_cast<const float4*>(a.T) + v);
-      float4 c, p;
-      price(S.x, X.x, T.x, a.r, sig, a.n_scen, c.x, p.x);
-      price(S.y, X.y, T.y, a.r, sig, a.n_scen, c.y, p.y);
-      price(S.z, X.z, T.z, a.r, sig, a.n_scen, c.z, p.z);
-      price(S.w, X.w, T.w, a.r, sig, a.n_scen, c.w, p.w);
-      __stcs(reinterpret_cast<float4*>(a.call) + v, c);
-      __stcs(reinterpret_cast<float4*>(a.put) + v, p);
+      const float4 s4 = __ldcs(reinterpret_cast<const float4*>(a.S) + v);
+      const float4 x4 = __ldcs(reinterpret_cast<const float4*>(a.X) + v);
+      const float4 t4 = __ldcs(reinterpret_cast<const float4*>(a.T) + v);
+      S[0] = s4.x; S[1] = s4.y; S[2] = s4.z; S[3] = s4.w;
+      X[0] = x4.x; X[1] = x4.y; X[2] = x4.z; X[3] = x4.w;
+      T[0] = t4.x; T[1] = t4.y; T[2] = t4.z; T[3] = t4.w;
+      price<4>(S, X, T, a.r, sig, a.n_scen, c, p);
+      __stcs(reinterpret_cast<float4*>(a.call) + v, make_float4(c[0], c[1], c[2], c[3]));
+      __stcs(reinterpret_cast<float4*>(a.put) + v, make_float4(p[0], p[1], p[2], p[3]));
     } else {
-      for (uint64_t i = i0; i < a.n && i < i0 + 4; ++i) {
-        float c, p;
-        price(reinterpret_cast<const float*>(a.S)[i], reinterpret_cast<const float*>(a.X)[i],
-              reinterpret_cast<const float*>(a.T)[i], a.r, sig, a.n_scen, c, p);
-        reinterpret_cast<float*>(a.call)[i] = c;
-        reinterpret_cast<float*>(a.put)[i] = p;
+      for (uint64_t i = i0; i < a.n && i < i0 + 4; ++i) {   // ragged tail: one option at a time
+        S[0] = reinterpret_cast<const float*>(a.S)[i];
+        X[0] = reinterpret_cast<const float*>(a.X)[i];
+        T[0] = reinterpret_cast<const float*>(a.T)[i];
+        price<1>(S, X, T, a.r, sig, a.n_scen, c, p);
+        reinterpret_cast<float*>(a.call)[i] = c[0];
+        reinterpret_cast<float*>(a.put)[i] = p[0];
       }
     }
   }
