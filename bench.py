@@ -332,6 +332,46 @@ def median_schedule(name, w, sA, sB, kA, kB, S, flush, reps):
     return rs[len(rs) // 2]
 
 
+def resize_storm(S, sess, job, n_sms, n_resizes=200, per_launch=12, gap_us=100.0, seed=20190520 + 303):
+    """SURVEY §8(d) C3 resize storm: during each GEMM launch, the host alternates a
+    shrink to a random sub-range (>= 16 SMs) and a grow back to all SMs every
+    gap_us, up to `per_launch` times, until n_resizes were issued; each resize's
+    latency is measured by the server on the device clock (reading Q30)."""
+    import random
+    rng = random.Random(seed)
+    k = sess.register_kernel(job.kind)
+    lat = {"shrink": [], "grow": []}
+    issued = 0
+    while issued < n_resizes:
+        lid = sess.launch(k, job.args, job.grid, placement=S.PLACE_CORUN, sm=(0, n_sms - 1))
+        spin_ms(0.05)
+        for i in range(min(per_launch, n_resizes - issued)):
+            if i % 2 == 0:
+                lo = rng.randrange(0, n_sms - 16)
+                hi = rng.randrange(lo + 15, n_sms)
+                if lo == 0 and hi == n_sms - 1:
+                    hi -= 1
+            else:
+                lo, hi = 0, n_sms - 1
+            st = sess.resize(lid, lo, hi)
+            issued += 1
+            if st == S.DONE:
+                break
+            spin_ms(gap_us * 1e-3)
+        sess.resize(lid, 0, n_sms - 1)
+        sess.sync(lid)
+        q = sess.query(lid)
+        for v, kind in zip(q["resize_us"], q["resize_kind"]):
+            lat[kind].append(v)
+
+    def stats(v):
+        return {"n": len(v), "p50": round(statistics.median(v), 2) if v else None,
+                "p99": round(float(np.percentile(v, 99)), 2) if v else None, "max": round(max(v), 2) if v else None}
+    return {"tenant": "gemm_bf16 8192^3, one launch per %d resizes" % per_launch, "resizes_issued": issued,
+            "gap_us": gap_us, "shrink_us": stats(lat["shrink"]), "grow_us": stats(lat["grow"]),
+            "clock": "device %globaltimer mapped to the host clock (DESIGN.md Q30)"}
+
+
 def prof_view(p):
     return {"solo_ms": round(p["solo_ms"], 4), "hbm_gbps": round(p["hbm_gbps"], 1),
             "fp32_gflops": round(p["fp32_gflops"], 1), "tc_tflops": round(p["tc_tflops"], 1),
@@ -504,6 +544,7 @@ def run_slate(args, world, rank, local):
         c3["config"] = C3
         c3["stp"] = r3["schedules"]["slate_corun"]["stp"]
         c3["antt"] = r3["schedules"]["slate_corun"]["antt"]
+        c3["resize_storm"] = resize_storm(S, sA, w3.a, sA.info()["num_sms"])
         del w3
 
     # ---- C4 (configs[3]): four client processes through the slated daemon (rank 0 only)

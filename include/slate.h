@@ -259,9 +259,12 @@ typedef struct {
   uint64_t t_first_ns;     /* %globaltimer at the first task start (device clock) */
   uint64_t t_last_ns;      /* %globaltimer when the last block finished */
   double start_ms, end_ms; /* CUDA-event times of the launch relative to the server's epoch */
-  double resize_us[16];    /* host-observed latency of the first 16 resizes (shrink: until
-                              no worker is live outside the range; grow: until the first
-                              task starts on a new rank); -1 if not observed */
+  double resize_us[16];    /* latency of the first 16 resizes applied while the launch ran
+                              (reading Q30: from the slate_resize call to, for a shrink, the
+                              last worker retiring outside the range, for a grow, the first
+                              worker joining on a new rank; device clock mapped to the host
+                              clock); -1 if not observed (e.g. the launch ended first) */
+  uint8_t resize_kind[16]; /* 1 shrink, 2 grow, 0 none, for each resize_us entry */
 } slate_launch_info;
 
 /* Counters and timing of a launch (copied out).  Errors: ENOTFOUND. */

@@ -246,7 +246,7 @@ uint32_t Server::open_queue() {
   Q->lo = 0;
   Q->hi = uint32_t(n_sms_ - 1);
   cudaStreamCreateWithFlags(&Q->stream, cudaStreamNonBlocking);
-  cudaStreamCreateWithFlags(&Q->aux, cudaStreamNonBlocking);
+  for (cudaStream_t& a : Q->aux) cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking);   // not on the resize path
   const uint32_t id = Q->id;
   queues_[id] = std::move(Q);
   return id;
@@ -261,11 +261,13 @@ int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
   Q.closed = true;
   if (rc == SLATE_OK) {
     cudaStreamSynchronize(Q.stream);
-    cudaStreamSynchronize(Q.aux);
+    for (cudaStream_t a : Q.aux)
+      if (a) cudaStreamSynchronize(a);
     const int slot = int((Q.d_ctrl - d_ctrl_pool_) / 16);
     free_ctrl_.push_back(slot);
     cudaStreamDestroy(Q.stream);
-    cudaStreamDestroy(Q.aux);
+    for (cudaStream_t a : Q.aux)
+      if (a) cudaStreamDestroy(a);
     queues_.erase(it);
   }
   return rc;
@@ -485,7 +487,6 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
   CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
   CK(cudaEventRecord(ev, ctrl_stream_));
   CK(cudaStreamWaitEvent(Q.stream, ev, 0));
-  CK(cudaStreamWaitEvent(Q.aux, ev, 0));
   cudaEventDestroy(ev);
   return SLATE_OK;
 }
@@ -521,9 +522,9 @@ void Server::drain_deferred(Queue& Q) {
 
 int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
   const KindOps* ops = L.k->ops;
-  if (Q.last_topup_end) {   // stream semantics: the predecessor's top-up workers must finish first
-    CK(cudaStreamWaitEvent(Q.stream, Q.last_topup_end, 0));
-  }
+  for (cudaEvent_t e : Q.topup_ends)   // stream semantics: the predecessor's top-up workers finish first
+    CK(cudaStreamWaitEvent(Q.stream, e, 0));
+  Q.topup_ends.clear();
   CK(cudaEventCreate(&L.ev_start));
   cudaEvent_t ev_end;
   CK(cudaEventCreate(&ev_end));
@@ -576,12 +577,37 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
 // queued behind it on the stream picks up the new range by itself); later
 // launches wait for the top-up's end (stream semantics).
 int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
-  if (Q.issued.size() != 1 || !Q.pending.empty() || !Q.deferred.empty()) return SLATE_OK;
-  Launch& R = *launches_[Q.issued.front()];
+  // only the last issued launch can get a top-up (later launches must stay behind
+  // it in stream order); launches before it that finished all their blocks but
+  // are not yet retired by the poller do not count
+  static const bool dbg = std::getenv("SLATE_DEBUG") != nullptr;
+  if (Q.issued.empty() || !Q.pending.empty() || !Q.deferred.empty()) {
+    if (dbg) fprintf(stderr, "[slate] grow: no top-up (issued %zu pending %zu deferred %zu)\n", Q.issued.size(),
+                     Q.pending.size(), Q.deferred.size());
+    return SLATE_OK;
+  }
+  for (size_t i = 0; i + 1 < Q.issued.size(); ++i) {
+    const Launch& E = *launches_[Q.issued[i]];
+    if (E.slot < 0 || !h_mirror_[E.slot].complete) {
+      if (dbg) fprintf(stderr, "[slate] grow: no top-up (an earlier launch is still running)\n");
+      return SLATE_OK;
+    }
+  }
+  Launch& R = *launches_[Q.issued.back()];
   if (R.state != 1 || R.slot < 0 || R.desc.mode == SLATE_MODE_STANDALONE) return SLATE_OK;
-  if (h_mirror_[R.slot].complete) return SLATE_OK;
+  if (h_mirror_[R.slot].complete) {
+    if (dbg) fprintf(stderr, "[slate] grow: no top-up (the launch finished its blocks)\n");
+    return SLATE_OK;
+  }
+  if (dbg) fprintf(stderr, "[slate] grow: top-up for launch %llu on [%u, %u]\n", (unsigned long long)R.id, Q.lo, Q.hi);
   const auto& g = R.desc.grid;
-  CK(cudaStreamWaitEvent(Q.aux, R.ev_start, 0));
+  cudaStream_t aux = Q.aux[Q.aux_next++ % Queue::kAux];
+  cudaEvent_t ev_ctrl;   // the top-up starts after the resize word it must see (and after R started)
+  CK(cudaEventCreateWithFlags(&ev_ctrl, cudaEventDisableTiming));
+  CK(cudaEventRecord(ev_ctrl, ctrl_stream_));
+  CK(cudaStreamWaitEvent(aux, ev_ctrl, 0));
+  cudaEventDestroy(ev_ctrl);
+  CK(cudaStreamWaitEvent(aux, R.ev_start, 0));
   WorkerCommon w{};
   w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = R.B; w.iters = R.iters; w.occ = uint32_t(R.k->occ);
   w.bound_lo = Q.lo; w.bound_hi = Q.hi; w.n_ranks = uint32_t(n_sms_);
@@ -589,10 +615,10 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   w.ctrl = Q.d_ctrl; w.tc = d_tc_ + R.slot; w.mirror = d_mirror_ + R.slot;
   w.cov = reinterpret_cast<uint32_t*>(R.desc.coverage);
   w.rank_of = d_rank_of_;
-  CK(R.k->ops->launch_worker(w, R.args.data(), uint32_t(R.k->occ) * uint32_t(n_sms_), Q.aux));
+  CK(R.k->ops->launch_worker(w, R.args.data(), uint32_t(R.k->occ) * uint32_t(n_sms_), aux));
   cudaEvent_t ev_end, ev_snap;
   CK(cudaEventCreate(&ev_end));
-  CK(cudaEventRecord(ev_end, Q.aux));
+  CK(cudaEventRecord(ev_end, aux));
   R.ev_end.push_back(ev_end);
   CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
   CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
@@ -600,7 +626,7 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
                      cudaMemcpyDeviceToHost, copy_stream_));
   CK(cudaEventRecord(ev_snap, copy_stream_));
   R.ev_done.push_back(ev_snap);
-  Q.last_topup_end = ev_end;
+  Q.topup_ends.push_back(ev_end);
   R.n_topups += 1;
   return SLATE_OK;
 }
@@ -666,10 +692,7 @@ int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_
         if (write_ctrl(A, nlo, nhi, true, err) == SLATE_OK && !A.issued.empty()) {
           Launch& R = *launches_[A.issued.front()];
           R.n_resizes += 1;
-          if (R.resize_us.size() < 16) {
-            R.pending_resize.push_back({A.epoch, 1, t0, int(R.resize_us.size())});
-            R.resize_us.push_back(-1);
-          }
+          track_resize(R, A.epoch, 1, t0);
         }
       }
     } else if (Q.lo != d->sm_lo || Q.hi != d->sm_hi) {
@@ -794,10 +817,7 @@ void Server::schedule() {
     write_ctrl(A, 0, uint32_t(n_sms_) - s - 1, true, &err);   // shrink the running kernel
     if (!A.issued.empty()) {
       Launch& R = *launches_[A.issued.front()];
-      if (R.resize_us.size() < 16) {
-        R.pending_resize.push_back({A.epoch, 1, t0, int(R.resize_us.size())});
-        R.resize_us.push_back(-1);
-      }
+      track_resize(R, A.epoch, 1, t0);
       R.n_resizes += 1;
     }
     (void)old_lo;
@@ -832,10 +852,7 @@ void Server::release(Queue& Q) {
       write_ctrl(A, 0, uint32_t(n_sms_ - 1), true, &err);
       if (!A.issued.empty()) {
         Launch& R = *launches_[A.issued.front()];
-        if (R.resize_us.size() < 16) {
-          R.pending_resize.push_back({A.epoch, 2, t0, int(R.resize_us.size())});
-          R.resize_us.push_back(-1);
-        }
+        track_resize(R, A.epoch, 2, t0);
         R.n_resizes += 1;
       }
       grow_running(A, old_lo, old_hi, &err);
@@ -870,13 +887,66 @@ int Server::resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string
   if (!Q.issued.empty()) {
     Launch& R = *launches_[Q.issued.front()];
     R.n_resizes += 1;
-    if (R.resize_us.size() < 16 && (shrink || grow)) {
-      R.pending_resize.push_back({Q.epoch, shrink ? 1 : 2, t0, int(R.resize_us.size())});
-      R.resize_us.push_back(-1);
-    }
+    if (shrink || grow) track_resize(R, Q.epoch, shrink ? 1 : 2, t0);
   }
   if (grow) rc = grow_running(Q, old_lo, old_hi, err);
   return rc;
+}
+
+// a resize applied while R runs: measured (Q30) for the first 16 of the launch
+void Server::track_resize(Launch& R, uint32_t epoch, int kind, double t0) {
+  if (R.resize_us.size() >= 16) return;
+  queues_[R.queue]->pending_resize.push_back({epoch, kind, t0, R.id, int(R.resize_us.size())});
+  R.resize_us.push_back(-1);
+  R.resize_kind.push_back(uint8_t(kind));
+}
+
+// completion stamp (device ns) -> latency from the host's resize call (Q30)
+void Server::record_resize(const Queue::PendingResize& pr, unsigned long long done_ns, double t) {
+  auto li = launches_.find(pr.lid);
+  if (li == launches_.end()) return;
+  Launch& R = *li->second;
+  double t0_dev;
+  if (clk_base_ns_ && done_ns && host_to_dev_us(pr.t0_us, &t0_dev))
+    R.resize_us[pr.idx] = std::max(0.0, double(int64_t(done_ns - clk_base_ns_)) * 1e-3 - t0_dev);
+  else
+    R.resize_us[pr.idx] = t - pr.t0_us;
+  if (std::getenv("SLATE_DEBUG"))
+    fprintf(stderr, "[slate] resize kind %d epoch %u: %.3f us on the device clock, %.3f us host-observed\n", pr.kind,
+            pr.epoch, R.resize_us[pr.idx], t - pr.t0_us);
+}
+
+// A resize applies to the queue, whichever of its launches is running: a
+// shrink ends when the launch holding workers outside the range has retired
+// them (its mirror's shrink epoch) or has ended altogether (`ended`, its last
+// block's stamp: later launches start inside the range); a grow ends when a
+// worker of any of the queue's launches joined under the new epoch.
+void Server::resolve_resizes(Queue& Q, double t, const Launch* ended) {
+  for (auto it = Q.pending_resize.begin(); it != Q.pending_resize.end();) {
+    unsigned long long done_ns = 0;
+    bool done = false;
+    for (uint64_t lid : Q.issued) {
+      const Launch& L = *launches_[lid];
+      if (L.slot < 0) continue;
+      const HostMirror& m = h_mirror_[L.slot];
+      if (it->kind == 1 ? m.shrink_epoch >= it->epoch : m.join_epoch >= it->epoch) {
+        done_ns = it->kind == 1 ? m.shrink_ns : m.join_ns;
+        done = true;
+        break;
+      }
+      if (it->kind == 1) break;   // only the oldest running launch can hold out-of-range workers
+    }
+    if (!done && ended && it->kind == 1 && ended->slot >= 0) {
+      done_ns = h_mirror_[ended->slot].t_last;
+      done = true;
+    }
+    if (done) {
+      record_resize(*it, done_ns, t);
+      it = Q.pending_resize.erase(it);
+    } else {
+      ++it;
+    }
+  }
 }
 
 // ------------------------------------------------------------------ poller
@@ -897,47 +967,23 @@ void Server::poll_once() {
   std::vector<uint32_t> idle;
   for (auto& kv : queues_) {
     Queue& Q = *kv.second;
-    bool first = true;
+    if (!Q.pending_resize.empty()) resolve_resizes(Q, t, nullptr);
     while (!Q.issued.empty()) {
       Launch& L = *launches_[Q.issued.front()];
-      if (first && L.slot >= 0) {
-        const HostMirror& m = h_mirror_[L.slot];
-        for (auto it = L.pending_resize.begin(); it != L.pending_resize.end();) {
-          const bool seen = it->kind == 1 ? (m.shrink_epoch >= it->epoch) : (m.join_epoch >= it->epoch);
-          if (seen) {
-            // completion time on the device clock (the last retire / the first join),
-            // start time = the host's resize call mapped onto the device clock
-            const unsigned long long done_ns = it->kind == 1 ? m.shrink_ns : m.join_ns;
-            double t0_dev;
-            if (clk_base_ns_ && host_to_dev_us(it->t0_us, &t0_dev)) {
-              const double dev_done_us = double(int64_t(done_ns - clk_base_ns_)) * 1e-3;
-              L.resize_us[it->idx] = std::max(0.0, dev_done_us - t0_dev);
-            } else {
-              L.resize_us[it->idx] = t - it->t0_us;
-            }
-            if (std::getenv("SLATE_DEBUG"))
-              fprintf(stderr, "[slate] resize kind %d epoch %u: %.3f us on the device clock, %.3f us host-observed\n",
-                      it->kind, it->epoch, L.resize_us[it->idx], t - it->t0_us);
-            it = L.pending_resize.erase(it);
-          } else {
-            ++it;
-          }
-        }
-      }
-      first = false;
       if (!launch_done_events(L)) break;
+      if (!Q.pending_resize.empty()) resolve_resizes(Q, t, &L);
       if (L.slot >= 0) {
         std::memcpy(L.snapshot, h_snap_ + size_t(L.slot) * kTaskCtlHeader, kTaskCtlHeader);
         L.has_snapshot = true;
         free_slot(L.slot);
         L.slot = -1;
       }
-      L.pending_resize.clear();
       L.state = 2;
       Q.issued.pop_front();
-      if (Q.last_topup_end && Q.issued.empty()) Q.last_topup_end = nullptr;
+      if (Q.issued.empty()) Q.topup_ends.clear();
       cv_.notify_all();
     }
+    if (Q.issued.empty()) Q.pending_resize.clear();   // nothing left to observe them on
     drain_deferred(Q);
     if (Q.active && Q.issued.empty() && Q.pending.empty() && Q.deferred.empty()) idle.push_back(Q.id);
   }
@@ -1014,7 +1060,10 @@ int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
   }
   out->n_resizes = L.n_resizes;
   out->n_topups = L.n_topups;
-  for (int i = 0; i < 16; ++i) out->resize_us[i] = i < int(L.resize_us.size()) ? L.resize_us[i] : -1.0;
+  for (int i = 0; i < 16; ++i) {
+    out->resize_us[i] = i < int(L.resize_us.size()) ? L.resize_us[i] : -1.0;
+    out->resize_kind[i] = i < int(L.resize_kind.size()) ? L.resize_kind[i] : 0;
+  }
   TaskCtl tc;
   std::memset(&tc, 0, sizeof(tc));
   if (L.desc.mode == SLATE_MODE_STANDALONE) {

@@ -43,9 +43,7 @@ struct Launch {
   bool mirror_complete_seen = false;
   uint32_t n_resizes = 0, n_topups = 0;
   std::vector<double> resize_us;
-  // pending resize measurements: epoch, kind (1 shrink, 2 grow), host t0
-  struct PendingResize { uint32_t epoch; int kind; double t0_us; int idx; };
-  std::vector<PendingResize> pending_resize;
+  std::vector<uint8_t> resize_kind;   // 1 shrink, 2 grow
   unsigned char snapshot[kTaskCtlHeader];   // final TaskCtl header copy
   bool has_snapshot = false;
 };
@@ -53,7 +51,10 @@ struct Launch {
 struct Queue {
   uint32_t id;
   cudaStream_t stream = nullptr;
-  cudaStream_t aux = nullptr;   // top-up launches
+  static constexpr int kAux = 8;
+  cudaStream_t aux[kAux] = {};  // top-up launches (round robin: a top-up whose workers joined runs
+                                // until the launch drains, so top-ups must not queue behind each other)
+  uint32_t aux_next = 0;
   uint64_t* d_ctrl = nullptr;   // the resize word {epoch, lo, hi}
   uint32_t epoch = 0, lo = 0, hi = 0;
   bool active = false;          // holds an SM range
@@ -61,7 +62,11 @@ struct Queue {
   std::deque<uint64_t> pending; // launches waiting for SMs (AUTO/SOLO)
   std::deque<uint64_t> deferred;  // granted SMs but waiting for a control block (stream order)
   std::deque<uint64_t> issued;  // issued, not complete (stream order)
-  cudaEvent_t last_topup_end = nullptr;  // successors must wait for it
+  std::vector<cudaEvent_t> topup_ends;  // top-ups of the last issued launch: successors wait for all
+  // resize latencies being measured (Q30): epoch, kind (1 shrink, 2 grow), host
+  // t0, and where the result goes (launch id, index in its resize_us)
+  struct PendingResize { uint32_t epoch; int kind; double t0_us; uint64_t lid; int idx; };
+  std::vector<PendingResize> pending_resize;
   bool closed = false;
 };
 
@@ -122,6 +127,9 @@ class Server {
   std::atomic<bool> clk_stop_{false};
   std::thread clock_;
   bool launch_done_events(Launch& L);
+  void track_resize(Launch& R, uint32_t epoch, int kind, double t0);
+  void resolve_resizes(Queue& Q, double t_host, const Launch* ended);
+  void record_resize(const Queue::PendingResize& pr, unsigned long long done_ns, double t_host);
   int alloc_slot();
   void free_slot(int slot);
   uint32_t auto_iters(uint32_t B, int occ, uint32_t cap, uint32_t per_worker) const;

@@ -103,11 +103,13 @@ class LaunchInfo(ctypes.Structure):
                 ("sm_lo", c_u32), ("sm_hi", c_u32), ("n_resizes", c_u32), ("n_topups", c_u32),
                 ("workers_started", c_u32), ("coverage_ok", c_u32), ("epoch", c_u32), ("shrink_epoch", c_u32),
                 ("join_epoch", c_u32), ("pad_", c_u32), ("t_first_ns", c_u64), ("t_last_ns", c_u64),
-                ("start_ms", c_f64), ("end_ms", c_f64), ("resize_us", c_f64 * 16)]
+                ("start_ms", c_f64), ("end_ms", c_f64), ("resize_us", c_f64 * 16), ("resize_kind", ctypes.c_uint8 * 16)]
 
     def as_dict(self):
         d = {f[0]: getattr(self, f[0]) for f in self._fields_}
         d["resize_us"] = [v for v in self.resize_us if v >= 0]
+        d["resize_kind"] = [("shrink", "grow")[k - 1] for v, k in zip(self.resize_us, self.resize_kind)
+                            if v >= 0 and k in (1, 2)]
         return d
 
 
