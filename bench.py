@@ -194,38 +194,54 @@ def run_reference(args, world, rank):
 
 # ------------------------------------------------------------------ clocks
 class Clocks:
+    """SM clock and clock-event reasons sampled through NVML every 10 ms while
+    the timed region runs (a thread; nvidia-smi -lms buffers its output and
+    lost the samples of sub-second regions)."""
+
+    NAMES = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+             ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+             ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+             ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"),
+             ("hw_power_brake", "nvmlClocksEventReasonHwPowerBrakeSlowdown"))
+
     def __init__(self, index):
-        self.path = "/tmp/slate_bench_clocks_%d.csv" % os.getpid()
-        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        import threading
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self.stop_ev = threading.Event()
+        self.th = None
         try:
-            self.f = open(self.path, "w")
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), "--query-gpu=" + q,
-                                       "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
-                                      stderr=subprocess.DEVNULL)
+            import pynvml as N
+            N.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            phys = int(vis.split(",")[index]) if vis and vis.split(",")[index].strip().isdigit() else index
+            self.N, self.h = N, N.nvmlDeviceGetHandleByIndex(phys)
+            self.max_mhz = N.nvmlDeviceGetMaxClockInfo(self.h, N.NVML_CLOCK_SM)
+            self.th = threading.Thread(target=self._run, daemon=True)
+            self.th.start()
         except Exception:
-            self.p = None
+            self.th = None
+
+    def _run(self):
+        N = self.N
+        bits = [(n, getattr(N, c, 0)) for n, c in self.NAMES]
+        while not self.stop_ev.is_set():
+            try:
+                self.samples.append(N.nvmlDeviceGetClockInfo(self.h, N.NVML_CLOCK_SM))
+                r = N.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.reasons.update(n for n, b in bits if b and (r & b))
+            except Exception:
+                pass
+            self.stop_ev.wait(0.01)
 
     def stop(self):
-        if not self.p:
+        if not self.th:
             return None
-        self.p.terminate()
-        try:
-            self.p.wait(timeout=5)
-        except Exception:
-            self.p.kill()
-        self.f.close()
-        rows = [l.strip().split(", ") for l in open(self.path) if l.strip()]
-        os.unlink(self.path)
-        if not rows:
+        self.stop_ev.set()
+        self.th.join(timeout=2)
+        if not self.samples:
             return None
-        sm = [float(r[1]) for r in rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in rows if len(r) >= 9 for i in range(4) if r[5 + i].strip() == "Active"})
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(rows)}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples), "source": "nvml, 10 ms"}
 
 
 # ------------------------------------------------------------------ the GPU workload

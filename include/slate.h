@@ -143,7 +143,8 @@ typedef struct {
   uint32_t kind;           /* slate_kind */
   uint32_t iters;          /* SLATE_ITERS, blocks per task; 0 -> auto per launch (reading
                               Q11): min(cap, max(1, B / (t * occ * N))), cap = 10, t = 8;
-                              SPMV_CSR cap 8, t = 4; GEMM_BF16 -> 1 */
+                              SPMV_CSR cap 32, t = 6; GEMM_BF16 -> 1.  SPMV_CSR accepts
+                              iters <= 32 (its task buffer holds 32 blocks' row pointers) */
   uint32_t flags;          /* SLATE_KFLAG_* */
 } slate_kernel_desc;
 
@@ -151,7 +152,8 @@ typedef struct {
  * worker's occupancy (the "maximum number of thread blocks that the
  * designated SMs can support").  Idempotent per
  * (kind, iters, flags): registering twice returns the same handle.
- * Errors: EINVAL (bad abi_version / kind / flags), EUNSUPPORTED. */
+ * Errors: EINVAL (bad abi_version / kind / flags, iters above the kind's
+ * maximum), EUNSUPPORTED. */
 slate_status slate_register_kernel(slate_session* s, const slate_kernel_desc* d, slate_kernel* out);
 
 /* ------------------------------------------------------------------ launch */

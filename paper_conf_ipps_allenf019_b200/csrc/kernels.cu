@@ -5,6 +5,7 @@
 #include "slate_device.cuh"
 #include "tenants.cuh"
 #include "gemm_tc.cuh"
+#include "spmv_ws.cuh"
 
 namespace slate {
 
@@ -65,7 +66,7 @@ const KindOps* kind_ops(uint32_t kind) {
     table[SLATE_KIND_TRIAD] = make_ops<Triad>(0);
     table[SLATE_KIND_COPY] = make_ops<Copy>(0);
     table[SLATE_KIND_SGEMM_NAIVE] = make_ops<SgemmNaive>(0);
-    table[SLATE_KIND_SPMV_CSR] = make_ops<SpmvCsr>(0);
+    table[SLATE_KIND_SPMV_CSR] = spmv_ws_ops();
     table[SLATE_KIND_BLACKSCHOLES] = make_ops<BlackScholes>(0);
     table[SLATE_KIND_STENCIL2D] = make_ops<Stencil2D>(0);
     table[SLATE_KIND_GEMM_BF16] = gemm_tc_ops();

@@ -74,6 +74,7 @@ struct KindOps {
   size_t args_size = 0;
   uint32_t default_iters = 0;   // 0: auto (reading Q11)
   uint32_t max_auto_iters = 10; // per-tenant cap of the automatic task size
+  uint32_t max_iters = 0;       // largest task size the worker supports (0: any)
   uint32_t tasks_per_worker = 8; // the automatic task size aims at >= this many tasks per worker
   uint32_t tile_m = 0;           // GEMM: output rows per original block
   uint32_t tile_n = 0;           // GEMM: output columns per original block

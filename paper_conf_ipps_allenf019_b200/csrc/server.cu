@@ -296,6 +296,10 @@ int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::stri
     if (err) *err = "kind not built into this library";
     return SLATE_EUNSUPPORTED;
   }
+  if (ops->max_iters && d->iters > ops->max_iters) {
+    if (err) *err = "iters exceeds the kind's maximum task size";
+    return SLATE_EINVAL;
+  }
   std::lock_guard<std::mutex> g(mu_);
   const uint32_t iters = d->iters ? d->iters : ops->default_iters;   // 0 = auto per launch
   for (auto& kv : kernels_) {
@@ -356,7 +360,8 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     }
     case SLATE_KIND_SPMV_CSR: {
       auto a = static_cast<const slate_args_spmv*>(d->args);
-      if (!al(a->col) || !al(a->val)) return fail("spmv col/val must be 16-byte aligned");
+      if (!al(a->rowptr) || !al(a->col) || !al(a->val) || !al(a->x))
+        return fail("spmv rowptr/col/val/x must be 16-byte aligned");
       g[0] = cdiv(a->n_rows, 32);
       break;
     }

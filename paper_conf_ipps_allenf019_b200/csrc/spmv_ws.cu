@@ -1,0 +1,475 @@
+// spmv_ws.cu -- the slate worker of the CSR SpMV kind, warp-specialised for
+// sm_100a (DESIGN.md §5 "SpMV tenant").
+//
+// What it computes is the original kernel's (tenants.cuh SpmvCsrT): original
+// block x owns rows 32x..32x+31; lane l of a row's 8-lane group sums
+// val[j] * x[col[j]] over j = rp[row]+l, +8, ... in ascending order (an fmaf
+// chain from 0) and the group reduces with a xor 4, 2, 1 butterfly.  Only
+// where the operands come from differs, so y is bit-identical to the original
+// kernel's (tests/test_gpu_parity.py).
+//
+// Why a separate worker: the register body is bound by the L1 gather of x (one
+// 128-B line per lane per instruction: ~1 nonzero per SM clock, 16.7 M
+// nonzeros in C2 -> ~60 us) and by the dependent rp -> col -> x round trips of
+// each task.  Here one CTA per SM runs three roles (the structure of the GEMM
+// tenant: the slate protocol lives in a producer thread):
+//   * task warp (warp 8, lane 0) -- the slate worker proper: Lst1 binding and
+//     standby (prologue), at every task boundary the resize word (retire, Lst1
+//     P:L185) and the task counter (Lst2 (2) P:L208); then for the task it
+//     pulls the row-pointer slice and a window of x into one of two task
+//     buffers by cp.async.bulk.  The window is read off the task's nonzeros:
+//     [first column of its first row, last column of its last row], widened to
+//     the buffer's capacity (a banded or near-diagonal matrix then finds every
+//     column in it; any column outside is read from global memory, so the
+//     window only decides speed, never the result);
+//   * chunk warp (warp 9, lane 0) -- streams the task's nonzeros as chunks of
+//     256 rows (8 original blocks) through a 4-slot ring: columns and values of
+//     [rp[r0], rp[r0+256]) by cp.async.bulk (HBM -> shared, evict-first);
+//   * compute warps 0..7 -- per chunk, 8 lanes per row, x from the window in
+//     shared memory.
+// The task warp runs up to two tasks ahead of the compute warps and the chunk
+// warp keeps four chunks (~128 KB) in flight, so HBM sees a continuous stream
+// instead of one round-trip chain per task.
+//
+// Resize: the task boundary is where the task warp re-reads the
+// resize word; a CTA that left the range stops fetching, its compute warps
+// finish the (at most two) tasks it already holds, then it retires.  Nothing
+// is abandoned, so coverage is exactly-once by construction.
+#include <cstring>
+#include "kernels.h"
+#include "slate_device.cuh"
+#include "tenants.cuh"
+#include "spmv_ws.cuh"
+
+namespace slate {
+namespace spmv {
+
+#ifndef SLATE_SPMV_WARPS
+#define SLATE_SPMV_WARPS 16
+#endif
+constexpr int kComputeWarps = SLATE_SPMV_WARPS;  // 4 rows per warp per pass (8 lanes per row)
+constexpr int kCompute = 32 * kComputeWarps;
+constexpr int kThreads = kCompute + 64;          // + task warp + chunk warp
+constexpr int kTaskWarp = kComputeWarps, kChunkWarp = kComputeWarps + 1;
+constexpr int kChunkBlocks = 8;                  // blocks per chunk (256 rows)
+constexpr int kChunkRows = 32 * kChunkBlocks;
+constexpr int kPasses = kChunkRows / (4 * kComputeWarps);
+static_assert(kPasses * 4 * kComputeWarps == kChunkRows, "rows per chunk");
+constexpr int kMaxTaskBlocks = 32;               // task-size cap (1024 rows)
+constexpr int kSlots = 4;                        // chunk ring depth
+constexpr int kCap = kChunkRows * 16 + 8;        // nonzeros per slot (16 per row + alignment)
+constexpr int kSlotBytes = 2 * kCap * 4;         // col + val
+constexpr int kRpInts = 32 * kMaxTaskBlocks + 4; // rp slice of one task (rounded to 16 B)
+constexpr int kWin = 11264;                      // x window per task (floats)
+constexpr int kTaskBytes = kRpInts * 4 + kWin * 4;
+constexpr int kHdrBytes = 1024;
+constexpr int kSmemBytes = kHdrBytes + kSlots * kSlotBytes + 2 * kTaskBytes;
+static_assert(kSmemBytes <= 227 * 1024, "one CTA per SM");
+static_assert(kSlotBytes % 16 == 0 && kTaskBytes % 16 == 0 && (kRpInts * 4) % 16 == 0, "16-B bulk granules");
+
+struct TaskMeta {                 // written by the task warp before its rp arrive
+  uint32_t g, n;                  // original blocks [g, g+n); n = 0: stop (sentinel)
+  int32_t wlo;                    // x window: columns [wlo, wlo + wlen)
+  uint32_t wlen;
+};
+struct ChunkMeta {                // written by the chunk warp before its slot arrive
+  uint32_t tb;                    // task buffer; 0xffffffff: stop (sentinel)
+  uint32_t row0;                  // first row of the chunk within the task
+  uint32_t nblk;                  // blocks in the chunk
+  int32_t a0;                     // nonzero index of col_s[0] (16-B aligned)
+  uint32_t mode;                  // 0 staged, 1 col/val from global memory (the chunk exceeds the slot)
+  uint32_t first, last;           // first / last chunk of its task
+  uint32_t pad;
+};
+struct Hdr {
+  uint64_t slot_full[kSlots], slot_empty[kSlots];
+  uint64_t task_rp[2], task_win[2], task_empty[2];
+  TaskMeta tmeta[2];
+  ChunkMeta cmeta[kSlots];
+  uint32_t go, rank, retired;
+  uint64_t ctrl;                  // the resize word last acted on (task warp)
+};
+static_assert(sizeof(Hdr) <= kHdrBytes, "header");
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+// x is re-read by every task (L2-resident): no evict-first hint
+__device__ __forceinline__ void bulk_g2s_keep(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+#ifdef SLATE_SPMV_TRACE
+// development trace (tools/probe/spmv_stream.cu): per CTA < 4 and role, 64 events {t, kind, a, b}
+__device__ unsigned long long spmv_trace[4][3][64][4];
+__device__ __forceinline__ void trace(int role, uint32_t& n, uint32_t kind, uint32_t a0, uint32_t b0) {
+  if (blockIdx.x < 4 && n < 64) {
+    unsigned long long* r = spmv_trace[blockIdx.x][role][n++];
+    r[0] = globaltimer(); r[1] = kind; r[2] = a0; r[3] = b0;
+  }
+}
+#define TRACE(role, kind, a0, b0) trace(role, tn, kind, a0, b0)
+#define TRACE_DECL uint32_t tn = 0
+#else
+#define TRACE(role, kind, a0, b0)
+#define TRACE_DECL
+#endif
+
+struct Smem {
+  Hdr* h;
+  char* slots;
+  char* tasks;
+  __device__ __forceinline__ int32_t* col(int s) const { return reinterpret_cast<int32_t*>(slots + s * kSlotBytes); }
+  __device__ __forceinline__ float* val(int s) const {
+    return reinterpret_cast<float*>(slots + s * kSlotBytes + kCap * 4);
+  }
+  __device__ __forceinline__ int32_t* rp(int b) const { return reinterpret_cast<int32_t*>(tasks + b * kTaskBytes); }
+  __device__ __forceinline__ float* xw(int b) const {
+    return reinterpret_cast<float*>(tasks + b * kTaskBytes + kRpInts * 4);
+  }
+};
+
+// ------------------------------------------------------------------ compute warps
+// Rows of one chunk: kPasses passes of 4 rows per compute warp; every pass's
+// shared-memory loads are issued before the first FMA, and the x reads are
+// branch-free (a column outside the window reads a clamped slot first and is
+// patched from global memory afterwards, under a warp vote that is false for
+// banded matrices), so a warp keeps ~16 loads in flight.
+__device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Smem& S, const ChunkMeta& m,
+                                              const TaskMeta& tm, int s) {
+  const float* __restrict__ xg = reinterpret_cast<const float*>(a.x);
+  const int32_t* rp = S.rp(int(m.tb)) + m.row0;          // rp of the chunk's first row
+  const float* xw = S.xw(int(m.tb));
+  const int32_t wlo = tm.wlo;
+  const uint32_t wlen = tm.wlen, wmax = tm.wlen ? tm.wlen - 1 : 0;
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int l = int(lane & 7);
+  const uint32_t row_first = tm.g * 32 + m.row0;        // global row of rp[0]
+  const uint32_t nrows = min(m.nblk * 32, a.n_rows - row_first);
+  auto xval = [&](int c) -> float {
+    const uint32_t d = uint32_t(c - wlo);
+    return d < wlen ? xw[d] : __ldg(xg + c);
+  };
+  constexpr int U = kPasses;
+  int lo[U], hi[U];
+  float acc[U];
+  if (m.mode == 0) {
+    const int32_t* col = S.col(s);
+    const float* val = S.val(s);
+    const int32_t a0 = m.a0;
+    int c0[U], c1[U];
+    float v0[U], v1[U], x0[U], x1[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint32_t lr = u * (kComputeWarps * 4) + w * 4 + (lane >> 3);
+      lo[u] = 0; hi[u] = 0; acc[u] = 0.f;
+      if (lr < nrows) { lo[u] = rp[lr] - a0 + l; hi[u] = rp[lr + 1] - a0; }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool h0 = lo[u] < hi[u], h1 = lo[u] + 8 < hi[u];
+      c0[u] = col[h0 ? lo[u] : 0];
+      v0[u] = val[h0 ? lo[u] : 0];
+      c1[u] = col[h1 ? lo[u] + 8 : 0];
+      v1[u] = val[h1 ? lo[u] + 8 : 0];
+    }
+    bool miss = false;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint32_t d0 = uint32_t(c0[u] - wlo), d1 = uint32_t(c1[u] - wlo);
+      x0[u] = xw[min(d0, wmax)];
+      x1[u] = xw[min(d1, wmax)];
+      miss |= (lo[u] < hi[u] && d0 >= wlen) || (lo[u] + 8 < hi[u] && d1 >= wlen);
+    }
+    if (__any_sync(0xffffffffu, miss)) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (lo[u] < hi[u] && uint32_t(c0[u] - wlo) >= wlen) x0[u] = __ldg(xg + c0[u]);
+        if (lo[u] + 8 < hi[u] && uint32_t(c1[u] - wlo) >= wlen) x1[u] = __ldg(xg + c1[u]);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (lo[u] < hi[u]) acc[u] = __fmaf_rn(v0[u], x0[u], acc[u]);
+      if (lo[u] + 8 < hi[u]) acc[u] = __fmaf_rn(v1[u], x1[u], acc[u]);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u)     // rows longer than 16: the rest of the chain, still ascending
+      for (int j = lo[u] + 16; j < hi[u]; j += 8) acc[u] = __fmaf_rn(val[j], xval(col[j]), acc[u]);
+  } else {
+    // the chunk's nonzeros did not fit the slot: the same chain from global memory
+    const int32_t* col = reinterpret_cast<const int32_t*>(a.col);
+    const float* val = reinterpret_cast<const float*>(a.val);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint32_t lr = u * (kComputeWarps * 4) + w * 4 + (lane >> 3);
+      lo[u] = 0; hi[u] = 0; acc[u] = 0.f;
+      if (lr < nrows) { lo[u] = rp[lr] + l; hi[u] = rp[lr + 1]; }
+      for (int j = lo[u]; j < hi[u]; j += 8) acc[u] = __fmaf_rn(__ldcs(val + j), xval(__ldcs(col + j)), acc[u]);
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    float v = acc[u];
+    v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 4));
+    v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 2));
+    v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 1));
+    const uint32_t lr = u * (kComputeWarps * 4) + w * 4 + (lane >> 3);
+    if (l == 0 && lr < nrows) __stcs(reinterpret_cast<float*>(a.y) + row_first + lr, v);
+  }
+}
+
+// ------------------------------------------------------------------ the worker
+__global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant__ WorkerParams<slate_args_spmv> p) {
+  extern __shared__ __align__(128) char smem_raw[];
+  Smem S;
+  S.h = reinterpret_cast<Hdr*>(smem_raw);
+  S.slots = smem_raw + kHdrBytes;
+  S.tasks = S.slots + kSlots * kSlotBytes;
+  Hdr& H = *S.h;
+  const slate_args_spmv& a = p.args;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (threadIdx.x == kTaskWarp * 32) {
+    for (int i = 0; i < kSlots; ++i) {
+      mbar_init(&H.slot_full[i], 1);              // the chunk warp's expect_tx arrive (+ bytes)
+      mbar_init(&H.slot_empty[i], kComputeWarps); // every compute warp
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&H.task_rp[i], 1);                // the task warp's expect_tx arrive (+ rp bytes)
+      mbar_init(&H.task_win[i], 1);               // the task warp's expect_tx arrive (+ x bytes)
+      mbar_init(&H.task_empty[i], kComputeWarps + 1);   // every compute warp + the chunk warp
+    }
+    fence_mbar_init();
+    // ---- Lst1: bind to the SM, standby while under-staffed
+    const uint32_t r = p.rank_of[smid()];
+    uint64_t c = 0;
+    H.rank = r;
+    H.retired = 0;
+    H.go = prologue(p, r, c) ? 1u : 0u;
+    H.ctrl = c;
+  }
+  __syncthreads();
+  if (!H.go) return;
+
+  if (warp == kTaskWarp) {
+    // ===================== task warp: the slate task protocol + task buffers =====================
+    uint64_t c = H.ctrl;
+    const uint32_t rank = H.rank;
+    TRACE_DECL;
+    for (uint32_t t = 0;; ++t) {
+      const int b = int(t & 1);
+      const uint32_t use = t >> 1;
+      uint32_t g = 0xffffffffu, chg = 0;
+      if (lane == 0) {
+        TRACE(0, 0, t, 0);
+        mbar_wait(&H.task_empty[b], (use & 1) ^ 1);   // task t-2 fully consumed
+        TRACE(0, 1, t, 0);
+        // task boundary: the resize word, then the counter
+        const uint64_t c2 = ld_acquire_u64(p.ctrl);
+        chg = ctrl_epoch(c2) != ctrl_epoch(c);
+        c = c2;
+        if (!in_range(p, rank, c) && try_retire(p.tc)) {
+          H.retired = 1;
+        } else {
+          const uint32_t f = atomicAdd(&p.tc->next, p.iters);          // Lst2 (2)
+          if (f < p.B) {
+            g = f;
+            TRACE(0, 2, t, g);
+            if (f == 0) p.tc->t_first = globaltimer();
+          } else {
+            atomicAdd(&p.tc->live_pending, ~0ull);                      // drained: live -= 1
+          }
+        }
+      }
+      g = __shfl_sync(0xffffffffu, g, 0);
+      chg = __shfl_sync(0xffffffffu, chg, 0);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if (chg && g != 0xffffffffu) check_shrink_done(p, c, lane);
+      if (lane == 0) {
+        TaskMeta& tm = H.tmeta[b];
+        if (g == 0xffffffffu) {
+          tm.g = 0; tm.n = 0; tm.wlo = 0; tm.wlen = 0;
+          mbar_expect_tx(&H.task_rp[b], 0);           // sentinel: publishes the stop
+        } else {
+          const uint32_t n = min(p.iters, p.B - g);
+          const uint32_t r0 = g * 32, r1 = min(r0 + n * 32, a.n_rows);
+          // rp[r0 .. r1]: whole 16-B granules by the bulk engine, the last
+          // (r1 - r0 + 1) mod 4 entries by this thread (never reads past rp's end)
+          const uint32_t nbulk = (r1 - r0 + 1) & ~3u;
+          tm.g = g; tm.n = n;
+          // the window comes from the task's first and last nonzero (two loads
+          // that ride alongside the rp slice; the rp ends are needed for them)
+          const int32_t* rpg = reinterpret_cast<const int32_t*>(a.rowptr);
+          const int32_t e0 = __ldg(rpg + r0), e1 = __ldg(rpg + r1);
+          for (uint32_t i = nbulk; i <= r1 - r0; ++i) S.rp(b)[i] = __ldg(rpg + r0 + i);
+          mbar_expect_tx(&H.task_rp[b], nbulk * 4);  // (its release publishes tm and the tail)
+          if (nbulk) bulk_g2s(S.rp(b), rpg + r0, nbulk * 4, &H.task_rp[b]);
+          int32_t wlo = 0;
+          uint32_t wlen = 0;
+          if (e1 > e0) {
+            const int32_t* colg = reinterpret_cast<const int32_t*>(a.col);
+            const int32_t cf = __ldg(colg + e0), cl = __ldg(colg + e1 - 1);
+            const int32_t cmin = min(cf, cl), cmax = max(cf, cl);
+            const int32_t ncols = int32_t(a.n_cols);
+            const int32_t span = cmax - cmin + 1;
+            int32_t lo = span >= kWin ? cmin : cmin - (kWin - span) / 2;
+            lo = max(0, min(lo, ncols - kWin)) & ~3;
+            wlo = lo;
+            // whole granules inside x; columns past the window read global memory
+            wlen = uint32_t(max(0, min(kWin, ncols - lo)) & ~3);
+          }
+          tm.wlo = wlo;
+          tm.wlen = wlen;
+          TRACE(0, 3, t, wlen);
+          mbar_expect_tx(&H.task_win[b], wlen * 4);
+          if (wlen)
+            bulk_g2s_keep(S.xw(b), reinterpret_cast<const float*>(a.x) + wlo, wlen * 4, &H.task_win[b]);
+        }
+      }
+      if (g == 0xffffffffu) {
+        if (lane == 0) H.ctrl = c;                  // the word the CTA acted on last
+        break;
+      }
+    }
+  } else if (warp == kChunkWarp) {
+    // ===================== chunk warp: nonzeros of each task through the slot ring =====================
+    if (lane == 0) {
+      TRACE_DECL;
+      uint32_t q = 0;   // chunks issued
+      for (uint32_t t = 0;; ++t) {
+        const int b = int(t & 1);
+        mbar_wait(&H.task_rp[b], (t >> 1) & 1);
+        TRACE(1, 10, t, 0);
+        const TaskMeta tm = H.tmeta[b];
+        const uint32_t nch = tm.n ? (tm.n + kChunkBlocks - 1) / kChunkBlocks : 1;
+        for (uint32_t k = 0; k < nch; ++k, ++q) {
+          const int s = int(q % kSlots);
+          mbar_wait(&H.slot_empty[s], ((q / kSlots) & 1) ^ 1);
+          TRACE(1, 11, q, 0);
+          ChunkMeta& m = H.cmeta[s];
+          if (tm.n == 0) {
+            m.tb = 0xffffffffu;
+            mbar_expect_tx(&H.slot_full[s], 0);
+            break;
+          }
+          const uint32_t row0 = k * kChunkRows;
+          const uint32_t nblk = min(uint32_t(kChunkBlocks), tm.n - k * kChunkBlocks);
+          const uint32_t r0 = tm.g * 32 + row0;
+          const uint32_t nrows = min(nblk * 32, a.n_rows - r0);
+          const int32_t* rp = S.rp(b) + row0;
+          const int32_t e0 = rp[0], e1 = rp[nrows];
+          // [a0, a1) in whole 16-B granules; at the end of the matrix the
+          // granule past nnz may lie outside the arrays: its entries are loaded
+          // by this thread instead
+          const bool end = r0 + nrows == a.n_rows;
+          const int32_t a0 = e0 & ~3, a1 = end ? (e1 & ~3) : ((e1 + 3) & ~3);
+          m.tb = uint32_t(b); m.row0 = row0; m.nblk = nblk; m.a0 = a0;
+          m.first = k == 0; m.last = k + 1 == nch;
+          if (max(a1, e1) - a0 > kCap) {
+            m.mode = 1;
+            mbar_expect_tx(&H.slot_full[s], 0);
+          } else {
+            m.mode = 0;
+            for (int32_t j = max(a1, a0); j < e1; ++j) {
+              S.col(s)[j - a0] = __ldg(reinterpret_cast<const int32_t*>(a.col) + j);
+              S.val(s)[j - a0] = __ldg(reinterpret_cast<const float*>(a.val) + j);
+            }
+            const uint32_t bytes = uint32_t(max(a1 - a0, 0)) * 4;
+            mbar_expect_tx(&H.slot_full[s], 2 * bytes);
+            if (bytes) {
+              bulk_g2s(S.col(s), reinterpret_cast<const int32_t*>(a.col) + a0, bytes, &H.slot_full[s]);
+              bulk_g2s(S.val(s), reinterpret_cast<const float*>(a.val) + a0, bytes, &H.slot_full[s]);
+            }
+          }
+        }
+        if (tm.n == 0) break;
+        mbar_arrive(&H.task_empty[b]);   // this warp is done reading the task's rp
+      }
+    }
+  } else {
+    // ===================== compute warps =====================
+    uint32_t q = 0, t = 0, my_blocks = 0, my_tasks = 0;
+    TRACE_DECL;
+    for (;; ++q) {
+      const int s = int(q % kSlots);
+      mbar_wait(&H.slot_full[s], (q / kSlots) & 1);
+      if (threadIdx.x == 0) TRACE(2, 20, q, 0);
+      const ChunkMeta m = H.cmeta[s];
+      if (m.tb == 0xffffffffu) break;
+      const int b = int(m.tb);
+      if (m.first) {
+        mbar_wait(&H.task_rp[b], (t >> 1) & 1);
+        mbar_wait(&H.task_win[b], (t >> 1) & 1);
+      }
+      const TaskMeta tm = H.tmeta[b];
+      if (threadIdx.x == 0) TRACE(2, 21, q, 0);
+      compute_chunk(a, S, m, tm, s);
+      __syncwarp();
+      if (threadIdx.x == 0) TRACE(2, 22, q, 0);
+      if (lane == 0) {
+        mbar_arrive(&H.slot_empty[s]);
+        if (m.last) mbar_arrive(&H.task_empty[b]);
+      }
+      if (threadIdx.x == 0) {
+        my_blocks += m.nblk;
+        if (p.cov)
+          for (uint32_t i = 0; i < m.nblk; ++i) atomicAdd(&p.cov[tm.g + m.row0 / 32 + i], 1u);
+      }
+      if (m.last) {
+        ++t;
+        ++my_tasks;
+      }
+    }
+    if (threadIdx.x == 0 && my_blocks) count_done(p, my_blocks, my_tasks);
+  }
+  __syncthreads();
+  if (warp == kTaskWarp) {
+    if (lane == 0) atomicAdd(&p.tc->live_rank[H.rank], 0xffffffffu);   // live_rank -= 1
+    if (H.retired) check_shrink_done(p, H.ctrl, lane);
+  }
+}
+
+static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32_t grid, cudaStream_t st) {
+  WorkerParams<slate_args_spmv> p;
+  std::memcpy(&p.args, args, sizeof(p.args));
+  p.gx = w.gx; p.gy = w.gy; p.gz = w.gz; p.B = w.B; p.iters = w.iters; p.occ = w.occ;
+  p.bound_lo = w.bound_lo; p.bound_hi = w.bound_hi; p.n_ranks = w.n_ranks;
+  p.standby_timeout_ns = w.standby_timeout_ns;
+  p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
+  void* kargs[] = {&p};
+  return cudaLaunchKernel(reinterpret_cast<const void*>(&spmv_worker), dim3(grid), dim3(kThreads), kargs, kSmemBytes,
+                          st);
+}
+
+static cudaError_t launch_standalone(const void* args, dim3 grid, cudaStream_t st) {
+  slate_args_spmv a;
+  std::memcpy(&a, args, sizeof(a));
+  void* kargs[] = {&a};
+  return cudaLaunchKernel(reinterpret_cast<const void*>(&standalone<SpmvCsrReg>), grid, dim3(SpmvCsrReg::kThreads),
+                          kargs, 0, st);
+}
+
+}  // namespace spmv
+
+KindOps spmv_ws_ops() {
+  KindOps o;
+  o.worker_fn = reinterpret_cast<const void*>(&spmv::spmv_worker);
+  o.standalone_fn = reinterpret_cast<const void*>(&standalone<SpmvCsrReg>);
+  o.threads = spmv::kThreads;
+  o.smem = spmv::kSmemBytes;
+  o.smem_standalone = 0;
+  o.args_size = sizeof(slate_args_spmv);
+  o.default_iters = 0;
+  o.max_auto_iters = spmv::kMaxTaskBlocks;
+  o.max_iters = spmv::kMaxTaskBlocks;        // the task buffer holds the rp slice of <= 32 blocks
+  o.tasks_per_worker = 6;
+  o.launch_worker = &spmv::launch_worker;
+  o.launch_standalone = &spmv::launch_standalone;
+  return o;
+}
+
+}  // namespace slate

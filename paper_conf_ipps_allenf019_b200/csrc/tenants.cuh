@@ -293,9 +293,11 @@ struct SpmvCsrT : TenantBase {
     if (i < n) rows<kU>(a, g + i, n - i);
   }
 };
-// the configuration in use: 8 blocks' rows in flight per thread, 4 CTAs/SM
-// (tools/probe/worker_overhead.cu: fastest of U in {1..8} x occupancy {4, 6, 8})
-using SpmvCsr = SpmvCsrT<8, 4>;
+// the register body: 8 blocks' rows in flight per thread, 4 CTAs/SM
+// (tools/probe/worker_overhead.cu: fastest of U in {1..8} x occupancy {4, 6, 8}).
+// It is the original kernel K(B,T) of the SpMV kind; the slate worker of the
+// kind is the warp-specialised one in spmv_ws.cu (same per-row arithmetic).
+using SpmvCsrReg = SpmvCsrT<8, 4>;
 
 // ============================================================== Black-Scholes
 // European call/put as in the CUDA SDK BlackScholes sample: the normal CDF by

@@ -71,6 +71,33 @@ def spmv_inputs(n_rows, seed, mode="float", nnz_per_row=16, band=4096, n_cols=No
     return rowptr.astype(np.int32), cols, val, x
 
 
+def spmv_ragged_inputs(n_rows, seed, mode="float", lengths=(0, 48), band=None, n_cols=None, long_rows=0,
+                       long_len=2000):
+    """CSR with irregular rows: each row's length uniform in ``lengths`` (empty
+    rows included), plus ``long_rows`` rows of ``long_len`` nonzeros at random
+    positions; distinct sorted columns uniform in [i - band, i + band] clipped to
+    [0, n_cols), or over all columns when ``band`` is None.  Same dtypes and
+    value ranges as spmv_inputs."""
+    n_cols = n_rows if n_cols is None else n_cols
+    g = rng(seed)
+    per_row = g.integers(lengths[0], lengths[1] + 1, size=n_rows)
+    if long_rows:
+        per_row[g.choice(n_rows, size=long_rows, replace=False)] = long_len
+    cols = []
+    for i in range(n_rows):
+        lo, hi = (0, n_cols) if band is None else (max(0, i - band), min(n_cols, i + band + 1))
+        k = min(int(per_row[i]), hi - lo)
+        per_row[i] = k
+        cols.append(np.sort(g.choice(hi - lo, size=k, replace=False)) + lo)
+    rowptr = np.zeros(n_rows + 1, dtype=np.int64)
+    rowptr[1:] = np.cumsum(per_row)
+    nnz = int(rowptr[-1])
+    col = np.concatenate(cols).astype(np.int32) if nnz else np.zeros(0, np.int32)
+    val = _vec(g, nnz, mode, -2, 2)
+    x = _vec(g, n_cols, mode, -2, 2)
+    return rowptr.astype(np.int32), col, val, x
+
+
 def bs_inputs(n, seed):
     """Option batch in the CUDA SDK BlackScholes sample's ranges: stock price
     S ~ U[5, 30], strike X ~ U[1, 100], expiry T ~ U[0.25, 10] years; SoA fp32.

@@ -81,8 +81,11 @@ def make_sgemm(m, n, k, seed, mode="float"):
     return Tenant(S.KIND_SGEMM_NAIVE, args, grid, [C_d], check, (A_d, B_d))
 
 
-def make_spmv(n_rows, seed, mode="float", band=4096):
-    rp, col, val, x = I.spmv_inputs(n_rows, seed, mode, band=band)
+def make_spmv(n_rows, seed, mode="float", band=4096, ragged=None):
+    if ragged is None:
+        rp, col, val, x = I.spmv_inputs(n_rows, seed, mode, band=band)
+    else:
+        rp, col, val, x = I.spmv_ragged_inputs(n_rows, seed, mode, band=band, **ragged)
     rp_d, col_d, val_d, x_d = dev(rp), dev(col), dev(val), dev(x)
     y_d = torch.zeros(n_rows, device=DEV)
     args, grid = S.spmv_args(rp_d, col_d, val_d, x_d, y_d)

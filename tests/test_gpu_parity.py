@@ -24,6 +24,14 @@ CASES = {
     "sgemm_int": lambda: make_sgemm(256, 256, 256, 105, "int"),
     "spmv_float": lambda: make_spmv(32 * 300 + 7, 106, band=512),
     "spmv_int": lambda: make_spmv(32 * 128, 107, "int", band=64),
+    # irregular rows (empty ones included): chunks over the staging slot's
+    # capacity take the global-memory path
+    "spmv_ragged": lambda: make_spmv(32 * 200 + 13, 115, band=3000, ragged=dict(lengths=(0, 48))),
+    # a non-square matrix with columns spread over all of x: the x window misses
+    "spmv_wide": lambda: make_spmv(32 * 150 + 5, 116, band=None, ragged=dict(lengths=(16, 16), n_cols=50001)),
+    # a few very long rows between short ones
+    "spmv_long_rows": lambda: make_spmv(32 * 100 + 31, 117, "int", band=None,
+                                        ragged=dict(lengths=(0, 4), n_cols=20000, long_rows=3, long_len=3000)),
     "bs": lambda: make_bs(1024 * 12 + 4 * 33 + 2, 108, n_scen=5),
     "stencil_float": lambda: make_stencil(8 * 37 + 3, 32 * 9 + 5, 109),
     "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
@@ -58,7 +66,7 @@ def test_tenant_parity(sess, name):
     assert ok, "standalone vs oracle: %s (worst %.3g of tolerance)" % (name, err)
     B = int(np.prod(t.grid))
     n = sess.info()["num_sms"]
-    for iters in (1, 10):
+    for iters in ((1, 10, 32) if t.kind == S.KIND_SPMV_CSR else (1, 10)):
         k = sess.register_kernel(t.kind, iters=iters, flags=S.KFLAG_COVERAGE)
         for sm in [(0, n - 1), (3, 3 + n // 3)]:
             lid, outs, cov = _run(sess, t, k, placement=S.PLACE_CORUN, sm=sm)

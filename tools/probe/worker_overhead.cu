@@ -1,5 +1,5 @@
 // Development probe: where does the slate worker's per-launch/per-task overhead
-// come from?  Runs the real slate_worker<SpmvCsr> (library headers) beside the
+// come from?  Runs the real slate_worker<SpmvCsrReg> (library headers) beside the
 // original kernel and stripped-down persistent variants, L2 flushed each run.
 #include <cuda_runtime.h>
 #include <cstdio>
@@ -21,7 +21,7 @@ __global__ void __launch_bounds__(256) v0(slate_args_spmv a, unsigned* ctr, int 
     const unsigned g = s_g;
     __syncthreads();
     if (g >= (unsigned)nblk) return;
-    SpmvCsr::cta_task(a, g, min((unsigned)it, nblk - g), nullptr);
+    SpmvCsrReg::cta_task(a, g, min((unsigned)it, nblk - g), nullptr);
   }
 }
 // V1: V0 + the done counter (64-bit atomic with return) per task
@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(256) v1(slate_args_spmv a, unsigned* ctr, unsi
     __syncthreads();
     if (g >= (unsigned)nblk) return;
     const unsigned n = min((unsigned)it, nblk - g);
-    SpmvCsr::cta_task(a, g, n, nullptr);
+    SpmvCsrReg::cta_task(a, g, n, nullptr);
     __syncthreads();
     if (threadIdx.x == 0) { unsigned long long o = atomicAdd(done, (1ull << 32) | n); if ((unsigned)o + n == (unsigned)nblk) done[1] = 1; }
   }
@@ -84,19 +84,19 @@ int main() {
     }
     printf("%-44s best %.4f ms  mean %.4f ms  %.0f GB/s\n", name, best, sum / cnt, bytes / best / 1e6);
   };
-  timeit("original kernel (standalone<SpmvCsr>)", [&] { standalone<SpmvCsr><<<nblk, 256>>>(a); });
+  timeit("original kernel (standalone<SpmvCsrReg>)", [&] { standalone<SpmvCsrReg><<<nblk, 256>>>(a); });
   for (int it : {4}) {
     int occ; cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, v0, 256, 0);
     printf("v0 occ %d\n", occ);
     timeit("v0 persistent, 1 atomic/task", [&] { v0<<<148 * occ, 256>>>(a, ctr, nblk, it); });
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, v1, 256, 0);
     timeit("v1 + done atomic/task", [&] { v1<<<148 * occ, 256>>>(a, ctr, done, nblk, it); });
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, slate_worker<SpmvCsr>, 256, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, slate_worker<SpmvCsrReg>, 256, 0);
     printf("worker occ %d\n", occ);
     WorkerParams<slate_args_spmv> p{};
     p.args = a; p.gx = nblk; p.gy = 1; p.gz = 1; p.B = nblk; p.iters = it; p.occ = occ; p.bound_lo = 0; p.bound_hi = 147;
     p.n_ranks = 148; p.standby_timeout_ns = 200000; p.ctrl = ctrl; p.tc = tc; p.mirror = nullptr; p.cov = nullptr; p.rank_of = lut;
-    timeit("slate_worker<SpmvCsr> (the real one)", [&] { slate_worker<SpmvCsr><<<148 * occ, 256>>>(p); });
+    timeit("slate_worker<SpmvCsrReg> (the real one)", [&] { slate_worker<SpmvCsrReg><<<148 * occ, 256>>>(p); });
     auto variant = [&](const char* name, auto kern, int it2) {
       int o; cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, 256, 0);
       WorkerParams<slate_args_spmv> q = p; q.occ = o; q.iters = it2;
