@@ -514,7 +514,7 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     top = max(durs, key=lambda k: sum(durs[k]))
     j, avg = job[top], sum(durs[top]) / len(durs[top])
     # the worker kernel's name as ncu prints it (the key of profiles/ncu_traffic.json)
-    kname = {"blackscholes": "slate_worker<BlackScholes>", "spmv": "slate_worker<SpmvCsrT<8, 4>>",
+    kname = {"blackscholes": "slate_worker<BlackScholes>", "spmv": "spmv::spmv_worker",
              "gemm_bf16": "gemm::gemm_kernel<1>", "copy": "slate_worker<Copy>"}[top]
     if j.tc:
         ach = j.tc / (avg * 1e-3) / 1e12

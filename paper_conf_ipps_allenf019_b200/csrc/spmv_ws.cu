@@ -12,28 +12,32 @@
 // 128-B line per lane per instruction: ~1 nonzero per SM clock, 16.7 M
 // nonzeros in C2 -> ~60 us) and by the dependent rp -> col -> x round trips of
 // each task.  Here one CTA per SM runs three roles (the structure of the GEMM
-// tenant: the slate protocol lives in a producer thread):
-//   * task warp (warp 8, lane 0) -- the slate worker proper: Lst1 binding and
-//     standby (prologue), at every task boundary the resize word (retire, Lst1
-//     P:L185) and the task counter (Lst2 (2) P:L208); then for the task it
-//     pulls the row-pointer slice and a window of x into one of two task
-//     buffers by cp.async.bulk.  The window is read off the task's nonzeros:
-//     [first column of its first row, last column of its last row], widened to
-//     the buffer's capacity (a banded or near-diagonal matrix then finds every
-//     column in it; any column outside is read from global memory, so the
-//     window only decides speed, never the result);
-//   * chunk warp (warp 9, lane 0) -- streams the task's nonzeros as chunks of
-//     256 rows (8 original blocks) through a 4-slot ring: columns and values of
+// tenant: the slate protocol lives in a producer warp):
+//   * task warp (warp 16) -- the slate worker proper: Lst1 binding and standby
+//     (prologue), at every task boundary the resize word (retire, Lst1 P:L185)
+//     and the task counter (Lst2 (2) P:L208), taken one task ahead
+//     (speculative boundary); then the task's row-pointer slice, loaded by the
+//     whole warp into one of four slice buffers, and the bounds of its x window,
+//     read off the task's nonzeros: [first column of its first row, last column
+//     of its last row] widened to the buffer's capacity (a banded or
+//     near-diagonal matrix then finds every column in it; a column outside is
+//     read from global memory, so the window decides speed, never the result);
+//   * chunk warp (warp 17, lane 0) -- per task the x window (cp.async.bulk,
+//     L2 -> shared, two buffers), then the task's nonzeros as chunks of 256 rows
+//     (8 original blocks) through a 4-slot ring: columns and values of
 //     [rp[r0], rp[r0+256]) by cp.async.bulk (HBM -> shared, evict-first);
-//   * compute warps 0..7 -- per chunk, 8 lanes per row, x from the window in
-//     shared memory.
-// The task warp runs up to two tasks ahead of the compute warps and the chunk
-// warp keeps four chunks (~128 KB) in flight, so HBM sees a continuous stream
-// instead of one round-trip chain per task.
+//   * compute warps 0..15 -- per chunk, 8 lanes per row, x from the window.
+// The task warp runs up to three tasks ahead of the compute warps and the chunk
+// warp keeps up to four chunks (~128 KB) in flight, so HBM sees a stream
+// instead of one round-trip chain per task.  What bounds it (DESIGN.md §5,
+// tools/probe/spmv_stream.cu, tools/probe/bulk_bw.cu): a bulk copy costs the
+// SM's copy engine ~190 ns however small it is, and 16-KB copies with the
+// ring's depth deliver ~50 GB/s per SM; the compute warps are issue-bound at
+// ~1150 clocks per 256-row chunk.
 //
 // Resize: the task boundary is where the task warp re-reads the
 // resize word; a CTA that left the range stops fetching, its compute warps
-// finish the (at most two) tasks it already holds, then it retires.  Nothing
+// finish the tasks it already holds (at most four), then it retires.  Nothing
 // is abandoned, so coverage is exactly-once by construction.
 #include <cstring>
 #include "kernels.h"
@@ -59,13 +63,14 @@ constexpr int kMaxTaskBlocks = 32;               // task-size cap (1024 rows)
 constexpr int kSlots = 4;                        // chunk ring depth
 constexpr int kCap = kChunkRows * 16 + 8;        // nonzeros per slot (16 per row + alignment)
 constexpr int kSlotBytes = 2 * kCap * 4;         // col + val
+constexpr int kRpBufs = 4;                       // row-pointer slices: the task warp runs <= 3 tasks ahead
 constexpr int kRpInts = 32 * kMaxTaskBlocks + 4; // rp slice of one task (rounded to 16 B)
-constexpr int kWin = 11264;                      // x window per task (floats)
-constexpr int kTaskBytes = kRpInts * 4 + kWin * 4;
+constexpr int kWinBufs = 2;
+constexpr int kWin = 10240;                      // x window per task (floats)
 constexpr int kHdrBytes = 1024;
-constexpr int kSmemBytes = kHdrBytes + kSlots * kSlotBytes + 2 * kTaskBytes;
+constexpr int kSmemBytes = kHdrBytes + kSlots * kSlotBytes + kRpBufs * kRpInts * 4 + kWinBufs * kWin * 4;
 static_assert(kSmemBytes <= 227 * 1024, "one CTA per SM");
-static_assert(kSlotBytes % 16 == 0 && kTaskBytes % 16 == 0 && (kRpInts * 4) % 16 == 0, "16-B bulk granules");
+static_assert(kSlotBytes % 16 == 0 && (kRpInts * 4) % 16 == 0 && (kWin * 4) % 16 == 0, "16-B bulk granules");
 
 struct TaskMeta {                 // written by the task warp before its rp arrive
   uint32_t g, n;                  // original blocks [g, g+n); n = 0: stop (sentinel)
@@ -73,18 +78,19 @@ struct TaskMeta {                 // written by the task warp before its rp arri
   uint32_t wlen;
 };
 struct ChunkMeta {                // written by the chunk warp before its slot arrive
-  uint32_t tb;                    // task buffer; 0xffffffff: stop (sentinel)
+  uint32_t tb;                    // rp buffer of the chunk's task; 0xffffffff: stop (sentinel)
+  uint32_t wb;                    // x-window buffer of the chunk's task
   uint32_t row0;                  // first row of the chunk within the task
   uint32_t nblk;                  // blocks in the chunk
   int32_t a0;                     // nonzero index of col_s[0] (16-B aligned)
   uint32_t mode;                  // 0 staged, 1 col/val from global memory (the chunk exceeds the slot)
   uint32_t first, last;           // first / last chunk of its task
-  uint32_t pad;
 };
 struct Hdr {
   uint64_t slot_full[kSlots], slot_empty[kSlots];
-  uint64_t task_rp[2], task_win[2], task_empty[2];
-  TaskMeta tmeta[2];
+  uint64_t rp_full[kRpBufs], rp_empty[kRpBufs];
+  uint64_t win_full[kWinBufs], win_empty[kWinBufs];
+  TaskMeta tmeta[kRpBufs];
   ChunkMeta cmeta[kSlots];
   uint32_t go, rank, retired;
   uint64_t ctrl;                  // the resize word last acted on (task warp)
@@ -118,18 +124,21 @@ __device__ __forceinline__ void trace(int role, uint32_t& n, uint32_t kind, uint
 #define TRACE_DECL
 #endif
 
+#ifdef SLATE_SPMV_PROFILE
+__device__ long long spmv_prof[148][32][5];   // per CTA, compute warp: {total, wait full, first-chunk waits, compute, chunks}
+#endif
+
 struct Smem {
   Hdr* h;
   char* slots;
-  char* tasks;
+  char* rpb;
+  char* win;
   __device__ __forceinline__ int32_t* col(int s) const { return reinterpret_cast<int32_t*>(slots + s * kSlotBytes); }
   __device__ __forceinline__ float* val(int s) const {
     return reinterpret_cast<float*>(slots + s * kSlotBytes + kCap * 4);
   }
-  __device__ __forceinline__ int32_t* rp(int b) const { return reinterpret_cast<int32_t*>(tasks + b * kTaskBytes); }
-  __device__ __forceinline__ float* xw(int b) const {
-    return reinterpret_cast<float*>(tasks + b * kTaskBytes + kRpInts * 4);
-  }
+  __device__ __forceinline__ int32_t* rp(int b) const { return reinterpret_cast<int32_t*>(rpb + b * kRpInts * 4); }
+  __device__ __forceinline__ float* xw(int b) const { return reinterpret_cast<float*>(win + b * kWin * 4); }
 };
 
 // ------------------------------------------------------------------ compute warps
@@ -142,7 +151,7 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
                                               const TaskMeta& tm, int s) {
   const float* __restrict__ xg = reinterpret_cast<const float*>(a.x);
   const int32_t* rp = S.rp(int(m.tb)) + m.row0;          // rp of the chunk's first row
-  const float* xw = S.xw(int(m.tb));
+  const float* xw = S.xw(int(m.wb));
   const int32_t wlo = tm.wlo;
   const uint32_t wlen = tm.wlen, wmax = tm.wlen ? tm.wlen - 1 : 0;
   const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -160,21 +169,29 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
     const int32_t* col = S.col(s);
     const float* val = S.val(s);
     const int32_t a0 = m.a0;
-    int c0[U], c1[U];
+    int base[U], len[U], c0[U], c1[U];
     float v0[U], v1[U], x0[U], x1[U];
+    bool longrow = false;
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       const uint32_t lr = u * (kComputeWarps * 4) + w * 4 + (lane >> 3);
-      lo[u] = 0; hi[u] = 0; acc[u] = 0.f;
-      if (lr < nrows) { lo[u] = rp[lr] - a0 + l; hi[u] = rp[lr + 1] - a0; }
+      const int32_t r0v = rp[lr], r1v = rp[lr + 1];   // inside the task buffer even past nrows
+      const bool in = lr < nrows;
+      len[u] = in ? r1v - r0v : 0;
+      base[u] = in ? r0v - a0 + l : 0;                 // >= 0; a row's reads stay inside shared memory
+      longrow |= len[u] > 16;
+      lo[u] = base[u];
+      hi[u] = base[u] - l + len[u];
+      acc[u] = 0.f;
     }
+    // the first two elements of each lane's chain (rows of <= 16 nonzeros end
+    // here): loads are unconditional, the predicate is applied at the FMA
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      const bool h0 = lo[u] < hi[u], h1 = lo[u] + 8 < hi[u];
-      c0[u] = col[h0 ? lo[u] : 0];
-      v0[u] = val[h0 ? lo[u] : 0];
-      c1[u] = col[h1 ? lo[u] + 8 : 0];
-      v1[u] = val[h1 ? lo[u] + 8 : 0];
+      c0[u] = col[base[u]];
+      v0[u] = val[base[u]];
+      c1[u] = col[base[u] + 8];
+      v1[u] = val[base[u] + 8];
     }
     bool miss = false;
 #pragma unroll
@@ -182,23 +199,25 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
       const uint32_t d0 = uint32_t(c0[u] - wlo), d1 = uint32_t(c1[u] - wlo);
       x0[u] = xw[min(d0, wmax)];
       x1[u] = xw[min(d1, wmax)];
-      miss |= (lo[u] < hi[u] && d0 >= wlen) || (lo[u] + 8 < hi[u] && d1 >= wlen);
+      miss |= (l < len[u] && d0 >= wlen) || (l + 8 < len[u] && d1 >= wlen);
     }
     if (__any_sync(0xffffffffu, miss)) {
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        if (lo[u] < hi[u] && uint32_t(c0[u] - wlo) >= wlen) x0[u] = __ldg(xg + c0[u]);
-        if (lo[u] + 8 < hi[u] && uint32_t(c1[u] - wlo) >= wlen) x1[u] = __ldg(xg + c1[u]);
+        if (l < len[u] && uint32_t(c0[u] - wlo) >= wlen) x0[u] = __ldg(xg + c0[u]);
+        if (l + 8 < len[u] && uint32_t(c1[u] - wlo) >= wlen) x1[u] = __ldg(xg + c1[u]);
       }
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      if (lo[u] < hi[u]) acc[u] = __fmaf_rn(v0[u], x0[u], acc[u]);
-      if (lo[u] + 8 < hi[u]) acc[u] = __fmaf_rn(v1[u], x1[u], acc[u]);
+      acc[u] = l < len[u] ? __fmaf_rn(v0[u], x0[u], 0.f) : 0.f;
+      acc[u] = l + 8 < len[u] ? __fmaf_rn(v1[u], x1[u], acc[u]) : acc[u];
     }
+    if (__any_sync(0xffffffffu, longrow)) {
 #pragma unroll
-    for (int u = 0; u < U; ++u)     // rows longer than 16: the rest of the chain, still ascending
-      for (int j = lo[u] + 16; j < hi[u]; j += 8) acc[u] = __fmaf_rn(val[j], xval(col[j]), acc[u]);
+      for (int u = 0; u < U; ++u)   // rows longer than 16: the rest of the chain, still ascending
+        for (int j = lo[u] + 16; j < hi[u]; j += 8) acc[u] = __fmaf_rn(val[j], xval(col[j]), acc[u]);
+    }
   } else {
     // the chunk's nonzeros did not fit the slot: the same chain from global memory
     const int32_t* col = reinterpret_cast<const int32_t*>(a.col);
@@ -228,7 +247,8 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   Smem S;
   S.h = reinterpret_cast<Hdr*>(smem_raw);
   S.slots = smem_raw + kHdrBytes;
-  S.tasks = S.slots + kSlots * kSlotBytes;
+  S.rpb = S.slots + kSlots * kSlotBytes;
+  S.win = S.rpb + kRpBufs * kRpInts * 4;
   Hdr& H = *S.h;
   const slate_args_spmv& a = p.args;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -238,10 +258,13 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       mbar_init(&H.slot_full[i], 1);              // the chunk warp's expect_tx arrive (+ bytes)
       mbar_init(&H.slot_empty[i], kComputeWarps); // every compute warp
     }
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&H.task_rp[i], 1);                // the task warp's expect_tx arrive (+ rp bytes)
-      mbar_init(&H.task_win[i], 1);               // the task warp's expect_tx arrive (+ x bytes)
-      mbar_init(&H.task_empty[i], kComputeWarps + 1);   // every compute warp + the chunk warp
+    for (int i = 0; i < kRpBufs; ++i) {
+      mbar_init(&H.rp_full[i], 32);               // every lane of the task warp (plain loads + stores)
+      mbar_init(&H.rp_empty[i], kComputeWarps);   // every compute warp, after the task's last chunk
+    }
+    for (int i = 0; i < kWinBufs; ++i) {
+      mbar_init(&H.win_full[i], 1);               // the chunk warp's expect_tx arrive (+ x bytes)
+      mbar_init(&H.win_empty[i], kComputeWarps);
     }
     fence_mbar_init();
     // ---- Lst1: bind to the SM, standby while under-staffed
@@ -256,84 +279,104 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   if (!H.go) return;
 
   if (warp == kTaskWarp) {
-    // ===================== task warp: the slate task protocol + task buffers =====================
+    // ===================== task warp: the slate task protocol + row-pointer slices =====================
     uint64_t c = H.ctrl;
     const uint32_t rank = H.rank;
     TRACE_DECL;
+    // Speculative boundary (as the generic worker's kSpeculative mode): the
+    // decision for task t+1 -- retire, or the counter atomic -- is taken when
+    // task t's slice is fetched, from the resize word loaded one boundary
+    // earlier, so neither round trip sits on the task warp's critical path; a
+    // resize is honoured within two task boundaries.
+    uint64_t c_pre = c;                   // the resize word for the next boundary (lane 0)
+    uint32_t g_next = 0xffffffffu;        // raw counter value fetched for the next task (lane 0)
+    bool next_ret = false;
+    if (lane == 0) {                      // the first boundary is not speculative
+      if (!in_range(p, rank, c) && try_retire(p.tc)) {
+        next_ret = true;
+      } else {
+        g_next = atomicAdd(&p.tc->next, p.iters);                     // Lst2 (2)
+      }
+      c_pre = ld_acquire_u64(p.ctrl);
+    }
     for (uint32_t t = 0;; ++t) {
-      const int b = int(t & 1);
-      const uint32_t use = t >> 1;
+      const int b = int(t % kRpBufs);
       uint32_t g = 0xffffffffu, chg = 0;
       if (lane == 0) {
         TRACE(0, 0, t, 0);
-        mbar_wait(&H.task_empty[b], (use & 1) ^ 1);   // task t-2 fully consumed
-        TRACE(0, 1, t, 0);
-        // task boundary: the resize word, then the counter
-        const uint64_t c2 = ld_acquire_u64(p.ctrl);
-        chg = ctrl_epoch(c2) != ctrl_epoch(c);
-        c = c2;
-        if (!in_range(p, rank, c) && try_retire(p.tc)) {
+        // resolve the fetch taken at the previous boundary
+        if (next_ret) {
           H.retired = 1;
+        } else if (g_next < p.B) {
+          g = g_next;
+          TRACE(0, 2, t, g);
+          if (g == 0) p.tc->t_first = globaltimer();
         } else {
-          const uint32_t f = atomicAdd(&p.tc->next, p.iters);          // Lst2 (2)
-          if (f < p.B) {
-            g = f;
-            TRACE(0, 2, t, g);
-            if (f == 0) p.tc->t_first = globaltimer();
-          } else {
-            atomicAdd(&p.tc->live_pending, ~0ull);                      // drained: live -= 1
-          }
+          atomicAdd(&p.tc->live_pending, ~0ull);                        // drained: live -= 1
         }
+        // task boundary for task t+1, taken now
+        next_ret = false;
+        g_next = 0xffffffffu;
+        if (g != 0xffffffffu) {
+          chg = ctrl_epoch(c_pre) != ctrl_epoch(c);
+          c = c_pre;
+          if (!in_range(p, rank, c) && try_retire(p.tc)) next_ret = true;
+          else g_next = atomicAdd(&p.tc->next, p.iters);              // Lst2 (2); result used next round
+          c_pre = ld_acquire_u64(p.ctrl);
+        }
+        mbar_wait(&H.rp_empty[b], ((t / kRpBufs) & 1) ^ 1);         // task t-4 fully consumed
+        TRACE(0, 1, t, 0);
       }
       g = __shfl_sync(0xffffffffu, g, 0);
       chg = __shfl_sync(0xffffffffu, chg, 0);
       c = __shfl_sync(0xffffffffu, c, 0);
-      if (chg && g != 0xffffffffu) check_shrink_done(p, c, lane);
-      if (lane == 0) {
-        TaskMeta& tm = H.tmeta[b];
-        if (g == 0xffffffffu) {
-          tm.g = 0; tm.n = 0; tm.wlo = 0; tm.wlen = 0;
-          mbar_expect_tx(&H.task_rp[b], 0);           // sentinel: publishes the stop
-        } else {
-          const uint32_t n = min(p.iters, p.B - g);
-          const uint32_t r0 = g * 32, r1 = min(r0 + n * 32, a.n_rows);
-          // rp[r0 .. r1]: whole 16-B granules by the bulk engine, the last
-          // (r1 - r0 + 1) mod 4 entries by this thread (never reads past rp's end)
-          const uint32_t nbulk = (r1 - r0 + 1) & ~3u;
-          tm.g = g; tm.n = n;
-          // the window comes from the task's first and last nonzero (two loads
-          // that ride alongside the rp slice; the rp ends are needed for them)
-          const int32_t* rpg = reinterpret_cast<const int32_t*>(a.rowptr);
-          const int32_t e0 = __ldg(rpg + r0), e1 = __ldg(rpg + r1);
-          for (uint32_t i = nbulk; i <= r1 - r0; ++i) S.rp(b)[i] = __ldg(rpg + r0 + i);
-          mbar_expect_tx(&H.task_rp[b], nbulk * 4);  // (its release publishes tm and the tail)
-          if (nbulk) bulk_g2s(S.rp(b), rpg + r0, nbulk * 4, &H.task_rp[b]);
-          int32_t wlo = 0;
-          uint32_t wlen = 0;
-          if (e1 > e0) {
-            const int32_t* colg = reinterpret_cast<const int32_t*>(a.col);
-            const int32_t cf = __ldg(colg + e0), cl = __ldg(colg + e1 - 1);
-            const int32_t cmin = min(cf, cl), cmax = max(cf, cl);
-            const int32_t ncols = int32_t(a.n_cols);
-            const int32_t span = cmax - cmin + 1;
-            int32_t lo = span >= kWin ? cmin : cmin - (kWin - span) / 2;
-            lo = max(0, min(lo, ncols - kWin)) & ~3;
-            wlo = lo;
-            // whole granules inside x; columns past the window read global memory
-            wlen = uint32_t(max(0, min(kWin, ncols - lo)) & ~3);
-          }
-          tm.wlo = wlo;
-          tm.wlen = wlen;
-          TRACE(0, 3, t, wlen);
-          mbar_expect_tx(&H.task_win[b], wlen * 4);
-          if (wlen)
-            bulk_g2s_keep(S.xw(b), reinterpret_cast<const float*>(a.x) + wlo, wlen * 4, &H.task_win[b]);
-        }
-      }
+      if (chg) check_shrink_done(p, c, lane);
+      TaskMeta& tm = H.tmeta[b];
       if (g == 0xffffffffu) {
-        if (lane == 0) H.ctrl = c;                  // the word the CTA acted on last
+        if (lane == 0) {
+          tm.g = 0; tm.n = 0; tm.wlo = 0; tm.wlen = 0;
+          H.ctrl = c;                                 // the word the CTA acted on last
+        }
+        mbar_arrive(&H.rp_full[b]);                   // sentinel: publishes the stop
         break;
       }
+      // rp[r0 .. r1] by the whole warp: 16-B loads (r0 = 32 g is 128-B aligned), then the tail
+      const uint32_t n = min(p.iters, p.B - g);
+      const uint32_t r0 = g * 32, r1 = min(r0 + n * 32, a.n_rows);
+      const uint32_t cnt = r1 - r0 + 1, n4 = cnt / 4;
+      const int32_t* rpg = reinterpret_cast<const int32_t*>(a.rowptr) + r0;
+      int32_t* rps = S.rp(b);
+      constexpr int kV = (kRpInts / 4 + 31) / 32;
+      int4 v[kV];
+#pragma unroll
+      for (int k = 0; k < kV; ++k)
+        if (lane + 32 * k < n4) v[k] = __ldg(reinterpret_cast<const int4*>(rpg) + lane + 32 * k);
+#pragma unroll
+      for (int k = 0; k < kV; ++k)
+        if (lane + 32 * k < n4) reinterpret_cast<int4*>(rps)[lane + 32 * k] = v[k];
+      if (lane < cnt - n4 * 4) rps[n4 * 4 + lane] = __ldg(rpg + n4 * 4 + lane);
+      __syncwarp();
+      if (lane == 0) {
+        // the x window from the task's first and last nonzero
+        const int32_t e0 = rps[0], e1 = rps[r1 - r0];
+        int32_t wlo = 0;
+        uint32_t wlen = 0;
+        if (e1 > e0) {
+          const int32_t* colg = reinterpret_cast<const int32_t*>(a.col);
+          const int32_t cf = __ldg(colg + e0), cl = __ldg(colg + e1 - 1);
+          const int32_t cmin = min(cf, cl), cmax = max(cf, cl);
+          const int32_t ncols = int32_t(a.n_cols);
+          const int32_t span = cmax - cmin + 1;
+          int32_t lo = span >= kWin ? cmin : cmin - (kWin - span) / 2;
+          lo = max(0, min(lo, ncols - kWin)) & ~3;
+          wlo = lo;
+          // whole granules inside x; columns past the window read global memory
+          wlen = uint32_t(max(0, min(kWin, ncols - lo)) & ~3);
+        }
+        tm.g = g; tm.n = n; tm.wlo = wlo; tm.wlen = wlen;
+        TRACE(0, 3, t, wlen);
+      }
+      mbar_arrive(&H.rp_full[b]);                     // each lane after its stores (count 32)
     }
   } else if (warp == kChunkWarp) {
     // ===================== chunk warp: nonzeros of each task through the slot ring =====================
@@ -341,10 +384,16 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       TRACE_DECL;
       uint32_t q = 0;   // chunks issued
       for (uint32_t t = 0;; ++t) {
-        const int b = int(t & 1);
-        mbar_wait(&H.task_rp[b], (t >> 1) & 1);
+        const int b = int(t % kRpBufs), wb = int(t % kWinBufs);
+        mbar_wait(&H.rp_full[b], (t / kRpBufs) & 1);
         TRACE(1, 10, t, 0);
         const TaskMeta tm = H.tmeta[b];
+        if (tm.n) {                                   // the task's x window (task t-2 is done with the buffer)
+          mbar_wait(&H.win_empty[wb], ((t / kWinBufs) & 1) ^ 1);
+          mbar_expect_tx(&H.win_full[wb], tm.wlen * 4);
+          if (tm.wlen)
+            bulk_g2s_keep(S.xw(wb), reinterpret_cast<const float*>(a.x) + tm.wlo, tm.wlen * 4, &H.win_full[wb]);
+        }
         const uint32_t nch = tm.n ? (tm.n + kChunkBlocks - 1) / kChunkBlocks : 1;
         for (uint32_t k = 0; k < nch; ++k, ++q) {
           const int s = int(q % kSlots);
@@ -367,7 +416,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           // by this thread instead
           const bool end = r0 + nrows == a.n_rows;
           const int32_t a0 = e0 & ~3, a1 = end ? (e1 & ~3) : ((e1 + 3) & ~3);
-          m.tb = uint32_t(b); m.row0 = row0; m.nblk = nblk; m.a0 = a0;
+          m.tb = uint32_t(b); m.wb = uint32_t(wb); m.row0 = row0; m.nblk = nblk; m.a0 = a0;
           m.first = k == 0; m.last = k + 1 == nch;
           if (max(a1, e1) - a0 > kCap) {
             m.mode = 1;
@@ -387,32 +436,51 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           }
         }
         if (tm.n == 0) break;
-        mbar_arrive(&H.task_empty[b]);   // this warp is done reading the task's rp
       }
     }
   } else {
     // ===================== compute warps =====================
     uint32_t q = 0, t = 0, my_blocks = 0, my_tasks = 0;
     TRACE_DECL;
+#ifdef SLATE_SPMV_PROFILE
+    long long pf_wait = 0, pf_first = 0, pf_comp = 0, pf_t0 = clock64();
+#endif
     for (;; ++q) {
       const int s = int(q % kSlots);
+#ifdef SLATE_SPMV_PROFILE
+      long long c0 = clock64();
+#endif
       mbar_wait(&H.slot_full[s], (q / kSlots) & 1);
+#ifdef SLATE_SPMV_PROFILE
+      long long c1 = clock64();
+      pf_wait += c1 - c0;
+#endif
       if (threadIdx.x == 0) TRACE(2, 20, q, 0);
       const ChunkMeta m = H.cmeta[s];
       if (m.tb == 0xffffffffu) break;
       const int b = int(m.tb);
       if (m.first) {
-        mbar_wait(&H.task_rp[b], (t >> 1) & 1);
-        mbar_wait(&H.task_win[b], (t >> 1) & 1);
+        mbar_wait(&H.rp_full[b], (t / kRpBufs) & 1);
+        mbar_wait(&H.win_full[m.wb], (t / kWinBufs) & 1);
       }
       const TaskMeta tm = H.tmeta[b];
       if (threadIdx.x == 0) TRACE(2, 21, q, 0);
+#ifdef SLATE_SPMV_PROFILE
+      long long c2 = clock64();
+      pf_first += c2 - c1;
+#endif
       compute_chunk(a, S, m, tm, s);
       __syncwarp();
+#ifdef SLATE_SPMV_PROFILE
+      pf_comp += clock64() - c2;
+#endif
       if (threadIdx.x == 0) TRACE(2, 22, q, 0);
       if (lane == 0) {
         mbar_arrive(&H.slot_empty[s]);
-        if (m.last) mbar_arrive(&H.task_empty[b]);
+        if (m.last) {
+          mbar_arrive(&H.rp_empty[b]);
+          mbar_arrive(&H.win_empty[m.wb]);
+        }
       }
       if (threadIdx.x == 0) {
         my_blocks += m.nblk;
@@ -425,6 +493,12 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       }
     }
     if (threadIdx.x == 0 && my_blocks) count_done(p, my_blocks, my_tasks);
+#ifdef SLATE_SPMV_PROFILE
+    if (lane == 0 && blockIdx.x < 148) {
+      long long* o = spmv_prof[blockIdx.x][warp];
+      o[0] = clock64() - pf_t0; o[1] = pf_wait; o[2] = pf_first; o[3] = pf_comp; o[4] = q;
+    }
+#endif
   }
   __syncthreads();
   if (warp == kTaskWarp) {

@@ -123,5 +123,15 @@ int main(int argc, char** argv) {
     for (auto& x : ev) printf("cta %d %9.3f us  %s\n", c, (x.first - t0) / 1e3, x.second.c_str());
   }
 #endif
+#ifdef SLATE_SPMV_PROFILE
+  ws_worker(32, 148);
+  static long long pr[148][32][5];
+  CK(cudaMemcpyFromSymbol(pr, spmv::spmv_prof, sizeof(pr)));
+  for (int c : {0, 1, 70, 147}) for (int w : {0, 7, 15}) {
+    long long* o = pr[c][w];
+    printf("cta %3d warp %2d: total %7lld clk  wait-full %6.1f%%  first-chunk %5.1f%%  compute %5.1f%%  chunks %lld  (%.0f clk/chunk compute)\n",
+           c, w, o[0], 100.0 * o[1] / o[0], 100.0 * o[2] / o[0], 100.0 * o[3] / o[0], o[4], o[4] ? double(o[3]) / o[4] : 0.0);
+  }
+#endif
   return 0;
 }
