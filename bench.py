@@ -316,7 +316,8 @@ def make_c3(S, dev):
 
 
 def submit(sess, kernel, job, **kw):
-    return [sess.launch(kernel, job.args, job.grid, **kw) for _ in range(job.reps)]
+    """A job: `reps` launches of its kernel in one slate_launch_n call."""
+    return sess.launch_n(kernel, job.args, job.grid, job.reps, **kw)
 
 
 def collect(sess, ids):
@@ -360,11 +361,25 @@ def run_schedule(name, w, sA, sB, kA, kB, S):
         spin_ms(w.arrival_ms)
         ib = submit(sB, kB, b, placement=S.PLACE_AUTO)
         qa, qb = collect(sA, ia), collect(sB, ib)
+    elif name == "slate_table":     # Slate AUTO with the paper's Tab I alone deciding (reading Q8)
+        sA.set_policy(S.POLICY_TABLE)
+        try:
+            ia = submit(sA, kA, a, placement=S.PLACE_AUTO)
+            spin_ms(w.arrival_ms)
+            ib = submit(sB, kB, b, placement=S.PLACE_AUTO)
+            qa, qb = collect(sA, ia), collect(sB, ib)
+        finally:
+            sA.set_policy(S.POLICY_HYBRID)
     elif name == "slate_forced":    # co-run regardless of Tab I, split from the T(s) curves
+        # B's first launch is placed on the top s_b SMs (A shrinks); the rest of
+        # B's job queues behind it on the same range, and when A's job drains
+        # the server grows B to every SM -- the AUTO co-run's shape
         n, s_b = w.n_sms, w.split
         ia = submit(sA, kA, a, placement=S.PLACE_AUTO)
         spin_ms(w.arrival_ms)
-        ib = submit(sB, kB, b, placement=S.PLACE_CORUN, sm=(n - s_b, n - 1))
+        ib = [sB.launch(kB, b.args, b.grid, placement=S.PLACE_CORUN, sm=(n - s_b, n - 1))]
+        if b.reps > 1:
+            ib += sB.launch_n(kB, b.args, b.grid, b.reps - 1, placement=S.PLACE_AUTO)
         qa, qb = collect(sA, ia), collect(sB, ib)
     else:
         raise ValueError(name)
@@ -457,10 +472,13 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     cap = frac < 1.0
     lo_b = w.n_sms - S.saturation_sms(ca, w.n_sms, frac) if cap and mem_a and not mem_b else 0
     hi_b = S.saturation_sms(cb, w.n_sms, frac) if cap and mem_b and not mem_a else 0
-    w.split, _ = S.choose_split(ca, cb, w.n_sms, 2, lo_b, hi_b)
+    # job-level curves: a job is `reps` launches of its kernel
+    ja = {k: v * w.a.reps for k, v in ca.items()}
+    jb = {k: v * w.b.reps for k, v in cb.items()}
+    w.split, _ = S.choose_split(ja, jb, w.n_sms, 2, lo_b, hi_b)
     w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
     base = {}
-    for name in ("seq_cuda", "seq_slate", "streams", "slate_forced"):
+    for name in ("seq_cuda", "seq_slate", "streams", "slate_table", "slate_forced"):
         run_schedule(name, w, sA, sB, kA, kB, S)
         base[name] = median_schedule(name, w, sA, sB, kA, kB, S, flush, 3)
     solo_a = base["seq_cuda"][1]

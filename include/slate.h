@@ -193,6 +193,16 @@ typedef struct {
  * ENOTFOUND (kernel), ENOMEM (control-block pool exhausted), ECUDA. */
 slate_status slate_launch(slate_session* s, slate_kernel k, const slate_launch_desc* d, slate_launch_id* out);
 
+/* n (>= 1) launches of the same kernel and descriptor in one call: a job of
+ * n back-to-back kernels (the paper's applications loop over their kernels,
+ * P:L291).  All n are queued before the selector considers the queue, so a
+ * co-run decision and its split see the whole job (reading Q31), and the
+ * client pays one round trip to the server instead of n.  The ids
+ * are *first .. *first + n - 1.  Errors: as slate_launch; on an error after
+ * some launches were queued, those stay queued and *first names the first. */
+slate_status slate_launch_n(slate_session* s, slate_kernel k, const slate_launch_desc* d, uint32_t n,
+                            slate_launch_id* first);
+
 /* Resize the SM range of the queue that owns launch l to [sm_lo, sm_hi]
  * (§III-C; the dispatcher's start_sm/end_sm, Lst3 P:L250-251).
  * Publishes {epoch+1, lo, hi} to the device with a stream memory write that
@@ -326,6 +336,29 @@ uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t 
  * gains little bandwidth but raises the HBM latency its compute-bound partner
  * sees. */
 uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n, uint32_t n_sms, double frac);
+/* Reading Q31 (the B200 selector): should kernel B co-run with the active A
+ * although Tab I says solo?  Job curves are `work` launches of each kernel
+ * (the launches queued or running) back to back, time = work * curve(s); the
+ * split is slate_choose_split over the job curves and the predicted gain is
+ * (T_A(n) + T_B(n)) / makespan(split).  Returns 1 iff gain >= min_gain;
+ * *split and *gain (may be NULL) receive the split and the gain. */
+int slate_fluid_corun(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, double work_a,
+                      const uint32_t* sms_b, const double* ms_b, uint32_t n_b, double work_b,
+                      uint32_t n_sms, uint32_t step, uint32_t lo_b, uint32_t hi_b, double min_gain,
+                      uint32_t* split, double* gain);
+
+/* Selector policy of the server (process-wide; the initial value comes from
+ * SLATE_POLICY = table | literal | hybrid in the server's environment, default
+ * hybrid).  TABLE: Tab I, symmetric reading (Q8); LITERAL: Tab I as printed;
+ * HYBRID: Tab I, and where it says solo the fluid model over the measured
+ * solo curves and the queued work (slate_fluid_corun, gain >= 1.05) may still
+ * co-run the pair (Q31).  In every policy a co-running pair's split is re-taken
+ * from the job curves as launches arrive (resizing both queues).
+ * Errors: EINVAL (unknown policy). */
+#define SLATE_POLICY_TABLE   0u
+#define SLATE_POLICY_LITERAL 1u
+#define SLATE_POLICY_HYBRID  2u
+slate_status slate_set_policy(slate_session* s, uint32_t policy);
 
 #ifdef __cplusplus
 }

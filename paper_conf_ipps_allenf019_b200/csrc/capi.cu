@@ -187,11 +187,28 @@ slate_status slate_launch(slate_session* s, slate_kernel k, const slate_launch_d
   return rc == SLATE_OK ? rc : fail(s, rc, err);
 }
 
+slate_status slate_launch_n(slate_session* s, slate_kernel k, const slate_launch_desc* d, uint32_t n,
+                            slate_launch_id* first) {
+  if (!s || !d || !first || n == 0) return fail(s, SLATE_EINVAL, "null argument or n == 0");
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  const int rc = s->srv ? s->srv->launch_n(s->queue, k, d, n, first, &err) : s->remote->launch_n(k, d, n, first, &err);
+  return rc == SLATE_OK ? rc : fail(s, rc, err);
+}
+
 slate_status slate_resize(slate_session* s, slate_launch_id l, uint32_t lo, uint32_t hi) {
   if (!s) return SLATE_EINVAL;
   std::lock_guard<std::mutex> g(s->mu);
   std::string err;
   const int rc = s->srv ? s->srv->resize(s->queue, l, lo, hi, &err) : s->remote->resize(l, lo, hi, &err);
+  return rc >= SLATE_OK ? rc : fail(s, rc, err);
+}
+
+slate_status slate_set_policy(slate_session* s, uint32_t policy) {
+  if (!s) return SLATE_EINVAL;
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  const int rc = s->srv ? s->srv->set_policy(policy, &err) : s->remote->set_policy(policy, &err);
   return rc >= SLATE_OK ? rc : fail(s, rc, err);
 }
 

@@ -220,12 +220,33 @@ int RemoteClient::launch(uint64_t k, const slate_launch_desc* d, uint64_t* out, 
   return rc;
 }
 
+int RemoteClient::launch_n(uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err) {
+  Request rq{};
+  rq.cmd = CMD_LAUNCH;
+  rq.id = k;
+  rq.lo = n;   // launches in the batch (0 or 1: one)
+  int rc = pack_launch(rq, d, err);
+  if (rc != SLATE_OK) return rc;
+  Response rs;
+  rc = call(rq, &rs, err);
+  if (rc == SLATE_OK) *first = rs.out;
+  return rc;
+}
+
 int RemoteClient::resize(uint64_t l, uint32_t lo, uint32_t hi, std::string* err) {
   Request rq{};
   rq.cmd = CMD_RESIZE;
   rq.id = l;
   rq.lo = lo;
   rq.hi = hi;
+  Response rs;
+  return call(rq, &rs, err);
+}
+
+int RemoteClient::set_policy(uint32_t policy, std::string* err) {
+  Request rq{};
+  rq.cmd = CMD_POLICY;
+  rq.lo = policy;
   Response rs;
   return call(rq, &rs, err);
 }

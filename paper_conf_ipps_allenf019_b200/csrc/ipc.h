@@ -28,7 +28,7 @@ constexpr int kMaxArgs = 256;
 
 enum Cmd : uint32_t {
   CMD_NONE = 0, CMD_INFO, CMD_SHARE, CMD_UNSHARE, CMD_REGISTER, CMD_LAUNCH, CMD_RESIZE, CMD_SYNC, CMD_PROFILE,
-  CMD_QUERY, CMD_DETACH
+  CMD_QUERY, CMD_DETACH, CMD_POLICY
 };
 
 struct Request {
@@ -94,7 +94,9 @@ class RemoteClient {
   int unshare(uint64_t handle, std::string* err);
   int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
   int launch(uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err);
+  int launch_n(uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err);
   int resize(uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
+  int set_policy(uint32_t policy, std::string* err);
   int sync(uint64_t l, int64_t timeout_us, std::string* err);
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);

@@ -106,4 +106,20 @@ uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t 
   return best_s;
 }
 
+int slate_fluid_corun(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, double work_a, const uint32_t* sms_b,
+                      const double* ms_b, uint32_t n_b, double work_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
+                      uint32_t hi_b, double min_gain, uint32_t* split, double* gain) {
+  // job curves: `work` launches of the kernel, back to back on the same SMs
+  std::vector<double> ja(ms_a, ms_a + n_a), jb(ms_b, ms_b + n_b);
+  for (double& v : ja) v *= work_a;
+  for (double& v : jb) v *= work_b;
+  double t_co = 0;
+  const uint32_t s = slate_choose_split(sms_a, ja.data(), n_a, sms_b, jb.data(), n_b, n_sms, step, lo_b, hi_b, &t_co);
+  const double t_seq = interp(sms_a, ja.data(), n_a, n_sms) + interp(sms_b, jb.data(), n_b, n_sms);
+  const double g = t_co > 0 ? t_seq / t_co : 0.0;
+  if (split) *split = s;
+  if (gain) *gain = g;
+  return g >= min_gain ? 1 : 0;
+}
+
 }  // extern "C"

@@ -164,7 +164,8 @@ int Session::handle(const Request& rq, Response& rs) {
         rc = SLATE_EINVAL;
         break;
       }
-      if (rq.cmd == CMD_LAUNCH) rc = srv_->launch(queue_, rq.id, &d, &rs.out, &err);
+      if (rq.cmd == CMD_LAUNCH && rq.lo > 1) rc = srv_->launch_n(queue_, rq.id, &d, rq.lo, &rs.out, &err);
+      else if (rq.cmd == CMD_LAUNCH) rc = srv_->launch(queue_, rq.id, &d, &rs.out, &err);
       else rc = srv_->profile(rq.id, &d, rq.flags, &rs.prof, &err);
       break;
     }
@@ -173,6 +174,9 @@ int Session::handle(const Request& rq, Response& rs) {
       break;
     case CMD_SYNC:
       rc = srv_->sync(queue_, rq.id, rq.timeout_us, &err);
+      break;
+    case CMD_POLICY:
+      rc = srv_->set_policy(rq.lo, &err);
       break;
     case CMD_QUERY:
       rc = srv_->query(rq.id, &rs.linfo, &err);

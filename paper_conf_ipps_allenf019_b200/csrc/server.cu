@@ -130,6 +130,11 @@ int Server::init(std::string* err) {
   peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
   standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
   saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.95);   // reading Q29 (1.0: no cap)
+  if (const char* pol = std::getenv("SLATE_POLICY")) {              // reading Q31
+    const std::string v(pol);
+    policy_ = v == "table" ? SLATE_POLICY_TABLE : v == "literal" ? SLATE_POLICY_LITERAL : SLATE_POLICY_HYBRID;
+  }
+  min_gain_ = env_double("SLATE_MIN_GAIN", 1.05);
   poller_ = std::thread([this] { poller_main(); });
   return SLATE_OK;
 }
@@ -639,6 +644,29 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
 // ------------------------------------------------------------------ launch
 int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_t* out, std::string* err) {
   std::unique_lock<std::mutex> g(mu_);
+  return launch_locked(q, kid, d, out, err, false);
+}
+
+// n launches of one kernel in one call (a job): all are queued before the
+// selector looks at them, so a co-run decision sees the whole job
+int Server::launch_n(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint32_t n, uint64_t* first,
+                     std::string* err) {
+  if (n == 0) {
+    if (err) *err = "n == 0";
+    return SLATE_EINVAL;
+  }
+  std::unique_lock<std::mutex> g(mu_);
+  int rc = SLATE_OK;
+  for (uint32_t i = 0; i < n && rc == SLATE_OK; ++i) {
+    uint64_t id = 0;
+    rc = launch_locked(q, kid, d, &id, err, i + 1 < n);
+    if (i == 0) *first = id;
+  }
+  return rc;
+}
+
+int Server::launch_locked(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_t* out, std::string* err,
+                          bool defer) {
   auto qi = queues_.find(q);
   if (qi == queues_.end()) return SLATE_ENOTFOUND;
   auto ki = kernels_.find(kid);
@@ -708,10 +736,11 @@ int Server::launch(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_
     if (rc == SLATE_OK) rc = issue(LL, Q, err);
   } else if (Q.active) {
     rc = issue(LL, Q, err);
+    if (rc == SLATE_OK && Q.auto_split && !defer) resplit();
   } else {
     Q.pending.push_back(LL.id);
     if (std::find(waiting_.begin(), waiting_.end(), Q.id) == waiting_.end()) waiting_.push_back(Q.id);
-    schedule();
+    if (!defer) schedule();
   }
   if (rc != SLATE_OK) fail_launch(LL, int(cudaErrorLaunchFailure));
   return rc;
@@ -744,6 +773,101 @@ int Server::category_of(const Launch& L) const {
 static const slate_profile_t* find_profile(const std::map<std::string, ProfileEntry>& t, const std::string& key) {
   auto it = t.find(key);
   return it == t.end() ? nullptr : &it->second.p;
+}
+
+int Server::set_policy(uint32_t policy, std::string* err) {
+  if (policy > SLATE_POLICY_HYBRID) {
+    if (err) *err = "unknown policy";
+    return SLATE_EINVAL;
+  }
+  std::lock_guard<std::mutex> g(mu_);
+  policy_ = policy;
+  return SLATE_OK;
+}
+
+// the launch's solo curve from the profile table, ascending in SMs
+bool Server::curve_of(const Launch& L, std::vector<uint32_t>* sms, std::vector<double>* ms) const {
+  slate_launch_desc d = L.desc;
+  d.args = L.args.data();
+  const slate_profile_t* p = find_profile(profiles_, profile_key(*L.k, &d));
+  if (!p || p->n_curve < 2) return false;
+  sms->clear();
+  ms->clear();
+  for (int i = int(p->n_curve) - 1; i >= 0; --i) {   // stored in descending SM order
+    sms->push_back(p->curve_sms[i]);
+    ms->push_back(p->curve_ms[i]);
+  }
+  return true;
+}
+
+// SMs for B's queue (A keeps the rest) from the job curves of both queues:
+// each queue's remaining launches (running + waiting) of its head kernel back
+// to back (reading Q10 over jobs, Q31), with the Q29 saturation cap; n/2 when
+// a curve is missing.  *gain = the predicted T_seq / T_corun.
+uint32_t Server::pair_split(const Launch& LA, const Queue& A, const Launch& LB, const Queue& B, int catA, int catB,
+                            double* gain) const {
+  *gain = 0;
+  std::vector<uint32_t> sa, sb;
+  std::vector<double> ta, tb;
+  if (!curve_of(LA, &sa, &ta) || !curve_of(LB, &sb, &tb)) return uint32_t(n_sms_ / 2);
+  const bool memA = catA >= 3, memB = catB >= 3;
+  uint32_t lo_b = 0, hi_b = 0;
+  if (saturation_frac_ < 1.0 && memB && !memA)
+    hi_b = slate_saturation_sms(sb.data(), tb.data(), uint32_t(sb.size()), uint32_t(n_sms_), saturation_frac_);
+  if (saturation_frac_ < 1.0 && memA && !memB)
+    lo_b = uint32_t(n_sms_) - slate_saturation_sms(sa.data(), ta.data(), uint32_t(sa.size()), uint32_t(n_sms_),
+                                                   saturation_frac_);
+  const double wa = double(std::max<size_t>(1, A.issued.size() + A.pending.size()));
+  const double wb = double(std::max<size_t>(1, B.issued.size() + B.pending.size()));
+  uint32_t s = uint32_t(n_sms_ / 2);
+  slate_fluid_corun(sa.data(), ta.data(), uint32_t(sa.size()), wa, sb.data(), tb.data(), uint32_t(sb.size()), wb,
+                    uint32_t(n_sms_), 2, lo_b, hi_b, min_gain_, &s, gain);
+  return s;
+}
+
+// A co-running pair on the selector's split: as launches arrive the jobs
+// grow, so the split is re-taken from the job curves; a change of >= 6 SMs
+// resizes both queues (shrink one, grow the other).
+void Server::resplit() {
+  if (active_.size() != 2) return;
+  Queue& A = *queues_[active_[0]];
+  Queue& B = *queues_[active_[1]];
+  if (!A.auto_split || !B.auto_split || A.explicit_range || B.explicit_range) return;
+  const uint64_t la = !A.pending.empty() ? A.pending.front() : (!A.issued.empty() ? A.issued.back() : 0);
+  const uint64_t lb = !B.pending.empty() ? B.pending.front() : (!B.issued.empty() ? B.issued.back() : 0);
+  if (!la || !lb) return;
+  const Launch& LA = *launches_[la];
+  const Launch& LB = *launches_[lb];
+  const int catA = category_of(LA), catB = category_of(LB);
+  if (catA < 0 || catB < 0) return;
+  double g = 0;
+  const uint32_t s = pair_split(LA, A, LB, B, catA, catB, &g);
+  const uint32_t cur = B.hi - B.lo + 1;
+  if ((s > cur ? s - cur : cur - s) < 6) return;
+  if (std::getenv("SLATE_DEBUG"))
+    fprintf(stderr, "[slate] resplit: B %u -> %u SMs (A work %zu, B work %zu, gain %.3f)\n", cur, s,
+            A.issued.size() + A.pending.size(), B.issued.size() + B.pending.size(), g);
+  std::string err;
+  const uint32_t n = uint32_t(n_sms_);
+  Queue& shrink = s > cur ? A : B;
+  Queue& grow = s > cur ? B : A;
+  const uint32_t g_lo = grow.lo, g_hi = grow.hi;
+  const double t0 = now_us();
+  if (&shrink == &A) write_ctrl(A, 0, n - s - 1, true, &err);
+  else write_ctrl(B, n - s, n - 1, true, &err);
+  if (!shrink.issued.empty()) {
+    Launch& R = *launches_[shrink.issued.front()];
+    R.n_resizes += 1;
+    track_resize(R, shrink.epoch, 1, t0);
+  }
+  if (&grow == &A) write_ctrl(A, 0, n - s - 1, true, &err);
+  else write_ctrl(B, n - s, n - 1, true, &err);
+  if (!grow.issued.empty()) {
+    Launch& R = *launches_[grow.issued.back()];
+    R.n_resizes += 1;
+    track_resize(R, grow.epoch, 2, t0);
+  }
+  grow_running(grow, g_lo, g_hi, &err);
 }
 
 void Server::schedule() {
@@ -784,39 +908,31 @@ void Server::schedule() {
       byp.push_back(bypassed_[qid]);
       qids.push_back(qid);
     }
-    const int idx = slate_select(uint32_t(catA), cats.data(), byp.data(), uint32_t(cats.size()), 4, 0);
+    int idx = slate_select(uint32_t(catA), cats.data(), byp.data(), uint32_t(cats.size()), 4,
+                           policy_ == SLATE_POLICY_LITERAL ? 1 : 0);
+    uint32_t s = uint32_t(n_sms_ / 2);
+    if (idx >= 0) {
+      const Launch& HB = *launches_[queues_[qids[idx]]->pending.front()];
+      double g = 0;
+      s = pair_split(*LA, A, HB, *queues_[qids[idx]], catA, int(cats[idx]), &g);
+    } else if (policy_ == SLATE_POLICY_HYBRID && cats[0] != 99u) {
+      // reading Q31: Tab I keeps the head of the queue waiting, but the measured
+      // solo curves and the queued work predict a co-run gain of >= min_gain_
+      const Launch& HB = *launches_[queues_[qids[0]]->pending.front()];
+      double g = 0;
+      const uint32_t s0 = pair_split(*LA, A, HB, *queues_[qids[0]], catA, int(cats[0]), &g);
+      if (g >= min_gain_) {
+        idx = 0;
+        s = s0;
+      }
+    }
+    if (std::getenv("SLATE_DEBUG"))
+      fprintf(stderr, "[slate] select: active cat %d, head cat %u, idx %d, split %u (A work %zu, B work %zu)\n", catA,
+              cats[0], idx, s, A.issued.size() + A.pending.size(),
+              idx >= 0 ? queues_[qids[idx]]->pending.size() : size_t(0));
     if (idx < 0) break;
     for (int i = 0; i < idx; ++i) bypassed_[qids[i]] += 1;
     Queue& Bq = *queues_[qids[idx]];
-    const Launch& HB = *launches_[Bq.pending.front()];
-    // split from the profile curves (reading Q10), else half
-    uint32_t s = uint32_t(n_sms_ / 2);
-    {
-      slate_launch_desc da = LA->desc, db = HB.desc;
-      da.args = LA->args.data();
-      db.args = HB.args.data();
-      const slate_profile_t* pa = find_profile(profiles_, profile_key(*LA->k, &da));
-      const slate_profile_t* pb = find_profile(profiles_, profile_key(*HB.k, &db));
-      if (pa && pb && pa->n_curve >= 2 && pb->n_curve >= 2) {
-        std::vector<uint32_t> sa, sb;
-        std::vector<double> ta, tb;
-        for (int i = int(pa->n_curve) - 1; i >= 0; --i) { sa.push_back(pa->curve_sms[i]); ta.push_back(pa->curve_ms[i]); }
-        for (int i = int(pb->n_curve) - 1; i >= 0; --i) { sb.push_back(pb->curve_sms[i]); tb.push_back(pb->curve_ms[i]); }
-        // curves are stored in descending SM order; interp wants ascending.
-        // Reading Q29: a memory-bound tenant paired with a compute-bound one gets
-        // no more SMs than it needs for 95% of its full-chip bandwidth
-        // (SLATE_SATURATION_FRAC; 1.0 turns the cap off).
-        const bool memA = catA >= 3, memB = category_of(HB) >= 3;
-        uint32_t lo_b = 0, hi_b = 0;
-        if (saturation_frac_ < 1.0 && memB && !memA)
-          hi_b = slate_saturation_sms(sb.data(), tb.data(), uint32_t(sb.size()), uint32_t(n_sms_), saturation_frac_);
-        if (saturation_frac_ < 1.0 && memA && !memB)
-          lo_b = uint32_t(n_sms_) -
-                 slate_saturation_sms(sa.data(), ta.data(), uint32_t(sa.size()), uint32_t(n_sms_), saturation_frac_);
-        s = slate_choose_split(sa.data(), ta.data(), uint32_t(sa.size()), sb.data(), tb.data(), uint32_t(sb.size()),
-                               uint32_t(n_sms_), 2, lo_b, hi_b, nullptr);
-      }
-    }
     const uint32_t old_lo = A.lo, old_hi = A.hi;
     const double t0 = now_us();
     write_ctrl(A, 0, uint32_t(n_sms_) - s - 1, true, &err);   // shrink the running kernel
@@ -831,6 +947,7 @@ void Server::schedule() {
     bypassed_.erase(Bq.id);
     Bq.active = true;
     Bq.explicit_range = false;
+    A.auto_split = Bq.auto_split = true;
     active_.push_back(Bq.id);
     write_ctrl(Bq, uint32_t(n_sms_) - s, uint32_t(n_sms_ - 1), false, &err);
     while (!Bq.pending.empty()) {
@@ -847,6 +964,8 @@ void Server::release(Queue& Q) {
   std::string err;
   Q.active = false;
   Q.explicit_range = false;
+  Q.auto_split = false;
+  for (uint32_t other : active_) queues_[other]->auto_split = false;
   active_.erase(std::remove(active_.begin(), active_.end(), Q.id), active_.end());
   if (active_.size() == 1) {
     // the survivor claims the released SMs, explicit placement or not

@@ -59,6 +59,7 @@ struct Queue {
   uint32_t epoch = 0, lo = 0, hi = 0;
   bool active = false;          // holds an SM range
   bool explicit_range = false;  // set by a CORUN placement
+  bool auto_split = false;      // co-running on a split the selector took (re-taken as work arrives)
   std::deque<uint64_t> pending; // launches waiting for SMs (AUTO/SOLO)
   std::deque<uint64_t> deferred;  // granted SMs but waiting for a control block (stream order)
   std::deque<uint64_t> issued;  // issued, not complete (stream order)
@@ -88,7 +89,9 @@ class Server {
 
   int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
   int launch(uint32_t q, uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err);
+  int launch_n(uint32_t q, uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err);
   int resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
+  int set_policy(uint32_t policy, std::string* err);
   int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);
@@ -96,6 +99,7 @@ class Server {
 
  private:
   // all private helpers are called with mu_ held
+  int launch_locked(uint32_t q, uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err, bool defer);
   int issue(Launch& L, Queue& Q, std::string* err);
   int issue_now(Launch& L, Queue& Q, std::string* err);
   void drain_deferred(Queue& Q);
@@ -104,6 +108,10 @@ class Server {
   int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
   void schedule();
   void release(Queue& Q);
+  bool curve_of(const Launch& L, std::vector<uint32_t>* sms, std::vector<double>* ms) const;
+  uint32_t pair_split(const Launch& LA, const Queue& A, const Launch& LB, const Queue& B, int catA, int catB,
+                      double* gain) const;
+  void resplit();
   void poll_once();
   void poller_main();
   int category_of(const Launch& L) const;
@@ -161,6 +169,8 @@ class Server {
   double peak_hbm_ = 6650.0, peak_fp32_ = 74400.0, peak_tc_ = 1590.0;
   uint32_t standby_timeout_ns_ = 200000;
   double saturation_frac_ = 0.95;
+  uint32_t policy_ = SLATE_POLICY_HYBRID;
+  double min_gain_ = 1.05;
 
   mutable std::mutex mu_;
   std::condition_variable cv_;       // state changes (completion, activation)

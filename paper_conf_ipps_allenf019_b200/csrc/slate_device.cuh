@@ -341,8 +341,10 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     } else if constexpr (!Tn::kSpeculative) {
       // the boundary's resize word is in flight during the task; the counter
       // atomic is one round trip at the boundary (fewer live registers than
-      // the speculative form below)
-      prefetch_ctrl();
+      // the speculative form below).  Long-task tenants (kLateCtrl) load the
+      // word at the boundary instead: one more round trip per task, but a
+      // resize is honoured after the running task rather than the next one.
+      if constexpr (!Tn::kLateCtrl) prefetch_ctrl();
       if constexpr (Tn::kHasTask) {
         Tn::cta_task(p.args, g, n, dyn_smem);
         if (p.cov && threadIdx.x == 0)
@@ -356,6 +358,7 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
           w.advance(p.gx, p.gy);
         }
       }
+      if constexpr (Tn::kLateCtrl) prefetch_ctrl();
       __syncthreads();
       my_blocks += n;
       my_tasks += 1;

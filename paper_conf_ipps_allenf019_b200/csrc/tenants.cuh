@@ -29,6 +29,7 @@ struct TenantBase {
   static constexpr bool kSpeculative = false; // fetch the next task while this one runs (+registers)
   static constexpr uint32_t kTasksPerWorker = 8; // auto task size aims at >= this many tasks per worker
   static constexpr bool kHasFini = false;   // cta_fini(smem): once per CTA before it exits
+  static constexpr bool kLateCtrl = false;  // read the resize word at the boundary, not at task start
 };
 
 // ------------------------------------------------------------------ bulk async copies (TMA engine)
@@ -316,6 +317,7 @@ struct BlackScholes : TenantBase {
   using Args = slate_args_bs;
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 4;
+  static constexpr bool kLateCtrl = true;    // a block is ~30 us at P = 32: honour a resize after it
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
   __device__ __forceinline__ static float poly(float K) {

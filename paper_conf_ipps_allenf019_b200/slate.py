@@ -133,6 +133,8 @@ for _name, _args in [
     ("slate_query", [ctypes.c_void_p, c_u64, _P(LaunchInfo)]),
     ("slate_serve", [ctypes.c_char_p, ctypes.c_int, c_u32]),
     ("slate_kind_geometry", [c_u32, _P(c_u32), _P(c_u32)]),
+    ("slate_set_policy", [ctypes.c_void_p, c_u32]),
+    ("slate_launch_n", [ctypes.c_void_p, c_u64, _P(LaunchDesc), c_u32, _P(c_u64)]),
 ]:
     getattr(_lib, _name).restype = c_i32
     getattr(_lib, _name).argtypes = _args
@@ -147,11 +149,16 @@ _lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c
                                     c_u32, _P(c_f64)]
 _lib.slate_saturation_sms.restype = c_u32
 _lib.slate_saturation_sms.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_u32, c_f64]
+_lib.slate_fluid_corun.restype = ctypes.c_int
+_lib.slate_fluid_corun.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_f64, _P(c_u32), _P(c_f64), c_u32, c_f64, c_u32,
+                                   c_u32, c_u32, c_u32, c_f64, _P(c_u32), _P(c_f64)]
+POLICY_TABLE, POLICY_LITERAL, POLICY_HYBRID = 0, 1, 2
 
 EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffer", "slate_unshare_buffer",
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
-            "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms"]
+            "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
+            "slate_fluid_corun", "slate_set_policy", "slate_launch_n"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -238,8 +245,19 @@ class Session:
         self._check(_lib.slate_launch(self._h, kernel, ctypes.byref(d), ctypes.byref(lid)), "slate_launch")
         return lid.value
 
+    def launch_n(self, kernel, args, grid, n, placement=PLACE_AUTO, sm=None, mode=MODE_SLATE, coverage=None):
+        """n launches of one kernel as one job; returns their ids."""
+        d = self._desc(args, grid, placement, sm, mode, coverage)
+        first = c_u64()
+        self._check(_lib.slate_launch_n(self._h, kernel, ctypes.byref(d), n, ctypes.byref(first)), "slate_launch_n")
+        return list(range(first.value, first.value + n))
+
     def resize(self, launch_id, lo, hi):
         return self._check(_lib.slate_resize(self._h, launch_id, lo, hi), "slate_resize")
+
+    def set_policy(self, policy):
+        """Selector policy of the server (POLICY_TABLE / LITERAL / HYBRID; reading Q31)."""
+        return self._check(_lib.slate_set_policy(self._h, policy), "slate_set_policy")
 
     def sync(self, launch_id=0, timeout_us=-1):
         return self._check(_lib.slate_sync(self._h, launch_id, timeout_us), "slate_sync")
@@ -286,6 +304,15 @@ def choose_split(curve_a, curve_b, n_sms, step=2, lo_b=0, hi_b=0):
     t = c_f64()
     s = _lib.slate_choose_split(sa, ta, na, sb, tb, nb, n_sms, step, lo_b, hi_b, ctypes.byref(t))
     return s, t.value
+
+
+def fluid_corun(curve_a, work_a, curve_b, work_b, n_sms, step=2, lo_b=0, hi_b=0, min_gain=1.05):
+    sa, ta, na = _curve(curve_a)
+    sb, tb, nb = _curve(curve_b)
+    s, g = c_u32(), c_f64()
+    r = _lib.slate_fluid_corun(sa, ta, na, work_a, sb, tb, nb, work_b, n_sms, step, lo_b, hi_b, min_gain,
+                               ctypes.byref(s), ctypes.byref(g))
+    return bool(r), s.value, g.value
 
 
 def saturation_sms(curve, n_sms, frac=0.9):

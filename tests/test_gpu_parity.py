@@ -127,3 +127,21 @@ def test_gemm_full_size_sampled(sess):
         tiles = [(0, 0), (63, 63)] + [(rng.randrange(64), rng.randrange(64)) for _ in range(22)]
         ok, err = t.check(outs, rows=tiles)
         assert ok, (mode, err)
+
+
+def test_launch_n_job(sess):
+    """slate_launch_n: a job of n launches in one call -- consecutive ids, every
+    launch complete with exact counters, the output the oracle's."""
+    t = make_triad(1024 * 40 + 3, 118, "int")
+    k = sess.register_kernel(t.kind, iters=4)
+    t.zero_outputs()
+    torch.cuda.synchronize()
+    ids = sess.launch_n(k, t.args, t.grid, 5)
+    assert ids == list(range(ids[0], ids[0] + 5))
+    sess.sync(0)
+    torch.cuda.synchronize()
+    B = int(np.prod(t.grid))
+    for i in ids:
+        q = sess.query(i)
+        assert q["state"] == 2 and q["blocks_done"] == B and q["tasks_done"] == -(-B // 4)
+    assert t.check(t.snapshot())[0]

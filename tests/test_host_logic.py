@@ -102,6 +102,22 @@ def test_choose_split_bounds_and_saturation_match_oracle(S):
         assert s1 == s2 or abs(OS.corun_makespan(ca, cb, 148, s1) - t2) <= 1e-9 * t2
 
 
+def test_fluid_corun_matches_oracle(S):
+    rng = random.Random(13)
+    pts = [148, 111, 74, 49, 37, 18]
+    for _ in range(200):
+        knee_a, knee_b = rng.uniform(10, 148), rng.uniform(10, 148)
+        ca = {s: rng.uniform(0.02, 0.5) * max(1.0, knee_a / s) for s in pts}
+        cb = {s: rng.uniform(0.02, 0.5) * max(1.0, knee_b / s) for s in pts}
+        wa, wb = rng.choice([1, 7, 64]), rng.choice([1, 13, 640])
+        lo = rng.choice([0, 0, rng.randrange(1, 148)])
+        hi = rng.choice([0, 0, rng.randrange(1, 148)])
+        r1 = S.fluid_corun(ca, wa, cb, wb, 148, 2, lo, hi)
+        r2 = OS.fluid_corun(ca, wa, cb, wb, 148, 2, lo, hi)
+        assert abs(r1[2] - r2[2]) <= 1e-9 * r2[2]
+        assert r1[0] == r2[0] or abs(r2[2] - 1.05) < 1e-9
+
+
 def test_kind_geometry(S):
     assert S.kind_geometry(S.KIND_TRIAD) == (1, 1024)
     assert S.kind_geometry(S.KIND_SGEMM_NAIVE) == (16, 16)

@@ -129,3 +129,24 @@ def test_metrics_closed_forms():
     assert M.utilisation(6.5e12, 1.0, 6.5e12) == 1.0
     # STP <= n for any schedule without super-linear speed-up
     assert M.stp([2, 3, 5], [2, 3, 5]) == 3.0
+
+
+def test_fluid_corun_reading_q31():
+    n = 148
+    pts = (18, 37, 74, 111, 148)
+    # both tenants scale linearly: no split beats running them back to back
+    lin = {k: 148.0 / k for k in pts}
+    ok, _, g = S.fluid_corun(lin, 1, lin, 1, n)
+    assert not ok and abs(g - 1.0) < 1e-9
+    # A scales linearly (1 ms on the chip), B saturates at 37 SMs (1 ms):
+    # by hand at s = 38, B ends at 1 ms while A ran at 110/148 of its rate, A's
+    # remaining 1 - 110/148 ends 38/148 ms later: makespan 1.2568 (the chooser
+    # may only do better), against 2 ms back to back
+    sat = {k: max(1.0, 37.0 / k) for k in pts}
+    ok, s, g = S.fluid_corun(lin, 1, sat, 1, n)
+    assert ok and g >= 2.0 / (1.0 + 38.0 / 148) - 1e-9 and 30 <= s <= 48
+    # the same pair with B's job 100x shorter: nothing worth a co-run
+    ok, _, g = S.fluid_corun(lin, 1, sat, 0.01, n)
+    assert not ok and g < 1.05
+    # work scales the jobs: 10 launches of A against 10 of B is the 1-vs-1 decision
+    assert S.fluid_corun(lin, 10, sat, 10, n)[1:] == pytest.approx(S.fluid_corun(lin, 1, sat, 1, n)[1:])
