@@ -548,6 +548,14 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
         roof = {"kernel": kname, "bound": "hbm", "achieved": round(ach, 1), "peak": peak_hbm,
                 "unit": "GB/s", "frac": round(ach / peak_hbm, 4), "peak_source": "MEASURED_PEAKS.json hbm_gbs"}
     roof["avg_launch_ms"] = round(avg, 5)
+    # the same kernel solo on every SM (the Slate-sequential schedule): in the
+    # co-run it holds only its share of the SMs, so its per-launch rate there
+    # is not its roofline position
+    solo_q = base["seq_slate"][3] if top == w.a.name else base["seq_slate"][4]
+    solo_avg = sum(q["end_ms"] - q["start_ms"] for q in solo_q) / len(solo_q)
+    roof["solo"] = {"avg_launch_ms": round(solo_avg, 5),
+                    "achieved": round(roof["achieved"] * avg / solo_avg, 3 if roof["unit"] != "GB/s" else 1),
+                    "frac": round(roof["frac"] * avg / solo_avg, 4)}
     roof["traffic"] = None
     ncu_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(ncu_path):
@@ -584,7 +592,12 @@ def run_slate(args, world, rank, local):
         clocks["c"] = Clocks(local)
         barrier(world)
         torch.cuda.synchronize()
+        nvtx = bool(os.environ.get("SLATE_NVTX"))   # profiling only: ncu --nvtx --nvtx-include "timed/"
+        if nvtx:
+            torch.cuda.nvtx.range_push("timed")
         out = loop()
+        if nvtx:
+            torch.cuda.nvtx.range_pop()
         torch.cuda.synchronize()
         barrier(world)
         clocks["r"] = clocks["c"].stop()
