@@ -29,7 +29,9 @@ model can show they are sufficient:
     workers than its target occ*|range| (so a launch cannot burn its whole grid
     on foreign SMs), and leaves when the target is met or the queue is drained;
     after a timeout with zero live workers it runs anyway;
-  * the last live worker of a tenant never retires while tasks remain.
+  * the last live worker of a tenant never retires while tasks remain (the
+    runtime decrements live and puts the unit back if it was the last:
+    ``Config.faa_retire``; the transient zero is explored too).
 
 ``simulate`` runs one seeded random interleaving; ``explore`` enumerates every
 interleaving of a tiny configuration (depth-first, memoised on state).  Both
@@ -43,7 +45,7 @@ class ProtocolViolation(AssertionError):
     pass
 
 
-PENDING, PROLOGUE, STANDBY, FETCH, EXEC, CHECK, EXITED = range(7)
+PENDING, PROLOGUE, STANDBY, FETCH, EXEC, CHECK, EXITED, RETIRING = range(8)
 
 
 @dataclass
@@ -57,6 +59,10 @@ class Config:
     resizes: list = field(default_factory=list)   # [(lo, hi), ...] applied in order at random times
     grid: int = 0             # CTAs per launch; default occ * ranks (one full wave)
     abort: bool = False       # long-task tenants: a retiring worker may abandon its task
+    faa_retire: bool = True   # retire as the runtime does it (Q22): live -= 1 in one atomic
+                              # step, and if that took live from 1 to 0, live += 1 in a later step
+                              # and stay; other CTAs may act in between.  False: one atomic
+                              # "retire unless last" step
                               # mid-way and return it (Q28)
 
 
@@ -111,7 +117,7 @@ class Model:
                 for r in range(self.cfg.ranks):
                     if self.resident[r] < self.cfg.occ:
                         acts.append(("place", i, r))
-            elif st in (PROLOGUE, FETCH, EXEC, CHECK):
+            elif st in (PROLOGUE, FETCH, EXEC, CHECK, RETIRING):
                 acts.append(("step", i))
                 # Q28: a worker outside the range may abandon its running task and
                 # retire, unless it is the last live worker (one atomic on {live, returned})
@@ -190,10 +196,22 @@ class Model:
         elif st == CHECK:
             # Lst2 (1) loop condition: retreat is examined only between tasks
             c[6] = self.epoch
-            if self.in_range(c) or (self.live == 1 and (self.next < cfg.blocks or self.returned)):
+            if self.in_range(c):
+                c[0] = FETCH
+            elif cfg.faa_retire:
+                was_last = self.live == 1
+                self.live -= 1             # fetch-and-add: live -= 1
+                c[0], c[5] = RETIRING, int(was_last)
+            elif self.live == 1 and (self.next < cfg.blocks or self.returned):
                 c[0] = FETCH               # stay (the last live worker never retires)
             else:
                 self.exit(c, True)         # exit (3): retreated
+        elif st == RETIRING:
+            if c[5]:                       # it was the last live worker: put the unit back, stay
+                self.live += 1
+                c[0] = FETCH
+            else:
+                self.exit(c, False)        # exit (3): retreated (its unit of live is already gone)
 
     # ------------------------------------------------------------ invariants
     def done(self):

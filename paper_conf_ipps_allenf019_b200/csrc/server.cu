@@ -34,6 +34,12 @@ static double env_double(const char* name, double dflt) {
 
 static uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
+// ranks in [a_lo, a_hi] ∩ [b_lo, b_hi] (empty ranges have lo > hi)
+static uint32_t overlap(uint32_t a_lo, uint32_t a_hi, uint32_t b_lo, uint32_t b_hi) {
+  const uint32_t lo = std::max(a_lo, b_lo), hi = std::min(a_hi, b_hi);
+  return lo > hi ? 0u : hi - lo + 1;
+}
+
 Server::Server(int device) : device_(device) {}
 
 Server::~Server() {
@@ -484,6 +490,8 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
   Q.epoch += 1;
   Q.lo = lo;
   Q.hi = hi;
+  Q.cov_lo = std::max(Q.cov_lo, lo);   // workers outside the new range retire
+  Q.cov_hi = std::min(Q.cov_hi, hi);
   const uint64_t v = pack_ctrl(Q.epoch, lo, hi);
   // a stream memory write needs no SM: it lands even while persistent workers fill every SM
   const CUresult r = reinterpret_cast<WriteValue64Fn>(write_value64_)(
@@ -577,6 +585,10 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     L.ev_done.push_back(ev_snap);
   }
   L.state = 1;
+  if (Q.issued.empty()) {
+    Q.cov_lo = Q.lo;
+    Q.cov_hi = Q.hi;
+  }
   Q.issued.push_back(L.id);
   cv_.notify_all();
   return SLATE_OK;
@@ -638,6 +650,13 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   R.ev_done.push_back(ev_snap);
   Q.topup_ends.push_back(ev_end);
   R.n_topups += 1;
+  if (Q.cov_lo > Q.cov_hi) {
+    Q.cov_lo = Q.lo;
+    Q.cov_hi = Q.hi;
+  } else {
+    Q.cov_lo = std::min(Q.cov_lo, Q.lo);
+    Q.cov_hi = std::max(Q.cov_hi, Q.hi);
+  }
   return SLATE_OK;
 }
 
@@ -842,7 +861,7 @@ void Server::resplit() {
   if (catA < 0 || catB < 0) return;
   double g = 0;
   const uint32_t s = pair_split(LA, A, LB, B, catA, catB, &g);
-  const uint32_t cur = B.hi - B.lo + 1;
+  const uint32_t cur = B.hi - B.lo + 1;   // B's SMs
   if ((s > cur ? s - cur : cur - s) < 6) return;
   if (std::getenv("SLATE_DEBUG"))
     fprintf(stderr, "[slate] resplit: B %u -> %u SMs (A work %zu, B work %zu, gain %.3f)\n", cur, s,
@@ -853,15 +872,18 @@ void Server::resplit() {
   Queue& grow = s > cur ? B : A;
   const uint32_t g_lo = grow.lo, g_hi = grow.hi;
   const double t0 = now_us();
-  if (&shrink == &A) write_ctrl(A, 0, n - s - 1, true, &err);
-  else write_ctrl(B, n - s, n - 1, true, &err);
+  // ranges for B holding s SMs on its side, A the rest
+  const uint32_t b_lo = B.low_side ? 0 : n - s, b_hi = B.low_side ? s - 1 : n - 1;
+  const uint32_t a_lo = B.low_side ? s : 0, a_hi = B.low_side ? n - 1 : n - s - 1;
+  if (&shrink == &A) write_ctrl(A, a_lo, a_hi, true, &err);
+  else write_ctrl(B, b_lo, b_hi, true, &err);
   if (!shrink.issued.empty()) {
     Launch& R = *launches_[shrink.issued.front()];
     R.n_resizes += 1;
     track_resize(R, shrink.epoch, 1, t0);
   }
-  if (&grow == &A) write_ctrl(A, 0, n - s - 1, true, &err);
-  else write_ctrl(B, n - s, n - 1, true, &err);
+  if (&grow == &A) write_ctrl(A, a_lo, a_hi, true, &err);
+  else write_ctrl(B, b_lo, b_hi, true, &err);
   if (!grow.issued.empty()) {
     Launch& R = *launches_[grow.issued.back()];
     R.n_resizes += 1;
@@ -935,7 +957,11 @@ void Server::schedule() {
     Queue& Bq = *queues_[qids[idx]];
     const uint32_t old_lo = A.lo, old_hi = A.hi;
     const double t0 = now_us();
-    write_ctrl(A, 0, uint32_t(n_sms_) - s - 1, true, &err);   // shrink the running kernel
+    // A keeps the side its running launch has workers on
+    const uint32_t n = uint32_t(n_sms_);
+    const bool a_high = !A.issued.empty() && overlap(A.cov_lo, A.cov_hi, s, n - 1) > overlap(A.cov_lo, A.cov_hi, 0, n - s - 1);
+    A.low_side = !a_high;
+    write_ctrl(A, a_high ? s : 0, a_high ? n - 1 : n - s - 1, true, &err);   // shrink the running kernel
     if (!A.issued.empty()) {
       Launch& R = *launches_[A.issued.front()];
       track_resize(R, A.epoch, 1, t0);
@@ -948,8 +974,9 @@ void Server::schedule() {
     Bq.active = true;
     Bq.explicit_range = false;
     A.auto_split = Bq.auto_split = true;
+    Bq.low_side = a_high;
     active_.push_back(Bq.id);
-    write_ctrl(Bq, uint32_t(n_sms_) - s, uint32_t(n_sms_ - 1), false, &err);
+    write_ctrl(Bq, a_high ? 0 : n - s, a_high ? s - 1 : n - 1, false, &err);
     while (!Bq.pending.empty()) {
       Launch& L = *launches_[Bq.pending.front()];
       Bq.pending.pop_front();
@@ -1105,6 +1132,10 @@ void Server::poll_once() {
       L.state = 2;
       Q.issued.pop_front();
       if (Q.issued.empty()) Q.topup_ends.clear();
+      else {                      // the next launch starts now, on the queue's current range
+        Q.cov_lo = Q.lo;
+        Q.cov_hi = Q.hi;
+      }
       cv_.notify_all();
     }
     if (Q.issued.empty()) Q.pending_resize.clear();   // nothing left to observe them on

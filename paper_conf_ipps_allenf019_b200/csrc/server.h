@@ -60,6 +60,12 @@ struct Queue {
   bool active = false;          // holds an SM range
   bool explicit_range = false;  // set by a CORUN placement
   bool auto_split = false;      // co-running on a split the selector took (re-taken as work arrives)
+  bool low_side = true;         // co-running: this queue holds the low ranks [0, k)
+  // ranks the running (front) launch has workers on: its range when it started,
+  // widened by top-ups, narrowed by shrinks (workers outside retire).  A queue
+  // is never shrunk onto ranks its running launch has no workers on (where a
+  // lone last worker would then carry the whole launch).
+  uint32_t cov_lo = 1, cov_hi = 0;
   std::deque<uint64_t> pending; // launches waiting for SMs (AUTO/SOLO)
   std::deque<uint64_t> deferred;  // granted SMs but waiting for a control block (stream order)
   std::deque<uint64_t> issued;  // issued, not complete (stream order)

@@ -152,9 +152,23 @@ __device__ void check_shrink_done(const P& p, uint64_t c, uint32_t lane) {
   }
 }
 
-// Retire unless this is the last live worker (liveness rule): CAS on live.
-// With `give_back`, the same atomic step also counts one returned task (Q28).
+// Retire unless this is the last live worker (liveness rule).  Without a
+// give-back this is one fetch-and-add: live -= 1, and if that took the count
+// from 1 to 0 the worker was the last and puts its unit back (the transient 0
+// is visible only to standby CTAs, which may then join -- a transition the
+// protocol allows anyway).  A CAS loop here serialises a mass retirement: with
+// N workers leaving at once only one CAS per L2 round trip succeeds, and a
+// shrink of half the SMs of a 4-CTA/SM tenant took ~90 us (tools/storm_tenant.py).
+// With `give_back`, retiring and returning the task must be one atomic step
+// (Q28: a returned task must never be taken while its giver could stay), so
+// that path keeps the CAS.
 __device__ __forceinline__ bool try_retire(TaskCtl* tc, bool give_back = false) {
+  if (!give_back) {
+    const unsigned long long old = atomicAdd(&tc->live_pending, ~0ull);   // live -= 1
+    if (uint32_t(old) > 1u) return true;
+    atomicAdd(&tc->live_pending, 1ull);                                    // the last one stays
+    return false;
+  }
   unsigned long long v = ld_relaxed_u64(&tc->live_pending);
   const unsigned long long delta = give_back ? (1ull << 32) - 1ull : ~0ull;   // live -1 (, returned +1)
   while (uint32_t(v) > 1u) {

@@ -67,6 +67,52 @@ def test_protocol_exhaustive(cfg):
     assert n > 10
 
 
+@pytest.mark.parametrize("cfg", [
+    P.Config(blocks=4, iters=2, ranks=2, occ=1, lo=0, hi=1, resizes=[(0, 0), (0, 1)], faa_retire=False),
+    P.Config(blocks=3, iters=1, ranks=2, occ=1, lo=1, hi=1, resizes=[(0, 1)], faa_retire=False),
+    P.Config(blocks=3, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1), (0, 1)], abort=True, faa_retire=False),
+])
+def test_protocol_exhaustive_single_step_retire(cfg):
+    """The same invariants with "retire unless last" as one atomic step."""
+    assert P.explore(cfg) > 10
+
+
+def test_faa_retire_needs_the_undo():
+    """Q22 with the runtime's fetch-and-add retire: a last live worker that
+    took live to 0 and left anyway (no undo) strands the remaining tasks: the
+    mutation must fail on some interleaving."""
+    class NoUndo(P.Model):
+        def apply(self, act):
+            if act[0] == "step":
+                c = self.ctas[act[1]]
+                if c[0] == P.RETIRING:
+                    self.exit(c, False)
+                    return
+            super().apply(act)
+
+    cfg = P.Config(blocks=4, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1)], grid=1)
+    with pytest.raises(P.ProtocolViolation):
+        stack, seen = [NoUndo(cfg)], set()
+        import copy
+        while stack:
+            x = stack.pop()
+            k = x.key()
+            if k in seen:
+                continue
+            seen.add(k)
+            if x.done():
+                x.check_final()
+                continue
+            acts = x.actions()
+            if not acts:
+                raise P.ProtocolViolation("deadlock")
+            for a in acts:
+                y = copy.deepcopy(x)
+                y.apply(a)
+                y.check_step()
+                stack.append(y)
+
+
 def test_protocol_random_seeds():
     cfgs = [
         P.Config(blocks=1000, iters=3, ranks=8, occ=2, lo=0, hi=7, resizes=[(0, 3), (5, 7), (0, 7)]),
