@@ -273,3 +273,158 @@ def expected_counters(total_blocks, iters):
         "task_starts": list(range(0, total_blocks, iters)),
         "next_clamped": tasks * iters,
     }
+
+
+# ================================================================ the paper's own workload (Tab II)
+# NEXT-2: the five applications of Tab II ("from the
+# NVIDIA CUDA 8.0 samples and the Rodinia benchmark suite") as tenants.
+# Black-Scholes (BS) is ``blackscholes`` above with one scenario (P = 1, the
+# SDK kernel).  The other four follow.  Readings (Q33-Q36): TR is the
+# SDK's tiled transpose, MM the SDK's shared-memory tiled matrixMul, RG the
+# SDK's quasirandomGenerator kernel (the Niederreiter-style XOR generator, the
+# inverse-CND pass not included), GS Rodinia's Gaussian elimination as its two
+# kernels Fan1 (multipliers of column t) and Fan2 (rank-1 update of the
+# trailing rows), one pair of launches per elimination step t.
+
+TR_TILE = 32          # 32x32 input tile per block
+MM_TILE = 32          # 32x32 C tile per block
+QRNG_E = 1024         # points per block (one dimension)
+QRNG_BITS = 31        # QRNG_RESOLUTION of the SDK sample
+GS_FAN1_E = 256       # rows per Fan1 block
+GS_FAN2_R, GS_FAN2_C = 16, 128   # rows x columns of the trailing submatrix per Fan2 block
+
+
+# ---------------------------------------------------------------- TR: transpose
+def transpose_grid(h, w):
+    return (cdiv(w, TR_TILE), cdiv(h, TR_TILE), 1)
+
+
+def transpose(inp, blocks=None):
+    """out[j][i] = in[i][j]; ``inp`` is h x w row-major, the output w x h.
+    Block (x, y) moves the input tile rows 32y.., columns 32x.."""
+    h, w = inp.shape
+    out = np.zeros((w, h), dtype=inp.dtype)
+
+    def block(x, y, z):
+        r0, r1 = y * TR_TILE, min((y + 1) * TR_TILE, h)
+        c0, c1 = x * TR_TILE, min((x + 1) * TR_TILE, w)
+        for i in range(r0, r1):
+            out[c0:c1, i] = inp[i, c0:c1]
+
+    run_grid(transpose_grid(h, w), block, blocks)
+    return out
+
+
+# ---------------------------------------------------------------- MM: tiled SGEMM
+def sgemm_tiled_grid(m, n):
+    return (cdiv(n, MM_TILE), cdiv(m, MM_TILE), 1)
+
+
+def sgemm_tiled(A, B, blocks=None):
+    """C = A @ B (A m x k, B k x n, row-major), the SDK matrixMul: block (x, y)
+    owns the 32x32 C tile rows 32y.., columns 32x..; every C element is the dot
+    product of its row of A and column of B (k ascending; summed here in double)."""
+    m, k = A.shape
+    k2, n = B.shape
+    assert k == k2
+    A64 = A.astype(np.float64)
+    B64 = B.astype(np.float64)
+    C = np.zeros((m, n), dtype=np.float64)
+
+    def block(x, y, z):
+        r0, r1 = y * MM_TILE, min((y + 1) * MM_TILE, m)
+        c0, c1 = x * MM_TILE, min((x + 1) * MM_TILE, n)
+        for r in range(r0, r1):
+            for c in range(c0, c1):
+                C[r, c] = float(np.dot(A64[r, :], B64[:, c]))
+
+    run_grid(sgemm_tiled_grid(m, n), block, blocks)
+    return C
+
+
+# ---------------------------------------------------------------- RG: quasirandom generator
+def qrng_grid(n, dims):
+    return (cdiv(n, QRNG_E), dims, 1)
+
+
+def qrng_point(table_row, k):
+    """q(k) = XOR of table_row[b] over the set bits b < 31 of k (the generator
+    matrix applied to the binary digits of k over GF(2))."""
+    r = 0
+    for b in range(QRNG_BITS):
+        if (k >> b) & 1:
+            r ^= int(table_row[b])
+    return r
+
+
+def qrng(table, n, seed, blocks=None):
+    """out[d][i] = float32(q_d(seed + i) + 1) * 2^-31 for i < n, d < dims: the
+    SDK kernel's ``(float)(result + 1) * INT_SCALE`` (INT_SCALE = 2^-31, the
+    float nearest 1/0x80000001).  ``table`` is dims x 31 uint32 (< 2^31).  The
+    integer -> float conversion rounds to nearest (fp32, as the kernel does);
+    the scaling by a power of two is exact.  Block (x, d) makes points
+    1024x .. of dimension d."""
+    dims = table.shape[0]
+    out = np.zeros((dims, n), dtype=np.float32)
+
+    def block(x, d, z):
+        for i in range(x * QRNG_E, min((x + 1) * QRNG_E, n)):
+            q = qrng_point(table[d], (seed + i) & 0xFFFFFFFF)
+            out[d, i] = np.float32(q + 1) * np.float32(2.0 ** -31)
+
+    run_grid(qrng_grid(n, dims), block, blocks)
+    return out
+
+
+# ---------------------------------------------------------------- GS: Gaussian elimination
+def gauss_fan1_grid(n, t):
+    return (max(cdiv(n - 1 - t, GS_FAN1_E), 1), 1, 1)
+
+
+def gauss_fan2_grid(n, t):
+    return (max(cdiv(n - t, GS_FAN2_C), 1), max(cdiv(n - 1 - t, GS_FAN2_R), 1), 1)
+
+
+def gauss_fan1(a, m, t, blocks=None):
+    """Rodinia Fan1 at step t: m[i][t] = a[i][t] / a[t][t] for rows i = t+1 .. n-1.
+    ``a`` and ``m`` are n x n float64 arrays, ``m`` updated in place."""
+    n = a.shape[0]
+
+    def block(x, y, z):
+        for i in range(t + 1 + x * GS_FAN1_E, min(t + 1 + (x + 1) * GS_FAN1_E, n)):
+            m[i, t] = a[i, t] / a[t, t]
+
+    run_grid(gauss_fan1_grid(n, t), block, blocks)
+
+
+def gauss_fan2(a, b, m, t, blocks=None):
+    """Rodinia Fan2 at step t: a[i][j] -= m[i][t] * a[t][j] for rows i = t+1 .. n-1
+    and columns j = t .. n-1 (column t included: it becomes ~0), and
+    b[i] -= m[i][t] * b[t].  In place on float64 arrays.  Block (x, y) owns rows
+    t+1+16y .., columns t+128x ..; the blocks with x = 0 update b."""
+    n = a.shape[0]
+
+    def block(x, y, z):
+        r0, r1 = t + 1 + y * GS_FAN2_R, min(t + 1 + (y + 1) * GS_FAN2_R, n)
+        c0, c1 = t + x * GS_FAN2_C, min(t + (x + 1) * GS_FAN2_C, n)
+        for i in range(r0, r1):
+            a[i, c0:c1] -= m[i, t] * a[t, c0:c1]
+            if x == 0:
+                b[i] -= m[i, t] * b[t]
+
+    run_grid(gauss_fan2_grid(n, t), block, blocks)
+
+
+def gaussian(a, b, steps=None):
+    """Forward elimination without pivoting (Rodinia ``ForwardSub``): for
+    t = 0 .. n-2, Fan1 then Fan2.  Returns (a, b, m) in float64: a upper
+    triangular below the diagonal up to rounding (column entries ~0), m the
+    unit-lower factor's multipliers below the diagonal (zero elsewhere)."""
+    n = a.shape[0]
+    a = a.astype(np.float64).copy()
+    b = b.astype(np.float64).copy()
+    m = np.zeros((n, n), dtype=np.float64)
+    for t in range(n - 1 if steps is None else steps):
+        gauss_fan1(a, m, t)
+        gauss_fan2(a, b, m, t)
+    return a, b, m

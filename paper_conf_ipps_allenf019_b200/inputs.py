@@ -140,3 +140,46 @@ def gemm_inputs(m, n, k, seed, mode="float"):
     A = _vec(g, m * k, mode, -2, 2).reshape(m, k)
     B = _vec(g, n * k, mode, -2, 2).reshape(n, k)
     return to_bf16_bits(A), to_bf16_bits(B)
+
+
+# ---------------------------------------------------------------- the paper's Tab II apps (NEXT-2)
+def transpose_inputs(h, w, seed, mode="float"):
+    """h x w fp32 matrix: U[-1,1) or integers in [-2^10, 2^10]."""
+    return _vec(rng(seed), h * w, mode, -1024, 1024).reshape(h, w)
+
+
+def qrng_table(dims, seed, bits=31):
+    """dims x bits uint32 generator table of a digital (0,1)-style sequence:
+    entry b of a dimension has its leading bit at position bits-1-b and random
+    bits below it (an upper unit-triangular generator matrix over GF(2)), so
+    every dimension is a permutation-preserving digital sequence.  Dimension 0
+    is the van der Corput sequence (no bits below the leading one)."""
+    g = rng(seed)
+    t = np.zeros((dims, bits), dtype=np.uint32)
+    for d in range(dims):
+        for b in range(bits):
+            lead = 1 << (bits - 1 - b)
+            low = 0 if d == 0 else int(g.integers(0, lead))
+            t[d, b] = lead | low
+    return t
+
+
+def gauss_inputs(n, seed=None, mode="rodinia"):
+    """Linear system a (n x n fp32) and right-hand side b (n fp32).
+
+    ``rodinia``: Rodinia gaussian's generated matrix (``-s n``):
+    a[i][j] = 10 exp(-0.01 |i - j|) (symmetric positive definite, so no pivoting
+    is needed), b = 1.  ``int``: a = L U with L unit lower triangular, entries
+    in {-1, 0, 1}, and U upper triangular with unit diagonal and entries in
+    [-2, 2], b integers in [-4, 4]: every multiplier and every intermediate
+    value of the elimination is a small integer, exact in fp32."""
+    if mode == "rodinia":
+        i = np.arange(n)
+        a = (10.0 * np.exp(-0.01 * np.abs(i[:, None] - i[None, :]))).astype(np.float32)
+        return a, np.ones(n, dtype=np.float32)
+    g = rng(seed)
+    L = np.tril(g.integers(-1, 2, size=(n, n)), -1) + np.eye(n, dtype=np.int64)
+    U = np.triu(g.integers(-2, 3, size=(n, n)), 1) + np.eye(n, dtype=np.int64)
+    a = (L @ U).astype(np.float32)
+    b = g.integers(-4, 5, size=n).astype(np.float32)
+    return a, b
