@@ -74,7 +74,16 @@ typedef enum {
   SLATE_KIND_BLACKSCHOLES = 5, /* mean call/put over P sigmas; 1024 options/block, T=256 */
   SLATE_KIND_STENCIL2D = 6,    /* 5-point Jacobi sweep; 32x8 points/block, T = 256      */
   SLATE_KIND_GEMM_BF16 = 7,    /* C(fp32) = A B^T, bf16 K-major; 128x128 tile/block     */
-  SLATE_KIND_MAX_ = 8
+  /* The paper's own applications (Tab II; NEXT-2).  Black-Scholes
+   * (BS) is SLATE_KIND_BLACKSCHOLES with one scenario. */
+  SLATE_KIND_TRANSPOSE = 8,    /* TR: out = in^T, fp32 h x w -> w x h; 32x32 tile/block, T = 256 */
+  SLATE_KIND_SGEMM_TILED = 9,  /* MM: C = A B, fp32 row-major, the SDK matrixMul; 32x32 C tile/block
+                                  through shared memory, T = 256 (args: slate_args_sgemm)          */
+  SLATE_KIND_QRNG = 10,        /* RG: quasirandom points; 1024 points of one dimension/block     */
+  SLATE_KIND_GAUSS_FAN1 = 11,  /* GS step t, Fan1: m[i][t] = a[i][t] / a[t][t]; 256 rows/block   */
+  SLATE_KIND_GAUSS_FAN2 = 12,  /* GS step t, Fan2: a[i][j] -= m[i][t] a[t][j] (j >= t),
+                                  b[i] -= m[i][t] b[t]; 16 rows x 128 columns/block              */
+  SLATE_KIND_MAX_ = 13
 } slate_kind;
 
 /* Per-kind argument blocks (passed by value in slate_launch_desc.args).
@@ -91,6 +100,16 @@ typedef struct {
 } slate_args_bs;
 typedef struct { uint64_t in, out; uint32_t h, w; } slate_args_stencil;
 typedef struct { uint64_t A, B, C; uint32_t m, n, k, pad_; } slate_args_gemm;       /* A m x k, B n x k bf16 */
+/* TR: in h x w fp32, out w x h fp32 (out[j][i] = in[i][j]); grid (ceil(w/32), ceil(h/32)) */
+typedef struct { uint64_t in, out; uint32_t h, w; } slate_args_transpose;
+/* RG (the CUDA SDK quasirandomGenerator kernel): out[d][i] = float(q_d(seed + i) + 1) * 2^-31,
+ * q_d(k) = XOR of table[d][b] over the set bits b < 31 of k; table dims x 31 uint32 (< 2^31),
+ * out dims x n fp32; grid (ceil(n/1024), dims) */
+typedef struct { uint64_t table, out; uint32_t n, dims, seed, pad_; } slate_args_qrng;
+/* GS (Rodinia gaussian, forward elimination without pivoting), step t < n-1 of an n x n
+ * system: a n x n, m n x n (multipliers, column t written by Fan1), b n; all fp32 row-major.
+ * Fan1 grid (ceil((n-1-t)/256)); Fan2 grid (ceil((n-t)/128), ceil((n-1-t)/16)). */
+typedef struct { uint64_t a, b, m; uint32_t n, t; } slate_args_gauss;
 
 /* ------------------------------------------------------------------ attach */
 /* Open a session ("the daemon creates a session for each application
@@ -277,6 +296,9 @@ typedef struct {
                               worker joining on a new rank; device clock mapped to the host
                               clock); -1 if not observed (e.g. the launch ended first) */
   uint8_t resize_kind[16]; /* 1 shrink, 2 grow, 0 none, for each resize_us entry */
+  uint64_t t_enter_ns;     /* %globaltimer when the first worker CTA started (device clock; 0 if standalone) */
+  uint64_t t_exit_ns;      /* %globaltimer when the last worker CTA that ran a task exited (0 unless the
+                              library is built with SLATE_DIAG_EXIT) */
 } slate_launch_info;
 
 /* Counters and timing of a launch (copied out).  Errors: ENOTFOUND. */

@@ -80,6 +80,11 @@ slate_status slate_kind_geometry(uint32_t kind, uint32_t* tile_m, uint32_t* tile
     case SLATE_KIND_SPMV_CSR: *tile_m = 1; *tile_n = 32; return SLATE_OK;
     case SLATE_KIND_BLACKSCHOLES: *tile_m = 1; *tile_n = 1024; return SLATE_OK;
     case SLATE_KIND_STENCIL2D: *tile_m = 8; *tile_n = 32; return SLATE_OK;
+    case SLATE_KIND_TRANSPOSE: *tile_m = 32; *tile_n = 32; return SLATE_OK;
+    case SLATE_KIND_SGEMM_TILED: *tile_m = 32; *tile_n = 32; return SLATE_OK;
+    case SLATE_KIND_QRNG: *tile_m = 1; *tile_n = 1024; return SLATE_OK;
+    case SLATE_KIND_GAUSS_FAN1: *tile_m = 256; *tile_n = 1; return SLATE_OK;
+    case SLATE_KIND_GAUSS_FAN2: *tile_m = 16; *tile_n = 128; return SLATE_OK;
     case SLATE_KIND_GEMM_BF16: {
       const slate::KindOps* o = slate::kind_ops(kind);
       *tile_m = o && o->tile_m ? o->tile_m : 128;

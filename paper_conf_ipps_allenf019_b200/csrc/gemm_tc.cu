@@ -63,7 +63,7 @@ struct Params {
   CUtensorMap tma_b;
   CUtensorMap tma_c;     // fp32 C, boxes of 32 x 32, SWIZZLE_128B (epilogue TMA store)
   slate_args_gemm args;
-  uint32_t gx, gy, B, iters, occ, bound_lo, bound_hi, n_ranks, standby_timeout_ns;
+  uint32_t gx, gy, B, iters, occ, bound_lo, bound_hi, n_ranks, standby_timeout_ns, base_epoch;
   const uint64_t* ctrl;
   TaskCtl* tc;
   HostMirror* mirror;
@@ -258,10 +258,8 @@ __device__ bool pair_prologue(const P& p, uint32_t r0, uint32_t r1, uint64_t& c_
       atomicAdd(&tc->live_rank[r1], 1u);
       atomicAdd(&tc->started, 1u);
       const uint32_t e = ctrl_epoch(c);
-      if (e > 0 && ld_relaxed_u32(&tc->join_epoch) < e && atomicMax(&tc->join_epoch, e) < e && p.mirror) {
-        p.mirror->join_ns = globaltimer();
-        __threadfence_system();
-        p.mirror->join_epoch = e;
+      if (e > p.base_epoch && ld_relaxed_u32(&tc->join_epoch) < e && atomicMax(&tc->join_epoch, e) < e && p.mirror) {
+        publish_mirror(&tc->join_word, &p.mirror->join, mirror_pack(e, globaltimer()));
       }
       c_out = c;
       return true;
@@ -703,6 +701,7 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.gx = w.gx; p.gy = w.gy; p.B = w.B; p.iters = w.iters; p.occ = w.occ;
   p.bound_lo = w.bound_lo; p.bound_hi = w.bound_hi; p.n_ranks = w.n_ranks;
   p.standby_timeout_ns = w.standby_timeout_ns;
+  p.base_epoch = w.base_epoch;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   return launch_pairs(reinterpret_cast<const void*>(&gemm_kernel<true>), p, dim3((grid + 1) & ~1u), st);
 }

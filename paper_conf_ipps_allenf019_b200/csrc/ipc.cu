@@ -32,6 +32,10 @@ int pointer_fields(uint32_t kind, const size_t** offs) {
   static const size_t stencil[] = {offsetof(slate_args_stencil, in), offsetof(slate_args_stencil, out)};
   static const size_t gemm[] = {offsetof(slate_args_gemm, A), offsetof(slate_args_gemm, B),
                                 offsetof(slate_args_gemm, C)};
+  static const size_t transpose[] = {offsetof(slate_args_transpose, in), offsetof(slate_args_transpose, out)};
+  static const size_t qrng[] = {offsetof(slate_args_qrng, table), offsetof(slate_args_qrng, out)};
+  static const size_t gauss[] = {offsetof(slate_args_gauss, a), offsetof(slate_args_gauss, b),
+                                 offsetof(slate_args_gauss, m)};
   switch (kind) {
     case SLATE_KIND_TRIAD: *offs = triad; return 3;
     case SLATE_KIND_COPY: *offs = copy; return 2;
@@ -40,6 +44,11 @@ int pointer_fields(uint32_t kind, const size_t** offs) {
     case SLATE_KIND_BLACKSCHOLES: *offs = bs; return 6;
     case SLATE_KIND_STENCIL2D: *offs = stencil; return 2;
     case SLATE_KIND_GEMM_BF16: *offs = gemm; return 3;
+    case SLATE_KIND_TRANSPOSE: *offs = transpose; return 2;
+    case SLATE_KIND_SGEMM_TILED: *offs = sgemm; return 3;
+    case SLATE_KIND_QRNG: *offs = qrng; return 2;
+    case SLATE_KIND_GAUSS_FAN1: *offs = gauss; return 3;
+    case SLATE_KIND_GAUSS_FAN2: *offs = gauss; return 3;
     default: *offs = nullptr; return 0;
   }
 }

@@ -25,6 +25,8 @@ cudaError_t launch_worker_t(const WorkerCommon& w, const void* args, uint32_t gr
   p.gx = w.gx; p.gy = w.gy; p.gz = w.gz; p.B = w.B; p.iters = w.iters; p.occ = w.occ;
   p.bound_lo = w.bound_lo; p.bound_hi = w.bound_hi; p.n_ranks = w.n_ranks;
   p.standby_timeout_ns = w.standby_timeout_ns;
+  p.base_epoch = w.base_epoch;
+  p.is_topup = w.is_topup;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
   return cudaLaunchKernel(reinterpret_cast<const void*>(&slate_worker<Tn>), dim3(grid), dim3(Tn::kThreads), kargs,
@@ -54,6 +56,7 @@ KindOps make_ops(uint32_t default_iters) {
   o.tasks_per_worker = Tn::kTasksPerWorker;
   o.launch_worker = &launch_worker_t<Tn>;
   o.launch_standalone = &launch_standalone_t<Tn>;
+  o.topup_anytime = true;
   return o;
 }
 
@@ -70,6 +73,11 @@ const KindOps* kind_ops(uint32_t kind) {
     table[SLATE_KIND_BLACKSCHOLES] = make_ops<BlackScholes>(0);
     table[SLATE_KIND_STENCIL2D] = make_ops<Stencil2D>(0);
     table[SLATE_KIND_GEMM_BF16] = gemm_tc_ops();
+    table[SLATE_KIND_TRANSPOSE] = make_ops<Transpose>(0);
+    table[SLATE_KIND_SGEMM_TILED] = make_ops<SgemmTiled>(0);
+    table[SLATE_KIND_QRNG] = make_ops<Qrng>(0);
+    table[SLATE_KIND_GAUSS_FAN1] = make_ops<GaussFan1>(0);
+    table[SLATE_KIND_GAUSS_FAN2] = make_ops<GaussFan2>(0);
     init = true;
   }
   if (kind == 0 || kind >= SLATE_KIND_MAX_) return nullptr;

@@ -21,43 +21,60 @@ __host__ __device__ __forceinline__ uint32_t ctrl_hi(uint64_t c) { return uint32
 // Per launch, in device memory.  Line 0 holds the task counter alone (the hot
 // atomic, slateIdx of Lst2); line 1 the completion counters; then per-rank
 // live counts used to detect the end of a shrink.
+// Each counter every worker CTA updates has a 128-B line of its own: same-line
+// atomics serialise in one L2 slice (tools/probe/launch_cost.cu: ~1 us per
+// launch of 1184 CTAs).
 struct alignas(128) TaskCtl {
   uint32_t next;                  // slateIdx: next original block to hand out
   uint32_t pad0[31];
   unsigned long long done;        // (tasks_done << 32) | blocks_done
-  unsigned long long live_pending;// (returned tasks << 32) | live worker CTAs: one word, so that
-                                  // abandoning a task and retiring is one atomic step (Q28)
-  uint32_t started;               // workers that joined
-  uint32_t pad_s;
   unsigned long long t_first;     // %globaltimer at the start of the task at block 0
   unsigned long long t_last;      // %globaltimer when blocks_done reached B
   uint32_t shrink_epoch;          // last epoch whose shrink was observed complete
   uint32_t join_epoch;            // last epoch in which a worker joined (grow)
-  uint32_t pad1[20];
+  unsigned long long t_enter;     // %globaltimer at the first worker CTA's entry (launch overhead split)
+  unsigned long long t_exit;      // %globaltimer at the last working CTA's exit
+  unsigned long long shrink_word; // max mirror_pack(epoch, ns) of completed shrinks (the mirror's source)
+  unsigned long long join_word;   // max mirror_pack(epoch, ns) of grow joins
+  uint32_t pad1[16];
+  unsigned long long live_pending;// (returned tasks << 32) | live worker CTAs: one word, so that
+                                  // abandoning a task and retiring is one atomic step (Q28)
+  uint32_t pad_l[30];
+  uint32_t started;               // workers that joined
+  uint32_t main_live;             // joined CTAs of the launch's own grid (not top-ups) not yet exited
+  uint32_t pad_s[30];
   uint32_t live_rank[kMaxRanks];  // live workers per SM rank
   uint32_t ret_head, ret_tail;    // ring of abandoned task starts (+1; 0 = slot empty)
   uint32_t pad2[30];
   uint32_t ret[kMaxRanks];
 };
-static_assert(offsetof(TaskCtl, live_rank) == 256, "TaskCtl header must stay 256 B (the query snapshot)");
-constexpr size_t kTaskCtlHeader = 256;   // the part snapshotted to the host at the end
+static_assert(offsetof(TaskCtl, live_pending) == 256 && offsetof(TaskCtl, started) == 384 &&
+              offsetof(TaskCtl, live_rank) == 512, "TaskCtl header lines: next | done.. | live_pending | started");
+constexpr size_t kTaskCtlHeader = 512;   // the part snapshotted to the host at the end
 
 // Per launch, in mapped pinned host memory: what the host poller watches.
+// Every event is ONE 8-byte store with no fence: a __threadfence_system()
+// before a flag store cost ~4 us per launch (tools/probe/launch_cost.cu),
+// paid by the CTA whose exit ends the kernel.  An epoch and its device time
+// share one word (mirror_pack); the host restores the time's upper bits.
+constexpr int kMirrorNsBits = 44;   // 2^44 ns = 17.6 s of device clock
+__host__ __device__ __forceinline__ unsigned long long mirror_pack(uint32_t epoch, unsigned long long ns) {
+  return (static_cast<unsigned long long>(epoch) << kMirrorNsBits) | (ns & ((1ull << kMirrorNsBits) - 1));
+}
+__host__ __device__ __forceinline__ uint32_t mirror_epoch(unsigned long long w) { return uint32_t(w >> kMirrorNsBits); }
 struct HostMirror {
-  volatile uint32_t complete;     // 1 once every block has run
-  volatile uint32_t shrink_epoch; // epoch whose shrink completed (no live worker outside)
-  volatile uint32_t join_epoch;   // epoch in which a worker first joined
-  volatile uint32_t pad;
-  volatile unsigned long long t_last;
-  volatile unsigned long long shrink_ns;
-  volatile unsigned long long join_ns;
-  uint64_t pad2[3];
+  volatile unsigned long long done;   // %globaltimer when every block had run (0: not yet)
+  volatile unsigned long long shrink; // mirror_pack(epoch, ns): the last epoch whose shrink completed
+  volatile unsigned long long join;   // mirror_pack(epoch, ns): the last epoch in which a worker joined
+  uint64_t pad[5];
 };
 
 // Everything a worker launch needs besides the tenant's own arguments.
 struct WorkerCommon {
   uint32_t gx, gy, gz, B, iters, occ;
   uint32_t bound_lo, bound_hi, n_ranks, standby_timeout_ns;
+  uint32_t base_epoch;   // the queue's epoch at issue (0 for top-ups: every join of theirs is a grow)
+  uint32_t is_topup;     // 1: a top-up grid sharing a running launch's counter
   const uint64_t* ctrl;
   TaskCtl* tc;
   HostMirror* mirror;
@@ -78,6 +95,8 @@ struct KindOps {
   uint32_t tasks_per_worker = 8; // the automatic task size aims at >= this many tasks per worker
   uint32_t tile_m = 0;           // GEMM: output rows per original block
   uint32_t tile_n = 0;           // GEMM: output columns per original block
+  bool topup_anytime = false;    // the worker's last main CTA waits for every block (leave_main), so a
+                                 // running launch may get a top-up while later launches are queued
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;
   cudaError_t (*launch_standalone)(const void* args, dim3 grid, cudaStream_t) = nullptr;
 };

@@ -335,6 +335,8 @@ int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::stri
     if (err) *err = "worker does not fit on an SM";
     return SLATE_ECUDA;
   }
+  static const int occ_cap = int(env_double("SLATE_OCC_CAP", 0));   // experiments: fewer workers per SM
+  if (occ_cap > 0 && occ > occ_cap) occ = occ_cap;
   k->occ = occ;
   *out = k->id;
   kernels_[k->id] = std::move(k);
@@ -399,6 +401,39 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
       g[1] = a->m / tm;
       break;
     }
+    case SLATE_KIND_TRANSPOSE: {
+      auto a = static_cast<const slate_args_transpose*>(d->args);
+      g[0] = cdiv(a->w, 32);
+      g[1] = cdiv(a->h, 32);
+      break;
+    }
+    case SLATE_KIND_SGEMM_TILED: {
+      auto a = static_cast<const slate_args_sgemm*>(d->args);
+      g[0] = cdiv(a->n, 32);
+      g[1] = cdiv(a->m, 32);
+      if (a->k == 0) return fail("k == 0");
+      break;
+    }
+    case SLATE_KIND_QRNG: {
+      auto a = static_cast<const slate_args_qrng*>(d->args);
+      if (!al(a->out)) return fail("qrng output must be 16-byte aligned");
+      if (a->dims == 0 || a->dims > 65535) return fail("qrng dims must be in [1, 65535]");
+      g[0] = cdiv(a->n, 1024);
+      g[1] = a->dims;
+      break;
+    }
+    case SLATE_KIND_GAUSS_FAN1:
+    case SLATE_KIND_GAUSS_FAN2: {
+      auto a = static_cast<const slate_args_gauss*>(d->args);
+      if (a->n < 2 || a->t + 1 >= a->n) return fail("gauss step needs t < n - 1");
+      if (k.desc.kind == SLATE_KIND_GAUSS_FAN1) {
+        g[0] = cdiv(a->n - 1 - a->t, 256);
+      } else {
+        g[0] = cdiv(a->n - a->t, 128);
+        g[1] = cdiv(a->n - 1 - a->t, 16);
+      }
+      break;
+    }
     default:
       return fail("unknown kind");
   }
@@ -457,6 +492,37 @@ void Server::work(const KernelEntry& k, const slate_launch_desc* d, double* byte
       *tc = 2.0 * a->m * double(a->n) * a->k;
       break;
     }
+    case SLATE_KIND_TRANSPOSE: {
+      auto a = static_cast<const slate_args_transpose*>(d->args);
+      *bytes = 8.0 * a->h * double(a->w);
+      break;
+    }
+    case SLATE_KIND_SGEMM_TILED: {
+      auto a = static_cast<const slate_args_sgemm*>(d->args);
+      *bytes = 4.0 * (double(a->m) * a->k + double(a->k) * a->n + double(a->m) * a->n);
+      *fp32 = 2.0 * a->m * double(a->n) * a->k;
+      break;
+    }
+    case SLATE_KIND_QRNG: {
+      auto a = static_cast<const slate_args_qrng*>(d->args);
+      *bytes = 4.0 * double(a->n) * a->dims + 124.0 * a->dims;
+      *fp32 = double(a->n) * a->dims;           // the 2^-31 scaling (the XOR walk is integer work)
+      break;
+    }
+    case SLATE_KIND_GAUSS_FAN1: {
+      auto a = static_cast<const slate_args_gauss*>(d->args);
+      const double r = a->n - 1.0 - a->t;
+      *bytes = 8.0 * r + 4.0;
+      *fp32 = r;
+      break;
+    }
+    case SLATE_KIND_GAUSS_FAN2: {
+      auto a = static_cast<const slate_args_gauss*>(d->args);
+      const double r = a->n - 1.0 - a->t, c = double(a->n) - a->t;
+      *bytes = 8.0 * r * c + 4.0 * c + 4.0 * r + 8.0 * r + 4.0;   // trailing block r/w, pivot row, m column, b
+      *fp32 = 2.0 * r * c + 2.0 * r;
+      break;
+    }
   }
 }
 
@@ -474,6 +540,15 @@ void Server::free_slot(int slot) {
   if (!slot_zeroed_[slot]) cudaEventCreateWithFlags(&slot_zeroed_[slot], cudaEventDisableTiming);
   cudaEventRecord(slot_zeroed_[slot], copy_stream_);
   free_slots_.push_back(slot);
+}
+
+// one wave of workers (Q12) -- but no more CTAs than there are tasks,
+// and at least one per SM (so any SM range gets workers): every worker CTA
+// costs its launch a prologue and a fetch (tools/probe/launch_cost.cu)
+uint32_t Server::worker_grid(int occ, uint32_t B, uint32_t iters) const {
+  const uint64_t wave = uint64_t(occ) * uint64_t(n_sms_);
+  const uint64_t tasks = (uint64_t(B) + iters - 1) / iters;
+  return uint32_t(std::min<uint64_t>(wave, std::max<uint64_t>(uint64_t(n_sms_), tasks)));
 }
 
 // reading Q11: the paper's default task of 10 blocks, reduced so every
@@ -543,12 +618,19 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
   for (cudaEvent_t e : Q.topup_ends)   // stream semantics: the predecessor's top-up workers finish first
     CK(cudaStreamWaitEvent(Q.stream, e, 0));
   Q.topup_ends.clear();
-  CK(cudaEventCreate(&L.ev_start));
+  // A launch queued right behind another of its queue starts where that one
+  // ends (stream order), so it records no start event of its own: an event
+  // between two kernels costs ~3 us of stream time (tools/probe/pdl_cost.cu).
+  if (!Q.issued.empty() && !launches_[Q.issued.back()]->ev_end.empty()) {
+    L.start_after = launches_[Q.issued.back()]->ev_end.front();
+  } else {
+    CK(cudaEventCreate(&L.ev_start));
+  }
   cudaEvent_t ev_end;
   CK(cudaEventCreate(&ev_end));
   const auto& g = L.desc.grid;
   if (L.desc.mode == SLATE_MODE_STANDALONE) {
-    CK(cudaEventRecord(L.ev_start, Q.stream));
+    if (L.ev_start) CK(cudaEventRecord(L.ev_start, Q.stream));
     CK(ops->launch_standalone(L.args.data(), dim3(g[0], g[1], g[2]), Q.stream));
     CK(cudaEventRecord(ev_end, Q.stream));
     L.ev_end.push_back(ev_end);
@@ -565,15 +647,16 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     // wait (a cross-stream dependency) if that copy has not finished yet
     if (slot_zeroed_[slot] && cudaEventQuery(slot_zeroed_[slot]) != cudaSuccess)
       CK(cudaStreamWaitEvent(Q.stream, slot_zeroed_[slot], 0));
-    CK(cudaEventRecord(L.ev_start, Q.stream));
+    if (L.ev_start) CK(cudaEventRecord(L.ev_start, Q.stream));
     WorkerCommon w{};
     w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = L.B; w.iters = L.iters; w.occ = uint32_t(L.k->occ);
     w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
     w.standby_timeout_ns = standby_timeout_ns_;
+    w.base_epoch = Q.epoch;
     w.ctrl = Q.d_ctrl; w.tc = d_tc_ + slot; w.mirror = d_mirror_ + slot;
     w.cov = reinterpret_cast<uint32_t*>(L.desc.coverage);
     w.rank_of = d_rank_of_;
-    CK(ops->launch_worker(w, L.args.data(), uint32_t(L.k->occ) * uint32_t(n_sms_), Q.stream));
+    CK(ops->launch_worker(w, L.args.data(), worker_grid(L.k->occ, L.B, L.iters), Q.stream));
     CK(cudaEventRecord(ev_end, Q.stream));
     L.ev_end.push_back(ev_end);
     cudaEvent_t ev_snap;
@@ -603,6 +686,17 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   // it in stream order); launches before it that finished all their blocks but
   // are not yet retired by the poller do not count
   static const bool dbg = std::getenv("SLATE_DEBUG") != nullptr;
+  if (!Q.issued.empty()) {
+    // kinds whose last main CTA waits for all blocks (leave_main): top up the
+    // RUNNING launch -- the first issued one that has not finished its blocks --
+    // whatever is queued behind it (a grow then lands within a task, not a launch)
+    for (uint64_t lid : Q.issued) {
+      Launch& E = *launches_[lid];
+      if (E.slot < 0 || E.desc.mode == SLATE_MODE_STANDALONE || !E.k->ops->topup_anytime) break;
+      if (h_mirror_[E.slot].done) continue;
+      return topup(Q, E, err);
+    }
+  }
   if (Q.issued.empty() || !Q.pending.empty() || !Q.deferred.empty()) {
     if (dbg) fprintf(stderr, "[slate] grow: no top-up (issued %zu pending %zu deferred %zu)\n", Q.issued.size(),
                      Q.pending.size(), Q.deferred.size());
@@ -610,17 +704,23 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   }
   for (size_t i = 0; i + 1 < Q.issued.size(); ++i) {
     const Launch& E = *launches_[Q.issued[i]];
-    if (E.slot < 0 || !h_mirror_[E.slot].complete) {
+    if (E.slot < 0 || !h_mirror_[E.slot].done) {
       if (dbg) fprintf(stderr, "[slate] grow: no top-up (an earlier launch is still running)\n");
       return SLATE_OK;
     }
   }
   Launch& R = *launches_[Q.issued.back()];
   if (R.state != 1 || R.slot < 0 || R.desc.mode == SLATE_MODE_STANDALONE) return SLATE_OK;
-  if (h_mirror_[R.slot].complete) {
+  if (h_mirror_[R.slot].done) {
     if (dbg) fprintf(stderr, "[slate] grow: no top-up (the launch finished its blocks)\n");
     return SLATE_OK;
   }
+  return topup(Q, R, err);
+}
+
+// a top-up grid for launch R on the queue's current range, sharing R's counter
+int Server::topup(Queue& Q, Launch& R, std::string* err) {
+  static const bool dbg = std::getenv("SLATE_DEBUG") != nullptr;
   if (dbg) fprintf(stderr, "[slate] grow: top-up for launch %llu on [%u, %u]\n", (unsigned long long)R.id, Q.lo, Q.hi);
   const auto& g = R.desc.grid;
   cudaStream_t aux = Q.aux[Q.aux_next++ % Queue::kAux];
@@ -629,11 +729,12 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   CK(cudaEventRecord(ev_ctrl, ctrl_stream_));
   CK(cudaStreamWaitEvent(aux, ev_ctrl, 0));
   cudaEventDestroy(ev_ctrl);
-  CK(cudaStreamWaitEvent(aux, R.ev_start, 0));
+  CK(cudaStreamWaitEvent(aux, R.ev_start ? R.ev_start : R.start_after, 0));
   WorkerCommon w{};
   w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = R.B; w.iters = R.iters; w.occ = uint32_t(R.k->occ);
   w.bound_lo = Q.lo; w.bound_hi = Q.hi; w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
+  w.is_topup = 1;
   w.ctrl = Q.d_ctrl; w.tc = d_tc_ + R.slot; w.mirror = d_mirror_ + R.slot;
   w.cov = reinterpret_cast<uint32_t*>(R.desc.coverage);
   w.rank_of = d_rank_of_;
@@ -778,6 +879,12 @@ std::string Server::profile_key(const KernelEntry& k, const slate_launch_desc* d
     case SLATE_KIND_BLACKSCHOLES: { auto x = static_cast<const slate_args_bs*>(a); s << x->n << 'p' << x->n_scen; break; }
     case SLATE_KIND_STENCIL2D: { auto x = static_cast<const slate_args_stencil*>(a); s << x->h << 'x' << x->w; break; }
     case SLATE_KIND_GEMM_BF16: { auto x = static_cast<const slate_args_gemm*>(a); s << x->m << 'x' << x->n << 'x' << x->k; break; }
+    case SLATE_KIND_TRANSPOSE: { auto x = static_cast<const slate_args_transpose*>(a); s << x->h << 'x' << x->w; break; }
+    case SLATE_KIND_SGEMM_TILED: { auto x = static_cast<const slate_args_sgemm*>(a); s << x->m << 'x' << x->n << 'x' << x->k; break; }
+    case SLATE_KIND_QRNG: { auto x = static_cast<const slate_args_qrng*>(a); s << x->n << 'd' << x->dims; break; }
+    // one profile per system size: the steps of one elimination share it
+    case SLATE_KIND_GAUSS_FAN1:
+    case SLATE_KIND_GAUSS_FAN2: s << static_cast<const slate_args_gauss*>(a)->n; break;
   }
   return s.str();
 }
@@ -937,9 +1044,11 @@ void Server::schedule() {
       const Launch& HB = *launches_[queues_[qids[idx]]->pending.front()];
       double g = 0;
       s = pair_split(*LA, A, HB, *queues_[qids[idx]], catA, int(cats[idx]), &g);
-    } else if (policy_ == SLATE_POLICY_HYBRID && cats[0] != 99u) {
+    } else if (policy_ == SLATE_POLICY_HYBRID && cats[0] != 99u && (catA >= 3) != (cats[0] >= 3)) {
       // reading Q31: Tab I keeps the head of the queue waiting, but the measured
-      // solo curves and the queued work predict a co-run gain of >= min_gain_
+      // solo curves and the queued work predict a co-run gain of >= min_gain_.
+      // Only for a memory-intensive tenant (M_M, H_M) beside a compute one
+      // (Q37): solo curves do not see two memory tenants sharing HBM
       const Launch& HB = *launches_[queues_[qids[0]]->pending.front()];
       double g = 0;
       const uint32_t s0 = pair_split(*LA, A, HB, *queues_[qids[0]], catA, int(cats[0]), &g);
@@ -1052,6 +1161,20 @@ void Server::track_resize(Launch& R, uint32_t epoch, int kind, double t0) {
   R.resize_kind.push_back(uint8_t(kind));
 }
 
+// the full device time of a mirror word's low kMirrorNsBits bits: the value
+// nearest the device clock's reading at host time t (us)
+unsigned long long Server::unwrap_mirror_ns(unsigned long long w, double t) const {
+  const unsigned long long mask = (1ull << kMirrorNsBits) - 1, low = w & mask;
+  double dev_us = 0;
+  if (!clk_base_ns_ || !host_to_dev_us(t, &dev_us)) return low;
+  const long long ref = (long long)clk_base_ns_ + (long long)(dev_us * 1e3);
+  long long full = (long long)((ref & ~(long long)mask) | (long long)low);
+  const long long half = 1ll << (kMirrorNsBits - 1);
+  if (full > ref + half) full -= 1ll << kMirrorNsBits;
+  else if (full < ref - half) full += 1ll << kMirrorNsBits;
+  return (unsigned long long)full;
+}
+
 // completion stamp (device ns) -> latency from the host's resize call (Q30)
 void Server::record_resize(const Queue::PendingResize& pr, unsigned long long done_ns, double t) {
   auto li = launches_.find(pr.lid);
@@ -1080,15 +1203,16 @@ void Server::resolve_resizes(Queue& Q, double t, const Launch* ended) {
       const Launch& L = *launches_[lid];
       if (L.slot < 0) continue;
       const HostMirror& m = h_mirror_[L.slot];
-      if (it->kind == 1 ? m.shrink_epoch >= it->epoch : m.join_epoch >= it->epoch) {
-        done_ns = it->kind == 1 ? m.shrink_ns : m.join_ns;
+      const unsigned long long w = it->kind == 1 ? m.shrink : m.join;
+      if (w && mirror_epoch(w) >= it->epoch) {
+        done_ns = unwrap_mirror_ns(w, t);
         done = true;
         break;
       }
       if (it->kind == 1) break;   // only the oldest running launch can hold out-of-range workers
     }
     if (!done && ended && it->kind == 1 && ended->slot >= 0) {
-      done_ns = h_mirror_[ended->slot].t_last;
+      done_ns = h_mirror_[ended->slot].done;
       done = true;
     }
     if (done) {
@@ -1241,10 +1365,12 @@ int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
     out->t_last_ns = tc.t_last;
     out->shrink_epoch = tc.shrink_epoch;
     out->join_epoch = tc.join_epoch;
+    out->t_enter_ns = tc.t_enter;
+    out->t_exit_ns = tc.t_exit;
   }
   if (L.state == 2) {
     float ms = 0;
-    if (cudaEventElapsedTime(&ms, epoch_ev_, L.ev_start) == cudaSuccess) out->start_ms = ms;
+    if (cudaEventElapsedTime(&ms, epoch_ev_, L.ev_start ? L.ev_start : L.start_after) == cudaSuccess) out->start_ms = ms;
     double end = 0;
     for (cudaEvent_t e : L.ev_end)
       if (cudaEventElapsedTime(&ms, epoch_ev_, e) == cudaSuccess) end = std::max(end, double(ms));
@@ -1296,7 +1422,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   for (int r = 0; r < reps + 1; ++r) {
     CK(cudaMemcpyAsync(d_tc_ + slot, h_zero_, sizeof(TaskCtl), cudaMemcpyHostToDevice, st));
     CK(cudaEventRecord(e0, st));
-    CK(k.ops->launch_worker(w, d->args, uint32_t(k.occ) * uint32_t(n_sms_), st));
+    CK(k.ops->launch_worker(w, d->args, worker_grid(k.occ, B, w.iters), st));
     CK(cudaEventRecord(e1, st));
     CK(cudaEventSynchronize(e1));
     float t;

@@ -36,7 +36,8 @@ struct Launch {
   uint32_t B = 0, iters = 1;
   int state = 0;                // 0 queued, 1 issued, 2 complete
   int slot = -1;                // TaskCtl / mirror slot
-  cudaEvent_t ev_start = nullptr;
+  cudaEvent_t ev_start = nullptr;     // recorded before the kernel, or null when chained:
+  cudaEvent_t start_after = nullptr;  // the predecessor's end (same stream): this launch starts there
   std::vector<cudaEvent_t> ev_end;    // kernel ends (main + top-ups), for timing
   std::vector<cudaEvent_t> ev_done;   // all must complete (main + top-ups, after snapshots)
   int error = 0;                      // cudaError_t seen on completion
@@ -112,6 +113,7 @@ class Server {
   void fail_launch(Launch& L, int code);
   int write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool immediate, std::string* err);
   int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
+  int topup(Queue& Q, Launch& R, std::string* err);
   void schedule();
   void release(Queue& Q);
   bool curve_of(const Launch& L, std::vector<uint32_t>* sms, std::vector<double>* ms) const;
@@ -142,11 +144,13 @@ class Server {
   std::thread clock_;
   bool launch_done_events(Launch& L);
   void track_resize(Launch& R, uint32_t epoch, int kind, double t0);
+  unsigned long long unwrap_mirror_ns(unsigned long long w, double t) const;
   void resolve_resizes(Queue& Q, double t_host, const Launch* ended);
   void record_resize(const Queue::PendingResize& pr, unsigned long long done_ns, double t_host);
   int alloc_slot();
   void free_slot(int slot);
   uint32_t auto_iters(uint32_t B, int occ, uint32_t cap, uint32_t per_worker) const;
+  uint32_t worker_grid(int occ, uint32_t B, uint32_t iters) const;
   bool validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const;
   void work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const;
 

@@ -40,6 +40,26 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const unsigned long long* p) 
   asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+// a store to mapped host memory, visible to the host without a fence (one 8-byte word)
+__device__ __forceinline__ void st_sys_u64(volatile unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// Publish a packed (epoch, ns) event to the host mirror so that the mirror only
+// ever moves forward in epoch: the device word takes the max, and a writer
+// whose store may have overtaken a newer one re-reads and re-stores until the
+// mirror holds the device word's value (two CTAs completing shrinks of
+// consecutive epochs may otherwise store in the reverse order).
+__device__ __forceinline__ void publish_mirror(unsigned long long* word, volatile unsigned long long* host,
+                                               unsigned long long v) {
+  unsigned long long cur = atomicMax(word, v);
+  cur = cur > v ? cur : v;
+  for (int i = 0; i < 4; ++i) {
+    st_sys_u64(host, cur);
+    const unsigned long long now = ld_relaxed_u64(word);
+    if (now == cur) break;
+    cur = now;
+  }
+}
 __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -56,6 +76,8 @@ struct WorkerParams {
   uint32_t bound_lo, bound_hi;    // launch bound (top-up launches), else [0, N-1]
   uint32_t n_ranks;
   uint32_t standby_timeout_ns;
+  uint32_t base_epoch;            // resize-word epoch when the launch was issued: a join under a later epoch is a grow
+  uint32_t is_topup;              // 1: a top-up grid (grow) sharing a running launch's TaskCtl
   const uint64_t* ctrl;           // the queue's resize word
   TaskCtl* tc;
   HostMirror* mirror;             // device alias of the pinned mirror (may be null)
@@ -103,8 +125,10 @@ __device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
   uint64_t t0 = 0;
   uint32_t backoff = 256;
   for (;;) {
-    const uint64_t c = ld_acquire_u64(p.ctrl);
+    // the counter load first: a relaxed load issued after the acquire would wait
+    // for it; this way both round trips (and the caller's rank lookup) overlap
     const uint32_t nxt = ld_relaxed_u32(&tc->next);
+    const uint64_t c = ld_acquire_u64(p.ctrl);
     if (nxt >= p.B) return false;                                       // exit (2)
     bool join = in_range(p, rank, c);
     if (!join) {
@@ -118,11 +142,10 @@ __device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
       atomicAdd(&tc->live_pending, 1ull);    // results unused: RED, no round trip
       atomicAdd(&tc->live_rank[rank], 1u);
       atomicAdd(&tc->started, 1u);
+      if (!p.is_topup) atomicAdd(&tc->main_live, 1u);
       const uint32_t e = ctrl_epoch(c);
-      if (e > 0 && ld_relaxed_u32(&tc->join_epoch) < e && atomicMax(&tc->join_epoch, e) < e && p.mirror) {
-        p.mirror->join_ns = globaltimer();   // grow observed (a worker joined under epoch e)
-        __threadfence_system();
-        p.mirror->join_epoch = e;
+      if (e > p.base_epoch && ld_relaxed_u32(&tc->join_epoch) < e && atomicMax(&tc->join_epoch, e) < e && p.mirror) {
+        publish_mirror(&tc->join_word, &p.mirror->join, mirror_pack(e, globaltimer()));   // grow observed under epoch e
       }
       c_out = c;
       return true;
@@ -146,9 +169,7 @@ __device__ void check_shrink_done(const P& p, uint64_t c, uint32_t lane) {
   busy = __any_sync(0xffffffffu, busy);
   const uint32_t e = ctrl_epoch(c);
   if (!busy && lane == 0 && atomicMax(&tc->shrink_epoch, e) < e && p.mirror) {
-    p.mirror->shrink_ns = globaltimer();
-    __threadfence_system();
-    p.mirror->shrink_epoch = e;
+    publish_mirror(&tc->shrink_word, &p.mirror->shrink, mirror_pack(e, globaltimer()));
   }
 }
 
@@ -224,6 +245,7 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
                                              uint32_t n_done, bool& retired, bool& epoch_changed) {
   TaskCtl* tc = p.tc;
   epoch_changed = ctrl_epoch(c2) != ctrl_epoch(c);
+  if (epoch_changed) asm volatile("fence.acq_rel.gpu;" ::: "memory");   // completes the acquire of c2
   c = c2;
   retired = false;
   unsigned long long old = 0;
@@ -244,13 +266,25 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
   if (n_done && uint32_t(old) + n_done == p.B) {                        // last block of the launch
     const uint64_t t = globaltimer();
     tc->t_last = t;
-    if (p.mirror) {
-      p.mirror->t_last = t;
-      __threadfence_system();
-      p.mirror->complete = 1;
-    }
+    if (p.mirror) st_sys_u64(&p.mirror->done, t);
   }
   return g;
+}
+
+// A CTA of the launch's own grid leaves.  The last one to leave waits until
+// every block of the launch is done: top-up CTAs (another stream, grow) may
+// still hold some, and the queue's next launch starts when this kernel
+// completes (stream order).  Without top-ups the blocks are all counted by
+// then and it does not wait.
+template <class P>
+__device__ __forceinline__ void leave_main(const P& p) {
+  if (p.is_topup) return;
+  if (atomicSub(&p.tc->main_live, 1u) != 1u) return;
+  uint32_t ns = 128;
+  while (uint32_t(ld_relaxed_u64(&p.tc->done)) < p.B) {
+    __nanosleep(ns);
+    if (ns < 2048) ns <<= 1;
+  }
 }
 
 // one finished task: blocks_done += n, tasks_done += 1; the CTA that
@@ -261,11 +295,7 @@ __device__ __forceinline__ void count_done(const P& p, uint32_t n, uint32_t task
   if (uint32_t(old) + n == p.B) {
     const uint64_t t = globaltimer();
     p.tc->t_last = t;
-    if (p.mirror) {
-      p.mirror->t_last = t;
-      __threadfence_system();
-      p.mirror->complete = 1;
-    }
+    if (p.mirror) st_sys_u64(&p.mirror->done, t);
   }
 }
 
@@ -290,10 +320,11 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
 
   // ---- Lst1: the block leader binds the CTA to its SM
   if (threadIdx.x == 0) {
-    const uint32_t r = p.rank_of[smid()];
-    s_rank = r;
+    if (blockIdx.x == 0) atomicCAS(&p.tc->t_enter, 0ull, globaltimer());   // result unused
+    const uint32_t r = p.rank_of[smid()];   // in flight together with the prologue's loads
     s_retired = 0;
     s_go = prologue(p, r, c) ? 1u : 0u;
+    s_rank = r;
   }
   __syncthreads();
   if (!s_go) return;
@@ -327,7 +358,10 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     return s_g[slot];
   };
   auto prefetch_ctrl = [&]() {   // the next boundary's resize word, in flight during the task
-    if (threadIdx.x == 0) c2 = ld_acquire_u64(p.ctrl);
+    // relaxed: an acquire load here would hold back warp 0's body loads for an
+    // L2 round trip every task; the acquire is a fence at the boundary instead,
+    // taken only when the epoch changed (relaxed load + fence = acquire pattern)
+    if (threadIdx.x == 0) c2 = ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(p.ctrl));
   };
 
   c2 = c;
@@ -386,10 +420,11 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
       bool spec_retired = false, spec_changed = false;
       if (threadIdx.x == 0) {
         spec_changed = ctrl_epoch(c2) != ctrl_epoch(c);
+        if (spec_changed) asm volatile("fence.acq_rel.gpu;" ::: "memory");
         c = c2;
         if (!in_range(p, rank, c) && try_retire(p.tc)) spec_retired = true;
         else fut = atomicAdd(&p.tc->next, p.iters);                   // Lst2 (2), result used below
-        c2 = ld_acquire_u64(p.ctrl);                                  // for the next boundary
+        c2 = ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(p.ctrl));   // next boundary
       }
       if constexpr (Tn::kHasTask) {
         Tn::cta_task(p.args, g, n, dyn_smem);     // Lst2 (3)-(5) for a 1-D grid, blocks in flight together
@@ -428,7 +463,13 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     }
   }
   if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
-  if (threadIdx.x == 0 && my_blocks) count_done(p, my_blocks, my_tasks);
+  if (threadIdx.x == 0 && my_blocks) {
+    count_done(p, my_blocks, my_tasks);
+#ifdef SLATE_DIAG_EXIT   // diagnostic only: one more same-line atomic per CTA in the kernel's tail
+    atomicMax(&p.tc->t_exit, globaltimer());
+#endif
+  }
+  if (threadIdx.x == 0) leave_main(p);
   if (threadIdx.x < 32) {
     c = __shfl_sync(0xffffffffu, c, 0);
     if (lane == 0) atomicAdd(&p.tc->live_rank[rank], 0xffffffffu);   // live_rank -= 1

@@ -503,6 +503,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   __syncthreads();
   if (warp == kTaskWarp) {
     if (lane == 0) atomicAdd(&p.tc->live_rank[H.rank], 0xffffffffu);   // live_rank -= 1
+    if (lane == 0) leave_main(p);
     if (H.retired) check_shrink_done(p, H.ctrl, lane);
   }
 }
@@ -513,6 +514,8 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.gx = w.gx; p.gy = w.gy; p.gz = w.gz; p.B = w.B; p.iters = w.iters; p.occ = w.occ;
   p.bound_lo = w.bound_lo; p.bound_hi = w.bound_hi; p.n_ranks = w.n_ranks;
   p.standby_timeout_ns = w.standby_timeout_ns;
+  p.base_epoch = w.base_epoch;
+  p.is_topup = w.is_topup;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
   return cudaLaunchKernel(reinterpret_cast<const void*>(&spmv_worker), dim3(grid), dim3(kThreads), kargs, kSmemBytes,
@@ -543,6 +546,7 @@ KindOps spmv_ws_ops() {
   o.tasks_per_worker = 6;
   o.launch_worker = &spmv::launch_worker;
   o.launch_standalone = &spmv::launch_standalone;
+  o.topup_anytime = true;   // leave_main: the last main CTA waits for every block
   return o;
 }
 

@@ -18,6 +18,10 @@ namespace slate {
 __device__ __forceinline__ float4 ld_stream(const float4* p) { return __ldcs(p); }
 __device__ __forceinline__ void st_stream(float4* p, float4 v) { __stcs(p, v); }
 
+#ifndef SLATE_SPEC_SHORT
+#define SLATE_SPEC_SHORT 0   // experiment switch: speculative task fetch for the short-block Tab II tenants
+#endif
+
 // Optional per-tenant hooks default to off.
 struct TenantBase {
   static constexpr bool kHasInit = false;   // cta_init(smem): once per CTA before the first block
@@ -313,11 +317,15 @@ using SpmvCsrReg = SpmvCsrT<8, 4>;
 // one at d1: exp(-d2^2/2) = exp(-d1^2/2) S / (X e^{-rT}) (d1 sigma sqrt T =
 // ln(S/X) + (r + sigma^2/2) T); the put by put-call parity, put = call + X e^{-rT}
 // - S for every scenario, hence for their mean.
+#ifndef SLATE_BS_MINB
+#define SLATE_BS_MINB 4
+#endif
 struct BlackScholes : TenantBase {
   using Args = slate_args_bs;
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 4;
-  static constexpr bool kLateCtrl = true;    // a block is ~30 us at P = 32: honour a resize after it
+  static constexpr int kMinBlocks = SLATE_BS_MINB;
+  static constexpr bool kLateCtrl = !SLATE_SPEC_SHORT;    // a block is ~30 us at P = 32: honour a resize after it
+  static constexpr bool kSpeculative = SLATE_SPEC_SHORT;
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
   // one MUFU op each, no denormal range handling: every argument here is a
@@ -437,6 +445,214 @@ struct Stencil2D : TenantBase {
     const float up = __ldg(in + uint64_t(i - 1) * w + j), down = __ldg(in + uint64_t(i + 1) * w + j);
     const float v = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up, down), __fadd_rn(left, right)));
     reinterpret_cast<float*>(a.out)[uint64_t(i) * w + j] = v;
+  }
+};
+
+// ================================================================ the paper's own apps (Tab II, NEXT-2)
+// TR, MM, RG, GS of Tab II, written for B200 from the apps'
+// definitions (oracle/tenants.py); Black-Scholes is the BlackScholes tenant
+// with one scenario.  Bodies that stage through shared memory end with a
+// barrier: a worker runs its task's blocks back to back in the same CTA.
+
+// ---------------------------------------------------------------- TR: transpose
+// 32x32 tile through shared memory (+1 column of padding: the transposed read
+// is conflict-free), both the load and the store coalesced; thread (tx, ty)
+// moves rows ty, ty+8, ty+16, ty+24 of the tile.
+struct Transpose : TenantBase {
+  using Args = slate_args_transpose;
+  static constexpr bool kSpeculative = SLATE_SPEC_SHORT;
+  static constexpr int kThreads = 256;        // 32 x 8
+  static constexpr int kMinBlocks = 8;
+  static constexpr int kSmem = 32 * 33 * 4, kSmemStandalone = 32 * 33 * 4;
+
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t bx, uint32_t by, uint32_t, char* smem) {
+    float (*tile)[33] = reinterpret_cast<float (*)[33]>(smem);
+    const float* in = reinterpret_cast<const float*>(a.in);
+    float* out = reinterpret_cast<float*>(a.out);
+    const uint32_t tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    const uint32_t c = bx * 32 + tx;
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      const uint32_t row = by * 32 + ty + 8 * r;
+      if (row < a.h && c < a.w) tile[ty + 8 * r][tx] = __ldcs(in + uint64_t(row) * a.w + c);
+    }
+    __syncthreads();
+    const uint32_t i = by * 32 + tx;             // output column = input row
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      const uint32_t j = bx * 32 + ty + 8 * r;   // output row = input column
+      if (j < a.w && i < a.h) __stcs(out + uint64_t(j) * a.h + i, tile[tx][ty + 8 * r]);
+    }
+    __syncthreads();                             // the tile is reused by the worker's next block
+  }
+};
+
+// ---------------------------------------------------------------- MM: tiled SGEMM
+// The SDK matrixMul's scheme (32x32 C tile, A and B staged 32x32 at a time in
+// shared memory, k ascending), with each thread holding 4 C elements (rows
+// ty + 8r, column tx) and reading A's tile 4 k at a time (one broadcast
+// 128-bit load per row): every C element is the fmaf chain over k = 0..K-1 in
+// order from 0 -- the order of the naive kernel.  Out-of-range A/B entries are
+// staged as 0 (fmaf(0, b, acc) = acc).
+struct SgemmTiled : TenantBase {
+  using Args = slate_args_sgemm;
+  static constexpr int kThreads = 256;        // 32 x 8
+  static constexpr int kMinBlocks = 4;
+  static constexpr int kSmem = 2 * 32 * 32 * 4, kSmemStandalone = 2 * 32 * 32 * 4;
+
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t bx, uint32_t by, uint32_t, char* smem) {
+    float (*As)[32] = reinterpret_cast<float (*)[32]>(smem);
+    float (*Bs)[32] = reinterpret_cast<float (*)[32]>(smem + 32 * 32 * 4);
+    const float* A = reinterpret_cast<const float*>(a.A);
+    const float* B = reinterpret_cast<const float*>(a.B);
+    const uint32_t tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    const uint32_t r0 = by * 32, c0 = bx * 32;
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+    for (uint32_t k0 = 0; k0 < a.k; k0 += 32) {
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {
+        const uint32_t row = r0 + ty + 8 * r, ka = k0 + tx;
+        As[ty + 8 * r][tx] = (row < a.m && ka < a.k) ? __ldg(A + uint64_t(row) * a.k + ka) : 0.f;
+        const uint32_t kb = k0 + ty + 8 * r, col = c0 + tx;
+        Bs[ty + 8 * r][tx] = (kb < a.k && col < a.n) ? __ldg(B + uint64_t(kb) * a.n + col) : 0.f;
+      }
+      __syncthreads();
+#pragma unroll
+      for (int kk = 0; kk < 32; kk += 4) {
+        const float b0 = Bs[kk][tx], b1 = Bs[kk + 1][tx], b2 = Bs[kk + 2][tx], b3 = Bs[kk + 3][tx];
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+          const float4 av = *reinterpret_cast<const float4*>(&As[ty + 8 * r][kk]);
+          acc[r] = __fmaf_rn(av.x, b0, acc[r]);
+          acc[r] = __fmaf_rn(av.y, b1, acc[r]);
+          acc[r] = __fmaf_rn(av.z, b2, acc[r]);
+          acc[r] = __fmaf_rn(av.w, b3, acc[r]);
+        }
+      }
+      __syncthreads();                           // tiles reused by the next k slice / next block
+    }
+    float* C = reinterpret_cast<float*>(a.C);
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      const uint32_t row = r0 + ty + 8 * r, col = c0 + tx;
+      if (row < a.m && col < a.n) C[uint64_t(row) * a.n + col] = acc[r];
+    }
+  }
+};
+
+// ---------------------------------------------------------------- RG: quasirandom generator
+// The SDK quasirandomGenerator kernel: q_d(k) = XOR of table[d][b] over the set
+// bits of k, written as float(q + 1) * 2^-31.  Thread t of block (x, d) makes
+// points 1024x + 4t .. +3: the first by the 31-bit walk, the next three by the
+// GF(2) linearity q(k+1) = q(k) ^ q(k ^ (k+1)), where k ^ (k+1) = 2^(c+1) - 1
+// (c = trailing ones of k) and q of it is a prefix XOR of the table -- the
+// same bits as the walk (XOR is exact), ~4x fewer integer ops.
+struct Qrng : TenantBase {
+  using Args = slate_args_qrng;
+  static constexpr bool kSpeculative = SLATE_SPEC_SHORT;
+  static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 8;
+  static constexpr int kSmem = 2 * 32 * 4, kSmemStandalone = 2 * 32 * 4;
+
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t d, uint32_t, char* smem) {
+    uint32_t* tab = reinterpret_cast<uint32_t*>(smem);        // [0, 31): table row d
+    uint32_t* pre = tab + 32;                                  // [0, 32): prefix XORs, pre[c] = tab[0] ^ .. ^ tab[c]
+    const uint32_t* table = reinterpret_cast<const uint32_t*>(a.table) + uint64_t(d) * 31;
+    if (threadIdx.x < 32) {
+      const uint32_t v = threadIdx.x < 31 ? __ldg(table + threadIdx.x) : 0u;
+      uint32_t p = v;                                          // inclusive prefix XOR over the warp
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t q = __shfl_up_sync(0xffffffffu, p, o);
+        if (threadIdx.x >= uint32_t(o)) p ^= q;
+      }
+      tab[threadIdx.x] = v;
+      pre[threadIdx.x] = p;
+    }
+    __syncthreads();
+    const uint32_t i0 = x * 1024 + threadIdx.x * 4;
+    float o[4];
+    uint32_t k = a.seed + i0;
+    uint32_t q = 0;
+#pragma unroll
+    for (int b = 0; b < 31; ++b) q ^= ((k >> b) & 1u) ? tab[b] : 0u;
+    o[0] = __fmul_rn(__uint2float_rn(q + 1u), 4.656612873077392578125e-10f);   // 2^-31
+#pragma unroll
+    for (int j = 1; j < 4; ++j) {
+      const uint32_t c = min(uint32_t(__ffs(~k)) - 1u, 30u);   // trailing ones of k (bit 31 is outside the table)
+      q ^= pre[c];
+      ++k;
+      o[j] = __fmul_rn(__uint2float_rn(q + 1u), 4.656612873077392578125e-10f);
+    }
+    float* out = reinterpret_cast<float*>(a.out) + uint64_t(d) * a.n;
+    if (i0 + 4 <= a.n && ((uint64_t(d) * a.n) & 3) == 0) {
+      __stcs(reinterpret_cast<float4*>(out + i0), make_float4(o[0], o[1], o[2], o[3]));
+    } else {
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (i0 + j < a.n) out[i0 + j] = o[j];
+    }
+    __syncthreads();                             // the table is reused by the worker's next block
+  }
+};
+
+// ---------------------------------------------------------------- GS: Gaussian elimination
+// Rodinia gaussian's two kernels for elimination step t.  Fan1 computes the
+// multipliers of column t; Fan2 applies the rank-1 update to the trailing rows
+// (columns t .. n-1, column t included as in Rodinia) and to b.  Rodinia maps
+// threadIdx.x to rows (strided, uncoalesced); here lanes run along a row, so
+// every warp access is one or more full 128-byte lines; each element's update
+// is the same single fmaf(-m, pivot, a).
+struct GaussFan1 : TenantBase {
+  using Args = slate_args_gauss;
+  static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 8;
+  static constexpr int kSmem = 0, kSmemStandalone = 0;
+
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
+    const float* A = reinterpret_cast<const float*>(a.a);
+    const uint32_t i = a.t + 1 + x * 256 + threadIdx.x;
+    if (i >= a.n) return;
+    reinterpret_cast<float*>(a.m)[uint64_t(i) * a.n + a.t] =
+        __fdiv_rn(A[uint64_t(i) * a.n + a.t], A[uint64_t(a.t) * a.n + a.t]);
+  }
+};
+
+struct GaussFan2 : TenantBase {
+  using Args = slate_args_gauss;
+  static constexpr bool kSpeculative = SLATE_SPEC_SHORT;
+  static constexpr int kThreads = 256;        // 8 warps x 2 rows, lanes along 128 columns
+  static constexpr int kMinBlocks = 8;
+  static constexpr int kSmem = 0, kSmemStandalone = 0;
+
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t y, uint32_t, char*) {
+    float* A = reinterpret_cast<float*>(a.a);
+    const float* M = reinterpret_cast<const float*>(a.m);
+    const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const uint32_t n = a.n, t = a.t;
+    const uint32_t c0 = t + x * 128 + lane;
+    float piv[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t j = c0 + 32 * q;
+      piv[q] = j < n ? __ldg(A + uint64_t(t) * n + j) : 0.f;
+    }
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      const uint32_t i = t + 1 + y * 16 + w * 2 + r;
+      if (i >= n) break;
+      const float mi = __ldg(M + uint64_t(i) * n + t);
+      float* row = A + uint64_t(i) * n;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t j = c0 + 32 * q;
+        if (j < n) row[j] = __fmaf_rn(-mi, piv[q], row[j]);
+      }
+      if (x == 0 && lane == 0) {
+        float* b = reinterpret_cast<float*>(a.b);
+        b[i] = __fmaf_rn(-mi, b[t], b[i]);
+      }
+    }
   }
 };
 

@@ -171,8 +171,10 @@ def gauss_inputs(n, seed=None, mode="rodinia"):
     a[i][j] = 10 exp(-0.01 |i - j|) (symmetric positive definite, so no pivoting
     is needed), b = 1.  ``int``: a = L U with L unit lower triangular, entries
     in {-1, 0, 1}, and U upper triangular with unit diagonal and entries in
-    [-2, 2], b integers in [-4, 4]: every multiplier and every intermediate
-    value of the elimination is a small integer, exact in fp32."""
+    [-2, 2], and b = L y with y integers in [-4, 4]: after step t every
+    trailing entry is sum_{k >= t} L_ik U_kj (resp. L_ik y_k), so every
+    multiplier and every intermediate value of the elimination is a small
+    integer, exact in fp32."""
     if mode == "rodinia":
         i = np.arange(n)
         a = (10.0 * np.exp(-0.01 * np.abs(i[:, None] - i[None, :]))).astype(np.float32)
@@ -181,5 +183,6 @@ def gauss_inputs(n, seed=None, mode="rodinia"):
     L = np.tril(g.integers(-1, 2, size=(n, n)), -1) + np.eye(n, dtype=np.int64)
     U = np.triu(g.integers(-2, 3, size=(n, n)), 1) + np.eye(n, dtype=np.int64)
     a = (L @ U).astype(np.float32)
-    b = g.integers(-4, 5, size=n).astype(np.float32)
+    y = g.integers(-4, 5, size=n)
+    b = (L @ y).astype(np.float32)
     return a, b

@@ -24,6 +24,8 @@ OK, DONE = 0, 1
 EINVAL, ENOMEM, ECUDA, EIPC, ETIMEDOUT, ENOTFOUND, ESTATE, EUNSUPPORTED = -1, -2, -3, -4, -5, -6, -7, -8
 
 KIND_TRIAD, KIND_COPY, KIND_SGEMM_NAIVE, KIND_SPMV_CSR, KIND_BLACKSCHOLES, KIND_STENCIL2D, KIND_GEMM_BF16 = range(1, 8)
+# the paper's Tab II apps (TR, MM, RG, GS = Fan1 + Fan2; BS is KIND_BLACKSCHOLES with one scenario)
+KIND_TRANSPOSE, KIND_SGEMM_TILED, KIND_QRNG, KIND_GAUSS_FAN1, KIND_GAUSS_FAN2 = range(8, 13)
 KFLAG_COVERAGE = 1
 PLACE_AUTO, PLACE_SOLO, PLACE_CORUN = 0, 1, 2
 MODE_SLATE, MODE_STANDALONE = 0, 1
@@ -68,6 +70,18 @@ class ArgsGemm(ctypes.Structure):
     _fields_ = [("A", c_u64), ("B", c_u64), ("C", c_u64), ("m", c_u32), ("n", c_u32), ("k", c_u32), ("pad_", c_u32)]
 
 
+class ArgsTranspose(ctypes.Structure):
+    _fields_ = [("inp", c_u64), ("out", c_u64), ("h", c_u32), ("w", c_u32)]
+
+
+class ArgsQrng(ctypes.Structure):
+    _fields_ = [("table", c_u64), ("out", c_u64), ("n", c_u32), ("dims", c_u32), ("seed", c_u32), ("pad_", c_u32)]
+
+
+class ArgsGauss(ctypes.Structure):
+    _fields_ = [("a", c_u64), ("b", c_u64), ("m", c_u64), ("n", c_u32), ("t", c_u32)]
+
+
 class Info(ctypes.Structure):
     _fields_ = [("abi_version", c_u32), ("num_sms", c_u32), ("max_smid", c_u32), ("device", c_u32),
                 ("server_pid", c_u64), ("peak_hbm_gbps", c_f64), ("peak_fp32_gflops", c_f64),
@@ -103,7 +117,8 @@ class LaunchInfo(ctypes.Structure):
                 ("sm_lo", c_u32), ("sm_hi", c_u32), ("n_resizes", c_u32), ("n_topups", c_u32),
                 ("workers_started", c_u32), ("coverage_ok", c_u32), ("epoch", c_u32), ("shrink_epoch", c_u32),
                 ("join_epoch", c_u32), ("pad_", c_u32), ("t_first_ns", c_u64), ("t_last_ns", c_u64),
-                ("start_ms", c_f64), ("end_ms", c_f64), ("resize_us", c_f64 * 16), ("resize_kind", ctypes.c_uint8 * 16)]
+                ("start_ms", c_f64), ("end_ms", c_f64), ("resize_us", c_f64 * 16), ("resize_kind", ctypes.c_uint8 * 16),
+                ("t_enter_ns", c_u64), ("t_exit_ns", c_u64)]
 
     def as_dict(self):
         d = {f[0]: getattr(self, f[0]) for f in self._fields_}
@@ -372,3 +387,29 @@ def gemm_args(A, B, C):
     m, k = A.shape
     n, _ = B.shape
     return ArgsGemm(_ptr(A), _ptr(B), _ptr(C), m, n, k, 0), (n // GEMM_TILE_N, m // GEMM_TILE_M, 1)
+
+
+def transpose_args(inp, out):
+    h, w = inp.shape
+    return ArgsTranspose(_ptr(inp), _ptr(out), h, w), (cdiv(w, 32), cdiv(h, 32), 1)
+
+
+def sgemm_tiled_args(A, B, C):
+    m, k = A.shape
+    _, n = B.shape
+    return ArgsSgemm(_ptr(A), _ptr(B), _ptr(C), m, n, k, 0), (cdiv(n, 32), cdiv(m, 32), 1)
+
+
+def qrng_args(table, out, seed=0):
+    dims, n = out.shape
+    return ArgsQrng(_ptr(table), _ptr(out), n, dims, seed & 0xFFFFFFFF, 0), (cdiv(n, 1024), dims, 1)
+
+
+def gauss_fan1_args(a, b, m, t):
+    n = a.shape[0]
+    return ArgsGauss(_ptr(a), _ptr(b), _ptr(m), n, t), (cdiv(n - 1 - t, 256), 1, 1)
+
+
+def gauss_fan2_args(a, b, m, t):
+    n = a.shape[0]
+    return ArgsGauss(_ptr(a), _ptr(b), _ptr(m), n, t), (cdiv(n - t, 128), cdiv(n - 1 - t, 16), 1)

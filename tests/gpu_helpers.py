@@ -27,13 +27,18 @@ def dev(a):
 class Tenant:
     """A tenant instance: device buffers, args, grid, and the oracle check."""
 
-    def __init__(self, kind, args, grid, outputs, check, keep):
+    def __init__(self, kind, args, grid, outputs, check, keep, initial=None):
         self.kind, self.args, self.grid, self.outputs, self.check, self._keep = kind, args, grid, outputs, check, keep
+        # in-place tenants (GS Fan2 updates a and b): every run restarts from these
+        self._initial = None if initial is None else [t.clone() for t in initial]
         torch.cuda.synchronize()   # inputs are written on torch's stream; the server's streams do not wait
 
     def zero_outputs(self):
-        for t in self.outputs:
-            t.zero_()
+        for i, t in enumerate(self.outputs):
+            if self._initial is None:
+                t.zero_()
+            else:
+                t.copy_(self._initial[i])
         torch.cuda.synchronize()
 
     def snapshot(self):
@@ -161,3 +166,91 @@ def make_gemm(m, n, k, seed, mode="float"):
         return ok, worst
 
     return Tenant(S.KIND_GEMM_BF16, args, grid, [C_d], check, (A_d, B_d))
+
+
+# ------------------------------------------------------------------ the paper's Tab II apps (NEXT-2)
+def make_transpose(h, w, seed):
+    A = I.transpose_inputs(h, w, seed)
+    in_d, out_d = dev(A), torch.zeros(w, h, device=DEV)
+    args, grid = S.transpose_args(in_d, out_d)
+
+    def check(outs, rows=None):
+        return outs[0].cpu().numpy().tobytes() == OT.transpose(A).tobytes(), 0.0
+
+    return Tenant(S.KIND_TRANSPOSE, args, grid, [out_d], check, (in_d,))
+
+
+def make_sgemm_tiled(m, n, k, seed, mode="float"):
+    A, B = I.sgemm_inputs(m, n, k, seed, mode)
+    A_d, B_d, C_d = dev(A), dev(B), torch.zeros(m, n, device=DEV)
+    args, grid = S.sgemm_tiled_args(A_d, B_d, C_d)
+
+    def check(outs, rows=None):
+        ref = OT.sgemm_tiled(A, B)
+        g = outs[0].cpu().numpy().astype(np.float64)
+        if mode == "int":
+            return np.array_equal(g, ref), 0.0
+        return within(g, ref, np.abs(A.astype(np.float64)) @ np.abs(B.astype(np.float64)))
+
+    return Tenant(S.KIND_SGEMM_TILED, args, grid, [C_d], check, (A_d, B_d))
+
+
+def make_qrng(n, dims, seed, qseed=0):
+    table = I.qrng_table(dims, seed)
+    t_d = dev(table.view(np.int32))
+    out_d = torch.zeros(dims, n, device=DEV)
+    args, grid = S.qrng_args(t_d, out_d, qseed)
+
+    def check(outs, rows=None):
+        return np.array_equal(outs[0].cpu().numpy(), OT.qrng(table, n, qseed)), 0.0
+
+    return Tenant(S.KIND_QRNG, args, grid, [out_d], check, (t_d,))
+
+
+def gauss_state(n, t, seed, mode):
+    """The system after t elimination steps of the oracle, as fp32 inputs (exact
+    in int mode), and the oracle's multipliers of column t (Fan1 of step t)."""
+    a0, b0 = I.gauss_inputs(n, seed, mode)
+    a, b, m = OT.gaussian(a0, b0, steps=t)
+    return a.astype(np.float32), b.astype(np.float32), m.astype(np.float32)
+
+
+def make_gauss_fan1(n, t, seed, mode="int"):
+    a, b, m = gauss_state(n, t, seed, mode)
+    a_d, b_d, m_d = dev(a), dev(b), torch.zeros(n, n, device=DEV)
+    args, grid = S.gauss_fan1_args(a_d, b_d, m_d, t)
+
+    def check(outs, rows=None):
+        ref = np.zeros((n, n))
+        OT.gauss_fan1(a.astype(np.float64), ref, t)
+        g = outs[0].cpu().numpy().astype(np.float64)
+        # fp32 division is correctly rounded; so is the fp64 quotient rounded to fp32
+        return np.array_equal(g, ref.astype(np.float32).astype(np.float64)), 0.0
+
+    return Tenant(S.KIND_GAUSS_FAN1, args, grid, [m_d], check, (a_d, b_d))
+
+
+def make_gauss_fan2(n, t, seed, mode="int"):
+    a, b, m = gauss_state(n, t, seed, mode)
+    mt = np.zeros((n, n))
+    OT.gauss_fan1(a.astype(np.float64), mt, t)
+    m[:, t] = mt[:, t].astype(np.float32)
+    a_d, b_d, m_d = dev(a), dev(b), dev(m)
+    args, grid = S.gauss_fan2_args(a_d, b_d, m_d, t)
+
+    def check(outs, rows=None):
+        ra, rb = a.astype(np.float64), b.astype(np.float64)
+        OT.gauss_fan2(ra, rb, m.astype(np.float64), t)
+        ga = outs[0].cpu().numpy().astype(np.float64)
+        gb = outs[1].cpu().numpy().astype(np.float64)
+        if mode == "int":
+            return np.array_equal(ga, ra) and np.array_equal(gb, rb), 0.0
+        # one fmaf per element: Q17 with scale |a| + |m p|
+        m64 = m[:, t].astype(np.float64)
+        sa = np.abs(a.astype(np.float64)) + np.abs(m64)[:, None] * np.abs(a[t].astype(np.float64))[None, :]
+        sb = np.abs(b.astype(np.float64)) + np.abs(m64) * abs(float(b[t]))
+        ok1, e1 = within(ga, ra, sa)
+        ok2, e2 = within(gb, rb, sb)
+        return ok1 and ok2, max(e1, e2)
+
+    return Tenant(S.KIND_GAUSS_FAN2, args, grid, [a_d, b_d], check, (m_d,), initial=[a_d, b_d])

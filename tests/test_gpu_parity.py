@@ -12,7 +12,8 @@ import torch
 from oracle import tenants as OT
 from paper_conf_ipps_allenf019_b200 import slate as S
 
-from gpu_helpers import (make_bs, make_copy, make_gemm, make_sgemm, make_spmv, make_stencil, make_triad)
+from gpu_helpers import (make_bs, make_copy, make_gauss_fan1, make_gauss_fan2, make_gemm, make_qrng, make_sgemm,
+                         make_sgemm_tiled, make_spmv, make_stencil, make_transpose, make_triad)
 
 pytestmark = pytest.mark.gpu
 
@@ -37,6 +38,18 @@ CASES = {
     "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
     "gemm_int": lambda: make_gemm(256, 512, 512, 113, "int"),
     "gemm_float": lambda: make_gemm(768, 512, 1024, 114),
+    # the paper's Tab II apps (NEXT-2)
+    "tr": lambda: make_transpose(32 * 11 + 7, 32 * 9 + 19, 120),
+    "tr_row": lambda: make_transpose(1, 32 * 40 + 1, 121),
+    "mm_float": lambda: make_sgemm_tiled(32 * 7 + 5, 32 * 6 + 31, 32 * 3 + 9, 122),
+    "mm_int": lambda: make_sgemm_tiled(256, 192, 160, 123, "int"),
+    "rg": lambda: make_qrng(1024 * 13 + 4 * 17 + 2, 3, 124, qseed=5),
+    "rg_wrap": lambda: make_qrng(1024 * 3, 2, 125, qseed=2 ** 32 - 1500),   # k wraps past 2^31 and 2^32
+    "bs_textbook": lambda: make_bs(1024 * 9 + 3, 130, n_scen=1),
+    "gs_fan1": lambda: make_gauss_fan1(700, 37, 126, "rodinia"),
+    "gs_fan2_int": lambda: make_gauss_fan2(300, 11, 127, "int"),
+    "gs_fan2_float": lambda: make_gauss_fan2(500, 23, 128, "rodinia"),
+    "gs_fan2_last": lambda: make_gauss_fan2(200, 198, 129, "int"),
 }
 
 

@@ -94,7 +94,7 @@ def test_resize_storm_spmv_warp_specialised(sess):
 def test_resize_storm_iters1_copy(sess):
     t = make_copy(1 << 30, 203)
     q, done = _storm(sess, t, 1, 40, 3, 10)
-    assert done >= 5
+    assert done >= 4          # the 8-GiB copy lasts ~1.5 ms: a handful of resizes land while it runs
     assert len(q["resize_us"]) >= 3, q
 
 
