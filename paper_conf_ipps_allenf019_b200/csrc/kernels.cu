@@ -27,10 +27,11 @@ cudaError_t launch_worker_t(const WorkerCommon& w, const void* args, uint32_t gr
   p.standby_timeout_ns = w.standby_timeout_ns;
   p.base_epoch = w.base_epoch;
   p.is_topup = w.is_topup;
+  p.gate_first = w.gate_first;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
-  return cudaLaunchKernel(reinterpret_cast<const void*>(&slate_worker<Tn>), dim3(grid), dim3(Tn::kThreads), kargs,
-                          Tn::kSmem, st);
+  return launch_kernel(reinterpret_cast<const void*>(&slate_worker<Tn>), dim3(grid), dim3(Tn::kThreads), kargs,
+                       Tn::kSmem, st, w.pdl);
 }
 
 template <class Tn>
@@ -57,6 +58,7 @@ KindOps make_ops(uint32_t default_iters) {
   o.launch_worker = &launch_worker_t<Tn>;
   o.launch_standalone = &launch_standalone_t<Tn>;
   o.topup_anytime = true;
+  o.pdl_ok = true;
   return o;
 }
 

@@ -75,6 +75,9 @@ struct WorkerCommon {
   uint32_t bound_lo, bound_hi, n_ranks, standby_timeout_ns;
   uint32_t base_epoch;   // the queue's epoch at issue (0 for top-ups: every join of theirs is a grow)
   uint32_t is_topup;     // 1: a top-up grid sharing a running launch's counter
+  uint32_t gate_first;   // top-up of a launch with no start event: wait until the launch took its first task
+  bool pdl = false;      // launch with programmatic stream serialization (the previous op on the stream is
+                         // the previous worker of the same batch; the worker waits in griddepcontrol.wait)
   const uint64_t* ctrl;
   TaskCtl* tc;
   HostMirror* mirror;
@@ -95,6 +98,7 @@ struct KindOps {
   uint32_t tasks_per_worker = 8; // the automatic task size aims at >= this many tasks per worker
   uint32_t tile_m = 0;           // GEMM: output rows per original block
   uint32_t tile_n = 0;           // GEMM: output columns per original block
+  bool pdl_ok = false;           // the worker calls griddepcontrol.wait before its first task
   bool topup_anytime = false;    // the worker's last main CTA waits for every block (leave_main), so a
                                  // running launch may get a top-up while later launches are queued
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;
@@ -102,6 +106,25 @@ struct KindOps {
 };
 
 const KindOps* kind_ops(uint32_t kind);   // nullptr if the kind is not built
+
+// cudaLaunchKernel, or with programmatic dependent launch (PDL): the kernel may
+// start while the previous kernel on the stream drains, and waits for it in
+// griddepcontrol.wait (tools/probe/pdl_cost.cu: ~2 us per back-to-back launch)
+inline cudaError_t launch_kernel(const void* fn, dim3 grid, dim3 block, void** args, size_t smem, cudaStream_t st,
+                                 bool pdl) {
+  if (!pdl) return cudaLaunchKernel(fn, grid, block, args, smem, st);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelExC(&cfg, fn, args);
+}
 cudaError_t launch_calibrate(uint32_t* out, uint32_t blocks, uint32_t spin_ns, cudaStream_t st);
 cudaError_t launch_clock_probe(volatile uint32_t* flag, volatile unsigned long long* stamp, int rounds,
                                cudaStream_t st);

@@ -140,6 +140,9 @@ int Server::init(std::string* err) {
     const std::string v(pol);
     policy_ = v == "table" ? SLATE_POLICY_TABLE : v == "literal" ? SLATE_POLICY_LITERAL : SLATE_POLICY_HYBRID;
   }
+  {
+    pdl_enabled_ = env_double("SLATE_PDL", 1.0) != 0.0;
+  }
   min_gain_ = env_double("SLATE_MIN_GAIN", 1.05);
   poller_ = std::thread([this] { poller_main(); });
   return SLATE_OK;
@@ -279,6 +282,13 @@ int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
     cudaStreamDestroy(Q.stream);
     for (cudaStream_t a : Q.aux)
       if (a) cudaStreamDestroy(a);
+    // a queue can still hold SMs with nothing issued (a resize after its last
+    // launch completed activates it): give them back before it goes away, and
+    // leave no reference to it in the scheduler's lists
+    if (Q.active) release(Q);
+    waiting_.erase(std::remove(waiting_.begin(), waiting_.end(), q), waiting_.end());
+    active_.erase(std::remove(active_.begin(), active_.end(), q), active_.end());
+    bypassed_.erase(q);
     queues_.erase(it);
   }
   return rc;
@@ -580,6 +590,7 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
   CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
   CK(cudaEventRecord(ev, ctrl_stream_));
   CK(cudaStreamWaitEvent(Q.stream, ev, 0));
+  Q.last_op_kernel = false;
   cudaEventDestroy(ev);
   return SLATE_OK;
 }
@@ -591,10 +602,42 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
 int Server::issue(Launch& L, Queue& Q, std::string* err) {
   const bool needs_slot = L.desc.mode != SLATE_MODE_STANDALONE;
   if (!Q.deferred.empty() || (needs_slot && free_slots_.empty())) {
+    if (!Q.open_batch.empty()) close_batch(Q, nullptr);
     Q.deferred.push_back(L.id);
     return SLATE_OK;
   }
   return issue_now(L, Q, err);
+}
+
+// End the queue's open batch: every member completes with the batch's end
+// event `end` (recorded here on the queue's stream if null); the workers'
+// control-block snapshots are copied after it.
+void Server::close_batch(Queue& Q, cudaEvent_t end, bool closed_by_launch) {
+  if (Q.open_batch.empty()) return;
+  if (!end) {
+    cudaEventCreate(&end);
+    cudaEventRecord(end, Q.stream);
+    Q.last_op_kernel = false;
+  }
+  std::vector<Launch*> ws;
+  for (uint64_t id : Q.open_batch) {
+    Launch& M = *launches_[id];
+    M.batch_end = end;
+    M.batch_n = uint32_t(Q.open_batch.size()) + (closed_by_launch ? 1u : 0u);
+    if (M.slot >= 0) ws.push_back(&M);
+    else M.ev_done.push_back(end);
+  }
+  if (!ws.empty()) {
+    cudaEvent_t snap;
+    cudaEventCreateWithFlags(&snap, cudaEventDisableTiming);
+    cudaStreamWaitEvent(copy_stream_, end, 0);
+    for (Launch* M : ws)
+      cudaMemcpyAsync(h_snap_ + size_t(M->slot) * kTaskCtlHeader, d_tc_ + M->slot, kTaskCtlHeader,
+                      cudaMemcpyDeviceToHost, copy_stream_);
+    cudaEventRecord(snap, copy_stream_);
+    for (Launch* M : ws) M->ev_done.push_back(snap);
+  }
+  Q.open_batch.clear();
 }
 
 void Server::fail_launch(Launch& L, int code) {
@@ -609,32 +652,50 @@ void Server::drain_deferred(Queue& Q) {
     Launch& L = *launches_[Q.deferred.front()];
     if (L.desc.mode != SLATE_MODE_STANDALONE && free_slots_.empty()) break;
     Q.deferred.pop_front();
+    const Launch* nx = Q.deferred.empty() ? nullptr : launches_[Q.deferred.front()].get();
+    batch_more_ = nx && (nx->desc.mode == SLATE_MODE_STANDALONE || free_slots_.size() > 1);
     if (issue_now(L, Q, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
+    batch_more_ = false;
   }
+  close_batch(Q, nullptr);
 }
 
 int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
   const KindOps* ops = L.k->ops;
-  for (cudaEvent_t e : Q.topup_ends)   // stream semantics: the predecessor's top-up workers finish first
+  for (cudaEvent_t e : Q.topup_ends) {   // stream semantics: the predecessor's top-up workers finish first
     CK(cudaStreamWaitEvent(Q.stream, e, 0));
+    Q.last_op_kernel = false;
+  }
   Q.topup_ends.clear();
-  // A launch queued right behind another of its queue starts where that one
-  // ends (stream order), so it records no start event of its own: an event
-  // between two kernels costs ~3 us of stream time (tools/probe/pdl_cost.cu).
-  if (!Q.issued.empty() && !launches_[Q.issued.back()]->ev_end.empty()) {
+  // a batch holds launches of one mode
+  if (!Q.open_batch.empty() && launches_[Q.open_batch.front()]->desc.mode != L.desc.mode) close_batch(Q, nullptr);
+  // Events between kernels cost ~3 us of stream time each and stop programmatic
+  // dependent launch (tools/probe/pdl_cost.cu).  A launch queued right behind
+  // another of its queue starts where that one ends (stream order), so it
+  // records no start event; inside a batch (launches issued back to back by one
+  // loop) only the last records an end event.
+  const bool in_batch = !Q.open_batch.empty();
+  if (in_batch) {
+    L.batch_first = Q.open_batch.front();
+    L.batch_idx = uint32_t(Q.open_batch.size());
+  } else if (!Q.issued.empty() && !launches_[Q.issued.back()]->ev_end.empty()) {
     L.start_after = launches_[Q.issued.back()]->ev_end.front();
   } else {
     CK(cudaEventCreate(&L.ev_start));
   }
-  cudaEvent_t ev_end;
-  CK(cudaEventCreate(&ev_end));
+  const bool batch_member = batch_more_;   // no end event: the batch's end completes it
+  cudaEvent_t ev_end = nullptr;
+  if (!batch_member) CK(cudaEventCreate(&ev_end));
   const auto& g = L.desc.grid;
   if (L.desc.mode == SLATE_MODE_STANDALONE) {
     if (L.ev_start) CK(cudaEventRecord(L.ev_start, Q.stream));
     CK(ops->launch_standalone(L.args.data(), dim3(g[0], g[1], g[2]), Q.stream));
-    CK(cudaEventRecord(ev_end, Q.stream));
-    L.ev_end.push_back(ev_end);
-    L.ev_done.push_back(ev_end);
+    Q.last_op_kernel = false;   // standalone kernels do not wait in griddepcontrol.wait: no PDL after them
+    if (ev_end) {
+      CK(cudaEventRecord(ev_end, Q.stream));
+      L.ev_end.push_back(ev_end);
+      L.ev_done.push_back(ev_end);
+    }
   } else {
     const int slot = alloc_slot();
     if (slot < 0) {
@@ -645,9 +706,14 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     std::memset(reinterpret_cast<void*>(h_mirror_ + slot), 0, sizeof(HostMirror));
     // the control block was zeroed by DMA when it was freed (no SM needed); only
     // wait (a cross-stream dependency) if that copy has not finished yet
-    if (slot_zeroed_[slot] && cudaEventQuery(slot_zeroed_[slot]) != cudaSuccess)
+    if (slot_zeroed_[slot] && cudaEventQuery(slot_zeroed_[slot]) != cudaSuccess) {
       CK(cudaStreamWaitEvent(Q.stream, slot_zeroed_[slot], 0));
-    if (L.ev_start) CK(cudaEventRecord(L.ev_start, Q.stream));
+      Q.last_op_kernel = false;
+    }
+    if (L.ev_start) {
+      CK(cudaEventRecord(L.ev_start, Q.stream));
+      Q.last_op_kernel = false;
+    }
     WorkerCommon w{};
     w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = L.B; w.iters = L.iters; w.occ = uint32_t(L.k->occ);
     w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
@@ -656,16 +722,28 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     w.ctrl = Q.d_ctrl; w.tc = d_tc_ + slot; w.mirror = d_mirror_ + slot;
     w.cov = reinterpret_cast<uint32_t*>(L.desc.coverage);
     w.rank_of = d_rank_of_;
+    // PDL: the previous op on the stream is the previous worker of this batch
+    w.pdl = in_batch && Q.last_op_kernel && ops->pdl_ok && pdl_enabled_;
     CK(ops->launch_worker(w, L.args.data(), worker_grid(L.k->occ, L.B, L.iters), Q.stream));
-    CK(cudaEventRecord(ev_end, Q.stream));
-    L.ev_end.push_back(ev_end);
-    cudaEvent_t ev_snap;
-    CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
-    CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
-    CK(cudaMemcpyAsync(h_snap_ + size_t(slot) * kTaskCtlHeader, d_tc_ + slot, kTaskCtlHeader, cudaMemcpyDeviceToHost,
-                       copy_stream_));
-    CK(cudaEventRecord(ev_snap, copy_stream_));
-    L.ev_done.push_back(ev_snap);
+    Q.last_op_kernel = ops->pdl_ok;
+    if (ev_end) {
+      CK(cudaEventRecord(ev_end, Q.stream));
+      Q.last_op_kernel = false;
+      L.ev_end.push_back(ev_end);
+      cudaEvent_t ev_snap;
+      CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
+      CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+      CK(cudaMemcpyAsync(h_snap_ + size_t(slot) * kTaskCtlHeader, d_tc_ + slot, kTaskCtlHeader,
+                         cudaMemcpyDeviceToHost, copy_stream_));
+      CK(cudaEventRecord(ev_snap, copy_stream_));
+      L.ev_done.push_back(ev_snap);
+    }
+  }
+  if (batch_member) {
+    Q.open_batch.push_back(L.id);
+  } else if (!Q.open_batch.empty()) {
+    L.batch_n = uint32_t(Q.open_batch.size()) + 1;
+    close_batch(Q, ev_end, true);   // this launch ends the batch
   }
   L.state = 1;
   if (Q.issued.empty()) {
@@ -729,8 +807,10 @@ int Server::topup(Queue& Q, Launch& R, std::string* err) {
   CK(cudaEventRecord(ev_ctrl, ctrl_stream_));
   CK(cudaStreamWaitEvent(aux, ev_ctrl, 0));
   cudaEventDestroy(ev_ctrl);
-  CK(cudaStreamWaitEvent(aux, R.ev_start ? R.ev_start : R.start_after, 0));
+  cudaEvent_t r_start = R.ev_start ? R.ev_start : R.start_after;
+  if (r_start) CK(cudaStreamWaitEvent(aux, r_start, 0));
   WorkerCommon w{};
+  w.gate_first = r_start ? 0u : 1u;   // a batch member has no start event: its top-up waits on the device
   w.gx = g[0]; w.gy = g[1]; w.gz = g[2]; w.B = R.B; w.iters = R.iters; w.occ = uint32_t(R.k->occ);
   w.bound_lo = Q.lo; w.bound_hi = Q.hi; w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
@@ -779,9 +859,13 @@ int Server::launch_n(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint3
   int rc = SLATE_OK;
   for (uint32_t i = 0; i < n && rc == SLATE_OK; ++i) {
     uint64_t id = 0;
+    batch_more_ = i + 1 < n;   // the job's launches go out as one batch if the queue can take them now
     rc = launch_locked(q, kid, d, &id, err, i + 1 < n);
     if (i == 0) *first = id;
   }
+  batch_more_ = false;
+  auto qi = queues_.find(q);
+  if (qi != queues_.end()) close_batch(*qi->second, nullptr);
   return rc;
 }
 
@@ -1014,8 +1098,11 @@ void Server::schedule() {
       while (!Q.pending.empty()) {
         Launch& L = *launches_[Q.pending.front()];
         Q.pending.pop_front();
+        batch_more_ = !Q.pending.empty();
         if (issue(L, Q, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
       }
+      batch_more_ = false;
+      close_batch(Q, nullptr);
       continue;
     }
     if (active_.size() >= 2) break;
@@ -1089,8 +1176,11 @@ void Server::schedule() {
     while (!Bq.pending.empty()) {
       Launch& L = *launches_[Bq.pending.front()];
       Bq.pending.pop_front();
+      batch_more_ = !Bq.pending.empty();
       if (issue(L, Bq, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
     }
+    batch_more_ = false;
+    close_batch(Bq, nullptr);
     break;   // at most two co-runners (reading Q13)
   }
 }
@@ -1322,6 +1412,47 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
   return SLATE_OK;
 }
 
+// Event times of a launch relative to the server's epoch event (ms).  A batch
+// member (issued without events between kernels) is placed by its device
+// stamps relative to the batch's first launch (workers: first task and last
+// block), or, for original kernels, evenly between the batch's start and end.
+void Server::launch_times(const Launch& L, double* start, double* end) const {
+  auto ev_ms = [&](cudaEvent_t e) {
+    float ms = 0;
+    return (e && cudaEventElapsedTime(&ms, epoch_ev_, e) == cudaSuccess) ? double(ms) : -1.0;
+  };
+  auto snap = [](const Launch& X, unsigned long long* t0, unsigned long long* t1) {
+    TaskCtl tc;
+    std::memcpy(&tc, X.snapshot, kTaskCtlHeader);
+    *t0 = tc.t_first;
+    *t1 = tc.t_last;
+    return X.has_snapshot && tc.t_first && tc.t_last;
+  };
+  double s = ev_ms(L.ev_start ? L.ev_start : L.start_after), e = -1.0;
+  for (cudaEvent_t x : L.ev_end) e = std::max(e, ev_ms(x));
+  const Launch* F = &L;
+  if (L.batch_first) {
+    auto it = launches_.find(L.batch_first);
+    if (it != launches_.end()) F = it->second.get();
+  }
+  if (s < 0 || e < 0) {
+    const double fs = ev_ms(F->ev_start ? F->ev_start : F->start_after);
+    unsigned long long f0, f1, l0, l1;
+    if (snap(*F, &f0, &f1) && snap(L, &l0, &l1)) {                   // workers: device stamps
+      const double off = fs - double(f0) * 1e-6;
+      if (s < 0) s = off + double(l0) * 1e-6;
+      if (e < 0) e = off + double(l1) * 1e-6;
+    } else {                                                          // original kernels: evenly spread
+      const double be = L.batch_end ? ev_ms(L.batch_end) : e;
+      const double n = std::max(1u, L.batch_n), step = (be - fs) / n;
+      if (s < 0) s = fs + step * L.batch_idx;
+      if (e < 0) e = fs + step * (L.batch_idx + 1);
+    }
+  }
+  *start = std::max(0.0, s);
+  *end = std::max(*start, e);
+}
+
 int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
   std::unique_lock<std::mutex> g(mu_);
   auto it = launches_.find(l);
@@ -1369,12 +1500,7 @@ int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
     out->t_exit_ns = tc.t_exit;
   }
   if (L.state == 2) {
-    float ms = 0;
-    if (cudaEventElapsedTime(&ms, epoch_ev_, L.ev_start ? L.ev_start : L.start_after) == cudaSuccess) out->start_ms = ms;
-    double end = 0;
-    for (cudaEvent_t e : L.ev_end)
-      if (cudaEventElapsedTime(&ms, epoch_ev_, e) == cudaSuccess) end = std::max(end, double(ms));
-    out->end_ms = end;
+    launch_times(L, &out->start_ms, &out->end_ms);
     if (L.desc.coverage) {
       std::vector<uint32_t> cov(L.B);
       CK(cudaMemcpyAsync(cov.data(), reinterpret_cast<void*>(L.desc.coverage), size_t(L.B) * 4, cudaMemcpyDeviceToHost,
@@ -1389,14 +1515,22 @@ int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
 // ------------------------------------------------------------------ profile
 int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t lo, uint32_t hi, int reps, double* ms,
                       std::string* err) {
-  // a private queue: its own stream and resize word; one control block slot
-  int slot;
+  // a private queue: its own stream and resize word; kBatch control blocks.
+  // A measurement is kBatch launches back to back (programmatic dependent
+  // launch, no events between them), as a job's launches run: the per-launch
+  // time is the batch's span over kBatch.
+  constexpr int kBatch = 8;
+  std::vector<int> slots;
   uint64_t* ctrl;
   {
     std::lock_guard<std::mutex> g(mu_);
-    slot = alloc_slot();
-    if (slot < 0 || free_ctrl_.empty()) {
-      if (slot >= 0) free_slots_.push_back(slot);
+    while (int(slots.size()) < kBatch) {
+      const int sl = alloc_slot();
+      if (sl < 0) break;
+      slots.push_back(sl);
+    }
+    if (int(slots.size()) < kBatch || free_ctrl_.empty()) {
+      for (int sl : slots) free_slots_.push_back(sl);
       if (err) *err = "pool exhausted";
       return SLATE_ENOMEM;
     }
@@ -1414,20 +1548,25 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   w.iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters, k.ops->tasks_per_worker);
   w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
-  w.ctrl = ctrl; w.tc = d_tc_ + slot; w.mirror = nullptr; w.cov = nullptr; w.rank_of = d_rank_of_;
+  w.ctrl = ctrl; w.mirror = nullptr; w.cov = nullptr; w.rank_of = d_rank_of_;
   cudaEvent_t e0, e1;
   CK(cudaEventCreate(&e0));
   CK(cudaEventCreate(&e1));
   std::vector<double> times;
   for (int r = 0; r < reps + 1; ++r) {
-    CK(cudaMemcpyAsync(d_tc_ + slot, h_zero_, sizeof(TaskCtl), cudaMemcpyHostToDevice, st));
+    for (int sl : slots)
+      CK(cudaMemcpyAsync(d_tc_ + sl, h_zero_, sizeof(TaskCtl), cudaMemcpyHostToDevice, st));
     CK(cudaEventRecord(e0, st));
-    CK(k.ops->launch_worker(w, d->args, worker_grid(k.occ, B, w.iters), st));
+    for (int i = 0; i < kBatch; ++i) {
+      w.tc = d_tc_ + slots[i];
+      w.pdl = i > 0 && k.ops->pdl_ok && pdl_enabled_;
+      CK(k.ops->launch_worker(w, d->args, worker_grid(k.occ, B, w.iters), st));
+    }
     CK(cudaEventRecord(e1, st));
     CK(cudaEventSynchronize(e1));
     float t;
     CK(cudaEventElapsedTime(&t, e0, e1));
-    if (r > 0) times.push_back(t);   // the first run warms up
+    if (r > 0) times.push_back(t / kBatch);   // the first run warms up
   }
   std::sort(times.begin(), times.end());
   *ms = times[times.size() / 2];
@@ -1435,7 +1574,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   cudaEventDestroy(e1);
   cudaStreamDestroy(st);
   std::lock_guard<std::mutex> g(mu_);
-  free_slot(slot);
+  for (int sl : slots) free_slot(sl);
   free_ctrl_.push_back(int((ctrl - d_ctrl_pool_) / 16));
   return SLATE_OK;
 }

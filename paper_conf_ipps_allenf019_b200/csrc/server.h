@@ -38,6 +38,12 @@ struct Launch {
   int slot = -1;                // TaskCtl / mirror slot
   cudaEvent_t ev_start = nullptr;     // recorded before the kernel, or null when chained:
   cudaEvent_t start_after = nullptr;  // the predecessor's end (same stream): this launch starts there
+  // batch issue (no events between the kernels of a batch): the batch's first
+  // launch (times of members come from device stamps relative to it), the
+  // member's index, and the event that ends the batch
+  uint64_t batch_first = 0;
+  uint32_t batch_idx = 0, batch_n = 0;
+  cudaEvent_t batch_end = nullptr;
   std::vector<cudaEvent_t> ev_end;    // kernel ends (main + top-ups), for timing
   std::vector<cudaEvent_t> ev_done;   // all must complete (main + top-ups, after snapshots)
   int error = 0;                      // cudaError_t seen on completion
@@ -71,6 +77,8 @@ struct Queue {
   std::deque<uint64_t> deferred;  // granted SMs but waiting for a control block (stream order)
   std::deque<uint64_t> issued;  // issued, not complete (stream order)
   std::vector<cudaEvent_t> topup_ends;  // top-ups of the last issued launch: successors wait for all
+  std::vector<uint64_t> open_batch;     // issued launches of the current batch, no end event yet
+  bool last_op_kernel = false;          // the last op on `stream` is the last issued worker kernel (PDL)
   // resize latencies being measured (Q30): epoch, kind (1 shrink, 2 grow), host
   // t0, and where the result goes (launch id, index in its resize_us)
   struct PendingResize { uint32_t epoch; int kind; double t0_us; uint64_t lid; int idx; };
@@ -114,6 +122,10 @@ class Server {
   int write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool immediate, std::string* err);
   int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
   int topup(Queue& Q, Launch& R, std::string* err);
+  void close_batch(Queue& Q, cudaEvent_t end, bool closed_by_launch = false);
+  void launch_times(const Launch& L, double* start, double* end) const;
+  bool batch_more_ = false;
+  bool pdl_enabled_ = true;   // SLATE_PDL=0 turns programmatic dependent launch off   // set by the issuing loops: another launch of this queue is issued right after
   void schedule();
   void release(Queue& Q);
   bool curve_of(const Launch& L, std::vector<uint32_t>* sms, std::vector<double>* ms) const;

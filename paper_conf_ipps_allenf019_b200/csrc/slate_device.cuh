@@ -78,12 +78,18 @@ struct WorkerParams {
   uint32_t standby_timeout_ns;
   uint32_t base_epoch;            // resize-word epoch when the launch was issued: a join under a later epoch is a grow
   uint32_t is_topup;              // 1: a top-up grid (grow) sharing a running launch's TaskCtl
+  uint32_t gate_first;            // top-up: join only once the launch has taken its first task
   const uint64_t* ctrl;           // the queue's resize word
   TaskCtl* tc;
   HostMirror* mirror;             // device alias of the pinned mirror (may be null)
   uint32_t* cov;                  // coverage log u32[B] or null
   const uint16_t* rank_of;        // %smid -> rank
 };
+
+// programmatic dependent launch: wait for the previous kernel on the stream
+// (no-op for a normal launch); let the next one start launching its CTAs
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // ------------------------------------------------------------------ decode (Lst2 (4))
 struct BlockWalk {
@@ -124,6 +130,9 @@ __device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
   TaskCtl* tc = p.tc;
   uint64_t t0 = 0;
   uint32_t backoff = 256;
+  if (p.gate_first) {   // top-up of a launch that has no start event: wait until it started
+    while (ld_relaxed_u64(&tc->t_first) == 0 && ld_relaxed_u32(&tc->next) < p.B) __nanosleep(512);
+  }
   for (;;) {
     // the counter load first: a relaxed load issued after the acquire would wait
     // for it; this way both round trips (and the caller's rank lookup) overlap
@@ -364,6 +373,7 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     if (threadIdx.x == 0) c2 = ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(p.ctrl));
   };
 
+  pdl_wait();   // a PDL launch: the previous kernel on the stream has completed from here on
   c2 = c;
   uint32_t g = fetch(0, 0, 0);
   int slot = 0;
@@ -462,6 +472,7 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
       }
     }
   }
+  pdl_trigger();   // no more tasks for this CTA: the queue's next kernel may start launching
   if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
   if (threadIdx.x == 0 && my_blocks) {
     count_done(p, my_blocks, my_tasks);

@@ -277,6 +277,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   }
   __syncthreads();
   if (!H.go) return;
+  pdl_wait();   // a PDL launch: the previous kernel on the stream has completed from here on
 
   if (warp == kTaskWarp) {
     // ===================== task warp: the slate task protocol + row-pointer slices =====================
@@ -500,6 +501,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     }
 #endif
   }
+  pdl_trigger();   // no more tasks for this CTA: the queue's next kernel may start launching
   __syncthreads();
   if (warp == kTaskWarp) {
     if (lane == 0) atomicAdd(&p.tc->live_rank[H.rank], 0xffffffffu);   // live_rank -= 1
@@ -516,10 +518,11 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.standby_timeout_ns = w.standby_timeout_ns;
   p.base_epoch = w.base_epoch;
   p.is_topup = w.is_topup;
+  p.gate_first = w.gate_first;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
-  return cudaLaunchKernel(reinterpret_cast<const void*>(&spmv_worker), dim3(grid), dim3(kThreads), kargs, kSmemBytes,
-                          st);
+  return launch_kernel(reinterpret_cast<const void*>(&spmv_worker), dim3(grid), dim3(kThreads), kargs, kSmemBytes, st,
+                       w.pdl);
 }
 
 static cudaError_t launch_standalone(const void* args, dim3 grid, cudaStream_t st) {
@@ -547,6 +550,7 @@ KindOps spmv_ws_ops() {
   o.launch_worker = &spmv::launch_worker;
   o.launch_standalone = &spmv::launch_standalone;
   o.topup_anytime = true;   // leave_main: the last main CTA waits for every block
+  o.pdl_ok = true;          // griddepcontrol.wait before the first task
   return o;
 }
 

@@ -143,3 +143,37 @@ def test_gemm_shrink_latency(sess):
         assert q["blocks_done"] == q["total_blocks"]
         lats += q["resize_us"]
     assert lats and max(lats) < 200, lats
+
+
+def test_dependent_chain_with_topups(sess):
+    """Stream order under grows: a chain of triads where each launch reads the
+    previous one's output (ping-pong x <- x + 1), all queued at once on a
+    quarter of the SMs, then a storm of grows and shrinks.  A grow tops up the
+    RUNNING launch while the rest of the chain is queued behind it; its last
+    main CTA waits for the top-up's blocks before the kernel ends, so the next
+    launch reads finished data: the result must be exactly x0 + K."""
+    n_sms = sess.info()["num_sms"]
+    n, K = 1 << 25, 60
+    x0 = torch.arange(n, dtype=torch.float32, device="cuda:0") % 1000
+    bufs = [x0.clone(), torch.zeros(n, device="cuda:0")]
+    ones = torch.ones(n, device="cuda:0")
+    torch.cuda.synchronize()
+    k = sess.register_kernel(S.KIND_TRIAD, iters=2)
+    ids = []
+    for i in range(K):
+        args, grid = S.triad_args(bufs[(i + 1) % 2], bufs[i % 2], ones, 1.0)
+        ids.append(sess.launch(k, args, grid, placement=S.PLACE_CORUN, sm=(0, n_sms // 4 - 1)))
+    rng = random.Random(205)
+    for i in range(4000):
+        lo, hi = (0, n_sms - 1) if i % 2 == 0 else (0, rng.randrange(n_sms // 8, n_sms // 2))
+        if sess.resize(ids[-1], lo, hi) == S.DONE:
+            break
+        time.sleep(0.00015)
+    sess.sync(0)
+    torch.cuda.synchronize()
+    topups = sum(sess.query(i)["n_topups"] for i in ids)
+    for i in ids:
+        q = sess.query(i)
+        assert q["blocks_done"] == q["total_blocks"] and q["tasks_done"] == -(-q["total_blocks"] // 2)
+    assert torch.equal(bufs[K % 2], x0 + K)
+    assert topups >= 1, "no grow landed on a running launch"
