@@ -419,7 +419,7 @@ def resize_storm(S, sess, job, n_sms, n_resizes=200, per_launch=12, gap_us=100.0
     rng = random.Random(seed)
     k = sess.register_kernel(job.kind)
     lat = {"shrink": [], "grow": []}
-    issued = 0
+    issued = superseded = 0
     while issued < n_resizes:
         lid = sess.launch(k, job.args, job.grid, placement=S.PLACE_CORUN, sm=(0, n_sms - 1))
         spin_ms(0.05)
@@ -441,12 +441,14 @@ def resize_storm(S, sess, job, n_sms, n_resizes=200, per_launch=12, gap_us=100.0
         q = sess.query(lid)
         for v, kind in zip(q["resize_us"], q["resize_kind"]):
             lat[kind].append(v)
+        superseded += q["n_superseded"]
 
     def stats(v):
         return {"n": len(v), "p50": round(statistics.median(v), 2) if v else None,
                 "p99": round(float(np.percentile(v, 99)), 2) if v else None, "max": round(max(v), 2) if v else None}
     return {"tenant": "gemm_bf16 8192^3, one launch per %d resizes" % per_launch, "resizes_issued": issued,
             "gap_us": gap_us, "shrink_us": stats(lat["shrink"]), "grow_us": stats(lat["grow"]),
+            "shrinks_superseded": superseded,   # overtaken by the next grow before completing: not timed
             "clock": "device %globaltimer mapped to the host clock (DESIGN.md Q30)"}
 
 

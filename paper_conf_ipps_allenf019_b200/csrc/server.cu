@@ -1245,8 +1245,23 @@ int Server::resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string
 
 // a resize applied while R runs: measured (Q30) for the first 16 of the launch
 void Server::track_resize(Launch& R, uint32_t epoch, int kind, double t0) {
+  Queue& Q = *queues_[R.queue];
+  if (kind == 2) {
+    // a grow re-admits ranks: a shrink still pending was overtaken before it
+    // completed (its workers may now stay) -- it has no completion to time;
+    // counted apart (n_superseded), not as a latency
+    for (auto it = Q.pending_resize.begin(); it != Q.pending_resize.end();) {
+      if (it->kind == 1 && it->epoch < epoch) {
+        auto li = launches_.find(it->lid);
+        if (li != launches_.end()) li->second->n_superseded += 1;
+        it = Q.pending_resize.erase(it);
+      } else {
+        ++it;
+      }
+    }
+  }
   if (R.resize_us.size() >= 16) return;
-  queues_[R.queue]->pending_resize.push_back({epoch, kind, t0, R.id, int(R.resize_us.size())});
+  Q.pending_resize.push_back({epoch, kind, t0, R.id, int(R.resize_us.size())});
   R.resize_us.push_back(-1);
   R.resize_kind.push_back(uint8_t(kind));
 }
@@ -1497,6 +1512,7 @@ int Server::query(uint64_t l, slate_launch_info* out, std::string* err) {
     out->shrink_epoch = tc.shrink_epoch;
     out->join_epoch = tc.join_epoch;
     out->t_enter_ns = tc.t_enter;
+    out->n_superseded = L.n_superseded;
     out->t_exit_ns = tc.t_exit;
   }
   if (L.state == 2) {

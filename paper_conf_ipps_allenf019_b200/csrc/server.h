@@ -48,7 +48,7 @@ struct Launch {
   std::vector<cudaEvent_t> ev_done;   // all must complete (main + top-ups, after snapshots)
   int error = 0;                      // cudaError_t seen on completion
   bool mirror_complete_seen = false;
-  uint32_t n_resizes = 0, n_topups = 0;
+  uint32_t n_resizes = 0, n_topups = 0, n_superseded = 0;
   std::vector<double> resize_us;
   std::vector<uint8_t> resize_kind;   // 1 shrink, 2 grow
   unsigned char snapshot[kTaskCtlHeader];   // final TaskCtl header copy

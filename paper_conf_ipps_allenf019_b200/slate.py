@@ -118,7 +118,7 @@ class LaunchInfo(ctypes.Structure):
                 ("workers_started", c_u32), ("coverage_ok", c_u32), ("epoch", c_u32), ("shrink_epoch", c_u32),
                 ("join_epoch", c_u32), ("pad_", c_u32), ("t_first_ns", c_u64), ("t_last_ns", c_u64),
                 ("start_ms", c_f64), ("end_ms", c_f64), ("resize_us", c_f64 * 16), ("resize_kind", ctypes.c_uint8 * 16),
-                ("t_enter_ns", c_u64), ("t_exit_ns", c_u64)]
+                ("t_enter_ns", c_u64), ("t_exit_ns", c_u64), ("n_superseded", c_u32), ("pad2_", c_u32)]
 
     def as_dict(self):
         d = {f[0]: getattr(self, f[0]) for f in self._fields_}
