@@ -222,6 +222,18 @@ slate_status slate_launch(slate_session* s, slate_kernel k, const slate_launch_d
 slate_status slate_launch_n(slate_session* s, slate_kernel k, const slate_launch_desc* d, uint32_t n,
                             slate_launch_id* first);
 
+/* n (>= 1) launches of possibly different kernels and descriptors in one call,
+ * in order: ks[i] with ds[i].  A job whose launches differ (e.g. Gaussian
+ * elimination, a Fan1 and a Fan2 launch per step with the step in the args,
+ * Tab II GS) goes out as one batch: no event between its kernels and
+ * programmatic dependent launch, as slate_launch_n.  Stream order between the
+ * launches is kept (launch i+1 starts after launch i completed).  ks and ds are
+ * caller-owned arrays of n entries, read during the call.  The ids are
+ * *first .. *first + n - 1.  Through an endpoint the launches are sent one by
+ * one (same ids and order, no batch).  Errors: as slate_launch_n. */
+slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel* ks, const slate_launch_desc* ds,
+                               slate_launch_id* first);
+
 /* Resize the SM range of the queue that owns launch l to [sm_lo, sm_hi]
  * (§III-C; the dispatcher's start_sm/end_sm, Lst3 P:L250-251).
  * Publishes {epoch+1, lo, hi} to the device with a stream memory write that

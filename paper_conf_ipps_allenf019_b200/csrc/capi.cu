@@ -201,6 +201,24 @@ slate_status slate_launch_n(slate_session* s, slate_kernel k, const slate_launch
   return rc == SLATE_OK ? rc : fail(s, rc, err);
 }
 
+slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel* ks, const slate_launch_desc* ds,
+                               slate_launch_id* first) {
+  if (!s || !ks || !ds || !first || n == 0) return fail(s, SLATE_EINVAL, "null argument or n == 0");
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  int rc = SLATE_OK;
+  if (s->srv) {
+    rc = s->srv->launch_many(s->queue, n, ks, ds, first, &err);
+  } else {
+    for (uint32_t i = 0; i < n && rc == SLATE_OK; ++i) {
+      slate_launch_id id = 0;
+      rc = s->remote->launch(ks[i], &ds[i], &id, &err);
+      if (i == 0) *first = id;
+    }
+  }
+  return rc == SLATE_OK ? rc : fail(s, rc, err);
+}
+
 slate_status slate_resize(slate_session* s, slate_launch_id l, uint32_t lo, uint32_t hi) {
   if (!s) return SLATE_EINVAL;
   std::lock_guard<std::mutex> g(s->mu);

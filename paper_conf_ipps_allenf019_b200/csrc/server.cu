@@ -112,8 +112,10 @@ int Server::init(std::string* err) {
   std::memset(reinterpret_cast<void*>(h_mirror_), 0, sizeof(HostMirror) * kSlots);
   CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&d_mirror_), h_mirror_, 0));
   CK(cudaHostAlloc(reinterpret_cast<void**>(&h_snap_), kTaskCtlHeader * kSlots, cudaHostAllocDefault));
-  CK(cudaHostAlloc(&h_zero_, sizeof(TaskCtl), cudaHostAllocDefault));
-  std::memset(h_zero_, 0, sizeof(TaskCtl));
+  CK(cudaHostAlloc(&h_zero_, sizeof(TaskCtl) * kZeroRun, cudaHostAllocDefault));
+  std::memset(h_zero_, 0, sizeof(TaskCtl) * kZeroRun);
+  zero_ev_.resize(kZeroEv);
+  for (auto& e : zero_ev_) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
   for (int i = 0; i < kSlots; ++i) free_slots_.push_back(i);
   slot_zeroed_.assign(kSlots, nullptr);
   CK(cudaMalloc(&d_ctrl_pool_, 128 * kQueues));
@@ -545,20 +547,42 @@ int Server::alloc_slot() {
 
 // a freed control block is zeroed by DMA on the copy stream right away, so the
 // next launch that takes the slot only waits on an (already complete) event
-void Server::free_slot(int slot) {
-  cudaMemcpyAsync(d_tc_ + slot, h_zero_, sizeof(TaskCtl), cudaMemcpyHostToDevice, copy_stream_);
-  if (!slot_zeroed_[slot]) cudaEventCreateWithFlags(&slot_zeroed_[slot], cudaEventDisableTiming);
-  cudaEventRecord(slot_zeroed_[slot], copy_stream_);
-  free_slots_.push_back(slot);
+void Server::free_slot(int slot) { pending_free_.push_back(slot); }
+
+// Zero the control blocks freed since the last flush by DMA, one copy per run
+// of consecutive slots (a batch's launches hold consecutive slots: a job of
+// 8190 launches is ~32 copies, not 8190).  A slot's event is its run's, from
+// a round-robin pool: an event re-recorded later only makes a waiter wait
+// longer (the copy stream is in order).
+void Server::flush_free() {
+  if (pending_free_.empty()) return;
+  std::sort(pending_free_.begin(), pending_free_.end());
+  size_t i = 0;
+  while (i < pending_free_.size()) {
+    size_t j = i + 1;
+    while (j < pending_free_.size() && pending_free_[j] == pending_free_[j - 1] + 1 && int(j - i) < kZeroRun) ++j;
+    const int s0 = pending_free_[i], len = int(j - i);
+    cudaMemcpyAsync(d_tc_ + s0, h_zero_, sizeof(TaskCtl) * len, cudaMemcpyHostToDevice, copy_stream_);
+    cudaEvent_t e = zero_ev_[zero_ev_next_++ % kZeroEv];
+    cudaEventRecord(e, copy_stream_);
+    for (size_t k = i; k < j; ++k) {
+      slot_zeroed_[pending_free_[k]] = e;
+      free_slots_.push_back(pending_free_[k]);
+    }
+    i = j;
+  }
+  pending_free_.clear();
 }
 
 // one wave of workers (Q12) -- but no more CTAs than there are tasks,
 // and at least one per SM (so any SM range gets workers): every worker CTA
 // costs its launch a prologue and a fetch (tools/probe/launch_cost.cu)
-uint32_t Server::worker_grid(int occ, uint32_t B, uint32_t iters) const {
+uint32_t Server::worker_grid(int occ, uint32_t B, uint32_t iters, bool full_range) const {
   const uint64_t wave = uint64_t(occ) * uint64_t(n_sms_);
   const uint64_t tasks = (uint64_t(B) + iters - 1) / iters;
-  return uint32_t(std::min<uint64_t>(wave, std::max<uint64_t>(uint64_t(n_sms_), tasks)));
+  // on the whole chip any SM will do: one CTA per task suffices (a 6-block
+  // Gaussian-elimination step gets 6 CTAs, not 148)
+  return uint32_t(std::min<uint64_t>(wave, full_range ? tasks : std::max<uint64_t>(uint64_t(n_sms_), tasks)));
 }
 
 // reading Q11: the paper's default task of 10 blocks, reduced so every
@@ -631,9 +655,15 @@ void Server::close_batch(Queue& Q, cudaEvent_t end, bool closed_by_launch) {
     cudaEvent_t snap;
     cudaEventCreateWithFlags(&snap, cudaEventDisableTiming);
     cudaStreamWaitEvent(copy_stream_, end, 0);
-    for (Launch* M : ws)
-      cudaMemcpyAsync(h_snap_ + size_t(M->slot) * kTaskCtlHeader, d_tc_ + M->slot, kTaskCtlHeader,
-                      cudaMemcpyDeviceToHost, copy_stream_);
+    // one strided copy per run of consecutive slots (headers out of 2.5-KB blocks)
+    for (size_t i = 0; i < ws.size();) {
+      size_t j = i + 1;
+      while (j < ws.size() && ws[j]->slot == ws[j - 1]->slot + 1) ++j;
+      const int s0 = ws[i]->slot;
+      cudaMemcpy2DAsync(h_snap_ + size_t(s0) * kTaskCtlHeader, kTaskCtlHeader, d_tc_ + s0, sizeof(TaskCtl),
+                        kTaskCtlHeader, j - i, cudaMemcpyDeviceToHost, copy_stream_);
+      i = j;
+    }
     cudaEventRecord(snap, copy_stream_);
     for (Launch* M : ws) M->ev_done.push_back(snap);
   }
@@ -724,7 +754,8 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     w.rank_of = d_rank_of_;
     // PDL: the previous op on the stream is the previous worker of this batch
     w.pdl = in_batch && Q.last_op_kernel && ops->pdl_ok && pdl_enabled_;
-    CK(ops->launch_worker(w, L.args.data(), worker_grid(L.k->occ, L.B, L.iters), Q.stream));
+    const bool full = Q.lo == 0 && Q.hi == uint32_t(n_sms_ - 1);
+    CK(ops->launch_worker(w, L.args.data(), worker_grid(L.k->occ, L.B, L.iters, full), Q.stream));
     Q.last_op_kernel = ops->pdl_ok;
     if (ev_end) {
       CK(cudaEventRecord(ev_end, Q.stream));
@@ -861,6 +892,27 @@ int Server::launch_n(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint3
     uint64_t id = 0;
     batch_more_ = i + 1 < n;   // the job's launches go out as one batch if the queue can take them now
     rc = launch_locked(q, kid, d, &id, err, i + 1 < n);
+    if (i == 0) *first = id;
+  }
+  batch_more_ = false;
+  auto qi = queues_.find(q);
+  if (qi != queues_.end()) close_batch(*qi->second, nullptr);
+  return rc;
+}
+
+// n launches of different kernels/descriptors in one call, issued as one batch
+int Server::launch_many(uint32_t q, uint32_t n, const uint64_t* ks, const slate_launch_desc* ds, uint64_t* first,
+                        std::string* err) {
+  if (n == 0) {
+    if (err) *err = "n == 0";
+    return SLATE_EINVAL;
+  }
+  std::unique_lock<std::mutex> g(mu_);
+  int rc = SLATE_OK;
+  for (uint32_t i = 0; i < n && rc == SLATE_OK; ++i) {
+    uint64_t id = 0;
+    batch_more_ = i + 1 < n;
+    rc = launch_locked(q, ks[i], &ds[i], &id, err, i + 1 < n);
     if (i == 0) *first = id;
   }
   batch_more_ = false;
@@ -1371,6 +1423,7 @@ void Server::poll_once() {
     drain_deferred(Q);
     if (Q.active && Q.issued.empty() && Q.pending.empty() && Q.deferred.empty()) idle.push_back(Q.id);
   }
+  flush_free();
   for (uint32_t q : idle) release(*queues_[q]);
 }
 
@@ -1576,7 +1629,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     for (int i = 0; i < kBatch; ++i) {
       w.tc = d_tc_ + slots[i];
       w.pdl = i > 0 && k.ops->pdl_ok && pdl_enabled_;
-      CK(k.ops->launch_worker(w, d->args, worker_grid(k.occ, B, w.iters), st));
+      CK(k.ops->launch_worker(w, d->args, worker_grid(k.occ, B, w.iters, lo == 0 && hi == uint32_t(n_sms_ - 1)), st));
     }
     CK(cudaEventRecord(e1, st));
     CK(cudaEventSynchronize(e1));
@@ -1591,6 +1644,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   cudaStreamDestroy(st);
   std::lock_guard<std::mutex> g(mu_);
   for (int sl : slots) free_slot(sl);
+  flush_free();
   free_ctrl_.push_back(int((ctrl - d_ctrl_pool_) / 16));
   return SLATE_OK;
 }

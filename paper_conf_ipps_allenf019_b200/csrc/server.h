@@ -105,6 +105,8 @@ class Server {
   int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
   int launch(uint32_t q, uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err);
   int launch_n(uint32_t q, uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err);
+  int launch_many(uint32_t q, uint32_t n, const uint64_t* ks, const slate_launch_desc* ds, uint64_t* first,
+                  std::string* err);
   int resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
   int set_policy(uint32_t policy, std::string* err);
   int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);
@@ -162,7 +164,7 @@ class Server {
   int alloc_slot();
   void free_slot(int slot);
   uint32_t auto_iters(uint32_t B, int occ, uint32_t cap, uint32_t per_worker) const;
-  uint32_t worker_grid(int occ, uint32_t B, uint32_t iters) const;
+  uint32_t worker_grid(int occ, uint32_t B, uint32_t iters, bool full_range) const;
   bool validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const;
   void work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const;
 
@@ -176,12 +178,18 @@ class Server {
   void* write_value64_ = nullptr;   // cuStreamWriteValue64 (driver entry point)
 
   // pools
-  static constexpr int kSlots = 4096;
+  static constexpr int kSlots = 16384;   // control blocks: a Gaussian elimination at n = 4096 is 8190 launches in one batch
   TaskCtl* d_tc_ = nullptr;
   HostMirror* h_mirror_ = nullptr;
   HostMirror* d_mirror_ = nullptr;
   unsigned char* h_snap_ = nullptr;   // pinned, kSlots * kTaskCtlHeader
-  void* h_zero_ = nullptr;            // pinned zeros (TaskCtl reset by DMA, no SM)
+  void* h_zero_ = nullptr;            // pinned zeros (TaskCtl reset by DMA, no SM), kZeroRun blocks
+  static constexpr int kZeroRun = 256;   // control blocks zeroed by one copy
+  static constexpr int kZeroEv = 1024;   // events marking zeroing copies (round robin)
+  std::vector<cudaEvent_t> zero_ev_;
+  uint32_t zero_ev_next_ = 0;
+  std::vector<int> pending_free_;     // freed this poll, zeroed together by flush_free()
+  void flush_free();
   std::deque<int> free_slots_;     // FIFO: a freed block is reused as late as possible
   std::vector<cudaEvent_t> slot_zeroed_;   // DMA zeroing of a freed slot, off the critical path
   static constexpr int kQueues = 64;

@@ -150,6 +150,7 @@ for _name, _args in [
     ("slate_kind_geometry", [c_u32, _P(c_u32), _P(c_u32)]),
     ("slate_set_policy", [ctypes.c_void_p, c_u32]),
     ("slate_launch_n", [ctypes.c_void_p, c_u64, _P(LaunchDesc), c_u32, _P(c_u64)]),
+    ("slate_launch_many", [ctypes.c_void_p, c_u32, _P(c_u64), _P(LaunchDesc), _P(c_u64)]),
 ]:
     getattr(_lib, _name).restype = c_i32
     getattr(_lib, _name).argtypes = _args
@@ -173,7 +174,7 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
-            "slate_fluid_corun", "slate_set_policy", "slate_launch_n"]
+            "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -265,6 +266,17 @@ class Session:
         d = self._desc(args, grid, placement, sm, mode, coverage)
         first = c_u64()
         self._check(_lib.slate_launch_n(self._h, kernel, ctypes.byref(d), n, ctypes.byref(first)), "slate_launch_n")
+        return list(range(first.value, first.value + n))
+
+    def launch_many(self, items, placement=PLACE_AUTO, sm=None, mode=MODE_SLATE):
+        """Launches [(kernel, args, grid), ...] in order as one job (one batch); returns their ids."""
+        n = len(items)
+        ks = (c_u64 * n)(*[k for k, _, _ in items])
+        ds = (LaunchDesc * n)()
+        for i, (_, args, grid) in enumerate(items):
+            ds[i] = self._desc(args, grid, placement, sm, mode)
+        first = c_u64()
+        self._check(_lib.slate_launch_many(self._h, n, ks, ds, ctypes.byref(first)), "slate_launch_many")
         return list(range(first.value, first.value + n))
 
     def resize(self, launch_id, lo, hi):

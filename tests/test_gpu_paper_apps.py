@@ -28,7 +28,7 @@ def sess():
     s.close()
 
 
-def _eliminate(sess, a0, b0, mode, iters=0, placement=S.PLACE_AUTO, sm=None):
+def _eliminate(sess, a0, b0, mode, iters=0, placement=S.PLACE_AUTO, sm=None, many=False):
     n = a0.shape[0]
     a = torch.from_numpy(a0).to(DEV)
     b = torch.from_numpy(b0).to(DEV)
@@ -36,12 +36,14 @@ def _eliminate(sess, a0, b0, mode, iters=0, placement=S.PLACE_AUTO, sm=None):
     torch.cuda.synchronize()
     k1 = sess.register_kernel(S.KIND_GAUSS_FAN1, iters=iters)
     k2 = sess.register_kernel(S.KIND_GAUSS_FAN2, iters=iters)
-    ids = []
+    ids, items = [], []
     for t in range(n - 1):
-        args, grid = S.gauss_fan1_args(a, b, m, t)
-        ids.append(sess.launch(k1, args, grid, placement=placement, sm=sm, mode=mode))
-        args, grid = S.gauss_fan2_args(a, b, m, t)
-        ids.append(sess.launch(k2, args, grid, placement=placement, sm=sm, mode=mode))
+        items.append((k1,) + S.gauss_fan1_args(a, b, m, t))
+        items.append((k2,) + S.gauss_fan2_args(a, b, m, t))
+    if many:    # one slate_launch_many call: one batch (no events between kernels, PDL)
+        ids = sess.launch_many(items, placement=placement, sm=sm, mode=mode)
+    else:
+        ids = [sess.launch(k, args, grid, placement=placement, sm=sm, mode=mode) for k, args, grid in items]
     sess.sync(0)
     torch.cuda.synchronize()
     for i in ids[-4:]:
@@ -50,11 +52,11 @@ def _eliminate(sess, a0, b0, mode, iters=0, placement=S.PLACE_AUTO, sm=None):
     return a.cpu().numpy(), b.cpu().numpy(), m.cpu().numpy()
 
 
-@pytest.mark.parametrize("n,iters", [(256, 0), (129, 1)])
-def test_gaussian_int_exact(sess, n, iters):
+@pytest.mark.parametrize("n,iters,many", [(256, 0, False), (129, 1, False), (300, 0, True)])
+def test_gaussian_int_exact(sess, n, iters, many):
     a0, b0 = I.gauss_inputs(n, 140 + n, mode="int")
     ra, rb, rm = OT.gaussian(a0, b0)
-    ga, gb, gm = _eliminate(sess, a0, b0, S.MODE_SLATE, iters=iters)
+    ga, gb, gm = _eliminate(sess, a0, b0, S.MODE_SLATE, iters=iters, many=many)
     assert np.array_equal(ga.astype(np.float64), ra)
     assert np.array_equal(gb.astype(np.float64), rb)
     assert np.array_equal(gm.astype(np.float64), rm)
@@ -64,8 +66,8 @@ def test_gaussian_rodinia_matrix(sess):
     n = 384
     a0, b0 = I.gauss_inputs(n)
     ra, rb, rm = OT.gaussian(a0, b0)
-    ga, gb, gm = _eliminate(sess, a0, b0, S.MODE_SLATE)
-    sa, sb, sm_ = _eliminate(sess, a0, b0, S.MODE_STANDALONE)
+    ga, gb, gm = _eliminate(sess, a0, b0, S.MODE_SLATE, many=True)
+    sa, sb, sm_ = _eliminate(sess, a0, b0, S.MODE_STANDALONE, many=True)
     assert np.array_equal(ga, sa) and np.array_equal(gb, sb) and np.array_equal(gm, sm_)
     tol = 4 * n * 2.0 ** -24 * float(np.abs(a0).max())
     assert np.abs(np.triu(ga).astype(np.float64) - np.triu(ra)).max() <= tol

@@ -109,7 +109,8 @@ class App:
         if len(self.launches) == 1:
             ki, args, grid = self.launches[0]
             return sess.launch_n(ks[ki], args, grid, self.reps, **kw)
-        return [sess.launch(ks[ki], args, grid, **kw) for ki, args, grid in self.launches]
+        # GS: the elimination's 2(n-1) launches in one call (one batch)
+        return sess.launch_many([(ks[ki], args, grid) for ki, args, grid in self.launches], **kw)
 
     def profile(self, sess, ks):
         # the representative (largest) launch: the job's first Fan2 for GS
