@@ -372,6 +372,12 @@ uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t 
  * gains little bandwidth but raises the HBM latency its compute-bound partner
  * sees. */
 uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n, uint32_t n_sms, double frac);
+/* NEXT-4, the task size from a solo profile: a
+ * worker's time per block is t = solo_ms * occ * n_sms / B; the task takes
+ * floor(budget_us / t) blocks, at most floor(B / (2 occ n_sms)) (every worker
+ * gets two tasks), clamped to [1, cap].  The server uses it for launches of
+ * kernels registered with iters 0 once their shape has been profiled. */
+uint32_t slate_choose_iters(double solo_ms, uint32_t occ, uint32_t n_sms, uint32_t B, uint32_t cap, double budget_us);
 /* Reading Q31 (the B200 selector): should kernel B co-run with the active A
  * although Tab I says solo?  Job curves are `work` launches of each kernel
  * (the launches queued or running) back to back, time = work * curve(s); the

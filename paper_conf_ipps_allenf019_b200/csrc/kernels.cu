@@ -43,6 +43,14 @@ cudaError_t launch_standalone_t(const void* args, dim3 grid, cudaStream_t st) {
                           Tn::kSmemStandalone, st);
 }
 
+// Black-Scholes: the few-scenario worker (task-level body) or the
+// many-scenario one, per launch; same occupancy (64 registers, 4 CTAs/SM)
+cudaError_t launch_worker_bs(const WorkerCommon& w, const void* args, uint32_t grid, cudaStream_t st) {
+  const slate_args_bs* a = static_cast<const slate_args_bs*>(args);
+  return a->n_scen <= BlackScholesShort::kPipelineMaxScen ? launch_worker_t<BlackScholesShort>(w, args, grid, st)
+                                                           : launch_worker_t<BlackScholes>(w, args, grid, st);
+}
+
 template <class Tn>
 KindOps make_ops(uint32_t default_iters) {
   KindOps o;
@@ -73,6 +81,7 @@ const KindOps* kind_ops(uint32_t kind) {
     table[SLATE_KIND_SGEMM_NAIVE] = make_ops<SgemmNaive>(0);
     table[SLATE_KIND_SPMV_CSR] = spmv_ws_ops();
     table[SLATE_KIND_BLACKSCHOLES] = make_ops<BlackScholes>(0);
+    table[SLATE_KIND_BLACKSCHOLES].launch_worker = &launch_worker_bs;
     table[SLATE_KIND_STENCIL2D] = make_ops<Stencil2D>(0);
     table[SLATE_KIND_GEMM_BF16] = gemm_tc_ops();
     table[SLATE_KIND_TRANSPOSE] = make_ops<Transpose>(0);

@@ -122,4 +122,12 @@ int slate_fluid_corun(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, d
   return g >= min_gain ? 1 : 0;
 }
 
+uint32_t slate_choose_iters(double solo_ms, uint32_t occ, uint32_t n_sms, uint32_t B, uint32_t cap, double budget_us) {
+  if (B == 0 || occ == 0 || n_sms == 0) return 1;
+  const double workers = double(occ) * n_sms;
+  const double t_block_us = std::max(solo_ms * 1e3 * workers / B, 1e-3);
+  const double it = std::min(std::floor(budget_us / t_block_us), std::floor(B / (2.0 * workers)));
+  return uint32_t(std::max(1.0, std::min(double(cap ? cap : 1), it)));
+}
+
 }  // extern "C"

@@ -144,6 +144,7 @@ int Server::init(std::string* err) {
   }
   {
     pdl_enabled_ = env_double("SLATE_PDL", 1.0) != 0.0;
+    task_budget_us_ = env_double("SLATE_TASK_BUDGET_US", 20.0);
   }
   min_gain_ = env_double("SLATE_MIN_GAIN", 1.05);
   poller_ = std::thread([this] { poller_main(); });
@@ -953,7 +954,7 @@ int Server::launch_locked(uint32_t q, uint64_t kid, const slate_launch_desc* d, 
   L->args.assign(static_cast<const unsigned char*>(d->args), static_cast<const unsigned char*>(d->args) + d->args_size);
   L->desc.args = nullptr;
   L->B = B;
-  L->iters = k.desc.iters ? k.desc.iters : auto_iters(B, k.occ, k.ops->max_auto_iters, k.ops->tasks_per_worker);
+  L->iters = k.desc.iters ? k.desc.iters : choose_iters(k, d, B);
   Launch& LL = *L;
   launches_[L->id] = std::move(L);
   *out = LL.id;
@@ -1035,6 +1036,20 @@ int Server::category_of(const Launch& L) const {
 static const slate_profile_t* find_profile(const std::map<std::string, ProfileEntry>& t, const std::string& key) {
   auto it = t.find(key);
   return it == t.end() ? nullptr : &it->second.p;
+}
+
+// NEXT-4 (the task size trades scheduling overhead
+// against imbalance and reaction time).  With a solo profile of the launch's
+// kernel and shape, a worker's time per block is t = T_solo * workers / B;
+// the task takes as many blocks as fit a budget (SLATE_TASK_BUDGET_US, default
+// 20 us: a resize is honoured within two tasks, reading Q23, inside the 50-us
+// target), at least one, at most the kind's cap, and leaves every worker at
+// least two tasks.  Without a profile: the occupancy rule (auto_iters, Q11).
+uint32_t Server::choose_iters(const KernelEntry& k, const slate_launch_desc* d, uint32_t B) const {
+  const uint32_t cap = k.ops->max_auto_iters;
+  const slate_profile_t* p = find_profile(profiles_, profile_key(k, d));
+  if (!p || p->solo_ms <= 0) return auto_iters(B, k.occ, cap, k.ops->tasks_per_worker);
+  return slate_choose_iters(p->solo_ms, uint32_t(k.occ), uint32_t(n_sms_), B, cap, task_budget_us_);
 }
 
 int Server::set_policy(uint32_t policy, std::string* err) {

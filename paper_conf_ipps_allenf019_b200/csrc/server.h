@@ -165,6 +165,8 @@ class Server {
   void free_slot(int slot);
   uint32_t auto_iters(uint32_t B, int occ, uint32_t cap, uint32_t per_worker) const;
   uint32_t worker_grid(int occ, uint32_t B, uint32_t iters, bool full_range) const;
+  uint32_t choose_iters(const KernelEntry& k, const slate_launch_desc* d, uint32_t B) const;
+  double task_budget_us_ = 20.0;
   bool validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const;
   void work(const KernelEntry& k, const slate_launch_desc* d, double* bytes, double* fp32, double* tc) const;
 

@@ -415,6 +415,63 @@ struct BlackScholes : TenantBase {
   }
 };
 
+// The Black-Scholes worker for launches with few scenarios (<= 4; the Tab II
+// BS is P = 1): same blocks and arithmetic, plus a task-level body.  A separate
+// kernel, chosen per launch by the server (kernels.cu), so the many-scenario
+// worker (C2's P = 32, compute-bound) keeps its own code and registers.
+struct BlackScholesShort : BlackScholes {
+  static constexpr bool kLateCtrl = false;   // blocks of a few us: the word is read when the task starts
+  // Task-level body: with few scenarios a block is a few us of HBM traffic,
+  // so the next block's S, X, T are copied into shared memory (cp.async, no
+  // extra registers) while this block is priced -- the original kernel hides
+  // its loads behind other CTAs, the worker runs its task's blocks back to
+  // back.  Each thread reads only the 48 bytes it copied, so no barrier is
+  // needed.  A task reaching the ragged last block takes the per-block path.
+  // Each option's arithmetic is price<4>'s (measured: a P = 1 launch of 2^23
+  // options 54 -> 46 us at 4 blocks per task).
+  static constexpr bool kHasTask = true;
+  static constexpr uint32_t kPipelineMaxScen = 4;
+  static constexpr int kSmem = 2 * 3 * 256 * 16;   // two cp.async stages
+  static constexpr int kStageBytes = 3 * 256 * 16;   // S, X, T float4 of 256 threads
+  __device__ __forceinline__ static void stage_in(const Args& a, uint64_t v, char* stage) {
+    const char* src[3] = {reinterpret_cast<const char*>(a.S), reinterpret_cast<const char*>(a.X),
+                          reinterpret_cast<const char*>(a.T)};
+#pragma unroll
+    for (int q = 0; q < 3; ++q)
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(stage + (q * 256 + threadIdx.x) * 16)),
+                   "l"(src[q] + v * 16)
+                   : "memory");
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  }
+  __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char* smem) {
+    const uint64_t n_full = a.n / 1024;            // blocks with 1024 options (no ragged tail)
+    if (g + n > n_full) {
+      for (uint32_t i = 0; i < n; ++i) cta_block(a, g + i, 0, 0, smem);
+      return;
+    }
+    const float* sig = reinterpret_cast<const float*>(a.sigmas);
+    uint64_t v = uint64_t(g) * 256 + threadIdx.x;
+    stage_in(a, v, smem);
+    for (uint32_t i = 0; i < n; ++i) {
+      const uint64_t cur = v;
+      if (i + 1 < n) {
+        v += 256;
+        stage_in(a, v, smem + ((i + 1) & 1) * kStageBytes);    // next block in flight
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+      }
+      const float4* st = reinterpret_cast<const float4*>(smem + (i & 1) * kStageBytes);
+      const float4 s4 = st[threadIdx.x], x4 = st[256 + threadIdx.x], t4 = st[512 + threadIdx.x];
+      float S[4] = {s4.x, s4.y, s4.z, s4.w}, X[4] = {x4.x, x4.y, x4.z, x4.w}, T[4] = {t4.x, t4.y, t4.z, t4.w};
+      float c[4], p[4];
+      price<4>(S, X, T, a.r, sig, a.n_scen, c, p);
+      __stcs(reinterpret_cast<float4*>(a.call) + cur, make_float4(c[0], c[1], c[2], c[3]));
+      __stcs(reinterpret_cast<float4*>(a.put) + cur, make_float4(p[0], p[1], p[2], p[3]));
+    }
+  }
+};
+
 // ============================================================== 2-D 5-point stencil
 // One Jacobi sweep of an h x w field; 32 x 8 points per block.  Each thread
 // owns one point; the up/down neighbours come from the rows above/below
@@ -463,7 +520,49 @@ struct Transpose : TenantBase {
   static constexpr bool kSpeculative = SLATE_SPEC_SHORT;
   static constexpr int kThreads = 256;        // 32 x 8
   static constexpr int kMinBlocks = 8;
-  static constexpr int kSmem = 32 * 33 * 4, kSmemStandalone = 32 * 33 * 4;
+  static constexpr int kSmem = 2 * 32 * 33 * 4, kSmemStandalone = 32 * 33 * 4;
+  static constexpr bool kHasTask = true;
+
+  __device__ __forceinline__ static void load(const Args& a, uint32_t bx, uint32_t by, float (&v)[4]) {
+    const float* in = reinterpret_cast<const float*>(a.in);
+    const uint32_t tx = threadIdx.x & 31, ty = threadIdx.x >> 5, c = bx * 32 + tx;
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      const uint32_t row = by * 32 + ty + 8 * r;
+      v[r] = (row < a.h && c < a.w) ? __ldcs(in + uint64_t(row) * a.w + c) : 0.f;
+    }
+  }
+  // The task's blocks as one pipeline (the worker's task-level body): the
+  // next tile's loads are in flight while this tile's transposed stores go
+  // out, two shared-memory tiles alternate, one barrier per block (measured:
+  // 138 -> 125 us per 8192^2 launch; a 3-stage cp.async ring was slower, 132).
+  // Every element moves exactly as in cta_block.
+  __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char* smem) {
+    float* out = reinterpret_cast<float*>(a.out);
+    const uint32_t gx = (a.w + 31) / 32;
+    const uint32_t tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    float v[4];
+    uint32_t bx = g % gx, by = g / gx;
+    load(a, bx, by, v);
+    for (uint32_t k = 0; k < n; ++k) {
+      float (*tile)[33] = reinterpret_cast<float (*)[33]>(smem + (k & 1) * (32 * 33 * 4));
+#pragma unroll
+      for (int r = 0; r < 4; ++r) tile[ty + 8 * r][tx] = v[r];
+      __syncthreads();
+      const uint32_t cbx = bx, cby = by;
+      if (k + 1 < n) {
+        if (++bx == gx) { bx = 0; ++by; }
+        load(a, bx, by, v);                      // in flight during the stores below
+      }
+      const uint32_t i = cby * 32 + tx;
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {
+        const uint32_t j = cbx * 32 + ty + 8 * r;
+        if (j < a.w && i < a.h) __stcs(out + uint64_t(j) * a.h + i, tile[tx][ty + 8 * r]);
+      }
+    }
+    __syncthreads();                             // the tiles are reused by the worker's next task
+  }
 
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t bx, uint32_t by, uint32_t, char* smem) {
     float (*tile)[33] = reinterpret_cast<float (*)[33]>(smem);

@@ -165,6 +165,8 @@ _lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c
                                     c_u32, _P(c_f64)]
 _lib.slate_saturation_sms.restype = c_u32
 _lib.slate_saturation_sms.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_u32, c_f64]
+_lib.slate_choose_iters.restype = c_u32
+_lib.slate_choose_iters.argtypes = [c_f64, c_u32, c_u32, c_u32, c_u32, c_f64]
 _lib.slate_fluid_corun.restype = ctypes.c_int
 _lib.slate_fluid_corun.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_f64, _P(c_u32), _P(c_f64), c_u32, c_f64, c_u32,
                                    c_u32, c_u32, c_u32, c_f64, _P(c_u32), _P(c_f64)]
@@ -174,7 +176,7 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
-            "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many"]
+            "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -340,6 +342,10 @@ def fluid_corun(curve_a, work_a, curve_b, work_b, n_sms, step=2, lo_b=0, hi_b=0,
     r = _lib.slate_fluid_corun(sa, ta, na, work_a, sb, tb, nb, work_b, n_sms, step, lo_b, hi_b, min_gain,
                                ctypes.byref(s), ctypes.byref(g))
     return bool(r), s.value, g.value
+
+
+def choose_iters(solo_ms, occ, n_sms, blocks, cap, budget_us=20.0):
+    return _lib.slate_choose_iters(solo_ms, occ, n_sms, blocks, cap, budget_us)
 
 
 def saturation_sms(curve, n_sms, frac=0.9):

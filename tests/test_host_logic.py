@@ -125,3 +125,19 @@ def test_kind_geometry(S):
     assert (tm, tn) == (256, 256)          # one CTA-pair tile per original block
     with pytest.raises(S.SlateError):
         S.kind_geometry(99)
+
+
+def test_choose_iters_closed_forms(S):
+    """NEXT-4 task size: budget / (T_solo * workers / B), capped by two tasks per
+    worker and by the kind's cap, at least 1."""
+    # Black-Scholes P = 1 on B200: 65.5 us, 4 x 148 workers, 8192 blocks -> 4.73 us per block -> 4
+    assert S.choose_iters(0.0655, 4, 148, 8192, 10, 20.0) == 4
+    # P = 32: 25 us per block, over the budget -> 1
+    assert S.choose_iters(0.349, 4, 148, 8192, 10, 20.0) == 1
+    # tiny blocks: the balance bound (two tasks per worker) or the cap decides
+    assert S.choose_iters(0.001, 8, 148, 65536, 10, 20.0) == 10
+    assert S.choose_iters(0.001, 8, 148, 4736, 10, 20.0) == 2
+    # fewer blocks than workers: 1
+    assert S.choose_iters(0.5, 8, 148, 100, 10, 20.0) == 1
+    # a longer budget buys longer tasks, linearly
+    assert S.choose_iters(0.0655, 4, 148, 8192, 10, 40.0) == 6
