@@ -620,7 +620,13 @@ def run_slate(args, world, rank, local):
         for k, v in w2.pinned.items():
             w2._keep[k].copy_(v, non_blocking=True)
         torch.cuda.synchronize()
-        run_schedule("slate", w2, sA, sB, kA, kB, S)
+        # what a user does: submit both jobs (AUTO placement), wait for them; no
+        # per-launch queries (run_schedule's timing reads) in this region
+        submit(sA, kA, w2.a, placement=S.PLACE_AUTO)
+        spin_ms(w2.arrival_ms)
+        submit(sB, kB, w2.b, placement=S.PLACE_AUTO)
+        sA.sync(0)
+        sB.sync(0)
         for k in w2.out_names:
             w2.out_pinned[k].copy_(w2._keep[k], non_blocking=True)
         torch.cuda.synchronize()

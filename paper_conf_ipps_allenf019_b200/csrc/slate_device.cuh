@@ -87,9 +87,13 @@ struct WorkerParams {
 };
 
 // programmatic dependent launch: wait for the previous kernel on the stream
-// (no-op for a normal launch); let the next one start launching its CTAs
+// (no-op for a normal launch).  The workers never trigger their dependents
+// early (griddepcontrol.launch_dependents): a CTA's exit is the trigger, so the
+// next grid's CTAs take SM slots only once every CTA of this grid has left --
+// the last main CTA waits for a top-up grid's blocks (leave_main), and an
+// early trigger let the next grid's waiting CTAs take the slots that top-up
+// needed (one C4 run stalled 320 ms that way).
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
-__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // ------------------------------------------------------------------ decode (Lst2 (4))
 struct BlockWalk {
@@ -472,7 +476,6 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
       }
     }
   }
-  pdl_trigger();   // no more tasks for this CTA: the queue's next kernel may start launching
   if constexpr (Tn::kHasFini) Tn::cta_fini(dyn_smem);
   if (threadIdx.x == 0 && my_blocks) {
     count_done(p, my_blocks, my_tasks);

@@ -501,7 +501,6 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     }
 #endif
   }
-  pdl_trigger();   // no more tasks for this CTA: the queue's next kernel may start launching
   __syncthreads();
   if (warp == kTaskWarp) {
     if (lane == 0) atomicAdd(&p.tc->live_rank[H.rank], 0xffffffffu);   // live_rank -= 1
