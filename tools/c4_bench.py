@@ -75,8 +75,13 @@ def client(endpoint, kind, steps, go_path):
         ids = [s.launch(kid, args, grid, placement=S.PLACE_AUTO) for _ in range(JOBS[kind])]
         s.sync(0)
         qs = [s.query(i) for i in ids]
+        slow = sorted(qs, key=lambda q: q["start_ms"] - q["end_ms"])[:3]   # the longest launches (diagnostics)
         out.append([min(q["start_ms"] for q in qs), max(q["end_ms"] for q in qs),
-                    sum(len(q["resize_us"]) for q in qs), [v for q in qs for v in q["resize_us"]]])
+                    sum(len(q["resize_us"]) for q in qs), [v for q in qs for v in q["resize_us"]],
+                    [{"ms": round(q["end_ms"] - q["start_ms"], 3), "start": round(q["start_ms"], 3),
+                      "workers": q["workers_started"], "topups": q["n_topups"], "resizes": q["n_resizes"],
+                      "iters": q["iters"], "sm": [q["sm_lo"], q["sm_hi"]]} for q in slow]])
+        open("%s.%d.%s" % (go_path, step, kind), "w").close()   # this client is ready for the next step
     print("RESULT " + json.dumps(out), flush=True)
     s.close()
 
@@ -144,9 +149,15 @@ def main():
                               stdout=subprocess.PIPE, text=True) for k in JOBS}
     for p in ps.values():
         assert "READY" in p.stdout.readline()
+    # a step is released once every client finished reading the previous one
+    # (the SpMV client's 256 per-launch queries once overran a fixed 0.3-s gap,
+    # so its next job started up to 0.5 s late and the step's span measured that)
     for step in range(a.steps):
+        if step:
+            while not all(os.path.exists("%s.%d.%s" % (go, step - 1, k)) for k in JOBS):
+                time.sleep(0.001)
+            time.sleep(0.05)
         open("%s.%d" % (go, step), "w").close()
-        time.sleep(0.3)
     res = {}
     for k, p in ps.items():
         out, _ = p.communicate(timeout=600)
@@ -155,6 +166,8 @@ def main():
     d.wait(timeout=30)
     for step in range(a.steps):
         os.unlink("%s.%d" % (go, step))
+        for k in JOBS:
+            os.unlink("%s.%d.%s" % (go, step, k))
     spans, stps, resize = [], [], []
     for step in range(a.steps):
         t0 = min(res[k][step][0] for k in JOBS)
@@ -165,6 +178,12 @@ def main():
         resize += [v for k in JOBS for v in res[k][step][3]]
     spans_sorted = sorted(spans)
     mk = spans_sorted[len(spans) // 2]
+    # a step far above the median: report each tenant's longest launches (stderr)
+    for step, sp in enumerate(spans):
+        if sp > 2 * mk:
+            sys.stderr.write("C4 step %d: %.1f ms\n" % (step, sp))
+            for k in JOBS:
+                sys.stderr.write("  %s span %.1f: %s\n" % (k, res[k][step][1] - res[k][step][0], json.dumps(res[k][step][4])))
     print(json.dumps({"config": "C4: triad 2^26, SpMV 2^20, stencil 8192^2, bf16 GEMM 4096^3 from 4 client processes "
                                 "via slated (AUTO)",
                       "jobs": JOBS, "seq_cuda_ms": round(seq_ms, 3), "solo_ms": {k: round(v, 3) for k, v in solo.items()},
