@@ -347,6 +347,130 @@ struct BlackScholes : TenantBase {
     return __fmul_rn(K, __fmaf_rn(K, __fmaf_rn(K, __fmaf_rn(K, __fmaf_rn(K, A5, A4), A3), A2), A1));
   }
   // options o = 0..k-1 of this thread (k = 4, or 1..3 on the ragged tail)
+  // ---- packed FP32x2 (sm_100: FFMA2 / FMUL2 / FADD2): two options per instruction
+  // The body is issue-bound (~39 instructions per option-scenario against ~30
+  // FP32-pipe cycles); a packed op does two options' work in one issue slot
+  // (tools/probe/ffma2_rate.cu: the FP32 pipe rate is the same, so this pays
+  // only where issue, not the pipe, is the limit).  Per element the same
+  // round-to-nearest ops as price<k>; ptxas may contract a packed mul + add
+  // into FFMA2, so results can differ from price<k> by an ulp (Q39).
+  typedef unsigned long long f2;
+  __device__ __forceinline__ static f2 pk(float a, float b) {
+    f2 r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+  }
+  __device__ __forceinline__ static void up(f2 v, float& a, float& b) { asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v)); }
+  __device__ __forceinline__ static f2 fma2(f2 a, f2 b, f2 c) {
+    f2 d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+    return d;
+  }
+  __device__ __forceinline__ static f2 mul2(f2 a, f2 b) {
+    f2 d;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+  }
+  __device__ __forceinline__ static f2 add2(f2 a, f2 b) {
+    f2 d;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+  }
+  __device__ __forceinline__ static f2 sub2(f2 a, f2 b) {
+    f2 d;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+  }
+  __device__ __forceinline__ static f2 abs2(f2 a) { return a & 0x7fffffff7fffffffull; }
+  __device__ __forceinline__ static f2 poly2(f2 K) {
+    const f2 A1 = pk(0.31938153f, 0.31938153f), A2 = pk(-0.356563782f, -0.356563782f),
+             A3 = pk(1.781477937f, 1.781477937f), A4 = pk(-1.821255978f, -1.821255978f),
+             A5 = pk(1.330274429f, 1.330274429f);
+    return mul2(K, fma2(K, fma2(K, fma2(K, fma2(K, A5, A4), A3), A2), A1));
+  }
+  // 4 options as two packed pairs (0,1) and (2,3); the per-option setup and the
+  // final mean are price<4>'s scalar code
+  __device__ __forceinline__ static void price4_x2(const float (&S)[4], const float (&X)[4], const float (&T)[4], float r,
+                                                   const float* sig, uint32_t P, float (&call)[4], float (&put)[4]) {
+    const float RSQRT2PI = 0.39894228040143267794f;
+    float sqt[4], rsqt[4], lsx[4], xd[4], sxd[4];
+#pragma unroll
+    for (int o = 0; o < 4; ++o) {
+      sqt[o] = sqrtf(T[o]);
+      rsqt[o] = __fdiv_rn(1.0f, sqt[o]);
+      lsx[o] = logf(__fdiv_rn(S[o], X[o]));
+      xd[o] = __fmul_rn(X[o], expf(__fmul_rn(-r, T[o])));
+      sxd[o] = __fdiv_rn(S[o], xd[o]);
+    }
+    f2 SQT[2], RSQT[2], LSX[2], TT[2], SS[2], XD[2], SXD[2], CS[2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      SQT[h] = pk(sqt[2 * h], sqt[2 * h + 1]);
+      RSQT[h] = pk(rsqt[2 * h], rsqt[2 * h + 1]);
+      LSX[h] = pk(lsx[2 * h], lsx[2 * h + 1]);
+      TT[h] = pk(T[2 * h], T[2 * h + 1]);
+      SS[h] = pk(S[2 * h], S[2 * h + 1]);
+      XD[h] = pk(xd[2 * h], xd[2 * h + 1]);
+      SXD[h] = pk(sxd[2 * h], sxd[2 * h + 1]);
+      CS[h] = pk(0.f, 0.f);
+    }
+    const f2 ONE = pk(1.0f, 1.0f), AK = pk(0.2316419f, 0.2316419f), MH = pk(-0.5f, -0.5f),
+             L2E = pk(1.44269504088896341f, 1.44269504088896341f), RS = pk(RSQRT2PI, RSQRT2PI);
+    for (uint32_t p = 0; p < P; ++p) {
+      const float sg = __ldg(sig + p);
+      const float rsg = rcp(sg);
+      const float hs2 = __fmaf_rn(__fmul_rn(0.5f, sg), sg, r);
+      const f2 SG = pk(sg, sg), RSG = pk(rsg, rsg), HS2 = pk(hs2, hs2);
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const f2 sst = mul2(SG, SQT[h]);
+        const f2 d1 = mul2(fma2(HS2, TT[h], LSX[h]), mul2(RSG, RSQT[h]));
+        const f2 d2 = sub2(d1, sst);
+        const f2 u1 = fma2(AK, abs2(d1), ONE), u2 = fma2(AK, abs2(d2), ONE);
+        float uu0, uu1, a0, a1;
+        up(mul2(u1, u2), uu0, uu1);
+        const f2 q = pk(rcp(uu0), rcp(uu1));
+        up(mul2(mul2(MH, mul2(d1, d1)), L2E), a0, a1);
+        float x0, x1;
+        asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x0) : "f"(a0));
+        asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x1) : "f"(a1));
+        const f2 e1 = mul2(RS, pk(x0, x1));
+        const f2 c1 = mul2(e1, poly2(mul2(u2, q)));
+        const f2 c2 = mul2(mul2(e1, SXD[h]), poly2(mul2(u1, q)));
+        const f2 o1 = sub2(ONE, c1), o2 = sub2(ONE, c2);
+        float d10, d11, d20, d21, c10, c11, c20, c21, o10, o11, o20, o21;
+        up(d1, d10, d11);
+        up(d2, d20, d21);
+        up(c1, c10, c11);
+        up(c2, c20, c21);
+        up(o1, o10, o11);
+        up(o2, o20, o21);
+        const f2 n1 = pk(d10 > 0.f ? o10 : c10, d11 > 0.f ? o11 : c11);
+        const f2 n2 = pk(d20 > 0.f ? o20 : c20, d21 > 0.f ? o21 : c21);
+        CS[h] = add2(CS[h], sub2(mul2(SS[h], n1), mul2(XD[h], n2)));
+      }
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      float c0, c1;
+      up(CS[h], c0, c1);
+      call[2 * h] = __fdiv_rn(c0, float(P));
+      call[2 * h + 1] = __fdiv_rn(c1, float(P));
+    }
+#pragma unroll
+    for (int o = 0; o < 4; ++o) put[o] = __fadd_rn(call[o], __fsub_rn(xd[o], S[o]));
+  }
+#ifndef SLATE_BS_X2
+#define SLATE_BS_X2 1
+#endif
+  __device__ __forceinline__ static void price4(const float (&S)[4], const float (&X)[4], const float (&T)[4], float r,
+                                                const float* sig, uint32_t P, float (&call)[4], float (&put)[4]) {
+#if SLATE_BS_X2
+    price4_x2(S, X, T, r, sig, P, call, put);
+#else
+    price<4>(S, X, T, r, sig, P, call, put);
+#endif
+  }
   template <int k>
   __device__ __forceinline__ static void price(const float (&S)[4], const float (&X)[4], const float (&T)[4],
                                                float r, const float* sig, uint32_t P, float (&call)[4],
@@ -399,7 +523,7 @@ struct BlackScholes : TenantBase {
       S[0] = s4.x; S[1] = s4.y; S[2] = s4.z; S[3] = s4.w;
       X[0] = x4.x; X[1] = x4.y; X[2] = x4.z; X[3] = x4.w;
       T[0] = t4.x; T[1] = t4.y; T[2] = t4.z; T[3] = t4.w;
-      price<4>(S, X, T, a.r, sig, a.n_scen, c, p);
+      price4(S, X, T, a.r, sig, a.n_scen, c, p);
       __stcs(reinterpret_cast<float4*>(a.call) + v, make_float4(c[0], c[1], c[2], c[3]));
       __stcs(reinterpret_cast<float4*>(a.put) + v, make_float4(p[0], p[1], p[2], p[3]));
     } else {
@@ -465,7 +589,7 @@ struct BlackScholesShort : BlackScholes {
       const float4 s4 = st[threadIdx.x], x4 = st[256 + threadIdx.x], t4 = st[512 + threadIdx.x];
       float S[4] = {s4.x, s4.y, s4.z, s4.w}, X[4] = {x4.x, x4.y, x4.z, x4.w}, T[4] = {t4.x, t4.y, t4.z, t4.w};
       float c[4], p[4];
-      price<4>(S, X, T, a.r, sig, a.n_scen, c, p);
+      price4(S, X, T, a.r, sig, a.n_scen, c, p);
       __stcs(reinterpret_cast<float4*>(a.call) + cur, make_float4(c[0], c[1], c[2], c[3]));
       __stcs(reinterpret_cast<float4*>(a.put) + cur, make_float4(p[0], p[1], p[2], p[3]));
     }
