@@ -261,14 +261,19 @@ class Workload:
         self.arrival_ms = 0.0
 
 
-def make_c2(S, dev):
+def make_c2(S, dev, pinned=None):
+    """The C2 pair on device buffers; `pinned` (another C2 workload's pinned host
+    inputs) gives a second device set over the same host data (e2e pipelining)."""
     import torch
     from paper_conf_ipps_allenf019_b200 import inputs as I
-    rp, col, val, x = I.spmv_inputs(N_ROWS, I.seed_for(2, 0))
-    S_, X_, T_, r = I.bs_inputs(N_OPT, I.seed_for(2, 1))
-    sig = I.bs_sigmas(P_SCEN)
-    host = {"rp": rp, "col": col, "val": val, "x": x, "S": S_, "X": X_, "T": T_, "sig": sig}
-    pinned = {k: torch.from_numpy(v).pin_memory() for k, v in host.items()}
+    r = I.bs_inputs(8, I.seed_for(2, 1))[3]
+    if pinned is None:
+        rp, col, val, x = I.spmv_inputs(N_ROWS, I.seed_for(2, 0))
+        S_, X_, T_, r = I.bs_inputs(N_OPT, I.seed_for(2, 1))
+        sig = I.bs_sigmas(P_SCEN)
+        host = {"rp": rp, "col": col, "val": val, "x": x, "S": S_, "X": X_, "T": T_, "sig": sig}
+        pinned = {k: torch.from_numpy(v).pin_memory() for k, v in host.items()}
+    rp = pinned["rp"].numpy()
     d = {k: v.to(dev) for k, v in pinned.items()}
     d["y"] = torch.zeros(N_ROWS, device=dev)
     d["call"] = torch.zeros(N_OPT, device=dev)
@@ -611,28 +616,58 @@ def run_slate(args, world, rank, local):
     value = aggregate(world, args.steps, total_ms_max)
     n_launch = sum(len(s[3]) + len(s[4]) + sum(q["n_topups"] for q in s[3] + s[4]) for s in r2["steps"])
 
-    # ---- e2e: host buffers in, the same co-run through the public API, results out
+    # ---- e2e: host buffers in, the same co-run through the public API, results out.
+    # Every step copies its inputs from pinned host memory and reads its results
+    # back; the copies run on a copy stream and overlap the neighbouring steps'
+    # kernels (step i+1's inputs go in while step i computes, into a second
+    # device set; step i's results come out while step i+1 computes).
     kA, kB = sA.register_kernel(w2.a.kind), sA.register_kernel(w2.b.kind)
-    e2e_times = []
-    for i in range(args.steps + 1):
-        flush_l2(flush)
-        t0 = time.perf_counter()
-        for k, v in w2.pinned.items():
-            w2._keep[k].copy_(v, non_blocking=True)
-        torch.cuda.synchronize()
-        # what a user does: submit both jobs (AUTO placement), wait for them; no
-        # per-launch queries (run_schedule's timing reads) in this region
-        submit(sA, kA, w2.a, placement=S.PLACE_AUTO)
-        spin_ms(w2.arrival_ms)
-        submit(sB, kB, w2.b, placement=S.PLACE_AUTO)
-        sA.sync(0)
-        sB.sync(0)
-        for k in w2.out_names:
-            w2.out_pinned[k].copy_(w2._keep[k], non_blocking=True)
-        torch.cuda.synchronize()
-        if i:
-            e2e_times.append(time.perf_counter() - t0)
-    e2e_s = allmax(world, statistics.median(e2e_times))
+    w2b = make_c2(S, dev, pinned=w2.pinned)
+    w2b.arrival_ms = w2.arrival_ms
+    sets = [w2, w2b]
+    cs = torch.cuda.Stream()
+
+    def h2d(w):
+        with torch.cuda.stream(cs):
+            for k, v in w2.pinned.items():
+                w._keep[k].copy_(v, non_blocking=True)
+            ev = torch.cuda.Event()
+            ev.record(cs)
+        return ev
+
+    def d2h(w):
+        with torch.cuda.stream(cs):
+            for k in w2.out_names:
+                w2.out_pinned[k].copy_(w._keep[k], non_blocking=True)
+            ev = torch.cuda.Event()
+            ev.record(cs)
+        return ev
+
+    def e2e_run(n):
+        ev_in = h2d(sets[0])
+        ev_out = [None, None]
+        for i in range(n):
+            cur = sets[i % 2]
+            ev_in.synchronize()                      # step i's inputs are in (the server's streams do not wait)
+            if ev_out[i % 2] is not None:
+                ev_out[i % 2].synchronize()          # step i-2's results are out of this set
+            submit(sA, kA, cur.a, placement=S.PLACE_AUTO)
+            spin_ms(cur.arrival_ms)
+            submit(sB, kB, cur.b, placement=S.PLACE_AUTO)
+            if i + 1 < n:
+                ev_in = h2d(sets[(i + 1) % 2])       # overlaps step i's kernels
+            sA.sync(0)
+            sB.sync(0)
+            ev_out[i % 2] = d2h(cur)                 # overlaps step i+1's kernels
+        cs.synchronize()
+
+    flush_l2(flush)
+    e2e_run(2)                                       # warm-up
+    flush_l2(flush)
+    t0 = time.perf_counter()
+    e2e_run(args.steps)
+    e2e_s = allmax(world, (time.perf_counter() - t0) / args.steps)
+    del w2b
     h2d_bytes, d2h_bytes = w2.h2d_bytes, w2.d2h_bytes
     del w2
 
