@@ -45,7 +45,7 @@ class ProtocolViolation(AssertionError):
     pass
 
 
-PENDING, PROLOGUE, STANDBY, FETCH, EXEC, CHECK, EXITED, RETIRING = range(8)
+PENDING, PROLOGUE, STANDBY, FETCH, EXEC, CHECK, EXITED, RETIRING, WAITDONE = range(9)
 
 
 @dataclass
@@ -59,6 +59,9 @@ class Config:
     resizes: list = field(default_factory=list)   # [(lo, hi), ...] applied in order at random times
     grid: int = 0             # CTAs per launch; default occ * ranks (one full wave)
     abort: bool = False       # long-task tenants: a retiring worker may abandon its task
+    leave_main: bool = True   # the CTA whose exit completes the launch's own grid waits until every block ran
+                              # (a top-up grid may still hold blocks, and the queue's next
+                              # launch starts when this grid completes).  False: it just exits
     faa_retire: bool = True   # retire as the runtime does it (Q22): live -= 1 in one atomic
                               # step, and if that took live from 1 to 0, live += 1 in a later step
                               # and stay; other CTAs may act in between.  False: one atomic
@@ -86,8 +89,11 @@ class Model:
         self.task_starts = []
         self.resize_i = 0
         grid = cfg.grid or cfg.occ * cfg.ranks
-        # per CTA: [state, rank, launch_lo, launch_hi, g, n, seen_epoch, was_worker]
-        self.ctas = [[PENDING, -1, 0, cfg.ranks - 1, 0, 0, -1, False] for _ in range(grid)]
+        # per CTA: [state, rank, launch_lo, launch_hi, g, n, seen_epoch, was_worker, main]
+        # (main: a CTA of the launch's own grid; top-up CTAs are not)
+        self.ctas = [[PENDING, -1, 0, cfg.ranks - 1, 0, 0, -1, False, True] for _ in range(grid)]
+        self.main_exited = 0               # main CTAs that have left (joined or not)
+        self.grid = grid
         self.resident = [0] * cfg.ranks    # resident CTAs per SM (placement capacity)
 
     # ------------------------------------------------------------ helpers
@@ -98,13 +104,19 @@ class Model:
         return _in(c[1], self.lo, self.hi) and _in(c[1], c[2], c[3])
 
     def exit(self, c, worker):
-        c[0] = EXITED
-        self.resident[c[1]] -= 1
         if worker:
             self.live -= 1
+        if c[8]:                           # a CTA of the launch's own grid leaves (worker or not)
+            self.main_exited += 1
+            if self.main_exited == self.grid and self.cfg.leave_main and self.blocks_done < self.cfg.blocks:
+                c[0] = WAITDONE            # the one completing the grid waits for every block (leave_main)
+                return
+        c[0] = EXITED
+        self.resident[c[1]] -= 1
 
     def key(self):
-        return (self.next, self.epoch, self.lo, self.hi, self.live, tuple(self.returned), tuple(self.cov), self.blocks_done,
+        return (self.next, self.epoch, self.lo, self.hi, self.live, self.main_exited, tuple(self.returned), tuple(self.cov),
+                self.blocks_done,
                 self.tasks_done, tuple(sorted(self.task_starts)), self.resize_i,
                 tuple(tuple(c) for c in self.ctas), tuple(self.resident))
 
@@ -127,6 +139,8 @@ class Model:
                 acts.append(("step", i))
                 if self.live == 0 and self.next < self.cfg.blocks:
                     acts.append(("timeout", i))
+            elif st == WAITDONE and self.blocks_done == self.cfg.blocks:
+                acts.append(("step", i))
         if self.resize_i < len(self.cfg.resizes):
             acts.append(("resize",))
         return acts
@@ -143,7 +157,7 @@ class Model:
             # (the runtime's rule); CTAs it places on old ranks leave
             if lo < old[0] or hi > old[1]:
                 for _ in range(cfg.occ * cfg.ranks):
-                    self.ctas.append([PENDING, -1, lo, hi, 0, 0, -1, False])
+                    self.ctas.append([PENDING, -1, lo, hi, 0, 0, -1, False, False])
             return
         if act[0] == "place":
             _, i, r = act
@@ -161,6 +175,10 @@ class Model:
         if act[0] == "timeout":            # standby with no live worker: run anyway (liveness)
             self.live += 1
             c[0], c[7] = FETCH, True
+            return
+        if st == WAITDONE:                 # every block ran: the last main CTA leaves, the grid completes
+            c[0] = EXITED
+            self.resident[c[1]] -= 1
             return
         if st in (PROLOGUE, STANDBY):
             # Lst1: leader reads the SM id and the bound; here also the queue state
@@ -236,6 +254,11 @@ class Model:
     def check_step(self):
         if any(v > 1 for v in self.cov):
             raise ProtocolViolation("block executed twice")
+        # stream order: the launch's own grid completes (its next launch may start)
+        # only when every block has run, whatever top-up grids still hold
+        if self.blocks_done < self.cfg.blocks and all(c[0] == EXITED for c in self.ctas if c[8]):
+            raise ProtocolViolation("the launch's grid completed with %d blocks still to run"
+                                    % (self.cfg.blocks - self.blocks_done))
 
 
 def simulate(cfg, seed, max_steps=10_000_000):

@@ -41,7 +41,7 @@ struct alignas(128) TaskCtl {
                                   // abandoning a task and retiring is one atomic step (Q28)
   uint32_t pad_l[30];
   uint32_t started;               // workers that joined
-  uint32_t main_live;             // joined CTAs of the launch's own grid (not top-ups) not yet exited
+  uint32_t main_exited;           // CTAs of the launch's own grid (not top-ups) that left, joined or not
   uint32_t pad_s[30];
   uint32_t live_rank[kMaxRanks];  // live workers per SM rank
   uint32_t ret_head, ret_tail;    // ring of abandoned task starts (+1; 0 = slot empty)

@@ -155,7 +155,6 @@ __device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
       atomicAdd(&tc->live_pending, 1ull);    // results unused: RED, no round trip
       atomicAdd(&tc->live_rank[rank], 1u);
       atomicAdd(&tc->started, 1u);
-      if (!p.is_topup) atomicAdd(&tc->main_live, 1u);
       const uint32_t e = ctrl_epoch(c);
       if (e > p.base_epoch && ld_relaxed_u32(&tc->join_epoch) < e && atomicMax(&tc->join_epoch, e) < e && p.mirror) {
         publish_mirror(&tc->join_word, &p.mirror->join, mirror_pack(e, globaltimer()));   // grow observed under epoch e
@@ -284,15 +283,19 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
   return g;
 }
 
-// A CTA of the launch's own grid leaves.  The last one to leave waits until
-// every block of the launch is done: top-up CTAs (another stream, grow) may
-// still hold some, and the queue's next launch starts when this kernel
-// completes (stream order).  Without top-ups the blocks are all counted by
-// then and it does not wait.
+// A CTA of the launch's own grid leaves -- every one, worker or not (a CTA
+// that finds the queue drained in its prologue too).  The one whose exit
+// completes the grid waits until every block of the launch is done: top-up
+// CTAs (another stream, grow) may still hold some, and the queue's next
+// launch starts when this grid completes (stream order).  Without top-ups the
+// blocks are all counted by then and it does not wait.  Modelled in
+// oracle/protocol.py (Config.leave_main; counting only joined CTAs was not
+// enough: a grid whose CTAs all arrived after a top-up took the last tasks
+// completed early).
 template <class P>
 __device__ __forceinline__ void leave_main(const P& p) {
   if (p.is_topup) return;
-  if (atomicSub(&p.tc->main_live, 1u) != 1u) return;
+  if (atomicAdd(&p.tc->main_exited, 1u) + 1u != gridDim.x) return;
   uint32_t ns = 128;
   while (uint32_t(ld_relaxed_u64(&p.tc->done)) < p.B) {
     __nanosleep(ns);
@@ -340,7 +343,10 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     s_rank = r;
   }
   __syncthreads();
-  if (!s_go) return;
+  if (!s_go) {
+    if (threadIdx.x == 0) leave_main(p);
+    return;
+  }
   const uint32_t rank = s_rank;
   c = __shfl_sync(0xffffffffu, c, 0);
   if constexpr (Tn::kHasInit) {

@@ -276,7 +276,10 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     H.ctrl = c;
   }
   __syncthreads();
-  if (!H.go) return;
+  if (!H.go) {
+    if (threadIdx.x == 0) leave_main(p);
+    return;
+  }
   pdl_wait();   // a PDL launch: the previous kernel on the stream has completed from here on
 
   if (warp == kTaskWarp) {

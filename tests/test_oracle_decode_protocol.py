@@ -193,3 +193,18 @@ def test_protocol_abort_needs_the_combined_word():
                 y = copy.deepcopy(x)
                 y.apply(a)
                 stack.append(y)
+
+
+def test_grid_completion_waits_for_topup_blocks():
+    """Stream order with top-ups (leave_main): the launch's own grid
+    completes only after every block ran, even when a top-up grid (a grow) took the
+    last tasks -- and the CTA that waits cannot starve the top-up (liveness is part
+    of the exhaustive exploration).  Without the rule the exploration finds a grid
+    that completes with blocks still running on the top-up."""
+    cfgs = [P.Config(blocks=4, iters=2, ranks=2, occ=1, lo=0, hi=1, resizes=[(0, 0), (0, 1)]),
+            P.Config(blocks=3, iters=1, ranks=2, occ=1, lo=0, hi=0, resizes=[(0, 1)])]
+    for cfg in cfgs:
+        assert P.explore(cfg) > 0
+    bad = P.Config(blocks=4, iters=2, ranks=2, occ=1, lo=0, hi=1, resizes=[(0, 0), (0, 1)], leave_main=False)
+    with pytest.raises(P.ProtocolViolation, match="grid completed"):
+        P.explore(bad)
