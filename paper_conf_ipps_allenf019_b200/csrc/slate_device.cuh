@@ -489,12 +489,14 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
     atomicMax(&p.tc->t_exit, globaltimer());
 #endif
   }
-  if (threadIdx.x == 0) leave_main(p);
   if (threadIdx.x < 32) {
     c = __shfl_sync(0xffffffffu, c, 0);
     if (lane == 0) atomicAdd(&p.tc->live_rank[rank], 0xffffffffu);   // live_rank -= 1
     if (s_retired) check_shrink_done(p, c, lane);
   }
+  // after the shrink bookkeeping: a retired CTA that ends up waiting here for
+  // the launch's blocks must not hold up the end of the shrink it retired for
+  if (threadIdx.x == 0) leave_main(p);
 }
 
 template <class Tn>

@@ -507,8 +507,8 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   __syncthreads();
   if (warp == kTaskWarp) {
     if (lane == 0) atomicAdd(&p.tc->live_rank[H.rank], 0xffffffffu);   // live_rank -= 1
-    if (lane == 0) leave_main(p);
     if (H.retired) check_shrink_done(p, H.ctrl, lane);
+    if (lane == 0) leave_main(p);   // after the shrink bookkeeping (see slate_device.cuh)
   }
 }
 

@@ -72,7 +72,9 @@ def client(endpoint, kind, steps, go_path):
     for step in range(steps):
         while not os.path.exists("%s.%d" % (go_path, step)):
             time.sleep(0.0005)
+        t_go = time.time()
         ids = [s.launch(kid, args, grid, placement=S.PLACE_AUTO) for _ in range(JOBS[kind])]
+        t_sub = time.time()
         s.sync(0)
         qs = [s.query(i) for i in ids]
         slow = sorted(qs, key=lambda q: q["start_ms"] - q["end_ms"])[:3]   # the longest launches (diagnostics)
@@ -80,7 +82,7 @@ def client(endpoint, kind, steps, go_path):
                     sum(len(q["resize_us"]) for q in qs), [v for q in qs for v in q["resize_us"]],
                     [{"ms": round(q["end_ms"] - q["start_ms"], 3), "start": round(q["start_ms"], 3),
                       "workers": q["workers_started"], "topups": q["n_topups"], "resizes": q["n_resizes"],
-                      "iters": q["iters"], "sm": [q["sm_lo"], q["sm_hi"]]} for q in slow]])
+                      "iters": q["iters"], "sm": [q["sm_lo"], q["sm_hi"]]} for q in slow], [t_go, t_sub]])
         open("%s.%d.%s" % (go_path, step, kind), "w").close()   # this client is ready for the next step
     print("RESULT " + json.dumps(out), flush=True)
     s.close()
@@ -183,7 +185,9 @@ def main():
         if sp > 2 * mk:
             sys.stderr.write("C4 step %d: %.1f ms\n" % (step, sp))
             for k in JOBS:
-                sys.stderr.write("  %s span %.1f: %s\n" % (k, res[k][step][1] - res[k][step][0], json.dumps(res[k][step][4])))
+                sys.stderr.write("  %s span %.1f, host go %.3f submitted %.3f: %s\n" % (
+                    k, res[k][step][1] - res[k][step][0], res[k][step][5][0], res[k][step][5][1],
+                    json.dumps(res[k][step][4])))
     print(json.dumps({"config": "C4: triad 2^26, SpMV 2^20, stencil 8192^2, bf16 GEMM 4096^3 from 4 client processes "
                                 "via slated (AUTO)",
                       "jobs": JOBS, "seq_cuda_ms": round(seq_ms, 3), "solo_ms": {k: round(v, 3) for k, v in solo.items()},
