@@ -83,7 +83,8 @@ typedef enum {
   SLATE_KIND_GAUSS_FAN1 = 11,  /* GS step t, Fan1: m[i][t] = a[i][t] / a[t][t]; 256 rows/block   */
   SLATE_KIND_GAUSS_FAN2 = 12,  /* GS step t, Fan2: a[i][j] -= m[i][t] a[t][j] (j >= t),
                                   b[i] -= m[i][t] b[t]; 16 rows x 128 columns/block              */
-  SLATE_KIND_MAX_ = 13
+  SLATE_KIND_USER = 13,        /* a user kernel compiled at run time (slate_register_source, NEXT-3) */
+  SLATE_KIND_MAX_ = 14
 } slate_kind;
 
 /* Per-kind argument blocks (passed by value in slate_launch_desc.args).
@@ -233,6 +234,42 @@ slate_status slate_launch_n(slate_session* s, slate_kernel k, const slate_launch
  * one (same ids and order, no batch).  Errors: as slate_launch_n. */
 slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel* ks, const slate_launch_desc* ds,
                                slate_launch_id* first);
+
+/* ------------------------------------------------------------------ runtime kernel transformation
+ * NEXT-3 (Slate scans a user kernel's source, injects its task
+ * loop and compiles it with NVRTC).  `source` holds a CUDA C++ kernel
+ *     __global__ void <kernel_name>(<parameters>) { ... blockIdx ... gridDim ... }
+ * with 1-D blocks of `block_threads` threads and `smem_bytes` of dynamic
+ * shared memory.  The server renames it into a device function that takes the
+ * block index and the original grid, generates the slate worker (Lst1/Lst2:
+ * SM binding, task counter, decode, resize word) and an original-kernel
+ * wrapper around the same body, compiles both for sm_100a with NVRTC and
+ * registers the result as a kernel of kind SLATE_KIND_USER.  Launch it with
+ * slate_launch / slate_launch_n: desc.grid is the original grid (any x, y, z),
+ * desc.args the parameters packed as a C struct in declaration order
+ * (args_size bytes).  bytes_per_block / flops_per_block declare its work for
+ * slate_profile's classification (0 if unknown).  In-process sessions only
+ * (through an endpoint the server cannot rewrite pointers it cannot see).
+ * Errors: EINVAL (no such kernel in the source, bad sizes), EUNSUPPORTED (no
+ * NVRTC, or an endpoint session), ECUDA (compile or load failed; the compiler
+ * log is in slate_last_error). */
+typedef struct {
+  uint32_t abi_version;
+  uint32_t block_threads;
+  uint32_t smem_bytes;
+  uint32_t args_size;
+  uint32_t iters;              /* task size; 0 = automatic */
+  uint32_t pad_;
+  const char* source;
+  const char* kernel_name;
+  double bytes_per_block, flops_per_block;
+} slate_source_desc;
+slate_status slate_register_source(slate_session* s, const slate_source_desc* d, slate_kernel* out);
+/* The transformed source slate_register_source would compile (no GPU, no
+ * NVRTC needed): writes up to cap bytes (NUL-terminated) to out and the full
+ * length to *len.  Errors: EINVAL (no such kernel). */
+slate_status slate_transform_source(const char* source, const char* kernel_name, uint32_t block_threads,
+                                    uint32_t smem_bytes, char* out, size_t cap, size_t* len);
 
 /* Resize the SM range of the queue that owns launch l to [sm_lo, sm_hi]
  * (§III-C; the dispatcher's start_sm/end_sm, Lst3 P:L250-251).

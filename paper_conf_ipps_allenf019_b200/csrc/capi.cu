@@ -219,6 +219,15 @@ slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel*
   return rc == SLATE_OK ? rc : fail(s, rc, err);
 }
 
+slate_status slate_register_source(slate_session* s, const slate_source_desc* d, slate_kernel* out) {
+  if (!s || !d || !out) return fail(s, SLATE_EINVAL, "null argument");
+  std::lock_guard<std::mutex> g(s->mu);
+  if (!s->srv) return fail(s, SLATE_EUNSUPPORTED, "runtime-compiled kernels need an in-process session");
+  std::string err;
+  const int rc = s->srv->register_source(d, out, &err);
+  return rc == SLATE_OK ? rc : fail(s, rc, err);
+}
+
 slate_status slate_resize(slate_session* s, slate_launch_id l, uint32_t lo, uint32_t hi) {
   if (!s) return SLATE_EINVAL;
   std::lock_guard<std::mutex> g(s->mu);

@@ -1,10 +1,11 @@
 // kernels.h -- host/device shared layout of the slate control structures and
 // the host-side dispatch table over tenant kinds.  No torch types anywhere.
 #pragma once
-#include <cstddef>
-#include <cstdint>
-#include <cuda_runtime.h>
+#include "rtc_types.h"
+#ifndef __CUDACC_RTC__
+#include <string>
 #include "../../include/slate.h"
+#endif
 
 namespace slate {
 
@@ -48,8 +49,10 @@ struct alignas(128) TaskCtl {
   uint32_t pad2[30];
   uint32_t ret[kMaxRanks];
 };
+#ifndef __CUDACC_RTC__
 static_assert(offsetof(TaskCtl, live_pending) == 256 && offsetof(TaskCtl, started) == 384 &&
               offsetof(TaskCtl, live_rank) == 512, "TaskCtl header lines: next | done.. | live_pending | started");
+#endif
 constexpr size_t kTaskCtlHeader = 512;   // the part snapshotted to the host at the end
 
 // Per launch, in mapped pinned host memory: what the host poller watches.
@@ -69,6 +72,21 @@ struct HostMirror {
   uint64_t pad[5];
 };
 
+// The second kernel parameter of a runtime-compiled user worker (NEXT-3): every
+// WorkerParams field but the user's arguments (the first parameter), in a
+// layout both nvcc (host) and NVRTC (the worker) see.
+struct UserWorkerCommon {
+  uint32_t gx, gy, gz, B, iters, occ;
+  uint32_t bound_lo, bound_hi, n_ranks, standby_timeout_ns;
+  uint32_t base_epoch, is_topup, gate_first, pad_;
+  const uint64_t* ctrl;
+  TaskCtl* tc;
+  HostMirror* mirror;
+  uint32_t* cov;
+  const uint16_t* rank_of;
+};
+
+#ifndef __CUDACC_RTC__   // host side (not needed by runtime-compiled user workers)
 // Everything a worker launch needs besides the tenant's own arguments.
 struct WorkerCommon {
   uint32_t gx, gy, gz, B, iters, occ;
@@ -83,6 +101,7 @@ struct WorkerCommon {
   HostMirror* mirror;
   uint32_t* cov;
   const uint16_t* rank_of;
+  const struct KindOps* ops = nullptr;   // the kind being launched (runtime-compiled kinds read their kernels here)
 };
 
 struct KindOps {
@@ -103,7 +122,21 @@ struct KindOps {
                                  // running launch may get a top-up while later launches are queued
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;
   cudaError_t (*launch_standalone)(const void* args, dim3 grid, cudaStream_t) = nullptr;
+  // runtime-compiled user kernels (NEXT-3): the original kernel needs its kind
+  cudaError_t (*launch_standalone_ops)(const KindOps*, const void* args, dim3 grid, cudaStream_t) = nullptr;
+  uint32_t user_threads = 0;     // T of a user kernel
+  void* user_ctx = nullptr;      // the loaded user kernels (user_kernels.cu)
+  double user_bytes_per_block = 0, user_flops_per_block = 0;
 };
+
+// NEXT-3 (the paper's runtime kernel transformation): scan a user's
+// CUDA source for its __global__ kernel and generate the slate worker around it
+// (and an original-kernel wrapper over the same body); compile it with NVRTC
+// for sm_100a and load it.  Returns false with *err set on failure.
+bool transform_user_kernel(const char* src, const char* name, uint32_t threads, uint32_t smem, std::string* out,
+                           std::string* err);
+bool build_user_kind(const char* src, const char* name, uint32_t threads, uint32_t smem, uint32_t args_size,
+                     KindOps* ops, std::string* err);
 
 const KindOps* kind_ops(uint32_t kind);   // nullptr if the kind is not built
 
@@ -128,5 +161,7 @@ inline cudaError_t launch_kernel(const void* fn, dim3 grid, dim3 block, void** a
 cudaError_t launch_calibrate(uint32_t* out, uint32_t blocks, uint32_t spin_ns, cudaStream_t st);
 cudaError_t launch_clock_probe(volatile uint32_t* flag, volatile unsigned long long* stamp, int rounds,
                                cudaStream_t st);
+
+#endif  // __CUDACC_RTC__
 
 }  // namespace slate

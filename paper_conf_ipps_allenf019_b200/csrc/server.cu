@@ -356,6 +356,47 @@ int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::stri
   return SLATE_OK;
 }
 
+// NEXT-3: a user kernel from source (user_kernels.cu), a kind of its own
+int Server::register_source(const slate_source_desc* d, uint64_t* out, std::string* err) {
+  if (!d || !out || d->abi_version != SLATE_ABI_VERSION || !d->source || !d->kernel_name || d->args_size == 0 ||
+      d->args_size > 4096 || d->block_threads == 0 || d->block_threads > 1024) {
+    if (err) *err = "bad source descriptor";
+    return SLATE_EINVAL;
+  }
+  auto ops = std::make_unique<KindOps>();
+  std::string e;
+  if (!build_user_kind(d->source, d->kernel_name, d->block_threads, d->smem_bytes, d->args_size, ops.get(), &e)) {
+    if (err) *err = e;
+    return e.find("not found") != std::string::npos ? SLATE_EUNSUPPORTED
+           : e.find("no `__global__") != std::string::npos ? SLATE_EINVAL : SLATE_ECUDA;
+  }
+  ops->user_bytes_per_block = d->bytes_per_block;
+  ops->user_flops_per_block = d->flops_per_block;
+  if (ops->smem > 48 * 1024) {
+    CK(cudaFuncSetAttribute(ops->worker_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem));
+    CK(cudaFuncSetAttribute(ops->standalone_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ops->smem));
+  }
+  int occ = 0;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ops->worker_fn, ops->threads, ops->smem));
+  if (occ < 1) {
+    if (err) *err = "the user worker does not fit on an SM";
+    return SLATE_ECUDA;
+  }
+  std::lock_guard<std::mutex> g(mu_);
+  auto k = std::make_unique<KernelEntry>();
+  k->id = next_kernel_id_++;
+  k->desc = slate_kernel_desc{};
+  k->desc.abi_version = SLATE_ABI_VERSION;
+  k->desc.kind = SLATE_KIND_USER;
+  k->desc.iters = d->iters;
+  k->occ = occ;
+  k->ops = ops.get();
+  k->own_ops = std::move(ops);
+  *out = k->id;
+  kernels_[k->id] = std::move(k);
+  return SLATE_OK;
+}
+
 bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t* B, std::string* err) const {
   auto fail = [&](const char* m) {
     if (err) *err = m;
@@ -447,6 +488,11 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
       }
       break;
     }
+    case SLATE_KIND_USER:        // the caller's grid is the original grid
+      g[0] = d->grid[0];
+      g[1] = d->grid[1];
+      g[2] = d->grid[2];
+      break;
     default:
       return fail("unknown kind");
   }
@@ -527,6 +573,12 @@ void Server::work(const KernelEntry& k, const slate_launch_desc* d, double* byte
       const double r = a->n - 1.0 - a->t;
       *bytes = 8.0 * r + 4.0;
       *fp32 = r;
+      break;
+    }
+    case SLATE_KIND_USER: {      // declared at registration, per block
+      const double B = double(d->grid[0]) * d->grid[1] * d->grid[2];
+      *bytes = k.ops->user_bytes_per_block * B;
+      *fp32 = k.ops->user_flops_per_block * B;
       break;
     }
     case SLATE_KIND_GAUSS_FAN2: {
@@ -720,7 +772,10 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
   const auto& g = L.desc.grid;
   if (L.desc.mode == SLATE_MODE_STANDALONE) {
     if (L.ev_start) CK(cudaEventRecord(L.ev_start, Q.stream));
-    CK(ops->launch_standalone(L.args.data(), dim3(g[0], g[1], g[2]), Q.stream));
+    if (ops->launch_standalone_ops)
+      CK(ops->launch_standalone_ops(ops, L.args.data(), dim3(g[0], g[1], g[2]), Q.stream));
+    else
+      CK(ops->launch_standalone(L.args.data(), dim3(g[0], g[1], g[2]), Q.stream));
     Q.last_op_kernel = false;   // standalone kernels do not wait in griddepcontrol.wait: no PDL after them
     if (ev_end) {
       CK(cudaEventRecord(ev_end, Q.stream));
@@ -753,6 +808,7 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     w.ctrl = Q.d_ctrl; w.tc = d_tc_ + slot; w.mirror = d_mirror_ + slot;
     w.cov = reinterpret_cast<uint32_t*>(L.desc.coverage);
     w.rank_of = d_rank_of_;
+    w.ops = ops;
     // PDL: the previous op on the stream is the previous worker of this batch
     w.pdl = in_batch && Q.last_op_kernel && ops->pdl_ok && pdl_enabled_;
     const bool full = Q.lo == 0 && Q.hi == uint32_t(n_sms_ - 1);
@@ -847,6 +903,7 @@ int Server::topup(Queue& Q, Launch& R, std::string* err) {
   w.bound_lo = Q.lo; w.bound_hi = Q.hi; w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
   w.is_topup = 1;
+  w.ops = R.k->ops;
   w.ctrl = Q.d_ctrl; w.tc = d_tc_ + R.slot; w.mirror = d_mirror_ + R.slot;
   w.cov = reinterpret_cast<uint32_t*>(R.desc.coverage);
   w.rank_of = d_rank_of_;
@@ -1022,6 +1079,7 @@ std::string Server::profile_key(const KernelEntry& k, const slate_launch_desc* d
     // one profile per system size: the steps of one elimination share it
     case SLATE_KIND_GAUSS_FAN1:
     case SLATE_KIND_GAUSS_FAN2: s << static_cast<const slate_args_gauss*>(a)->n; break;
+    case SLATE_KIND_USER: s << k.id << ':' << d->grid[0] << 'x' << d->grid[1] << 'x' << d->grid[2]; break;
   }
   return s.str();
 }
@@ -1633,6 +1691,7 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
   w.bound_lo = 0; w.bound_hi = uint32_t(n_sms_ - 1); w.n_ranks = uint32_t(n_sms_);
   w.standby_timeout_ns = standby_timeout_ns_;
   w.ctrl = ctrl; w.mirror = nullptr; w.cov = nullptr; w.rank_of = d_rank_of_;
+  w.ops = k.ops;
   cudaEvent_t e0, e1;
   CK(cudaEventCreate(&e0));
   CK(cudaEventCreate(&e1));

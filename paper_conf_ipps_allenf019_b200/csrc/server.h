@@ -25,6 +25,7 @@ struct KernelEntry {
   slate_kernel_desc desc;
   const KindOps* ops;
   int occ;                      // resident worker CTAs per SM
+  std::unique_ptr<KindOps> own_ops;   // a runtime-compiled user kernel's kind (NEXT-3)
 };
 
 struct Launch {
@@ -103,6 +104,7 @@ class Server {
   int close_queue(uint32_t q, int64_t timeout_us, std::string* err);
 
   int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
+  int register_source(const slate_source_desc* d, uint64_t* out, std::string* err);
   int launch(uint32_t q, uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err);
   int launch_n(uint32_t q, uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err);
   int launch_many(uint32_t q, uint32_t n, const uint64_t* ks, const slate_launch_desc* ds, uint64_t* first,

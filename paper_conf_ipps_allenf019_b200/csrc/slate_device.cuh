@@ -13,11 +13,24 @@
 // retire; grow = waiting CTAs join / a top-up launch adds workers on the new
 // ranks; progress lives only in the counter.  No relaunch (north star).
 #pragma once
-#include <cstdint>
-#include <cuda_runtime.h>
+#include "rtc_types.h"
 #include "kernels.h"
 
 namespace slate {
+
+// Optional per-tenant hooks default to off.
+struct TenantBase {
+  static constexpr bool kHasInit = false;   // cta_init(smem): once per CTA before the first block
+  static constexpr bool kHasTask = false;   // cta_task(args, g, n, smem): task [g, g+n) of a 1-D grid at once
+  static constexpr bool kLookahead = false; // cta_task2(args, g, n, g2, n2, smem): run task [g, g+n) of a
+                                            // 1-D grid knowing the CTA's next task [g2, g2+n2) (n2 = 0: none)
+  static constexpr uint32_t kMaxIters = 10; // cap of the automatic task size (P:L303 default 10)
+  static constexpr int kMinBlocks = 1;      // __launch_bounds__ min blocks per SM of the worker
+  static constexpr bool kSpeculative = false; // fetch the next task while this one runs (+registers)
+  static constexpr uint32_t kTasksPerWorker = 8; // auto task size aims at >= this many tasks per worker
+  static constexpr bool kHasFini = false;   // cta_fini(smem): once per CTA before it exits
+  static constexpr bool kLateCtrl = false;  // read the resize word at the boundary, not at task start
+};
 
 // ------------------------------------------------------------------ PTX helpers
 __device__ __forceinline__ uint32_t smid() {

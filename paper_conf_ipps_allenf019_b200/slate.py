@@ -26,6 +26,7 @@ EINVAL, ENOMEM, ECUDA, EIPC, ETIMEDOUT, ENOTFOUND, ESTATE, EUNSUPPORTED = -1, -2
 KIND_TRIAD, KIND_COPY, KIND_SGEMM_NAIVE, KIND_SPMV_CSR, KIND_BLACKSCHOLES, KIND_STENCIL2D, KIND_GEMM_BF16 = range(1, 8)
 # the paper's Tab II apps (TR, MM, RG, GS = Fan1 + Fan2; BS is KIND_BLACKSCHOLES with one scenario)
 KIND_TRANSPOSE, KIND_SGEMM_TILED, KIND_QRNG, KIND_GAUSS_FAN1, KIND_GAUSS_FAN2 = range(8, 13)
+KIND_USER = 13   # a user kernel compiled at run time (register_source, NEXT-3)
 KFLAG_COVERAGE = 1
 PLACE_AUTO, PLACE_SOLO, PLACE_CORUN = 0, 1, 2
 MODE_SLATE, MODE_STANDALONE = 0, 1
@@ -80,6 +81,12 @@ class ArgsQrng(ctypes.Structure):
 
 class ArgsGauss(ctypes.Structure):
     _fields_ = [("a", c_u64), ("b", c_u64), ("m", c_u64), ("n", c_u32), ("t", c_u32)]
+
+
+class SourceDesc(ctypes.Structure):
+    _fields_ = [("abi_version", c_u32), ("block_threads", c_u32), ("smem_bytes", c_u32), ("args_size", c_u32),
+                ("iters", c_u32), ("pad_", c_u32), ("source", ctypes.c_char_p), ("kernel_name", ctypes.c_char_p),
+                ("bytes_per_block", c_f64), ("flops_per_block", c_f64)]
 
 
 class Info(ctypes.Structure):
@@ -151,6 +158,9 @@ for _name, _args in [
     ("slate_set_policy", [ctypes.c_void_p, c_u32]),
     ("slate_launch_n", [ctypes.c_void_p, c_u64, _P(LaunchDesc), c_u32, _P(c_u64)]),
     ("slate_launch_many", [ctypes.c_void_p, c_u32, _P(c_u64), _P(LaunchDesc), _P(c_u64)]),
+    ("slate_register_source", [ctypes.c_void_p, _P(SourceDesc), _P(c_u64)]),
+    ("slate_transform_source", [ctypes.c_char_p, ctypes.c_char_p, c_u32, c_u32, ctypes.c_char_p, ctypes.c_size_t,
+                                _P(ctypes.c_size_t)]),
 ]:
     getattr(_lib, _name).restype = c_i32
     getattr(_lib, _name).argtypes = _args
@@ -176,7 +186,8 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_register_kernel", "slate_launch", "slate_resize", "slate_sync", "slate_profile", "slate_query",
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
-            "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters"]
+            "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters",
+            "slate_register_source", "slate_transform_source"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -237,6 +248,16 @@ class Session:
 
     def unshare_buffer(self, handle):
         self._check(_lib.slate_unshare_buffer(self._h, handle), "slate_unshare_buffer")
+
+    def register_source(self, source, name, args_struct, threads=256, smem=0, iters=0, bytes_per_block=0.0,
+                        flops_per_block=0.0):
+        """A user CUDA kernel compiled at run time (NEXT-3); `args_struct` is the
+        ctypes Structure type of its parameters, in declaration order."""
+        d = SourceDesc(ABI_VERSION, threads, smem, ctypes.sizeof(args_struct), iters, 0, source.encode(), name.encode(),
+                       bytes_per_block, flops_per_block)
+        k = c_u64()
+        self._check(_lib.slate_register_source(self._h, ctypes.byref(d), ctypes.byref(k)), "slate_register_source")
+        return k.value
 
     def register_kernel(self, kind, iters=0, flags=0):
         d = KernelDesc(ABI_VERSION, kind, iters, flags)
@@ -342,6 +363,17 @@ def fluid_corun(curve_a, work_a, curve_b, work_b, n_sms, step=2, lo_b=0, hi_b=0,
     r = _lib.slate_fluid_corun(sa, ta, na, work_a, sb, tb, nb, work_b, n_sms, step, lo_b, hi_b, min_gain,
                                ctypes.byref(s), ctypes.byref(g))
     return bool(r), s.value, g.value
+
+
+def transform_source(source, name, threads=256, smem=0):
+    """The generated worker source for a user kernel (no GPU needed)."""
+    n = ctypes.c_size_t()
+    st = _lib.slate_transform_source(source.encode(), name.encode(), threads, smem, None, 0, ctypes.byref(n))
+    if st != OK:
+        raise SlateError(st, "slate_transform_source")
+    buf = ctypes.create_string_buffer(n.value + 1)
+    _lib.slate_transform_source(source.encode(), name.encode(), threads, smem, buf, n.value + 1, ctypes.byref(n))
+    return buf.value.decode()
 
 
 def choose_iters(solo_ms, occ, n_sms, blocks, cap, budget_us=20.0):
