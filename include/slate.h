@@ -415,6 +415,17 @@ uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n,
  * gets two tasks), clamped to [1, cap].  The server uses it for launches of
  * kernels registered with iters 0 once their shape has been profiled. */
 uint32_t slate_choose_iters(double solo_ms, uint32_t occ, uint32_t n_sms, uint32_t B, uint32_t cap, double budget_us);
+/* NEXT-4, k co-runners: the fluid-model makespan of k jobs (curve i: npts[i]
+ * points sms[i][*] -> ms[i][*], job times) on disjoint shares, a finishing
+ * job's SMs going to the unfinished one with the most time left; and the
+ * shares (multiples of step, each >= step, summing to n_sms) minimising it,
+ * by exhaustive search (returns the makespan, -1 if n_sms / step < k).  Pure
+ * functions for the selector and its tests; the server co-runs at most two
+ * queues (Q13, Q37). */
+double slate_corun_makespan_k(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, uint32_t k,
+                              const uint32_t* shares);
+double slate_choose_split_k(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, uint32_t k,
+                            uint32_t n_sms, uint32_t step, uint32_t* shares_out);
 /* Reading Q31 (the B200 selector): should kernel B co-run with the active A
  * although Tab I says solo?  Job curves are `work` launches of each kernel
  * (the launches queued or running) back to back, time = work * curve(s); the

@@ -3,6 +3,7 @@
 // DESIGN.md).  Pure host functions, exported through the C ABI so they can be
 // checked against the oracle without a GPU.
 #include <cmath>
+#include <functional>
 #include <cstdint>
 #include <limits>
 #include <vector>
@@ -128,6 +129,82 @@ uint32_t slate_choose_iters(double solo_ms, uint32_t occ, uint32_t n_sms, uint32
   const double t_block_us = std::max(solo_ms * 1e3 * workers / B, 1e-3);
   const double it = std::min(std::floor(budget_us / t_block_us), std::floor(B / (2.0 * workers)));
   return uint32_t(std::max(1.0, std::min(double(cap ? cap : 1), it)));
+}
+
+// NEXT-4: k co-runners (oracle selector.corun_makespan_k / choose_split_k).
+// curve i: npts[i] points sms[i][*] -> ms[i][*].
+static double makespan_k(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, uint32_t k,
+                         const uint32_t* shares) {
+  std::vector<double> left(k, 1.0), s(k);
+  std::vector<bool> alive(k, true);
+  for (uint32_t i = 0; i < k; ++i) s[i] = shares[i];
+  double t = 0;
+  for (;;) {
+    double dt = std::numeric_limits<double>::infinity();
+    bool any = false;
+    std::vector<double> rate(k, 0.0);
+    for (uint32_t i = 0; i < k; ++i)
+      if (alive[i]) {
+        any = true;
+        rate[i] = 1.0 / interp(sms[i], ms[i], npts[i], s[i]);
+        dt = std::min(dt, left[i] / rate[i]);
+      }
+    if (!any) return t;
+    t += dt;
+    double freed = 0;
+    std::vector<uint32_t> done;
+    for (uint32_t i = 0; i < k; ++i)
+      if (alive[i]) {
+        if (left[i] - rate[i] * dt <= 1e-12) done.push_back(i);
+        left[i] = std::max(0.0, left[i] - rate[i] * dt);
+      }
+    for (uint32_t i : done) {
+      alive[i] = false;
+      freed += s[i];
+      s[i] = 0;
+    }
+    if (freed > 0) {
+      int best = -1;
+      double most = -1;
+      for (uint32_t i = 0; i < k; ++i)
+        if (alive[i]) {
+          const double rem = left[i] * interp(sms[i], ms[i], npts[i], s[i]);
+          if (rem > most) { most = rem; best = int(i); }
+        }
+      if (best >= 0) s[best] += freed;
+    }
+  }
+}
+
+double slate_corun_makespan_k(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, uint32_t k,
+                              const uint32_t* shares) {
+  return makespan_k(sms, ms, npts, k, shares);
+}
+
+double slate_choose_split_k(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, uint32_t k,
+                            uint32_t n_sms, uint32_t step, uint32_t* shares_out) {
+  if (k == 0 || step == 0 || n_sms / step < k) return -1.0;
+  const uint32_t units = n_sms / step;
+  std::vector<uint32_t> u(k, 1), best;
+  double best_t = std::numeric_limits<double>::infinity();
+  // enumerate compositions of `units` into k positive parts, lexicographic order
+  std::vector<uint32_t> sh(k);
+  std::function<void(uint32_t, uint32_t)> rec = [&](uint32_t pos, uint32_t rest) {
+    if (pos == k - 1) {
+      u[pos] = rest;
+      for (uint32_t i = 0; i < k; ++i) sh[i] = u[i] * step;
+      const double t = makespan_k(sms, ms, npts, k, sh.data());
+      if (t < best_t - 1e-12) { best_t = t; best = sh; }
+      return;
+    }
+    for (uint32_t v = 1; v + (k - 1 - pos) <= rest; ++v) {
+      u[pos] = v;
+      rec(pos + 1, rest - v);
+    }
+  };
+  rec(0, units);
+  for (uint32_t i = 0; i < k; ++i) shares_out[i] = best[i];
+  return best_t;
 }
 
 }  // extern "C"

@@ -175,6 +175,10 @@ _lib.slate_choose_split.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c
                                     c_u32, _P(c_f64)]
 _lib.slate_saturation_sms.restype = c_u32
 _lib.slate_saturation_sms.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_u32, c_f64]
+_lib.slate_corun_makespan_k.restype = c_f64
+_lib.slate_corun_makespan_k.argtypes = [ctypes.c_void_p, ctypes.c_void_p, _P(c_u32), c_u32, _P(c_u32)]
+_lib.slate_choose_split_k.restype = c_f64
+_lib.slate_choose_split_k.argtypes = [ctypes.c_void_p, ctypes.c_void_p, _P(c_u32), c_u32, c_u32, c_u32, _P(c_u32)]
 _lib.slate_choose_iters.restype = c_u32
 _lib.slate_choose_iters.argtypes = [c_f64, c_u32, c_u32, c_u32, c_u32, c_f64]
 _lib.slate_fluid_corun.restype = ctypes.c_int
@@ -187,7 +191,7 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
             "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters",
-            "slate_register_source", "slate_transform_source"]
+            "slate_register_source", "slate_transform_source", "slate_corun_makespan_k", "slate_choose_split_k"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -363,6 +367,28 @@ def fluid_corun(curve_a, work_a, curve_b, work_b, n_sms, step=2, lo_b=0, hi_b=0,
     r = _lib.slate_fluid_corun(sa, ta, na, work_a, sb, tb, nb, work_b, n_sms, step, lo_b, hi_b, min_gain,
                                ctypes.byref(s), ctypes.byref(g))
     return bool(r), s.value, g.value
+
+
+def _curves_k(curves):
+    keep = [_curve(c) for c in curves]
+    sms = (ctypes.POINTER(c_u32) * len(curves))(*[ctypes.cast(a, ctypes.POINTER(c_u32)) for a, _, _ in keep])
+    ms = (ctypes.POINTER(c_f64) * len(curves))(*[ctypes.cast(b, ctypes.POINTER(c_f64)) for _, b, _ in keep])
+    npts = (c_u32 * len(curves))(*[n for _, _, n in keep])
+    return keep, sms, ms, npts
+
+
+def corun_makespan_k(curves, shares):
+    keep, sms, ms, npts = _curves_k(curves)
+    return _lib.slate_corun_makespan_k(ctypes.cast(sms, ctypes.c_void_p), ctypes.cast(ms, ctypes.c_void_p), npts,
+                                       len(curves), (c_u32 * len(shares))(*shares))
+
+
+def choose_split_k(curves, n_sms, step=2):
+    keep, sms, ms, npts = _curves_k(curves)
+    out = (c_u32 * len(curves))()
+    t = _lib.slate_choose_split_k(ctypes.cast(sms, ctypes.c_void_p), ctypes.cast(ms, ctypes.c_void_p), npts,
+                                  len(curves), n_sms, step, out)
+    return list(out), t
 
 
 def transform_source(source, name, threads=256, smem=0):

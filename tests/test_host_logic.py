@@ -141,3 +141,20 @@ def test_choose_iters_closed_forms(S):
     assert S.choose_iters(0.5, 8, 148, 100, 10, 20.0) == 1
     # a longer budget buys longer tasks, linearly
     assert S.choose_iters(0.0655, 4, 148, 8192, 10, 40.0) == 6
+
+
+def test_k_way_split_matches_oracle(S):
+    """slate_choose_split_k / slate_corun_makespan_k == oracle selector (random curves)."""
+    rng = random.Random(170)
+    for trial in range(6):
+        k = 3 if trial % 2 else 2
+        curves = []
+        for _ in range(k):
+            t148 = rng.uniform(0.5, 3.0)
+            curves.append({148: t148, 74: t148 * rng.uniform(1.05, 2.0), 37: t148 * rng.uniform(2.1, 4.0)})
+        n, step = 148, 4 if k == 3 else 2
+        s_c, t_c = S.choose_split_k(curves, n, step)
+        s_o, t_o = OS.choose_split_k(curves, n, step)
+        assert s_c == s_o and abs(t_c - t_o) < 1e-9 * t_o
+        shares = s_o
+        assert abs(S.corun_makespan_k(curves, shares) - OS.corun_makespan_k(curves, shares)) < 1e-9 * t_o

@@ -150,3 +150,30 @@ def test_fluid_corun_reading_q31():
     assert not ok and g < 1.05
     # work scales the jobs: 10 launches of A against 10 of B is the 1-vs-1 decision
     assert S.fluid_corun(lin, 10, sat, 10, n)[1:] == pytest.approx(S.fluid_corun(lin, 1, sat, 1, n)[1:])
+
+
+# ------------------------------------------------------------------ k-way split (NEXT-4)
+def test_k_way_makespan_closed_forms():
+    n = 48
+    lin = {s: 48.0 / s for s in (6, 12, 24, 48)}          # perfectly linear: T(s) = 48 / s, T(n) = 1
+    # work conservation: with linear curves and SMs handed on, any split of k jobs
+    # finishes at the sum of their full-chip times
+    for shares in ([24, 24], [6, 42], [12, 12, 24], [6, 18, 12, 12]):
+        assert abs(S.corun_makespan_k([lin] * len(shares), shares) - len(shares)) < 1e-9
+    # two co-runners: the k-way model is the 2-way one (pinned separately)
+    a = {148: 1.0, 74: 1.3, 37: 2.4}
+    b = {148: 2.0, 74: 2.1, 37: 2.9}
+    for s in (20, 74, 100):
+        assert abs(S.corun_makespan_k([a, b], [148 - s, s]) - S.corun_makespan(a, b, 148, s)) < 1e-9
+    s2, t2 = S.choose_split(a, b, 148)
+    sk, tk = S.choose_split_k([a, b], 148)
+    assert sk == [148 - s2, s2] and abs(tk - t2) < 1e-9
+
+
+def test_k_way_saturating_jobs_overlap_fully():
+    # three jobs that each reach full speed on a third of the chip run side by side
+    n = 48
+    sat = {16: 1.0, 48: 1.0}                              # T(s) = 1 for s >= 16 (and s/16 below)
+    shares, t = S.choose_split_k([sat, sat, sat], n, step=4)
+    assert shares == [16, 16, 16] and abs(t - 1.0) < 1e-9
+    assert S.corun_makespan_k([sat] * 3, [8, 20, 20]) > 1.0 + 1e-9
