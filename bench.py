@@ -555,6 +555,12 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
         roof = {"kernel": kname, "bound": "hbm", "achieved": round(ach, 1), "peak": peak_hbm,
                 "unit": "GB/s", "frac": round(ach / peak_hbm, 4), "peak_source": "MEASURED_PEAKS.json hbm_gbs"}
     roof["avg_launch_ms"] = round(avg, 5)
+    # in the co-run the kernel holds only its share of the SMs (the split): its
+    # rate against that share of the peak (the job also grows to every SM once
+    # its co-runner drains, so this is a lower bound on the share's use)
+    share = (w.n_sms - w.split) if top == w.a.name else w.split
+    roof["corun_sms"] = int(share)
+    roof["frac_of_share"] = round(roof["frac"] * w.n_sms / max(share, 1), 4)
     # the same kernel solo on every SM (the Slate-sequential schedule): in the
     # co-run it holds only its share of the SMs, so its per-launch rate there
     # is not its roofline position
