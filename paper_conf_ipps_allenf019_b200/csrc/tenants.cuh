@@ -370,17 +370,18 @@ struct BlackScholes : TenantBase {
     return d;
   }
   __device__ __forceinline__ static f2 abs2(f2 a) { return a & 0x7fffffff7fffffffull; }
-  __device__ __forceinline__ static f2 poly2(f2 K) {
-    const f2 A1 = pk(0.31938153f, 0.31938153f), A2 = pk(-0.356563782f, -0.356563782f),
-             A3 = pk(1.781477937f, 1.781477937f), A4 = pk(-1.821255978f, -1.821255978f),
-             A5 = pk(1.330274429f, 1.330274429f);
+  // the A&S polynomial with 1/sqrt(2 pi) folded into its coefficients
+  __device__ __forceinline__ static f2 poly2r(f2 K) {
+    const float R = 0.39894228040143267794f;
+    const f2 A1 = pk(0.31938153f * R, 0.31938153f * R), A2 = pk(-0.356563782f * R, -0.356563782f * R),
+             A3 = pk(1.781477937f * R, 1.781477937f * R), A4 = pk(-1.821255978f * R, -1.821255978f * R),
+             A5 = pk(1.330274429f * R, 1.330274429f * R);
     return mul2(K, fma2(K, fma2(K, fma2(K, fma2(K, A5, A4), A3), A2), A1));
   }
   // 4 options as two packed pairs (0,1) and (2,3); the per-option setup and the
   // final mean are price<4>'s scalar code
   __device__ __forceinline__ static void price4_x2(const float (&S)[4], const float (&X)[4], const float (&T)[4], float r,
                                                    const float* sig, uint32_t P, float (&call)[4], float (&put)[4]) {
-    const float RSQRT2PI = 0.39894228040143267794f;
     float sqt[4], rsqt[4], lsx[4], xd[4], sxd[4];
 #pragma unroll
     for (int o = 0; o < 4; ++o) {
@@ -402,8 +403,8 @@ struct BlackScholes : TenantBase {
       SXD[h] = pk(sxd[2 * h], sxd[2 * h + 1]);
       CS[h] = pk(0.f, 0.f);
     }
-    const f2 ONE = pk(1.0f, 1.0f), AK = pk(0.2316419f, 0.2316419f), MH = pk(-0.5f, -0.5f),
-             L2E = pk(1.44269504088896341f, 1.44269504088896341f), RS = pk(RSQRT2PI, RSQRT2PI);
+    const float HL2E = -0.5f * 1.44269504088896341f;   // exp(-d^2/2) = 2^(d^2 * -log2(e)/2)
+    const f2 ONE = pk(1.0f, 1.0f), AK = pk(0.2316419f, 0.2316419f), MHL = pk(HL2E, HL2E);
     for (uint32_t p = 0; p < P; ++p) {
       const float sg = __ldg(sig + p);
       const float rsg = rcp(sg);
@@ -415,16 +416,19 @@ struct BlackScholes : TenantBase {
         const f2 d1 = mul2(fma2(HS2, TT[h], LSX[h]), mul2(RSG, RSQT[h]));
         const f2 d2 = sub2(d1, sst);
         const f2 u1 = fma2(AK, abs2(d1), ONE), u2 = fma2(AK, abs2(d2), ONE);
-        float uu0, uu1, a0, a1;
-        up(mul2(u1, u2), uu0, uu1);
-        const f2 q = pk(rcp(uu0), rcp(uu1));
-        up(mul2(mul2(MH, mul2(d1, d1)), L2E), a0, a1);
+        // the two A&S K = 1/u by two reciprocals: the MUFU pipe has the slack
+        // the FP32 pipe (the limit) lacks -- one more MUFU op, three fewer FP32
+        float u10, u11, u20, u21, a0, a1;
+        up(u1, u10, u11);
+        up(u2, u20, u21);
+        const f2 k1 = pk(rcp(u10), rcp(u11)), k2 = pk(rcp(u20), rcp(u21));
+        up(mul2(mul2(d1, d1), MHL), a0, a1);
         float x0, x1;
         asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x0) : "f"(a0));
         asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x1) : "f"(a1));
-        const f2 e1 = mul2(RS, pk(x0, x1));
-        const f2 c1 = mul2(e1, poly2(mul2(u2, q)));
-        const f2 c2 = mul2(mul2(e1, SXD[h]), poly2(mul2(u1, q)));
+        const f2 e1 = pk(x0, x1);                       // exp(-d1^2/2); 1/sqrt(2 pi) is in poly2r
+        const f2 c1 = mul2(e1, poly2r(k1));
+        const f2 c2 = mul2(mul2(e1, SXD[h]), poly2r(k2));
         const f2 o1 = sub2(ONE, c1), o2 = sub2(ONE, c2);
         float d10, d11, d20, d21, c10, c11, c20, c21, o10, o11, o20, o21;
         up(d1, d10, d11);
