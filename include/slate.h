@@ -250,6 +250,7 @@ slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel*
  * (args_size bytes).  bytes_per_block / flops_per_block declare its work for
  * slate_profile's classification (0 if unknown).  In-process sessions only
  * (through an endpoint the server cannot rewrite pointers it cannot see).
+ * flags: SLATE_KFLAG_COVERAGE as for slate_register_kernel.
  * Errors: EINVAL (no such kernel in the source, bad sizes), EUNSUPPORTED (no
  * NVRTC, or an endpoint session), ECUDA (compile or load failed; the compiler
  * log is in slate_last_error). */
@@ -259,7 +260,7 @@ typedef struct {
   uint32_t smem_bytes;
   uint32_t args_size;
   uint32_t iters;              /* task size; 0 = automatic */
-  uint32_t pad_;
+  uint32_t flags;              /* SLATE_KFLAG_COVERAGE: launches may pass a coverage log */
   const char* source;
   const char* kernel_name;
   double bytes_per_block, flops_per_block;

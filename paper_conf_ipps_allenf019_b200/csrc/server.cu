@@ -389,6 +389,7 @@ int Server::register_source(const slate_source_desc* d, uint64_t* out, std::stri
   k->desc.abi_version = SLATE_ABI_VERSION;
   k->desc.kind = SLATE_KIND_USER;
   k->desc.iters = d->iters;
+  k->desc.flags = d->flags & SLATE_KFLAG_COVERAGE;
   k->occ = occ;
   k->ops = ops.get();
   k->own_ops = std::move(ops);

@@ -85,7 +85,7 @@ class ArgsGauss(ctypes.Structure):
 
 class SourceDesc(ctypes.Structure):
     _fields_ = [("abi_version", c_u32), ("block_threads", c_u32), ("smem_bytes", c_u32), ("args_size", c_u32),
-                ("iters", c_u32), ("pad_", c_u32), ("source", ctypes.c_char_p), ("kernel_name", ctypes.c_char_p),
+                ("iters", c_u32), ("flags", c_u32), ("source", ctypes.c_char_p), ("kernel_name", ctypes.c_char_p),
                 ("bytes_per_block", c_f64), ("flops_per_block", c_f64)]
 
 
@@ -254,10 +254,10 @@ class Session:
         self._check(_lib.slate_unshare_buffer(self._h, handle), "slate_unshare_buffer")
 
     def register_source(self, source, name, args_struct, threads=256, smem=0, iters=0, bytes_per_block=0.0,
-                        flops_per_block=0.0):
+                        flops_per_block=0.0, flags=0):
         """A user CUDA kernel compiled at run time (NEXT-3); `args_struct` is the
         ctypes Structure type of its parameters, in declaration order."""
-        d = SourceDesc(ABI_VERSION, threads, smem, ctypes.sizeof(args_struct), iters, 0, source.encode(), name.encode(),
+        d = SourceDesc(ABI_VERSION, threads, smem, ctypes.sizeof(args_struct), iters, flags, source.encode(), name.encode(),
                        bytes_per_block, flops_per_block)
         k = c_u64()
         self._check(_lib.slate_register_source(self._h, ctypes.byref(d), ctypes.byref(k)), "slate_register_source")

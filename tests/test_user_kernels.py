@@ -3,7 +3,8 @@ source is scanned, turned into a device body, wrapped into the slate worker
 and the original kernel, and compiled with NVRTC.  CPU tests check the
 transformation and that NVRTC compiles its output for sm_100a (no GPU needed);
 the -m gpu test runs a 2-D user kernel through the worker against its original
-kernel (bit-exact), numpy (exact: integer inputs) and the exact counters."""
+kernel (bit-exact), numpy (exact: integer inputs), the exact counters and the
+coverage log (every original block exactly once)."""
 import ctypes
 import os
 
@@ -97,12 +98,12 @@ def test_user_kernel_through_the_worker(S):
         n = s.info()["num_sms"]
         B = grid[0] * grid[1]
         for iters in (1, 3):
-            k = s.register_source(USER_SRC, "axpb2d", Args, threads=T, iters=iters)
+            k = s.register_source(USER_SRC, "axpb2d", Args, threads=T, iters=iters, flags=S.KFLAG_COVERAGE)
             for sm in [(0, n - 1), (5, 5 + n // 4)]:
                 yd.zero_()
                 cov = torch.zeros(B, dtype=torch.int32, device="cuda:0")
                 torch.cuda.synchronize()
-                lid = s.launch(k, args, grid, placement=S.PLACE_CORUN, sm=sm, coverage=None)
+                lid = s.launch(k, args, grid, placement=S.PLACE_CORUN, sm=sm, coverage=cov)
                 s.sync(lid)
                 torch.cuda.synchronize()
                 assert torch.equal(yd, ref), (iters, sm)
@@ -110,3 +111,4 @@ def test_user_kernel_through_the_worker(S):
                 ex = OT.expected_counters(B, iters)
                 assert (q["blocks_done"], q["tasks_done"], q["next_clamped"]) == \
                     (ex["blocks_done"], ex["tasks_done"], ex["next_clamped"])
+                assert q["coverage_ok"] == 1 and np.array_equal(cov.cpu().numpy(), ex["coverage"].astype(np.int32))
