@@ -1442,12 +1442,14 @@ void Server::resolve_resizes(Queue& Q, double t, const Launch* ended) {
       }
       if (it->kind == 1) break;   // only the oldest running launch can hold out-of-range workers
     }
+    bool via_end = false;
     if (!done && ended && it->kind == 1 && ended->slot >= 0) {
       done_ns = h_mirror_[ended->slot].done;
-      done = true;
+      done = via_end = true;
     }
     if (done) {
       record_resize(*it, done_ns, t);
+      if (std::getenv("SLATE_DEBUG") && via_end) fprintf(stderr, "[slate]   (resolved by the launch's end)\n");
       it = Q.pending_resize.erase(it);
     } else {
       ++it;
