@@ -699,7 +699,7 @@ def run_slate(args, world, rank, local):
             sA.close()
             sB.close()
             sA = sB = None
-            c4 = c4_bench.run(max(3, args.steps // 2))
+            c4 = c4_bench.run(max(3, args.steps // 2), local)
         except Exception as e:   # reported, never fatal for the headline
             c4 = {"error": str(e)[:300]}
 

@@ -58,11 +58,13 @@ def build(kind, S, dev):
     return k, args, grid, keep
 
 
-def client(endpoint, kind, steps, go_path):
+def client(endpoint, kind, steps, go_path, device=0):
     """One tenant process: profile, then `steps` jobs, each released by the parent."""
     from paper_conf_ipps_allenf019_b200 import slate as S
+    import torch
+    torch.cuda.set_device(device)
     s = S.Session(endpoint)
-    k, args, grid, keep = build(kind, S, "cuda:0")
+    k, args, grid, keep = build(kind, S, "cuda:%d" % device)
     for t in keep:
         s.share_buffer(t)
     kid = s.register_kernel(k)
@@ -88,11 +90,13 @@ def client(endpoint, kind, steps, go_path):
     s.close()
 
 
-def sequential(endpoint):
+def sequential(endpoint, device=0):
     """The four jobs back to back with the original kernels, one client (vanilla CUDA)."""
     from paper_conf_ipps_allenf019_b200 import slate as S
+    import torch
+    torch.cuda.set_device(device)
     s = S.Session(endpoint)
-    built = {k: build(k, S, "cuda:0") for k in JOBS}
+    built = {k: build(k, S, "cuda:%d" % device) for k in JOBS}
     for k, (_, _, _, keep) in built.items():
         for t in keep:
             s.share_buffer(t)
@@ -117,10 +121,10 @@ def sequential(endpoint):
     return times[len(times) // 2]
 
 
-def run(steps):
-    """Run the C4 measurement (daemon + 4 client processes); returns the result dict."""
+def run(steps, device=0):
+    """Run the C4 measurement (daemon + 4 client processes) on GPU `device`; returns the result dict."""
     from paper_conf_ipps_allenf019_b200 import slate as S
-    cmd = [sys.executable, __file__, "--steps", str(steps)]
+    cmd = [sys.executable, __file__, "--steps", str(steps), "--device", str(device)]
     out = subprocess.run(cmd, capture_output=True, text=True, timeout=900)
     lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
     if not lines:
@@ -132,22 +136,24 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--client", nargs=3)
+    ap.add_argument("--device", type=int, default=0)
     a = ap.parse_args()
     if a.client:
-        client(a.client[0], a.client[1], a.steps, a.client[2])
+        client(a.client[0], a.client[1], a.steps, a.client[2], a.device)
         return
     from paper_conf_ipps_allenf019_b200 import slate as S
     ep = "/slate-c4-%d" % os.getpid()
     go = "/tmp/slate_c4_go_%d" % os.getpid()
-    d = subprocess.Popen([S.DAEMON, "--endpoint", ep], stderr=subprocess.DEVNULL)
+    d = subprocess.Popen([S.DAEMON, "--device", str(a.device), "--endpoint", ep], stderr=subprocess.DEVNULL)
     for _ in range(300):
         try:
             S.Session(ep).close()
             break
         except S.SlateError:
             time.sleep(0.2)
-    seq_ms, solo = sequential(ep)
-    ps = {k: subprocess.Popen([sys.executable, __file__, "--steps", str(a.steps), "--client", ep, k, go],
+    seq_ms, solo = sequential(ep, a.device)
+    ps = {k: subprocess.Popen([sys.executable, __file__, "--steps", str(a.steps), "--device", str(a.device),
+                               "--client", ep, k, go],
                               stdout=subprocess.PIPE, text=True) for k in JOBS}
     for p in ps.values():
         assert "READY" in p.stdout.readline()
