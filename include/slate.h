@@ -349,7 +349,8 @@ typedef struct {
   uint64_t t_enter_ns;     /* %globaltimer when the first worker CTA started (device clock; 0 if standalone) */
   uint64_t t_exit_ns;      /* %globaltimer when the last worker CTA that ran a task exited (0 unless the
                               library is built with SLATE_DIAG_EXIT) */
-  uint32_t n_superseded;   /* shrinks overtaken by a grow before they completed (not timed) */
+  uint32_t n_superseded;   /* resizes with no completion to time: shrinks overtaken by a grow before
+                              they completed, grows of a queue with no block left to run */
   uint32_t pad2_;
 } slate_launch_info;
 

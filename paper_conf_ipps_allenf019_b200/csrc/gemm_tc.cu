@@ -64,6 +64,7 @@ struct Params {
   CUtensorMap tma_c;     // fp32 C, boxes of 32 x 32, SWIZZLE_128B (epilogue TMA store)
   slate_args_gemm args;
   uint32_t gx, gy, B, iters, occ, bound_lo, bound_hi, n_ranks, standby_timeout_ns, base_epoch;
+  uint32_t is_topup, gate_first;   // as WorkerParams (slate_device.cuh)
   const uint64_t* ctrl;
   TaskCtl* tc;
   HostMirror* mirror;
@@ -241,6 +242,9 @@ __device__ bool pair_prologue(const P& p, uint32_t r0, uint32_t r1, uint64_t& c_
   TaskCtl* tc = p.tc;
   uint64_t t0 = 0;
   uint32_t backoff = 256;
+  if (p.gate_first) {   // top-up of a launch that has no start event: wait until it started
+    while (ld_relaxed_u64(&tc->t_first) == 0 && ld_relaxed_u32(&tc->next) < p.B) __nanosleep(512);
+  }
   for (;;) {
     const uint64_t c = ld_acquire_u64(p.ctrl);
     if (ld_relaxed_u32(&tc->next) >= p.B) return false;
@@ -316,7 +320,10 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       st_cluster(mapa(&S.go, 1), go);
     }
     cluster_sync();
-    if (!S.go) return;
+    if (!S.go) {
+      if (threadIdx.x == 0) leave_main(p);   // every CTA of the grid counts (slate_device.cuh)
+      return;
+    }
   }
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&p.tma_a);
@@ -623,6 +630,9 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       }
       if (S.retired) check_shrink_done(p, c, lane);
     }
+    // after the shrink bookkeeping; tiles are counted done one by one by the
+    // epilogue, so the CTA completing the grid can wait for a top-up's tiles
+    if (threadIdx.x == 0) leave_main(p);
   }
 }
 
@@ -702,6 +712,8 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.bound_lo = w.bound_lo; p.bound_hi = w.bound_hi; p.n_ranks = w.n_ranks;
   p.standby_timeout_ns = w.standby_timeout_ns;
   p.base_epoch = w.base_epoch;
+  p.is_topup = w.is_topup;
+  p.gate_first = w.gate_first;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   return launch_pairs(reinterpret_cast<const void*>(&gemm_kernel<true>), p, dim3((grid + 1) & ~1u), st);
 }
@@ -730,6 +742,7 @@ KindOps gemm_tc_ops() {
   o.tile_m = gemm::kTileM;
   o.tile_n = gemm::BN;
   o.launch_worker = &gemm::launch_worker;
+  o.topup_anytime = true;   // leave_main: the CTA completing the grid waits for every tile
   o.launch_standalone = &gemm::launch_standalone;
   return o;
 }

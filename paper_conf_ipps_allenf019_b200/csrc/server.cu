@@ -867,6 +867,7 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   if (Q.issued.empty() || !Q.pending.empty() || !Q.deferred.empty()) {
     if (dbg) fprintf(stderr, "[slate] grow: no top-up (issued %zu pending %zu deferred %zu)\n", Q.issued.size(),
                      Q.pending.size(), Q.deferred.size());
+    if (Q.pending.empty() && Q.deferred.empty()) drop_idle_grow(Q);
     return SLATE_OK;
   }
   for (size_t i = 0; i + 1 < Q.issued.size(); ++i) {
@@ -880,9 +881,25 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   if (R.state != 1 || R.slot < 0 || R.desc.mode == SLATE_MODE_STANDALONE) return SLATE_OK;
   if (h_mirror_[R.slot].done) {
     if (dbg) fprintf(stderr, "[slate] grow: no top-up (the launch finished its blocks)\n");
+    drop_idle_grow(Q);
     return SLATE_OK;
   }
   return topup(Q, R, err);
+}
+
+// A grow when the queue has no block left to run (its launches finished their
+// blocks, nothing queued): no worker can join until the client's next launch,
+// so the grow has no completion of its own to time -- counted with the
+// superseded resizes (n_superseded), not as a latency.
+void Server::drop_idle_grow(Queue& Q) {
+  for (auto it = Q.pending_resize.rbegin(); it != Q.pending_resize.rend(); ++it) {
+    if (it->kind == 2 && it->epoch == Q.epoch) {
+      auto li = launches_.find(it->lid);
+      if (li != launches_.end()) li->second->n_superseded += 1;
+      Q.pending_resize.erase(std::next(it).base());
+      return;
+    }
+  }
 }
 
 // a top-up grid for launch R on the queue's current range, sharing R's counter

@@ -126,6 +126,7 @@ class Server {
   int write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool immediate, std::string* err);
   int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
   int topup(Queue& Q, Launch& R, std::string* err);
+  void drop_idle_grow(Queue& Q);
   void close_batch(Queue& Q, cudaEvent_t end, bool closed_by_launch = false);
   void launch_times(const Launch& L, double* start, double* end) const;
   bool batch_more_ = false;

@@ -144,7 +144,9 @@ def main():
     from paper_conf_ipps_allenf019_b200 import slate as S
     ep = "/slate-c4-%d" % os.getpid()
     go = "/tmp/slate_c4_go_%d" % os.getpid()
-    d = subprocess.Popen([S.DAEMON, "--device", str(a.device), "--endpoint", ep], stderr=subprocess.DEVNULL)
+    log = os.environ.get("C4_DAEMON_LOG")           # diagnostics: the daemon's stderr (SLATE_DEBUG output)
+    d = subprocess.Popen([S.DAEMON, "--device", str(a.device), "--endpoint", ep],
+                         stderr=open(log, "w") if log else subprocess.DEVNULL)
     for _ in range(300):
         try:
             S.Session(ep).close()
