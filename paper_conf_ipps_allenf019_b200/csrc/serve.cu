@@ -31,13 +31,39 @@ const bool g_debug = std::getenv("SLATE_DEBUG") != nullptr;
 #define DBG(...) do { if (g_debug) { std::fprintf(stderr, __VA_ARGS__); std::fflush(stderr); } } while (0)
 void on_signal(int) { g_stop = 1; }
 
-// server-wide cache of opened IPC allocations (a handle can be opened once per context)
+// server-wide cache of opened IPC allocations (a handle can be opened once per context).
+// An allocation no session references any more (refs 0) stays mapped until the
+// device has no work queued: cudaIpcCloseMemHandle waits for the device and
+// holds the driver while it does, so closing while other tenants run stalled
+// every session's issue (no grows reached the running launches) for 12-360 ms
+// at the end of C4 runs.  reap_ipc closes them from the watcher thread.
 struct Opened {
   void* ptr;
   int refs;
 };
 std::mutex g_ipc_mu;
 std::map<std::string, Opened> g_ipc;
+constexpr int kMaxUnreferenced = 64;   // beyond this, close even while the device is busy
+
+void unref_ipc_locked(const std::string& key) {
+  auto it = g_ipc.find(key);
+  if (it != g_ipc.end() && it->second.refs > 0) it->second.refs -= 1;
+}
+
+void reap_ipc(Server* srv, bool force) {
+  std::lock_guard<std::mutex> g(g_ipc_mu);
+  int unreferenced = 0;
+  for (const auto& kv : g_ipc) unreferenced += kv.second.refs == 0;
+  if (!unreferenced || (!force && unreferenced <= kMaxUnreferenced && srv->busy())) return;
+  for (auto it = g_ipc.begin(); it != g_ipc.end();) {
+    if (it->second.refs == 0) {
+      cudaIpcCloseMemHandle(it->second.ptr);
+      it = g_ipc.erase(it);
+    } else {
+      ++it;
+    }
+  }
+}
 
 struct Import {
   uint64_t id, client_base, size;
@@ -75,13 +101,7 @@ bool Session::translate(uint64_t& p, std::string* err) const {
 
 void Session::release_imports() {
   std::lock_guard<std::mutex> g(g_ipc_mu);
-  for (const Import& im : imports_) {
-    auto it = g_ipc.find(im.key);
-    if (it != g_ipc.end() && --it->second.refs == 0) {
-      cudaIpcCloseMemHandle(it->second.ptr);
-      g_ipc.erase(it);
-    }
-  }
+  for (const Import& im : imports_) unref_ipc_locked(im.key);   // closed by reap_ipc
   imports_.clear();
 }
 
@@ -122,11 +142,9 @@ int Session::handle(const Request& rq, Response& rs) {
       rc = SLATE_ENOTFOUND;
       for (size_t i = 0; i < imports_.size(); ++i)
         if (imports_[i].id == rq.id) {
-          std::lock_guard<std::mutex> g(g_ipc_mu);
-          auto it = g_ipc.find(imports_[i].key);
-          if (it != g_ipc.end() && --it->second.refs == 0) {
-            cudaIpcCloseMemHandle(it->second.ptr);
-            g_ipc.erase(it);
+          {
+            std::lock_guard<std::mutex> g(g_ipc_mu);
+            unref_ipc_locked(imports_[i].key);
           }
           imports_.erase(imports_.begin() + long(i));
           rc = SLATE_OK;
@@ -211,8 +229,15 @@ void Session::run() {
       std::memset(&rs, 0, sizeof(rs));
       if (rq.cmd == CMD_DETACH) {
         std::string err;
+        const auto t0 = std::chrono::steady_clock::now();
         rs.status = srv_->close_queue(queue_, 60000000, &err);
+        const auto t1 = std::chrono::steady_clock::now();
         release_imports();
+        const auto t2 = std::chrono::steady_clock::now();
+        if (getenv("SLATE_CLOSE_TIMING"))
+          fprintf(stderr, "slated[q%u]: detach close %.3f ms, release %.3f ms\n", queue_,
+                  std::chrono::duration<double, std::milli>(t1 - t0).count(),
+                  std::chrono::duration<double, std::milli>(t2 - t1).count());
         detached = true;
       } else {
         handle(rq, rs);
@@ -234,8 +259,15 @@ void Session::run() {
   }
   if (!detached && queue_) {
     std::string err;
+    const auto t0 = std::chrono::steady_clock::now();
     srv_->close_queue(queue_, 60000000, &err);
+    const auto t1 = std::chrono::steady_clock::now();
     release_imports();
+    const auto t2 = std::chrono::steady_clock::now();
+    if (getenv("SLATE_CLOSE_TIMING"))
+      fprintf(stderr, "slated[q%u]: close %.3f ms, release %.3f ms\n", queue_,
+              std::chrono::duration<double, std::milli>(t1 - t0).count(),
+              std::chrono::duration<double, std::milli>(t2 - t1).count());
   }
   if (detached) {   // the client is reading its DETACH response: wait for its ack (or its exit)
     const auto t0 = std::chrono::steady_clock::now();
@@ -281,6 +313,7 @@ extern "C" slate_status slate_serve(const char* endpoint, int device, uint32_t f
   shm->hdr.alive.store(1, std::memory_order_release);
   fprintf(stderr, "slated: serving %s on device %d (%u SMs)\n", endpoint, device, srv->info().num_sms);
   std::vector<std::thread> threads;
+  uint32_t tick = 0;
   while (!g_stop) {
     for (int i = 0; i < kSlots; ++i) {
       Slot& s = shm->slots[i];
@@ -290,10 +323,12 @@ extern "C" slate_status slate_serve(const char* endpoint, int device, uint32_t f
         threads.emplace_back([srv, &s, device] { Session(srv, &s, device).run(); });
       }
     }
+    if (++tick % 256 == 0) reap_ipc(srv, false);   // ~every 50 ms
     std::this_thread::sleep_for(std::chrono::microseconds(200));
   }
   shm->hdr.alive.store(0);
   for (auto& t : threads) t.join();
+  reap_ipc(srv, true);
   munmap(p, sizeof(ShmLayout));
   close(fd);
   shm_unlink(endpoint);

@@ -269,6 +269,15 @@ uint32_t Server::open_queue() {
   return id;
 }
 
+bool Server::busy() {
+  std::lock_guard<std::mutex> g(mu_);
+  for (const auto& kv : queues_) {
+    const Queue& Q = *kv.second;
+    if (!Q.issued.empty() || !Q.pending.empty() || !Q.deferred.empty()) return true;
+  }
+  return false;
+}
+
 int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
   const int rc = sync(q, 0, timeout_us, err);
   std::lock_guard<std::mutex> g(mu_);

@@ -102,6 +102,7 @@ class Server {
 
   uint32_t open_queue();
   int close_queue(uint32_t q, int64_t timeout_us, std::string* err);
+  bool busy();   // any queue has launches pending, deferred or issued and not complete
 
   int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
   int register_source(const slate_source_desc* d, uint64_t* out, std::string* err);
