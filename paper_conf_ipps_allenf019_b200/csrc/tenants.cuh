@@ -370,9 +370,9 @@ struct BlackScholes : TenantBase {
     return d;
   }
   __device__ __forceinline__ static f2 abs2(f2 a) { return a & 0x7fffffff7fffffffull; }
-  // the A&S polynomial with 1/sqrt(2 pi) folded into its coefficients
-  __device__ __forceinline__ static f2 poly2r(f2 K) {
-    const float R = 0.39894228040143267794f;
+  // the A&S polynomial, negated, with 1/sqrt(2 pi) folded into its coefficients
+  __device__ __forceinline__ static f2 poly2rn(f2 K) {
+    const float R = -0.39894228040143267794f;
     const f2 A1 = pk(0.31938153f * R, 0.31938153f * R), A2 = pk(-0.356563782f * R, -0.356563782f * R),
              A3 = pk(1.781477937f * R, 1.781477937f * R), A4 = pk(-1.821255978f * R, -1.821255978f * R),
              A5 = pk(1.330274429f * R, 1.330274429f * R);
@@ -404,17 +404,20 @@ struct BlackScholes : TenantBase {
       SXD[h] = pk(sxd[2 * h], sxd[2 * h + 1]);
       CS[h] = pk(0.f, 0.f);
     }
-    const float HL2E = -0.5f * 1.44269504088896341f;   // exp(-d^2/2) = 2^(d^2 * -log2(e)/2)
-    const f2 ONE = pk(1.0f, 1.0f), AK = pk(0.2316419f, 0.2316419f), MHL = pk(HL2E, HL2E);
+    // d1, d2 are carried scaled by C = sqrt(log2(e)/2): exp(-d1^2/2) = 2^-(C d1)^2
+    // (the scale rides on 1/sigma and sigma, the A&S constant is divided by it)
+    const float C = 0.84932180028801904f;
+    const f2 ONE = pk(1.0f, 1.0f), HALF = pk(0.5f, 0.5f), AK = pk(0.2316419f / C, 0.2316419f / C);
+    const f2 SGN = 0x8000000080000000ull;
     for (uint32_t p = 0; p < P; ++p) {
       const float sg = __ldg(sig + p);
       const float rsg = rcp(sg);
       const float hs2 = __fmaf_rn(__fmul_rn(0.5f, sg), sg, r);
-      const f2 NSG = pk(-sg, -sg), RSG = pk(rsg, rsg), HS2 = pk(hs2, hs2);
+      const f2 NSG = pk(-sg * C, -sg * C), RSG = pk(rsg * C, rsg * C), HS2 = pk(hs2, hs2);
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const f2 d1 = mul2(fma2(HS2, SQT[h], LQ[h]), RSG);
-        const f2 d2 = fma2(NSG, SQT[h], d1);
+        const f2 d1 = mul2(fma2(HS2, SQT[h], LQ[h]), RSG);   // C d1
+        const f2 d2 = fma2(NSG, SQT[h], d1);                 // C d2
         const f2 u1 = fma2(AK, abs2(d1), ONE), u2 = fma2(AK, abs2(d2), ONE);
         // the two A&S K = 1/u by two reciprocals: the MUFU pipe has the slack
         // the FP32 pipe (the limit) lacks -- one more MUFU op, three fewer FP32
@@ -422,24 +425,17 @@ struct BlackScholes : TenantBase {
         up(u1, u10, u11);
         up(u2, u20, u21);
         const f2 k1 = pk(rcp(u10), rcp(u11)), k2 = pk(rcp(u20), rcp(u21));
-        up(mul2(mul2(d1, d1), MHL), a0, a1);
+        up(mul2(d1, d1), a0, a1);
         float x0, x1;
-        asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x0) : "f"(a0));
-        asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x1) : "f"(a1));
-        const f2 e1 = pk(x0, x1);                       // exp(-d1^2/2); 1/sqrt(2 pi) is in poly2r
-        const f2 c1 = mul2(e1, poly2r(k1));
-        const f2 c2 = mul2(mul2(e1, SXD[h]), poly2r(k2));
-        const f2 o1 = sub2(ONE, c1), o2 = sub2(ONE, c2);
-        float d10, d11, d20, d21, c10, c11, c20, c21, o10, o11, o20, o21;
-        up(d1, d10, d11);
-        up(d2, d20, d21);
-        up(c1, c10, c11);
-        up(c2, c20, c21);
-        up(o1, o10, o11);
-        up(o2, o20, o21);
-        const f2 n1 = pk(d10 > 0.f ? o10 : c10, d11 > 0.f ? o11 : c11);
-        const f2 n2 = pk(d20 > 0.f ? o20 : c20, d21 > 0.f ? o21 : c21);
-        CS[h] = fma2(NXD[h], n2, fma2(SS[h], n1, CS[h]));   // += S n1 - X e^{-rT} n2
+        asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x0) : "f"(-a0));
+        asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(x1) : "f"(-a1));
+        const f2 e1 = pk(x0, x1);                       // exp(-d1^2/2); 1/sqrt(2 pi) is in poly2rn
+        // N(d) = 1/2 + sign(d) (1/2 - c), c the A&S tail e poly(K): the 1/2 - c
+        // is one FFMA2 (negated polynomial), the sign one LOP3 per element, and
+        // the constant 1/2 (S - X e^{-rT}) of every scenario is added after the loop
+        const f2 m1 = fma2(e1, poly2rn(k1), HALF) ^ (d1 & SGN);
+        const f2 m2 = fma2(mul2(e1, SXD[h]), poly2rn(k2), HALF) ^ (d2 & SGN);
+        CS[h] = fma2(NXD[h], m2, fma2(SS[h], m1, CS[h]));   // += S (n1 - 1/2) - X e^{-rT} (n2 - 1/2)
       }
     }
 #pragma unroll
@@ -450,7 +446,10 @@ struct BlackScholes : TenantBase {
       call[2 * h + 1] = __fdiv_rn(c1, float(P));
     }
 #pragma unroll
-    for (int o = 0; o < 4; ++o) put[o] = __fadd_rn(call[o], __fsub_rn(xd[o], S[o]));
+    for (int o = 0; o < 4; ++o) {
+      call[o] = __fmaf_rn(0.5f, __fsub_rn(S[o], xd[o]), call[o]);
+      put[o] = __fadd_rn(call[o], __fsub_rn(xd[o], S[o]));
+    }
   }
 #ifndef SLATE_BS_X2
 #define SLATE_BS_X2 1
