@@ -199,7 +199,10 @@ constexpr uint32_t kIdesc =
 // standalone and slate use the same map; every tile is computed exactly once).
 // 8 rows of 256 x 256 tiles = 2048 rows of A per group: each B column panel is
 // fetched from DRAM 4 times at 8192^3 (measured with 128-row tiles: 16 rows
-// 0.91 GB of DRAM reads per launch, 8 rows 1.33 GB, 32 rows 1.20 GB).
+// 0.91 GB of DRAM reads per launch, 8 rows 1.33 GB, 32 rows 1.20 GB; with the
+// current 256 x 256 CTA-pair tiles, profiles/r1_gemm_groupm_sweep.md: 4 rows
+// 1.36 GB, 8 rows 0.94 GB, 16 rows 1.29 GB, 32 rows 2.45 GB, and 8 is also the
+// fastest solo and in the C3 co-run).
 #ifndef SLATE_GEMM_GROUP_M
 #define SLATE_GEMM_GROUP_M 8
 #endif
