@@ -151,12 +151,28 @@ slate_status slate_get_info(slate_session* s, slate_info* out);
  *   handle  receives an opaque id (for slate_unshare_buffer).
  * Ownership: the CLIENT owns the memory and must keep it alive until every
  * launch that uses it has completed and the buffer is unshared/detached.
+ * Through an endpoint the server drops its mapping asynchronously once no
+ * session references the allocation: when the device is idle, else within
+ * ~0.5 s (a mapping is never closed on a session's issue path, because
+ * closing waits for the device).  CUDA leaves freeing exported memory before
+ * every importer closed it undefined, so a client that frees a buffer while
+ * other tenants keep the server busy should wait ~0.5 s after unsharing.
  * Errors: EINVAL (null/zero range, not device memory), EIPC. */
 slate_status slate_share_buffer(slate_session* s, uint64_t dev_ptr, size_t bytes, uint64_t* handle);
 slate_status slate_unshare_buffer(slate_session* s, uint64_t handle);
 
 /* ------------------------------------------------------------------ kernels */
 #define SLATE_KFLAG_COVERAGE 1u   /* launches may pass a coverage log (debug) */
+/* Rank log (debug; needs SLATE_KFLAG_COVERAGE): the coverage log is then
+ * u32[2B], and for every original block b the word cov[B + b] records who
+ * took the task holding b, written by the fetching thread when it hands the
+ * task out: bits 0-7 the worker's SM rank (for a GEMM CTA pair, the leader's),
+ * bits 8-15 / 16-23 the range [lo, hi] of the resize word the worker acted on
+ * (intersected with a top-up's bound), bit 24 set if the worker was outside
+ * that range and kept the task only because it was the last live worker
+ * (reading Q22), bit 31 set (valid).  It makes "the kernel only runs on these
+ * SMs" (§IV-C, Lst1) checkable per task. */
+#define SLATE_KFLAG_RANKLOG 2u
 
 typedef struct {
   uint32_t abi_version;    /* SLATE_ABI_VERSION */
@@ -195,7 +211,8 @@ typedef struct {
   uint32_t args_size;      /* sizeof the kind's slate_args_* */
   const void* args;        /* copied before the call returns */
   uint64_t coverage;       /* 0, or device u32[Gx*Gy*Gz] zero-filled by the caller:
-                              every executed original block b does cov[b] += 1 */
+                              every executed original block b does cov[b] += 1;
+                              u32[2*Gx*Gy*Gz] for a kernel with SLATE_KFLAG_RANKLOG */
 } slate_launch_desc;
 
 /* Submit one kernel launch, asynchronously (the API "wraps ... launch",
@@ -237,40 +254,57 @@ slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel*
 
 /* ------------------------------------------------------------------ runtime kernel transformation
  * NEXT-3 (Slate scans a user kernel's source, injects its task
- * loop and compiles it with NVRTC).  `source` holds a CUDA C++ kernel
- *     __global__ void <kernel_name>(<parameters>) { ... blockIdx ... gridDim ... }
- * with 1-D blocks of `block_threads` threads and `smem_bytes` of dynamic
- * shared memory.  The server renames it into a device function that takes the
- * block index and the original grid, generates the slate worker (Lst1/Lst2:
- * SM binding, task counter, decode, resize word) and an original-kernel
- * wrapper around the same body, compiles both for sm_100a with NVRTC and
- * registers the result as a kernel of kind SLATE_KIND_USER.  Launch it with
- * slate_launch / slate_launch_n: desc.grid is the original grid (any x, y, z),
- * desc.args the parameters packed as a C struct in declaration order
- * (args_size bytes).  bytes_per_block / flops_per_block declare its work for
- * slate_profile's classification (0 if unknown).  In-process sessions only
- * (through an endpoint the server cannot rewrite pointers it cannot see).
- * flags: SLATE_KFLAG_COVERAGE as for slate_register_kernel.
- * Errors: EINVAL (no such kernel in the source, bad sizes), EUNSUPPORTED (no
- * NVRTC, or an endpoint session), ECUDA (compile or load failed; the compiler
- * log is in slate_last_error). */
+ * loop and compiles it with NVRTC; "a compiled kernel image can be further
+ * cached").  `source` holds a CUDA C++ kernel
+ *     __global__ void <kernel_name>(<parameters>) { ... blockIdx ... threadIdx ... }
+ * with blocks of block_threads x block_y x block_z threads (block_y, block_z:
+ * 0 means 1) and `smem_bytes` of dynamic shared memory.  The server renames
+ * it into a device function that takes the block index, the original grid,
+ * the thread index and the block shape (every blockIdx / gridDim / threadIdx /
+ * blockDim token of the source is renamed), generates the slate worker
+ * (Lst1/Lst2: SM binding, task counter, decode, resize word) -- a 1-D worker
+ * CTA of the same thread count, threads linearised x-fastest as the hardware
+ * forms warps -- and an original-kernel wrapper around the same body launched
+ * with the real block shape, compiles both for sm_100a with NVRTC and
+ * registers the result as a kernel of kind SLATE_KIND_USER.  If the source
+ * uses shared memory (a __shared__ declaration or smem_bytes > 0) the worker
+ * puts a CTA barrier between the blocks it runs back to back.
+ * Compiled images are cached, keyed by a hash of the generated source, the
+ * options and the NVRTC version: in process (a second registration, e.g. with
+ * another task size, reuses the loaded image) and on disk in
+ * $SLATE_RTC_CACHE (default $HOME/.cache/slate-rtc; "off" disables it).
+ * Launch it with slate_launch / slate_launch_n: desc.grid is the original grid
+ * (any x, y, z), desc.args the parameters packed as a C struct in declaration
+ * order (args_size bytes; checked against the compiled struct's size).
+ * bytes_per_block / flops_per_block declare its work for slate_profile's
+ * classification (0 if unknown).  Through an endpoint the source travels over
+ * the command channel and the server rewrites every pointer parameter (a
+ * parameter whose type contains '*') to its mapping of the shared buffers.
+ * flags: SLATE_KFLAG_COVERAGE / SLATE_KFLAG_RANKLOG as for slate_register_kernel.
+ * Errors: EINVAL (no such kernel in the source, bad sizes, args_size not the
+ * parameter struct's), EUNSUPPORTED (no NVRTC), ECUDA (compile or load
+ * failed; the compiler log is in slate_last_error). */
 typedef struct {
   uint32_t abi_version;
-  uint32_t block_threads;
+  uint32_t block_threads;      /* blockDim.x */
   uint32_t smem_bytes;
   uint32_t args_size;
   uint32_t iters;              /* task size; 0 = automatic */
-  uint32_t flags;              /* SLATE_KFLAG_COVERAGE: launches may pass a coverage log */
+  uint32_t flags;              /* SLATE_KFLAG_COVERAGE / SLATE_KFLAG_RANKLOG */
   const char* source;
   const char* kernel_name;
   double bytes_per_block, flops_per_block;
+  uint32_t block_y, block_z;   /* blockDim.y, blockDim.z (0 = 1) */
 } slate_source_desc;
 slate_status slate_register_source(slate_session* s, const slate_source_desc* d, slate_kernel* out);
 /* The transformed source slate_register_source would compile (no GPU, no
  * NVRTC needed): writes up to cap bytes (NUL-terminated) to out and the full
- * length to *len.  Errors: EINVAL (no such kernel). */
-slate_status slate_transform_source(const char* source, const char* kernel_name, uint32_t block_threads,
-                                    uint32_t smem_bytes, char* out, size_t cap, size_t* len);
+ * length to *len.  Errors: EINVAL (no such kernel, bad block shape). */
+slate_status slate_transform_source(const char* source, const char* kernel_name, uint32_t block_x, uint32_t block_y,
+                                    uint32_t block_z, uint32_t smem_bytes, char* out, size_t cap, size_t* len);
+/* Counters of this process's compiled-image cache: NVRTC compiles, in-process
+ * hits, on-disk hits (any pointer may be NULL). */
+void slate_rtc_stats(uint64_t* compiles, uint64_t* mem_hits, uint64_t* disk_hits);
 
 /* Resize the SM range of the queue that owns launch l to [sm_lo, sm_hi]
  * (§III-C; the dispatcher's start_sm/end_sm, Lst3 P:L250-251).
@@ -382,7 +416,7 @@ slate_status slate_kind_geometry(uint32_t kind, uint32_t* tile_m, uint32_t* tile
  * The selector's pure functions, exported so they can be checked without a GPU.
  * Categories: 0 L_C, 1 M_C, 2 H_C, 3 M_M, 4 H_M. */
 /* Classify fractions of peak (reading Q9). Returns the category;
- * *c_level/*m_level receive 0 = L, 1 = M, 2 = H (may be NULL). */
+ * *c_level and *m_level receive 0 = L, 1 = M, 2 = H (may be NULL). */
 uint32_t slate_classify(double hbm_frac, double fp32_frac, double tc_frac, uint32_t* c_level, uint32_t* m_level);
 /* Tab I: 1 = corun, 0 = solo.  literal != 0 uses the table as
  * printed, otherwise the symmetric reading (Q8). */

@@ -255,6 +255,37 @@ def gemm_bf16(A_bits, B_bits, blocks=None):
     return C
 
 
+# ---------------------------------------------------------------- probe3d (a 3-D grid of 3-D blocks)
+# The user kernel of the NEXT-3 / 3-D-grid parity test (tests/test_user_kernels.py):
+#   i = blockIdx.x*blockDim.x + threadIdx.x (and j, k on y, z); inside the field
+#   out[k][j][i] = 2*in[k][j][i] + (blockIdx.x + 3*blockIdx.y + 7*blockIdx.z)
+# so every element records which original block wrote it: the block's (x,y,z)
+# comes from decode() of its linear index (reading Q18 for z), the
+# threads of a block are enumerated x-fastest (CUDA's threadIdx order).
+def probe3d_grid(shape, block):
+    nz, ny, nx = shape
+    bx, by, bz = block
+    return (cdiv(nx, bx), cdiv(ny, by), cdiv(nz, bz))
+
+
+def probe3d(inp, block, blocks=None):
+    nz, ny, nx = inp.shape
+    bx, by, bz = block
+    out = np.zeros(inp.shape, dtype=np.float64)
+    src = inp.astype(np.float64)
+
+    def body(x, y, z):
+        for tz in range(bz):
+            for ty in range(by):
+                for tx in range(bx):
+                    i, j, k = x * bx + tx, y * by + ty, z * bz + tz
+                    if i < nx and j < ny and k < nz:
+                        out[k, j, i] = 2.0 * src[k, j, i] + (x + 3 * y + 7 * z)
+
+    run_grid(probe3d_grid(inp.shape, block), body, blocks)
+    return out
+
+
 # ---------------------------------------------------------------- coverage
 def expected_counters(total_blocks, iters):
     """Deterministic counters of one complete slate launch.

@@ -222,9 +222,8 @@ slate_status slate_launch_many(slate_session* s, uint32_t n, const slate_kernel*
 slate_status slate_register_source(slate_session* s, const slate_source_desc* d, slate_kernel* out) {
   if (!s || !d || !out) return fail(s, SLATE_EINVAL, "null argument");
   std::lock_guard<std::mutex> g(s->mu);
-  if (!s->srv) return fail(s, SLATE_EUNSUPPORTED, "runtime-compiled kernels need an in-process session");
   std::string err;
-  const int rc = s->srv->register_source(d, out, &err);
+  const int rc = s->srv ? s->srv->register_source(d, out, &err) : s->remote->register_source(d, out, &err);
   return rc == SLATE_OK ? rc : fail(s, rc, err);
 }
 

@@ -64,7 +64,7 @@ struct Params {
   CUtensorMap tma_c;     // fp32 C, boxes of 32 x 32, SWIZZLE_128B (epilogue TMA store)
   slate_args_gemm args;
   uint32_t gx, gy, B, iters, occ, bound_lo, bound_hi, n_ranks, standby_timeout_ns, base_epoch;
-  uint32_t is_topup, gate_first;   // as WorkerParams (slate_device.cuh)
+  uint32_t is_topup, gate_first, ranklog;   // as WorkerParams (slate_device.cuh)
   const uint64_t* ctrl;
   TaskCtl* tc;
   HostMirror* mirror;
@@ -246,7 +246,15 @@ __device__ bool pair_prologue(const P& p, uint32_t r0, uint32_t r1, uint64_t& c_
   uint64_t t0 = 0;
   uint32_t backoff = 256;
   if (p.gate_first) {   // top-up of a launch that has no start event: wait until it started
-    while (ld_relaxed_u64(&tc->t_first) == 0 && ld_relaxed_u32(&tc->next) < p.B) __nanosleep(512);
+    // bounded: the gated launch may be queued behind other work and need the
+    // very SM slots this top-up's waiting CTAs hold; a launch that starts later
+    // reads the resize word by itself (its own grid is a full wave), so the
+    // top-up may leave without joining
+    const uint64_t tg = globaltimer();
+    while (ld_relaxed_u64(&tc->t_first) == 0 && ld_relaxed_u32(&tc->next) < p.B) {
+      if (globaltimer() - tg > p.standby_timeout_ns) return false;
+      __nanosleep(512);
+    }
   }
   for (;;) {
     const uint64_t c = ld_acquire_u64(p.ctrl);
@@ -370,7 +378,8 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       if constexpr (kSlate) {
         // task boundary: resize word, returned tasks, then the counter
         c = ld_acquire_u64(p.ctrl);
-        if (!pair_in_range(p, S.rank, S.peer_rank, c) && try_retire(p.tc)) {
+        const bool inr = pair_in_range(p, S.rank, S.peer_rank, c);
+        if (!inr && try_retire(p.tc)) {
           S.retired = 1;
         } else {
           bool leave;
@@ -385,6 +394,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
               g = take_returned(p.tc, true, leave);          // drained: leave unless one was returned
             }
           }
+          if (g != 0xffffffffu) log_task(p, g, S.rank, c, !inr);   // the leader's rank (the pair is in or out together)
         }
       } else {
         g = t == 0 ? blockIdx.y * (gridDim.x >> 1) + (blockIdx.x >> 1) : 0xffffffffu;
@@ -717,6 +727,7 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.base_epoch = w.base_epoch;
   p.is_topup = w.is_topup;
   p.gate_first = w.gate_first;
+  p.ranklog = w.ranklog;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   return launch_pairs(reinterpret_cast<const void*>(&gemm_kernel<true>), p, dim3((grid + 1) & ~1u), st);
 }

@@ -1,3 +1,4 @@
+#include <algorithm>
 // ipc.cu -- client side of the shared-memory transport (see ipc.h) and the
 // per-kind pointer-field table used by the server to translate launch
 // arguments.
@@ -202,6 +203,38 @@ int RemoteClient::register_kernel(const slate_kernel_desc* d, uint64_t* out, std
   rq.kdesc = *d;
   Response rs;
   const int rc = call(rq, &rs, err);
+  if (rc == SLATE_OK) *out = rs.out;
+  return rc;
+}
+
+// NEXT-3 through an endpoint: the source in 256-byte chunks, then the registration
+int RemoteClient::register_source(const slate_source_desc* d, uint64_t* out, std::string* err) {
+  const size_t name_len = d->kernel_name ? std::strlen(d->kernel_name) : 0;
+  if (!d->source || !d->kernel_name || name_len == 0 || name_len >= sizeof(SourceReg::name)) {
+    if (err) *err = "need a source and a kernel name (< 192 characters)";
+    return SLATE_EINVAL;
+  }
+  const size_t n = std::strlen(d->source);
+  Response rs;
+  for (size_t off = 0; off < n || off == 0; off += size_t(kMaxArgs)) {
+    Request rq{};
+    rq.cmd = CMD_SOURCE_CHUNK;
+    rq.flags = off == 0 ? 1u : 0u;
+    rq.lo = uint32_t(std::min(n - off, size_t(kMaxArgs)));
+    std::memcpy(rq.args, d->source + off, rq.lo);
+    const int rc = call(rq, &rs, err);
+    if (rc != SLATE_OK) return rc;
+    if (n == 0) break;
+  }
+  Request rq{};
+  rq.cmd = CMD_REGISTER_SOURCE;
+  SourceReg r{};
+  r.bx = d->block_threads; r.by = d->block_y; r.bz = d->block_z; r.smem = d->smem_bytes;
+  r.args_size = d->args_size; r.iters = d->iters; r.flags = d->flags;
+  r.bytes_per_block = d->bytes_per_block; r.flops_per_block = d->flops_per_block;
+  std::memcpy(r.name, d->kernel_name, name_len + 1);
+  std::memcpy(rq.args, &r, sizeof(r));
+  const int rc = call(rq, &rs, err, true);   // NVRTC: ~0.2 s on a cache miss
   if (rc == SLATE_OK) *out = rs.out;
   return rc;
 }

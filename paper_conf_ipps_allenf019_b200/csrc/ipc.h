@@ -28,8 +28,18 @@ constexpr int kMaxArgs = 256;
 
 enum Cmd : uint32_t {
   CMD_NONE = 0, CMD_INFO, CMD_SHARE, CMD_UNSHARE, CMD_REGISTER, CMD_LAUNCH, CMD_RESIZE, CMD_SYNC, CMD_PROFILE,
-  CMD_QUERY, CMD_DETACH, CMD_POLICY
+  CMD_QUERY, CMD_DETACH, CMD_POLICY,
+  CMD_SOURCE_CHUNK,        // append args[0, lo) to the session's source buffer (flags & 1: start a new one)
+  CMD_REGISTER_SOURCE      // compile the buffered source: args holds a SourceReg (NEXT-3 through an endpoint)
 };
+
+// CMD_REGISTER_SOURCE's argument block (slate_source_desc without the strings)
+struct SourceReg {
+  uint32_t bx, by, bz, smem, args_size, iters, flags, pad;
+  double bytes_per_block, flops_per_block;
+  char name[192];
+};
+static_assert(sizeof(SourceReg) <= 256, "fits Request::args");
 
 struct Request {
   uint32_t cmd;
@@ -93,6 +103,7 @@ class RemoteClient {
   int share(uint64_t dev_ptr, size_t bytes, uint64_t* handle, std::string* err);
   int unshare(uint64_t handle, std::string* err);
   int register_kernel(const slate_kernel_desc* d, uint64_t* out, std::string* err);
+  int register_source(const slate_source_desc* d, uint64_t* out, std::string* err);
   int launch(uint64_t k, const slate_launch_desc* d, uint64_t* out, std::string* err);
   int launch_n(uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err);
   int resize(uint64_t l, uint32_t lo, uint32_t hi, std::string* err);

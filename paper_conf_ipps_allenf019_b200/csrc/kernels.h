@@ -4,6 +4,7 @@
 #include "rtc_types.h"
 #ifndef __CUDACC_RTC__
 #include <string>
+#include <vector>
 #include "../../include/slate.h"
 #endif
 
@@ -78,7 +79,7 @@ struct HostMirror {
 struct UserWorkerCommon {
   uint32_t gx, gy, gz, B, iters, occ;
   uint32_t bound_lo, bound_hi, n_ranks, standby_timeout_ns;
-  uint32_t base_epoch, is_topup, gate_first, pad_;
+  uint32_t base_epoch, is_topup, gate_first, ranklog;
   const uint64_t* ctrl;
   TaskCtl* tc;
   HostMirror* mirror;
@@ -94,6 +95,7 @@ struct WorkerCommon {
   uint32_t base_epoch;   // the queue's epoch at issue (0 for top-ups: every join of theirs is a grow)
   uint32_t is_topup;     // 1: a top-up grid sharing a running launch's counter
   uint32_t gate_first;   // top-up of a launch with no start event: wait until the launch took its first task
+  uint32_t ranklog = 0;  // cov holds 2B words: the rank log follows the coverage counts (SLATE_KFLAG_RANKLOG)
   bool pdl = false;      // launch with programmatic stream serialization (the previous op on the stream is
                          // the previous worker of the same batch; the worker waits in griddepcontrol.wait)
   const uint64_t* ctrl;
@@ -127,16 +129,18 @@ struct KindOps {
   uint32_t user_threads = 0;     // T of a user kernel
   void* user_ctx = nullptr;      // the loaded user kernels (user_kernels.cu)
   double user_bytes_per_block = 0, user_flops_per_block = 0;
+  std::vector<size_t> user_ptr_offsets;   // pointer parameters of a user kernel's argument struct
 };
 
 // NEXT-3 (the paper's runtime kernel transformation): scan a user's
 // CUDA source for its __global__ kernel and generate the slate worker around it
 // (and an original-kernel wrapper over the same body); compile it with NVRTC
 // for sm_100a and load it.  Returns false with *err set on failure.
-bool transform_user_kernel(const char* src, const char* name, uint32_t threads, uint32_t smem, std::string* out,
-                           std::string* err);
-bool build_user_kind(const char* src, const char* name, uint32_t threads, uint32_t smem, uint32_t args_size,
-                     KindOps* ops, std::string* err);
+bool transform_user_kernel(const char* src, const char* name, uint32_t bx, uint32_t by, uint32_t bz, uint32_t smem,
+                           std::string* out, std::string* err);
+// compiled images are cached: *compiled says whether NVRTC ran
+bool build_user_kind(const char* src, const char* name, uint32_t bx, uint32_t by, uint32_t bz, uint32_t smem,
+                     uint32_t args_size, KindOps* ops, std::string* err, bool* compiled = nullptr);
 
 const KindOps* kind_ops(uint32_t kind);   // nullptr if the kind is not built
 

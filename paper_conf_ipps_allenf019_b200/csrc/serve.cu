@@ -32,37 +32,62 @@ const bool g_debug = std::getenv("SLATE_DEBUG") != nullptr;
 void on_signal(int) { g_stop = 1; }
 
 // server-wide cache of opened IPC allocations (a handle can be opened once per context).
-// An allocation no session references any more (refs 0) stays mapped until the
-// device has no work queued: cudaIpcCloseMemHandle waits for the device and
-// holds the driver while it does, so closing while other tenants run stalled
-// every session's issue (no grows reached the running launches) for 12-360 ms
-// at the end of C4 runs.  reap_ipc closes them from the watcher thread.
+// An allocation no session references any more (refs 0) is closed by the
+// watcher thread (reap_ipc), never on a session's issue path, and never under
+// g_ipc_mu: cudaIpcCloseMemHandle waits for the device and holds the driver
+// while it does, so closing from a session thread while other tenants ran
+// stalled every session's issue (no grows reached the running launches) for
+// 12-360 ms at the end of C4 runs.  The reaper waits for an idle device, but
+// only so long: an unreferenced mapping is closed anyway once it is older than
+// kMaxUnrefAge or the unreferenced mappings exceed kMaxUnrefBytes, so memory of
+// clients that left is given back under continuous load.  Contract (slate.h):
+// a client keeps a shared allocation alive until slate_unshare_buffer /
+// slate_detach of it returned; the server's mapping goes within kMaxUnrefAge.
 struct Opened {
   void* ptr;
   int refs;
+  uint64_t bytes;
+  std::chrono::steady_clock::time_point unref_since;
 };
-std::mutex g_ipc_mu;
+std::mutex g_ipc_mu;      // the map
+std::mutex g_ipc_close_mu;  // held while mappings are being closed (and by an open of a new handle)
 std::map<std::string, Opened> g_ipc;
-constexpr int kMaxUnreferenced = 64;   // beyond this, close even while the device is busy
+constexpr auto kMaxUnrefAge = std::chrono::milliseconds(500);
+constexpr uint64_t kMaxUnrefBytes = 8ull << 30;
 
 void unref_ipc_locked(const std::string& key) {
   auto it = g_ipc.find(key);
-  if (it != g_ipc.end() && it->second.refs > 0) it->second.refs -= 1;
+  if (it != g_ipc.end() && it->second.refs > 0 && --it->second.refs == 0)
+    it->second.unref_since = std::chrono::steady_clock::now();
 }
 
 void reap_ipc(Server* srv, bool force) {
-  std::lock_guard<std::mutex> g(g_ipc_mu);
-  int unreferenced = 0;
-  for (const auto& kv : g_ipc) unreferenced += kv.second.refs == 0;
-  if (!unreferenced || (!force && unreferenced <= kMaxUnreferenced && srv->busy())) return;
-  for (auto it = g_ipc.begin(); it != g_ipc.end();) {
-    if (it->second.refs == 0) {
-      cudaIpcCloseMemHandle(it->second.ptr);
-      it = g_ipc.erase(it);
-    } else {
-      ++it;
+  std::lock_guard<std::mutex> gc(g_ipc_close_mu);
+  std::vector<void*> close_now;
+  {
+    std::lock_guard<std::mutex> g(g_ipc_mu);
+    const auto now = std::chrono::steady_clock::now();
+    uint64_t unref_bytes = 0;
+    bool any = false, old = false;
+    for (const auto& kv : g_ipc)
+      if (kv.second.refs == 0) {
+        any = true;
+        unref_bytes += kv.second.bytes;
+        old = old || now - kv.second.unref_since > kMaxUnrefAge;
+      }
+    if (!any) return;
+    const bool go = force || old || unref_bytes > kMaxUnrefBytes || !srv->busy();
+    if (!go) return;
+    for (auto it = g_ipc.begin(); it != g_ipc.end();) {
+      if (it->second.refs == 0) {
+        close_now.push_back(it->second.ptr);
+        it = g_ipc.erase(it);
+      } else {
+        ++it;
+      }
     }
   }
+  for (void* p : close_now) cudaIpcCloseMemHandle(p);   // outside g_ipc_mu: sessions keep issuing
 }
 
 struct Import {
@@ -84,6 +109,7 @@ class Session {
   Slot* slot_;
   int device_;
   uint32_t queue_ = 0;
+  std::string source_;   // a user kernel's source being received (CMD_SOURCE_CHUNK)
   std::vector<Import> imports_;
   uint64_t next_import_ = 1;
 };
@@ -118,7 +144,13 @@ int Session::handle(const Request& rq, Response& rs) {
       std::string key(reinterpret_cast<const char*>(&rq.handle), sizeof(rq.handle));
       void* ptr = nullptr;
       {
-        std::lock_guard<std::mutex> g(g_ipc_mu);
+        std::unique_lock<std::mutex> gc(g_ipc_close_mu, std::defer_lock);
+        std::unique_lock<std::mutex> g(g_ipc_mu);
+        if (g_ipc.find(key) == g_ipc.end()) {   // a new mapping: not while the reaper closes (lock order close -> map)
+          g.unlock();
+          gc.lock();
+          g.lock();
+        }
         auto it = g_ipc.find(key);
         if (it != g_ipc.end()) {
           it->second.refs += 1;
@@ -131,7 +163,7 @@ int Session::handle(const Request& rq, Response& rs) {
             rc = SLATE_EIPC;
             break;
           }
-          g_ipc[key] = {ptr, 1};
+          g_ipc[key] = {ptr, 1, rq.alloc_size, std::chrono::steady_clock::time_point()};
         }
       }
       imports_.push_back({next_import_, rq.alloc_base, rq.alloc_size, static_cast<char*>(ptr), key});
@@ -155,6 +187,30 @@ int Session::handle(const Request& rq, Response& rs) {
     case CMD_REGISTER:
       rc = srv_->register_kernel(&rq.kdesc, &rs.out, &err);
       break;
+    case CMD_SOURCE_CHUNK:
+      if (rq.flags & 1) source_.clear();
+      if (rq.lo > uint32_t(kMaxArgs) || source_.size() + rq.lo > (16u << 20)) {
+        rc = SLATE_EINVAL;
+        err = "source chunk too large (a source is at most 16 MiB)";
+        break;
+      }
+      source_.append(reinterpret_cast<const char*>(rq.args), rq.lo);
+      break;
+    case CMD_REGISTER_SOURCE: {
+      SourceReg r;
+      std::memcpy(&r, rq.args, sizeof(r));
+      r.name[sizeof(r.name) - 1] = 0;
+      slate_source_desc d{};
+      d.abi_version = SLATE_ABI_VERSION;
+      d.block_threads = r.bx; d.block_y = r.by; d.block_z = r.bz;
+      d.smem_bytes = r.smem; d.args_size = r.args_size; d.iters = r.iters; d.flags = r.flags;
+      d.source = source_.c_str();
+      d.kernel_name = r.name;
+      d.bytes_per_block = r.bytes_per_block; d.flops_per_block = r.flops_per_block;
+      rc = srv_->register_source(&d, &rs.out, &err);
+      source_.clear();
+      break;
+    }
     case CMD_LAUNCH:
     case CMD_PROFILE: {
       // rewrite every pointer argument into the server's address space
@@ -169,8 +225,15 @@ int Session::handle(const Request& rq, Response& rs) {
         break;
       }
       const size_t* offs;
-      const int nf = pointer_fields(kind, &offs);
+      int nf = pointer_fields(kind, &offs);
+      std::vector<size_t> user_offs;   // a runtime-compiled kernel: its own pointer parameters
+      if (kind == SLATE_KIND_USER && srv_->kernel_ptr_fields(rq.id, &user_offs)) {
+        offs = user_offs.data();
+        nf = int(user_offs.size());
+      }
       bool ok = d.args_size <= sizeof(args);
+      for (int i = 0; ok && i < nf; ++i) ok = offs[i] + 8 <= d.args_size;
+      if (!ok && err.empty()) err = "argument block smaller than the kernel's pointer parameters";
       for (int i = 0; ok && i < nf; ++i) {
         uint64_t p;
         std::memcpy(&p, args + offs[i], 8);

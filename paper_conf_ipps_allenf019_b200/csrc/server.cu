@@ -5,6 +5,7 @@
 // completion of kernels, selection (Tab I), dynamic resizing
 // (P:L123-127).  B200 design in DESIGN.md §Runtime.
 #include <algorithm>
+#include <unordered_set>
 #include <chrono>
 #include <cmath>
 #include <cstdlib>
@@ -137,6 +138,7 @@ int Server::init(std::string* err) {
   peak_fp32_ = env_double("SLATE_PEAK_FP32_GFLOPS", 2.0 * 128 * prop.multiProcessorCount * (prop.clockRate / 1e6));
   peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
   standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
+  keep_finished_ = size_t(std::max(16.0, env_double("SLATE_KEEP_FINISHED", 65536.0)));
   saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.95);   // reading Q29 (1.0: no cap)
   if (const char* pol = std::getenv("SLATE_POLICY")) {              // reading Q31
     const std::string v(pol);
@@ -307,6 +309,14 @@ int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
 }
 
 // ------------------------------------------------------------------ kernels
+bool Server::kernel_ptr_fields(uint64_t k, std::vector<size_t>* offs) const {
+  std::lock_guard<std::mutex> g(mu_);
+  auto it = kernels_.find(k);
+  if (it == kernels_.end()) return false;
+  *offs = it->second->ops->user_ptr_offsets;
+  return true;
+}
+
 bool Server::kernel_kind(uint64_t k, uint32_t* kind) const {
   std::lock_guard<std::mutex> g(mu_);
   auto it = kernels_.find(k);
@@ -320,7 +330,8 @@ int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::stri
     if (err) *err = "bad kernel descriptor";
     return SLATE_EINVAL;
   }
-  if (d->kind == 0 || d->kind >= SLATE_KIND_MAX_ || (d->flags & ~SLATE_KFLAG_COVERAGE)) {
+  if (d->kind == 0 || d->kind >= SLATE_KIND_MAX_ || (d->flags & ~(SLATE_KFLAG_COVERAGE | SLATE_KFLAG_RANKLOG)) ||
+      ((d->flags & SLATE_KFLAG_RANKLOG) && !(d->flags & SLATE_KFLAG_COVERAGE))) {
     if (err) *err = "bad kind or flags";
     return SLATE_EINVAL;
   }
@@ -367,17 +378,20 @@ int Server::register_kernel(const slate_kernel_desc* d, uint64_t* out, std::stri
 
 // NEXT-3: a user kernel from source (user_kernels.cu), a kind of its own
 int Server::register_source(const slate_source_desc* d, uint64_t* out, std::string* err) {
+  const uint64_t threads = d ? uint64_t(d->block_threads) * (d->block_y ? d->block_y : 1) * (d->block_z ? d->block_z : 1)
+                             : 0;
   if (!d || !out || d->abi_version != SLATE_ABI_VERSION || !d->source || !d->kernel_name || d->args_size == 0 ||
-      d->args_size > 4096 || d->block_threads == 0 || d->block_threads > 1024) {
+      d->args_size > 4096 || threads == 0 || threads > 1024) {
     if (err) *err = "bad source descriptor";
     return SLATE_EINVAL;
   }
   auto ops = std::make_unique<KindOps>();
   std::string e;
-  if (!build_user_kind(d->source, d->kernel_name, d->block_threads, d->smem_bytes, d->args_size, ops.get(), &e)) {
+  if (!build_user_kind(d->source, d->kernel_name, d->block_threads, d->block_y, d->block_z, d->smem_bytes,
+                       d->args_size, ops.get(), &e)) {
     if (err) *err = e;
     return e.find("not found") != std::string::npos ? SLATE_EUNSUPPORTED
-           : e.find("no `__global__") != std::string::npos ? SLATE_EINVAL : SLATE_ECUDA;
+           : (e.find("no `__global__") != std::string::npos || e.find("args_size") == 0) ? SLATE_EINVAL : SLATE_ECUDA;
   }
   ops->user_bytes_per_block = d->bytes_per_block;
   ops->user_flops_per_block = d->flops_per_block;
@@ -398,7 +412,11 @@ int Server::register_source(const slate_source_desc* d, uint64_t* out, std::stri
   k->desc.abi_version = SLATE_ABI_VERSION;
   k->desc.kind = SLATE_KIND_USER;
   k->desc.iters = d->iters;
-  k->desc.flags = d->flags & SLATE_KFLAG_COVERAGE;
+  k->desc.flags = d->flags & (SLATE_KFLAG_COVERAGE | SLATE_KFLAG_RANKLOG);
+  if ((k->desc.flags & SLATE_KFLAG_RANKLOG) && !(k->desc.flags & SLATE_KFLAG_COVERAGE)) {
+    if (err) *err = "SLATE_KFLAG_RANKLOG needs SLATE_KFLAG_COVERAGE";
+    return SLATE_EINVAL;
+  }
   k->occ = occ;
   k->ops = ops.get();
   k->own_ops = std::move(ops);
@@ -736,7 +754,46 @@ void Server::close_batch(Queue& Q, cudaEvent_t end, bool closed_by_launch) {
 void Server::fail_launch(Launch& L, int code) {
   L.error = code;
   L.state = 2;
+  finished_.push_back(L.id);
+  auto qi = queues_.find(L.queue);
+  if (qi != queues_.end() && !qi->second->first_error) qi->second->first_error = code;
   cv_.notify_all();
+}
+
+// Drop the oldest completed launch records beyond the retention window, with
+// the CUDA events only they reference.  Events are shared between launches (a
+// batch's end and snapshot events, a chained launch's start = its
+// predecessor's end, top-up ends), so an event is destroyed only when no
+// retained launch or queue names it.  Bulk: one scan per keep_finished_
+// evictions.
+void Server::retire_finished() {
+  if (finished_.size() <= keep_finished_) return;
+  std::unordered_set<cudaEvent_t> cand;
+  const size_t n = finished_.size() - keep_finished_;
+  for (size_t i = 0; i < n; ++i) {
+    const uint64_t id = finished_.front();
+    finished_.pop_front();
+    auto it = launches_.find(id);
+    if (it == launches_.end()) continue;
+    const Launch& L = *it->second;
+    cand.insert(L.ev_start);
+    cand.insert(L.batch_end);
+    for (cudaEvent_t e : L.ev_end) cand.insert(e);
+    for (cudaEvent_t e : L.ev_done) cand.insert(e);
+    launches_.erase(it);
+  }
+  for (const auto& kv : launches_) {
+    const Launch& L = *kv.second;
+    cand.erase(L.ev_start);
+    cand.erase(L.start_after);
+    cand.erase(L.batch_end);
+    for (cudaEvent_t e : L.ev_end) cand.erase(e);
+    for (cudaEvent_t e : L.ev_done) cand.erase(e);
+  }
+  for (const auto& kv : queues_)
+    for (cudaEvent_t e : kv.second->topup_ends) cand.erase(e);
+  for (cudaEvent_t e : cand)
+    if (e) cudaEventDestroy(e);
 }
 
 void Server::drain_deferred(Queue& Q) {
@@ -817,6 +874,7 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     w.base_epoch = Q.epoch;
     w.ctrl = Q.d_ctrl; w.tc = d_tc_ + slot; w.mirror = d_mirror_ + slot;
     w.cov = reinterpret_cast<uint32_t*>(L.desc.coverage);
+    w.ranklog = (L.k->desc.flags & SLATE_KFLAG_RANKLOG) && w.cov ? 1u : 0u;
     w.rank_of = d_rank_of_;
     w.ops = ops;
     // PDL: the previous op on the stream is the previous worker of this batch
@@ -933,6 +991,7 @@ int Server::topup(Queue& Q, Launch& R, std::string* err) {
   w.ops = R.k->ops;
   w.ctrl = Q.d_ctrl; w.tc = d_tc_ + R.slot; w.mirror = d_mirror_ + R.slot;
   w.cov = reinterpret_cast<uint32_t*>(R.desc.coverage);
+  w.ranklog = (R.k->desc.flags & SLATE_KFLAG_RANKLOG) && w.cov ? 1u : 0u;
   w.rank_of = d_rank_of_;
   CK(R.k->ops->launch_worker(w, R.args.data(), uint32_t(R.k->occ) * uint32_t(n_sms_), aux));
   cudaEvent_t ev_end, ev_snap;
@@ -1513,6 +1572,8 @@ void Server::poll_once() {
         L.slot = -1;
       }
       L.state = 2;
+      finished_.push_back(L.id);
+      if (L.error && !Q.first_error) Q.first_error = L.error;
       Q.issued.pop_front();
       if (Q.issued.empty()) Q.topup_ends.clear();
       else {                      // the next launch starts now, on the queue's current range
@@ -1527,6 +1588,7 @@ void Server::poll_once() {
   }
   flush_free();
   for (uint32_t q : idle) release(*queues_[q]);
+  if (finished_.size() > 2 * keep_finished_) retire_finished();
 }
 
 void Server::poller_main() {
@@ -1560,7 +1622,8 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
     return qi == queues_.end() ||
            (qi->second->issued.empty() && qi->second->pending.empty() && qi->second->deferred.empty());
   };
-  if (l && launches_.find(l) == launches_.end()) return SLATE_ENOTFOUND;
+  // a launch id below the retention window completed long ago (ids are monotonic)
+  if (l && launches_.find(l) == launches_.end()) return l < next_launch_id_ ? SLATE_OK : SLATE_ENOTFOUND;
   while (!done()) {
     if (timeout_us < 0) {
       cv_.wait_for(g, std::chrono::milliseconds(5));
@@ -1572,12 +1635,17 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
       cv_.wait_until(g, std::min(deadline, std::chrono::steady_clock::now() + std::chrono::milliseconds(5)));
     }
   }
-  for (auto& kv : launches_) {
-    const Launch& L = *kv.second;
-    if ((l ? L.id == l : L.queue == q) && L.error) {
-      if (err) *err = std::string("CUDA error: ") + cudaGetErrorString(cudaError_t(L.error));
-      return SLATE_ECUDA;
-    }
+  int e = 0;   // per launch, or the queue's first error (no scan over every launch ever made)
+  if (l) {
+    auto it = launches_.find(l);
+    if (it != launches_.end()) e = it->second->error;
+  } else {
+    auto qi = queues_.find(q);
+    if (qi != queues_.end()) e = qi->second->first_error;
+  }
+  if (e) {
+    if (err) *err = std::string("CUDA error: ") + cudaGetErrorString(cudaError_t(e));
+    return SLATE_ECUDA;
   }
   return SLATE_OK;
 }

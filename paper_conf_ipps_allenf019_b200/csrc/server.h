@@ -85,6 +85,7 @@ struct Queue {
   struct PendingResize { uint32_t epoch; int kind; double t0_us; uint64_t lid; int idx; };
   std::vector<PendingResize> pending_resize;
   bool closed = false;
+  int first_error = 0;          // the first cudaError_t a launch of this queue completed with
 };
 
 struct ProfileEntry {
@@ -116,6 +117,7 @@ class Server {
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);
   bool kernel_kind(uint64_t k, uint32_t* kind) const;
+  bool kernel_ptr_fields(uint64_t k, std::vector<size_t>* offs) const;   // a user kernel's pointer parameters
 
  private:
   // all private helpers are called with mu_ held
@@ -213,6 +215,12 @@ class Server {
   std::map<uint64_t, std::unique_ptr<KernelEntry>> kernels_;
   std::map<uint32_t, std::unique_ptr<Queue>> queues_;
   std::map<uint64_t, std::unique_ptr<Launch>> launches_;
+  // completed launches in completion order: records (and their CUDA events)
+  // are kept for slate_query until kKeepFinished newer ones completed, then
+  // dropped in bulk (retire_finished), so a long-running slated stays bounded
+  std::deque<uint64_t> finished_;
+  size_t keep_finished_ = 65536;   // SLATE_KEEP_FINISHED (tests use a small window)
+  void retire_finished();
   std::deque<uint32_t> waiting_;     // queues waiting for SMs, FIFO
   std::map<uint32_t, uint32_t> bypassed_;
   std::vector<uint32_t> active_;     // queues holding SMs

@@ -92,6 +92,7 @@ struct WorkerParams {
   uint32_t base_epoch;            // resize-word epoch when the launch was issued: a join under a later epoch is a grow
   uint32_t is_topup;              // 1: a top-up grid (grow) sharing a running launch's TaskCtl
   uint32_t gate_first;            // top-up: join only once the launch has taken its first task
+  uint32_t ranklog;               // 1: cov holds 2B words, cov[B + b] = the rank log entry of block b
   const uint64_t* ctrl;           // the queue's resize word
   TaskCtl* tc;
   HostMirror* mirror;             // device alias of the pinned mirror (may be null)
@@ -127,6 +128,25 @@ struct BlockWalk {
   }
 };
 
+// ------------------------------------------------------------------ rank log (debug, SLATE_KFLAG_RANKLOG)
+// Who took each task: written by the fetching lane when it hands out task
+// [g, g+n), one word per block at cov[B + b]: the worker's SM rank, the range
+// [lo, hi] of the resize word it acted on (intersected with the launch bound),
+// and flags -- bit 0: the worker was outside that range and kept the task only
+// under the last-live-worker rule (Q22), bit 7: valid.  Tests check that every
+// task ran on a rank inside the range in force ("ensures that the
+// kernel only runs on these SMs") and that co-runners' rank sets are disjoint.
+__device__ __forceinline__ uint32_t ranklog_entry(uint32_t rank, uint32_t lo, uint32_t hi, bool outside) {
+  return (rank & 0xffu) | ((lo & 0xffu) << 8) | ((hi & 0xffu) << 16) | ((0x80u | (outside ? 1u : 0u)) << 24);
+}
+template <class P>
+__device__ __forceinline__ void log_task(const P& p, uint32_t g, uint32_t rank, uint64_t c, bool outside) {
+  if (!p.ranklog || !p.cov || g >= p.B) return;
+  const uint32_t lo = max(ctrl_lo(c), p.bound_lo), hi = min(ctrl_hi(c), p.bound_hi);
+  const uint32_t e = ranklog_entry(rank, lo, hi, outside), n = min(p.iters, p.B - g);
+  for (uint32_t i = 0; i < n; ++i) p.cov[p.B + g + i] = e;
+}
+
 // ------------------------------------------------------------------ bookkeeping
 // Latency discipline: every bookkeeping atomic whose result is not needed is a
 // fire-and-forget reduction (RED), the resize word for a task boundary is
@@ -148,7 +168,15 @@ __device__ bool prologue(const P& p, uint32_t rank, uint64_t& c_out) {
   uint64_t t0 = 0;
   uint32_t backoff = 256;
   if (p.gate_first) {   // top-up of a launch that has no start event: wait until it started
-    while (ld_relaxed_u64(&tc->t_first) == 0 && ld_relaxed_u32(&tc->next) < p.B) __nanosleep(512);
+    // bounded: the gated launch may be queued behind other work and need the
+    // very SM slots this top-up's waiting CTAs hold; a launch that starts later
+    // reads the resize word by itself (its own grid is a full wave), so the
+    // top-up may leave without joining
+    const uint64_t tg = globaltimer();
+    while (ld_relaxed_u64(&tc->t_first) == 0 && ld_relaxed_u32(&tc->next) < p.B) {
+      if (globaltimer() - tg > p.standby_timeout_ns) return false;
+      __nanosleep(512);
+    }
   }
   for (;;) {
     // the counter load first: a relaxed load issued after the acquire would wait
@@ -277,15 +305,17 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
   // task_done: one 64-bit atomic; its result is needed only to spot the last block
   if (n_done) old = atomicAdd(&tc->done, (1ull << 32) | n_done);
   uint32_t g = 0xffffffffu;
-  if (!in_range(p, rank, c2) && try_retire(tc)) {
+  const bool inr = in_range(p, rank, c2);
+  if (!inr && try_retire(tc)) {
     retired = true;
   } else {
     g = atomicAdd(&tc->next, p.iters);                                  // Lst2 (2)
     if (g >= p.B) {                                                     // Q3: nothing to run
       atomicAdd(&tc->live_pending, ~0ull);                               // live -= 1 (RED)
       g = 0xffffffffu;
-    } else if (g == 0) {
-      tc->t_first = globaltimer();
+    } else {
+      if (g == 0) tc->t_first = globaltimer();
+      log_task(p, g, rank, c2, !inr);
     }
   }
   if (n_done && uint32_t(old) + n_done == p.B) {                        // last block of the launch
@@ -455,8 +485,12 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
         spec_changed = ctrl_epoch(c2) != ctrl_epoch(c);
         if (spec_changed) asm volatile("fence.acq_rel.gpu;" ::: "memory");
         c = c2;
-        if (!in_range(p, rank, c) && try_retire(p.tc)) spec_retired = true;
-        else fut = atomicAdd(&p.tc->next, p.iters);                   // Lst2 (2), result used below
+        const bool inr = in_range(p, rank, c);
+        if (!inr && try_retire(p.tc)) spec_retired = true;
+        else {
+          fut = atomicAdd(&p.tc->next, p.iters);                       // Lst2 (2), result used below
+          log_task(p, fut, rank, c, !inr);
+        }
         c2 = ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(p.ctrl));   // next boundary
       }
       if constexpr (Tn::kHasTask) {

@@ -296,10 +296,12 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     uint32_t g_next = 0xffffffffu;        // raw counter value fetched for the next task (lane 0)
     bool next_ret = false;
     if (lane == 0) {                      // the first boundary is not speculative
-      if (!in_range(p, rank, c) && try_retire(p.tc)) {
+      const bool inr = in_range(p, rank, c);
+      if (!inr && try_retire(p.tc)) {
         next_ret = true;
       } else {
         g_next = atomicAdd(&p.tc->next, p.iters);                     // Lst2 (2)
+        log_task(p, g_next, rank, c, !inr);
       }
       c_pre = ld_acquire_u64(p.ctrl);
     }
@@ -324,8 +326,12 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
         if (g != 0xffffffffu) {
           chg = ctrl_epoch(c_pre) != ctrl_epoch(c);
           c = c_pre;
-          if (!in_range(p, rank, c) && try_retire(p.tc)) next_ret = true;
-          else g_next = atomicAdd(&p.tc->next, p.iters);              // Lst2 (2); result used next round
+          const bool inr = in_range(p, rank, c);
+          if (!inr && try_retire(p.tc)) next_ret = true;
+          else {
+            g_next = atomicAdd(&p.tc->next, p.iters);                 // Lst2 (2); result used next round
+            log_task(p, g_next, rank, c, !inr);
+          }
           c_pre = ld_acquire_u64(p.ctrl);
         }
         mbar_wait(&H.rp_empty[b], ((t / kRpBufs) & 1) ^ 1);         // task t-4 fully consumed
@@ -521,6 +527,7 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.base_epoch = w.base_epoch;
   p.is_topup = w.is_topup;
   p.gate_first = w.gate_first;
+  p.ranklog = w.ranklog;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
   return launch_kernel(reinterpret_cast<const void*>(&spmv_worker), dim3(grid), dim3(kThreads), kargs, kSmemBytes, st,

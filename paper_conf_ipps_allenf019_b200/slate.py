@@ -28,6 +28,7 @@ KIND_TRIAD, KIND_COPY, KIND_SGEMM_NAIVE, KIND_SPMV_CSR, KIND_BLACKSCHOLES, KIND_
 KIND_TRANSPOSE, KIND_SGEMM_TILED, KIND_QRNG, KIND_GAUSS_FAN1, KIND_GAUSS_FAN2 = range(8, 13)
 KIND_USER = 13   # a user kernel compiled at run time (register_source, NEXT-3)
 KFLAG_COVERAGE = 1
+KFLAG_RANKLOG = 2   # with KFLAG_COVERAGE: the coverage log is u32[2B], cov[B + b] = who took block b (slate.h)
 PLACE_AUTO, PLACE_SOLO, PLACE_CORUN = 0, 1, 2
 MODE_SLATE, MODE_STANDALONE = 0, 1
 PROF_CURVE, PROF_FORCE = 1, 2
@@ -86,7 +87,7 @@ class ArgsGauss(ctypes.Structure):
 class SourceDesc(ctypes.Structure):
     _fields_ = [("abi_version", c_u32), ("block_threads", c_u32), ("smem_bytes", c_u32), ("args_size", c_u32),
                 ("iters", c_u32), ("flags", c_u32), ("source", ctypes.c_char_p), ("kernel_name", ctypes.c_char_p),
-                ("bytes_per_block", c_f64), ("flops_per_block", c_f64)]
+                ("bytes_per_block", c_f64), ("flops_per_block", c_f64), ("block_y", c_u32), ("block_z", c_u32)]
 
 
 class Info(ctypes.Structure):
@@ -159,8 +160,8 @@ for _name, _args in [
     ("slate_launch_n", [ctypes.c_void_p, c_u64, _P(LaunchDesc), c_u32, _P(c_u64)]),
     ("slate_launch_many", [ctypes.c_void_p, c_u32, _P(c_u64), _P(LaunchDesc), _P(c_u64)]),
     ("slate_register_source", [ctypes.c_void_p, _P(SourceDesc), _P(c_u64)]),
-    ("slate_transform_source", [ctypes.c_char_p, ctypes.c_char_p, c_u32, c_u32, ctypes.c_char_p, ctypes.c_size_t,
-                                _P(ctypes.c_size_t)]),
+    ("slate_transform_source", [ctypes.c_char_p, ctypes.c_char_p, c_u32, c_u32, c_u32, c_u32, ctypes.c_char_p,
+                                ctypes.c_size_t, _P(ctypes.c_size_t)]),
 ]:
     getattr(_lib, _name).restype = c_i32
     getattr(_lib, _name).argtypes = _args
@@ -184,6 +185,8 @@ _lib.slate_choose_iters.argtypes = [c_f64, c_u32, c_u32, c_u32, c_u32, c_f64]
 _lib.slate_fluid_corun.restype = ctypes.c_int
 _lib.slate_fluid_corun.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_f64, _P(c_u32), _P(c_f64), c_u32, c_f64, c_u32,
                                    c_u32, c_u32, c_u32, c_f64, _P(c_u32), _P(c_f64)]
+_lib.slate_rtc_stats.restype = None
+_lib.slate_rtc_stats.argtypes = [_P(c_u64), _P(c_u64), _P(c_u64)]
 POLICY_TABLE, POLICY_LITERAL, POLICY_HYBRID = 0, 1, 2
 
 EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffer", "slate_unshare_buffer",
@@ -191,7 +194,8 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_status_string", "slate_last_error", "slate_classify", "slate_policy", "slate_select",
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
             "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters",
-            "slate_register_source", "slate_transform_source", "slate_corun_makespan_k", "slate_choose_split_k"]
+            "slate_register_source", "slate_transform_source", "slate_corun_makespan_k", "slate_choose_split_k",
+            "slate_rtc_stats"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -254,11 +258,13 @@ class Session:
         self._check(_lib.slate_unshare_buffer(self._h, handle), "slate_unshare_buffer")
 
     def register_source(self, source, name, args_struct, threads=256, smem=0, iters=0, bytes_per_block=0.0,
-                        flops_per_block=0.0, flags=0):
+                        flops_per_block=0.0, flags=0, block=None):
         """A user CUDA kernel compiled at run time (NEXT-3); `args_struct` is the
-        ctypes Structure type of its parameters, in declaration order."""
-        d = SourceDesc(ABI_VERSION, threads, smem, ctypes.sizeof(args_struct), iters, flags, source.encode(), name.encode(),
-                       bytes_per_block, flops_per_block)
+        ctypes Structure type of its parameters, in declaration order; `block`
+        an (x, y, z) block shape (default (threads, 1, 1))."""
+        bx, by, bz = block if block is not None else (threads, 1, 1)
+        d = SourceDesc(ABI_VERSION, bx, smem, ctypes.sizeof(args_struct), iters, flags, source.encode(), name.encode(),
+                       bytes_per_block, flops_per_block, by, bz)
         k = c_u64()
         self._check(_lib.slate_register_source(self._h, ctypes.byref(d), ctypes.byref(k)), "slate_register_source")
         return k.value
@@ -391,15 +397,23 @@ def choose_split_k(curves, n_sms, step=2):
     return list(out), t
 
 
-def transform_source(source, name, threads=256, smem=0):
+def transform_source(source, name, threads=256, smem=0, block=None):
     """The generated worker source for a user kernel (no GPU needed)."""
+    bx, by, bz = block if block is not None else (threads, 1, 1)
     n = ctypes.c_size_t()
-    st = _lib.slate_transform_source(source.encode(), name.encode(), threads, smem, None, 0, ctypes.byref(n))
+    st = _lib.slate_transform_source(source.encode(), name.encode(), bx, by, bz, smem, None, 0, ctypes.byref(n))
     if st != OK:
         raise SlateError(st, "slate_transform_source")
     buf = ctypes.create_string_buffer(n.value + 1)
-    _lib.slate_transform_source(source.encode(), name.encode(), threads, smem, buf, n.value + 1, ctypes.byref(n))
+    _lib.slate_transform_source(source.encode(), name.encode(), bx, by, bz, smem, buf, n.value + 1, ctypes.byref(n))
     return buf.value.decode()
+
+
+def rtc_stats():
+    """(NVRTC compiles, in-process cache hits, on-disk cache hits) of this process."""
+    a, b, c = c_u64(), c_u64(), c_u64()
+    _lib.slate_rtc_stats(ctypes.byref(a), ctypes.byref(b), ctypes.byref(c))
+    return a.value, b.value, c.value
 
 
 def choose_iters(solo_ms, occ, n_sms, blocks, cap, budget_us=20.0):

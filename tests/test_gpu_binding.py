@@ -1,0 +1,153 @@
+"""The kernel-SM mapping, checked per task (-m gpu).  P:L163 §IV-C: Slate
+"ensures that the kernel only runs on these SMs" (Lst1's sm_low/sm_high); the
+north star: workers "bound to a per-tenant SM range".  With SLATE_KFLAG_RANKLOG
+every task records the SM rank of the worker that took it and the range of the
+resize word that worker acted on (slate.h), so the binding is checked
+directly, not through timing:
+  * two co-runners on disjoint ranges: every task of each ran on a rank inside
+    its own range, and the two rank sets are disjoint (while both ran);
+  * under a random resize storm: every task ran inside the range of a resize
+    word the host published (the initial range or one it requested), except
+    tasks kept by the last live worker (reading Q22), which are flagged;
+and outputs, coverage and counters stay exact throughout."""
+import random
+import time
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import tenants as OT
+from paper_conf_ipps_allenf019_b200 import slate as S
+
+from gpu_helpers import make_bs, make_copy, make_gemm, make_sgemm, make_spmv, make_stencil, make_triad
+
+pytestmark = pytest.mark.gpu
+
+
+def decode_log(cov, B):
+    c = cov.cpu().numpy().view(np.uint32)
+    counts, log = c[:B], c[B:]
+    assert np.all(counts == 1), "coverage"
+    assert np.all(log >> 31 == 1), "every task logged"
+    return log & 0xff, (log >> 8) & 0xff, (log >> 16) & 0xff, (log >> 24) & 1
+
+
+def _run_pair(t_a, t_b, ra, rb, iters_a, iters_b, reps=1):
+    """Launch A and B from two sessions (two queues) at once on disjoint ranges."""
+    sa, sb = S.Session(None, 0), S.Session(None, 0)
+    try:
+        ka = sa.register_kernel(t_a.kind, iters=iters_a, flags=S.KFLAG_COVERAGE | S.KFLAG_RANKLOG)
+        kb = sb.register_kernel(t_b.kind, iters=iters_b, flags=S.KFLAG_COVERAGE | S.KFLAG_RANKLOG)
+        Ba, Bb = int(np.prod(t_a.grid)), int(np.prod(t_b.grid))
+        covs_a = [torch.zeros(2 * Ba, dtype=torch.int32, device="cuda:0") for _ in range(reps)]
+        covs_b = [torch.zeros(2 * Bb, dtype=torch.int32, device="cuda:0") for _ in range(reps)]
+        t_a.zero_outputs()
+        t_b.zero_outputs()
+        torch.cuda.synchronize()
+        la = [sa.launch(ka, t_a.args, t_a.grid, placement=S.PLACE_CORUN, sm=ra, coverage=c) for c in covs_a]
+        lb = [sb.launch(kb, t_b.args, t_b.grid, placement=S.PLACE_CORUN, sm=rb, coverage=c) for c in covs_b]
+        for l in la:
+            sa.sync(l)
+        for l in lb:
+            sb.sync(l)
+        torch.cuda.synchronize()
+        qa, qb = sa.query(la[-1]), sb.query(lb[-1])
+        return covs_a, covs_b, Ba, Bb, (qa, qb)
+    finally:
+        sa.close()
+        sb.close()
+
+
+PAIRS = {
+    "triad+sgemm": (lambda: make_triad(1 << 24, 401), lambda: make_sgemm(512, 512, 512, 402), 10, 2),
+    "spmv+bs": (lambda: make_spmv(1 << 18, 403), lambda: make_bs(1 << 20, 404, n_scen=32), 16, 1),
+    "gemm+copy": (lambda: make_gemm(2048, 2048, 2048, 405, "int"), lambda: make_copy(1 << 26, 406), 1, 10),
+    "stencil+bs": (lambda: make_stencil(4096, 4096, 407), lambda: make_bs(1 << 20, 408, n_scen=8), 10, 2),
+}
+
+
+@pytest.mark.parametrize("name", sorted(PAIRS))
+def test_corunners_run_only_on_their_own_ranks(name):
+    mk_a, mk_b, ia, ib = PAIRS[name]
+    t_a, t_b = mk_a(), mk_b()
+    n = S.Session(None, 0).info()["num_sms"]
+    split = n // 2 if "gemm" not in name else (n // 2) & ~1
+    ra, rb = (0, split - 1), (split, n - 1)
+    covs_a, covs_b, Ba, Bb, _ = _run_pair(t_a, t_b, ra, rb, ia, ib, reps=2)
+    ok_a, _ = t_a.check(t_a.snapshot())
+    ok_b, _ = t_b.check(t_b.snapshot())
+    assert ok_a and ok_b
+    ranks_a, ranks_b = set(), set()
+    for covs, B, (lo_r, hi_r), acc in ((covs_a, Ba, ra, ranks_a), (covs_b, Bb, rb, ranks_b)):
+        for cov in covs:
+            rank, lo, hi, outside = decode_log(cov, B)
+            # the range each task's worker acted on: its own range, or (after the
+            # partner finished first) the whole chip it grew to
+            own = (lo == lo_r) & (hi == hi_r)
+            grown = (lo == 0) & (hi == n - 1)
+            assert np.all(own | grown), (name, set(zip(lo.tolist(), hi.tolist())))
+            assert np.all((rank >= lo) & (rank <= hi) | (outside == 1)), name
+            assert outside.sum() == 0, name
+            acc.update(rank[own].tolist())
+    assert ranks_a and ranks_b
+    assert ranks_a <= set(range(ra[0], ra[1] + 1)) and ranks_b <= set(range(rb[0], rb[1] + 1))
+    assert not (ranks_a & ranks_b), name
+
+
+STORMS = {
+    "bs": (lambda: make_bs(1 << 21, 411, n_scen=64), 1),
+    "stencil": (lambda: make_stencil(8192, 4096, 412), 4),
+    "spmv": (lambda: make_spmv(1 << 20, 413), 8),
+    "gemm": (lambda: make_gemm(8192, 8192, 8192, 414, "int"), 1),
+}
+
+
+@pytest.mark.parametrize("name", sorted(STORMS))
+def test_rank_log_under_resize_storm(name):
+    mk, iters = STORMS[name]
+    t = mk()
+    s = S.Session(None, 0)
+    try:
+        n = s.info()["num_sms"]
+        k_std = s.register_kernel(t.kind)
+        t.zero_outputs()
+        s.sync(s.launch(k_std, t.args, t.grid, mode=S.MODE_STANDALONE))
+        torch.cuda.synchronize()
+        ref = t.snapshot()   # bit-exact reference: the original kernel (oracle parity: test_gpu_parity.py)
+        k = s.register_kernel(t.kind, iters=iters, flags=S.KFLAG_COVERAGE | S.KFLAG_RANKLOG)
+        B = int(np.prod(t.grid))
+        cov = torch.zeros(2 * B, dtype=torch.int32, device="cuda:0")
+        t.zero_outputs()
+        torch.cuda.synchronize()
+        rng = random.Random(7)
+        requested = {(0, n - 1)}
+        lid = s.launch(k, t.args, t.grid, placement=S.PLACE_CORUN, sm=(0, n - 1), coverage=cov)
+        resizes = 0
+        for _ in range(40):
+            lo = rng.randrange(0, n - 16)
+            hi = rng.randrange(lo + 15, n)
+            if t.kind == S.KIND_GEMM_BF16:   # CTA pairs: even-aligned ranges
+                lo &= ~1
+                hi |= 1
+            requested.add((lo, hi))
+            resizes += 1
+            if s.resize(lid, lo, hi) == S.DONE:
+                break
+            time.sleep(50e-6)
+        s.sync(lid)
+        torch.cuda.synchronize()
+        q = s.query(lid)
+        ex = OT.expected_counters(B, iters)
+        assert (q["blocks_done"], q["tasks_done"]) == (ex["blocks_done"], ex["tasks_done"])
+        for a, b in zip(t.snapshot(), ref):
+            assert torch.equal(a, b), name
+        rank, lo, hi, outside = decode_log(cov, B)
+        ranges = set(zip(lo.tolist(), hi.tolist()))
+        assert ranges <= requested, (name, ranges - requested)
+        assert np.all((rank >= lo) & (rank <= hi) | (outside == 1)), name
+        # only the last live worker may keep a task outside the range (Q22): rare
+        assert outside.sum() <= max(4, B // 100), (name, int(outside.sum()))
+        assert len(ranges) >= 2 or resizes < 2, name   # the storm reached the workers
+    finally:
+        s.close()

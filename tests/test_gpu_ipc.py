@@ -82,3 +82,29 @@ def test_unshared_pointer_is_rejected(daemon):
         s.launch(k, args, grid)
     assert e.value.status == S.EINVAL
     s.close()
+
+
+def test_user_kernel_through_the_daemon(daemon):
+    """NEXT-3 through an endpoint: the source goes over the command channel, the
+    daemon compiles it and rewrites the kernel's pointer parameters (found by
+    the transformation) to its mappings of this client's shared buffers."""
+    import numpy as np
+    import torch
+    from oracle import tenants as OT
+    from paper_conf_ipps_allenf019_b200 import slate as S
+    from test_user_kernels import PROBE3D_SRC, Args3D
+    shape, block = (5, 9, 70), (16, 2, 2)
+    grid = OT.probe3d_grid(shape, block)
+    rng = np.random.default_rng(11)
+    x = rng.integers(-300, 300, size=shape).astype(np.float32)
+    xd = torch.from_numpy(x).cuda()
+    yd = torch.zeros(shape, device="cuda:0")
+    torch.cuda.synchronize()
+    s = S.Session(daemon)
+    s.share_buffer(xd)
+    s.share_buffer(yd)
+    k = s.register_source(PROBE3D_SRC, "probe3d", Args3D, block=block, iters=3)
+    args = Args3D(xd.data_ptr(), yd.data_ptr(), shape[2], shape[1], shape[0])
+    s.sync(s.launch(k, args, grid))
+    assert np.array_equal(yd.cpu().numpy().astype(np.float64), OT.probe3d(x, block))
+    s.close()

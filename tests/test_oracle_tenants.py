@@ -155,3 +155,23 @@ def test_gemm_bf16_int_exact_and_sums():
     Af, Bf = I.gemm_inputs(130, 129, 64, 15)
     np.testing.assert_allclose(T.gemm_bf16(Af, Bf),
                                T.bf16_to_f64(Af) @ T.bf16_to_f64(Bf).T, rtol=1e-13, atol=1e-13)
+
+
+# ------------------------------------------------------------------ probe3d (3-D grid of 3-D blocks)
+def test_probe3d_block_ids_and_linearity():
+    """With a zero input each element holds the id term of the block that
+    wrote it: the block is the element's coordinates integer-divided by the
+    block shape (not decode(): an independent route), and every element of the
+    ragged 3-D field is written exactly once; the input term is linear."""
+    shape, block = (7, 11, 37), (8, 4, 2)          # (nz, ny, nx), (bx, by, bz): ragged in all three
+    assert T.probe3d_grid(shape, block) == (5, 3, 4)
+    z = T.probe3d(np.zeros(shape, np.float32), block)
+    k, j, i = np.meshgrid(np.arange(7), np.arange(11), np.arange(37), indexing="ij")
+    assert np.array_equal(z, (i // 8) + 3 * (j // 4) + 7 * (k // 2))
+    rng = np.random.default_rng(3)
+    x = rng.integers(-50, 50, size=shape).astype(np.float32)
+    assert np.array_equal(T.probe3d(x, block) - z, 2.0 * x.astype(np.float64))
+    # a subset of blocks writes only the elements of those blocks
+    part = T.probe3d(np.ones(shape, np.float32), block, blocks=[17])   # block 17 = (2, 0, 1)
+    nz_ = np.argwhere(part != 0)
+    assert nz_.size and set(map(tuple, (nz_ // [2, 4, 8]).tolist())) == {(1, 0, 2)}

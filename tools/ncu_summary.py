@@ -18,7 +18,8 @@ KEYS = {
     "gpu__time_duration.sum": "duration_us",
     "dram__bytes_read.sum": "dram_read",
     "dram__bytes_write.sum": "dram_write",
-    "FBSP.TriageCompute.dram__throughput.avg.pct_of_peak_sustained_elapsed": "dram_pct",
+    "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed": "dram_pct",
+    "dram__throughput.avg.pct_of_peak_sustained_elapsed": "dram_pct",
     "dram__bytes.sum.per_second": "dram_bytes_per_s",
     "sm__throughput.avg.pct_of_peak_sustained_elapsed": "sm_pct",
     "sm__warps_active.avg.pct_of_peak_sustained_active": "achieved_occupancy_pct",
@@ -32,6 +33,14 @@ KEYS = {
     "lts__t_sectors_op_atom.sum": "l2_atom_sectors",
     "smsp__inst_executed.sum": "inst_executed",
 }
+def _hbm_gbs():
+    for p in ("MEASURED_PEAKS.json", os.path.join(os.path.dirname(__file__), "..", "MEASURED_PEAKS.json")):
+        if os.path.exists(p):
+            return float(json.load(open(p))["hbm_gbs"])
+    return 6465.8   # the driver's measured figure on this pool (MEASURED_PEAKS.json, round 1)
+
+
+HBM_GBS = _hbm_gbs()
 B = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9}
 UNIT = {"dram_read": B, "dram_write": B,
         "duration_us": {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "ns": 1e-3, "us": 1.0, "ms": 1e3}}
@@ -55,6 +64,9 @@ def main(rep, out):
                     continue
                 v *= UNIT.get(name, {}).get(units[i], 1.0)
                 d[name] = v
+        if "dram_pct" not in d and d.get("duration_us"):
+            # no throughput metric in the capture: DRAM bytes / duration against the measured peak
+            d["dram_pct"] = 100.0 * (d.get("dram_read", 0) + d.get("dram_write", 0)) / (d["duration_us"] * 1e-6) / (HBM_GBS * 1e9)
         stalls = []
         for i in stall_cols:
             try:
@@ -65,7 +77,15 @@ def main(rep, out):
         d["top_stalls"] = [[h.split("stalled_")[-1].replace("_per_issue_active.ratio", ""), round(v, 2)]
                            for v, h in stalls[:5]]
         launches.append(d)
-    json.dump({"report": os.path.basename(rep), "launches": launches}, open(out + ".json", "w"), indent=1)
+    write(launches, os.path.basename(rep), out)
+
+
+def write(launches, rep_name, out):
+    for d in launches:
+        if d.get("dram_pct") is None and d.get("duration_us"):
+            d["dram_pct"] = 100.0 * (d.get("dram_read", 0) + d.get("dram_write", 0)) / (d["duration_us"] * 1e-6) / (HBM_GBS * 1e9)
+    json.dump({"report": rep_name, "launches": launches}, open(out + ".json", "w"), indent=1)
+    rep = rep_name
     with open(out + ".md", "w") as f:
         f.write("# ncu summary: %s\n\n" % os.path.basename(rep))
         f.write("| kernel | us | DRAM read MB | DRAM write MB | DRAM % | SM % | occ % | regs | grid | top stalls |\n")
@@ -89,4 +109,8 @@ def main(rep, out):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2])
+    if sys.argv[1] == "--from-json":   # re-render a summary already extracted (the .ncu-rep is scratch)
+        j = json.load(open(sys.argv[2] + ".json"))
+        write(j["launches"], j["report"], sys.argv[2])
+    else:
+        main(sys.argv[1], sys.argv[2])
