@@ -168,8 +168,9 @@ slate_status slate_unshare_buffer(slate_session* s, uint64_t handle);
  * took the task holding b, written by the fetching thread when it hands the
  * task out: bits 0-7 the worker's SM rank (for a GEMM CTA pair, the leader's),
  * bits 8-15 / 16-23 the range [lo, hi] of the resize word the worker acted on
- * (intersected with a top-up's bound), bit 24 set if the worker was outside
- * that range and kept the task only because it was the last live worker
+ * (as published; a top-up worker is also bound to the ranks it was launched
+ * for), bit 24 set if the worker was outside its range and kept the task only
+ * because it was the last live worker
  * (reading Q22), bit 31 set (valid).  It makes "the kernel only runs on these
  * SMs" (§IV-C, Lst1) checkable per task. */
 #define SLATE_KFLAG_RANKLOG 2u

@@ -131,9 +131,10 @@ struct BlockWalk {
 // ------------------------------------------------------------------ rank log (debug, SLATE_KFLAG_RANKLOG)
 // Who took each task: written by the fetching lane when it hands out task
 // [g, g+n), one word per block at cov[B + b]: the worker's SM rank, the range
-// [lo, hi] of the resize word it acted on (intersected with the launch bound),
-// and flags -- bit 0: the worker was outside that range and kept the task only
-// under the last-live-worker rule (Q22), bit 7: valid.  Tests check that every
+// [lo, hi] of the resize word it acted on (as the host published it; a top-up
+// worker is further bound to the ranks it was launched for), and flags --
+// bit 0: the worker was outside its range and kept the task only under the
+// last-live-worker rule (Q22), bit 7: valid.  Tests check that every
 // task ran on a rank inside the range in force ("ensures that the
 // kernel only runs on these SMs") and that co-runners' rank sets are disjoint.
 __device__ __forceinline__ uint32_t ranklog_entry(uint32_t rank, uint32_t lo, uint32_t hi, bool outside) {
@@ -142,8 +143,7 @@ __device__ __forceinline__ uint32_t ranklog_entry(uint32_t rank, uint32_t lo, ui
 template <class P>
 __device__ __forceinline__ void log_task(const P& p, uint32_t g, uint32_t rank, uint64_t c, bool outside) {
   if (!p.ranklog || !p.cov || g >= p.B) return;
-  const uint32_t lo = max(ctrl_lo(c), p.bound_lo), hi = min(ctrl_hi(c), p.bound_hi);
-  const uint32_t e = ranklog_entry(rank, lo, hi, outside), n = min(p.iters, p.B - g);
+  const uint32_t e = ranklog_entry(rank, ctrl_lo(c), ctrl_hi(c), outside), n = min(p.iters, p.B - g);
   for (uint32_t i = 0; i < n; ++i) p.cov[p.B + g + i] = e;
 }
 

@@ -76,7 +76,9 @@ def run_user(s, n_sms):
 
 
 def main():
+    import faulthandler
     groups = sys.argv[1:] or list(GROUPS) + ["user"]
+    faulthandler.dump_traceback_later(float(os.environ.get("SANITIZE_DUMP_S", "600")), exit=True)
     with S.Session(None, 0) as s:
         n = s.info()["num_sms"]
         for g in groups:
@@ -86,6 +88,7 @@ def main():
                 for mk in GROUPS[g]:
                     run(s, mk(), n)
             print("SANITIZE-OK", g, flush=True)
+    print("SANITIZE-CLOSED", flush=True)
 
 
 if __name__ == "__main__":
