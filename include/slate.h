@@ -438,6 +438,18 @@ uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t 
                             const uint32_t* sms_b, const double* ms_b, uint32_t n_b,
                             uint32_t n_sms, uint32_t step, uint32_t lo_b, uint32_t hi_b,
                             double* makespan_ms);
+/* The split objective (reading Q41).  MAKESPAN: slate_choose_split's.  ANTT:
+ * among the splits whose fluid-model makespan is within `slack` (e.g. 0.05) of
+ * the best, the one with the least ANTT = mean over the two jobs of co-run
+ * completion / solo time on all SMs (Eyerman; a makespan-only split can double
+ * the shorter job's turnaround).  *makespan_ms and *antt (may be NULL) receive
+ * the chosen split's predictions. */
+#define SLATE_SPLIT_MAKESPAN 0u
+#define SLATE_SPLIT_ANTT     1u
+uint32_t slate_choose_split_obj(const uint32_t* sms_a, const double* ms_a, uint32_t n_a,
+                                const uint32_t* sms_b, const double* ms_b, uint32_t n_b,
+                                uint32_t n_sms, uint32_t step, uint32_t lo_b, uint32_t hi_b,
+                                uint32_t objective, double slack, double* makespan_ms, double* antt);
 /* Reading Q29 (bandwidth saturation cap): the fewest SMs (1..n_sms) on which
  * a solo curve (sms ascending, ms) comes within frac (0 < frac <= 1) of its
  * full-chip rate: interp(s) <= interp(n_sms) / frac.  The scheduler caps a
@@ -473,6 +485,18 @@ int slate_fluid_corun(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, d
                       const uint32_t* sms_b, const double* ms_b, uint32_t n_b, double work_b,
                       uint32_t n_sms, uint32_t step, uint32_t lo_b, uint32_t hi_b, double min_gain,
                       uint32_t* split, double* gain);
+
+/* slate_fluid_corun with the split taken under `objective` / `slack`
+ * (slate_choose_split_obj); the gain is T_seq over that split's makespan. */
+int slate_fluid_corun_obj(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, double work_a,
+                          const uint32_t* sms_b, const double* ms_b, uint32_t n_b, double work_b,
+                          uint32_t n_sms, uint32_t step, uint32_t lo_b, uint32_t hi_b, double min_gain,
+                          uint32_t objective, double slack, uint32_t* split, double* gain);
+
+/* The split objective of the server's co-runs (process-wide; initial value
+ * from SLATE_SPLIT_OBJECTIVE = makespan | antt and SLATE_SPLIT_SLACK in the
+ * server's environment, default antt with slack 0.05).  Errors: EINVAL. */
+slate_status slate_set_split_objective(slate_session* s, uint32_t objective, double slack);
 
 /* Selector policy of the server (process-wide; the initial value comes from
  * SLATE_POLICY = table | literal | hybrid in the server's environment, default

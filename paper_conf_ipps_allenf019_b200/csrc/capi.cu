@@ -243,6 +243,15 @@ slate_status slate_set_policy(slate_session* s, uint32_t policy) {
   return rc >= SLATE_OK ? rc : fail(s, rc, err);
 }
 
+slate_status slate_set_split_objective(slate_session* s, uint32_t objective, double slack) {
+  if (!s) return SLATE_EINVAL;
+  std::lock_guard<std::mutex> g(s->mu);
+  std::string err;
+  const int rc = s->srv ? s->srv->set_split_objective(objective, slack, &err)
+                        : s->remote->set_split_objective(objective, slack, &err);
+  return rc >= SLATE_OK ? rc : fail(s, rc, err);
+}
+
 slate_status slate_sync(slate_session* s, slate_launch_id l, int64_t timeout_us) {
   if (!s) return SLATE_EINVAL;
   std::string err;

@@ -91,9 +91,21 @@ __device__ __forceinline__ void cluster_sync() {
 __device__ __forceinline__ void st_cluster(uint32_t raddr, uint32_t v) {
   asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(raddr), "r"(v) : "memory");
 }
+// the leader's progress word in the peer's shared memory: only ever raised
+// (K slices issued, bit 31 when it stopped), so the writer is an atomic max and
+// the reader an atomic read -- both cluster-scope atomics, no plain access
+__device__ __forceinline__ void red_max_cluster(uint32_t raddr, uint32_t v) {
+  asm volatile("red.relaxed.cluster.shared::cluster.max.u32 [%0], %1;" ::"r"(raddr), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint32_t ld_relaxed_cluster(const volatile uint32_t* p) {
   uint32_t v;
-  asm volatile("ld.relaxed.cluster.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(s_u32((const void*)p)) : "memory");
+  asm volatile("atom.relaxed.cluster.shared::cta.or.b32 %0, [%1], 0;" : "=r"(v) : "r"(s_u32((const void*)p)) : "memory");
+  return v;
+}
+// a 32-bit word of another CTA's shared memory (after a cluster barrier)
+__device__ __forceinline__ uint32_t ld_shared_cluster(uint32_t raddr) {
+  uint32_t v;
+  asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(raddr) : "memory");
   return v;
 }
 __device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t n) {
@@ -319,13 +331,13 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
     if (threadIdx.x == 0) {
       S.rank = p.rank_of[smid()];
       S.retired = 0;
-      if (!leader) st_cluster(mapa(&S.peer_rank, 0), S.rank);
     }
   }
-  cluster_sync();
+  cluster_sync();   // the peer's rank is written (and both CTAs run) before any DSMEM access
   if constexpr (kSlate) {
     // ---- Lst1 binding + standby, by the leader for the pair
     if (leader && threadIdx.x == 0) {
+      S.peer_rank = ld_shared_cluster(mapa(&S.rank, 1));
       const uint32_t go = pair_prologue(p, S.rank, S.peer_rank, c) ? 1u : 0u;
       S.go = go;
       st_cluster(mapa(&S.go, 1), go);
@@ -419,7 +431,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
                 c = c2;
                 S.retired = 1;
                 S.kb_limit[j] = kb;            // the MMA consumes the kb slices issued, then aborts
-                st_cluster(r_issued, it | 0x80000000u);   // ... and the peer issues exactly those
+                red_max_cluster(r_issued, it | 0x80000000u);   // ... and the peer issues exactly those
                 stop = true;
                 break;
               }
@@ -431,7 +443,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
           mbar_expect_tx(&S.full[s], kPairStageBytes);
           tma_load_half(sa, &p.tma_a, int(kb * BK), int(m0), full0 + s * 8);
           tma_load_half(sa + kHalfBytes, &p.tma_b, int(kb * BK), int(n0), full0 + s * 8);
-          st_cluster(r_issued, it + 1);   // one location, so the peer sees the counts in order
+          red_max_cluster(r_issued, it + 1);   // one location, so the peer sees the counts in order
         }
       }
     }

@@ -293,6 +293,15 @@ int RemoteClient::set_policy(uint32_t policy, std::string* err) {
   return call(rq, &rs, err);
 }
 
+int RemoteClient::set_split_objective(uint32_t objective, double slack, std::string* err) {
+  Request rq{};
+  rq.cmd = CMD_SPLIT;
+  rq.lo = objective;
+  std::memcpy(rq.args, &slack, sizeof(slack));
+  Response rs;
+  return call(rq, &rs, err);
+}
+
 int RemoteClient::sync(uint64_t l, int64_t timeout_us, std::string* err) {
   Request rq{};
   rq.cmd = CMD_SYNC;

@@ -30,7 +30,8 @@ enum Cmd : uint32_t {
   CMD_NONE = 0, CMD_INFO, CMD_SHARE, CMD_UNSHARE, CMD_REGISTER, CMD_LAUNCH, CMD_RESIZE, CMD_SYNC, CMD_PROFILE,
   CMD_QUERY, CMD_DETACH, CMD_POLICY,
   CMD_SOURCE_CHUNK,        // append args[0, lo) to the session's source buffer (flags & 1: start a new one)
-  CMD_REGISTER_SOURCE      // compile the buffered source: args holds a SourceReg (NEXT-3 through an endpoint)
+  CMD_REGISTER_SOURCE,     // compile the buffered source: args holds a SourceReg (NEXT-3 through an endpoint)
+  CMD_SPLIT                // the split objective: lo = objective, args = the slack (double)
 };
 
 // CMD_REGISTER_SOURCE's argument block (slate_source_desc without the strings)
@@ -108,6 +109,7 @@ class RemoteClient {
   int launch_n(uint64_t k, const slate_launch_desc* d, uint32_t n, uint64_t* first, std::string* err);
   int resize(uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
   int set_policy(uint32_t policy, std::string* err);
+  int set_split_objective(uint32_t objective, double slack, std::string* err);
   int sync(uint64_t l, int64_t timeout_us, std::string* err);
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);

@@ -2,6 +2,7 @@
 // algorithm and the SM split (§III-B; readings Q8-Q10, Q13 in
 // DESIGN.md).  Pure host functions, exported through the C ABI so they can be
 // checked against the oracle without a GPU.
+#include <algorithm>
 #include <cmath>
 #include <functional>
 #include <cstdint>
@@ -81,46 +82,88 @@ uint32_t slate_saturation_sms(const uint32_t* sms, const double* ms, uint32_t n,
   return n_sms;
 }
 
-uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, const uint32_t* sms_b,
-                            const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
-                            uint32_t hi_b, double* makespan_ms) {
+// fluid model: completion times of A on n-s SMs and B on s SMs, the
+// first to finish handing its SMs to the other (oracle selector.corun_times)
+static void corun_times(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, const uint32_t* sms_b,
+                        const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t s, double* t_a, double* t_b) {
+  const double ta = interp(sms_a, ms_a, n_a, double(n_sms - s));
+  const double tb = interp(sms_b, ms_b, n_b, double(s));
+  if (tb <= ta) {
+    *t_a = tb + (1.0 - tb / ta) * interp(sms_a, ms_a, n_a, n_sms);
+    *t_b = tb;
+  } else {
+    *t_a = ta;
+    *t_b = ta + (1.0 - ta / tb) * interp(sms_b, ms_b, n_b, n_sms);
+  }
+}
+
+uint32_t slate_choose_split_obj(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, const uint32_t* sms_b,
+                                const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
+                                uint32_t hi_b, uint32_t objective, double slack, double* makespan_ms, double* antt) {
   if (step == 0) step = 1;
-  double best_t = std::numeric_limits<double>::infinity();
-  uint32_t best_s = n_sms / 2;
   const double ta_full = interp(sms_a, ms_a, n_a, n_sms), tb_full = interp(sms_b, ms_b, n_b, n_sms);
   std::vector<uint32_t> cands;
   for (uint32_t s = step; s + step <= n_sms; s += step)
     if ((!lo_b || s >= lo_b) && (!hi_b || s <= hi_b)) cands.push_back(s);
   if (cands.empty())   // the bounds exclude every candidate: the bound nearest the range
     cands.push_back(std::min(std::max(step, lo_b ? lo_b : step), n_sms - step));
-  for (uint32_t s : cands) {
-    const double ta = interp(sms_a, ms_a, n_a, double(n_sms - s));
-    const double tb = interp(sms_b, ms_b, n_b, double(s));
-    // fluid model: the first to finish hands its SMs to the other
-    const double t = tb <= ta ? tb + (1.0 - tb / ta) * ta_full : ta + (1.0 - ta / tb) * tb_full;
-    if (t < best_t - 1e-12) {
-      best_t = t;
-      best_s = s;
+  std::vector<double> mk(cands.size()), an(cands.size());
+  double best_t = std::numeric_limits<double>::infinity();
+  size_t best = 0;
+  for (size_t i = 0; i < cands.size(); ++i) {
+    double a, b;
+    corun_times(sms_a, ms_a, n_a, sms_b, ms_b, n_b, n_sms, cands[i], &a, &b);
+    mk[i] = std::max(a, b);
+    an[i] = 0.5 * (a / ta_full + b / tb_full);
+    if (mk[i] < best_t - 1e-12) {
+      best_t = mk[i];
+      best = i;
     }
   }
-  if (makespan_ms) *makespan_ms = best_t;
-  return best_s;
+  if (objective == SLATE_SPLIT_ANTT) {   // reading Q41: least ANTT within `slack` of the best makespan
+    const double bound = best_t * (1.0 + slack);
+    double best_a = std::numeric_limits<double>::infinity();
+    for (size_t i = 0; i < cands.size(); ++i)
+      if (mk[i] <= bound + 1e-12 && an[i] < best_a - 1e-12) {
+        best_a = an[i];
+        best = i;
+      }
+  }
+  if (makespan_ms) *makespan_ms = mk[best];
+  if (antt) *antt = an[best];
+  return cands[best];
 }
 
-int slate_fluid_corun(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, double work_a, const uint32_t* sms_b,
-                      const double* ms_b, uint32_t n_b, double work_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
-                      uint32_t hi_b, double min_gain, uint32_t* split, double* gain) {
+uint32_t slate_choose_split(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, const uint32_t* sms_b,
+                            const double* ms_b, uint32_t n_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
+                            uint32_t hi_b, double* makespan_ms) {
+  return slate_choose_split_obj(sms_a, ms_a, n_a, sms_b, ms_b, n_b, n_sms, step, lo_b, hi_b, SLATE_SPLIT_MAKESPAN,
+                                0.0, makespan_ms, nullptr);
+}
+
+int slate_fluid_corun_obj(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, double work_a,
+                          const uint32_t* sms_b, const double* ms_b, uint32_t n_b, double work_b, uint32_t n_sms,
+                          uint32_t step, uint32_t lo_b, uint32_t hi_b, double min_gain, uint32_t objective,
+                          double slack, uint32_t* split, double* gain) {
   // job curves: `work` launches of the kernel, back to back on the same SMs
   std::vector<double> ja(ms_a, ms_a + n_a), jb(ms_b, ms_b + n_b);
   for (double& v : ja) v *= work_a;
   for (double& v : jb) v *= work_b;
   double t_co = 0;
-  const uint32_t s = slate_choose_split(sms_a, ja.data(), n_a, sms_b, jb.data(), n_b, n_sms, step, lo_b, hi_b, &t_co);
+  const uint32_t s = slate_choose_split_obj(sms_a, ja.data(), n_a, sms_b, jb.data(), n_b, n_sms, step, lo_b, hi_b,
+                                            objective, slack, &t_co, nullptr);
   const double t_seq = interp(sms_a, ja.data(), n_a, n_sms) + interp(sms_b, jb.data(), n_b, n_sms);
   const double g = t_co > 0 ? t_seq / t_co : 0.0;
   if (split) *split = s;
   if (gain) *gain = g;
   return g >= min_gain ? 1 : 0;
+}
+
+int slate_fluid_corun(const uint32_t* sms_a, const double* ms_a, uint32_t n_a, double work_a, const uint32_t* sms_b,
+                      const double* ms_b, uint32_t n_b, double work_b, uint32_t n_sms, uint32_t step, uint32_t lo_b,
+                      uint32_t hi_b, double min_gain, uint32_t* split, double* gain) {
+  return slate_fluid_corun_obj(sms_a, ms_a, n_a, work_a, sms_b, ms_b, n_b, work_b, n_sms, step, lo_b, hi_b, min_gain,
+                               SLATE_SPLIT_MAKESPAN, 0.0, split, gain);
 }
 
 uint32_t slate_choose_iters(double solo_ms, uint32_t occ, uint32_t n_sms, uint32_t B, uint32_t cap, double budget_us) {

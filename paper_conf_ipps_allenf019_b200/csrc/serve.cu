@@ -259,6 +259,12 @@ int Session::handle(const Request& rq, Response& rs) {
     case CMD_POLICY:
       rc = srv_->set_policy(rq.lo, &err);
       break;
+    case CMD_SPLIT: {
+      double slack;
+      std::memcpy(&slack, rq.args, sizeof(slack));
+      rc = srv_->set_split_objective(rq.lo, slack, &err);
+      break;
+    }
     case CMD_QUERY:
       rc = srv_->query(rq.id, &rs.linfo, &err);
       break;

@@ -149,6 +149,9 @@ int Server::init(std::string* err) {
     task_budget_us_ = env_double("SLATE_TASK_BUDGET_US", 20.0);
   }
   min_gain_ = env_double("SLATE_MIN_GAIN", 1.05);
+  if (const char* o = std::getenv("SLATE_SPLIT_OBJECTIVE"))
+    split_objective_ = std::string(o) == "makespan" ? SLATE_SPLIT_MAKESPAN : SLATE_SPLIT_ANTT;
+  split_slack_ = env_double("SLATE_SPLIT_SLACK", 0.05);
   poller_ = std::thread([this] { poller_main(); });
   return SLATE_OK;
 }
@@ -1206,6 +1209,17 @@ int Server::set_policy(uint32_t policy, std::string* err) {
   return SLATE_OK;
 }
 
+int Server::set_split_objective(uint32_t objective, double slack, std::string* err) {
+  if (objective > SLATE_SPLIT_ANTT || !(slack >= 0.0 && slack <= 1.0)) {
+    if (err) *err = "unknown split objective or slack outside [0, 1]";
+    return SLATE_EINVAL;
+  }
+  std::lock_guard<std::mutex> g(mu_);
+  split_objective_ = objective;
+  split_slack_ = slack;
+  return SLATE_OK;
+}
+
 // the launch's solo curve from the profile table, ascending in SMs
 bool Server::curve_of(const Launch& L, std::vector<uint32_t>* sms, std::vector<double>* ms) const {
   slate_launch_desc d = L.desc;
@@ -1241,8 +1255,8 @@ uint32_t Server::pair_split(const Launch& LA, const Queue& A, const Launch& LB, 
   const double wa = double(std::max<size_t>(1, A.issued.size() + A.pending.size()));
   const double wb = double(std::max<size_t>(1, B.issued.size() + B.pending.size()));
   uint32_t s = uint32_t(n_sms_ / 2);
-  slate_fluid_corun(sa.data(), ta.data(), uint32_t(sa.size()), wa, sb.data(), tb.data(), uint32_t(sb.size()), wb,
-                    uint32_t(n_sms_), 2, lo_b, hi_b, min_gain_, &s, gain);
+  slate_fluid_corun_obj(sa.data(), ta.data(), uint32_t(sa.size()), wa, sb.data(), tb.data(), uint32_t(sb.size()), wb,
+                        uint32_t(n_sms_), 2, lo_b, hi_b, min_gain_, split_objective_, split_slack_, &s, gain);
   return s;
 }
 

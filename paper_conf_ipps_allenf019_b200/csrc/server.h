@@ -113,6 +113,7 @@ class Server {
                   std::string* err);
   int resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
   int set_policy(uint32_t policy, std::string* err);
+  int set_split_objective(uint32_t objective, double slack, std::string* err);
   int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);
@@ -209,6 +210,8 @@ class Server {
   double saturation_frac_ = 0.95;
   uint32_t policy_ = SLATE_POLICY_HYBRID;
   double min_gain_ = 1.05;
+  uint32_t split_objective_ = SLATE_SPLIT_ANTT;   // reading Q41
+  double split_slack_ = 0.05;
 
   mutable std::mutex mu_;
   std::condition_variable cv_;       // state changes (completion, activation)

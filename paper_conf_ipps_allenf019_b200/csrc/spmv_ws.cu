@@ -286,6 +286,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     // ===================== task warp: the slate task protocol + row-pointer slices =====================
     uint64_t c = H.ctrl;
     const uint32_t rank = H.rank;
+    __syncwarp();   // every lane has read H.ctrl before lane 0 may rewrite it (the stop sentinel)
     TRACE_DECL;
     // Speculative boundary (as the generic worker's kSpeculative mode): the
     // decision for task t+1 -- retire, or the counter atomic -- is taken when

@@ -182,6 +182,14 @@ _lib.slate_choose_split_k.restype = c_f64
 _lib.slate_choose_split_k.argtypes = [ctypes.c_void_p, ctypes.c_void_p, _P(c_u32), c_u32, c_u32, c_u32, _P(c_u32)]
 _lib.slate_choose_iters.restype = c_u32
 _lib.slate_choose_iters.argtypes = [c_f64, c_u32, c_u32, c_u32, c_u32, c_f64]
+_lib.slate_choose_split_obj.restype = c_u32
+_lib.slate_choose_split_obj.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), _P(c_f64), c_u32, c_u32, c_u32, c_u32,
+                                        c_u32, c_u32, c_f64, _P(c_f64), _P(c_f64)]
+_lib.slate_fluid_corun_obj.restype = ctypes.c_int
+_lib.slate_fluid_corun_obj.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_f64, _P(c_u32), _P(c_f64), c_u32, c_f64, c_u32,
+                                       c_u32, c_u32, c_u32, c_f64, c_u32, c_f64, _P(c_u32), _P(c_f64)]
+_lib.slate_set_split_objective.restype = c_i32
+_lib.slate_set_split_objective.argtypes = [ctypes.c_void_p, c_u32, c_f64]
 _lib.slate_fluid_corun.restype = ctypes.c_int
 _lib.slate_fluid_corun.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_f64, _P(c_u32), _P(c_f64), c_u32, c_f64, c_u32,
                                    c_u32, c_u32, c_u32, c_f64, _P(c_u32), _P(c_f64)]
@@ -195,7 +203,7 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
             "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters",
             "slate_register_source", "slate_transform_source", "slate_corun_makespan_k", "slate_choose_split_k",
-            "slate_rtc_stats"]
+            "slate_rtc_stats", "slate_choose_split_obj", "slate_fluid_corun_obj", "slate_set_split_objective"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -319,6 +327,10 @@ class Session:
         """Selector policy of the server (POLICY_TABLE / LITERAL / HYBRID; reading Q31)."""
         return self._check(_lib.slate_set_policy(self._h, policy), "slate_set_policy")
 
+    def set_split_objective(self, objective="antt", slack=0.05):
+        """The split objective of the server's co-runs (reading Q41): "makespan" or "antt"."""
+        return self._check(_lib.slate_set_split_objective(self._h, _OBJ[objective], slack), "slate_set_split_objective")
+
     def sync(self, launch_id=0, timeout_us=-1):
         return self._check(_lib.slate_sync(self._h, launch_id, timeout_us), "slate_sync")
 
@@ -358,20 +370,26 @@ def _curve(c):
     return (c_u32 * len(k))(*k), (c_f64 * len(k))(*[c[x] for x in k]), len(k)
 
 
-def choose_split(curve_a, curve_b, n_sms, step=2, lo_b=0, hi_b=0):
+SPLIT_MAKESPAN, SPLIT_ANTT = 0, 1
+_OBJ = {"makespan": SPLIT_MAKESPAN, "antt": SPLIT_ANTT}
+
+
+def choose_split(curve_a, curve_b, n_sms, step=2, lo_b=0, hi_b=0, objective="makespan", slack=0.05, with_antt=False):
     sa, ta, na = _curve(curve_a)
     sb, tb, nb = _curve(curve_b)
-    t = c_f64()
-    s = _lib.slate_choose_split(sa, ta, na, sb, tb, nb, n_sms, step, lo_b, hi_b, ctypes.byref(t))
-    return s, t.value
+    t, a = c_f64(), c_f64()
+    s = _lib.slate_choose_split_obj(sa, ta, na, sb, tb, nb, n_sms, step, lo_b, hi_b, _OBJ[objective], slack,
+                                    ctypes.byref(t), ctypes.byref(a))
+    return (s, t.value, a.value) if with_antt else (s, t.value)
 
 
-def fluid_corun(curve_a, work_a, curve_b, work_b, n_sms, step=2, lo_b=0, hi_b=0, min_gain=1.05):
+def fluid_corun(curve_a, work_a, curve_b, work_b, n_sms, step=2, lo_b=0, hi_b=0, min_gain=1.05,
+                objective="makespan", slack=0.05):
     sa, ta, na = _curve(curve_a)
     sb, tb, nb = _curve(curve_b)
     s, g = c_u32(), c_f64()
-    r = _lib.slate_fluid_corun(sa, ta, na, work_a, sb, tb, nb, work_b, n_sms, step, lo_b, hi_b, min_gain,
-                               ctypes.byref(s), ctypes.byref(g))
+    r = _lib.slate_fluid_corun_obj(sa, ta, na, work_a, sb, tb, nb, work_b, n_sms, step, lo_b, hi_b, min_gain,
+                                   _OBJ[objective], slack, ctypes.byref(s), ctypes.byref(g))
     return bool(r), s.value, g.value
 
 

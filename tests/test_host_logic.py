@@ -102,6 +102,25 @@ def test_choose_split_bounds_and_saturation_match_oracle(S):
         assert s1 == s2 or abs(OS.corun_makespan(ca, cb, 148, s1) - t2) <= 1e-9 * t2
 
 
+def test_turnaround_split_matches_oracle(S):
+    """Reading Q41: slate_choose_split_obj(ANTT) == oracle choose_split(objective="antt")."""
+    rng = random.Random(41)
+    pts = [148, 111, 74, 49, 37, 18]
+    for _ in range(300):
+        knee_a, knee_b = rng.uniform(10, 148), rng.uniform(10, 148)
+        ca = {s: rng.uniform(0.2, 5) * max(1.0, knee_a / s) for s in pts}
+        cb = {s: rng.uniform(0.2, 5) * max(1.0, knee_b / s) for s in pts}
+        slack = rng.choice([0.0, 0.02, 0.05, 0.2])
+        lo = rng.choice([0, 0, rng.randrange(1, 148)])
+        s1, t1, a1 = S.choose_split(ca, cb, 148, 2, lo, 0, objective="antt", slack=slack, with_antt=True)
+        s2, t2 = OS.choose_split(ca, cb, 148, 2, lo, 0, objective="antt", slack=slack)
+        a2 = OS.corun_antt(ca, cb, 148, s2)
+        assert abs(a1 - a2) <= 1e-9 * a2 and abs(t1 - t2) <= 1e-9 * t2 or s1 == s2
+        r1 = S.fluid_corun(ca, 7, cb, 13, 148, 2, lo, 0, objective="antt", slack=slack)
+        r2 = OS.fluid_corun(ca, 7, cb, 13, 148, 2, lo, 0, objective="antt", slack=slack)
+        assert abs(r1[2] - r2[2]) <= 1e-9 * r2[2]
+
+
 def test_fluid_corun_matches_oracle(S):
     rng = random.Random(13)
     pts = [148, 111, 74, 49, 37, 18]

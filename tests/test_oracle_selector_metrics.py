@@ -95,6 +95,44 @@ def test_split_fluid_model():
     assert S.interp_time(curve_a, 148) == 1.0 and S.interp_time(curve_a, 200) == 1.0
 
 
+def test_turnaround_split_reading_q41():
+    """The ANTT objective against closed forms.  Linear curves T_i(s) = W_i n / s
+    are work-conserving: every split has makespan W_A + W_B, so all are feasible,
+    A's completion is W_A + W_B whatever s, and B's is W_B n / s while B runs
+    first -- ANTT falls as B (the shorter job) gets more SMs: the objective gives
+    it all but one step, the textbook shortest-job-first limit."""
+    n = 148
+    wa, wb = 3.0, 1.0
+    lin_a = {k: wa * n / k for k in (37, 74, 148)}
+    lin_b = {k: wb * n / k for k in (37, 74, 148)}
+    s, t = S.choose_split(lin_a, lin_b, n, objective="antt")
+    assert s == n - 2 and abs(t - (wa + wb)) < 1e-9
+    ta, tb = S.corun_times(lin_a, lin_b, n, s)
+    assert abs(ta - (wa + wb)) < 1e-9 and abs(tb - wb * n / (n - 2)) < 1e-9
+    assert abs(S.corun_antt(lin_a, lin_b, n, s) - 0.5 * ((wa + wb) / wa + n / (n - 2))) < 1e-12
+    # swapped roles: the shorter job is A, so B gets the least
+    s2, _ = S.choose_split(lin_b, lin_a, n, objective="antt")
+    assert s2 == 2
+    # a memory job B saturating at 37 SMs beside a linear compute job A: every
+    # s >= 37 finishes B at its solo time and A then loses time with every SM
+    # more, so the turnaround objective stops at the knee rounded up to the
+    # step (38); the makespan objective gives B fewer (30: B finishes later,
+    # A earlier, the two ends closer together)
+    curve_a = {k: n / k for k in (18, 37, 74, 111, 148)}
+    curve_b = {k: max(1.0, 37.0 / k) for k in (18, 37, 74, 111, 148)}
+    s_m, t_m = S.choose_split(curve_a, curve_b, n)
+    s_a, t_a = S.choose_split(curve_a, curve_b, n, objective="antt", slack=0.5)
+    assert s_m == 30 and abs(t_m - 1.25) < 1e-12
+    assert s_a == 38 and S.corun_times(curve_a, curve_b, n, 38)[1] == 1.0
+    assert S.corun_antt(curve_a, curve_b, n, 38) < S.corun_antt(curve_a, curve_b, n, 30)
+    # the slack bounds the makespan given up for turnaround
+    for slack in (0.0, 0.02, 0.1):
+        _, tt = S.choose_split(curve_a, curve_b, n, objective="antt", slack=slack)
+        assert tt <= t_m * (1 + slack) + 1e-12
+    _, t0 = S.choose_split(curve_a, curve_b, n, objective="antt", slack=0.0)
+    assert abs(t0 - t_m) < 1e-12
+
+
 def test_saturation_cap_reading_q29():
     # throughput linear between (37, 1/2T) and (74, 1/T): rate(s) = s / (74 T) there,
     # so rate >= 0.9 / T first holds at s = ceil(0.9 * 74) = 67

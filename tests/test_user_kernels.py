@@ -265,12 +265,12 @@ def test_image_cache_in_process_and_on_disk(S):
         with pytest.raises(S.SlateError) as e:
             s.register_source(BCAST_SRC, "bcast", Args3D, threads=96)   # 32-byte struct vs the kernel's 24
         assert e.value.status == S.EINVAL
-    code = ("import sys; sys.path.insert(0, %r)\n"
-            "from tests.test_user_kernels import BCAST_SRC, ArgsBcast\n"
+    code = ("import sys; sys.path.insert(0, %r); sys.path.insert(0, %r)\n"
+            "from test_user_kernels import BCAST_SRC, ArgsBcast\n"
             "from paper_conf_ipps_allenf019_b200 import slate as S\n"
             "with S.Session(None, 0) as s:\n"
             "    s.register_source(BCAST_SRC.replace('64', '65'), 'bcast', ArgsBcast, threads=160)\n"
-            "print(*S.rtc_stats())\n") % ROOT
+            "print(*S.rtc_stats())\n") % (ROOT, os.path.join(ROOT, "tests"))
     with tempfile.TemporaryDirectory() as d:
         env = dict(os.environ, SLATE_RTC_CACHE=os.path.join(d, "rtc"))
         runs = [subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)

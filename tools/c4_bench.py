@@ -90,8 +90,9 @@ def client(endpoint, kind, steps, go_path, device=0):
     s.close()
 
 
-def sequential(endpoint, device=0):
-    """The four jobs back to back with the original kernels, one client (vanilla CUDA)."""
+def sequential(endpoint, device=0, slate=False):
+    """The four jobs back to back, one client: the original kernels (vanilla
+    CUDA), or with slate=True the workers on every SM (Slate-sequential)."""
     from paper_conf_ipps_allenf019_b200 import slate as S
     import torch
     torch.cuda.set_device(device)
@@ -106,7 +107,11 @@ def sequential(endpoint, device=0):
         ids = []
         per = {}
         for k, (_, args, grid, _) in built.items():
-            li = [s.launch(kids[k], args, grid, mode=S.MODE_STANDALONE) for _ in range(JOBS[k])]
+            if slate:
+                first = s.launch_n(kids[k], args, grid, JOBS[k], placement=S.PLACE_SOLO)
+                li = list(first) if isinstance(first, (list, tuple)) else list(range(first, first + JOBS[k]))
+            else:
+                li = [s.launch(kids[k], args, grid, mode=S.MODE_STANDALONE) for _ in range(JOBS[k])]
             ids += li
             per[k] = li
         s.sync(0)
@@ -153,7 +158,11 @@ def main():
             break
         except S.SlateError:
             time.sleep(0.2)
-    seq_ms, solo = sequential(ep, a.device)
+    seq_ms, solo_cuda = sequential(ep, a.device)
+    seq_slate_ms, solo_slate = sequential(ep, a.device, slate=True)
+    # every job's best solo time (original kernels or workers), the baseline of the gains
+    solo = {k: min(solo_cuda[k], solo_slate[k]) for k in JOBS}
+    best_seq = sum(solo.values())
     ps = {k: subprocess.Popen([sys.executable, __file__, "--steps", str(a.steps), "--device", str(a.device),
                                "--client", ep, k, go],
                               stdout=subprocess.PIPE, text=True) for k in JOBS}
@@ -198,8 +207,13 @@ def main():
                     json.dumps(res[k][step][4])))
     print(json.dumps({"config": "C4: triad 2^26, SpMV 2^20, stencil 8192^2, bf16 GEMM 4096^3 from 4 client processes "
                                 "via slated (AUTO)",
-                      "jobs": JOBS, "seq_cuda_ms": round(seq_ms, 3), "solo_ms": {k: round(v, 3) for k, v in solo.items()},
-                      "corun_makespan_ms": round(mk, 3), "gain_vs_sequential": round(seq_ms / mk, 4),
+                      "jobs": JOBS, "seq_cuda_ms": round(seq_ms, 3), "seq_slate_ms": round(seq_slate_ms, 3),
+                      "best_sequential_ms": round(best_seq, 3),
+                      "solo_ms": {k: round(v, 3) for k, v in solo.items()},
+                      "solo_cuda_ms": {k: round(v, 3) for k, v in solo_cuda.items()},
+                      "solo_slate_ms": {k: round(v, 3) for k, v in solo_slate.items()},
+                      "corun_makespan_ms": round(mk, 3), "gain_vs_sequential": round(best_seq / mk, 4),
+                      "gain_vs_seq_cuda": round(seq_ms / mk, 4),
                       "stp_median": round(sorted(stps)[len(stps) // 2], 4), "makespans_ms": [round(x, 3) for x in spans],
                       "resize_us": {"n": len(resize), "p50": round(sorted(resize)[len(resize) // 2], 2) if resize else None,
                                     "max": round(max(resize), 2) if resize else None}}))
