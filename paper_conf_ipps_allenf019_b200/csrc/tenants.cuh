@@ -221,76 +221,89 @@ struct SgemmNaive : TenantBase {
 };
 
 // ============================================================== CSR SpMV  y = A x
-// 32 rows per block; warp w handles rows 4w..4w+3 with 8 lanes per row: lane l
-// sums j = rp[row]+l, +8, +16, ... in ascending order (an fmaf chain from 0),
-// then a butterfly (xor 4, 2, 1) inside the 8-lane group.  The task body runs
-// the task's blocks (up to kMaxIters = kU) at once, each thread holding one row
-// per block, so the row-pointer, column/value and x loads of 4 rows are in
-// flight together (tools/probe/spmv_variants.cu: 1.7x the original kernel);
-// per row the arithmetic is exactly cta_block's.
-template <int kU, int kMB>
-struct SpmvCsrT : TenantBase {
-  using Args = slate_args_spmv;
-  static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = kMB;     // latency-bound: occupancy is throughput
-  static constexpr int kSmem = 0, kSmemStandalone = 0;
-  static constexpr bool kHasTask = true;
-  static constexpr uint32_t kMaxIters = kU;
-  static constexpr uint32_t kTasksPerWorker = 4;   // full kU-block tasks (the body holds kU rows per thread)
+// The row reduction order, shared by the original kernel below and the worker
+// (spmv_ws.cu), so their y are bit-identical: a row's nonzeros are taken in
+// aligned 16-byte segments -- entries 4s .. 4s+3 of the col / val arrays, those
+// outside the row's [rp[row], rp[row+1]) skipped -- and lane q of the row's
+// 4-lane group sums segments s0+q, s0+q+4, ... (s0 = rp[row] / 4) in ascending
+// order, each segment's entries ascending, as one fmaf chain from 0; the group
+// then adds with a xor 2, 1 butterfly.  One 128-bit load of columns and one of
+// values per lane and segment (coalesced: a warp reads 8 rows x 16 nonzeros as
+// 512 contiguous bytes of each array).  The oracle is order-free (fp64; exact
+// on integer inputs), so the order is this build's choice.
+namespace spmvseg {
+struct Seg {
+  int4 c;
+  float4 v;
+};
+// entries base .. base+3 (base a multiple of 4) that exist in the arrays (< nnz)
+__device__ __forceinline__ Seg load(const int* __restrict__ col, const float* __restrict__ val, int base, int nnz,
+                                    bool any) {
+  Seg s;
+  s.c = make_int4(0, 0, 0, 0);
+  s.v = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (!any) return s;
+  if (base + 4 <= nnz) {
+    s.c = __ldcs(reinterpret_cast<const int4*>(col + base));
+    s.v = __ldcs(reinterpret_cast<const float4*>(val + base));
+  } else {   // the array's last, partial segment
+    if (base + 0 < nnz) { s.c.x = __ldcs(col + base + 0); s.v.x = __ldcs(val + base + 0); }
+    if (base + 1 < nnz) { s.c.y = __ldcs(col + base + 1); s.v.y = __ldcs(val + base + 1); }
+    if (base + 2 < nnz) { s.c.z = __ldcs(col + base + 2); s.v.z = __ldcs(val + base + 2); }
+  }
+  return s;
+}
+// acc <- the segment's entries of the row [lo, hi), ascending
+template <class XF>
+__device__ __forceinline__ float fma_seg(float acc, const Seg& s, int base, int lo, int hi, XF xval) {
+  if (base + 0 >= lo && base + 0 < hi) acc = __fmaf_rn(s.v.x, xval(s.c.x), acc);
+  if (base + 1 >= lo && base + 1 < hi) acc = __fmaf_rn(s.v.y, xval(s.c.y), acc);
+  if (base + 2 >= lo && base + 2 < hi) acc = __fmaf_rn(s.v.z, xval(s.c.z), acc);
+  if (base + 3 >= lo && base + 3 < hi) acc = __fmaf_rn(s.v.w, xval(s.c.w), acc);
+  return acc;
+}
+// lane q's chain over segments s0+q+4m for m >= m0 (the row's remaining segments)
+template <class XF>
+__device__ __forceinline__ float row_tail(float acc, const int* col, const float* val, int nnz, int lo, int hi, int q,
+                                          int m0, XF xval) {
+  for (int base = ((lo >> 2) + q + 4 * m0) * 4; base < hi; base += 16)
+    acc = fma_seg(acc, load(col, val, base, nnz, true), base, lo, hi, xval);
+  return acc;
+}
+__device__ __forceinline__ float reduce4(float v) {
+  v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 2));
+  v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 1));
+  return v;
+}
+}  // namespace spmvseg
 
-  template <int U>
-  __device__ __forceinline__ static void rows(const Args& a, uint32_t x0, uint32_t nblk) {
+// The original kernel K(B,T): 32 rows per block, 4 lanes per row (T = 128), x
+// from global memory.  Its slate worker is the warp-specialised one in
+// spmv_ws.cu (same per-row arithmetic).
+struct SpmvSeg : TenantBase {
+  using Args = slate_args_spmv;
+  static constexpr int kThreads = 128;
+  static constexpr int kMinBlocks = 16;
+  static constexpr int kSmem = 0, kSmemStandalone = 0;
+
+  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
     const int* __restrict__ rp = reinterpret_cast<const int*>(a.rowptr);
     const int* __restrict__ col = reinterpret_cast<const int*>(a.col);
     const float* __restrict__ val = reinterpret_cast<const float*>(a.val);
     const float* __restrict__ xv = reinterpret_cast<const float*>(a.x);
-    const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int l = int(lane & 7);
-    int lo[U], hi[U], c0[U], c1[U];
-    float v0[U], v1[U], acc[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const uint32_t row = (x0 + u) * 32 + w * 4 + (lane >> 3);
-      lo[u] = 0; hi[u] = 0; acc[u] = 0.f;
-      if (uint32_t(u) < nblk && row < a.n_rows) { lo[u] = __ldg(rp + row) + l; hi[u] = __ldg(rp + row + 1); }
+    const uint32_t row = x * 32 + (threadIdx.x >> 2);
+    const int q = int(threadIdx.x & 3);
+    const int nnz = __ldg(rp + a.n_rows);
+    int lo = 0, hi = 0;
+    if (row < a.n_rows) {
+      lo = __ldg(rp + row);
+      hi = __ldg(rp + row + 1);
     }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {        // first round: j = lo and lo + 8 (rows of <= 16 nonzeros end here)
-      c0[u] = lo[u] < hi[u] ? __ldcs(col + lo[u]) : 0;
-      v0[u] = lo[u] < hi[u] ? __ldcs(val + lo[u]) : 0.f;
-      c1[u] = lo[u] + 8 < hi[u] ? __ldcs(col + lo[u] + 8) : 0;
-      v1[u] = lo[u] + 8 < hi[u] ? __ldcs(val + lo[u] + 8) : 0.f;
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (lo[u] < hi[u]) acc[u] = __fmaf_rn(v0[u], __ldg(xv + c0[u]), acc[u]);
-      if (lo[u] + 8 < hi[u]) acc[u] = __fmaf_rn(v1[u], __ldg(xv + c1[u]), acc[u]);
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {        // longer rows: the rest of the chain, still ascending
-      for (int j = lo[u] + 16; j < hi[u]; j += 8) acc[u] = __fmaf_rn(__ldcs(val + j), __ldg(xv + __ldcs(col + j)), acc[u]);
-      float v = acc[u];
-      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 4));
-      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 2));
-      v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, 1));
-      const uint32_t row = (x0 + u) * 32 + w * 4 + (lane >> 3);
-      if (l == 0 && uint32_t(u) < nblk && row < a.n_rows) __stcs(reinterpret_cast<float*>(a.y) + row, v);
-    }
-  }
-  __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char*) {
-    rows<1>(a, x, 1);
-  }
-  __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char*) {
-    uint32_t i = 0;
-    for (; i + kU <= n; i += kU) rows<kU>(a, g + i, kU);
-    if (i < n) rows<kU>(a, g + i, n - i);
+    const float acc = spmvseg::row_tail(0.f, col, val, nnz, lo, hi, q, 0, [&](int c) { return __ldg(xv + c); });
+    const float v = spmvseg::reduce4(acc);
+    if (q == 0 && row < a.n_rows) __stcs(reinterpret_cast<float*>(a.y) + row, v);
   }
 };
-// the register body: 8 blocks' rows in flight per thread, 4 CTAs/SM
-// (tools/probe/worker_overhead.cu: fastest of U in {1..8} x occupancy {4, 6, 8}).
-// It is the original kernel K(B,T) of the SpMV kind; the slate worker of the
-// kind is the warp-specialised one in spmv_ws.cu (same per-row arithmetic).
-using SpmvCsrReg = SpmvCsrT<8, 4>;
 
 // ============================================================== Black-Scholes
 // European call/put as in the CUDA SDK BlackScholes sample: the normal CDF by
