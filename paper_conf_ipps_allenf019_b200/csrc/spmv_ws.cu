@@ -4,35 +4,36 @@
 // What it computes is the original kernel's (tenants.cuh SpmvSeg): a row's
 // nonzeros in aligned 16-byte segments, lane q of the row's 4-lane group
 // summing segments s0+q, s0+q+4, ... ascending as one fmaf chain, then a xor
-// 2, 1 butterfly.  Only where x comes from differs (a shared-memory window
+// 2, 1 butterfly.  Only where the operands come from differs (shared memory
 // here, global memory there), so y is bit-identical to the original kernel's
 // (tests/test_gpu_parity.py).
 //
-// Why a separate worker.  Per SM the kernel must move ~136 bytes per row
-// (16 nonzeros: 64 B of columns, 64 B of values, rp, y) while gathering 16
-// random x values per row.  Gathered from global memory, x costs one L1 tag
-// per lane (~1 nonzero per SM clock, the original kernel's bound); gathered
-// from a shared-memory window it costs a few bank wavefronts per warp load.
-// The columns and values stream through registers by 128-bit loads (one L1
-// wavefront per 128 B, no shared-memory round trip), software-pipelined: a
-// compute warp has the next group's loads in flight while it computes the
-// current group, so each SM keeps ~64 KB in flight -- what HBM needs to run
-// near its peak from half the chip (the co-run split).
-//
-// One CTA per SM, two roles:
+// Why a separate worker: the original kernel is bound by the L1 gather of x
+// (one 128-B line per lane per instruction: ~1 nonzero per SM clock) and, at
+// the co-run's SM share, by the bytes each SM can keep in flight (a register
+// pipeline holds ~45 KB per SM; at HBM's loaded latency that is ~25 GB/s per
+// SM -- measured, round 2).  Here one CTA per SM runs three roles (the
+// structure of the GEMM tenant: the slate protocol lives in a producer warp):
 //   * task warp (warp 16) -- the slate worker proper: Lst1 binding and standby
 //     (prologue), at every task boundary the resize word (retire, Lst1 P:L185)
 //     and the task counter (Lst2 (2) P:L208), taken one task ahead
-//     (speculative boundary); then the task's row-pointer slice into one of
-//     four slice buffers and the task's x window -- [first column of its first
-//     row, last column of its last row] widened to the buffer (a banded or
+//     (speculative boundary); then the task's row-pointer slice, loaded by the
+//     whole warp into one of four slice buffers, and the bounds of its x window,
+//     read off the task's nonzeros: [first column of its first row, last column
+//     of its last row] widened to the buffer's capacity (a banded or
 //     near-diagonal matrix then finds every column in it; a column outside is
-//     read from global memory, so the window decides speed, never the result)
-//     -- by one bulk copy (L2 -> shared, cp.async.bulk) into one of three windows;
-//   * compute warps 0..14 -- the 128 passes of 8 rows of a task (4 lanes per
-//     row) dealt round-robin, 9 per warp in three groups of three: the columns
-//     and values of the next group (this task's, or the next task's first) are
-//     loaded while the current group is computed.
+//     read from global memory, so the window decides speed, never the result);
+//   * chunk warp (warp 17, lane 0) -- per task the x window (cp.async.bulk,
+//     L2 -> shared, two buffers), then the task's nonzeros as chunks of 256 rows
+//     (8 original blocks) through a 4-slot ring: columns and values of
+//     [rp[r0], rp[r0+256]) by cp.async.bulk (HBM -> shared, evict-first), up to
+//     128 KB in flight per SM;
+//   * compute warps 0..15 -- per chunk, two passes of 8 rows, 4 lanes per row:
+//     one 128-bit shared load of columns and one of values per lane and
+//     segment, x from the window.
+// The task warp runs up to three tasks ahead of the compute warps and the chunk
+// warp keeps up to four chunks in flight, so HBM sees a stream instead of one
+// round-trip chain per task.
 //
 // Resize: the task boundary is where the task warp re-reads the
 // resize word; a CTA that left the range stops fetching, its compute warps
@@ -47,36 +48,53 @@
 namespace slate {
 namespace spmv {
 
-constexpr int kComputeWarps = 15;                  // + the task warp = 16 warps: 128 registers per thread
-constexpr int kThreads = 32 * kComputeWarps + 32;
-constexpr int kTaskWarp = kComputeWarps;
-constexpr int kMaxTaskBlocks = 32;                 // task-size cap (1024 rows)
-constexpr int kTaskRows = 32 * kMaxTaskBlocks;
-constexpr int kPassRows = 8;                       // rows per warp pass (4 lanes per row)
-constexpr int kTaskPasses = kTaskRows / kPassRows; // 128 passes per task, dealt round-robin to the warps
-constexpr int kU = 3;                              // passes per group (loads in flight together)
-constexpr int kGroups = (kTaskPasses + kComputeWarps * kU - 1) / (kComputeWarps * kU);   // 3 groups per warp
-constexpr int kRpBufs = 4;                         // row-pointer slices: the task warp runs <= 3 tasks ahead
-constexpr int kRpInts = kTaskRows + 4;             // rp slice of one task (rounded to 16 B)
-constexpr int kWinBufs = 3;                        // the task warp issues windows up to two tasks ahead
-constexpr int kWin = 10240;                        // x window per task (floats): 1024 rows of a +-4096 band
-constexpr int kHdrBytes = 512;
-constexpr int kSmemBytes = kHdrBytes + kRpBufs * kRpInts * 4 + kWinBufs * kWin * 4;
+#ifndef SLATE_SPMV_WARPS
+#define SLATE_SPMV_WARPS 16
+#endif
+constexpr int kComputeWarps = SLATE_SPMV_WARPS;
+constexpr int kCompute = 32 * kComputeWarps;
+constexpr int kThreads = kCompute + 64;          // + task warp + chunk warp
+constexpr int kTaskWarp = kComputeWarps, kChunkWarp = kComputeWarps + 1;
+constexpr int kChunkBlocks = 8;                  // blocks per chunk (256 rows)
+constexpr int kChunkRows = 32 * kChunkBlocks;
+constexpr int kPassRows = 8;                     // rows per warp pass (4 lanes per row)
+constexpr int kPasses = kChunkRows / (kPassRows * kComputeWarps);
+static_assert(kPasses * kPassRows * kComputeWarps == kChunkRows, "rows per chunk");
+constexpr int kMaxTaskBlocks = 32;               // task-size cap (1024 rows)
+constexpr int kSlots = 4;                        // chunk ring depth
+constexpr int kCap = kChunkRows * 16 + 8;        // nonzeros per slot (16 per row + alignment)
+constexpr int kSlotBytes = 2 * kCap * 4;         // col + val
+constexpr int kRpBufs = 4;                       // row-pointer slices: the task warp runs <= 3 tasks ahead
+constexpr int kRpInts = 32 * kMaxTaskBlocks + 4; // rp slice of one task (rounded to 16 B)
+constexpr int kWinBufs = 2;
+constexpr int kWin = 10240;                      // x window per task (floats)
+constexpr int kHdrBytes = 1024;
+constexpr int kSmemBytes = kHdrBytes + kSlots * kSlotBytes + kRpBufs * kRpInts * 4 + kWinBufs * kWin * 4;
 static_assert(kSmemBytes <= 227 * 1024, "one CTA per SM");
-static_assert((kRpInts * 4) % 16 == 0 && (kWin * 4) % 16 == 0, "16-B bulk granules");
+static_assert(kSlotBytes % 16 == 0 && (kRpInts * 4) % 16 == 0 && (kWin * 4) % 16 == 0, "16-B bulk granules");
 
 struct TaskMeta {                 // written by the task warp before its rp arrive
   uint32_t g, n;                  // original blocks [g, g+n); n = 0: stop (sentinel)
   int32_t wlo;                    // x window: columns [wlo, wlo + wlen)
   uint32_t wlen;
 };
+struct ChunkMeta {                // written by the chunk warp before its slot arrive
+  uint32_t tb;                    // rp buffer of the chunk's task; 0xffffffff: stop (sentinel)
+  uint32_t wb;                    // x-window buffer of the chunk's task
+  uint32_t row0;                  // first row of the chunk within the task
+  uint32_t nblk;                  // blocks in the chunk
+  int32_t a0;                     // nonzero index of col_s[0] (16-B aligned)
+  uint32_t mode;                  // 0 staged, 1 col/val from global memory (the chunk exceeds the slot)
+  uint32_t first, last;           // first / last chunk of its task
+};
 struct Hdr {
-  uint64_t rp_full[kRpBufs], rp_empty[kRpBufs], rp_tx[kRpBufs];
+  uint64_t slot_full[kSlots], slot_empty[kSlots];
+  uint64_t rp_full[kRpBufs], rp_empty[kRpBufs];
   uint64_t win_full[kWinBufs], win_empty[kWinBufs];
   TaskMeta tmeta[kRpBufs];
+  ChunkMeta cmeta[kSlots];
   uint32_t go, rank, retired;
-  int32_t nnz;
-  uint32_t blocks, tasks;         // counted by compute warp 0 (it runs a part of every task the CTA took)
+  int32_t nnz;                    // rp[n_rows]
   uint64_t ctrl;                  // the resize word last acted on (task warp)
 };
 static_assert(sizeof(Hdr) <= kHdrBytes, "header");
@@ -92,82 +110,110 @@ __device__ __forceinline__ void bulk_g2s_keep(void* dst, const void* src, uint32
                : "memory");
 }
 
+#ifdef SLATE_SPMV_TRACE
+// development trace (tools/probe/spmv_stream.cu): per CTA < 4 and role, 64 events {t, kind, a, b}
+__device__ unsigned long long spmv_trace[4][3][64][4];
+__device__ __forceinline__ void trace(int role, uint32_t& n, uint32_t kind, uint32_t a0, uint32_t b0) {
+  if (blockIdx.x < 4 && n < 64) {
+    unsigned long long* r = spmv_trace[blockIdx.x][role][n++];
+    r[0] = globaltimer(); r[1] = kind; r[2] = a0; r[3] = b0;
+  }
+}
+#define TRACE(role, kind, a0, b0) trace(role, tn, kind, a0, b0)
+#define TRACE_DECL uint32_t tn = 0
+#else
+#define TRACE(role, kind, a0, b0)
+#define TRACE_DECL
+#endif
+
+#ifdef SLATE_SPMV_PROFILE
+__device__ long long spmv_prof[148][32][5];   // per CTA, compute warp: {total, wait full, first-chunk waits, compute, chunks}
+#endif
+
 struct Smem {
   Hdr* h;
+  char* slots;
   char* rpb;
   char* win;
+  __device__ __forceinline__ int32_t* col(int s) const { return reinterpret_cast<int32_t*>(slots + s * kSlotBytes); }
+  __device__ __forceinline__ float* val(int s) const {
+    return reinterpret_cast<float*>(slots + s * kSlotBytes + kCap * 4);
+  }
   __device__ __forceinline__ int32_t* rp(int b) const { return reinterpret_cast<int32_t*>(rpb + b * kRpInts * 4); }
   __device__ __forceinline__ float* xw(int b) const { return reinterpret_cast<float*>(win + b * kWin * 4); }
 };
 
-// one group of kU passes of a compute warp: per lane, its row's first segment
-// (loads in flight until compute_group reads them; the row bounds are re-read
-// from the task's rp slice then, to keep two groups within the register budget)
-struct Group {
-  spmvseg::Seg s[kU];
-};
-__device__ __forceinline__ void row_bounds(const int32_t* rps, uint32_t nrows, uint32_t lr, int& lo, int& hi) {
-  const bool in = lr < nrows;
-  lo = in ? rps[lr] : 0;
-  hi = in ? rps[lr + 1] : 0;
-}
-
-// the row (within its task) of lane `lane` in pass u of group `grp` of warp w
-__device__ __forceinline__ uint32_t task_row(uint32_t w, uint32_t lane, int grp, int u) {
-  return (w + kComputeWarps * uint32_t(grp * kU + u)) * kPassRows + (lane >> 2);
-}
-
-// issue the loads of group `grp` of task `tm` (its rp slice `rps`)
-__device__ __forceinline__ void load_group(Group& G, const slate_args_spmv& a, const int32_t* rps,
-                                           const TaskMeta& tm, uint32_t w, uint32_t lane, int grp, int nnz) {
-  const int* __restrict__ col = reinterpret_cast<const int*>(a.col);
-  const float* __restrict__ val = reinterpret_cast<const float*>(a.val);
-  const uint32_t nrows = min(tm.n * 32u, a.n_rows - tm.g * 32u);
-  const int q = int(lane & 3);
-#pragma unroll
-  for (int u = 0; u < kU; ++u) {
-    const uint32_t lr = task_row(w, lane, grp, u);
-    int lo, hi;
-    row_bounds(rps, nrows, lr, lo, hi);
-    const int base = ((lo >> 2) + q) * 4;
-    G.s[u] = spmvseg::load(col, val, base, nnz, base < hi);
-  }
-}
-
-// compute group `grp` of task `tm` with x from window `xw` (columns [wlo, wlo + wlen))
-__device__ __forceinline__ void compute_group(const Group& G, const slate_args_spmv& a, const int32_t* rps,
-                                              const float* xw, const TaskMeta& tm, uint32_t w, uint32_t lane, int grp,
-                                              int nnz) {
-  const int* __restrict__ col = reinterpret_cast<const int*>(a.col);
-  const float* __restrict__ val = reinterpret_cast<const float*>(a.val);
+// ------------------------------------------------------------------ compute warps
+// Rows of one chunk: kPasses passes of 8 rows per compute warp, 4 lanes per
+// row; every pass's shared-memory loads are issued before the first FMA.  x
+// comes from the task's window, or global memory for a column outside it.
+__device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Smem& S, const ChunkMeta& m,
+                                              const TaskMeta& tm, int s, int nnz) {
   const float* __restrict__ xg = reinterpret_cast<const float*>(a.x);
+  const int32_t* rp = S.rp(int(m.tb)) + m.row0;          // rp of the chunk's first row
+  const float* xw = S.xw(int(m.wb));
   const int32_t wlo = tm.wlo;
   const uint32_t wlen = tm.wlen;
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int q = int(lane & 3);
+  const uint32_t row_first = tm.g * 32 + m.row0;        // global row of rp[0]
+  const uint32_t nrows = min(m.nblk * 32, a.n_rows - row_first);
   auto xval = [&](int c) -> float {
     const uint32_t d = uint32_t(c - wlo);
     return d < wlen ? xw[d] : __ldg(xg + c);
   };
-  const uint32_t nrows = min(tm.n * 32u, a.n_rows - tm.g * 32u);
-  const int q = int(lane & 3);
-  float acc[kU];
-  int lo[kU], hi[kU];
+  constexpr int U = kPasses;
+  int lo[U], hi[U];
+  float acc[U];
   bool longrow = false;
 #pragma unroll
-  for (int u = 0; u < kU; ++u) {
-    row_bounds(rps, nrows, task_row(w, lane, grp, u), lo[u], hi[u]);
-    const int base = ((lo[u] >> 2) + q) * 4;
-    acc[u] = spmvseg::fma_seg(0.f, G.s[u], base, lo[u], hi[u], xval);
-    longrow |= ((lo[u] >> 2) + 4) * 4 < hi[u];   // the row has segments past its first four
+  for (int u = 0; u < U; ++u) {
+    const uint32_t lr = (u * kComputeWarps + w) * kPassRows + (lane >> 2);
+    const bool in = lr < nrows;
+    lo[u] = in ? rp[lr] : 0;
+    hi[u] = in ? rp[lr + 1] : 0;
+    longrow |= ((lo[u] >> 2) + 4) * 4 < hi[u];   // segments past the lane's first
   }
-  if (__any_sync(0xffffffffu, longrow)) {
+  if (m.mode == 0) {
+    const int32_t* col = S.col(s);
+    const float* val = S.val(s);
+    const int32_t a0 = m.a0;   // the slot holds entries [a0, ...), a0 a multiple of 4
+    auto seg = [&](int base) {
+      spmvseg::Seg r;
+      r.c = *reinterpret_cast<const int4*>(col + (base - a0));
+      r.v = *reinterpret_cast<const float4*>(val + (base - a0));
+      return r;
+    };
+    spmvseg::Seg sg[U];
 #pragma unroll
-    for (int u = 0; u < kU; ++u) acc[u] = spmvseg::row_tail(acc[u], col, val, nnz, lo[u], hi[u], q, 1, xval);
+    for (int u = 0; u < U; ++u) {   // a lane with no entry of its row reads nothing (its offset may be negative)
+      const int base = ((lo[u] >> 2) + q) * 4;
+      if (base < hi[u]) sg[u] = seg(base);
+      else sg[u] = spmvseg::Seg{make_int4(0, 0, 0, 0), make_float4(0.f, 0.f, 0.f, 0.f)};
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int base = ((lo[u] >> 2) + q) * 4;
+      acc[u] = spmvseg::fma_seg(0.f, sg[u], base, lo[u], hi[u], xval);
+    }
+    if (__any_sync(0xffffffffu, longrow)) {
+#pragma unroll
+      for (int u = 0; u < U; ++u)   // rows longer than 16: the rest of the chain, still ascending
+        for (int base = ((lo[u] >> 2) + q + 4) * 4; base < hi[u]; base += 16)
+          acc[u] = spmvseg::fma_seg(acc[u], seg(base), base, lo[u], hi[u], xval);
+    }
+  } else {
+    // the chunk's nonzeros did not fit the slot: the same chain from global memory
+    const int* col = reinterpret_cast<const int*>(a.col);
+    const float* val = reinterpret_cast<const float*>(a.val);
+#pragma unroll
+    for (int u = 0; u < U; ++u) acc[u] = spmvseg::row_tail(0.f, col, val, nnz, lo[u], hi[u], q, 0, xval);
   }
 #pragma unroll
-  for (int u = 0; u < kU; ++u) {
+  for (int u = 0; u < U; ++u) {
     const float v = spmvseg::reduce4(acc[u]);
-    const uint32_t lr = task_row(w, lane, grp, u);
-    if (q == 0 && lr < nrows) __stcs(reinterpret_cast<float*>(a.y) + tm.g * 32u + lr, v);
+    const uint32_t lr = (u * kComputeWarps + w) * kPassRows + (lane >> 2);
+    if (q == 0 && lr < nrows) __stcs(reinterpret_cast<float*>(a.y) + row_first + lr, v);
   }
 }
 
@@ -176,20 +222,24 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   extern __shared__ __align__(128) char smem_raw[];
   Smem S;
   S.h = reinterpret_cast<Hdr*>(smem_raw);
-  S.rpb = smem_raw + kHdrBytes;
+  S.slots = smem_raw + kHdrBytes;
+  S.rpb = S.slots + kSlots * kSlotBytes;
   S.win = S.rpb + kRpBufs * kRpInts * 4;
   Hdr& H = *S.h;
   const slate_args_spmv& a = p.args;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
   if (threadIdx.x == kTaskWarp * 32) {
+    for (int i = 0; i < kSlots; ++i) {
+      mbar_init(&H.slot_full[i], 1);              // the chunk warp's expect_tx arrive (+ bytes)
+      mbar_init(&H.slot_empty[i], kComputeWarps); // every compute warp
+    }
     for (int i = 0; i < kRpBufs; ++i) {
       mbar_init(&H.rp_full[i], 32);               // every lane of the task warp (plain loads + stores)
-      mbar_init(&H.rp_empty[i], kComputeWarps);   // every compute warp, after the task
-      mbar_init(&H.rp_tx[i], 1);                  // the task warp's expect_tx arrive (+ the slice's bytes)
+      mbar_init(&H.rp_empty[i], kComputeWarps);   // every compute warp, after the task's last chunk
     }
     for (int i = 0; i < kWinBufs; ++i) {
-      mbar_init(&H.win_full[i], 1);               // the task warp's expect_tx arrive (+ x bytes)
+      mbar_init(&H.win_full[i], 1);               // the chunk warp's expect_tx arrive (+ x bytes)
       mbar_init(&H.win_empty[i], kComputeWarps);
     }
     fence_mbar_init();
@@ -198,8 +248,6 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     uint64_t c = 0;
     H.rank = r;
     H.retired = 0;
-    H.blocks = 0;
-    H.tasks = 0;
     H.nnz = __ldg(reinterpret_cast<const int*>(a.rowptr) + a.n_rows);
     H.go = prologue(p, r, c) ? 1u : 0u;
     H.ctrl = c;
@@ -213,10 +261,11 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   const int nnz = H.nnz;
 
   if (warp == kTaskWarp) {
-    // ===================== task warp: the slate task protocol, rp slices, x windows =====================
+    // ===================== task warp: the slate task protocol + row-pointer slices =====================
     uint64_t c = H.ctrl;
     const uint32_t rank = H.rank;
     __syncwarp();   // every lane has read H.ctrl before lane 0 may rewrite it (the stop sentinel)
+    TRACE_DECL;
     // Speculative boundary (as the generic worker's kSpeculative mode): the
     // decision for task t+1 -- retire, or the counter atomic -- is taken when
     // task t's slice is fetched, from the resize word loaded one boundary
@@ -236,14 +285,16 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       c_pre = ld_acquire_u64(p.ctrl);
     }
     for (uint32_t t = 0;; ++t) {
-      const int b = int(t % kRpBufs), wb = int(t % kWinBufs);
+      const int b = int(t % kRpBufs);
       uint32_t g = 0xffffffffu, chg = 0;
       if (lane == 0) {
+        TRACE(0, 0, t, 0);
         // resolve the fetch taken at the previous boundary
         if (next_ret) {
           H.retired = 1;
         } else if (g_next < p.B) {
           g = g_next;
+          TRACE(0, 2, t, g);
           if (g == 0) p.tc->t_first = globaltimer();
         } else {
           atomicAdd(&p.tc->live_pending, ~0ull);                        // drained: live -= 1
@@ -263,6 +314,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           c_pre = ld_acquire_u64(p.ctrl);
         }
         mbar_wait(&H.rp_empty[b], ((t / kRpBufs) & 1) ^ 1);         // task t-4 fully consumed
+        TRACE(0, 1, t, 0);
       }
       g = __shfl_sync(0xffffffffu, g, 0);
       chg = __shfl_sync(0xffffffffu, chg, 0);
@@ -277,19 +329,21 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
         mbar_arrive(&H.rp_full[b]);                   // sentinel: publishes the stop
         break;
       }
-      // rp[r0 .. r1]: whole 16-B granules by one bulk copy (r0 = 32 g is 128-B
-      // aligned; no registers hold the slice), the last 1-3 entries by lanes
+      // rp[r0 .. r1] by the whole warp: 16-B loads (r0 = 32 g is 128-B aligned), then the tail
       const uint32_t n = min(p.iters, p.B - g);
       const uint32_t r0 = g * 32, r1 = min(r0 + n * 32, a.n_rows);
       const uint32_t cnt = r1 - r0 + 1, n4 = cnt / 4;
       const int32_t* rpg = reinterpret_cast<const int32_t*>(a.rowptr) + r0;
       int32_t* rps = S.rp(b);
-      if (lane == 0) {
-        mbar_expect_tx(&H.rp_tx[b], n4 * 16);
-        bulk_g2s_keep(rps, rpg, n4 * 16, &H.rp_tx[b]);
-      }
+      constexpr int kV = (kRpInts / 4 + 31) / 32;
+      int4 v[kV];
+#pragma unroll
+      for (int k = 0; k < kV; ++k)
+        if (lane + 32 * k < n4) v[k] = __ldg(reinterpret_cast<const int4*>(rpg) + lane + 32 * k);
+#pragma unroll
+      for (int k = 0; k < kV; ++k)
+        if (lane + 32 * k < n4) reinterpret_cast<int4*>(rps)[lane + 32 * k] = v[k];
       if (lane < cnt - n4 * 4) rps[n4 * 4 + lane] = __ldg(rpg + n4 * 4 + lane);
-      if (lane == 0) mbar_wait(&H.rp_tx[b], (t / kRpBufs) & 1);
       __syncwarp();
       if (lane == 0) {
         // the x window from the task's first and last nonzero
@@ -309,69 +363,134 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           wlen = uint32_t(max(0, min(kWin, ncols - lo)) & ~3);
         }
         tm.g = g; tm.n = n; tm.wlo = wlo; tm.wlen = wlen;
-        mbar_wait(&H.win_empty[wb], ((t / kWinBufs) & 1) ^ 1);     // task t-3 is done with the window
-        mbar_expect_tx(&H.win_full[wb], wlen * 4);
-        if (wlen) bulk_g2s_keep(S.xw(wb), reinterpret_cast<const float*>(a.x) + wlo, wlen * 4, &H.win_full[wb]);
+        TRACE(0, 3, t, wlen);
       }
-      __syncwarp();
       mbar_arrive(&H.rp_full[b]);                     // each lane after its stores (count 32)
     }
-  } else {
-    // ===================== compute warps: loads of the next group in flight during this one =====================
-    // the groups of every task in order -- (t, 0), (t, 1), .., (t + 1, 0), ... --
-    // with two register sets alternating statically (the loop body is two steps)
-    uint32_t my_blocks = 0, my_tasks = 0;
-    struct Item {
-      uint32_t t;
-      int grp;
-      TaskMeta tm;
-    };
-    // the item after `it` (a new task's first group waits for its slice; n = 0: the stop)
-    auto advance = [&](const Item& it) -> Item {
-      if (it.grp + 1 < kGroups) return Item{it.t, it.grp + 1, it.tm};
-      const uint32_t t1 = it.t + 1;
-      mbar_wait(&H.rp_full[t1 % kRpBufs], (t1 / kRpBufs) & 1);
-      return Item{t1, 0, H.tmeta[t1 % kRpBufs]};
-    };
-    auto finish = [&](const Item& it, const Group& G) {
-      const int b = int(it.t % kRpBufs), wb = int(it.t % kWinBufs);
-      if (it.grp == 0) mbar_wait(&H.win_full[wb], (it.t / kWinBufs) & 1);
-      compute_group(G, a, S.rp(b), S.xw(wb), it.tm, warp, lane, it.grp, nnz);
-      if (it.grp + 1 == kGroups) {   // the task's last group: its slice and window are free
-        __syncwarp();
-        if (lane == 0) {
-          mbar_arrive(&H.rp_empty[b]);
-          mbar_arrive(&H.win_empty[wb]);
-          if (warp == 0 && p.cov)
-            for (uint32_t i = 0; i < it.tm.n; ++i) atomicAdd(&p.cov[it.tm.g + i], 1u);
+  } else if (warp == kChunkWarp) {
+    // ===================== chunk warp: nonzeros of each task through the slot ring =====================
+    if (lane == 0) {
+      TRACE_DECL;
+      uint32_t q = 0;   // chunks issued
+      for (uint32_t t = 0;; ++t) {
+        const int b = int(t % kRpBufs), wb = int(t % kWinBufs);
+        mbar_wait(&H.rp_full[b], (t / kRpBufs) & 1);
+        TRACE(1, 10, t, 0);
+        const TaskMeta tm = H.tmeta[b];
+        if (tm.n) {                                   // the task's x window (task t-2 is done with the buffer)
+          mbar_wait(&H.win_empty[wb], ((t / kWinBufs) & 1) ^ 1);
+          mbar_expect_tx(&H.win_full[wb], tm.wlen * 4);
+          if (tm.wlen)
+            bulk_g2s_keep(S.xw(wb), reinterpret_cast<const float*>(a.x) + tm.wlo, tm.wlen * 4, &H.win_full[wb]);
         }
-        my_blocks += it.tm.n;
-        my_tasks += 1;
+        const uint32_t nch = tm.n ? (tm.n + kChunkBlocks - 1) / kChunkBlocks : 1;
+        for (uint32_t k = 0; k < nch; ++k, ++q) {
+          const int s = int(q % kSlots);
+          mbar_wait(&H.slot_empty[s], ((q / kSlots) & 1) ^ 1);
+          TRACE(1, 11, q, 0);
+          ChunkMeta& m = H.cmeta[s];
+          if (tm.n == 0) {
+            m.tb = 0xffffffffu;
+            mbar_expect_tx(&H.slot_full[s], 0);
+            break;
+          }
+          const uint32_t row0 = k * kChunkRows;
+          const uint32_t nblk = min(uint32_t(kChunkBlocks), tm.n - k * kChunkBlocks);
+          const uint32_t r0 = tm.g * 32 + row0;
+          const uint32_t nrows = min(nblk * 32, a.n_rows - r0);
+          const int32_t* rp = S.rp(b) + row0;
+          const int32_t e0 = rp[0], e1 = rp[nrows];
+          // [a0, a1) in whole 16-B granules; at the end of the matrix the
+          // granule past nnz may lie outside the arrays: its entries are loaded
+          // by this thread instead
+          const bool end = r0 + nrows == a.n_rows;
+          const int32_t a0 = e0 & ~3, a1 = end ? (e1 & ~3) : ((e1 + 3) & ~3);
+          m.tb = uint32_t(b); m.wb = uint32_t(wb); m.row0 = row0; m.nblk = nblk; m.a0 = a0;
+          m.first = k == 0; m.last = k + 1 == nch;
+          if (max(a1, e1) - a0 > kCap) {
+            m.mode = 1;
+            mbar_expect_tx(&H.slot_full[s], 0);
+          } else {
+            m.mode = 0;
+            for (int32_t j = max(a1, a0); j < e1; ++j) {
+              S.col(s)[j - a0] = __ldg(reinterpret_cast<const int32_t*>(a.col) + j);
+              S.val(s)[j - a0] = __ldg(reinterpret_cast<const float*>(a.val) + j);
+            }
+            const uint32_t bytes = uint32_t(max(a1 - a0, 0)) * 4;
+            mbar_expect_tx(&H.slot_full[s], 2 * bytes);
+            if (bytes) {
+              bulk_g2s(S.col(s), reinterpret_cast<const int32_t*>(a.col) + a0, bytes, &H.slot_full[s]);
+              bulk_g2s(S.val(s), reinterpret_cast<const float*>(a.val) + a0, bytes, &H.slot_full[s]);
+            }
+          }
+        }
+        if (tm.n == 0) break;
       }
-    };
-    mbar_wait(&H.rp_full[0], 0);
-    Item cur{0, 0, H.tmeta[0]};
-    Group G0, G1;
-    if (cur.tm.n) load_group(G0, a, S.rp(0), cur.tm, warp, lane, 0, nnz);
-    while (cur.tm.n) {
-      Item nx = advance(cur);
-      if (nx.tm.n) load_group(G1, a, S.rp(nx.t % kRpBufs), nx.tm, warp, lane, nx.grp, nnz);
-      finish(cur, G0);
-      cur = nx;
-      if (!cur.tm.n) break;
-      nx = advance(cur);
-      if (nx.tm.n) load_group(G0, a, S.rp(nx.t % kRpBufs), nx.tm, warp, lane, nx.grp, nnz);
-      finish(cur, G1);
-      cur = nx;
     }
-    if (warp == 0 && lane == 0) {
-      H.blocks = my_blocks;
-      H.tasks = my_tasks;
+  } else {
+    // ===================== compute warps =====================
+    uint32_t q = 0, t = 0, my_blocks = 0, my_tasks = 0;
+    TRACE_DECL;
+#ifdef SLATE_SPMV_PROFILE
+    long long pf_wait = 0, pf_first = 0, pf_comp = 0, pf_t0 = clock64();
+#endif
+    for (;; ++q) {
+      const int s = int(q % kSlots);
+#ifdef SLATE_SPMV_PROFILE
+      long long c0 = clock64();
+#endif
+      mbar_wait(&H.slot_full[s], (q / kSlots) & 1);
+#ifdef SLATE_SPMV_PROFILE
+      long long c1 = clock64();
+      pf_wait += c1 - c0;
+#endif
+      if (threadIdx.x == 0) TRACE(2, 20, q, 0);
+      const ChunkMeta m = H.cmeta[s];
+      if (m.tb == 0xffffffffu) break;
+      const int b = int(m.tb);
+      if (m.first) {
+        mbar_wait(&H.rp_full[b], (t / kRpBufs) & 1);
+        mbar_wait(&H.win_full[m.wb], (t / kWinBufs) & 1);
+      }
+      const TaskMeta tm = H.tmeta[b];
+      if (threadIdx.x == 0) TRACE(2, 21, q, 0);
+#ifdef SLATE_SPMV_PROFILE
+      long long c2 = clock64();
+      pf_first += c2 - c1;
+#endif
+      compute_chunk(a, S, m, tm, s, nnz);
+      __syncwarp();
+#ifdef SLATE_SPMV_PROFILE
+      pf_comp += clock64() - c2;
+#endif
+      if (threadIdx.x == 0) TRACE(2, 22, q, 0);
+      if (lane == 0) {
+        mbar_arrive(&H.slot_empty[s]);
+        if (m.last) {
+          mbar_arrive(&H.rp_empty[b]);
+          mbar_arrive(&H.win_empty[m.wb]);
+        }
+      }
+      if (threadIdx.x == 0) {
+        my_blocks += m.nblk;
+        if (p.cov)
+          for (uint32_t i = 0; i < m.nblk; ++i) atomicAdd(&p.cov[tm.g + m.row0 / 32 + i], 1u);
+      }
+      if (m.last) {
+        ++t;
+        ++my_tasks;
+      }
     }
+    if (threadIdx.x == 0 && my_blocks) count_done(p, my_blocks, my_tasks);
+#ifdef SLATE_SPMV_PROFILE
+    if (lane == 0 && blockIdx.x < 148) {
+      long long* o = spmv_prof[blockIdx.x][warp];
+      o[0] = clock64() - pf_t0; o[1] = pf_wait; o[2] = pf_first; o[3] = pf_comp; o[4] = q;
+    }
+#endif
   }
-  __syncthreads();   // every compute warp is done: the CTA's blocks are complete
+  __syncthreads();
   if (warp == kTaskWarp) {
-    if (lane == 0 && H.blocks) count_done(p, H.blocks, H.tasks);
     if (lane == 0) atomicAdd(&p.tc->live_rank[H.rank], 0xffffffffu);   // live_rank -= 1
     if (H.retired) check_shrink_done(p, H.ctrl, lane);
     if (lane == 0) leave_main(p);   // after the shrink bookkeeping (see slate_device.cuh)
@@ -398,8 +517,8 @@ static cudaError_t launch_standalone(const void* args, dim3 grid, cudaStream_t s
   slate_args_spmv a;
   std::memcpy(&a, args, sizeof(a));
   void* kargs[] = {&a};
-  return cudaLaunchKernel(reinterpret_cast<const void*>(&standalone<SpmvSeg>), grid, dim3(SpmvSeg::kThreads), kargs,
-                          0, st);
+  return cudaLaunchKernel(reinterpret_cast<const void*>(&standalone<SpmvSeg>), grid, dim3(SpmvSeg::kThreads),
+                          kargs, 0, st);
 }
 
 }  // namespace spmv
