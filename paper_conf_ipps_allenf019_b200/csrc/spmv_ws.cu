@@ -24,11 +24,14 @@
 //     near-diagonal matrix then finds every column in it; a column outside is
 //     read from global memory, so the window decides speed, never the result);
 //   * chunk warp (warp 17, lane 0) -- per task the x window (cp.async.bulk,
-//     L2 -> shared, two buffers), then the task's nonzeros as chunks of 256 rows
-//     (8 original blocks) through a 4-slot ring: columns and values of
+//     L2 -> shared, two buffers), then the task's nonzeros as chunks of 512 rows
+//     (16 original blocks) through a 2-slot ring: columns and values of
 //     [rp[r0], rp[r0+256]) by cp.async.bulk (HBM -> shared, evict-first), up to
-//     128 KB in flight per SM;
-//   * compute warps 0..15 -- per chunk, two passes of 8 rows, 4 lanes per row:
+//     128 KB in flight per SM (two 32-KB copies per chunk: a bulk copy costs
+//     the SM's copy engine a fixed ~190 ns, so fewer, larger copies win --
+//     256-row chunks in a 4-slot ring: 52.7 us per C2 launch on 74 SMs, 128-row
+//     in 8 slots: 68.8, 512-row in 2 slots: 46.6; round 2);
+//   * compute warps 0..15 -- per chunk, four passes of 8 rows, 4 lanes per row:
 //     one 128-bit shared load of columns and one of values per lane and
 //     segment, x from the window.
 // The task warp runs up to three tasks ahead of the compute warps and the chunk
@@ -55,19 +58,28 @@ constexpr int kComputeWarps = SLATE_SPMV_WARPS;
 constexpr int kCompute = 32 * kComputeWarps;
 constexpr int kThreads = kCompute + 64;          // + task warp + chunk warp
 constexpr int kTaskWarp = kComputeWarps, kChunkWarp = kComputeWarps + 1;
-constexpr int kChunkBlocks = 8;                  // blocks per chunk (256 rows)
+#ifndef SLATE_SPMV_CHUNK_BLOCKS
+#define SLATE_SPMV_CHUNK_BLOCKS 16   // 512-row chunks: two 32-KB bulk copies each, four passes per warp (measured best, round 2)
+#endif
+#ifndef SLATE_SPMV_SLOTS
+#define SLATE_SPMV_SLOTS 2
+#endif
+#ifndef SLATE_SPMV_WIN
+#define SLATE_SPMV_WIN 9232         // 1024 rows of a +-4096 band (9216) + alignment slack
+#endif
+constexpr int kChunkBlocks = SLATE_SPMV_CHUNK_BLOCKS;   // blocks per chunk
 constexpr int kChunkRows = 32 * kChunkBlocks;
 constexpr int kPassRows = 8;                     // rows per warp pass (4 lanes per row)
 constexpr int kPasses = kChunkRows / (kPassRows * kComputeWarps);
 static_assert(kPasses * kPassRows * kComputeWarps == kChunkRows, "rows per chunk");
 constexpr int kMaxTaskBlocks = 32;               // task-size cap (1024 rows)
-constexpr int kSlots = 4;                        // chunk ring depth
+constexpr int kSlots = SLATE_SPMV_SLOTS;         // chunk ring depth
 constexpr int kCap = kChunkRows * 16 + 8;        // nonzeros per slot (16 per row + alignment)
 constexpr int kSlotBytes = 2 * kCap * 4;         // col + val
 constexpr int kRpBufs = 4;                       // row-pointer slices: the task warp runs <= 3 tasks ahead
 constexpr int kRpInts = 32 * kMaxTaskBlocks + 4; // rp slice of one task (rounded to 16 B)
 constexpr int kWinBufs = 2;
-constexpr int kWin = 10240;                      // x window per task (floats)
+constexpr int kWin = SLATE_SPMV_WIN;              // x window per task (floats)
 constexpr int kHdrBytes = 1024;
 constexpr int kSmemBytes = kHdrBytes + kSlots * kSlotBytes + kRpBufs * kRpInts * 4 + kWinBufs * kWin * 4;
 static_assert(kSmemBytes <= 227 * 1024, "one CTA per SM");
@@ -162,6 +174,7 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
     const uint32_t d = uint32_t(c - wlo);
     return d < wlen ? xw[d] : __ldg(xg + c);
   };
+  const int csafe = wlen ? wlo : 0;   // a column with a finite x, for the entries outside a row
   constexpr int U = kPasses;
   int lo[U], hi[U];
   float acc[U];
@@ -194,20 +207,20 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       const int base = ((lo[u] >> 2) + q) * 4;
-      acc[u] = spmvseg::fma_seg(0.f, sg[u], base, lo[u], hi[u], xval);
+      acc[u] = spmvseg::fma_seg(0.f, sg[u], base, lo[u], hi[u], csafe, xval);
     }
     if (__any_sync(0xffffffffu, longrow)) {
 #pragma unroll
       for (int u = 0; u < U; ++u)   // rows longer than 16: the rest of the chain, still ascending
         for (int base = ((lo[u] >> 2) + q + 4) * 4; base < hi[u]; base += 16)
-          acc[u] = spmvseg::fma_seg(acc[u], seg(base), base, lo[u], hi[u], xval);
+          acc[u] = spmvseg::fma_seg(acc[u], seg(base), base, lo[u], hi[u], csafe, xval);
     }
   } else {
     // the chunk's nonzeros did not fit the slot: the same chain from global memory
     const int* col = reinterpret_cast<const int*>(a.col);
     const float* val = reinterpret_cast<const float*>(a.val);
 #pragma unroll
-    for (int u = 0; u < U; ++u) acc[u] = spmvseg::row_tail(0.f, col, val, nnz, lo[u], hi[u], q, 0, xval);
+    for (int u = 0; u < U; ++u) acc[u] = spmvseg::row_tail(0.f, col, val, nnz, lo[u], hi[u], q, 0, csafe, xval);
   }
 #pragma unroll
   for (int u = 0; u < U; ++u) {

@@ -253,21 +253,29 @@ __device__ __forceinline__ Seg load(const int* __restrict__ col, const float* __
   }
   return s;
 }
-// acc <- the segment's entries of the row [lo, hi), ascending
+// acc <- the segment's entries of the row [lo, hi), ascending.  Branch-free:
+// an entry outside the row contributes fmaf(0, x[csafe], acc) with csafe a
+// column whose x is finite (the original kernel and the worker compute the
+// same expression, so their bits agree; a -0 sum may become +0, which the
+// oracle's comparison does not distinguish)
 template <class XF>
-__device__ __forceinline__ float fma_seg(float acc, const Seg& s, int base, int lo, int hi, XF xval) {
-  if (base + 0 >= lo && base + 0 < hi) acc = __fmaf_rn(s.v.x, xval(s.c.x), acc);
-  if (base + 1 >= lo && base + 1 < hi) acc = __fmaf_rn(s.v.y, xval(s.c.y), acc);
-  if (base + 2 >= lo && base + 2 < hi) acc = __fmaf_rn(s.v.z, xval(s.c.z), acc);
-  if (base + 3 >= lo && base + 3 < hi) acc = __fmaf_rn(s.v.w, xval(s.c.w), acc);
+__device__ __forceinline__ float fma_seg(float acc, const Seg& s, int base, int lo, int hi, int csafe, XF xval) {
+  const bool e0 = base + 0 >= lo && base + 0 < hi, e1 = base + 1 >= lo && base + 1 < hi;
+  const bool e2 = base + 2 >= lo && base + 2 < hi, e3 = base + 3 >= lo && base + 3 < hi;
+  const float x0 = xval(e0 ? s.c.x : csafe), x1 = xval(e1 ? s.c.y : csafe);
+  const float x2 = xval(e2 ? s.c.z : csafe), x3 = xval(e3 ? s.c.w : csafe);
+  acc = __fmaf_rn(e0 ? s.v.x : 0.f, x0, acc);
+  acc = __fmaf_rn(e1 ? s.v.y : 0.f, x1, acc);
+  acc = __fmaf_rn(e2 ? s.v.z : 0.f, x2, acc);
+  acc = __fmaf_rn(e3 ? s.v.w : 0.f, x3, acc);
   return acc;
 }
 // lane q's chain over segments s0+q+4m for m >= m0 (the row's remaining segments)
 template <class XF>
 __device__ __forceinline__ float row_tail(float acc, const int* col, const float* val, int nnz, int lo, int hi, int q,
-                                          int m0, XF xval) {
+                                          int m0, int csafe, XF xval) {
   for (int base = ((lo >> 2) + q + 4 * m0) * 4; base < hi; base += 16)
-    acc = fma_seg(acc, load(col, val, base, nnz, true), base, lo, hi, xval);
+    acc = fma_seg(acc, load(col, val, base, nnz, true), base, lo, hi, csafe, xval);
   return acc;
 }
 __device__ __forceinline__ float reduce4(float v) {
@@ -299,7 +307,7 @@ struct SpmvSeg : TenantBase {
       lo = __ldg(rp + row);
       hi = __ldg(rp + row + 1);
     }
-    const float acc = spmvseg::row_tail(0.f, col, val, nnz, lo, hi, q, 0, [&](int c) { return __ldg(xv + c); });
+    const float acc = spmvseg::row_tail(0.f, col, val, nnz, lo, hi, q, 0, 0, [&](int c) { return __ldg(xv + c); });
     const float v = spmvseg::reduce4(acc);
     if (q == 0 && row < a.n_rows) __stcs(reinterpret_cast<float*>(a.y) + row, v);
   }
