@@ -94,29 +94,37 @@ struct Triad : TenantBase {
 // ============================================================== copy  a = b
 // 4096 elements (16 KiB) per block, moved global -> shared -> global by the
 // bulk-copy (TMA) engine: one thread issues, no registers hold data.  The
-// worker pipelines the blocks of a task through kStages shared-memory buffers
-// (loads of later blocks in flight while earlier ones are stored), which is
-// what lets a few SMs saturate HBM (the E1 knee).
+// worker streams a task's blocks -- contiguous in memory -- through kStages
+// shared-memory stages of kUnit blocks each: one bulk load and one bulk store
+// per unit, loads of later units in flight while earlier ones are stored.
+// Units never cross a task boundary (the next task's blocks are elsewhere in
+// memory).  Measured (round 2, tools/copy_probe.py): with 1-block units in 4
+// stages (64 KiB, 3 CTAs per SM) an SM moves ~100 GB/s of copy traffic (read +
+// write), HBM saturates at ~70 of 148 SMs; 64-KiB units in 3 stages (1 CTA
+// per SM) reach only ~64 GB/s per SM, 32-KiB units x 2 stages (3 CTAs) the
+// same ~100: the SM's own memory interface, not the per-copy cost, is the
+// limit, and a copy tenant cannot saturate HBM on fewer SMs.
 struct Copy : TenantBase {
   using Args = slate_args_copy;
   static constexpr int kThreads = 128;
 #ifndef SLATE_COPY_STAGES
 #define SLATE_COPY_STAGES 4
 #endif
-#ifndef SLATE_COPY_SMEM_PAD
-#define SLATE_COPY_SMEM_PAD 0
+#ifndef SLATE_COPY_UNIT
+#define SLATE_COPY_UNIT 1
 #endif
   static constexpr int kStages = SLATE_COPY_STAGES;
+  static constexpr int kUnit = SLATE_COPY_UNIT;           // blocks per stage
   static constexpr int kBlockBytes = 16384;
-  static constexpr int kHdr = 128;                       // barriers + parity word
-  static constexpr int kSmem = kHdr + kStages * kBlockBytes + SLATE_COPY_SMEM_PAD;
+  static constexpr int kHdr = 128;                        // barriers + parity word
+  static constexpr int kSmem = kHdr + kStages * kUnit * kBlockBytes;
   static constexpr int kSmemStandalone = kHdr + kBlockBytes;
   static constexpr bool kHasInit = true, kLookahead = true, kHasFini = true;
 
   __device__ __forceinline__ static uint64_t* bars(char* smem) { return reinterpret_cast<uint64_t*>(smem); }
   __device__ __forceinline__ static uint32_t* parity(char* smem) { return reinterpret_cast<uint32_t*>(smem + 64); }
-  __device__ __forceinline__ static uint32_t* state(char* smem);
-  __device__ __forceinline__ static char* stage(char* smem, int s) { return smem + kHdr + s * kBlockBytes; }
+  __device__ __forceinline__ static uint32_t* state(char* smem) { return reinterpret_cast<uint32_t*>(smem + 72); }
+  __device__ __forceinline__ static char* stage(char* smem, int s) { return smem + kHdr + s * kUnit * kBlockBytes; }
 
   __device__ __forceinline__ static void cta_init(char* smem) {
     if (threadIdx.x == 0) {
@@ -130,21 +138,21 @@ struct Copy : TenantBase {
   __device__ __forceinline__ static void cta_fini(char*) {
     if (threadIdx.x == 0) bulk_wait0();          // stores complete before the CTA exits
   }
-  // bytes of block x moved by the bulk engine (multiple of 16); the rest by threads
-  __device__ __forceinline__ static uint32_t bulk_bytes(const Args& a, uint32_t x) {
-    const uint64_t e0 = uint64_t(x) * 4096;
-    const uint64_t e1 = min(e0 + 4096, a.n);
-    return uint32_t(((e1 - e0) * 4) & ~uint64_t(15));
+  // bytes of blocks [x0, x1) moved by the bulk engine (a multiple of 16); the rest by threads
+  __device__ __forceinline__ static uint32_t bulk_bytes(const Args& a, uint32_t x0, uint32_t x1) {
+    const uint64_t e0 = uint64_t(x0) * 4096;
+    const uint64_t e1 = min(uint64_t(x1) * 4096, a.n);
+    return e1 > e0 ? uint32_t(((e1 - e0) * 4) & ~uint64_t(15)) : 0u;
   }
-  __device__ __forceinline__ static void tail(const Args& a, uint32_t x) {
-    const uint64_t e0 = uint64_t(x) * 4096 + bulk_bytes(a, x) / 4;
-    const uint64_t e1 = min(uint64_t(x) * 4096 + 4096, a.n);
+  __device__ __forceinline__ static void tail(const Args& a, uint32_t x0, uint32_t x1) {
+    const uint64_t e0 = uint64_t(x0) * 4096 + bulk_bytes(a, x0, x1) / 4;
+    const uint64_t e1 = min(uint64_t(x1) * 4096, a.n);
     for (uint64_t i = e0; i < e1; ++i) reinterpret_cast<float*>(a.a)[i] = reinterpret_cast<const float*>(a.b)[i];
   }
-  __device__ __forceinline__ static void issue_load(const Args& a, char* smem, uint32_t x, int s) {
-    const uint32_t nb = bulk_bytes(a, x);
+  __device__ __forceinline__ static void issue_load(const Args& a, char* smem, uint32_t x0, uint32_t x1, int s) {
+    const uint32_t nb = bulk_bytes(a, x0, x1);
     mbar_expect_tx(bars(smem) + s, nb);
-    bulk_g2s(stage(smem, s), reinterpret_cast<const char*>(a.b) + uint64_t(x) * kBlockBytes, nb, bars(smem) + s);
+    bulk_g2s(stage(smem, s), reinterpret_cast<const char*>(a.b) + uint64_t(x0) * kBlockBytes, nb, bars(smem) + s);
   }
   __device__ __forceinline__ static void wait_load(char* smem, int s) {
     uint32_t& par = *parity(smem);
@@ -154,51 +162,52 @@ struct Copy : TenantBase {
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t x, uint32_t, uint32_t, char* smem) {
     if (threadIdx.x != 0) return;
     bulk_wait_read0();                           // the buffer is free
-    if (bulk_bytes(a, x)) {
-      issue_load(a, smem, x, 0);
+    if (bulk_bytes(a, x, x + 1)) {
+      issue_load(a, smem, x, x + 1, 0);
       wait_load(smem, 0);
-      bulk_s2g(reinterpret_cast<char*>(a.a) + uint64_t(x) * kBlockBytes, stage(smem, 0), bulk_bytes(a, x));
+      bulk_s2g(reinterpret_cast<char*>(a.a) + uint64_t(x) * kBlockBytes, stage(smem, 0), bulk_bytes(a, x, x + 1));
       bulk_commit();
     }
-    tail(a, x);
+    tail(a, x, x + 1);
   }
-  // The blocks of this task and of the next one form one stream through the
-  // stage ring: while the last stores of this task drain, the first loads of
-  // the next task are already in flight.  state: [0] blocks of this task
-  // already loaded by the previous call, [1] stage of this task's first block.
+  // The units of this task (blocks [g, g+n)) and of the next one ([g2, g2+n2))
+  // form one stream through the stage ring: while the last stores of this task
+  // drain, the first loads of the next task are already in flight.  state: [0]
+  // units of this task already loaded by the previous call, [1] stage of this
+  // task's first unit.
   __device__ __forceinline__ static void cta_task2(const Args& a, uint32_t g, uint32_t n, uint32_t g2, uint32_t n2,
                                                    char* smem) {
     if (threadIdx.x != 0) return;
     uint32_t* st = state(smem);
     const uint32_t pre = st[0], seq = st[1];
-    const uint32_t total = n + n2;
-    auto blk = [&](uint32_t k) { return k < n ? g + k : g2 + (k - n); };
+    const uint32_t ua = (n + kUnit - 1) / kUnit, ub = (n2 + kUnit - 1) / kUnit;
+    const uint32_t total = ua + ub;
+    auto first = [&](uint32_t k) { return k < ua ? g + k * kUnit : g2 + (k - ua) * kUnit; };
+    auto last = [&](uint32_t k) { return k < ua ? min(g + (k + 1) * kUnit, g + n) : min(g2 + (k - ua + 1) * kUnit, g2 + n2); };
     auto stg = [&](uint32_t k) { return int((seq + k) % kStages); };
     uint32_t issued = pre;
     if (issued < kStages) bulk_wait_read0();   // stages about to be refilled have been read out
     for (; issued < min(total, uint32_t(kStages)); ++issued)
-      if (bulk_bytes(a, blk(issued))) issue_load(a, smem, blk(issued), stg(issued));
-    for (uint32_t i = 0; i < n; ++i) {
-      const uint32_t x = g + i;
-      const uint32_t nb = bulk_bytes(a, x);
+      if (bulk_bytes(a, first(issued), last(issued))) issue_load(a, smem, first(issued), last(issued), stg(issued));
+    for (uint32_t i = 0; i < ua; ++i) {
+      const uint32_t x0 = first(i), x1 = last(i);
+      const uint32_t nb = bulk_bytes(a, x0, x1);
       if (nb) {
         wait_load(smem, stg(i));
-        bulk_s2g(reinterpret_cast<char*>(a.a) + uint64_t(x) * kBlockBytes, stage(smem, stg(i)), nb);
+        bulk_s2g(reinterpret_cast<char*>(a.a) + uint64_t(x0) * kBlockBytes, stage(smem, stg(i)), nb);
         bulk_commit();
       }
-      tail(a, x);
+      tail(a, x0, x1);
       if (issued < total && issued == i + kStages) {
-        bulk_wait_read0();                       // stage of block i has been read by its store
-        if (bulk_bytes(a, blk(issued))) issue_load(a, smem, blk(issued), stg(issued));
+        bulk_wait_read0();                       // the stage of unit i has been read by its store
+        if (bulk_bytes(a, first(issued), last(issued))) issue_load(a, smem, first(issued), last(issued), stg(issued));
         ++issued;
       }
     }
-    st[0] = issued > n ? issued - n : 0;
-    st[1] = (seq + n) % kStages;
+    st[0] = issued > ua ? issued - ua : 0;
+    st[1] = (seq + ua) % kStages;
   }
 };
-
-__device__ __forceinline__ uint32_t* Copy::state(char* smem) { return reinterpret_cast<uint32_t*>(smem + 72); }
 
 // ============================================================== naive SGEMM  C = A B
 // The CUDA-sample-style naive kernel: one thread per C element, no tiling.
