@@ -72,7 +72,7 @@ typedef enum {
   SLATE_KIND_SGEMM_NAIVE = 3,  /* C = A B, fp32 row-major; 16x16 C tile/block, T = 256  */
   SLATE_KIND_SPMV_CSR = 4,     /* y = A x, CSR int32/fp32; 32 rows/block, T = 256       */
   SLATE_KIND_BLACKSCHOLES = 5, /* mean call/put over P sigmas; 1024 options/block, T=256 */
-  SLATE_KIND_STENCIL2D = 6,    /* 5-point Jacobi sweep; 32x8 points/block, T = 256      */
+  SLATE_KIND_STENCIL2D = 6,    /* 5-point Jacobi sweep; 128x8 points/block, T = 256     */
   SLATE_KIND_GEMM_BF16 = 7,    /* C(fp32) = A B^T, bf16 K-major; 128x128 tile/block     */
   /* The paper's own applications (Tab II; NEXT-2).  Black-Scholes
    * (BS) is SLATE_KIND_BLACKSCHOLES with one scenario. */
@@ -153,10 +153,11 @@ slate_status slate_get_info(slate_session* s, slate_info* out);
  * launch that uses it has completed and the buffer is unshared/detached.
  * Through an endpoint the server drops its mapping asynchronously once no
  * session references the allocation: when the device is idle, else within
- * ~0.5 s (a mapping is never closed on a session's issue path, because
- * closing waits for the device).  CUDA leaves freeing exported memory before
- * every importer closed it undefined, so a client that frees a buffer while
- * other tenants keep the server busy should wait ~0.5 s after unsharing.
+ * 30 s or once unreferenced mappings exceed 8 GiB (a mapping is never closed
+ * on a session's issue path, because closing waits for the device).  CUDA
+ * leaves freeing exported memory before every importer closed it undefined:
+ * a client that frees a buffer while other tenants keep the server busy
+ * relies on the driver's reference to the allocation until then.
  * Errors: EINVAL (null/zero range, not device memory), EIPC. */
 slate_status slate_share_buffer(slate_session* s, uint64_t dev_ptr, size_t bytes, uint64_t* handle);
 slate_status slate_unshare_buffer(slate_session* s, uint64_t handle);

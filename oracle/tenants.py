@@ -38,7 +38,7 @@ COPY_E = 4096
 SGEMM_TILE = 16
 SPMV_ROWS = 32
 BS_E = 1024
-STENCIL_BX, STENCIL_BY = 32, 8
+STENCIL_BX, STENCIL_BY = 128, 8   # 128 columns x 8 rows per block (the tenant's float4 geometry)
 GEMM_TILE = 128
 
 

@@ -79,7 +79,7 @@ slate_status slate_kind_geometry(uint32_t kind, uint32_t* tile_m, uint32_t* tile
     case SLATE_KIND_SGEMM_NAIVE: *tile_m = 16; *tile_n = 16; return SLATE_OK;
     case SLATE_KIND_SPMV_CSR: *tile_m = 1; *tile_n = 32; return SLATE_OK;
     case SLATE_KIND_BLACKSCHOLES: *tile_m = 1; *tile_n = 1024; return SLATE_OK;
-    case SLATE_KIND_STENCIL2D: *tile_m = 8; *tile_n = 32; return SLATE_OK;
+    case SLATE_KIND_STENCIL2D: *tile_m = 8; *tile_n = 128; return SLATE_OK;
     case SLATE_KIND_TRANSPOSE: *tile_m = 32; *tile_n = 32; return SLATE_OK;
     case SLATE_KIND_SGEMM_TILED: *tile_m = 32; *tile_n = 32; return SLATE_OK;
     case SLATE_KIND_QRNG: *tile_m = 1; *tile_n = 1024; return SLATE_OK;

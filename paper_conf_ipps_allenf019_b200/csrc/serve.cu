@@ -40,7 +40,8 @@ void on_signal(int) { g_stop = 1; }
 // 12-360 ms at the end of C4 runs.  The reaper waits for an idle device, but
 // only so long: an unreferenced mapping is closed anyway once it is older than
 // kMaxUnrefAge or the unreferenced mappings exceed kMaxUnrefBytes, so memory of
-// clients that left is given back under continuous load.  Contract (slate.h):
+// clients that left is given back under continuous load (the age is long: a
+// close stalls every session's issue, so it should land between jobs).  Contract (slate.h):
 // a client keeps a shared allocation alive until slate_unshare_buffer /
 // slate_detach of it returned; the server's mapping goes within kMaxUnrefAge.
 struct Opened {
@@ -52,7 +53,7 @@ struct Opened {
 std::mutex g_ipc_mu;      // the map
 std::mutex g_ipc_close_mu;  // held while mappings are being closed (and by an open of a new handle)
 std::map<std::string, Opened> g_ipc;
-constexpr auto kMaxUnrefAge = std::chrono::milliseconds(500);
+constexpr auto kMaxUnrefAge = std::chrono::seconds(30);   // 0.5 s closed C4's buffers mid-run (steps 41 -> 61 ms)
 constexpr uint64_t kMaxUnrefBytes = 8ull << 30;
 
 void unref_ipc_locked(const std::string& key) {

@@ -472,7 +472,7 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     }
     case SLATE_KIND_STENCIL2D: {
       auto a = static_cast<const slate_args_stencil*>(d->args);
-      g[0] = cdiv(a->w, 32);
+      g[0] = cdiv(a->w, 128);
       g[1] = cdiv(a->h, 8);
       break;
     }

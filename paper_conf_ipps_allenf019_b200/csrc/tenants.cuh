@@ -618,35 +618,69 @@ struct BlackScholesShort : BlackScholes {
 };
 
 // ============================================================== 2-D 5-point stencil
-// One Jacobi sweep of an h x w field; 32 x 8 points per block.  Each thread
-// owns one point; the up/down neighbours come from the rows above/below
-// (L1/L2 reuse across the block's warps), left/right via warp shuffles with
-// the two block-edge columns loaded directly.
+// One Jacobi sweep of an h x w field; 128 x 8 points per block (north star:
+// 128-bit HBM access).  Warp r owns row 8y + r, lane l the 4 columns
+// 128x + 4l .. +3: one float4 load of the point row and one each of the rows
+// above and below (the block's other warps load those rows too: L1/L2 hits,
+// HBM reads every row once), left/right neighbours by warp shuffles inside the
+// float4s and across lanes, the block's two edge columns by scalar loads.
+// Fields whose width is not a multiple of 4 (or the ragged right edge) take a
+// scalar path.  Arithmetic per point as the oracle's parenthesisation:
+// 0.25 * ((up + down) + (left + right)); boundary points copied.
 struct Stencil2D : TenantBase {
   using Args = slate_args_stencil;
-  static constexpr int kThreads = 256;        // 32 x 8
-  static constexpr int kMinBlocks = 8;       // 32 registers, no spill
+  static constexpr int kThreads = 256;        // 8 warps: 8 rows x 32 lanes x 4 columns
+  static constexpr int kMinBlocks = 8;
   static constexpr int kSmem = 0, kSmemStandalone = 0;
 
+  __device__ __forceinline__ static float pt(float up, float down, float left, float right) {
+    return __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up, down), __fadd_rn(left, right)));
+  }
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t bx, uint32_t by, uint32_t, char*) {
     const float* in = reinterpret_cast<const float*>(a.in);
-    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
-    const int i = int(by) * 8 + ty, j = int(bx) * 32 + tx;
+    float* out = reinterpret_cast<float*>(a.out);
+    const int lane = int(threadIdx.x & 31), r = int(threadIdx.x >> 5);
     const int h = int(a.h), w = int(a.w);
-    const bool inside = i < h && j < w;
-    const float c = inside ? __ldg(in + uint64_t(i) * w + j) : 0.f;
-    float left = __shfl_up_sync(0xffffffffu, c, 1);
-    float right = __shfl_down_sync(0xffffffffu, c, 1);
-    if (!inside) return;
-    if (i == 0 || j == 0 || i == h - 1 || j == w - 1) {
-      reinterpret_cast<float*>(a.out)[uint64_t(i) * w + j] = c;
+    const int i = int(by) * 8 + r, j0 = int(bx) * 128 + lane * 4;
+    if ((w & 3) == 0) {
+      // vector path: every lane with j0 < w holds 4 whole columns
+      const bool inside = i < h && j0 < w;
+      const bool interior_row = i > 0 && i < h - 1;
+      float4 c = make_float4(0.f, 0.f, 0.f, 0.f), u = c, d = c;
+      if (inside) {
+        c = __ldg(reinterpret_cast<const float4*>(in + uint64_t(i) * w + j0));
+        if (interior_row) {
+          u = __ldg(reinterpret_cast<const float4*>(in + uint64_t(i - 1) * w + j0));
+          d = __ldg(reinterpret_cast<const float4*>(in + uint64_t(i + 1) * w + j0));
+        }
+      }
+      float left = __shfl_up_sync(0xffffffffu, c.w, 1);     // column j0 - 1 (lane - 1's last)
+      float right = __shfl_down_sync(0xffffffffu, c.x, 1);  // column j0 + 4 (lane + 1's first)
+      if (!inside) return;
+      if (lane == 0 && j0 > 0) left = __ldg(in + uint64_t(i) * w + j0 - 1);
+      if ((lane == 31 || j0 + 4 >= w) && j0 + 4 < w) right = __ldg(in + uint64_t(i) * w + j0 + 4);
+      float4 o = c;
+      if (interior_row) {
+        if (j0 > 0) o.x = pt(u.x, d.x, left, c.y);
+        o.y = pt(u.y, d.y, c.x, c.z);
+        o.z = pt(u.z, d.z, c.y, c.w);
+        if (j0 + 3 < w - 1) o.w = pt(u.w, d.w, c.z, right);
+      }
+      __stcs(reinterpret_cast<float4*>(out + uint64_t(i) * w + j0), o);
       return;
     }
-    if (tx == 0) left = __ldg(in + uint64_t(i) * w + j - 1);
-    if (tx == 31) right = __ldg(in + uint64_t(i) * w + j + 1);
-    const float up = __ldg(in + uint64_t(i - 1) * w + j), down = __ldg(in + uint64_t(i + 1) * w + j);
-    const float v = __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up, down), __fadd_rn(left, right)));
-    reinterpret_cast<float*>(a.out)[uint64_t(i) * w + j] = v;
+    // scalar path (w not a multiple of 4): the same points one at a time
+    if (i >= h) return;
+    for (int k = 0; k < 4; ++k) {
+      const int j = j0 + k;
+      if (j >= w) break;
+      const float cc = in[uint64_t(i) * w + j];
+      float v = cc;
+      if (i > 0 && i < h - 1 && j > 0 && j < w - 1)
+        v = pt(in[uint64_t(i - 1) * w + j], in[uint64_t(i + 1) * w + j], in[uint64_t(i) * w + j - 1],
+               in[uint64_t(i) * w + j + 1]);
+      out[uint64_t(i) * w + j] = v;
+    }
   }
 };
 

@@ -477,7 +477,7 @@ def bs_args(S, X, T, call, put, sigmas, r):
 
 def stencil_args(inp, out):
     h, w = inp.shape
-    return ArgsStencil(_ptr(inp), _ptr(out), h, w), (cdiv(w, 32), cdiv(h, 8), 1)
+    return ArgsStencil(_ptr(inp), _ptr(out), h, w), (cdiv(w, 128), cdiv(h, 8), 1)
 
 
 def kind_geometry(kind):

@@ -36,6 +36,9 @@ CASES = {
     "bs": lambda: make_bs(1024 * 12 + 4 * 33 + 2, 108, n_scen=5),
     "stencil_float": lambda: make_stencil(8 * 37 + 3, 32 * 9 + 5, 109),
     "stencil_int": lambda: make_stencil(77, 130, 110, "int"),
+    # width a multiple of 4: the float4 path, a ragged last block of 64 columns
+    "stencil_vec_float": lambda: make_stencil(8 * 13 + 5, 128 * 3 + 64, 113),
+    "stencil_vec_int": lambda: make_stencil(8 * 5 + 2, 128 * 2 + 4, 114, "int"),
     "gemm_int": lambda: make_gemm(256, 512, 512, 113, "int"),
     "gemm_float": lambda: make_gemm(768, 512, 1024, 114),
     # the paper's Tab II apps (NEXT-2)
