@@ -308,6 +308,28 @@ slate_status slate_transform_source(const char* source, const char* kernel_name,
  * hits, on-disk hits (any pointer may be NULL). */
 void slate_rtc_stats(uint64_t* compiles, uint64_t* mem_hits, uint64_t* disk_hits);
 
+/* NEXT-1, the fused co-run worker (a kernel shrinks when another
+ * arrives and "seamlessly claims" the SMs of one that completes
+ * the workers' exit conditions).  Launches da (session sa) and db (session
+ * sb) as ONE persistent kernel: every CTA holds the uniform shape of the pair
+ * and, at each task boundary, works for the tenant whose range (its session's
+ * resize word) holds its SM rank -- or for the other one once its own tenant
+ * has no task left -- so a resize in either direction and the grow on
+ * completion need no launch, no top-up grid and no standby CTA.  B starts on
+ * the top sm_b ranks, A on the rest.  Each launch keeps its own id, control
+ * block, coverage / rank log, counters and resize-latency stamps: slate_sync,
+ * slate_query and slate_resize work on either as on separate launches.
+ * Both sessions must be in-process sessions of the same server with no launch
+ * queued or running.  Pairs: any two of TRIAD, SGEMM_NAIVE, SGEMM_TILED,
+ * BLACKSCHOLES, STENCIL2D, TRANSPOSE (the kinds sharing a 256-thread CTA with
+ * no per-CTA state).  *la / *lb receive the two ids.
+ * Errors: EINVAL (sm_b outside [1, N-1], bad descriptors, sa == sb's queue),
+ * ESTATE (a session busy), EUNSUPPORTED (kind pair, or not in-process),
+ * ENOMEM (control blocks), ECUDA. */
+slate_status slate_launch_fused(slate_session* sa, slate_kernel ka, const slate_launch_desc* da, slate_session* sb,
+                                slate_kernel kb, const slate_launch_desc* db, uint32_t sm_b, slate_launch_id* la,
+                                slate_launch_id* lb);
+
 /* Resize the SM range of the queue that owns launch l to [sm_lo, sm_hi]
  * (§III-C; the dispatcher's start_sm/end_sm, Lst3 P:L250-251).
  * Publishes {epoch+1, lo, hi} to the device with a stream memory write that

@@ -243,6 +243,18 @@ slate_status slate_set_policy(slate_session* s, uint32_t policy) {
   return rc >= SLATE_OK ? rc : fail(s, rc, err);
 }
 
+slate_status slate_launch_fused(slate_session* sa, slate_kernel ka, const slate_launch_desc* da, slate_session* sb,
+                                slate_kernel kb, const slate_launch_desc* db, uint32_t sm_b, slate_launch_id* la,
+                                slate_launch_id* lb) {
+  if (!sa || !sb || !da || !db || !la || !lb) return fail(sa, SLATE_EINVAL, "null argument");
+  if (!sa->srv || sa->srv != sb->srv)
+    return fail(sa, SLATE_EUNSUPPORTED, "a fused pair needs two in-process sessions of one server");
+  std::scoped_lock g(sa->mu, sb->mu);
+  std::string err;
+  const int rc = sa->srv->launch_fused(sa->queue, ka, da, sb->queue, kb, db, sm_b, la, lb, &err);
+  return rc == SLATE_OK ? rc : fail(sa, rc, err);
+}
+
 slate_status slate_set_split_objective(slate_session* s, uint32_t objective, double slack) {
   if (!s) return SLATE_EINVAL;
   std::lock_guard<std::mutex> g(s->mu);

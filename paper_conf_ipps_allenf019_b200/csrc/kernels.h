@@ -144,6 +144,13 @@ bool build_user_kind(const char* src, const char* name, uint32_t bx, uint32_t by
 
 const KindOps* kind_ops(uint32_t kind);   // nullptr if the kind is not built
 
+// NEXT-1 (fused.cu): one persistent kernel running two tenants (kind_a, kind_b)
+bool fused_supported(uint32_t kind_a, uint32_t kind_b);
+cudaError_t fused_shape(uint32_t kind_a, uint32_t kind_b, const void** fn, int* threads, int* smem);
+cudaError_t launch_fused(uint32_t kind_a, uint32_t kind_b, const WorkerCommon& wa, const void* args_a,
+                         const WorkerCommon& wb, const void* args_b, uint32_t grow_on_drain, uint32_t grid,
+                         cudaStream_t st);
+
 // cudaLaunchKernel, or with programmatic dependent launch (PDL): the kernel may
 // start while the previous kernel on the stream drains, and waits for it in
 // griddepcontrol.wait (tools/probe/pdl_cost.cu: ~2 us per back-to-back launch)

@@ -923,6 +923,8 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   // it in stream order); launches before it that finished all their blocks but
   // are not yet retired by the poller do not count
   static const bool dbg = std::getenv("SLATE_DEBUG") != nullptr;
+  for (uint64_t lid : Q.issued)   // a fused co-run kernel (NEXT-1): its CTAs switch tenant, no launch
+    if (launches_[lid]->fused) return SLATE_OK;
   if (!Q.issued.empty()) {
     // kinds whose last main CTA waits for all blocks (leave_main): top up the
     // RUNNING launch -- the first issued one that has not finished its blocks --
@@ -1066,6 +1068,131 @@ int Server::launch_many(uint32_t q, uint32_t n, const uint64_t* ks, const slate_
   auto qi = queues_.find(q);
   if (qi != queues_.end()) close_batch(*qi->second, nullptr);
   return rc;
+}
+
+// NEXT-1 (fused.cuh): one persistent kernel runs both launches; each keeps its
+// own control block, resize word (its queue's) and records, so sync, query
+// and resize work as for separate launches, but a resize -- and the grow when
+// one tenant drains -- needs no top-up launch: the CTAs switch tenant
+// at their next task boundary.
+int Server::launch_fused(uint32_t qa, uint64_t ka, const slate_launch_desc* da, uint32_t qb, uint64_t kb,
+                         const slate_launch_desc* db, uint32_t sm_b, uint64_t* la, uint64_t* lb, std::string* err) {
+  std::unique_lock<std::mutex> g(mu_);
+  auto fail = [&](int rc, const char* m) {
+    if (err) *err = m;
+    return rc;
+  };
+  if (qa == qb) return fail(SLATE_EINVAL, "a fused pair needs two sessions (queues)");
+  auto qia = queues_.find(qa), qib = queues_.find(qb);
+  auto kia = kernels_.find(ka), kib = kernels_.find(kb);
+  if (qia == queues_.end() || qib == queues_.end() || kia == kernels_.end() || kib == kernels_.end())
+    return fail(SLATE_ENOTFOUND, "unknown session or kernel");
+  const KernelEntry& KA = *kia->second;
+  const KernelEntry& KB = *kib->second;
+  if (!fused_supported(KA.desc.kind, KB.desc.kind))
+    return fail(SLATE_EUNSUPPORTED, "no fused worker for this pair of kinds");
+  if (da->mode != SLATE_MODE_SLATE || db->mode != SLATE_MODE_SLATE) return fail(SLATE_EINVAL, "fused launches are slate mode");
+  if (sm_b == 0 || sm_b >= uint32_t(n_sms_)) return fail(SLATE_EINVAL, "sm_b must be in [1, N-1]");
+  if ((da->coverage && !(KA.desc.flags & SLATE_KFLAG_COVERAGE)) || (db->coverage && !(KB.desc.flags & SLATE_KFLAG_COVERAGE)))
+    return fail(SLATE_EINVAL, "coverage log given but the kernel was not registered with SLATE_KFLAG_COVERAGE");
+  Queue& A = *qia->second;
+  Queue& B = *qib->second;
+  auto idle = [](const Queue& Q) { return Q.issued.empty() && Q.pending.empty() && Q.deferred.empty(); };
+  if (!idle(A) || !idle(B)) return fail(SLATE_ESTATE, "both sessions must have no launch queued or running");
+  uint32_t BA = 0, BB = 0;
+  if (!validate(KA, da, &BA, err) || !validate(KB, db, &BB, err)) return SLATE_EINVAL;
+  if (free_slots_.size() < 2) return fail(SLATE_ENOMEM, "control-block pool exhausted");
+  const uint32_t n = uint32_t(n_sms_);
+  // the ranges: A [0, n - sm_b - 1], B [n - sm_b, n - 1]; both queues hold SMs
+  for (Queue* Q : {&A, &B}) {
+    if (!Q->active) {
+      Q->active = true;
+      active_.push_back(Q->id);
+    }
+    Q->explicit_range = true;
+    Q->auto_split = false;
+  }
+  int rc = write_ctrl(A, 0, n - sm_b - 1, false, err);
+  if (rc == SLATE_OK) rc = write_ctrl(B, n - sm_b, n - 1, false, err);
+  if (rc != SLATE_OK) return rc;
+  Launch* Ls[2];
+  WorkerCommon w[2];
+  const KernelEntry* Ks[2] = {&KA, &KB};
+  const slate_launch_desc* Ds[2] = {da, db};
+  Queue* Qs[2] = {&A, &B};
+  const uint32_t Bs[2] = {BA, BB};
+  cudaEvent_t ev_start = nullptr, ev_end = nullptr, ev_snap = nullptr;
+  CK(cudaEventCreate(&ev_start));
+  CK(cudaEventCreate(&ev_end));
+  CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
+  // the kernel goes on A's stream after B's stream is ready (its resize word written)
+  cudaEvent_t ev_b;
+  CK(cudaEventCreateWithFlags(&ev_b, cudaEventDisableTiming));
+  CK(cudaEventRecord(ev_b, B.stream));
+  CK(cudaStreamWaitEvent(A.stream, ev_b, 0));
+  cudaEventDestroy(ev_b);
+  for (int i = 0; i < 2; ++i) {
+    auto L = std::make_unique<Launch>();
+    L->id = next_launch_id_++;
+    L->queue = Qs[i]->id;
+    L->k = Ks[i];
+    L->desc = *Ds[i];
+    L->args.assign(static_cast<const unsigned char*>(Ds[i]->args),
+                   static_cast<const unsigned char*>(Ds[i]->args) + Ds[i]->args_size);
+    L->desc.args = nullptr;
+    L->B = Bs[i];
+    L->iters = Ks[i]->desc.iters ? Ks[i]->desc.iters : choose_iters(*Ks[i], Ds[i], Bs[i]);
+    L->fused = true;
+    L->slot = alloc_slot();
+    std::memset(reinterpret_cast<void*>(h_mirror_ + L->slot), 0, sizeof(HostMirror));
+    if (slot_zeroed_[L->slot] && cudaEventQuery(slot_zeroed_[L->slot]) != cudaSuccess)
+      CK(cudaStreamWaitEvent(A.stream, slot_zeroed_[L->slot], 0));
+    L->ev_start = ev_start;
+    L->ev_end.push_back(ev_end);
+    L->ev_done.push_back(ev_snap);
+    L->state = 1;
+    const auto& gd = L->desc.grid;
+    WorkerCommon& c = w[i];
+    c.gx = gd[0]; c.gy = gd[1]; c.gz = gd[2]; c.B = L->B; c.iters = L->iters; c.occ = 1;
+    c.bound_lo = 0; c.bound_hi = n - 1; c.n_ranks = n;
+    c.standby_timeout_ns = standby_timeout_ns_;
+    c.base_epoch = Qs[i]->epoch;
+    c.is_topup = 0;
+    c.gate_first = 0;
+    c.ctrl = Qs[i]->d_ctrl; c.tc = d_tc_ + L->slot; c.mirror = d_mirror_ + L->slot;
+    c.cov = reinterpret_cast<uint32_t*>(L->desc.coverage);
+    c.ranklog = (Ks[i]->desc.flags & SLATE_KFLAG_RANKLOG) && c.cov ? 1u : 0u;
+    c.rank_of = d_rank_of_;
+    Ls[i] = L.get();
+    launches_[L->id] = std::move(L);
+  }
+  const void* fn = nullptr;
+  int threads = 0, smem = 0, occ = 0;
+  CK(fused_shape(KA.desc.kind, KB.desc.kind, &fn, &threads, &smem));
+  if (smem > 48 * 1024) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
+  if (occ < 1) return fail(SLATE_ECUDA, "the fused worker does not fit on an SM");
+  w[0].occ = w[1].occ = uint32_t(occ);
+  CK(cudaEventRecord(ev_start, A.stream));
+  CK(slate::launch_fused(KA.desc.kind, KB.desc.kind, w[0], Ls[0]->args.data(), w[1], Ls[1]->args.data(), 1u,
+                  uint32_t(occ) * n, A.stream));
+  CK(cudaEventRecord(ev_end, A.stream));
+  CK(cudaStreamWaitEvent(B.stream, ev_end, 0));   // B's later launches follow the fused kernel
+  A.last_op_kernel = B.last_op_kernel = false;
+  CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+  for (Launch* L : Ls)
+    CK(cudaMemcpyAsync(h_snap_ + size_t(L->slot) * kTaskCtlHeader, d_tc_ + L->slot, kTaskCtlHeader,
+                       cudaMemcpyDeviceToHost, copy_stream_));
+  CK(cudaEventRecord(ev_snap, copy_stream_));
+  for (int i = 0; i < 2; ++i) {
+    Qs[i]->issued.push_back(Ls[i]->id);
+    Qs[i]->cov_lo = 0;
+    Qs[i]->cov_hi = n - 1;
+  }
+  *la = Ls[0]->id;
+  *lb = Ls[1]->id;
+  cv_.notify_all();
+  return SLATE_OK;
 }
 
 int Server::launch_locked(uint32_t q, uint64_t kid, const slate_launch_desc* d, uint64_t* out, std::string* err,
@@ -1680,6 +1807,16 @@ void Server::launch_times(const Launch& L, double* start, double* end) const {
     *t1 = tc.t_last;
     return X.has_snapshot && tc.t_first && tc.t_last;
   };
+  if (L.fused && L.has_snapshot) {   // one tenant of a fused kernel: its own first task to its last block
+    TaskCtl tc;
+    std::memcpy(&tc, L.snapshot, kTaskCtlHeader);
+    const double k0 = ev_ms(L.ev_start);
+    if (k0 >= 0 && tc.t_enter && tc.t_first && tc.t_last) {
+      *start = std::max(0.0, k0 + double(tc.t_first - tc.t_enter) * 1e-6);
+      *end = std::max(*start, k0 + double(tc.t_last - tc.t_enter) * 1e-6);
+      return;
+    }
+  }
   double s = ev_ms(L.ev_start ? L.ev_start : L.start_after), e = -1.0;
   for (cudaEvent_t x : L.ev_end) e = std::max(e, ev_ms(x));
   const Launch* F = &L;

@@ -54,6 +54,7 @@ struct Launch {
   std::vector<uint8_t> resize_kind;   // 1 shrink, 2 grow
   unsigned char snapshot[kTaskCtlHeader];   // final TaskCtl header copy
   bool has_snapshot = false;
+  bool fused = false;           // one tenant of a fused co-run kernel (NEXT-1): no top-ups; times from device stamps
 };
 
 struct Queue {
@@ -112,6 +113,10 @@ class Server {
   int launch_many(uint32_t q, uint32_t n, const uint64_t* ks, const slate_launch_desc* ds, uint64_t* first,
                   std::string* err);
   int resize(uint32_t q, uint64_t l, uint32_t lo, uint32_t hi, std::string* err);
+  // NEXT-1: launches da (queue qa) and db (queue qb) as ONE fused worker kernel,
+  // B on the top sm_b ranks, A on the rest; both queues must be idle
+  int launch_fused(uint32_t qa, uint64_t ka, const slate_launch_desc* da, uint32_t qb, uint64_t kb,
+                   const slate_launch_desc* db, uint32_t sm_b, uint64_t* la, uint64_t* lb, std::string* err);
   int set_policy(uint32_t policy, std::string* err);
   int set_split_objective(uint32_t objective, double slack, std::string* err);
   int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);

@@ -188,6 +188,9 @@ _lib.slate_choose_split_obj.argtypes = [_P(c_u32), _P(c_f64), c_u32, _P(c_u32), 
 _lib.slate_fluid_corun_obj.restype = ctypes.c_int
 _lib.slate_fluid_corun_obj.argtypes = [_P(c_u32), _P(c_f64), c_u32, c_f64, _P(c_u32), _P(c_f64), c_u32, c_f64, c_u32,
                                        c_u32, c_u32, c_u32, c_f64, c_u32, c_f64, _P(c_u32), _P(c_f64)]
+_lib.slate_launch_fused.restype = c_i32
+_lib.slate_launch_fused.argtypes = [ctypes.c_void_p, c_u64, ctypes.c_void_p, ctypes.c_void_p, c_u64, ctypes.c_void_p,
+                                    c_u32, _P(c_u64), _P(c_u64)]
 _lib.slate_set_split_objective.restype = c_i32
 _lib.slate_set_split_objective.argtypes = [ctypes.c_void_p, c_u32, c_f64]
 _lib.slate_fluid_corun.restype = ctypes.c_int
@@ -203,7 +206,7 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
             "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters",
             "slate_register_source", "slate_transform_source", "slate_corun_makespan_k", "slate_choose_split_k",
-            "slate_rtc_stats", "slate_choose_split_obj", "slate_fluid_corun_obj", "slate_set_split_objective"]
+            "slate_rtc_stats", "slate_choose_split_obj", "slate_fluid_corun_obj", "slate_set_split_objective", "slate_launch_fused"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -413,6 +416,19 @@ def choose_split_k(curves, n_sms, step=2):
     t = _lib.slate_choose_split_k(ctypes.cast(sms, ctypes.c_void_p), ctypes.cast(ms, ctypes.c_void_p), npts,
                                   len(curves), n_sms, step, out)
     return list(out), t
+
+
+def launch_fused(sa, ka, args_a, grid_a, sb, kb, args_b, grid_b, sm_b, coverage_a=None, coverage_b=None):
+    """NEXT-1: launches A (session sa) and B (session sb) as one fused co-run
+    kernel, B on the top sm_b SM ranks; returns (id_a, id_b)."""
+    da = sa._desc(args_a, grid_a, coverage=coverage_a)
+    db = sb._desc(args_b, grid_b, coverage=coverage_b)
+    la, lb = c_u64(), c_u64()
+    st = _lib.slate_launch_fused(sa._h, ka, ctypes.byref(da), sb._h, kb, ctypes.byref(db), sm_b, ctypes.byref(la),
+                                 ctypes.byref(lb))
+    if st < 0:
+        raise SlateError(st, "slate_launch_fused: " + _lib.slate_last_error(sa._h).decode())
+    return la.value, lb.value
 
 
 def transform_source(source, name, threads=256, smem=0, block=None):
