@@ -137,60 +137,100 @@ __device__ __forceinline__ void fused_body(const FusedParams<TA, TB>& fp) {
     pre_nb = ld_relaxed_u32(&pb.tc->next);
   }
   uint32_t backoff = 128;
+  // speculative boundary: once a task is decided, the counter atomic for the
+  // same tenant's next task is issued and its result read at the next
+  // boundary, so the round trip overlaps the task (the generic worker's
+  // kSpeculative mode; a resize is honoured within two tasks, reading Q23).
+  // A task fetched that way is always run -- fetched means owned.
+  uint32_t spec_g = 0xffffffffu;
+  int spec_t = -1;
+  uint64_t spec_c = 0;
+  // the tenant this CTA should work for now, from the prefetched words and
+  // counters: 0 / 1, -1 standby (outside both ranges), -2 exit (both drained);
+  // *c the range in force (the tenant's word, or the whole chip when it works
+  // for a tenant because the partner drained)
+  auto choose = [&](uint64_t* c) -> int {
+    const uint64_t ca = pre_ca, cb = pre_cb;
+    if (ctrl_epoch(ca) != seen_ea || ctrl_epoch(cb) != seen_eb) {
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");   // completes the acquire of the new word
+      seen_ea = ctrl_epoch(ca);
+      seen_eb = ctrl_epoch(cb);
+    }
+    const bool da = pre_na >= pa.B, db = pre_nb >= pb.B;
+    if (da && db) return -2;                                           // exit (2): both queues drained
+    const bool ina = in_range(pa, rank, ca), inb = in_range(pb, rank, cb);
+    const uint64_t all_a = pack_ctrl(ctrl_epoch(ca), 0, pa.n_ranks - 1);
+    const uint64_t all_b = pack_ctrl(ctrl_epoch(cb), 0, pb.n_ranks - 1);
+    if (ina && !da) { *c = ca; return 0; }
+    if (inb && !db) { *c = cb; return 1; }
+    if (fp.grow_on_drain && da && !db) { *c = all_b; return 1; }       // the drained tenant's SMs
+    if (fp.grow_on_drain && db && !da) { *c = all_a; return 0; }
+    return -1;
+  };
   for (;;) {
     if (threadIdx.x == 0) {
       uint32_t ten = 2, g = 0xffffffffu;
-      for (;;) {
-        const uint64_t ca = pre_ca, cb = pre_cb;
-        if (ctrl_epoch(ca) != seen_ea || ctrl_epoch(cb) != seen_eb) {
-          asm volatile("fence.acq_rel.gpu;" ::: "memory");   // completes the acquire of the new word
-          seen_ea = ctrl_epoch(ca);
-          seen_eb = ctrl_epoch(cb);
-        }
-        const bool da = pre_na >= pa.B, db = pre_nb >= pb.B;
-        if (da && db) break;                                           // exit (2): both queues drained
-        const bool ina = in_range(pa, rank, ca), inb = in_range(pb, rank, cb);
-        int want = -1;
-        if (ina && !da) want = 0;
-        else if (inb && !db) want = 1;
-        else if (fp.grow_on_drain && da && !db) want = 1;               // the drained tenant's SMs
-        else if (fp.grow_on_drain && db && !da) want = 0;
-        if (want < 0) {                                                 // outside both ranges: standby
-          leave();
-          __nanosleep(backoff);
-          if (backoff < 2048) backoff <<= 1;
-          prefetch();
-          continue;
-        }
-        backoff = 128;
-        const uint64_t c = want == 0 ? ca : cb;
-        if (want != cur) {
-          leave();
-          cur = want;
-          if (cur == 0) fused_join(pa, rank, c);
-          else fused_join(pb, rank, c);
-        }
-        // the range in force for this task: the tenant's word, or the whole
-        // chip when the CTA works for it because its partner drained
-        const bool by_drain = want == 0 ? !ina : !inb;
-        c_cur = by_drain ? pack_ctrl(ctrl_epoch(c), 0, pa.n_ranks - 1) : c;
-        // Lst2 (2): the task counter of the chosen tenant
-        g = cur == 0 ? atomicAdd(&pa.tc->next, pa.iters) : atomicAdd(&pb.tc->next, pb.iters);
-        if (cur == 0 ? g >= pa.B : g >= pb.B) {                        // drained meanwhile: decide again
-          prefetch();
-          if (cur == 0) pre_na = pa.B;
-          else pre_nb = pb.B;
-          continue;
-        }
-        if (g == 0) (cur == 0 ? pa.tc : pb.tc)->t_first = globaltimer();
-        if (cur == 0) log_task(pa, g, rank, c_cur, false);
+      bool keep = false;
+      if (spec_t >= 0 && spec_g < (spec_t == 0 ? pa.B : pb.B)) {
+        // a task fetched at the previous boundary: owned, so run it; keep
+        // speculating only if this CTA would still choose the same tenant
+        ten = uint32_t(spec_t);
+        g = spec_g;
+        c_cur = spec_c;
+        if (ten == 0) log_task(pa, g, rank, c_cur, false);
         else log_task(pb, g, rank, c_cur, false);
-        ten = uint32_t(cur);
-        break;
+        uint64_t c = 0;
+        keep = choose(&c) == int(ten);
+        if (keep) c_cur = c;
+      } else {
+        if (spec_t == 0) pre_na = pa.B;   // the speculative fetch found the tenant drained
+        if (spec_t == 1) pre_nb = pb.B;
+        for (;;) {
+          uint64_t c = 0;
+          const int want = choose(&c);
+          if (want == -2) break;
+          if (want == -1) {                                               // outside both ranges: standby
+            leave();
+            __nanosleep(backoff);
+            if (backoff < 2048) backoff <<= 1;
+            prefetch();
+            continue;
+          }
+          backoff = 128;
+          if (want != cur) {
+            leave();
+            cur = want;
+            if (cur == 0) fused_join(pa, rank, c);
+            else fused_join(pb, rank, c);
+          }
+          c_cur = c;
+          // Lst2 (2): the task counter of the chosen tenant
+          g = cur == 0 ? atomicAdd(&pa.tc->next, pa.iters) : atomicAdd(&pb.tc->next, pb.iters);
+          if (cur == 0 ? g >= pa.B : g >= pb.B) {                        // drained meanwhile: decide again
+            prefetch();
+            if (cur == 0) pre_na = pa.B;
+            else pre_nb = pb.B;
+            continue;
+          }
+          if (cur == 0) log_task(pa, g, rank, c_cur, false);
+          else log_task(pb, g, rank, c_cur, false);
+          ten = uint32_t(cur);
+          keep = true;
+          break;
+        }
+      }
+      spec_t = -1;
+      if (ten != 2) {
+        if (g == 0) (ten == 0 ? pa.tc : pb.tc)->t_first = globaltimer();
+        prefetch();                              // the next boundary's words, in flight during the task
+        if (keep) {                              // the same tenant's next task, in flight during this one
+          spec_t = int(ten);
+          spec_c = c_cur;
+          spec_g = ten == 0 ? atomicAdd(&pa.tc->next, pa.iters) : atomicAdd(&pb.tc->next, pb.iters);
+        }
       }
       s_ten = ten;
       s_g = g;
-      if (ten != 2) prefetch();                  // in flight during the task
     }
     __syncthreads();
     const uint32_t ten = s_ten, g = s_g;

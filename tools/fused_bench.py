@@ -89,7 +89,7 @@ out["gain_fused_vs_seq"] = round(out["seq"]["makespan_ms"] / out["fused"]["makes
 
 # resize storm on fused pairs: complementary ranges, 100 us apart
 rng = random.Random(7)
-lat = {1: [], 2: []}
+lat = {"shrink": [], "grow": []}
 issued = 0
 while issued < 120:
     la, lb = S.launch_fused(sa, ka, A[0], A[1], sb, kb, B[0], B[1], split)
@@ -106,7 +106,7 @@ while issued < 120:
     sb.sync(lb)
     for q in (sa.query(la), sb.query(lb)):
         for v, kd in zip(q["resize_us"], q["resize_kind"]):
-            if kd and v >= 0:
+            if kd in lat and v >= 0:
                 lat[kd].append(v)
 
 
@@ -115,7 +115,7 @@ def stats(v):
             "p99": round(float(np.percentile(v, 99)), 2) if v else None, "max": round(max(v), 2) if v else None}
 
 
-out["fused_resize_us"] = {"shrink": stats(lat[1]), "grow": stats(lat[2]), "resizes_issued": issued}
+out["fused_resize_us"] = {"shrink": stats(lat["shrink"]), "grow": stats(lat["grow"]), "resizes_issued": issued}
 bs_task_us = pa["solo_ms"] * 1e3 * 4 * n / (8192)   # a worker's time per BS block (4 CTAs/SM x n SMs)
 out["bs_block_us"] = round(bs_task_us, 2)
 print(json.dumps(out))
