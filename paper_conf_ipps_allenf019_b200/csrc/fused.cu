@@ -31,6 +31,7 @@ struct Pair {
     fill<TA>(p.a, wa, aa);
     fill<TB>(p.b, wb, ab);
     p.grow_on_drain = grow;
+    p.speculative = 0;
     void* kargs[] = {&p};
     return cudaLaunchKernel(reinterpret_cast<const void*>(&slate_fused<TA, TB>), dim3(grid), dim3(TA::kThreads), kargs,
                             kSmem, st);

@@ -35,6 +35,7 @@ struct FusedParams {
   WorkerParams<typename TA::Args> a;
   WorkerParams<typename TB::Args> b;
   uint32_t grow_on_drain;   // a drained tenant's SMs go to the other at once
+  uint32_t speculative;     // fetch the same tenant's next task during this one (see fused_body)
 };
 
 // whole-CTA-free (thread 0) version of check_shrink_done for the fused worker
@@ -137,11 +138,13 @@ __device__ __forceinline__ void fused_body(const FusedParams<TA, TB>& fp) {
     pre_nb = ld_relaxed_u32(&pb.tc->next);
   }
   uint32_t backoff = 128;
-  // speculative boundary: once a task is decided, the counter atomic for the
-  // same tenant's next task is issued and its result read at the next
-  // boundary, so the round trip overlaps the task (the generic worker's
-  // kSpeculative mode; a resize is honoured within two tasks, reading Q23).
-  // A task fetched that way is always run -- fetched means owned.
+  // speculative boundary (optional): once a task is decided, the counter
+  // atomic for the same tenant's next task is issued and its result read at
+  // the next boundary, so the round trip overlaps the task (the generic
+  // worker's kSpeculative mode); a task fetched that way is always run --
+  // fetched means owned -- so a resize is then honoured within two tasks, not
+  // one.  Measured (tools/fused_bench.py): no throughput gain on the pairs
+  // tried, twice the grow latency; off by default.
   uint32_t spec_g = 0xffffffffu;
   int spec_t = -1;
   uint64_t spec_c = 0;
@@ -223,7 +226,7 @@ __device__ __forceinline__ void fused_body(const FusedParams<TA, TB>& fp) {
       if (ten != 2) {
         if (g == 0) (ten == 0 ? pa.tc : pb.tc)->t_first = globaltimer();
         prefetch();                              // the next boundary's words, in flight during the task
-        if (keep) {                              // the same tenant's next task, in flight during this one
+        if (keep && fp.speculative) {            // the same tenant's next task, in flight during this one
           spec_t = int(ten);
           spec_c = c_cur;
           spec_g = ten == 0 ? atomicAdd(&pa.tc->next, pa.iters) : atomicAdd(&pb.tc->next, pb.iters);
@@ -251,8 +254,13 @@ __device__ __forceinline__ void fused_body(const FusedParams<TA, TB>& fp) {
   if (threadIdx.x == 0) leave();
 }
 
+// the uniform CTA shape's occupancy is the lower of the two tenants' (the
+// register budget of the hungrier body): a memory tenant paired with a
+// register-heavy compute tenant runs with fewer CTAs -- less memory in flight
+// -- than on its own (tools/fused_bench.py)
 template <class TA, class TB>
-__global__ void __launch_bounds__(TA::kThreads, 4) slate_fused(const __grid_constant__ FusedParams<TA, TB> p) {
+__global__ void __launch_bounds__(TA::kThreads, (TA::kMinBlocks < TB::kMinBlocks ? TA::kMinBlocks : TB::kMinBlocks))
+    slate_fused(const __grid_constant__ FusedParams<TA, TB> p) {
   fused_body<TA, TB>(p);
 }
 

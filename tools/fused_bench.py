@@ -29,17 +29,27 @@ from paper_conf_ipps_allenf019_b200 import slate as S  # noqa: E402
 dev = "cuda:0"
 sa, sb = S.Session(None, 0), S.Session(None, 0)
 n = sa.info()["num_sms"]
-Sx, X, T, r = I.bs_inputs(1 << 23, I.seed_for(2, 1))
-Sx, X, T = (torch.from_numpy(v).to(dev) for v in (Sx, X, T))
-sig = torch.from_numpy(I.bs_sigmas(32)).to(dev)
-cl, pu = torch.zeros(1 << 23, device=dev), torch.zeros(1 << 23, device=dev)
-f = torch.rand(16384, 16384, device=dev)
-o = torch.zeros_like(f)
+PAIR = sys.argv[1] if len(sys.argv) > 1 else "bs+stencil"
+if PAIR == "bs+stencil":
+    Sx, X, T, r = I.bs_inputs(1 << 23, I.seed_for(2, 1))
+    Sx, X, T = (torch.from_numpy(v).to(dev) for v in (Sx, X, T))
+    sig = torch.from_numpy(I.bs_sigmas(32)).to(dev)
+    cl, pu = torch.zeros(1 << 23, device=dev), torch.zeros(1 << 23, device=dev)
+    f = torch.rand(16384, 16384, device=dev)
+    o = torch.zeros_like(f)
+    A = S.bs_args(Sx, X, T, cl, pu, sig, r)
+    B = S.stencil_args(f, o)
+    kinds = (S.KIND_BLACKSCHOLES, S.KIND_STENCIL2D)
+    desc = "Black-Scholes 2^23 x 32 scenarios (A) + stencil 16384^2 (B), one launch each"
+else:   # the C1 kinds at a size that runs ~1 ms: naive SGEMM 1024^3 (A) + triad 2^27 (B)
+    Am, Bm, Cm = (torch.rand(1024, 1024, device=dev) for _ in range(3))
+    a, b, c = (torch.rand(1 << 27, device=dev) for _ in range(3))
+    A = S.sgemm_args(Am, Bm, Cm)
+    B = S.triad_args(a, b, c, 3.0)
+    kinds = (S.KIND_SGEMM_NAIVE, S.KIND_TRIAD)
+    desc = "naive SGEMM 1024^3 (A) + STREAM triad 2^27 (B), one launch each (config C1's kinds)"
 torch.cuda.synchronize()
-A = S.bs_args(Sx, X, T, cl, pu, sig, r)
-B = S.stencil_args(f, o)
-ka, kb = sa.register_kernel(S.KIND_BLACKSCHOLES), sb.register_kernel(S.KIND_STENCIL2D)
-ka_s, kb_s = sa.register_kernel(S.KIND_BLACKSCHOLES), sb.register_kernel(S.KIND_STENCIL2D)
+ka, kb = sa.register_kernel(kinds[0]), sb.register_kernel(kinds[1])
 pa = sa.profile(ka, *A, S.PROF_CURVE)
 pb = sb.profile(kb, *B, S.PROF_CURVE)
 ca = dict(zip(pa["curve_sms"], pa["curve_ms"]))
@@ -76,7 +86,7 @@ def run(kind):
     return max(a1, b1) - min(a0, b0), [a1 - min(a0, b0), b1 - min(a0, b0), qa["n_topups"] + qb["n_topups"]]
 
 
-out = {"pair": "Black-Scholes 2^23 x 32 scenarios (A) + stencil 16384^2 (B), one launch each",
+out = {"pair": desc,
        "split_sms_b": split, "predicted_makespan_ms": round(pred, 4)}
 for kind in ("seq", "corun", "fused"):
     for _ in range(2):
@@ -116,8 +126,6 @@ def stats(v):
 
 
 out["fused_resize_us"] = {"shrink": stats(lat["shrink"]), "grow": stats(lat["grow"]), "resizes_issued": issued}
-bs_task_us = pa["solo_ms"] * 1e3 * 4 * n / (8192)   # a worker's time per BS block (4 CTAs/SM x n SMs)
-out["bs_block_us"] = round(bs_task_us, 2)
 print(json.dumps(out))
 sa.close()
 sb.close()
