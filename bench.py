@@ -96,6 +96,30 @@ def aggregate(world, steps, total_ms_per_rank_max):
     return world * steps / (total_ms_per_rank_max / 1e3)
 
 
+def gather(world, obj):
+    """Every rank's `obj` (a small JSON-able dict) on every rank."""
+    if world == 1:
+        return [obj]
+    import torch.distributed as dist
+    out = [None] * world
+    dist.all_gather_object(out, obj)
+    return out
+
+
+def c5_aggregate(per_rank):
+    """SURVEY §8(e) / BASELINE configs[4] (C5): independent per-GPU Slate
+    instances, two client sessions per GPU (the C2 pair).  The box's wall-clock
+    gain G_agg = max_g T_g^seq / max_g makespan_g (the slowest GPU sets both),
+    the sum of the per-GPU STPs, and the per-GPU gains (to expose stragglers).
+    per_rank: [{"t_seq_ms", "makespan_ms", "stp"}] in rank order."""
+    t_seq = max(r["t_seq_ms"] for r in per_rank)
+    mk = max(r["makespan_ms"] for r in per_rank)
+    return {"gpus": len(per_rank), "clients": 2 * len(per_rank),
+            "g_agg": round(t_seq / mk, 4), "stp_sum": round(sum(r["stp"] for r in per_rank), 4),
+            "per_gpu_gain": [round(r["t_seq_ms"] / r["makespan_ms"], 4) for r in per_rank],
+            "t_seq_ms_max": round(t_seq, 3), "makespan_ms_max": round(mk, 3)}
+
+
 # ------------------------------------------------------------------ CPU oracle (reference / cpu_baseline)
 _ORACLE_INPUTS = {}
 
@@ -739,9 +763,14 @@ def run_slate(args, world, rank, local):
         c3["resize_storm"] = resize_storm(S, sA, w3.a, sA.info()["num_sms"])
         del w3
 
-    # ---- C4 (configs[3]): four client processes through the slated daemon (rank 0 only)
+    # ---- C5 (configs[4]): the C2 pair on every GPU, aggregated over the ranks
+    med = r2["med"]
+    c5 = c5_aggregate(gather(world, {"t_seq_ms": r2["best_sequential"]["ms"], "makespan_ms": med[0],
+                                     "stp": r2["schedules"]["slate_corun"]["stp"]}))
+
+    # ---- C4 (configs[3]): four client processes through a slated daemon, on every rank's GPU
     c4 = None
-    if rank == 0 and not args.no_c4:
+    if not args.no_c4:
         try:
             sys.path.insert(0, os.path.join(ROOT, "tools"))
             import c4_bench
@@ -785,7 +814,9 @@ def run_slate(args, world, rank, local):
     if c3:
         line["c3"] = c3
     if c4:
-        line["c4"] = c4
+        c4s = gather(world, c4)
+        line["c4"] = c4s[0] if world == 1 else {"per_rank": c4s}
+    line["c5"] = c5
     if cpu:
         line["cpu_baseline"] = cpu
         line["cpu_baseline_all_cores"] = cpu_all

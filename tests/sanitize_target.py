@@ -75,15 +75,41 @@ def run_user(s, n_sms):
     assert np.array_equal(yd.cpu().numpy().astype(np.float64), OT.probe3d(x, block))
 
 
+def run_fused(s, n_sms):
+    """NEXT-1: a fused pair (triad + naive SGEMM, integer inputs) with a resize in flight."""
+    sb = S.Session(None, 0)
+    try:
+        ta, tb = G.make_triad(1024 * 30 + 5, 914, "int"), G.make_sgemm(64, 48, 40, 915, "int")
+        ka = s.register_kernel(ta.kind, iters=3, flags=S.KFLAG_COVERAGE | S.KFLAG_RANKLOG)
+        kb = sb.register_kernel(tb.kind, iters=2, flags=S.KFLAG_COVERAGE | S.KFLAG_RANKLOG)
+        Ba, Bb = int(np.prod(ta.grid)), int(np.prod(tb.grid))
+        ca = torch.zeros(2 * Ba, dtype=torch.int32, device="cuda:0")
+        cb = torch.zeros(2 * Bb, dtype=torch.int32, device="cuda:0")
+        ta.zero_outputs()
+        tb.zero_outputs()
+        la, lb = S.launch_fused(s, ka, ta.args, ta.grid, sb, kb, tb.args, tb.grid, n_sms // 3, ca, cb)
+        s.resize(la, 0, n_sms // 2 - 1)
+        sb.resize(lb, n_sms // 2, n_sms - 1)
+        s.sync(la)
+        sb.sync(lb)
+        torch.cuda.synchronize()
+        assert ta.check(ta.snapshot())[0] and tb.check(tb.snapshot())[0]
+        assert s.query(la)["coverage_ok"] == 1 and sb.query(lb)["coverage_ok"] == 1
+    finally:
+        sb.close()
+
+
 def main():
     import faulthandler
-    groups = sys.argv[1:] or list(GROUPS) + ["user"]
+    groups = sys.argv[1:] or list(GROUPS) + ["user", "fused"]
     faulthandler.dump_traceback_later(float(os.environ.get("SANITIZE_DUMP_S", "600")), exit=True)
     with S.Session(None, 0) as s:
         n = s.info()["num_sms"]
         for g in groups:
             if g == "user":
                 run_user(s, n)
+            elif g == "fused":
+                run_fused(s, n)
             else:
                 for mk in GROUPS[g]:
                     run(s, mk(), n)

@@ -17,7 +17,7 @@ pytestmark = pytest.mark.gpu
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
-GROUPS = ["generic", "apps", "spmv", "gemm", "user"]
+GROUPS = ["generic", "apps", "spmv", "gemm", "user", "fused"]
 
 
 @pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
