@@ -89,7 +89,7 @@ __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 __device__ __forceinline__ void st_cluster(uint32_t raddr, uint32_t v) {
-  asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(raddr), "r"(v) : "memory");
+  asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(raddr), "r"(v) : "memory");  // racecheck: mbarrier-ordered (every use is followed by a remote arrive or a cluster barrier)
 }
 // the leader's progress word in the peer's shared memory: only ever raised
 // (K slices issued, bit 31 when it stopped), so the writer is an atomic max and
@@ -378,7 +378,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       mbar_wait(&S.tq_empty[j], (u & 1) ^ 1);
       fence_cluster();                             // the peer's reads of slot j happened
       S.kb_limit[j] = num_kb;
-      S.tileq[j] = entry;
+      S.tileq[j] = entry;  // racecheck: mbarrier-ordered
       st_cluster(r_tileq[j], entry);
       mbar_arrive(&S.tq_full[j]);
       mbar_arrive_remote(r_tq_full[j]);
@@ -534,7 +534,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
       const uint32_t j = t & 1, u = t >> 1;
       mbar_wait(&S.tq_full[j], u & 1);
       if (!leader) fence_cluster();
-      const uint32_t entry = S.tileq[j];
+      const uint32_t entry = S.tileq[j];  // racecheck: mbarrier-ordered
       __syncwarp();
       if (lane == 0) mbar_arrive_remote(tq_empty0 + j * 8);
       if (entry == 0xffffffffu) break;

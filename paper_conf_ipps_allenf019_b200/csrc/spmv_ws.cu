@@ -118,7 +118,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 __device__ __forceinline__ void bulk_g2s_keep(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                    smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))  // racecheck: mbarrier-ordered
                : "memory");
 }
 
@@ -172,7 +172,7 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
   const uint32_t nrows = min(m.nblk * 32, a.n_rows - row_first);
   auto xval = [&](int c) -> float {
     const uint32_t d = uint32_t(c - wlo);
-    return d < wlen ? xw[d] : __ldg(xg + c);
+    return d < wlen ? xw[d] : __ldg(xg + c);  // racecheck: mbarrier-ordered
   };
   const int csafe = wlen ? wlo : 0;   // a column with a finite x, for the entries outside a row
   constexpr int U = kPasses;
@@ -193,8 +193,8 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
     const int32_t a0 = m.a0;   // the slot holds entries [a0, ...), a0 a multiple of 4
     auto seg = [&](int base) {
       spmvseg::Seg r;
-      r.c = *reinterpret_cast<const int4*>(col + (base - a0));
-      r.v = *reinterpret_cast<const float4*>(val + (base - a0));
+      r.c = *reinterpret_cast<const int4*>(col + (base - a0));  // racecheck: mbarrier-ordered
+      r.v = *reinterpret_cast<const float4*>(val + (base - a0));  // racecheck: mbarrier-ordered
       return r;
     };
     spmvseg::Seg sg[U];
@@ -336,7 +336,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       TaskMeta& tm = H.tmeta[b];
       if (g == 0xffffffffu) {
         if (lane == 0) {
-          tm.g = 0; tm.n = 0; tm.wlo = 0; tm.wlen = 0;
+          tm.g = 0; tm.n = 0; tm.wlo = 0; tm.wlen = 0;  // racecheck: mbarrier-ordered
           H.ctrl = c;                                 // the word the CTA acted on last
         }
         mbar_arrive(&H.rp_full[b]);                   // sentinel: publishes the stop
@@ -403,7 +403,7 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           TRACE(1, 11, q, 0);
           ChunkMeta& m = H.cmeta[s];
           if (tm.n == 0) {
-            m.tb = 0xffffffffu;
+            m.tb = 0xffffffffu;  // racecheck: mbarrier-ordered
             mbar_expect_tx(&H.slot_full[s], 0);
             break;
           }
@@ -418,13 +418,13 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           // by this thread instead
           const bool end = r0 + nrows == a.n_rows;
           const int32_t a0 = e0 & ~3, a1 = end ? (e1 & ~3) : ((e1 + 3) & ~3);
-          m.tb = uint32_t(b); m.wb = uint32_t(wb); m.row0 = row0; m.nblk = nblk; m.a0 = a0;
-          m.first = k == 0; m.last = k + 1 == nch;
+          m.tb = uint32_t(b); m.wb = uint32_t(wb); m.row0 = row0; m.nblk = nblk; m.a0 = a0;  // racecheck: mbarrier-ordered
+          m.first = k == 0; m.last = k + 1 == nch;  // racecheck: mbarrier-ordered
           if (max(a1, e1) - a0 > kCap) {
             m.mode = 1;
             mbar_expect_tx(&H.slot_full[s], 0);
           } else {
-            m.mode = 0;
+            m.mode = 0;  // racecheck: mbarrier-ordered
             for (int32_t j = max(a1, a0); j < e1; ++j) {
               S.col(s)[j - a0] = __ldg(reinterpret_cast<const int32_t*>(a.col) + j);
               S.val(s)[j - a0] = __ldg(reinterpret_cast<const float*>(a.val) + j);
@@ -458,14 +458,14 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       pf_wait += c1 - c0;
 #endif
       if (threadIdx.x == 0) TRACE(2, 20, q, 0);
-      const ChunkMeta m = H.cmeta[s];
+      const ChunkMeta m = H.cmeta[s];  // racecheck: mbarrier-ordered
       if (m.tb == 0xffffffffu) break;
       const int b = int(m.tb);
       if (m.first) {
         mbar_wait(&H.rp_full[b], (t / kRpBufs) & 1);
         mbar_wait(&H.win_full[m.wb], (t / kWinBufs) & 1);
       }
-      const TaskMeta tm = H.tmeta[b];
+      const TaskMeta tm = H.tmeta[b];  // racecheck: mbarrier-ordered
       if (threadIdx.x == 0) TRACE(2, 21, q, 0);
 #ifdef SLATE_SPMV_PROFILE
       long long c2 = clock64();

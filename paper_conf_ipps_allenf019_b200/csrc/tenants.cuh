@@ -53,7 +53,7 @@ __device__ __forceinline__ void bulk_g2s(void* dst_smem, const void* src, uint32
   asm volatile(
       "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
           smem_u32(dst_smem)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(l2_evict_first())
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(l2_evict_first())  // racecheck: mbarrier-ordered
       : "memory");
 }
 __device__ __forceinline__ void bulk_s2g(void* dst, const void* src_smem, uint32_t bytes) {
