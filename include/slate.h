@@ -343,8 +343,13 @@ slate_status slate_launch_fused(slate_session* sa, slate_kernel ka, const slate_
 slate_status slate_resize(slate_session* s, slate_launch_id l, uint32_t sm_lo, uint32_t sm_hi);
 
 /* Wait until launch l (0 = every launch of this session) has run every block
- * and all its worker CTAs have exited.  timeout_us < 0 waits forever.
- * Errors: ETIMEDOUT, ECUDA (sticky kernel error), ENOTFOUND. */
+ * and all its worker CTAs have exited.  timeout_us < 0 waits forever.  A
+ * launch id older than the server's retention window (SLATE_KEEP_FINISHED,
+ * default 65536 completed launches) has completed: SLATE_OK.
+ * The server watchdog: a launch still running SLATE_WATCHDOG_S seconds after
+ * its issue (default 120, 0 = off) is reported -- this call returns ECUDA
+ * ("watchdog") instead of waiting; the kernel itself cannot be preempted.
+ * Errors: ETIMEDOUT, ECUDA (sticky kernel error, watchdog), ENOTFOUND. */
 slate_status slate_sync(slate_session* s, slate_launch_id l, int64_t timeout_us);
 
 /* ------------------------------------------------------------------ profile */

@@ -139,6 +139,7 @@ int Server::init(std::string* err) {
   peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
   standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
   keep_finished_ = size_t(std::max(16.0, env_double("SLATE_KEEP_FINISHED", 65536.0)));
+  watchdog_us_ = env_double("SLATE_WATCHDOG_S", 120.0) * 1e6;
   saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.95);   // reading Q29 (1.0: no cap)
   if (const char* pol = std::getenv("SLATE_POLICY")) {              // reading Q31
     const std::string v(pol);
@@ -905,6 +906,7 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     close_batch(Q, ev_end, true);   // this launch ends the batch
   }
   L.state = 1;
+  L.t_issue_us = now_us();
   if (Q.issued.empty()) {
     Q.cov_lo = Q.lo;
     Q.cov_hi = Q.hi;
@@ -1185,6 +1187,7 @@ int Server::launch_fused(uint32_t qa, uint64_t ka, const slate_launch_desc* da, 
                        cudaMemcpyDeviceToHost, copy_stream_));
   CK(cudaEventRecord(ev_snap, copy_stream_));
   for (int i = 0; i < 2; ++i) {
+    Ls[i]->t_issue_us = now_us();
     Qs[i]->issued.push_back(Ls[i]->id);
     Qs[i]->cov_lo = 0;
     Qs[i]->cov_hi = n - 1;
@@ -1704,7 +1707,20 @@ void Server::poll_once() {
     if (!Q.pending_resize.empty()) resolve_resizes(Q, t, nullptr);
     while (!Q.issued.empty()) {
       Launch& L = *launches_[Q.issued.front()];
-      if (!launch_done_events(L)) break;
+      if (!launch_done_events(L)) {
+        // the server watchdog: a kernel cannot be preempted, but a
+        // launch running past the limit is reported -- its syncs return
+        // ECUDA instead of waiting forever (the context may be wedged)
+        if (watchdog_us_ > 0 && !L.watchdog_fired && t - L.t_issue_us > watchdog_us_) {
+          L.watchdog_fired = true;
+          Q.watchdog = true;
+          if (!Q.first_error) Q.first_error = int(cudaErrorLaunchTimeout);
+          fprintf(stderr, "[slate] watchdog: launch %llu of queue %u running for %.1f s (limit %.1f s)\n",
+                  (unsigned long long)L.id, Q.id, (t - L.t_issue_us) * 1e-6, watchdog_us_ * 1e-6);
+          cv_.notify_all();
+        }
+        break;
+      }
       if (!Q.pending_resize.empty()) resolve_resizes(Q, t, &L);
       if (L.slot >= 0) {
         std::memcpy(L.snapshot, h_snap_ + size_t(L.slot) * kTaskCtlHeader, kTaskCtlHeader);
@@ -1757,10 +1773,10 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
   auto done = [&]() -> bool {
     if (l) {
       auto it = launches_.find(l);
-      return it == launches_.end() || it->second->state == 2;
+      return it == launches_.end() || it->second->state == 2 || it->second->watchdog_fired;
     }
     auto qi = queues_.find(q);
-    return qi == queues_.end() ||
+    return qi == queues_.end() || qi->second->watchdog ||
            (qi->second->issued.empty() && qi->second->pending.empty() && qi->second->deferred.empty());
   };
   // a launch id below the retention window completed long ago (ids are monotonic)
@@ -1779,7 +1795,13 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
   int e = 0;   // per launch, or the queue's first error (no scan over every launch ever made)
   if (l) {
     auto it = launches_.find(l);
-    if (it != launches_.end()) e = it->second->error;
+    if (it != launches_.end()) {
+      e = it->second->error;
+      if (it->second->watchdog_fired) {
+        if (err) *err = "watchdog: the launch ran longer than SLATE_WATCHDOG_S";
+        return SLATE_ECUDA;
+      }
+    }
   } else {
     auto qi = queues_.find(q);
     if (qi != queues_.end()) e = qi->second->first_error;

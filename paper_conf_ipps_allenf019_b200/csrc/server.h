@@ -55,6 +55,8 @@ struct Launch {
   unsigned char snapshot[kTaskCtlHeader];   // final TaskCtl header copy
   bool has_snapshot = false;
   bool fused = false;           // one tenant of a fused co-run kernel (NEXT-1): no top-ups; times from device stamps
+  double t_issue_us = 0;        // host time of the issue (the watchdog's clock)
+  bool watchdog_fired = false;  // ran longer than the watchdog limit: its syncs report an error
 };
 
 struct Queue {
@@ -87,6 +89,7 @@ struct Queue {
   std::vector<PendingResize> pending_resize;
   bool closed = false;
   int first_error = 0;          // the first cudaError_t a launch of this queue completed with
+  bool watchdog = false;        // a launch of this queue outlived the watchdog limit
 };
 
 struct ProfileEntry {
@@ -228,6 +231,7 @@ class Server {
   // dropped in bulk (retire_finished), so a long-running slated stays bounded
   std::deque<uint64_t> finished_;
   size_t keep_finished_ = 65536;   // SLATE_KEEP_FINISHED (tests use a small window)
+  double watchdog_us_ = 120e6;     // SLATE_WATCHDOG_S: a launch issued longer ago is reported (0: off)
   void retire_finished();
   std::deque<uint32_t> waiting_;     // queues waiting for SMs, FIFO
   std::map<uint32_t, uint32_t> bypassed_;
