@@ -285,7 +285,7 @@ bool Server::busy() {
 }
 
 int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
-  const int rc = sync(q, 0, timeout_us, err);
+  const int rc = sync(q, 0, timeout_us, err, true);   // until every launch really finished
   std::lock_guard<std::mutex> g(mu_);
   auto it = queues_.find(q);
   if (it == queues_.end()) return SLATE_ENOTFOUND;
@@ -1714,7 +1714,6 @@ void Server::poll_once() {
         if (watchdog_us_ > 0 && !L.watchdog_fired && t - L.t_issue_us > watchdog_us_) {
           L.watchdog_fired = true;
           Q.watchdog = true;
-          if (!Q.first_error) Q.first_error = int(cudaErrorLaunchTimeout);
           fprintf(stderr, "[slate] watchdog: launch %llu of queue %u running for %.1f s (limit %.1f s)\n",
                   (unsigned long long)L.id, Q.id, (t - L.t_issue_us) * 1e-6, watchdog_us_ * 1e-6);
           cv_.notify_all();
@@ -1767,16 +1766,16 @@ void Server::poller_main() {
 }
 
 // ------------------------------------------------------------------ sync / query
-int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
+int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err, bool through_watchdog) {
   std::unique_lock<std::mutex> g(mu_);
   const auto deadline = std::chrono::steady_clock::now() + std::chrono::microseconds(timeout_us < 0 ? 0 : timeout_us);
   auto done = [&]() -> bool {
     if (l) {
       auto it = launches_.find(l);
-      return it == launches_.end() || it->second->state == 2 || it->second->watchdog_fired;
+      return it == launches_.end() || it->second->state == 2 || (it->second->watchdog_fired && !through_watchdog);
     }
     auto qi = queues_.find(q);
-    return qi == queues_.end() || qi->second->watchdog ||
+    return qi == queues_.end() || (qi->second->watchdog && !through_watchdog) ||
            (qi->second->issued.empty() && qi->second->pending.empty() && qi->second->deferred.empty());
   };
   // a launch id below the retention window completed long ago (ids are monotonic)
@@ -1797,14 +1796,20 @@ int Server::sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err) {
     auto it = launches_.find(l);
     if (it != launches_.end()) {
       e = it->second->error;
-      if (it->second->watchdog_fired) {
+      if (it->second->watchdog_fired && !through_watchdog && it->second->state != 2) {
         if (err) *err = "watchdog: the launch ran longer than SLATE_WATCHDOG_S";
         return SLATE_ECUDA;
       }
     }
   } else {
     auto qi = queues_.find(q);
-    if (qi != queues_.end()) e = qi->second->first_error;
+    if (qi != queues_.end()) {
+      e = qi->second->first_error;
+      if (!e && qi->second->watchdog && !through_watchdog) {
+        if (err) *err = "watchdog: a launch of this session ran longer than SLATE_WATCHDOG_S";
+        return SLATE_ECUDA;
+      }
+    }
   }
   if (e) {
     if (err) *err = std::string("CUDA error: ") + cudaGetErrorString(cudaError_t(e));

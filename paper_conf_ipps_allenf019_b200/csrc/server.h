@@ -122,7 +122,8 @@ class Server {
                    const slate_launch_desc* db, uint32_t sm_b, uint64_t* la, uint64_t* lb, std::string* err);
   int set_policy(uint32_t policy, std::string* err);
   int set_split_objective(uint32_t objective, double slack, std::string* err);
-  int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err);
+  // through_watchdog: wait for the launches to really finish (detach), not only until the watchdog reported
+  int sync(uint32_t q, uint64_t l, int64_t timeout_us, std::string* err, bool through_watchdog = false);
   int profile(uint64_t k, const slate_launch_desc* d, uint32_t flags, slate_profile_t* out, std::string* err);
   int query(uint64_t l, slate_launch_info* out, std::string* err);
   bool kernel_kind(uint64_t k, uint32_t* kind) const;

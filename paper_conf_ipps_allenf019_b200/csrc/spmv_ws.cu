@@ -432,8 +432,17 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
             const uint32_t bytes = uint32_t(max(a1 - a0, 0)) * 4;
             mbar_expect_tx(&H.slot_full[s], 2 * bytes);
             if (bytes) {
-              bulk_g2s(S.col(s), reinterpret_cast<const int32_t*>(a.col) + a0, bytes, &H.slot_full[s]);
-              bulk_g2s(S.val(s), reinterpret_cast<const float*>(a.val) + a0, bytes, &H.slot_full[s]);
+#ifndef SLATE_SPMV_SPLIT
+#define SLATE_SPMV_SPLIT 1   // experiment: each array's chunk as this many bulk copies
+#endif
+              const uint32_t piece = ((bytes + SLATE_SPMV_SPLIT - 1) / SLATE_SPMV_SPLIT + 15) & ~15u;
+              for (uint32_t o = 0; o < bytes; o += piece) {
+                const uint32_t nb = min(piece, bytes - o);
+                bulk_g2s(reinterpret_cast<char*>(S.col(s)) + o, reinterpret_cast<const char*>(a.col) + uint64_t(a0) * 4 + o,
+                         nb, &H.slot_full[s]);
+                bulk_g2s(reinterpret_cast<char*>(S.val(s)) + o, reinterpret_cast<const char*>(a.val) + uint64_t(a0) * 4 + o,
+                         nb, &H.slot_full[s]);
+              }
             }
           }
         }
