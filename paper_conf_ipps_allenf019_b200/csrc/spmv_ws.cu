@@ -76,7 +76,10 @@ constexpr int kMaxTaskBlocks = 32;               // task-size cap (1024 rows)
 constexpr int kSlots = SLATE_SPMV_SLOTS;         // chunk ring depth
 constexpr int kCap = kChunkRows * 16 + 8;        // nonzeros per slot (16 per row + alignment)
 constexpr int kSlotBytes = 2 * kCap * 4;         // col + val
-constexpr int kRpBufs = 4;                       // row-pointer slices: the task warp runs <= 3 tasks ahead
+#ifndef SLATE_SPMV_RPBUFS
+#define SLATE_SPMV_RPBUFS 4
+#endif
+constexpr int kRpBufs = SLATE_SPMV_RPBUFS;       // row-pointer slices: the task warp runs <= kRpBufs-1 tasks ahead
 constexpr int kRpInts = 32 * kMaxTaskBlocks + 4; // rp slice of one task (rounded to 16 B)
 constexpr int kWinBufs = 2;
 constexpr int kWin = SLATE_SPMV_WIN;              // x window per task (floats)
@@ -297,6 +300,10 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       }
       c_pre = ld_acquire_u64(p.ctrl);
     }
+    bool prev_valid = false;              // task t-1: slice in shared memory, not yet published
+    int prev_b = 0;
+    uint32_t prev_g = 0, prev_n = 0;
+    int32_t prev_e0 = 0, prev_e1 = 0;
     for (uint32_t t = 0;; ++t) {
       const int b = int(t % kRpBufs);
       uint32_t g = 0xffffffffu, chg = 0;
@@ -333,6 +340,45 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       chg = __shfl_sync(0xffffffffu, chg, 0);
       c = __shfl_sync(0xffffffffu, c, 0);
       if (chg) check_shrink_done(p, c, lane);
+      // Two tasks in flight (one round trip per task instead of two): this
+      // iteration loads task t's row-pointer slice while lane 0 loads the two
+      // column indices that bound task t-1's x window (its slice arrived in the
+      // previous iteration), then publishes t-1.  Tasks are published in order.
+      const uint32_t n = g == 0xffffffffu ? 0u : min(p.iters, p.B - g);
+      const uint32_t r0 = g * 32, r1 = g == 0xffffffffu ? r0 : min(r0 + n * 32, a.n_rows);
+      const uint32_t cnt = g == 0xffffffffu ? 0u : r1 - r0 + 1, n4 = cnt / 4;
+      const int32_t* rpg = reinterpret_cast<const int32_t*>(a.rowptr) + r0;
+      int32_t* rps = S.rp(b);
+      constexpr int kV = (kRpInts / 4 + 31) / 32;
+      int4 v[kV];
+#pragma unroll
+      for (int k = 0; k < kV; ++k)
+        if (lane + 32 * k < n4) v[k] = __ldg(reinterpret_cast<const int4*>(rpg) + lane + 32 * k);
+      const bool tail = lane < cnt - n4 * 4;
+      const int32_t vt = tail ? __ldg(rpg + n4 * 4 + lane) : 0;
+      if (prev_valid) {
+        if (lane == 0) {
+          // the x window from task t-1's first and last nonzero
+          int32_t wlo = 0;
+          uint32_t wlen = 0;
+          if (prev_e1 > prev_e0) {
+            const int32_t* colg = reinterpret_cast<const int32_t*>(a.col);
+            const int32_t cf = __ldg(colg + prev_e0), cl = __ldg(colg + prev_e1 - 1);
+            const int32_t cmin = min(cf, cl), cmax = max(cf, cl);
+            const int32_t ncols = int32_t(a.n_cols);
+            const int32_t span = cmax - cmin + 1;
+            int32_t lo = span >= kWin ? cmin : cmin - (kWin - span) / 2;
+            lo = max(0, min(lo, ncols - kWin)) & ~3;
+            wlo = lo;
+            // whole granules inside x; columns past the window read global memory
+            wlen = uint32_t(max(0, min(kWin, ncols - lo)) & ~3);
+          }
+          TaskMeta& tp = H.tmeta[prev_b];
+          tp.g = prev_g; tp.n = prev_n; tp.wlo = wlo; tp.wlen = wlen;  // racecheck: mbarrier-ordered
+        }
+        mbar_arrive(&H.rp_full[prev_b]);              // each lane after its stores (count 32)
+        prev_valid = false;
+      }
       TaskMeta& tm = H.tmeta[b];
       if (g == 0xffffffffu) {
         if (lane == 0) {
@@ -342,43 +388,17 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
         mbar_arrive(&H.rp_full[b]);                   // sentinel: publishes the stop
         break;
       }
-      // rp[r0 .. r1] by the whole warp: 16-B loads (r0 = 32 g is 128-B aligned), then the tail
-      const uint32_t n = min(p.iters, p.B - g);
-      const uint32_t r0 = g * 32, r1 = min(r0 + n * 32, a.n_rows);
-      const uint32_t cnt = r1 - r0 + 1, n4 = cnt / 4;
-      const int32_t* rpg = reinterpret_cast<const int32_t*>(a.rowptr) + r0;
-      int32_t* rps = S.rp(b);
-      constexpr int kV = (kRpInts / 4 + 31) / 32;
-      int4 v[kV];
-#pragma unroll
-      for (int k = 0; k < kV; ++k)
-        if (lane + 32 * k < n4) v[k] = __ldg(reinterpret_cast<const int4*>(rpg) + lane + 32 * k);
 #pragma unroll
       for (int k = 0; k < kV; ++k)
         if (lane + 32 * k < n4) reinterpret_cast<int4*>(rps)[lane + 32 * k] = v[k];
-      if (lane < cnt - n4 * 4) rps[n4 * 4 + lane] = __ldg(rpg + n4 * 4 + lane);
+      if (tail) rps[n4 * 4 + lane] = vt;
       __syncwarp();
-      if (lane == 0) {
-        // the x window from the task's first and last nonzero
-        const int32_t e0 = rps[0], e1 = rps[r1 - r0];
-        int32_t wlo = 0;
-        uint32_t wlen = 0;
-        if (e1 > e0) {
-          const int32_t* colg = reinterpret_cast<const int32_t*>(a.col);
-          const int32_t cf = __ldg(colg + e0), cl = __ldg(colg + e1 - 1);
-          const int32_t cmin = min(cf, cl), cmax = max(cf, cl);
-          const int32_t ncols = int32_t(a.n_cols);
-          const int32_t span = cmax - cmin + 1;
-          int32_t lo = span >= kWin ? cmin : cmin - (kWin - span) / 2;
-          lo = max(0, min(lo, ncols - kWin)) & ~3;
-          wlo = lo;
-          // whole granules inside x; columns past the window read global memory
-          wlen = uint32_t(max(0, min(kWin, ncols - lo)) & ~3);
-        }
-        tm.g = g; tm.n = n; tm.wlo = wlo; tm.wlen = wlen;
-        TRACE(0, 3, t, wlen);
-      }
-      mbar_arrive(&H.rp_full[b]);                     // each lane after its stores (count 32)
+      prev_valid = true;
+      prev_b = b;
+      prev_g = g;
+      prev_n = n;
+      prev_e0 = rps[0];
+      prev_e1 = rps[r1 - r0];
     }
   } else if (warp == kChunkWarp) {
     // ===================== chunk warp: nonzeros of each task through the slot ring =====================
