@@ -503,6 +503,17 @@ double slate_corun_makespan_k(const uint32_t* const* sms, const double* const* m
                               const uint32_t* shares);
 double slate_choose_split_k(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, uint32_t k,
                             uint32_t n_sms, uint32_t step, uint32_t* shares_out);
+/* NEXT-4 / reading Q49 ("examines other kernels in the queue"): should
+ * a candidate job (curve k, category cats[k]) join a co-running group of k
+ * jobs (curves 0..k-1 on shares_cur)?  Only if the group keeps at most one
+ * memory-intensive job (categories 3, 4; reading Q37) and the fluid model
+ * predicts gain = (slate_corun_makespan_k(group, shares_cur) + T_k(n_sms)) /
+ * the best (k+1)-way makespan >= min_gain.  shares_out (k+1 entries) receives
+ * the best shares, *gain the prediction.  Returns 1 to admit.  The server
+ * admits a third co-runner this way (SLATE_MAX_CORUN, default 3). */
+int slate_kway_admit(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, const uint32_t* cats,
+                     uint32_t k, const uint32_t* shares_cur, uint32_t n_sms, uint32_t step, double min_gain,
+                     uint32_t* shares_out, double* gain);
 /* Reading Q31 (the B200 selector): should kernel B co-run with the active A
  * although Tab I says solo?  Job curves are `work` launches of each kernel
  * (the launches queued or running) back to back, time = work * curve(s); the

@@ -250,4 +250,24 @@ double slate_choose_split_k(const uint32_t* const* sms, const double* const* ms,
   return best_t;
 }
 
+// NEXT-4 (reading Q49): should the candidate (curve k) join a co-running group
+// of k jobs on shares_cur?  At most one memory-intensive job per group (Q37);
+// gain = (makespan_k(group) + T_candidate(n)) / makespan_{k+1}(best shares).
+// oracle selector.kway_admit
+int slate_kway_admit(const uint32_t* const* sms, const double* const* ms, const uint32_t* npts, const uint32_t* cats,
+                     uint32_t k, const uint32_t* shares_cur, uint32_t n_sms, uint32_t step, double min_gain,
+                     uint32_t* shares_out, double* gain) {
+  if (gain) *gain = 0.0;
+  uint32_t mem = 0;
+  for (uint32_t i = 0; i <= k; ++i) mem += cats[i] >= 3 ? 1u : 0u;
+  if (mem > 1 || k == 0) return 0;
+  const double t_cur = makespan_k(sms, ms, npts, k, shares_cur);
+  const double t_c = interp(sms[k], ms[k], npts[k], double(n_sms));
+  const double t_new = slate_choose_split_k(sms, ms, npts, k + 1, n_sms, step, shares_out);
+  if (t_new <= 0) return 0;
+  const double g = (t_cur + t_c) / t_new;
+  if (gain) *gain = g;
+  return g >= min_gain ? 1 : 0;
+}
+
 }  // extern "C"

@@ -153,6 +153,7 @@ int Server::init(std::string* err) {
   if (const char* o = std::getenv("SLATE_SPLIT_OBJECTIVE"))
     split_objective_ = std::string(o) == "makespan" ? SLATE_SPLIT_MAKESPAN : SLATE_SPLIT_ANTT;
   split_slack_ = env_double("SLATE_SPLIT_SLACK", 0.05);
+  max_corun_ = uint32_t(std::max(2.0, std::min(4.0, env_double("SLATE_MAX_CORUN", 3.0))));
   poller_ = std::thread([this] { poller_main(); });
   return SLATE_OK;
 }
@@ -1390,10 +1391,158 @@ uint32_t Server::pair_split(const Launch& LA, const Queue& A, const Launch& LB, 
   return s;
 }
 
+// ------------------------------------------------------------------ k-way co-runs (NEXT-4, reading Q49)
+bool Server::job_curve(const Queue& Q, std::vector<uint32_t>* sms, std::vector<double>* ms) const {
+  const uint64_t lid = !Q.pending.empty() ? Q.pending.front() : (!Q.issued.empty() ? Q.issued.back() : 0);
+  if (!lid) return false;
+  auto it = launches_.find(lid);
+  if (it == launches_.end() || !curve_of(*it->second, sms, ms)) return false;
+  const double work = double(std::max<size_t>(1, Q.issued.size() + Q.pending.size()));
+  for (double& v : *ms) v *= work;
+  return true;
+}
+
+// Contiguous ranges in `qids` order (the first queue on the low ranks).  Queues
+// that only shrink are written first, so SMs are given up before they are
+// granted; growing queues get top-ups for their running launch.
+void Server::apply_shares(const std::vector<uint32_t>& qids, const std::vector<uint32_t>& shares) {
+  std::string err;
+  const double t0 = now_us();
+  std::vector<uint32_t> lo(qids.size()), hi(qids.size());
+  uint32_t at = 0;
+  for (size_t i = 0; i < qids.size(); ++i) {
+    lo[i] = at;
+    hi[i] = at + shares[i] - 1;
+    at += shares[i];
+  }
+  hi.back() = uint32_t(n_sms_ - 1);
+  for (int pass = 0; pass < 2; ++pass) {
+    for (size_t i = 0; i < qids.size(); ++i) {
+      Queue& Q = *queues_[qids[i]];
+      const bool grows = lo[i] < Q.lo || hi[i] > Q.hi || !Q.active;
+      if ((pass == 0) == grows || (Q.lo == lo[i] && Q.hi == hi[i])) continue;
+      const uint32_t old_lo = Q.lo, old_hi = Q.hi;
+      write_ctrl(Q, lo[i], hi[i], true, &err);
+      if (!Q.issued.empty()) {
+        Launch& R = *launches_[grows ? Q.issued.back() : Q.issued.front()];
+        R.n_resizes += 1;
+        track_resize(R, Q.epoch, grows ? 2 : 1, t0);
+      }
+      if (grows) grow_running(Q, old_lo, old_hi, &err);
+    }
+  }
+  if (qids.size() == 2) {   // the pair's re-split (resplit) keeps each on its side
+    queues_[qids[0]]->low_side = true;
+    queues_[qids[1]]->low_side = false;
+  }
+}
+
+// A third co-runner (the selection "examines other kernels in the
+// queue"): the head of the waiting queue joins a co-running group if the group
+// keeps at most one memory-intensive job (Q37) and the fluid model predicts a
+// gain against running it after the group (slate_kway_admit).
+bool Server::try_admit_kway() {
+  if (waiting_.empty() || active_.size() < 2 || active_.size() >= max_corun_) return false;
+  std::vector<std::vector<uint32_t>> sms;
+  std::vector<std::vector<double>> ms;
+  std::vector<uint32_t> cats, shares_cur;
+  for (uint32_t qid : active_) {
+    const Queue& Q = *queues_[qid];
+    if (!Q.auto_split || Q.explicit_range || Q.issued.empty()) return false;
+    std::vector<uint32_t> s;
+    std::vector<double> t;
+    if (!job_curve(Q, &s, &t)) return false;
+    const int c = category_of(*launches_[Q.issued.back()]);
+    if (c < 0) return false;
+    sms.push_back(s);
+    ms.push_back(t);
+    cats.push_back(uint32_t(c));
+    shares_cur.push_back(Q.hi - Q.lo + 1);
+  }
+  const uint32_t cand = waiting_.front();
+  Queue& C = *queues_[cand];
+  if (C.pending.empty()) return false;
+  const Launch& H = *launches_[C.pending.front()];
+  if (H.desc.placement == SLATE_PLACE_SOLO) return false;
+  const int cc = category_of(H);
+  std::vector<uint32_t> s;
+  std::vector<double> t;
+  if (cc < 0 || !job_curve(C, &s, &t)) return false;
+  sms.push_back(s);
+  ms.push_back(t);
+  cats.push_back(uint32_t(cc));
+  std::vector<const uint32_t*> sp;
+  std::vector<const double*> mp;
+  std::vector<uint32_t> np;
+  for (size_t i = 0; i < sms.size(); ++i) {
+    sp.push_back(sms[i].data());
+    mp.push_back(ms[i].data());
+    np.push_back(uint32_t(sms[i].size()));
+  }
+  std::vector<uint32_t> shares(sms.size());
+  double g = 0;
+  const int admit = slate_kway_admit(sp.data(), mp.data(), np.data(), cats.data(), uint32_t(active_.size()),
+                                     shares_cur.data(), uint32_t(n_sms_), 2, min_gain_, shares.data(), &g);
+  if (std::getenv("SLATE_DEBUG"))
+    fprintf(stderr, "[slate] k-way: candidate queue %u (cat %d) into a group of %zu: gain %.3f -> %s\n", cand, cc,
+            active_.size(), g, admit ? "admit" : "wait");
+  if (!admit) return false;
+  waiting_.erase(std::find(waiting_.begin(), waiting_.end(), cand));
+  bypassed_.erase(cand);
+  std::vector<uint32_t> group(active_.begin(), active_.end());
+  group.push_back(cand);
+  apply_shares(group, shares);
+  C.active = true;
+  C.explicit_range = false;
+  C.auto_split = true;
+  active_.push_back(cand);
+  std::string err;
+  while (!C.pending.empty()) {
+    Launch& L = *launches_[C.pending.front()];
+    C.pending.pop_front();
+    batch_more_ = !C.pending.empty();
+    if (issue(L, C, &err) != SLATE_OK) fail_launch(L, int(cudaErrorLaunchFailure));
+  }
+  batch_more_ = false;
+  close_batch(C, nullptr);
+  return true;
+}
+
 // A co-running pair on the selector's split: as launches arrive the jobs
 // grow, so the split is re-taken from the job curves; a change of >= 6 SMs
 // resizes both queues (shrink one, grow the other).
 void Server::resplit() {
+  if (active_.size() > 2) {   // a k-way group: re-take the shares from the job curves (NEXT-4)
+    std::vector<std::vector<uint32_t>> sms;
+    std::vector<std::vector<double>> ms;
+    std::vector<uint32_t> cur;
+    for (uint32_t qid : active_) {
+      const Queue& Q = *queues_[qid];
+      if (!Q.auto_split || Q.explicit_range) return;
+      std::vector<uint32_t> s;
+      std::vector<double> t;
+      if (!job_curve(Q, &s, &t)) return;
+      sms.push_back(s);
+      ms.push_back(t);
+      cur.push_back(Q.hi - Q.lo + 1);
+    }
+    std::vector<const uint32_t*> sp;
+    std::vector<const double*> mp;
+    std::vector<uint32_t> np;
+    for (size_t i = 0; i < sms.size(); ++i) {
+      sp.push_back(sms[i].data());
+      mp.push_back(ms[i].data());
+      np.push_back(uint32_t(sms[i].size()));
+    }
+    std::vector<uint32_t> shares(sms.size());
+    if (slate_choose_split_k(sp.data(), mp.data(), np.data(), uint32_t(sms.size()), uint32_t(n_sms_), 2,
+                             shares.data()) <= 0)
+      return;
+    bool big = false;
+    for (size_t i = 0; i < shares.size(); ++i) big = big || (shares[i] > cur[i] ? shares[i] - cur[i] : cur[i] - shares[i]) >= 6;
+    if (big) apply_shares(active_, shares);
+    return;
+  }
   if (active_.size() != 2) return;
   Queue& A = *queues_[active_[0]];
   Queue& B = *queues_[active_[1]];
@@ -1460,7 +1609,10 @@ void Server::schedule() {
       close_batch(Q, nullptr);
       continue;
     }
-    if (active_.size() >= 2) break;
+    if (active_.size() >= 2) {   // a co-running group: a k-way admission (NEXT-4), or wait
+      if (!try_admit_kway()) break;
+      continue;
+    }
     Queue& A = *queues_[active_[0]];
     if (A.explicit_range) break;
     // the active kernel: the last launch issued on A (or pending on it)
@@ -1543,11 +1695,44 @@ void Server::schedule() {
 // the queue has nothing left: its SMs go to the co-runner
 void Server::release(Queue& Q) {
   std::string err;
+  const bool kway = active_.size() > 2;
   Q.active = false;
   Q.explicit_range = false;
   Q.auto_split = false;
-  for (uint32_t other : active_) queues_[other]->auto_split = false;
   active_.erase(std::remove(active_.begin(), active_.end(), Q.id), active_.end());
+  if (kway) {   // a k-way group loses a member: the others share its SMs, re-split from the job curves
+    bool all_auto = true;
+    for (uint32_t other : active_) all_auto = all_auto && queues_[other]->auto_split && !queues_[other]->explicit_range;
+    if (all_auto) {
+      std::vector<std::vector<uint32_t>> sms;
+      std::vector<std::vector<double>> ms;
+      bool ok = true;
+      for (uint32_t other : active_) {
+        std::vector<uint32_t> s;
+        std::vector<double> t;
+        ok = ok && job_curve(*queues_[other], &s, &t);
+        sms.push_back(s);
+        ms.push_back(t);
+      }
+      std::vector<uint32_t> shares(active_.size(), uint32_t(n_sms_) / uint32_t(active_.size()));
+      if (ok) {
+        std::vector<const uint32_t*> sp;
+        std::vector<const double*> mp;
+        std::vector<uint32_t> np;
+        for (size_t i = 0; i < sms.size(); ++i) {
+          sp.push_back(sms[i].data());
+          mp.push_back(ms[i].data());
+          np.push_back(uint32_t(sms[i].size()));
+        }
+        slate_choose_split_k(sp.data(), mp.data(), np.data(), uint32_t(sms.size()), uint32_t(n_sms_), 2,
+                             shares.data());
+      }
+      apply_shares(active_, shares);
+      schedule();
+      return;
+    }
+  }
+  for (uint32_t other : active_) queues_[other]->auto_split = false;
   if (active_.size() == 1) {
     // the survivor claims the released SMs, explicit placement or not
     Queue& A = *queues_[active_[0]];

@@ -149,6 +149,11 @@ class Server {
   bool curve_of(const Launch& L, std::vector<uint32_t>* sms, std::vector<double>* ms) const;
   uint32_t pair_split(const Launch& LA, const Queue& A, const Launch& LB, const Queue& B, int catA, int catB,
                       double* gain) const;
+  // NEXT-4 (Q49): job curve of a queue's head kernel (x its queued launches),
+  // a third co-runner's admission, and contiguous SM shares for a group
+  bool job_curve(const Queue& Q, std::vector<uint32_t>* sms, std::vector<double>* ms) const;
+  bool try_admit_kway();
+  void apply_shares(const std::vector<uint32_t>& qids, const std::vector<uint32_t>& shares);
   void resplit();
   void poll_once();
   void poller_main();
@@ -220,6 +225,7 @@ class Server {
   uint32_t policy_ = SLATE_POLICY_HYBRID;
   double min_gain_ = 1.05;
   uint32_t split_objective_ = SLATE_SPLIT_ANTT;   // reading Q41
+  uint32_t max_corun_ = 3;                         // SLATE_MAX_CORUN: co-runners per group (NEXT-4, Q49)
   double split_slack_ = 0.05;
 
   mutable std::mutex mu_;

@@ -180,6 +180,9 @@ _lib.slate_corun_makespan_k.restype = c_f64
 _lib.slate_corun_makespan_k.argtypes = [ctypes.c_void_p, ctypes.c_void_p, _P(c_u32), c_u32, _P(c_u32)]
 _lib.slate_choose_split_k.restype = c_f64
 _lib.slate_choose_split_k.argtypes = [ctypes.c_void_p, ctypes.c_void_p, _P(c_u32), c_u32, c_u32, c_u32, _P(c_u32)]
+_lib.slate_kway_admit.restype = ctypes.c_int
+_lib.slate_kway_admit.argtypes = [ctypes.c_void_p, ctypes.c_void_p, _P(c_u32), _P(c_u32), c_u32, _P(c_u32), c_u32, c_u32,
+                                  c_f64, _P(c_u32), _P(c_f64)]
 _lib.slate_choose_iters.restype = c_u32
 _lib.slate_choose_iters.argtypes = [c_f64, c_u32, c_u32, c_u32, c_u32, c_f64]
 _lib.slate_choose_split_obj.restype = c_u32
@@ -206,7 +209,7 @@ EXPORTED = ["slate_attach", "slate_detach", "slate_get_info", "slate_share_buffe
             "slate_choose_split", "slate_serve", "slate_kind_geometry", "slate_saturation_sms",
             "slate_fluid_corun", "slate_set_policy", "slate_launch_n", "slate_launch_many", "slate_choose_iters",
             "slate_register_source", "slate_transform_source", "slate_corun_makespan_k", "slate_choose_split_k",
-            "slate_rtc_stats", "slate_choose_split_obj", "slate_fluid_corun_obj", "slate_set_split_objective", "slate_launch_fused"]
+            "slate_rtc_stats", "slate_choose_split_obj", "slate_fluid_corun_obj", "slate_set_split_objective", "slate_launch_fused", "slate_kway_admit"]
 DAEMON = os.path.join(_PKG, "bin", "slated")
 
 
@@ -429,6 +432,16 @@ def launch_fused(sa, ka, args_a, grid_a, sb, kb, args_b, grid_b, sm_b, coverage_
     if st < 0:
         raise SlateError(st, "slate_launch_fused: " + _lib.slate_last_error(sa._h).decode())
     return la.value, lb.value
+
+
+def kway_admit(curves, cats, shares_cur, n_sms, step=2, min_gain=1.05):
+    keep, sms, ms, npts = _curves_k(curves)
+    out = (c_u32 * len(curves))()
+    g = c_f64()
+    r = _lib.slate_kway_admit(ctypes.cast(sms, ctypes.c_void_p), ctypes.cast(ms, ctypes.c_void_p), npts,
+                              (c_u32 * len(cats))(*cats), len(shares_cur), (c_u32 * len(shares_cur))(*shares_cur),
+                              n_sms, step, min_gain, out, ctypes.byref(g))
+    return bool(r), list(out), g.value
 
 
 def transform_source(source, name, threads=256, smem=0, block=None):

@@ -177,3 +177,21 @@ def test_k_way_split_matches_oracle(S):
         assert s_c == s_o and abs(t_c - t_o) < 1e-9 * t_o
         shares = s_o
         assert abs(S.corun_makespan_k(curves, shares) - OS.corun_makespan_k(curves, shares)) < 1e-9 * t_o
+
+
+def test_kway_admit_matches_oracle(S):
+    """NEXT-4 (Q49): slate_kway_admit == oracle selector.kway_admit on random groups."""
+    rng = random.Random(49)
+    pts = [148, 111, 74, 49, 37, 18]
+    for _ in range(60):
+        curves, cats = [], []
+        for _ in range(3):
+            knee = rng.uniform(10, 148)
+            curves.append({s: rng.uniform(0.2, 3) * max(1.0, knee / s) for s in pts})
+            cats.append(rng.choice([2, 2, 3, 4]))
+        a = rng.randrange(2, 147, 2)
+        r1 = S.kway_admit(curves, cats, [a, 148 - a], 148, 2)
+        r2 = OS.kway_admit(curves, cats, [a, 148 - a], 148, 2)
+        assert r1[0] == r2[0]
+        if r2[1] is not None:
+            assert abs(r1[2] - r2[2]) <= 1e-9 * r2[2]

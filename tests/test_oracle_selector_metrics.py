@@ -215,3 +215,28 @@ def test_k_way_saturating_jobs_overlap_fully():
     shares, t = S.choose_split_k([sat, sat, sat], n, step=4)
     assert shares == [16, 16, 16] and abs(t - 1.0) < 1e-9
     assert S.corun_makespan_k([sat] * 3, [8, 20, 20]) > 1.0 + 1e-9
+
+
+def test_kway_admission_reading_q49():
+    """Closed forms on linear and saturating curves.  Work-conserving (linear)
+    compute jobs gain nothing from joining: whatever the shares, the chip does
+    the same total work (gain exactly 1), and a linear job joining a pair that
+    already gives its compute partner every SM past the memory job's knee gains
+    nothing either.  A small-grid compute job that saturates at 30 SMs joins a
+    (linear compute, memory) pair: the pair alone ends at 1.257 and C after it
+    at 1.757; joined on shares (80, 38, 30), by hand: A progresses on 80 SMs
+    until C ends (0.5), on 110 until B ends (1.0), then on all 148, so the
+    makespan is 1 + (148 - 80*0.5 - 110*0.5)/148 = 1.358 -- the best shares do
+    a little better, gain 1.3.  A second memory job never joins (Q37)."""
+    n = 148
+    lin = lambda w: {k: w * n / k for k in (18, 30, 37, 74, 110, 111, 148)}
+    sat = lambda w, knee: {k: w * max(1.0, knee / k) for k in (18, 30, 37, 74, 111, 148)}
+    ok, shares, g = S.kway_admit([lin(1.0), lin(1.0), lin(1.0)], [2, 2, 2], [74, 74], n, 2)
+    assert not ok and abs(g - 1.0) < 1e-9 and sum(shares) == n
+    ok, _, g = S.kway_admit([lin(1.0), sat(1.0, 37), lin(1.0)], [2, 4, 2], [110, 38], n, 2)
+    assert not ok and g < 1.01
+    assert abs(S.corun_makespan_k([lin(1.0), sat(1.0, 37), sat(0.5, 30)], [80, 38, 30]) - 1.358108) < 1e-5
+    ok, shares, g = S.kway_admit([lin(1.0), sat(1.0, 37), sat(0.5, 30)], [2, 4, 2], [110, 38], n, 2)
+    assert ok and g >= 1.29 and sum(shares) == n and all(x % 2 == 0 and x >= 2 for x in shares)
+    ok, _, _ = S.kway_admit([lin(1.0), sat(1.0, 37), sat(1.0, 37)], [2, 4, 3], [110, 38], n, 2)
+    assert not ok
