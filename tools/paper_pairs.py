@@ -9,7 +9,7 @@ few tens of ms solo on B200.  Measured here:
   * Tab II on B200: each app's solo profile (HBM GB/s, FP32 GFLOP/s) and its
     class under reading Q9 (the paper's Titan Xp labels beside it);
   * §V-B solo study (P:L295-305): original kernels vs Slate workers on all SMs;
-  * Fig 5 task-size sweep (P:L361-363): Slate solo at iters 1, 10 and auto;
+  * Fig 5 task-size sweep (P:L361-363): Slate solo at iters 1, 2, 4, 10, 20 and auto;
   * Fig 7: all 15 pairings under sequential CUDA, plain
     concurrent streams (the hardware leftover policy, in place of MPS),
     Slate with Tab I alone (TABLE) and Slate HYBRID (Q31), with G = T_seq /
@@ -201,8 +201,11 @@ def main():
                "curve": {str(s): round(t, 4) for s, t in zip(p["curve_sms"], p["curve_ms"])},
                "launches_per_job": len(A.launches) * A.reps}
         solo = {}
+        # Fig 5's task sizes: 1, 2, 4, 10, 20 blocks per task, and the automatic size (Q38)
         for label, iters, mode in (("cuda", 0, S.MODE_STANDALONE), ("slate_auto", 0, S.MODE_SLATE),
-                                   ("slate_iters1", 1, S.MODE_SLATE), ("slate_iters10", 10, S.MODE_SLATE)):
+                                   ("slate_iters1", 1, S.MODE_SLATE), ("slate_iters2", 2, S.MODE_SLATE),
+                                   ("slate_iters4", 4, S.MODE_SLATE), ("slate_iters10", 10, S.MODE_SLATE),
+                                   ("slate_iters20", 20, S.MODE_SLATE)):
             ks = A.register(sA, iters) if iters else kern[n][0]
             ts = []
             for _ in range(args.reps + 1):
@@ -214,6 +217,7 @@ def main():
             solo[label] = round(statistics.median(ts[1:]), 3)
         rec["job_ms"] = solo
         rec["slate_vs_cuda"] = round(solo["cuda"] / solo["slate_auto"], 4)
+        rec["best_slate_vs_cuda"] = round(solo["cuda"] / min(v for k, v in solo.items() if k != "cuda"), 4)
         out["apps"][n] = rec
         print(n, json.dumps(rec), flush=True)
 
