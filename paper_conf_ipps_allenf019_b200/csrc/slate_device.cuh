@@ -101,13 +101,17 @@ struct WorkerParams {
 };
 
 // programmatic dependent launch: wait for the previous kernel on the stream
-// (no-op for a normal launch).  The workers never trigger their dependents
-// early (griddepcontrol.launch_dependents): a CTA's exit is the trigger, so the
-// next grid's CTAs take SM slots only once every CTA of this grid has left --
-// the last main CTA waits for a top-up grid's blocks (leave_main), and an
-// early trigger let the next grid's waiting CTAs take the slots that top-up
-// needed (one C4 run stalled 320 ms that way).
+// (no-op for a normal launch).  A worker CTA triggers its dependents
+// (griddepcontrol.launch_dependents) once every task of the launch has been
+// handed out -- the fetch that returned the last task start, a drained queue,
+// or its retirement -- so the next grid of the batch is launched, and its CTAs
+// run their prologue, while this grid's last tasks finish (the next grid reads
+// no tenant data before griddepcontrol.wait).  Not earlier: round 1 triggered
+// at entry, and the next grid's waiting CTAs took the SM slots a top-up of the
+// running launch needed (one C4 run stalled 320 ms); once every task is handed
+// out a top-up has nothing left to run.
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // ------------------------------------------------------------------ decode (Lst2 (4))
 struct BlockWalk {
@@ -308,8 +312,10 @@ __device__ __forceinline__ uint32_t boundary(const P& p, uint32_t rank, uint64_t
   const bool inr = in_range(p, rank, c2);
   if (!inr && try_retire(tc)) {
     retired = true;
+    pdl_trigger();                                                      // this CTA fetches no more
   } else {
     g = atomicAdd(&tc->next, p.iters);                                  // Lst2 (2)
+    if (g + p.iters >= p.B) pdl_trigger();                              // every task is handed out
     if (g >= p.B) {                                                     // Q3: nothing to run
       atomicAdd(&tc->live_pending, ~0ull);                               // live -= 1 (RED)
       g = 0xffffffffu;
@@ -486,9 +492,12 @@ __device__ __forceinline__ void worker_body(const WorkerParams<typename Tn::Args
         if (spec_changed) asm volatile("fence.acq_rel.gpu;" ::: "memory");
         c = c2;
         const bool inr = in_range(p, rank, c);
-        if (!inr && try_retire(p.tc)) spec_retired = true;
-        else {
+        if (!inr && try_retire(p.tc)) {
+          spec_retired = true;
+          pdl_trigger();
+        } else {
           fut = atomicAdd(&p.tc->next, p.iters);                       // Lst2 (2), result used below
+          if (fut + p.iters >= p.B) pdl_trigger();
           log_task(p, fut, rank, c, !inr);
         }
         c2 = ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(p.ctrl));   // next boundary

@@ -109,7 +109,6 @@ struct Hdr {
   TaskMeta tmeta[kRpBufs];
   ChunkMeta cmeta[kSlots];
   uint32_t go, rank, retired;
-  int32_t nnz;                    // rp[n_rows]
   uint64_t ctrl;                  // the resize word last acted on (task warp)
 };
 static_assert(sizeof(Hdr) <= kHdrBytes, "header");
@@ -264,7 +263,6 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     uint64_t c = 0;
     H.rank = r;
     H.retired = 0;
-    H.nnz = __ldg(reinterpret_cast<const int*>(a.rowptr) + a.n_rows);
     H.go = prologue(p, r, c) ? 1u : 0u;
     H.ctrl = c;
   }
@@ -274,7 +272,8 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     return;
   }
   pdl_wait();   // a PDL launch: the previous kernel on the stream has completed from here on
-  const int nnz = H.nnz;
+  // tenant data only after the wait (the previous launch may have written it)
+  const int nnz = __ldg(reinterpret_cast<const int*>(a.rowptr) + a.n_rows);
 
   if (warp == kTaskWarp) {
     // ===================== task warp: the slate task protocol + row-pointer slices =====================
@@ -294,8 +293,10 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       const bool inr = in_range(p, rank, c);
       if (!inr && try_retire(p.tc)) {
         next_ret = true;
+        pdl_trigger();                                                 // this CTA fetches no more
       } else {
         g_next = atomicAdd(&p.tc->next, p.iters);                     // Lst2 (2)
+        if (g_next + p.iters >= p.B) pdl_trigger();                   // every task is handed out
         log_task(p, g_next, rank, c, !inr);
       }
       c_pre = ld_acquire_u64(p.ctrl);
@@ -326,9 +327,12 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
           chg = ctrl_epoch(c_pre) != ctrl_epoch(c);
           c = c_pre;
           const bool inr = in_range(p, rank, c);
-          if (!inr && try_retire(p.tc)) next_ret = true;
-          else {
+          if (!inr && try_retire(p.tc)) {
+            next_ret = true;
+            pdl_trigger();
+          } else {
             g_next = atomicAdd(&p.tc->next, p.iters);                 // Lst2 (2); result used next round
+            if (g_next + p.iters >= p.B) pdl_trigger();
             log_task(p, g_next, rank, c, !inr);
           }
           c_pre = ld_acquire_u64(p.ctrl);
