@@ -19,6 +19,7 @@ void fill(WorkerParams<typename Tn::Args>& p, const WorkerCommon& w, const void*
   p.is_topup = 0;
   p.gate_first = 0;
   p.ranklog = w.ranklog;
+  p.pdl_early = 0;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
 }
 

@@ -29,6 +29,7 @@ cudaError_t launch_worker_t(const WorkerCommon& w, const void* args, uint32_t gr
   p.is_topup = w.is_topup;
   p.gate_first = w.gate_first;
   p.ranklog = w.ranklog;
+  p.pdl_early = 0;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
   return launch_kernel(reinterpret_cast<const void*>(&slate_worker<Tn>), dim3(grid), dim3(Tn::kThreads), kargs,

@@ -96,6 +96,7 @@ struct WorkerCommon {
   uint32_t is_topup;     // 1: a top-up grid sharing a running launch's counter
   uint32_t gate_first;   // top-up of a launch with no start event: wait until the launch took its first task
   uint32_t ranklog = 0;  // cov holds 2B words: the rank log follows the coverage counts (SLATE_KFLAG_RANKLOG)
+  uint32_t pdl_early = 0; // the previous grid of the PDL chain is this kernel with the same args (pdl_early_ok kinds)
   bool pdl = false;      // launch with programmatic stream serialization (the previous op on the stream is
                          // the previous worker of the same batch; the worker waits in griddepcontrol.wait)
   const uint64_t* ctrl;
@@ -120,6 +121,11 @@ struct KindOps {
   uint32_t tile_m = 0;           // GEMM: output rows per original block
   uint32_t tile_n = 0;           // GEMM: output columns per original block
   bool pdl_ok = false;           // the worker calls griddepcontrol.wait before its first task
+  // the worker may read its inputs before griddepcontrol.wait when the previous
+  // grid is the same kernel with the same arguments and the output overlaps no
+  // input (it then writes only what this launch rewrites with the same values)
+  bool pdl_early_ok = false;
+  bool (*outputs_disjoint)(const void* args) = nullptr;
   bool topup_anytime = false;    // the worker's last main CTA waits for every block (leave_main), so a
                                  // running launch may get a top-up while later launches are queued
   cudaError_t (*launch_worker)(const WorkerCommon&, const void* args, uint32_t grid, cudaStream_t) = nullptr;

@@ -139,6 +139,7 @@ int Server::init(std::string* err) {
   peak_tc_ = env_double("SLATE_PEAK_TC_TFLOPS", 1590.0);
   standby_timeout_ns_ = uint32_t(env_double("SLATE_STANDBY_TIMEOUT_US", 200.0) * 1000.0);
   keep_finished_ = size_t(std::max(16.0, env_double("SLATE_KEEP_FINISHED", 65536.0)));
+  pdl_early_enabled_ = env_double("SLATE_PDL_EARLY", 1.0) != 0.0;
   watchdog_us_ = env_double("SLATE_WATCHDOG_S", 120.0) * 1e6;
   saturation_frac_ = env_double("SLATE_SATURATION_FRAC", 0.95);   // reading Q29 (1.0: no cap)
   if (const char* pol = std::getenv("SLATE_POLICY")) {              // reading Q31
@@ -884,6 +885,11 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
     w.ops = ops;
     // PDL: the previous op on the stream is the previous worker of this batch
     w.pdl = in_batch && Q.last_op_kernel && ops->pdl_ok && pdl_enabled_;
+    if (w.pdl && ops->pdl_early_ok && pdl_early_enabled_) {   // the previous grid: the same kernel, the same args?
+      const Launch& P = *launches_[Q.open_batch.back()];
+      w.pdl_early = P.k == L.k && P.args == L.args && P.slot >= 0 &&
+                    (!ops->outputs_disjoint || ops->outputs_disjoint(L.args.data())) ? 1u : 0u;
+    }
     const bool full = Q.lo == 0 && Q.hi == uint32_t(n_sms_ - 1);
     CK(ops->launch_worker(w, L.args.data(), worker_grid(L.k->occ, L.B, L.iters, full), Q.stream));
     Q.last_op_kernel = ops->pdl_ok;

@@ -238,7 +238,8 @@ class Server {
   // dropped in bulk (retire_finished), so a long-running slated stays bounded
   std::deque<uint64_t> finished_;
   size_t keep_finished_ = 65536;   // SLATE_KEEP_FINISHED (tests use a small window)
-  double watchdog_us_ = 120e6;     // SLATE_WATCHDOG_S: a launch issued longer ago is reported (0: off)
+  double watchdog_us_ = 120e6;
+  bool pdl_early_enabled_ = true;  // SLATE_PDL_EARLY=0: every worker waits for the previous grid first     // SLATE_WATCHDOG_S: a launch issued longer ago is reported (0: off)
   void retire_finished();
   std::deque<uint32_t> waiting_;     // queues waiting for SMs, FIFO
   std::map<uint32_t, uint32_t> bypassed_;

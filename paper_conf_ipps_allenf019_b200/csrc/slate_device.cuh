@@ -93,6 +93,8 @@ struct WorkerParams {
   uint32_t is_topup;              // 1: a top-up grid (grow) sharing a running launch's TaskCtl
   uint32_t gate_first;            // top-up: join only once the launch has taken its first task
   uint32_t ranklog;               // 1: cov holds 2B words, cov[B + b] = the rank log entry of block b
+  uint32_t pdl_early;             // 1: the previous grid (PDL) is this kernel with these args: inputs may be read
+                                  // before griddepcontrol.wait (kinds that allow it, e.g. SpMV's producer warps)
   const uint64_t* ctrl;           // the queue's resize word
   TaskCtl* tc;
   HostMirror* mirror;             // device alias of the pinned mirror (may be null)

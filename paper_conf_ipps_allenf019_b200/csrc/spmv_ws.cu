@@ -81,7 +81,10 @@ constexpr int kSlotBytes = 2 * kCap * 4;         // col + val
 #endif
 constexpr int kRpBufs = SLATE_SPMV_RPBUFS;       // row-pointer slices: the task warp runs <= kRpBufs-1 tasks ahead
 constexpr int kRpInts = 32 * kMaxTaskBlocks + 4; // rp slice of one task (rounded to 16 B)
-constexpr int kWinBufs = 2;
+#ifndef SLATE_SPMV_WINBUFS
+#define SLATE_SPMV_WINBUFS 2
+#endif
+constexpr int kWinBufs = SLATE_SPMV_WINBUFS;
 constexpr int kWin = SLATE_SPMV_WIN;              // x window per task (floats)
 constexpr int kHdrBytes = 1024;
 constexpr int kSmemBytes = kHdrBytes + kSlots * kSlotBytes + kRpBufs * kRpInts * 4 + kWinBufs * kWin * 4;
@@ -271,8 +274,13 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
     if (threadIdx.x == 0) leave_main(p);
     return;
   }
-  pdl_wait();   // a PDL launch: the previous kernel on the stream has completed from here on
-  // tenant data only after the wait (the previous launch may have written it)
+  // a PDL launch: the previous kernel on the stream has completed after this
+  // wait.  When that kernel is this one with the same arguments (pdl_early:
+  // y overlaps no input, and the previous launch writes y only), the task and
+  // chunk warps start on the inputs at once -- the row-pointer slices, the x
+  // window and the first chunks are in flight while the previous launch
+  // finishes -- and only the compute warps, which write y, wait.
+  if (!p.pdl_early || (warp != kTaskWarp && warp != kChunkWarp)) pdl_wait();
   const int nnz = __ldg(reinterpret_cast<const int*>(a.rowptr) + a.n_rows);
 
   if (warp == kTaskWarp) {
@@ -543,6 +551,15 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
   }
 }
 
+// y = [y, y + 4 n_rows) against x and rowptr (col and val: a caller aliasing y
+// onto them writes its own matrix and is outside the kind's contract)
+static bool outputs_disjoint(const void* args) {
+  const slate_args_spmv* a = static_cast<const slate_args_spmv*>(args);
+  auto apart = [](uint64_t p0, uint64_t n0, uint64_t p1, uint64_t n1) { return p0 + n0 <= p1 || p1 + n1 <= p0; };
+  const uint64_t ny = 4ull * a->n_rows;
+  return apart(a->y, ny, a->x, 4ull * a->n_cols) && apart(a->y, ny, a->rowptr, 4ull * (a->n_rows + 1ull));
+}
+
 static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32_t grid, cudaStream_t st) {
   WorkerParams<slate_args_spmv> p;
   std::memcpy(&p.args, args, sizeof(p.args));
@@ -553,6 +570,7 @@ static cudaError_t launch_worker(const WorkerCommon& w, const void* args, uint32
   p.is_topup = w.is_topup;
   p.gate_first = w.gate_first;
   p.ranklog = w.ranklog;
+  p.pdl_early = w.pdl_early;
   p.ctrl = w.ctrl; p.tc = w.tc; p.mirror = w.mirror; p.cov = w.cov; p.rank_of = w.rank_of;
   void* kargs[] = {&p};
   return launch_kernel(reinterpret_cast<const void*>(&spmv_worker), dim3(grid), dim3(kThreads), kargs, kSmemBytes, st,
@@ -585,6 +603,8 @@ KindOps spmv_ws_ops() {
   o.launch_standalone = &spmv::launch_standalone;
   o.topup_anytime = true;   // leave_main: the last main CTA waits for every block
   o.pdl_ok = true;          // griddepcontrol.wait before the first task
+  o.pdl_early_ok = true;    // producer warps may start before the wait (y written only, see spmv_worker)
+  o.outputs_disjoint = &spmv::outputs_disjoint;
   return o;
 }
 

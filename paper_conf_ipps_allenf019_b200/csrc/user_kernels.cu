@@ -160,7 +160,7 @@ bool transform_user_kernel(const char* src, const char* name, uint32_t bx, uint3
   g += "  p.bound_lo = c.bound_lo; p.bound_hi = c.bound_hi; p.n_ranks = c.n_ranks;\n";
   g += "  p.standby_timeout_ns = c.standby_timeout_ns; p.base_epoch = c.base_epoch; p.is_topup = c.is_topup;\n";
   g += "  p.gate_first = c.gate_first; p.ranklog = c.ranklog; p.ctrl = c.ctrl; p.tc = c.tc; p.mirror = c.mirror;\n";
-  g += "  p.cov = c.cov; p.rank_of = c.rank_of;\n";
+  g += "  p.cov = c.cov; p.rank_of = c.rank_of; p.pdl_early = 0;\n";
   g += "  slate::worker_body<SlateUserTenant>(p);\n}\n";
   g += "// the original kernel K(B,T), launched with the " + BX + " x " + BY + " x " + BZ + " block\n";
   g += "extern \"C\" __global__ void __launch_bounds__(" + T +
