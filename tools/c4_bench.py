@@ -10,6 +10,8 @@ CUDA events (slate_query start/end, one clock for every client).
 """
 import argparse
 import json
+
+import numpy as np
 import os
 import signal
 import subprocess
@@ -216,7 +218,9 @@ def main():
                       "gain_vs_seq_cuda": round(seq_ms / mk, 4),
                       "stp_median": round(sorted(stps)[len(stps) // 2], 4), "makespans_ms": [round(x, 3) for x in spans],
                       "resize_us": {"n": len(resize), "p50": round(sorted(resize)[len(resize) // 2], 2) if resize else None,
-                                    "max": round(max(resize), 2) if resize else None}}))
+                                    "p99": round(float(np.percentile(resize, 99)), 2) if resize else None,
+                                    "max": round(max(resize), 2) if resize else None,
+                                    "over_50us": sum(1 for v in resize if v > 50.0)}}))
 
 
 if __name__ == "__main__":
