@@ -2125,9 +2125,9 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
                       std::string* err) {
   // a private queue: its own stream and resize word; kBatch control blocks.
   // A measurement is kBatch launches back to back (programmatic dependent
-  // launch, no events between them), as a job's launches run: the per-launch
-  // time is the batch's span over kBatch.
-  constexpr int kBatch = 8;
+  // launch, no events between them, the early start where the kind allows it),
+  // as a job's launches run: the per-launch time is the batch's span over kBatch.
+  constexpr int kBatch = 16;
   std::vector<int> slots;
   uint64_t* ctrl;
   {
@@ -2169,6 +2169,8 @@ int Server::run_timed(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     for (int i = 0; i < kBatch; ++i) {
       w.tc = d_tc_ + slots[i];
       w.pdl = i > 0 && k.ops->pdl_ok && pdl_enabled_;
+      w.pdl_early = w.pdl && k.ops->pdl_early_ok && pdl_early_enabled_ &&
+                    (!k.ops->outputs_disjoint || k.ops->outputs_disjoint(d->args)) ? 1u : 0u;
       CK(k.ops->launch_worker(w, d->args, worker_grid(k.occ, B, w.iters, lo == 0 && hi == uint32_t(n_sms_ - 1)), st));
     }
     CK(cudaEventRecord(e1, st));
