@@ -188,8 +188,8 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
   for (int u = 0; u < U; ++u) {
     const uint32_t lr = (u * kComputeWarps + w) * kPassRows + (lane >> 2);
     const bool in = lr < nrows;
-    lo[u] = in ? rp[lr] : 0;
-    hi[u] = in ? rp[lr + 1] : 0;
+    lo[u] = in ? rp[lr] : 0;  // racecheck: mbarrier-ordered
+    hi[u] = in ? rp[lr + 1] : 0;  // racecheck: mbarrier-ordered
     longrow |= ((lo[u] >> 2) + 4) * 4 < hi[u];   // segments past the lane's first
   }
   if (m.mode == 0) {
@@ -402,8 +402,8 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       }
 #pragma unroll
       for (int k = 0; k < kV; ++k)
-        if (lane + 32 * k < n4) reinterpret_cast<int4*>(rps)[lane + 32 * k] = v[k];
-      if (tail) rps[n4 * 4 + lane] = vt;
+        if (lane + 32 * k < n4) reinterpret_cast<int4*>(rps)[lane + 32 * k] = v[k];  // racecheck: mbarrier-ordered
+      if (tail) rps[n4 * 4 + lane] = vt;  // racecheck: mbarrier-ordered
       __syncwarp();
       prev_valid = true;
       prev_b = b;
