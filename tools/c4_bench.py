@@ -77,7 +77,12 @@ def client(endpoint, kind, steps, go_path, device=0):
         while not os.path.exists("%s.%d" % (go_path, step)):
             time.sleep(0.0005)
         t_go = time.time()
-        ids = [s.launch(kid, args, grid, placement=S.PLACE_AUTO) for _ in range(JOBS[kind])]
+        # the job in one call (slate_launch_n: the selector sees the whole job, its
+        # launches go out as one batch; C4_PER_LAUNCH=1: one call per launch)
+        if os.environ.get("C4_PER_LAUNCH"):
+            ids = [s.launch(kid, args, grid, placement=S.PLACE_AUTO) for _ in range(JOBS[kind])]
+        else:
+            ids = s.launch_n(kid, args, grid, JOBS[kind], placement=S.PLACE_AUTO)
         t_sub = time.time()
         s.sync(0)
         qs = [s.query(i) for i in ids]
