@@ -576,8 +576,12 @@ struct BlackScholesShort : BlackScholes {
   // options 54 -> 46 us at 4 blocks per task).
   static constexpr bool kHasTask = true;
   static constexpr uint32_t kPipelineMaxScen = 4;
-  static constexpr int kSmem = 2 * 3 * 256 * 16;   // two cp.async stages
+#ifndef SLATE_BS_STAGES
+#define SLATE_BS_STAGES 4
+#endif
+  static constexpr int kStages = SLATE_BS_STAGES;    // blocks staged ahead + the one being priced
   static constexpr int kStageBytes = 3 * 256 * 16;   // S, X, T float4 of 256 threads
+  static constexpr int kSmem = kStages * kStageBytes;
   __device__ __forceinline__ static void stage_in(const Args& a, uint64_t v, char* stage) {
     const char* src[3] = {reinterpret_cast<const char*>(a.S), reinterpret_cast<const char*>(a.X),
                           reinterpret_cast<const char*>(a.T)};
@@ -588,29 +592,42 @@ struct BlackScholesShort : BlackScholes {
                    : "memory");
     asm volatile("cp.async.commit_group;" ::: "memory");
   }
+  // wait until at most `pending` of this thread's cp.async groups are still in flight
+  __device__ __forceinline__ static void wait_pending(int pending) {
+    switch (pending) {
+      case 0: asm volatile("cp.async.wait_group 0;" ::: "memory"); break;
+      case 1: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
+      case 2: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
+      default: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
+    }
+  }
+  // A task's blocks through a kStages-deep ring of cp.async stages: block i is
+  // priced while blocks i+1 .. i+kStages-1 are in flight (round 2: a 2-stage
+  // ring kept ~half the bytes in flight of the original kernel's 8 CTAs/SM).
   __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char* smem) {
+    static_assert(kStages >= 2 && kStages <= 4, "wait_pending covers up to 3 groups in flight");
     const uint64_t n_full = a.n / 1024;            // blocks with 1024 options (no ragged tail)
     if (g + n > n_full) {
       for (uint32_t i = 0; i < n; ++i) cta_block(a, g + i, 0, 0, smem);
       return;
     }
     const float* sig = reinterpret_cast<const float*>(a.sigmas);
-    uint64_t v = uint64_t(g) * 256 + threadIdx.x;
-    stage_in(a, v, smem);
+    const uint64_t v0 = uint64_t(g) * 256 + threadIdx.x;
+    uint32_t issued = 0;
+    for (; issued < n && issued < uint32_t(kStages - 1); ++issued)
+      stage_in(a, v0 + uint64_t(issued) * 256, smem + (issued % kStages) * kStageBytes);
     for (uint32_t i = 0; i < n; ++i) {
-      const uint64_t cur = v;
-      if (i + 1 < n) {
-        v += 256;
-        stage_in(a, v, smem + ((i + 1) & 1) * kStageBytes);    // next block in flight
-        asm volatile("cp.async.wait_group 1;" ::: "memory");
-      } else {
-        asm volatile("cp.async.wait_group 0;" ::: "memory");
+      if (issued < n) {
+        stage_in(a, v0 + uint64_t(issued) * 256, smem + (issued % kStages) * kStageBytes);   // keep the ring full
+        ++issued;
       }
-      const float4* st = reinterpret_cast<const float4*>(smem + (i & 1) * kStageBytes);
+      wait_pending(int(issued - 1 - i));             // block i's group has landed
+      const float4* st = reinterpret_cast<const float4*>(smem + (i % kStages) * kStageBytes);
       const float4 s4 = st[threadIdx.x], x4 = st[256 + threadIdx.x], t4 = st[512 + threadIdx.x];
       float S[4] = {s4.x, s4.y, s4.z, s4.w}, X[4] = {x4.x, x4.y, x4.z, x4.w}, T[4] = {t4.x, t4.y, t4.z, t4.w};
       float c[4], p[4];
       price4(S, X, T, a.r, sig, a.n_scen, c, p);
+      const uint64_t cur = v0 + uint64_t(i) * 256;
       __stcs(reinterpret_cast<float4*>(a.call) + cur, make_float4(c[0], c[1], c[2], c[3]));
       __stcs(reinterpret_cast<float4*>(a.put) + cur, make_float4(p[0], p[1], p[2], p[3]));
     }
