@@ -574,11 +574,9 @@ struct BlackScholesShort : BlackScholes {
   // needed.  A task reaching the ragged last block takes the per-block path.
   // Each option's arithmetic is price<4>'s (measured: a P = 1 launch of 2^23
   // options 54 -> 46 us at 4 blocks per task).
+  static constexpr bool kHasTask = true;
   static constexpr uint32_t kPipelineMaxScen = 4;
-#ifndef SLATE_BS_STAGES
-#define SLATE_BS_STAGES 3   // 36 KB: with the worker's static shared memory under the 48-KB default limit
-#endif
-  static constexpr int kStages = SLATE_BS_STAGES;    // blocks staged ahead + the one being priced
+  static constexpr int kSmem = 2 * 3 * 256 * 16;   // two cp.async stages
   static constexpr int kStageBytes = 3 * 256 * 16;   // S, X, T float4 of 256 threads
   __device__ __forceinline__ static void stage_in(const Args& a, uint64_t v, char* stage) {
     const char* src[3] = {reinterpret_cast<const char*>(a.S), reinterpret_cast<const char*>(a.X),
@@ -590,71 +588,31 @@ struct BlackScholesShort : BlackScholes {
                    : "memory");
     asm volatile("cp.async.commit_group;" ::: "memory");
   }
-  // wait until at most `pending` of this thread's cp.async groups are still in flight
-  __device__ __forceinline__ static void wait_pending(int pending) {
-    switch (pending) {
-      case 0: asm volatile("cp.async.wait_group 0;" ::: "memory"); break;
-      case 1: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
-      case 2: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
-      default: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
-    }
-  }
-  // The blocks of this task and of the next one ([g2, g2+n2), fetched before
-  // this one runs: kLookahead) form one stream through a kStages-deep ring of
-  // cp.async stages: block i is priced while the next kStages-1 blocks are in
-  // flight, the next task's first blocks included, so neither the fetch nor
-  // the first loads of a task are exposed (round 2: 4 blocks per task exposed
-  // ~1 us of fill per task).  state (uniform over the CTA): [0] blocks of this
-  // task already staged by the previous call, [1] ring index of this task's
-  // first block.  A ragged task (the array's last, partial block) takes the
-  // per-block path and stages nothing ahead.
-  static constexpr bool kHasInit = true, kLookahead = true;
-  static constexpr int kSmemRing = kStages * kStageBytes;
-  static constexpr int kSmem = kSmemRing + 16;
-  __device__ __forceinline__ static uint32_t* state(char* smem) { return reinterpret_cast<uint32_t*>(smem + kSmemRing); }
-  __device__ __forceinline__ static void cta_init(char* smem) {
-    if (threadIdx.x == 0) {
-      state(smem)[0] = 0;
-      state(smem)[1] = 0;
-    }
-  }
-  __device__ __forceinline__ static void cta_task2(const Args& a, uint32_t g, uint32_t n, uint32_t g2, uint32_t n2,
-                                                   char* smem) {
-    static_assert(kStages >= 2 && kStages <= 4, "wait_pending covers up to 3 groups in flight");
-    const uint32_t pre = state(smem)[0], seq = state(smem)[1];
-    __syncthreads();                               // every thread has read the state before it is rewritten
+  __device__ __forceinline__ static void cta_task(const Args& a, uint32_t g, uint32_t n, char* smem) {
     const uint64_t n_full = a.n / 1024;            // blocks with 1024 options (no ragged tail)
-    if (g + n > n_full) {                          // never staged ahead (see below): pre == 0
+    if (g + n > n_full) {
       for (uint32_t i = 0; i < n; ++i) cta_block(a, g + i, 0, 0, smem);
-      if (threadIdx.x == 0) state(smem)[0] = 0;
       return;
     }
-    const bool next_ok = n2 && uint64_t(g2) + n2 <= n_full;
-    const uint32_t total = n + (next_ok ? n2 : 0u);
-    auto blk = [&](uint32_t k) { return k < n ? g + k : g2 + (k - n); };
-    auto stage = [&](uint32_t k) { return smem + ((seq + k) % kStages) * kStageBytes; };
     const float* sig = reinterpret_cast<const float*>(a.sigmas);
-    uint32_t issued = pre;
-    for (; issued < total && issued < uint32_t(kStages - 1); ++issued)
-      stage_in(a, uint64_t(blk(issued)) * 256 + threadIdx.x, stage(issued));
+    uint64_t v = uint64_t(g) * 256 + threadIdx.x;
+    stage_in(a, v, smem);
     for (uint32_t i = 0; i < n; ++i) {
-      if (issued < total && issued < i + kStages) {   // keep the ring full
-        stage_in(a, uint64_t(blk(issued)) * 256 + threadIdx.x, stage(issued));
-        ++issued;
+      const uint64_t cur = v;
+      if (i + 1 < n) {
+        v += 256;
+        stage_in(a, v, smem + ((i + 1) & 1) * kStageBytes);    // next block in flight
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
       }
-      wait_pending(int(issued - 1 - i));             // block i's group has landed
-      const float4* st = reinterpret_cast<const float4*>(stage(i));
+      const float4* st = reinterpret_cast<const float4*>(smem + (i & 1) * kStageBytes);
       const float4 s4 = st[threadIdx.x], x4 = st[256 + threadIdx.x], t4 = st[512 + threadIdx.x];
       float S[4] = {s4.x, s4.y, s4.z, s4.w}, X[4] = {x4.x, x4.y, x4.z, x4.w}, T[4] = {t4.x, t4.y, t4.z, t4.w};
       float c[4], p[4];
       price4(S, X, T, a.r, sig, a.n_scen, c, p);
-      const uint64_t cur = uint64_t(g + i) * 256 + threadIdx.x;
       __stcs(reinterpret_cast<float4*>(a.call) + cur, make_float4(c[0], c[1], c[2], c[3]));
       __stcs(reinterpret_cast<float4*>(a.put) + cur, make_float4(p[0], p[1], p[2], p[3]));
-    }
-    if (threadIdx.x == 0) {
-      state(smem)[0] = issued > n ? issued - n : 0u;
-      state(smem)[1] = (seq + n) % kStages;
     }
   }
 };
