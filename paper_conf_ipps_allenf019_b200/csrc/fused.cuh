@@ -60,11 +60,16 @@ __device__ __forceinline__ void fused_join(const P& p, uint32_t rank, uint64_t c
     publish_mirror(&tc->join_word, &p.mirror->join, mirror_pack(e, globaltimer()));   // grow observed under e
 }
 
-template <class Tn, class P>
+// kRegs: the register budget of the pair's kernel (the fused task body needs >= 64)
+template <class Tn, int kRegs, class P>
 __device__ __forceinline__ void fused_run_task(const P& p, uint32_t g, char* smem) {
   const uint32_t n = min(p.iters, p.B - g);
-  if constexpr (Tn::kHasTask) {
-    Tn::cta_task(p.args, g, n, smem);
+  constexpr bool kFusedBody = Tn::kHasFusedTask && kRegs >= 64;
+  if constexpr (kFusedBody || Tn::kHasTask) {
+    if constexpr (kFusedBody)
+      Tn::cta_task_fused(p.args, g, n, smem);
+    else
+      Tn::cta_task(p.args, g, n, smem);
     if (p.cov && threadIdx.x == 0)
       for (uint32_t i = 0; i < n; ++i) atomicAdd(&p.cov[g + i], 1u);
   } else {
@@ -238,8 +243,10 @@ __device__ __forceinline__ void fused_body(const FusedParams<TA, TB>& fp) {
     __syncthreads();
     const uint32_t ten = s_ten, g = s_g;
     if (ten == 2) break;
-    if (ten == 0) fused_run_task<TA>(pa, g, dyn_smem);
-    else fused_run_task<TB>(pb, g, dyn_smem);
+    constexpr int kMinB = TA::kMinBlocks < TB::kMinBlocks ? TA::kMinBlocks : TB::kMinBlocks;
+    constexpr int kRegs = 65536 / (TA::kThreads * (kMinB > 0 ? kMinB : 1));
+    if (ten == 0) fused_run_task<TA, kRegs>(pa, g, dyn_smem);
+    else fused_run_task<TB, kRegs>(pb, g, dyn_smem);
     __syncthreads();                             // the task's blocks are done; s_ten / s_g may be rewritten
     if (threadIdx.x == 0) {
       if (ten == 0) {

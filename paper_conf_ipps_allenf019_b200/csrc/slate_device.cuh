@@ -22,6 +22,8 @@ namespace slate {
 struct TenantBase {
   static constexpr bool kHasInit = false;   // cta_init(smem): once per CTA before the first block
   static constexpr bool kHasTask = false;   // cta_task(args, g, n, smem): task [g, g+n) of a 1-D grid at once
+  static constexpr bool kHasFusedTask = false; // cta_task_fused(args, g, n, smem): the task body used inside a
+                                               // fused co-run kernel (at the pair's lower occupancy) instead
   static constexpr bool kLookahead = false; // cta_task2(args, g, n, g2, n2, smem): run task [g, g+n) of a
                                             // 1-D grid knowing the CTA's next task [g2, g2+n2) (n2 = 0: none)
   static constexpr uint32_t kMaxIters = 10; // cap of the automatic task size (P:L303 default 10)

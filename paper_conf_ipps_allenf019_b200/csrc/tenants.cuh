@@ -636,6 +636,87 @@ struct Stencil2D : TenantBase {
   __device__ __forceinline__ static float pt(float up, float down, float left, float right) {
     return __fmul_rn(0.25f, __fadd_rn(__fadd_rn(up, down), __fadd_rn(left, right)));
   }
+  // the 4 points of a lane: interior points 0.25 ((up + down) + (left + right)), boundary copied
+  __device__ __forceinline__ static float4 out4(float4 c, float4 u, float4 d, float left, float right, int j0, int w,
+                                                bool interior_row) {
+    float4 o = c;
+    if (interior_row) {
+      if (j0 > 0) o.x = pt(u.x, d.x, left, c.y);
+      o.y = pt(u.y, d.y, c.x, c.z);
+      o.z = pt(u.z, d.z, c.y, c.w);
+      if (j0 + 3 < w - 1) o.w = pt(u.w, d.w, c.z, right);
+    }
+    return o;
+  }
+  // Task body inside a fused co-run kernel (w a multiple of 4): two x-neighbouring
+  // blocks of a row band at once -- a lane's 4 columns in each, all six float4
+  // loads in flight together.  A fused pair runs at its lower occupancy (4 CTAs/SM
+  // with Black-Scholes), where this restores the stencil's bytes in flight; the
+  // stand-alone worker (8 CTAs/SM, 32 registers) keeps cta_block, which this body
+  // would spill (profiles/r2_kernels.md).  Every point is out4's, as in cta_block.
+  static constexpr bool kHasFusedTask = true;
+  __device__ __forceinline__ static void cta_task_fused(const Args& a, uint32_t g, uint32_t n, char* smem) {
+    const uint32_t gx = (a.w + 127) / 128;
+    uint32_t bx = g % gx, by = g / gx;
+    uint32_t k = 0;
+    while (k < n) {
+      if ((a.w & 3) == 0 && k + 1 < n && bx + 1 < gx) {
+        pair(a, bx, by);
+        k += 2;
+        bx += 2;
+      } else {
+        cta_block(a, bx, by, 0, smem);
+        k += 1;
+        bx += 1;
+      }
+      if (bx >= gx) {
+        bx -= gx;
+        ++by;
+      }
+    }
+  }
+  __device__ __forceinline__ static void pair(const Args& a, uint32_t bx, uint32_t by) {
+    const float* in = reinterpret_cast<const float*>(a.in);
+    float* out = reinterpret_cast<float*>(a.out);
+    const int lane = int(threadIdx.x & 31), r = int(threadIdx.x >> 5);
+    const int h = int(a.h), w = int(a.w);
+    const int i = int(by) * 8 + r, j0 = int(bx) * 128 + lane * 4, j1 = j0 + 128;
+    const bool row_in = i < h, interior_row = i > 0 && i < h - 1;
+    const bool in0 = row_in && j0 < w, in1 = row_in && j1 < w;
+    const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+    float4 c0 = z, u0 = z, d0 = z, c1 = z, u1 = z, d1 = z;
+    const uint64_t base = uint64_t(i) * w;
+    if (in0) {
+      c0 = __ldg(reinterpret_cast<const float4*>(in + base + j0));
+      if (interior_row) {
+        u0 = __ldg(reinterpret_cast<const float4*>(in + base - w + j0));
+        d0 = __ldg(reinterpret_cast<const float4*>(in + base + w + j0));
+      }
+    }
+    if (in1) {
+      c1 = __ldg(reinterpret_cast<const float4*>(in + base + j1));
+      if (interior_row) {
+        u1 = __ldg(reinterpret_cast<const float4*>(in + base - w + j1));
+        d1 = __ldg(reinterpret_cast<const float4*>(in + base + w + j1));
+      }
+    }
+    // neighbours: within a block from the adjacent lanes, across the two blocks
+    // from lane 31 / lane 0 of the other, at the outer edges by scalar loads
+    float left0 = __shfl_up_sync(0xffffffffu, c0.w, 1), right0 = __shfl_down_sync(0xffffffffu, c0.x, 1);
+    float left1 = __shfl_up_sync(0xffffffffu, c1.w, 1), right1 = __shfl_down_sync(0xffffffffu, c1.x, 1);
+    const float c0_last = __shfl_sync(0xffffffffu, c0.w, 31), c1_first = __shfl_sync(0xffffffffu, c1.x, 0);
+    if (!row_in) return;
+    if (lane == 0) {
+      if (j0 > 0) left0 = __ldg(in + base + j0 - 1);
+      left1 = c0_last;                                 // column j1 - 1 = the first block's last
+    }
+    if (lane == 31) {
+      right0 = c1_first;                               // column j0 + 4 = the second block's first (< w here)
+      if (in1 && j1 + 4 < w) right1 = __ldg(in + base + j1 + 4);
+    }
+    __stcs(reinterpret_cast<float4*>(out + base + j0), out4(c0, u0, d0, left0, right0, j0, w, interior_row));
+    if (in1) __stcs(reinterpret_cast<float4*>(out + base + j1), out4(c1, u1, d1, left1, right1, j1, w, interior_row));
+  }
   __device__ __forceinline__ static void cta_block(const Args& a, uint32_t bx, uint32_t by, uint32_t, char*) {
     const float* in = reinterpret_cast<const float*>(a.in);
     float* out = reinterpret_cast<float*>(a.out);
@@ -659,14 +740,7 @@ struct Stencil2D : TenantBase {
       if (!inside) return;
       if (lane == 0 && j0 > 0) left = __ldg(in + uint64_t(i) * w + j0 - 1);
       if ((lane == 31 || j0 + 4 >= w) && j0 + 4 < w) right = __ldg(in + uint64_t(i) * w + j0 + 4);
-      float4 o = c;
-      if (interior_row) {
-        if (j0 > 0) o.x = pt(u.x, d.x, left, c.y);
-        o.y = pt(u.y, d.y, c.x, c.z);
-        o.z = pt(u.z, d.z, c.y, c.w);
-        if (j0 + 3 < w - 1) o.w = pt(u.w, d.w, c.z, right);
-      }
-      __stcs(reinterpret_cast<float4*>(out + uint64_t(i) * w + j0), o);
+      __stcs(reinterpret_cast<float4*>(out + uint64_t(i) * w + j0), out4(c, u, d, left, right, j0, w, interior_row));
       return;
     }
     // scalar path (w not a multiple of 4): the same points one at a time

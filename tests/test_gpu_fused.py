@@ -91,10 +91,15 @@ def test_fused_c1_pair_matches_the_oracle():
     assert own_a and own_b and not (own_a & own_b)
 
 
-@pytest.mark.parametrize("pair", ["bs+stencil", "transpose+sgemm"])
+@pytest.mark.parametrize("pair", ["bs+stencil", "bs+stencil_ragged", "transpose+sgemm"])
 def test_fused_resize_storm_exactly_once(pair):
     if pair == "bs+stencil":
         ta, tb, ia, ib = make_bs(1 << 21, 503, n_scen=64), make_stencil(8192, 4096, 504), 1, 4
+    elif pair == "bs+stencil_ragged":
+        # the fused stencil body pairs x-neighbouring blocks: 33 blocks a row band
+        # (the last one ragged, w % 128 = 4) and 3 blocks a task, so pairs start at
+        # both parities and tasks straddle row bands; h % 8 = 1
+        ta, tb, ia, ib = make_bs(1 << 20, 509, n_scen=32), make_stencil(1001, 4100, 510), 1, 3
     else:
         ta, tb, ia, ib = make_transpose(4096, 4096, 505), make_sgemm(512, 512, 512, 506), 4, 2
     refs = []
@@ -110,6 +115,9 @@ def test_fused_resize_storm_exactly_once(pair):
     for t, ref in zip((ta, tb), refs):
         for x, y in zip(t.snapshot(), ref):
             assert torch.equal(x, y), pair
+    if pair == "bs+stencil_ragged":
+        ok, err = tb.check(tb.snapshot())
+        assert ok, err
     _check_log(ca, Ba, req, ia)
     _check_log(cb, Bb, req, ib)
     for q, B, it in ((qa, Ba, ia), (qb, Bb, ib)):
