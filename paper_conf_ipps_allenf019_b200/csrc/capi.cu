@@ -4,6 +4,7 @@
 #include <cstring>
 #include <map>
 #include <memory>
+#include <cstdlib>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -29,6 +30,13 @@ namespace slate {
 static std::mutex g_servers_mu;
 static std::map<int, Server*> g_servers;   // in-process servers live until process exit
 
+// At exit: stop every server's threads before the CUDA runtime tears the
+// context down (registered after the runtime's own handler, so it runs first).
+static void stop_servers_at_exit() {
+  std::lock_guard<std::mutex> g(g_servers_mu);
+  for (auto& kv : g_servers) kv.second->stop_threads();
+}
+
 Server* get_local_server(int device, std::string* err, int* rc) {
   std::lock_guard<std::mutex> g(g_servers_mu);
   auto it = g_servers.find(device);
@@ -40,6 +48,10 @@ Server* get_local_server(int device, std::string* err, int* rc) {
     return nullptr;
   }
   g_servers[device] = s;
+  // registered once the runtime is initialised (init made CUDA calls), so the
+  // handler runs before the runtime's teardown
+  static const bool registered = (std::atexit(stop_servers_at_exit), true);
+  (void)registered;
   return s;
 }
 }  // namespace slate

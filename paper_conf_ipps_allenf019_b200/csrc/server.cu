@@ -43,15 +43,17 @@ static uint32_t overlap(uint32_t a_lo, uint32_t a_hi, uint32_t b_lo, uint32_t b_
 
 Server::Server(int device) : device_(device) {}
 
-Server::~Server() {
+Server::~Server() { stop_threads(); }
+
+void Server::stop_threads() {
+  clk_stop_.store(true);                       // a clock probe in flight is released (clock_anchor)
+  if (clock_.joinable()) clock_.join();
   {
     std::lock_guard<std::mutex> g(mu_);
     stop_ = true;
   }
   cv_.notify_all();
   if (poller_.joinable()) poller_.join();
-  clk_stop_.store(true);
-  if (clock_.joinable()) clock_.join();
 }
 
 double Server::now_us() const {

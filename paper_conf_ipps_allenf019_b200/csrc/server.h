@@ -101,6 +101,11 @@ class Server {
   explicit Server(int device);
   ~Server();
   int init(std::string* err);
+  // Stops and joins the poller and clock threads (idempotent).  In-process
+  // servers live until process exit; this runs from an atexit handler, before
+  // the CUDA runtime's own teardown, so no server thread is inside a CUDA call
+  // (or has a clock probe kernel waiting on it) while the context is destroyed.
+  void stop_threads();
 
   int num_sms() const { return n_sms_; }
   slate_info info() const;
