@@ -273,6 +273,11 @@ uint32_t Server::open_queue() {
   Q->lo = 0;
   Q->hi = uint32_t(n_sms_ - 1);
   cudaStreamCreateWithFlags(&Q->stream, cudaStreamNonBlocking);
+  {
+    int lo_prio = 0, hi_prio = 0;
+    cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
+    cudaStreamCreateWithPriority(&Q->snap, cudaStreamNonBlocking, hi_prio);
+  }
   for (cudaStream_t& a : Q->aux) cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking);   // not on the resize path
   const uint32_t id = Q->id;
   queues_[id] = std::move(Q);
@@ -299,9 +304,11 @@ int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
     cudaStreamSynchronize(Q.stream);
     for (cudaStream_t a : Q.aux)
       if (a) cudaStreamSynchronize(a);
+    cudaStreamSynchronize(Q.snap);
     const int slot = int((Q.d_ctrl - d_ctrl_pool_) / 16);
     free_ctrl_.push_back(slot);
     cudaStreamDestroy(Q.stream);
+    cudaStreamDestroy(Q.snap);
     for (cudaStream_t a : Q.aux)
       if (a) cudaStreamDestroy(a);
     // a queue can still hold SMs with nothing issued (a resize after its last
@@ -743,17 +750,17 @@ void Server::close_batch(Queue& Q, cudaEvent_t end, bool closed_by_launch) {
   if (!ws.empty()) {
     cudaEvent_t snap;
     cudaEventCreateWithFlags(&snap, cudaEventDisableTiming);
-    cudaStreamWaitEvent(copy_stream_, end, 0);
+    cudaStreamWaitEvent(Q.snap, end, 0);
     // one strided copy per run of consecutive slots (headers out of 2.5-KB blocks)
     for (size_t i = 0; i < ws.size();) {
       size_t j = i + 1;
       while (j < ws.size() && ws[j]->slot == ws[j - 1]->slot + 1) ++j;
       const int s0 = ws[i]->slot;
       cudaMemcpy2DAsync(h_snap_ + size_t(s0) * kTaskCtlHeader, kTaskCtlHeader, d_tc_ + s0, sizeof(TaskCtl),
-                        kTaskCtlHeader, j - i, cudaMemcpyDeviceToHost, copy_stream_);
+                        kTaskCtlHeader, j - i, cudaMemcpyDeviceToHost, Q.snap);
       i = j;
     }
-    cudaEventRecord(snap, copy_stream_);
+    cudaEventRecord(snap, Q.snap);
     for (Launch* M : ws) M->ev_done.push_back(snap);
   }
   Q.open_batch.clear();
@@ -901,10 +908,10 @@ int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
       L.ev_end.push_back(ev_end);
       cudaEvent_t ev_snap;
       CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
-      CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+      CK(cudaStreamWaitEvent(Q.snap, ev_end, 0));
       CK(cudaMemcpyAsync(h_snap_ + size_t(slot) * kTaskCtlHeader, d_tc_ + slot, kTaskCtlHeader,
-                         cudaMemcpyDeviceToHost, copy_stream_));
-      CK(cudaEventRecord(ev_snap, copy_stream_));
+                         cudaMemcpyDeviceToHost, Q.snap));
+      CK(cudaEventRecord(ev_snap, Q.snap));
       L.ev_done.push_back(ev_snap);
     }
   }
@@ -1015,10 +1022,10 @@ int Server::topup(Queue& Q, Launch& R, std::string* err) {
   CK(cudaEventRecord(ev_end, aux));
   R.ev_end.push_back(ev_end);
   CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
-  CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+  CK(cudaStreamWaitEvent(Q.snap, ev_end, 0));
   CK(cudaMemcpyAsync(h_snap_ + size_t(R.slot) * kTaskCtlHeader, d_tc_ + R.slot, kTaskCtlHeader,
-                     cudaMemcpyDeviceToHost, copy_stream_));
-  CK(cudaEventRecord(ev_snap, copy_stream_));
+                     cudaMemcpyDeviceToHost, Q.snap));
+  CK(cudaEventRecord(ev_snap, Q.snap));
   R.ev_done.push_back(ev_snap);
   Q.topup_ends.push_back(ev_end);
   R.n_topups += 1;
@@ -1190,11 +1197,11 @@ int Server::launch_fused(uint32_t qa, uint64_t ka, const slate_launch_desc* da, 
   CK(cudaEventRecord(ev_end, A.stream));
   CK(cudaStreamWaitEvent(B.stream, ev_end, 0));   // B's later launches follow the fused kernel
   A.last_op_kernel = B.last_op_kernel = false;
-  CK(cudaStreamWaitEvent(copy_stream_, ev_end, 0));
+  CK(cudaStreamWaitEvent(A.snap, ev_end, 0));
   for (Launch* L : Ls)
     CK(cudaMemcpyAsync(h_snap_ + size_t(L->slot) * kTaskCtlHeader, d_tc_ + L->slot, kTaskCtlHeader,
-                       cudaMemcpyDeviceToHost, copy_stream_));
-  CK(cudaEventRecord(ev_snap, copy_stream_));
+                       cudaMemcpyDeviceToHost, A.snap));
+  CK(cudaEventRecord(ev_snap, A.snap));
   for (int i = 0; i < 2; ++i) {
     Ls[i]->t_issue_us = now_us();
     Qs[i]->issued.push_back(Ls[i]->id);

@@ -62,6 +62,12 @@ struct Launch {
 struct Queue {
   uint32_t id;
   cudaStream_t stream = nullptr;
+  // the queue's own stream for its control-block snapshot copies (each waits
+  // for a launch's or batch's end): per queue, so one queue's long batch never
+  // holds back the completion of another's (a shared copy stream serialised
+  // them in issue order: a co-runner's end was observed only after the other
+  // job's whole batch, delaying its release and the survivor's grow)
+  cudaStream_t snap = nullptr;
   static constexpr int kAux = 8;
   cudaStream_t aux[kAux] = {};  // top-up launches (round robin: a top-up whose workers joined runs
                                 // until the launch drains, so top-ups must not queue behind each other)

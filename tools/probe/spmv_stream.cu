@@ -19,6 +19,9 @@
 using namespace slate;
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("CUDA %s at %d\n", cudaGetErrorString(e), __LINE__); exit(1); } } while (0)
 
+#ifdef SLATE_SPMV_PROFILE
+static void* spmv_prof_ptr() { void* p; CK(cudaGetSymbolAddress(&p, spmv::spmv_prof)); return p; }
+#endif
 int main(int argc, char** argv) {
   const int n = 1 << 20, band = 4096;
   const int nnzr = argc > 1 ? atoi(argv[1]) : 16;
@@ -80,7 +83,7 @@ int main(int argc, char** argv) {
   };
   const KindOps ws = spmv_ws_ops();
   CK(cudaFuncSetAttribute(ws.worker_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ws.smem));
-  timeit("original, register body", 148, [&] { standalone<SpmvCsrReg><<<nblk, SpmvCsrReg::kThreads>>>(a); });
+  timeit("original (SpmvSeg)", 148, [&] { standalone<SpmvSeg><<<nblk, SpmvSeg::kThreads>>>(a); });
   auto worker = [&](const char* name, auto kern, int threads, int smem, uint32_t iters, int sms) {
     int o; CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, threads, smem));
     WorkerParams<slate_args_spmv> p{};
@@ -99,7 +102,6 @@ int main(int argc, char** argv) {
     timeit(buf, sms, [&] { CK(ws.launch_worker(w, &a, 148, 0)); });
   };
   for (int sms : {148, 111, 74, 56, 37}) {
-    worker("worker, register body", slate_worker<SpmvCsrReg>, SpmvCsrReg::kThreads, 0, 8, sms);
     ws_worker(32, sms);
     if (sms == 148) { ws_worker(16, sms); ws_worker(8, sms); ws_worker(1, sms); }
   }
@@ -124,13 +126,18 @@ int main(int argc, char** argv) {
   }
 #endif
 #ifdef SLATE_SPMV_PROFILE
-  ws_worker(32, 148);
+  for (int sms : {148, 74, 37}) {
   static long long pr[148][32][5];
+  CK(cudaMemset(spmv_prof_ptr(), 0, sizeof(pr)));
+  ws_worker(32, sms);
   CK(cudaMemcpyFromSymbol(pr, spmv::spmv_prof, sizeof(pr)));
-  for (int c : {0, 1, 70, 147}) for (int w : {0, 7, 15}) {
+  printf("-- %d SMs\n", sms);
+  for (int c = 0; c < 148; ++c) for (int w : {0, 15}) {
+    if (!pr[c][w][4] || (c % 16 != 0)) continue;
     long long* o = pr[c][w];
     printf("cta %3d warp %2d: total %7lld clk  wait-full %6.1f%%  first-chunk %5.1f%%  compute %5.1f%%  chunks %lld  (%.0f clk/chunk compute)\n",
            c, w, o[0], 100.0 * o[1] / o[0], 100.0 * o[2] / o[0], 100.0 * o[3] / o[0], o[4], o[4] ? double(o[3]) / o[4] : 0.0);
+  }
   }
 #endif
   return 0;
