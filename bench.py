@@ -399,15 +399,15 @@ def run_schedule(name, w, sA, sB, kA, kB, S):
         spin_ms(w.arrival_ms)
         ib = submit(sB, kB, b, placement=S.PLACE_AUTO)
         qa, qb = collect(sA, ia), collect(sB, ib)
-    elif name == "slate_makespan":  # Slate AUTO with the makespan-only split (reading Q10; the default is Q41)
-        sA.set_split_objective("makespan")
+    elif name == "slate_antt":      # Slate AUTO with the turnaround-aware split (reading Q41; the default is Q10's)
+        sA.set_split_objective("antt", SPLIT_SLACK)
         try:
             ia = submit(sA, kA, a, placement=S.PLACE_AUTO)
             spin_ms(w.arrival_ms)
             ib = submit(sB, kB, b, placement=S.PLACE_AUTO)
             qa, qb = collect(sA, ia), collect(sB, ib)
         finally:
-            sA.set_split_objective("antt", SPLIT_SLACK)
+            sA.set_split_objective("makespan")
     elif name == "slate_table":     # Slate AUTO with the paper's Tab I alone deciding (reading Q8)
         sA.set_policy(S.POLICY_TABLE)
         try:
@@ -530,7 +530,7 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
     base = {}
     for name in ("seq_cuda", "seq_cuda_ba", "seq_slate", "seq_slate_ba", "streams", "slate_table", "slate_forced",
-                 "slate_makespan"):
+                 "slate_antt"):
         run_schedule(name, w, sA, sB, kA, kB, S)
         base[name] = median_schedule(name, w, sA, sB, kA, kB, S, flush, 3)
     # every job's solo time: alone on the whole GPU, as original kernels or as
@@ -672,7 +672,7 @@ def run_slate(args, world, rank, local):
         os.environ.setdefault("SLATE_PEAK_HBM_GBPS", str(peaks.get("hbm_gbs", 6650.0)))
         os.environ.setdefault("SLATE_PEAK_TC_TFLOPS", str(peaks.get("bf16_tflops", 1590.0)))
     sA, sB = S.Session(None, local), S.Session(None, local)
-    sA.set_split_objective("antt", SPLIT_SLACK)   # reading Q41 (the server's default, made explicit)
+    sA.set_split_objective("makespan")   # reading Q10, the server's default (made explicit); Q41's ANTT split is the slate_antt schedule
     flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MB > L2
 
     # ---- C2, the headline (BASELINE configs[1]); its timed loop is the bench's timed region
@@ -809,7 +809,8 @@ def run_slate(args, world, rank, local):
         "gain_vs_slate_sequential": r2["gain_vs_slate_sequential"], "best_sequential": r2["best_sequential"],
         "stp": r2["schedules"]["slate_corun"]["stp"], "antt": r2["schedules"]["slate_corun"]["antt"],
         "stp_vs_sequential": r2["stp_vs_sequential"], "antt_vs_sequential": r2["antt_vs_sequential"],
-        "split_objective": {"objective": "antt", "slack": SPLIT_SLACK, "reading": "DESIGN.md Q41"},
+        "split_objective": {"objective": "makespan", "reading": "DESIGN.md Q10/Q41",
+                            "alternative": "schedules.slate_antt: ANTT within %.2f of the best makespan" % SPLIT_SLACK},
         "schedules": r2["schedules"], "forced_split_sms_spmv": r2["split_sms_b"], "resize_us": r2["resize_us"],
         "corun_utilisation": r2["utilisation"], "profiles": r2["profiles"], "roofline": r2["roofline"],
         "clocks": clocks.get("r"),

@@ -534,7 +534,7 @@ int slate_fluid_corun_obj(const uint32_t* sms_a, const double* ms_a, uint32_t n_
 
 /* The split objective of the server's co-runs (process-wide; initial value
  * from SLATE_SPLIT_OBJECTIVE = makespan | antt and SLATE_SPLIT_SLACK in the
- * server's environment, default antt with slack 0.05).  Errors: EINVAL. */
+ * server's environment, default makespan; slack 0.05).  Errors: EINVAL. */
 slate_status slate_set_split_objective(slate_session* s, uint32_t objective, double slack);
 
 /* Selector policy of the server (process-wide; the initial value comes from

@@ -154,7 +154,7 @@ int Server::init(std::string* err) {
   }
   min_gain_ = env_double("SLATE_MIN_GAIN", 1.05);
   if (const char* o = std::getenv("SLATE_SPLIT_OBJECTIVE"))
-    split_objective_ = std::string(o) == "makespan" ? SLATE_SPLIT_MAKESPAN : SLATE_SPLIT_ANTT;
+    split_objective_ = std::string(o) == "antt" ? SLATE_SPLIT_ANTT : SLATE_SPLIT_MAKESPAN;
   split_slack_ = env_double("SLATE_SPLIT_SLACK", 0.05);
   max_corun_ = uint32_t(std::max(2.0, std::min(4.0, env_double("SLATE_MAX_CORUN", 3.0))));
   poller_ = std::thread([this] { poller_main(); });

@@ -235,7 +235,7 @@ class Server {
   double saturation_frac_ = 0.95;
   uint32_t policy_ = SLATE_POLICY_HYBRID;
   double min_gain_ = 1.05;
-  uint32_t split_objective_ = SLATE_SPLIT_ANTT;   // reading Q41
+  uint32_t split_objective_ = SLATE_SPLIT_MAKESPAN;   // reading Q41 (ANTT opt-in)
   uint32_t max_corun_ = 3;                         // SLATE_MAX_CORUN: co-runners per group (NEXT-4, Q49)
   double split_slack_ = 0.05;
 

@@ -333,7 +333,7 @@ class Session:
         """Selector policy of the server (POLICY_TABLE / LITERAL / HYBRID; reading Q31)."""
         return self._check(_lib.slate_set_policy(self._h, policy), "slate_set_policy")
 
-    def set_split_objective(self, objective="antt", slack=0.05):
+    def set_split_objective(self, objective="makespan", slack=0.05):
         """The split objective of the server's co-runs (reading Q41): "makespan" or "antt"."""
         return self._check(_lib.slate_set_split_objective(self._h, _OBJ[objective], slack), "slate_set_split_objective")
 
