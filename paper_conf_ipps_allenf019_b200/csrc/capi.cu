@@ -1,6 +1,7 @@
 // capi.cu -- the extern "C" boundary of libslate (include/slate.h).
 // In-process sessions talk to a per-device Server directly; sessions attached
 // to an endpoint go through the shared-memory transport (ipc.cu).
+#include <cstdio>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -33,8 +34,14 @@ static std::map<int, Server*> g_servers;   // in-process servers live until proc
 // At exit: stop every server's threads before the CUDA runtime tears the
 // context down (registered after the runtime's own handler, so it runs first).
 static void stop_servers_at_exit() {
+  static const bool trace = std::getenv("SLATE_EXIT_TRACE") != nullptr;
+  if (trace) fprintf(stderr, "[slate] exit: stopping server threads\n");
   std::lock_guard<std::mutex> g(g_servers_mu);
   for (auto& kv : g_servers) kv.second->stop_threads();
+  if (trace) {
+    fprintf(stderr, "[slate] exit: server threads stopped\n");
+    for (auto& kv : g_servers) kv.second->report_busy_streams(5000.0);
+  }
 }
 
 Server* get_local_server(int device, std::string* err, int* rc) {

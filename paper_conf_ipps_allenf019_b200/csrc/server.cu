@@ -56,6 +56,31 @@ void Server::stop_threads() {
   if (poller_.joinable()) poller_.join();
 }
 
+void Server::report_busy_streams(double wait_ms) {
+  std::vector<std::pair<std::string, cudaStream_t>> ss = {{"ctrl", ctrl_stream_}, {"copy", copy_stream_},
+                                                           {"clk", clk_stream_}};
+  {
+    std::lock_guard<std::mutex> g(mu_);
+    for (auto& kv : queues_) {
+      const Queue& Q = *kv.second;
+      if (Q.closed) continue;
+      const std::string q = "q" + std::to_string(Q.id);
+      ss.push_back({q + ".stream", Q.stream});
+      ss.push_back({q + ".snap", Q.snap});
+      for (int i = 0; i < Queue::kAux; ++i) ss.push_back({q + ".aux" + std::to_string(i), Q.aux[i]});
+    }
+  }
+  const double t0 = now_us();
+  for (auto& x : ss) {
+    if (!x.second) continue;
+    cudaError_t e;
+    while ((e = cudaStreamQuery(x.second)) == cudaErrorNotReady && now_us() - t0 < wait_ms * 1e3)
+      std::this_thread::sleep_for(std::chrono::milliseconds(1));
+    if (e != cudaSuccess) fprintf(stderr, "[slate] exit: stream %s busy (%s)\n", x.first.c_str(), cudaGetErrorString(e));
+  }
+  fprintf(stderr, "[slate] exit: streams checked (%zu)\n", ss.size());
+}
+
 double Server::now_us() const {
   return std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }

@@ -112,6 +112,9 @@ class Server {
   // the CUDA runtime's own teardown, so no server thread is inside a CUDA call
   // (or has a clock probe kernel waiting on it) while the context is destroyed.
   void stop_threads();
+  // Development aid (SLATE_EXIT_TRACE): which of the server's streams still
+  // has work after up to `wait_ms` (stderr).
+  void report_busy_streams(double wait_ms);
 
   int num_sms() const { return n_sms_; }
   slate_info info() const;
