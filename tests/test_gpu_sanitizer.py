@@ -60,9 +60,32 @@ def unexplained_hazards(report):
     return bad
 
 
+def _closed_reason():
+    """The GPU pool may close compute-sanitizer (its runs have left GPUs needing a
+    reset there); the stub then answers every call, `--version` included, with a
+    one-line notice and no tool banner.  Such a pool cannot run this tier: skip
+    it, naming the notice, rather than fail the GPU suite."""
+    try:
+        r = subprocess.run([SAN, "--version"], capture_output=True, text=True, timeout=60)
+    except (OSError, subprocess.TimeoutExpired) as e:
+        return "compute-sanitizer not runnable: %s" % e
+    out = r.stdout + r.stderr
+    if "closed" in out or "NVIDIA" not in out:
+        return "compute-sanitizer unavailable on this pool: " + out.strip()[:200]
+    return None
+
+
+@pytest.fixture(scope="module")
+def sanitizer():
+    why = _closed_reason()
+    if why:
+        pytest.skip(why)
+    return SAN
+
+
 @pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
 @pytest.mark.parametrize("group", GROUPS)
-def test_sanitizer(tool, group):
+def test_sanitizer(sanitizer, tool, group):
     cmd = [SAN, "--tool", tool, "--error-exitcode", "97", "--print-limit", "20"]
     if tool == "memcheck":
         cmd += ["--leak-check", "no"]
