@@ -71,6 +71,63 @@ __global__ void bulk_read(const char* src, uint32_t n_pieces, uint32_t* ctr, int
   for (int s = 0; s < stages; ++s) if (pend & (1u << s)) wait(s);
 }
 
+// one CTA, `issuers` warps each keeping its own ring of `stages` copies
+// (is the single-CTA ceiling per CTA or per issuing thread?)
+__global__ void bulk_multi(const char* src, uint32_t n_pieces, uint32_t* ctr, int k, uint32_t bytes, int stages) {
+  extern __shared__ __align__(128) char sm[];
+  __shared__ uint64_t bar[4][16];
+  if ((int)smid() >= k) return;
+  const int w = threadIdx.x >> 5;
+  if ((threadIdx.x & 31) != 0) return;
+  uint64_t* b = bar[w];
+  char* ring = sm + size_t(w) * stages * bytes;
+  for (int i = 0; i < stages; ++i) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(&b[i])));
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  const uint32_t cpp = kPiece / bytes;
+  uint32_t par = 0, pend = 0, sub = 0, p = atomicAdd(ctr, 1u);
+  auto wait = [&](int s) {
+    const uint32_t ph = (par >> s) & 1u;
+    asm volatile("{\n\t.reg .pred p;\nW_%=:\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W_%=;\n}" ::"r"(su32(&b[s])), "r"(ph) : "memory");
+    par ^= 1u << s; pend &= ~(1u << s);
+  };
+  for (uint32_t i = 0; p < n_pieces; ++i) {
+    const int s = int(i % stages);
+    if (pend & (1u << s)) wait(s);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(&b[s])), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(ring + size_t(s) * bytes)),
+                 "l"(src + size_t(p) * kPiece + size_t(sub) * bytes), "r"(bytes), "r"(su32(&b[s])) : "memory");
+    pend |= 1u << s;
+    if (++sub == cpp) { sub = 0; p = atomicAdd(ctr, 1u); }
+  }
+  for (int s = 0; s < stages; ++s) if (pend & (1u << s)) wait(s);
+}
+
+// cp.async 16 B per thread (LDGSTS), a ring of `stages` 16-KB slots filled by
+// all threads of the CTA, committed per slot
+template <int G>
+__global__ void ldgsts_read(const char* src, uint32_t n_pieces, uint32_t* ctr, int k, int stages) {
+  extern __shared__ __align__(128) char sm[];
+  __shared__ uint32_t s_p;
+  if ((int)smid() >= k) return;
+  const uint32_t slot = 16384;
+  for (;;) {
+    if (threadIdx.x == 0) s_p = atomicAdd(ctr, 1u);
+    __syncthreads();
+    const uint32_t p = s_p;
+    __syncthreads();
+    if (p >= n_pieces) break;
+    const char* b = src + size_t(p) * kPiece;
+    for (uint32_t c = 0; c < kPiece / slot; ++c) {
+      char* d = sm + size_t(c % stages) * slot;
+      for (uint32_t o = threadIdx.x * 16; o < slot; o += blockDim.x * 16)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(su32(d + o)), "l"(b + c * slot + o) : "memory");
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      asm volatile("cp.async.wait_group %0;" ::"n"(G - 1) : "memory");
+    }
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+}
+
 int main() {
   const size_t total = size_t(2) << 30;  // 2 GiB > L2
   char* src; CK(cudaMalloc(&src, total)); CK(cudaMemset(src, 1, total));
@@ -93,6 +150,11 @@ int main() {
     printf("sms %3d  %-40s %8.1f GB/s  %6.1f GB/s per SM\n", sms, what, gbs, gbs / sms);
   };
   char name[128];
+  CK(cudaFuncSetAttribute(bulk_multi, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  CK(cudaFuncSetAttribute(ldgsts_read<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  CK(cudaFuncSetAttribute(ldgsts_read<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  CK(cudaFuncSetAttribute(ldgsts_read<12>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+  // (1) LDG.128 and one-issuer bulk copies vs CTAs per SM (profiles/r2_read_bw_probe.txt)
   for (int sms : {148, 74, 37, 18}) {
     for (int cps : {1, 2, 4, 8}) for (int thr : {256, 512}) {
       if (cps * thr > 2048) continue;
@@ -106,6 +168,24 @@ int main() {
       if (smem * cps > 220 * 1024) continue;
       snprintf(name, sizeof name, "bulk %d CTA/SM  %2u KB x %d", cps, bytes / 1024, st);
       timeit([&] { bulk_read<<<nsm * cps, 32, smem>>>(src, n_pieces, ctr, sms, bytes, st); }, sms, name);
+    }
+  }
+  // (2) one CTA, several issuing warps; LDGSTS (profiles/r2_read_bw_probe_issuers.txt)
+  for (int sms : {74, 37}) {
+    for (int iss : {1, 2, 3, 4}) for (uint32_t bytes : {16384u, 32768u}) for (int st : {2, 3, 4}) {
+      const size_t smem = size_t(bytes) * st * iss;
+      if (smem > 200 * 1024) continue;
+      snprintf(name, sizeof name, "bulk 1 CTA, %d issuer warps, %2u KB x %d", iss, bytes / 1024, st);
+      timeit([&] { bulk_multi<<<nsm, 32 * iss, smem>>>(src, n_pieces, ctr, sms, bytes, st); }, sms, name);
+    }
+    for (int thr : {256, 512, 1024}) for (int st : {4, 8, 12}) {
+      snprintf(name, sizeof name, "ldgsts 1 CTA x %d thr, 16 KB x %d", thr, st);
+      auto l = [&] {
+        if (st == 4) ldgsts_read<4><<<nsm, thr, size_t(16384) * st>>>(src, n_pieces, ctr, sms, st);
+        else if (st == 8) ldgsts_read<8><<<nsm, thr, size_t(16384) * st>>>(src, n_pieces, ctr, sms, st);
+        else ldgsts_read<12><<<nsm, thr, size_t(16384) * st>>>(src, n_pieces, ctr, sms, st);
+      };
+      timeit(l, sms, name);
     }
   }
   return 0;

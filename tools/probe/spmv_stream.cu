@@ -101,12 +101,13 @@ int main(int argc, char** argv) {
     char buf[96]; snprintf(buf, sizeof buf, "worker, warp-specialised it %u", iters);
     timeit(buf, sms, [&] { CK(ws.launch_worker(w, &a, 148, 0)); });
   };
+  const uint32_t IT = getenv("SPMV_ITERS") ? atoi(getenv("SPMV_ITERS")) : 32;
   for (int sms : {148, 111, 74, 56, 37}) {
-    ws_worker(32, sms);
+    ws_worker(IT, sms);
     if (sms == 148) { ws_worker(16, sms); ws_worker(8, sms); ws_worker(1, sms); }
   }
 #ifdef SLATE_SPMV_TRACE
-  ws_worker(32, 148);
+  ws_worker(IT, 74);
   static unsigned long long t[4][3][64][4];
   CK(cudaMemcpyFromSymbol(t, spmv::spmv_trace, sizeof(t)));
   unsigned long long t0 = ~0ull;
@@ -129,7 +130,7 @@ int main(int argc, char** argv) {
   for (int sms : {148, 74, 37}) {
   static long long pr[148][32][5];
   CK(cudaMemset(spmv_prof_ptr(), 0, sizeof(pr)));
-  ws_worker(32, sms);
+  ws_worker(IT, sms);
   CK(cudaMemcpyFromSymbol(pr, spmv::spmv_prof, sizeof(pr)));
   printf("-- %d SMs\n", sms);
   for (int c = 0; c < 148; ++c) for (int w : {0, 15}) {
