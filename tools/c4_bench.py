@@ -202,6 +202,11 @@ def main():
         # turnaround of each job from the step's release (all four arrive together)
         stps.append(sum(solo[k] / (res[k][step][1] - t0) for k in JOBS))
         resize += [v for k in JOBS for v in res[k][step][3]]
+    if os.environ.get("C4_TIMELINE"):   # diagnostics: each job's [start, end] from the step's first start (ms)
+        for step in range(a.steps):
+            t0 = min(res[k][step][0] for k in JOBS)
+            sys.stderr.write("C4 step %d: %s\n" % (step, "  ".join(
+                "%s %.2f-%.2f" % (k, res[k][step][0] - t0, res[k][step][1] - t0) for k in JOBS)))
     spans_sorted = sorted(spans)
     mk = spans_sorted[len(spans) // 2]
     # a step far above the median: report each tenant's longest launches (stderr)
