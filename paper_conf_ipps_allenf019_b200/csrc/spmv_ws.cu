@@ -164,8 +164,17 @@ struct Smem {
 // Rows of one chunk: kPasses passes of 8 rows per compute warp, 4 lanes per
 // row; every pass's shared-memory loads are issued before the first FMA.  x
 // comes from the task's window, or global memory for a column outside it.
-__device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Smem& S, const ChunkMeta& m,
-                                              const TaskMeta& tm, int s, int nnz) {
+#ifndef SLATE_SPMV_EARLY_RELEASE
+#define SLATE_SPMV_EARLY_RELEASE 1
+#endif
+// Returns true when it already released the slot (arrived on `empty`): a warp
+// whose rows all fit their first segment is done with the slot once its
+// columns and values are in registers, so the chunk warp can refill the slot
+// while the warp still gathers x and accumulates (the gathers are ~55% of the
+// chunk's shared-memory work; profiles/r2_spmv_limits.md).
+__device__ __forceinline__ bool compute_chunk(const slate_args_spmv& a, const Smem& S, const ChunkMeta& m,
+                                              const TaskMeta& tm, int s, int nnz, uint64_t* empty) {
+  bool released = false;
   const float* __restrict__ xg = reinterpret_cast<const float*>(a.x);
   const int32_t* rp = S.rp(int(m.tb)) + m.row0;          // rp of the chunk's first row
   const float* xw = S.xw(int(m.wb));
@@ -209,6 +218,13 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
       if (base < hi[u]) sg[u] = seg(base);
       else sg[u] = spmvseg::Seg{make_int4(0, 0, 0, 0), make_float4(0.f, 0.f, 0.f, 0.f)};
     }
+    if (SLATE_SPMV_EARLY_RELEASE && !__any_sync(0xffffffffu, longrow)) {
+      // every lane's slot reads are issued above; the warp barrier orders them
+      // before lane 0's release arrive (as at the end of a chunk)
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) mbar_arrive(empty);
+      released = true;
+    }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       const int base = ((lo[u] >> 2) + q) * 4;
@@ -233,6 +249,7 @@ __device__ __forceinline__ void compute_chunk(const slate_args_spmv& a, const Sm
     const uint32_t lr = (u * kComputeWarps + w) * kPassRows + (lane >> 2);
     if (q == 0 && lr < nrows) __stcs(reinterpret_cast<float*>(a.y) + row_first + lr, v);
   }
+  return released;
 }
 
 // ------------------------------------------------------------------ the worker
@@ -512,14 +529,14 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       long long c2 = clock64();
       pf_first += c2 - c1;
 #endif
-      compute_chunk(a, S, m, tm, s, nnz);
+      const bool released = compute_chunk(a, S, m, tm, s, nnz, &H.slot_empty[s]);
       __syncwarp();
 #ifdef SLATE_SPMV_PROFILE
       pf_comp += clock64() - c2;
 #endif
       if (threadIdx.x == 0) TRACE(2, 22, q, 0);
       if (lane == 0) {
-        mbar_arrive(&H.slot_empty[s]);
+        if (!released) mbar_arrive(&H.slot_empty[s]);
         if (m.last) {
           mbar_arrive(&H.rp_empty[b]);
           mbar_arrive(&H.win_empty[m.wb]);
