@@ -127,6 +127,13 @@ __device__ __forceinline__ void bulk_g2s_keep(void* dst, const void* src, uint32
                : "memory");
 }
 
+#ifndef SLATE_SPMV_PF
+#define SLATE_SPMV_PF 0   // experiment (measured: no gain, profiles/r2_spmv_limits.md)
+#endif
+__device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
 #ifdef SLATE_SPMV_TRACE
 // development trace (tools/probe/spmv_stream.cu): per CTA < 4 and role, 64 events {t, kind, a, b}
 __device__ unsigned long long spmv_trace[4][3][64][4];
@@ -428,6 +435,21 @@ __global__ void __launch_bounds__(kThreads, 1) spmv_worker(const __grid_constant
       prev_n = n;
       prev_e0 = rps[0];
       prev_e1 = rps[r1 - r0];
+#if SLATE_SPMV_PF
+      {
+        // experiment: the task's columns and values into L2 now, up to three
+        // tasks before the chunk warp copies them (four lanes, one bulk
+        // prefetch each: the two halves of both arrays)
+        const int32_t e0 = prev_e0 & ~3, e1 = min((prev_e1 + 3) & ~3, nnz & ~3);
+        const int32_t half = ((e1 - e0) / 2) & ~3;
+        const int32_t o = e0 + ((lane & 1) ? half : 0);
+        const int32_t len = (lane & 1) ? (e1 - e0 - half) : half;
+        if (lane < 4 && len > 0)
+          bulk_prefetch_l2(lane < 2 ? static_cast<const void*>(reinterpret_cast<const int32_t*>(a.col) + o)
+                                    : static_cast<const void*>(reinterpret_cast<const float*>(a.val) + o),
+                           uint32_t(len) * 4);
+      }
+#endif
     }
   } else if (warp == kChunkWarp) {
     // ===================== chunk warp: nonzeros of each task through the slot ring =====================
