@@ -1871,8 +1871,9 @@ void Server::record_resize(const Queue::PendingResize& pr, unsigned long long do
   else
     R.resize_us[pr.idx] = t - pr.t0_us;
   if (std::getenv("SLATE_DEBUG"))
-    fprintf(stderr, "[slate] resize kind %d epoch %u: %.3f us on the device clock, %.3f us host-observed\n", pr.kind,
-            pr.epoch, R.resize_us[pr.idx], t - pr.t0_us);
+    fprintf(stderr, "[slate] resize kind %d (%s) epoch %u of launch %llu (tenant kind %u, %u top-ups): %.3f us on the device clock, %.3f us host-observed\n",
+            pr.kind, pr.kind == 1 ? "shrink" : "grow", pr.epoch, (unsigned long long)R.id, R.k->desc.kind,
+            unsigned(R.n_topups), R.resize_us[pr.idx], t - pr.t0_us);
 }
 
 // A resize applies to the queue, whichever of its launches is running: a
