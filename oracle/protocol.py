@@ -45,7 +45,7 @@ class ProtocolViolation(AssertionError):
     pass
 
 
-PENDING, PROLOGUE, STANDBY, FETCH, EXEC, CHECK, EXITED, RETIRING, WAITDONE = range(9)
+PENDING, PROLOGUE, STANDBY, FETCH, EXEC, CHECK, EXITED, RETIRING, WAITDONE, CLAIMED, ABORT_OK, ABORT_LAST = range(12)
 
 
 @dataclass
@@ -67,6 +67,13 @@ class Config:
                               # and stay; other CTAs may act in between.  False: one atomic
                               # "retire unless last" step
                               # mid-way and return it (Q28)
+    faa_abort: bool = True    # abandon-and-retire as the runtime does it (Q50): one
+                              # fetch-and-add on {live, returned} (live -1, returned +1); the
+                              # task is published to the ring in a later step.  If live went
+                              # 1 -> 0 the worker, in a later step, takes the unit back and
+                              # resumes its task unless the returned count is 0 (a taker claimed
+                              # it: then it publishes and leaves).  Takers claim a count and wait
+                              # for a publication.  False: one atomic "abandon unless last" step
 
 
 def _in(rank, lo, hi):
@@ -82,7 +89,8 @@ class Model:
         self.epoch = 0
         self.lo, self.hi = cfg.lo, cfg.hi  # the resize word {epoch, lo, hi}
         self.live = 0                      # live worker CTAs of the tenant
-        self.returned = []                 # abandoned task starts, FIFO (Q28)
+        self.ret_count = 0                 # returned units committed and not yet claimed (Q28)
+        self.ret_pub = []                  # published returned task starts, FIFO (the ring)
         self.cov = [0] * cfg.blocks        # executions per original block
         self.blocks_done = 0
         self.tasks_done = 0
@@ -115,7 +123,8 @@ class Model:
         self.resident[c[1]] -= 1
 
     def key(self):
-        return (self.next, self.epoch, self.lo, self.hi, self.live, self.main_exited, tuple(self.returned), tuple(self.cov),
+        return (self.next, self.epoch, self.lo, self.hi, self.live, self.main_exited, self.ret_count, tuple(self.ret_pub),
+                tuple(self.cov),
                 self.blocks_done,
                 self.tasks_done, tuple(sorted(self.task_starts)), self.resize_i,
                 tuple(tuple(c) for c in self.ctas), tuple(self.resident))
@@ -129,15 +138,19 @@ class Model:
                 for r in range(self.cfg.ranks):
                     if self.resident[r] < self.cfg.occ:
                         acts.append(("place", i, r))
-            elif st in (PROLOGUE, FETCH, EXEC, CHECK, RETIRING):
+            elif st in (PROLOGUE, FETCH, EXEC, CHECK, RETIRING, ABORT_OK, ABORT_LAST):
                 acts.append(("step", i))
                 # Q28: a worker outside the range may abandon its running task and
-                # retire, unless it is the last live worker (one atomic on {live, returned})
-                if st == EXEC and self.cfg.abort and not self.in_range(c) and self.live > 1:
+                # retire -- one fetch-and-add (faa_abort), or one atomic step that
+                # refuses the last live worker
+                if st == EXEC and self.cfg.abort and not self.in_range(c) and (self.cfg.faa_abort or self.live > 1):
                     acts.append(("abort", i))
+            elif st == CLAIMED:
+                if self.ret_pub:                   # the claimed unit has been published
+                    acts.append(("step", i))
             elif st == STANDBY:
                 acts.append(("step", i))
-                if self.live == 0 and self.next < self.cfg.blocks:
+                if self.live == 0 and (self.next < self.cfg.blocks or self.ret_count or self.ret_pub):
                     acts.append(("timeout", i))
             elif st == WAITDONE and self.blocks_done == self.cfg.blocks:
                 acts.append(("step", i))
@@ -168,8 +181,15 @@ class Model:
         i = act[1]
         c = self.ctas[i]
         st = c[0]
-        if act[0] == "abort":              # return the task, retire (live -1, returned +1 at once)
-            self.returned.append(c[4])
+        if act[0] == "abort":
+            if cfg.faa_abort:                  # fetch-and-add: live -1, returned +1; publish later
+                was_last = self.live == 1
+                self.live -= 1
+                self.ret_count += 1
+                c[0] = ABORT_LAST if was_last else ABORT_OK
+                return
+            self.ret_count += 1                # one atomic step: return the task, retire
+            self.ret_pub.append(c[4])
             self.exit(c, True)
             return
         if act[0] == "timeout":            # standby with no live worker: run anyway (liveness)
@@ -180,9 +200,26 @@ class Model:
             c[0] = EXITED
             self.resident[c[1]] -= 1
             return
+        if st == ABORT_OK:                 # publish the abandoned task, leave (live already -1)
+            self.ret_pub.append(c[4])
+            self.exit(c, False)
+            return
+        if st == ABORT_LAST:               # it was the last live worker: take the unit back ...
+            if self.ret_count >= 1:
+                self.ret_count -= 1
+                self.live += 1
+                c[0] = EXEC                # ... and resume its task (none of it ran)
+            else:                          # a taker claimed it: publish for the taker, leave
+                self.ret_pub.append(c[4])
+                self.exit(c, False)
+            return
+        if st == CLAIMED:                  # the ring slot of the claim is published
+            g = self.ret_pub.pop(0)
+            c[0], c[4], c[5] = EXEC, g, min(cfg.iters, cfg.blocks - g)
+            return
         if st in (PROLOGUE, STANDBY):
             # Lst1: leader reads the SM id and the bound; here also the queue state
-            if self.next >= cfg.blocks and not self.returned:
+            if self.next >= cfg.blocks and not self.ret_count:
                 self.exit(c, False)        # exit (2): nothing left to do
             elif self.in_range(c):
                 self.live += 1
@@ -192,9 +229,9 @@ class Model:
             else:
                 c[0] = STANDBY             # wait: the tenant is under-staffed
         elif st == FETCH:
-            if self.returned:              # Q28: returned tasks first
-                g = self.returned.pop(0)
-                c[0], c[4], c[5] = EXEC, g, min(cfg.iters, cfg.blocks - g)
+            if self.ret_count:             # Q28: returned tasks first -- claim a unit, then wait for its slot
+                self.ret_count -= 1
+                c[0] = CLAIMED
                 return
             # Lst2 (2): globIdx = atomicAdd(&slateIdx, SLATE_ITERS)
             g = self.next
@@ -220,7 +257,7 @@ class Model:
                 was_last = self.live == 1
                 self.live -= 1             # fetch-and-add: live -= 1
                 c[0], c[5] = RETIRING, int(was_last)
-            elif self.live == 1 and (self.next < cfg.blocks or self.returned):
+            elif self.live == 1 and (self.next < cfg.blocks or self.ret_count):
                 c[0] = FETCH               # stay (the last live worker never retires)
             else:
                 self.exit(c, True)         # exit (3): retreated
@@ -248,7 +285,7 @@ class Model:
             raise ProtocolViolation("next_clamped")
         if self.live != 0:
             raise ProtocolViolation("live workers at the end")
-        if self.returned:
+        if self.ret_count or self.ret_pub:
             raise ProtocolViolation("returned tasks never executed")
 
     def check_step(self):

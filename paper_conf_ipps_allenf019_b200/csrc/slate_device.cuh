@@ -241,9 +241,17 @@ __device__ void check_shrink_done(const P& p, uint64_t c, uint32_t lane) {
 // protocol allows anyway).  A CAS loop here serialises a mass retirement: with
 // N workers leaving at once only one CAS per L2 round trip succeeds, and a
 // shrink of half the SMs of a 4-CTA/SM tenant took ~90 us (tools/storm_tenant.py).
-// With `give_back`, retiring and returning the task must be one atomic step
-// (Q28: a returned task must never be taken while its giver could stay), so
-// that path keeps the CAS.
+// With `give_back` (Q28: retiring and returning the task must be one atomic
+// step, so a returned task is never orphaned) it is one fetch-and-add too
+// (reading Q50): live -1 and returned +1 in the same word.  A worker that was
+// not the last has retired and returned its task (true: the caller publishes
+// the task in the ring).  The last one takes the unit back -- returned -1,
+// live +1, by CAS, and keeps its task (false) -- unless the returned count is
+// already 0: a taker has claimed the unit and waits for its publication, and
+// that taker is live, so the worker publishes and leaves (true).  Only the
+// last worker ever loops.  Round 2 kept a CAS loop for every give-back, and a
+// GEMM shrink of ~60 CTA pairs serialised on it (storm shrink p50 34-42 us
+// against 13 us for grows).  Modelled in oracle/protocol.py (Config.faa_abort).
 __device__ __forceinline__ bool try_retire(TaskCtl* tc, bool give_back = false) {
   if (!give_back) {
     const unsigned long long old = atomicAdd(&tc->live_pending, ~0ull);   // live -= 1
@@ -251,14 +259,16 @@ __device__ __forceinline__ bool try_retire(TaskCtl* tc, bool give_back = false) 
     atomicAdd(&tc->live_pending, 1ull);                                    // the last one stays
     return false;
   }
-  unsigned long long v = ld_relaxed_u64(&tc->live_pending);
-  const unsigned long long delta = give_back ? (1ull << 32) - 1ull : ~0ull;   // live -1 (, returned +1)
-  while (uint32_t(v) > 1u) {
-    const unsigned long long w = atomicCAS(&tc->live_pending, v, v + delta);
-    if (w == v) return true;
+  const unsigned long long delta = (1ull << 32) - 1ull;                    // live -1, returned +1
+  const unsigned long long old = atomicAdd(&tc->live_pending, delta);
+  if (uint32_t(old) > 1u) return true;
+  unsigned long long v = old + delta;
+  while ((v >> 32) != 0) {
+    const unsigned long long w = atomicCAS(&tc->live_pending, v, v - delta);   // take it back: live +1, returned -1
+    if (w == v) return false;   // the last live worker stays, with its task
     v = w;
   }
-  return false;   // the last live worker stays (its next fetch exits if the queue is drained)
+  return true;                  // claimed by a live taker: publish it and leave
 }
 
 // Q28 returned-task ring (long-task tenants only).  A retiring worker that

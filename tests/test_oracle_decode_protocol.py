@@ -171,7 +171,8 @@ def test_protocol_abort_needs_the_combined_word():
                     acts.append(("abort", i))
             return acts
 
-    cfg = P.Config(blocks=2, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1)], grid=1, abort=True)
+    cfg = P.Config(blocks=2, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1)], grid=1, abort=True,
+                   faa_abort=False)
     m = Split(cfg)
     with pytest.raises(P.ProtocolViolation):
         # explore every interleaving of the broken model
@@ -193,6 +194,67 @@ def test_protocol_abort_needs_the_combined_word():
                 y = copy.deepcopy(x)
                 y.apply(a)
                 stack.append(y)
+
+
+@pytest.mark.parametrize("cfg", [
+    P.Config(blocks=3, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1), (0, 1)], abort=True, faa_abort=False),
+    P.Config(blocks=4, iters=2, ranks=2, occ=1, lo=0, hi=1, resizes=[(0, 0)], abort=True, faa_abort=False),
+])
+def test_protocol_exhaustive_single_step_abort(cfg):
+    """Q28 with "abandon unless last" as one atomic step (the round-1 CAS loop)."""
+    assert P.explore(cfg) > 10
+
+
+@pytest.mark.parametrize("cfg", [
+    P.Config(blocks=2, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1)], grid=1, abort=True),
+    P.Config(blocks=2, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(0, 0), (1, 1)], abort=True),
+])
+def test_protocol_exhaustive_faa_abort(cfg):
+    """Q50: abandon-and-retire by one fetch-and-add on {live, returned}, the last
+    live worker taking its unit back (or, if a taker claimed it, publishing it
+    and leaving): exactly-once, no orphaned return, termination, in every
+    interleaving -- including a single-CTA grid, where the abandoning worker is
+    always the last.  (The abort configurations of test_protocol_exhaustive and
+    the random-seed runs use this model too: it is the default.)"""
+    assert P.explore(cfg) > 10
+
+
+def test_faa_abort_needs_the_take_back():
+    """Mutation: a last live worker that abandons by fetch-and-add and simply
+    leaves (no take-back) orphans its task -- the model must find it."""
+    class NoTakeBack(P.Model):
+        def apply(self, act):
+            if act[0] == "step" and self.ctas[act[1]][0] == P.ABORT_LAST:
+                c = self.ctas[act[1]]
+                self.ret_pub.append(c[4])
+                self.exit(c, False)
+                return
+            super().apply(act)
+
+    cfg = P.Config(blocks=2, iters=1, ranks=2, occ=1, lo=0, hi=1, resizes=[(1, 1)], grid=1, abort=True)
+    import copy
+    stack, seen, failed = [NoTakeBack(cfg)], set(), False
+    while stack and not failed:
+        x = stack.pop()
+        k = x.key()
+        if k in seen:
+            continue
+        seen.add(k)
+        try:
+            if x.done():
+                x.check_final()
+                continue
+            acts = x.actions()
+            if not acts:
+                raise P.ProtocolViolation("deadlock")
+            for a in acts:
+                y = copy.deepcopy(x)
+                y.apply(a)
+                y.check_step()
+                stack.append(y)
+        except P.ProtocolViolation:
+            failed = True
+    assert failed
 
 
 def test_grid_completion_waits_for_topup_blocks():
