@@ -1020,7 +1020,13 @@ void Server::drop_idle_grow(Queue& Q) {
 // a top-up grid for launch R on the queue's current range, sharing R's counter
 int Server::topup(Queue& Q, Launch& R, std::string* err) {
   static const bool dbg = std::getenv("SLATE_DEBUG") != nullptr;
-  if (dbg) fprintf(stderr, "[slate] grow: top-up for launch %llu on [%u, %u]\n", (unsigned long long)R.id, Q.lo, Q.hi);
+  if (dbg) {
+    double since = -1;   // host time since the queue's latest grow call (us)
+    for (auto it = Q.pending_resize.rbegin(); it != Q.pending_resize.rend(); ++it)
+      if (it->kind == 2) { since = now_us() - it->t0_us; break; }
+    fprintf(stderr, "[slate] grow: top-up for launch %llu on [%u, %u], %.1f us after the grow call\n",
+            (unsigned long long)R.id, Q.lo, Q.hi, since);
+  }
   const auto& g = R.desc.grid;
   cudaStream_t aux = Q.aux[Q.aux_next++ % Queue::kAux];
   cudaEvent_t ev_ctrl;   // the top-up starts after the resize word it must see (and after R started)
