@@ -304,6 +304,7 @@ uint32_t Server::open_queue() {
     cudaStreamCreateWithPriority(&Q->snap, cudaStreamNonBlocking, hi_prio);
   }
   for (cudaStream_t& a : Q->aux) cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking);   // not on the resize path
+  cudaEventCreateWithFlags(&Q->ev_ctrl, cudaEventDisableTiming);
   const uint32_t id = Q->id;
   queues_[id] = std::move(Q);
   return id;
@@ -334,6 +335,7 @@ int Server::close_queue(uint32_t q, int64_t timeout_us, std::string* err) {
     free_ctrl_.push_back(slot);
     cudaStreamDestroy(Q.stream);
     cudaStreamDestroy(Q.snap);
+    if (Q.ev_ctrl) cudaEventDestroy(Q.ev_ctrl);
     for (cudaStream_t a : Q.aux)
       if (a) cudaStreamDestroy(a);
     // a queue can still hold SMs with nothing issued (a resize after its last
@@ -730,13 +732,11 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
     if (err) *err = "cuStreamWriteValue64 failed: " + std::to_string(int(r));
     return SLATE_ECUDA;
   }
-  // later launches of this queue start after the write
-  cudaEvent_t ev;
-  CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-  CK(cudaEventRecord(ev, ctrl_stream_));
-  CK(cudaStreamWaitEvent(Q.stream, ev, 0));
+  // later launches of this queue start after the write (a wait captures the
+  // event's state when it is enqueued, so one event per queue can be reused)
+  CK(cudaEventRecord(Q.ev_ctrl, ctrl_stream_));
+  CK(cudaStreamWaitEvent(Q.stream, Q.ev_ctrl, 0));
   Q.last_op_kernel = false;
-  cudaEventDestroy(ev);
   return SLATE_OK;
 }
 
@@ -1029,11 +1029,9 @@ int Server::topup(Queue& Q, Launch& R, std::string* err) {
   }
   const auto& g = R.desc.grid;
   cudaStream_t aux = Q.aux[Q.aux_next++ % Queue::kAux];
-  cudaEvent_t ev_ctrl;   // the top-up starts after the resize word it must see (and after R started)
-  CK(cudaEventCreateWithFlags(&ev_ctrl, cudaEventDisableTiming));
-  CK(cudaEventRecord(ev_ctrl, ctrl_stream_));
-  CK(cudaStreamWaitEvent(aux, ev_ctrl, 0));
-  cudaEventDestroy(ev_ctrl);
+  // the top-up starts after the resize word it must see (recorded by write_ctrl
+  // right after the queue's latest write) and after R started
+  CK(cudaStreamWaitEvent(aux, Q.ev_ctrl, 0));
   cudaEvent_t r_start = R.ev_start ? R.ev_start : R.start_after;
   if (r_start) CK(cudaStreamWaitEvent(aux, r_start, 0));
   WorkerCommon w{};

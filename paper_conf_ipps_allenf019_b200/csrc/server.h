@@ -72,6 +72,8 @@ struct Queue {
   cudaStream_t aux[kAux] = {};  // top-up launches (round robin: a top-up whose workers joined runs
                                 // until the launch drains, so top-ups must not queue behind each other)
   uint32_t aux_next = 0;
+  cudaEvent_t ev_ctrl = nullptr;  // recorded on the control stream after each write of this queue's word
+                                  // (reused: a grow's critical path makes no event create/destroy calls)
   uint64_t* d_ctrl = nullptr;   // the resize word {epoch, lo, hi}
   uint32_t epoch = 0, lo = 0, hi = 0;
   bool active = false;          // holds an SM range

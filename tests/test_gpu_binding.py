@@ -146,8 +146,13 @@ def test_rank_log_under_resize_storm(name):
         ranges = set(zip(lo.tolist(), hi.tolist()))
         assert ranges <= requested, (name, ranges - requested)
         assert np.all((rank >= lo) & (rank <= hi) | (outside == 1)), name
-        # only the last live worker may keep a task outside the range (Q22): rare
-        assert outside.sum() <= max(4, B // 100), (name, int(outside.sum()))
+        # only the last live worker may keep a task outside the range (Q22), and
+        # only until a worker of the new range joins: a few tasks per resize.
+        # (With retire-and-give-back as one fetch-and-add, Q50, a GEMM pair
+        # whose range jumped away is left alone sooner than the top-up's pairs
+        # arrive -- 13 tiles of 1024 over 40 resizes were seen -- where the
+        # round-1 CAS loop had taken ~40 us per mass retirement.)
+        assert outside.sum() <= max(4, B // 100, 2 * resizes), (name, int(outside.sum()), resizes)
         assert len(ranges) >= 2 or resizes < 2, name   # the storm reached the workers
     finally:
         s.close()
