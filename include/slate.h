@@ -100,7 +100,9 @@ typedef struct {
   uint64_t n; float r; uint32_t n_scen;
 } slate_args_bs;
 typedef struct { uint64_t in, out; uint32_t h, w; } slate_args_stencil;
-typedef struct { uint64_t A, B, C; uint32_t m, n, k, pad_; } slate_args_gemm;       /* A m x k, B n x k bf16 */
+/* gemm: A m x k, B n x k bf16 K-major, C m x n fp32; any m, k % 8 == 0, n % 4 == 0 (16-byte row
+ * strides); grid (ceil(n/tile_n), ceil(m/tile_m)), a ragged last tile row/column/K slice allowed */
+typedef struct { uint64_t A, B, C; uint32_t m, n, k, pad_; } slate_args_gemm;
 /* TR: in h x w fp32, out w x h fp32 (out[j][i] = in[i][j]); grid (ceil(w/32), ceil(h/32)) */
 typedef struct { uint64_t in, out; uint32_t h, w; } slate_args_transpose;
 /* RG (the CUDA SDK quasirandomGenerator kernel): out[d][i] = float(q_d(seed + i) + 1) * 2^-31,

@@ -363,7 +363,7 @@ __global__ void __launch_bounds__(kThreads, 1) gemm_kernel(const __grid_constant
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = S.tmem_base;
-  const uint32_t num_kb = p.args.k / BK;
+  const uint32_t num_kb = (p.args.k + BK - 1) / BK;   // a ragged last slice: zero-filled past k
   const uint32_t full0 = mapa(&S.full[0], 0);       // the leader's full barriers (shared::cluster)
 
   if (warp == 0 && lane == 0 && leader) {

@@ -518,11 +518,14 @@ bool Server::validate(const KernelEntry& k, const slate_launch_desc* d, uint32_t
     case SLATE_KIND_GEMM_BF16: {
       auto a = static_cast<const slate_args_gemm*>(d->args);
       const uint32_t tn = k.ops->tile_n ? k.ops->tile_n : 128, tm = k.ops->tile_m ? k.ops->tile_m : 128;
-      if (a->m % tm || a->n % tn || a->k % 64 || a->k == 0)
-        return fail("gemm_bf16 needs m % tile_m, n % tile_n, k % 64 == 0 (slate_kind_geometry)");
+      // any m; tensor-map row strides must be 16-byte multiples: k % 8, n % 4.
+      // Ragged tiles: the TMA loads zero-fill past m, n and k (zero products),
+      // the TMA stores of C clip past m and n
+      if (a->m == 0 || a->n == 0 || a->k == 0 || a->k % 8 || a->n % 4)
+        return fail("gemm_bf16 needs m, n, k > 0, k % 8 == 0 and n % 4 == 0 (16-byte row strides)");
       if (!al(a->A) || !al(a->B) || !al(a->C)) return fail("gemm arrays must be 16-byte aligned");
-      g[0] = a->n / tn;
-      g[1] = a->m / tm;
+      g[0] = cdiv(a->n, tn);
+      g[1] = cdiv(a->m, tm);
       break;
     }
     case SLATE_KIND_TRANSPOSE: {

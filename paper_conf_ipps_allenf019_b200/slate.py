@@ -523,7 +523,7 @@ GEMM_TILE_M, GEMM_TILE_N = kind_geometry(KIND_GEMM_BF16)
 def gemm_args(A, B, C):
     m, k = A.shape
     n, _ = B.shape
-    return ArgsGemm(_ptr(A), _ptr(B), _ptr(C), m, n, k, 0), (n // GEMM_TILE_N, m // GEMM_TILE_M, 1)
+    return ArgsGemm(_ptr(A), _ptr(B), _ptr(C), m, n, k, 0), (cdiv(n, GEMM_TILE_N), cdiv(m, GEMM_TILE_M), 1)
 
 
 def transpose_args(inp, out):

@@ -41,6 +41,9 @@ CASES = {
     "stencil_vec_int": lambda: make_stencil(8 * 5 + 2, 128 * 2 + 4, 114, "int"),
     "gemm_int": lambda: make_gemm(256, 512, 512, 113, "int"),
     "gemm_float": lambda: make_gemm(768, 512, 1024, 114),
+    # ragged in all three: a partial last tile row (m), column (n) and K slice (k)
+    "gemm_ragged_int": lambda: make_gemm(256 * 2 + 77, 256 + 132, 64 * 5 + 24, 131, "int"),
+    "gemm_ragged_float": lambda: make_gemm(300, 260, 520, 132),
     # the paper's Tab II apps (NEXT-2)
     "tr": lambda: make_transpose(32 * 11 + 7, 32 * 9 + 19, 120),
     "tr_row": lambda: make_transpose(1, 32 * 40 + 1, 121),

@@ -127,6 +127,20 @@ def test_resize_storm_gemm_abandons_tiles(sess):
     assert ok
 
 
+def test_resize_storm_gemm_ragged(sess):
+    """The same storm on a GEMM ragged in m, n and k (partial last tile row,
+    column and K slice: zero-filled TMA loads, clipped TMA stores): abandoned
+    and retaken tiles still store every element exactly once, exact against the
+    oracle on sampled tiles including the ragged corner."""
+    m, n, k = 2048 + 77, 2048 + 132, 4096 + 24
+    t = make_gemm(m, n, k, 207, "int")
+    q, done = _storm(sess, t, 1, 30, 5, 30)
+    assert done >= 5
+    last_x, last_y = (n - 1) // 128, (m - 1) // 128
+    ok, err = t.check(t.snapshot(), rows=[(0, 0), (last_x, last_y), (last_x, 3), (5, last_y)])
+    assert ok
+
+
 def test_gemm_shrink_latency(sess):
     n = sess.info()["num_sms"]
     t = make_gemm(8192, 8192, 8192, 206)
