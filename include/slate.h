@@ -161,7 +161,7 @@ slate_status slate_get_info(slate_session* s, slate_info* out);
  * a client that frees a buffer while other tenants keep the server busy
  * relies on the driver's reference to the allocation until then.
  * Errors: EINVAL (null/zero range, not device memory), EIPC. */
-slate_status slate_share_buffer(slate_session* s, uint64_t dev_ptr, size_t bytes, uint64_t* handle);
+slate_status slate_share_buffer(slate_session* s, void* dev_ptr, size_t bytes, uint64_t* handle);
 slate_status slate_unshare_buffer(slate_session* s, uint64_t handle);
 
 /* ------------------------------------------------------------------ kernels */

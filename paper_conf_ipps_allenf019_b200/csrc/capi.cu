@@ -160,7 +160,8 @@ slate_status slate_get_info(slate_session* s, slate_info* out) {
   return rc == SLATE_OK ? rc : fail(s, rc, err);
 }
 
-slate_status slate_share_buffer(slate_session* s, uint64_t dev_ptr, size_t bytes, uint64_t* handle) {
+slate_status slate_share_buffer(slate_session* s, void* ptr, size_t bytes, uint64_t* handle) {
+  const uint64_t dev_ptr = reinterpret_cast<uint64_t>(ptr);
   if (!s || !handle || !dev_ptr || !bytes) return fail(s, SLATE_EINVAL, "null or empty buffer");
   std::lock_guard<std::mutex> g(s->mu);
   cudaPointerAttributes attr;

@@ -146,7 +146,7 @@ for _name, _args in [
     ("slate_attach", [ctypes.c_char_p, ctypes.c_int, _P(ctypes.c_void_p)]),
     ("slate_detach", [ctypes.c_void_p]),
     ("slate_get_info", [ctypes.c_void_p, _P(Info)]),
-    ("slate_share_buffer", [ctypes.c_void_p, c_u64, ctypes.c_size_t, _P(c_u64)]),
+    ("slate_share_buffer", [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, _P(c_u64)]),
     ("slate_unshare_buffer", [ctypes.c_void_p, c_u64]),
     ("slate_register_kernel", [ctypes.c_void_p, _P(KernelDesc), _P(c_u64)]),
     ("slate_launch", [ctypes.c_void_p, c_u64, _P(LaunchDesc), _P(c_u64)]),
