@@ -98,7 +98,9 @@ def test_corunners_run_only_on_their_own_ranks(name):
 STORMS = {
     "bs": (lambda: make_bs(1 << 21, 411, n_scen=64), 1),
     "stencil": (lambda: make_stencil(8192, 4096, 412), 4),
-    "spmv": (lambda: make_spmv(1 << 20, 413), 8),
+    # 2^22 rows: ~100 us per launch, so the storm's resizes land while it runs
+    # (a 2^20-row launch, ~25 us since the early slot release, could end first)
+    "spmv": (lambda: make_spmv(1 << 22, 413), 8),
     "gemm": (lambda: make_gemm(8192, 8192, 8192, 414, "int"), 1),
 }
 
