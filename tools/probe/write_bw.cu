@@ -79,6 +79,42 @@ __global__ void bulk_write(char* dst, uint32_t n_pieces, uint32_t* ctr, int k, u
   asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
+// reads and writes on the same SMs at once: odd CTAs stream-read (LDG.128,
+// summed), even CTAs stream-write (STG.128); each half has its own counter over
+// its own buffer.  Is ~100 GB/s of copy traffic per SM (copy tenant) the sum of
+// the two paths, or a limit of mixed traffic?
+__global__ void mixed(const float4* __restrict__ src, float4* __restrict__ dst, uint32_t n_pieces, uint32_t* ctr, int k,
+                      float* sink) {
+  __shared__ uint32_t s_p;
+  if ((int)smid() >= k) return;
+  const bool rd = blockIdx.x & 1;
+  uint32_t* c = ctr + (rd ? 1 : 0);
+  const uint32_t per = kPiece / 16;
+  float acc = 0.f;
+  const float4 v = make_float4(1.f, 2.f, 3.f, 4.f);
+  for (;;) {
+    if (threadIdx.x == 0) s_p = atomicAdd(c, 1u);
+    __syncthreads();
+    const uint32_t p = s_p;
+    __syncthreads();
+    if (p >= n_pieces) break;
+    if (rd) {
+      const float4* b = src + size_t(p) * per;
+      for (uint32_t i = threadIdx.x; i < per; i += blockDim.x * 4) {
+        float4 x[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) x[u] = __ldcs(b + i + u * blockDim.x);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc += x[u].x + x[u].y + x[u].z + x[u].w;
+      }
+    } else {
+      float4* b = dst + size_t(p) * per;
+      for (uint32_t i = threadIdx.x; i < per; i += blockDim.x) __stcs(b + i, v);
+    }
+  }
+  if (acc == 1234.5f) sink[0] = acc;
+}
+
 int main() {
   const size_t total = size_t(2) << 30;
   char *src, *dst; CK(cudaMalloc(&src, total)); CK(cudaMalloc(&dst, total)); CK(cudaMemset(src, 1, total));
@@ -101,7 +137,17 @@ int main() {
     printf("sms %3d  %-44s %8.1f GB/s  %6.1f GB/s per SM (traffic)\n", sms, what, gbs, gbs / sms);
   };
   char name[128];
+  float* sink; CK(cudaMalloc(&sink, 4));
+  uint32_t* ctr2; CK(cudaMalloc(&ctr2, 8));
   for (int sms : {74, 37}) {
+    // mixed: each half moves `total` bytes; traffic = 2 x total over the time both took
+    for (int cps : {2, 4}) {
+      snprintf(name, sizeof name, "mixed read+write %d CTA/SM x 512 thr", cps);
+      timeit([&] {
+        CK(cudaMemset(ctr2, 0, 8));
+        mixed<<<nsm * cps, 512>>>((const float4*)src, (float4*)dst, n_pieces, ctr2, sms, sink);
+      }, sms, name, 2.0);
+    }
     for (int cps : {1, 2, 4}) {
       snprintf(name, sizeof name, "stg.128 %d CTA/SM x 512 thr", cps);
       timeit([&] { stg_write<4><<<nsm * cps, 512>>>((float4*)dst, n_pieces, ctr, sms); }, sms, name, 1.0);
