@@ -219,9 +219,13 @@ def run_reference(args, world, rank):
 
 # ------------------------------------------------------------------ clocks
 class Clocks:
-    """SM clock and clock-event reasons sampled through NVML every 10 ms while
+    """SM clock and clock-event reasons sampled through NVML every 50 ms while
     the timed region runs (a thread; nvidia-smi -lms buffers its output and
-    lost the samples of sub-second regions)."""
+    lost the samples of sub-second regions).  Not more often: an NVML query --
+    from this process or another -- delays a resize-word write the GPU has not
+    yet taken by up to ~0.4 ms (measured: 1-2 of 10 C2 shrinks at 393/356 us
+    with a 10-ms sampler, none above 38 us without, tools/c2_timeline.py
+    TL_CLOCKS / TL_NVML_ONLY); the co-run makespan is unaffected."""
 
     NAMES = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
              ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
@@ -256,7 +260,7 @@ class Clocks:
                 self.reasons.update(n for n, b in bits if b and (r & b))
             except Exception:
                 pass
-            self.stop_ev.wait(0.01)
+            self.stop_ev.wait(0.05)
 
     def stop(self):
         if not self.th:
@@ -266,7 +270,7 @@ class Clocks:
         if not self.samples:
             return None
         return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
-                "reasons": sorted(self.reasons), "samples": len(self.samples), "source": "nvml, 10 ms"}
+                "reasons": sorted(self.reasons), "samples": len(self.samples), "source": "nvml, 50 ms"}
 
 
 # ------------------------------------------------------------------ the GPU workload

@@ -728,19 +728,52 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
   Q.cov_lo = std::max(Q.cov_lo, lo);   // workers outside the new range retire
   Q.cov_hi = std::min(Q.cov_hi, hi);
   const uint64_t v = pack_ctrl(Q.epoch, lo, hi);
+  static const bool dbg_t = std::getenv("SLATE_DEBUG_TIMING") != nullptr;
+  const double tw0 = dbg_t ? now_us() : 0.0;
   // a stream memory write needs no SM: it lands even while persistent workers fill every SM
   const CUresult r = reinterpret_cast<WriteValue64Fn>(write_value64_)(
       reinterpret_cast<CUstream>(ctrl_stream_), reinterpret_cast<CUdeviceptr>(Q.d_ctrl), v, 0);
+  if (dbg_t) fprintf(stderr, "[slate] write_ctrl q%u: WriteValue64 %.1f us\n", Q.id, now_us() - tw0);
   if (r != CUDA_SUCCESS) {
     if (err) *err = "cuStreamWriteValue64 failed: " + std::to_string(int(r));
     return SLATE_ECUDA;
   }
-  // later launches of this queue start after the write (a wait captures the
-  // event's state when it is enqueued, so one event per queue can be reused)
+  // later launches of this queue start after the write: the event is recorded
+  // now, and the queue's stream waits for it just before its next kernel
+  // (settle_ctrl).  Not here: the stream may hold a long batch of queued
+  // kernels, and a wait enqueued behind them can block the host until the
+  // driver's queue has room -- measured ~110 us, which delayed a grow's
+  // top-up by as much (the top-up waits for the event on its own stream).
   CK(cudaEventRecord(Q.ev_ctrl, ctrl_stream_));
-  CK(cudaStreamWaitEvent(Q.stream, Q.ev_ctrl, 0));
-  Q.last_op_kernel = false;
+  if (dbg_t) fprintf(stderr, "[slate] write_ctrl q%u: + EventRecord %.1f us\n", Q.id, now_us() - tw0);
+  Q.ctrl_wait_pending = true;
   return SLATE_OK;
+}
+
+// The first issued launch of the queue that has not finished its blocks, by
+// binary search: launches of a queue run in stream order, so the done ones are
+// a prefix of `issued`.  A batch's members stay in `issued` until the batch's
+// end event (no events between them), so the prefix can hold hundreds of
+// launches: the linear scans this replaces cost ~120 us of the server lock per
+// grow in C2 (640-launch SpMV jobs), delaying the top-up by as much.
+size_t Server::first_running(const Queue& Q) const {
+  size_t lo = 0, hi = Q.issued.size();
+  while (lo < hi) {
+    const size_t mid = (lo + hi) / 2;
+    const Launch& E = *launches_.at(Q.issued[mid]);
+    const bool done = E.slot < 0 || h_mirror_[E.slot].done != 0;
+    if (done) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+void Server::settle_ctrl(Queue& Q) {
+  if (!Q.ctrl_wait_pending) return;
+  cudaStreamWaitEvent(Q.stream, Q.ev_ctrl, 0);   // the latest record: the queue's latest word (a failure
+                                                 // here is sticky and surfaces at the next launch's CK)
+  Q.last_op_kernel = false;
+  Q.ctrl_wait_pending = false;
 }
 
 // ------------------------------------------------------------------ issue
@@ -855,6 +888,7 @@ void Server::drain_deferred(Queue& Q) {
 
 int Server::issue_now(Launch& L, Queue& Q, std::string* err) {
   const KindOps* ops = L.k->ops;
+  settle_ctrl(Q);
   for (cudaEvent_t e : Q.topup_ends) {   // stream semantics: the predecessor's top-up workers finish first
     CK(cudaStreamWaitEvent(Q.stream, e, 0));
     Q.last_op_kernel = false;
@@ -969,17 +1003,15 @@ int Server::grow_running(Queue& Q, uint32_t, uint32_t, std::string* err) {
   // it in stream order); launches before it that finished all their blocks but
   // are not yet retired by the poller do not count
   static const bool dbg = std::getenv("SLATE_DEBUG") != nullptr;
-  for (uint64_t lid : Q.issued)   // a fused co-run kernel (NEXT-1): its CTAs switch tenant, no launch
-    if (launches_[lid]->fused) return SLATE_OK;
+  if (Q.n_fused) return SLATE_OK;   // a fused co-run kernel (NEXT-1): its CTAs switch tenant, no launch
   if (!Q.issued.empty()) {
     // kinds whose last main CTA waits for all blocks (leave_main): top up the
     // RUNNING launch -- the first issued one that has not finished its blocks --
     // whatever is queued behind it (a grow then lands within a task, not a launch)
-    for (uint64_t lid : Q.issued) {
-      Launch& E = *launches_[lid];
-      if (E.slot < 0 || E.desc.mode == SLATE_MODE_STANDALONE || !E.k->ops->topup_anytime) break;
-      if (h_mirror_[E.slot].done) continue;
-      return topup(Q, E, err);
+    const size_t i = first_running(Q);
+    if (i < Q.issued.size()) {
+      Launch& E = *launches_[Q.issued[i]];
+      if (E.slot >= 0 && E.desc.mode != SLATE_MODE_STANDALONE && E.k->ops->topup_anytime) return topup(Q, E, err);
     }
   }
   if (Q.issued.empty() || !Q.pending.empty() || !Q.deferred.empty()) {
@@ -1176,6 +1208,8 @@ int Server::launch_fused(uint32_t qa, uint64_t ka, const slate_launch_desc* da, 
   CK(cudaEventCreate(&ev_end));
   CK(cudaEventCreateWithFlags(&ev_snap, cudaEventDisableTiming));
   // the kernel goes on A's stream after B's stream is ready (its resize word written)
+  settle_ctrl(A);
+  settle_ctrl(B);
   cudaEvent_t ev_b;
   CK(cudaEventCreateWithFlags(&ev_b, cudaEventDisableTiming));
   CK(cudaEventRecord(ev_b, B.stream));
@@ -1193,6 +1227,7 @@ int Server::launch_fused(uint32_t qa, uint64_t ka, const slate_launch_desc* da, 
     L->B = Bs[i];
     L->iters = Ks[i]->desc.iters ? Ks[i]->desc.iters : choose_iters(*Ks[i], Ds[i], Bs[i]);
     L->fused = true;
+    Qs[i]->n_fused += 1;
     L->slot = alloc_slot();
     std::memset(reinterpret_cast<void*>(h_mirror_ + L->slot), 0, sizeof(HostMirror));
     if (slot_zeroed_[L->slot] && cudaEventQuery(slot_zeroed_[L->slot]) != cudaSuccess)
@@ -1792,6 +1827,8 @@ void Server::release(Queue& Q) {
         track_resize(R, A.epoch, 2, t0);
         R.n_resizes += 1;
       }
+      if (std::getenv("SLATE_DEBUG_TIMING"))
+        fprintf(stderr, "[slate] survivor grow: %.1f us before grow_running (%zu issued)\n", now_us() - t0, A.issued.size());
       grow_running(A, old_lo, old_hi, &err);
     }
   }
@@ -1892,8 +1929,13 @@ void Server::resolve_resizes(Queue& Q, double t, const Launch* ended) {
   for (auto it = Q.pending_resize.begin(); it != Q.pending_resize.end();) {
     unsigned long long done_ns = 0;
     bool done = false;
-    for (uint64_t lid : Q.issued) {
-      const Launch& L = *launches_[lid];
+    // Only launches running at the call can stamp it: the oldest one that has
+    // not finished (first_running) and those after it, plus a few just before
+    // it that may have finished since -- not the whole done prefix, which in a
+    // batch can be hundreds of launches long (see first_running).
+    const size_t fr = first_running(Q);
+    for (size_t j = fr > 4 ? fr - 4 : 0; j < Q.issued.size(); ++j) {
+      const Launch& L = *launches_[Q.issued[j]];
       if (L.slot < 0) continue;
       const HostMirror& m = h_mirror_[L.slot];
       const unsigned long long w = it->kind == 1 ? m.shrink : m.join;
@@ -1902,12 +1944,21 @@ void Server::resolve_resizes(Queue& Q, double t, const Launch* ended) {
         done = true;
         break;
       }
-      if (it->kind == 1) break;   // only the oldest running launch can hold out-of-range workers
+      if (it->kind == 1 && j >= fr) break;   // only the oldest running launch can hold out-of-range workers
     }
     bool via_end = false;
     if (!done && ended && it->kind == 1 && ended->slot >= 0) {
-      done_ns = h_mirror_[ended->slot].done;
-      done = via_end = true;
+      // a launch that ended without retiring a worker ends the shrink -- but not
+      // one that had ended before the call (a batch's finished members retire
+      // together at the batch's end; their stamps predate the resize)
+      const unsigned long long e = h_mirror_[ended->slot].done;
+      double t0_dev;
+      const bool before = clk_base_ns_ && e && host_to_dev_us(it->t0_us, &t0_dev) &&
+                          double(int64_t(e - clk_base_ns_)) * 1e-3 < t0_dev;
+      if (!before) {
+        done_ns = e;
+        done = via_end = true;
+      }
     }
     if (done) {
       record_resize(*it, done_ns, t);
@@ -1963,6 +2014,7 @@ void Server::poll_once() {
       L.state = 2;
       finished_.push_back(L.id);
       if (L.error && !Q.first_error) Q.first_error = L.error;
+      if (L.fused && Q.n_fused) Q.n_fused -= 1;
       Q.issued.pop_front();
       if (Q.issued.empty()) Q.topup_ends.clear();
       else {                      // the next launch starts now, on the queue's current range

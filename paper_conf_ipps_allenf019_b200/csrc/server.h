@@ -74,6 +74,7 @@ struct Queue {
   uint32_t aux_next = 0;
   cudaEvent_t ev_ctrl = nullptr;  // recorded on the control stream after each write of this queue's word
                                   // (reused: a grow's critical path makes no event create/destroy calls)
+  bool ctrl_wait_pending = false; // the queue's stream has not waited for ev_ctrl yet (settle_ctrl)
   uint64_t* d_ctrl = nullptr;   // the resize word {epoch, lo, hi}
   uint32_t epoch = 0, lo = 0, hi = 0;
   bool active = false;          // holds an SM range
@@ -88,6 +89,7 @@ struct Queue {
   std::deque<uint64_t> pending; // launches waiting for SMs (AUTO/SOLO)
   std::deque<uint64_t> deferred;  // granted SMs but waiting for a control block (stream order)
   std::deque<uint64_t> issued;  // issued, not complete (stream order)
+  uint32_t n_fused = 0;         // fused co-run launches (NEXT-1) among `issued`
   std::vector<cudaEvent_t> topup_ends;  // top-ups of the last issued launch: successors wait for all
   std::vector<uint64_t> open_batch;     // issued launches of the current batch, no end event yet
   bool last_op_kernel = false;          // the last op on `stream` is the last issued worker kernel (PDL)
@@ -153,6 +155,8 @@ class Server {
   void drain_deferred(Queue& Q);
   void fail_launch(Launch& L, int code);
   int write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool immediate, std::string* err);
+  void settle_ctrl(Queue& Q);   // the queue's stream waits for its latest resize-word write
+  size_t first_running(const Queue& Q) const;   // index in Q.issued of the first launch not done
   int grow_running(Queue& Q, uint32_t old_lo, uint32_t old_hi, std::string* err);
   int topup(Queue& Q, Launch& R, std::string* err);
   void drop_idle_grow(Queue& Q);

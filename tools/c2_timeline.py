@@ -27,12 +27,31 @@ w.split = 0
 w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
 print("profiles", json.dumps({"a": [pa["category_name"], pa["solo_ms"]], "b": [pb["category_name"], pb["solo_ms"]]}))
 flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)
-for rep in range(3):
+clk = bench.Clocks(0) if os.environ.get("TL_CLOCKS") else None   # the bench's NVML sampler, as in its timed region
+if os.environ.get("TL_NVML_ONLY"):   # diagnostics: one NVML call kind every 10 ms in a thread ("clock" or "reasons")
+    import threading
+    import pynvml as N
+    N.nvmlInit()
+    h = N.nvmlDeviceGetHandleByIndex(0)
+    which = os.environ["TL_NVML_ONLY"]
+
+    def _poll():
+        while True:
+            if which == "clock":
+                N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
+            else:
+                N.nvmlDeviceGetCurrentClocksEventReasons(h)
+            import time as _t
+            _t.sleep(0.01)
+    threading.Thread(target=_poll, daemon=True).start()
+REPS = int(os.environ.get("TL_REPS", "3"))
+for rep in range(REPS):
     bench.flush_l2(flush)
     mk, ta, tb, qa, qb, ja, jb = bench.run_schedule("slate", w, sA, sB, kA, kB, S)
     t0 = min(min(q["start_ms"] for q in qa), min(q["start_ms"] for q in qb))
-    print("rep %d makespan %.3f ms  turnaround A %.3f  B %.3f" % (rep, mk, ta, tb))
-    if rep < 2:
+    rz = [(k, round(v, 1)) for q in qa + qb for k, v in zip(q["resize_kind"], q["resize_us"])]
+    print("rep %d makespan %.3f ms  turnaround A %.3f  B %.3f  resizes %s" % (rep, mk, ta, tb, rz))
+    if rep < REPS - 1:
         continue
     for name, qs in (("A", qa), ("B", qb)):
         last = None
@@ -43,3 +62,5 @@ for rep in range(3):
                       (name, i, q["start_ms"] - t0, q["end_ms"] - t0, q["sm_lo"], q["sm_hi"], q["n_resizes"],
                        q["n_topups"], list(zip(q["resize_kind"], [round(v, 1) for v in q["resize_us"]]))))
                 last = key
+if clk:
+    print("clocks", clk.stop())
