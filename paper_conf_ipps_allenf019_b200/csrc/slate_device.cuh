@@ -115,7 +115,14 @@ struct WorkerParams {
 // running launch needed (one C4 run stalled 320 ms); once every task is handed
 // out a top-up has nothing left to run.
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
-__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+#ifndef SLATE_EARLY_TRIGGER
+#define SLATE_EARLY_TRIGGER 1   // experiment switch: 0 = the next grid of a batch launches when this one completes (measured: C2 32.2-32.5 ms instead of 31.9, C4 shrink tail unchanged)
+#endif
+__device__ __forceinline__ void pdl_trigger() {
+#if SLATE_EARLY_TRIGGER
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
+}
 
 // ------------------------------------------------------------------ decode (Lst2 (4))
 struct BlockWalk {
