@@ -245,22 +245,24 @@ class Clocks:
             phys = int(vis.split(",")[index]) if vis and vis.split(",")[index].strip().isdigit() else index
             self.N, self.h = N, N.nvmlDeviceGetHandleByIndex(phys)
             self.max_mhz = N.nvmlDeviceGetMaxClockInfo(self.h, N.NVML_CLOCK_SM)
+            self._sample()   # the first sample before the timed work starts (the recipe: start before)
             self.th = threading.Thread(target=self._run, daemon=True)
             self.th.start()
         except Exception:
             self.th = None
 
-    def _run(self):
+    def _sample(self):
         N = self.N
-        bits = [(n, getattr(N, c, 0)) for n, c in self.NAMES]
-        while not self.stop_ev.is_set():
-            try:
-                self.samples.append(N.nvmlDeviceGetClockInfo(self.h, N.NVML_CLOCK_SM))
-                r = N.nvmlDeviceGetCurrentClocksEventReasons(self.h)
-                self.reasons.update(n for n, b in bits if b and (r & b))
-            except Exception:
-                pass
-            self.stop_ev.wait(0.05)
+        try:
+            self.samples.append(N.nvmlDeviceGetClockInfo(self.h, N.NVML_CLOCK_SM))
+            r = N.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            self.reasons.update(n for n, c in self.NAMES if getattr(N, c, 0) and (r & getattr(N, c, 0)))
+        except Exception:
+            pass
+
+    def _run(self):
+        while not self.stop_ev.wait(0.05):
+            self._sample()
 
     def stop(self):
         if not self.th:
@@ -585,7 +587,8 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     sched = {k: summary(v) for k, v in base.items()}
     sched["slate_corun"] = summary(med)
     qa, qb = med[3], med[4]
-    resize = [v for q in qa + qb for v in q["resize_us"]]
+    # resize latencies of every timed step (the median step alone holds two)
+    resize = [v for r in steps_out for q in r[3] + r[4] for v in q["resize_us"]]
     mk = med[0]
     peak_hbm = float(peaks.get("hbm_gbs", 6650.0))
     peak_fp32 = info["peak_fp32_gflops"] / 1e3
@@ -659,6 +662,7 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
             "resize_us": {"n": len(resize), "p50": round(statistics.median(resize), 2) if resize else None,
                           "p99": round(float(np.percentile(resize, 99)), 2) if resize else None,
                           "max": round(max(resize), 2) if resize else None,
+                          "over_50us": sum(1 for v in resize if v > 50.0), "scope": "every timed step",
                           "topups": sum(q["n_topups"] for q in qa + qb)},
             "split_sms_b": w.split, "arrival_ms": round(w.arrival_ms, 3),
             "utilisation": util, "profiles": {w.a.name: prof_view(pa), w.b.name: prof_view(pb)}, "roofline": roof}

@@ -1885,7 +1885,9 @@ void Server::track_resize(Launch& R, uint32_t epoch, int kind, double t0) {
     }
   }
   if (R.resize_us.size() >= 16) return;
-  Q.pending_resize.push_back({epoch, kind, t0, R.id, int(R.resize_us.size())});
+  const size_t fr = first_running(Q);
+  const uint64_t run = fr < Q.issued.size() ? Q.issued[fr] : (Q.issued.empty() ? 0 : Q.issued.back());
+  Q.pending_resize.push_back({epoch, kind, t0, R.id, int(R.resize_us.size()), run});
   R.resize_us.push_back(-1);
   R.resize_kind.push_back(uint8_t(kind));
 }
@@ -1929,12 +1931,13 @@ void Server::resolve_resizes(Queue& Q, double t, const Launch* ended) {
   for (auto it = Q.pending_resize.begin(); it != Q.pending_resize.end();) {
     unsigned long long done_ns = 0;
     bool done = false;
-    // Only launches running at the call can stamp it: the oldest one that has
-    // not finished (first_running) and those after it, plus a few just before
-    // it that may have finished since -- not the whole done prefix, which in a
-    // batch can be hundreds of launches long (see first_running).
+    // Only launches running at the call can stamp it: from the one that was
+    // running then (recorded at the call; it may have finished since -- the
+    // poller cannot run while a long launch_n holds the lock) onward -- not the
+    // whole done prefix, which in a batch can be hundreds of launches long
     const size_t fr = first_running(Q);
-    for (size_t j = fr > 4 ? fr - 4 : 0; j < Q.issued.size(); ++j) {
+    const size_t j0 = size_t(std::lower_bound(Q.issued.begin(), Q.issued.end(), it->run) - Q.issued.begin());
+    for (size_t j = std::min(j0, fr); j < Q.issued.size(); ++j) {
       const Launch& L = *launches_[Q.issued[j]];
       if (L.slot < 0) continue;
       const HostMirror& m = h_mirror_[L.slot];

@@ -95,7 +95,8 @@ struct Queue {
   bool last_op_kernel = false;          // the last op on `stream` is the last issued worker kernel (PDL)
   // resize latencies being measured (Q30): epoch, kind (1 shrink, 2 grow), host
   // t0, and where the result goes (launch id, index in its resize_us)
-  struct PendingResize { uint32_t epoch; int kind; double t0_us; uint64_t lid; int idx; };
+  // lid: the launch the latency is recorded on; run: the queue's running launch at the call
+  struct PendingResize { uint32_t epoch; int kind; double t0_us; uint64_t lid; int idx; uint64_t run = 0; };
   std::vector<PendingResize> pending_resize;
   bool closed = false;
   int first_error = 0;          // the first cudaError_t a launch of this queue completed with
