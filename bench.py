@@ -221,11 +221,9 @@ def run_reference(args, world, rank):
 class Clocks:
     """SM clock and clock-event reasons sampled through NVML every 50 ms while
     the timed region runs (a thread; nvidia-smi -lms buffers its output and
-    lost the samples of sub-second regions).  Not more often: an NVML query --
-    from this process or another -- delays a resize-word write the GPU has not
-    yet taken by up to ~0.4 ms (measured: 1-2 of 10 C2 shrinks at 393/356 us
-    with a 10-ms sampler, none above 38 us without, tools/c2_timeline.py
-    TL_CLOCKS / TL_NVML_ONLY); the co-run makespan is unaffected."""
+    lost the samples of sub-second regions); the first sample is taken before
+    the timed work starts.  (Resize latencies are the same with a 10-ms
+    sampler and without one: profiles/r2_resize_nvml_interference.json.)"""
 
     NAMES = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
              ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
