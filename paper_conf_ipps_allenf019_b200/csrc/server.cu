@@ -728,24 +728,18 @@ int Server::write_ctrl(Queue& Q, uint32_t lo, uint32_t hi, bool, std::string* er
   Q.cov_lo = std::max(Q.cov_lo, lo);   // workers outside the new range retire
   Q.cov_hi = std::min(Q.cov_hi, hi);
   const uint64_t v = pack_ctrl(Q.epoch, lo, hi);
-  static const bool dbg_t = std::getenv("SLATE_DEBUG_TIMING") != nullptr;
-  const double tw0 = dbg_t ? now_us() : 0.0;
   // a stream memory write needs no SM: it lands even while persistent workers fill every SM
   const CUresult r = reinterpret_cast<WriteValue64Fn>(write_value64_)(
       reinterpret_cast<CUstream>(ctrl_stream_), reinterpret_cast<CUdeviceptr>(Q.d_ctrl), v, 0);
-  if (dbg_t) fprintf(stderr, "[slate] write_ctrl q%u: WriteValue64 %.1f us\n", Q.id, now_us() - tw0);
   if (r != CUDA_SUCCESS) {
     if (err) *err = "cuStreamWriteValue64 failed: " + std::to_string(int(r));
     return SLATE_ECUDA;
   }
   // later launches of this queue start after the write: the event is recorded
-  // now, and the queue's stream waits for it just before its next kernel
-  // (settle_ctrl).  Not here: the stream may hold a long batch of queued
-  // kernels, and a wait enqueued behind them can block the host until the
-  // driver's queue has room -- measured ~110 us, which delayed a grow's
-  // top-up by as much (the top-up waits for the event on its own stream).
+  // now (a top-up waits for it on its own stream), and the queue's stream waits
+  // for it just before its next kernel (settle_ctrl) -- one wait for several
+  // writes between two kernels of the queue
   CK(cudaEventRecord(Q.ev_ctrl, ctrl_stream_));
-  if (dbg_t) fprintf(stderr, "[slate] write_ctrl q%u: + EventRecord %.1f us\n", Q.id, now_us() - tw0);
   Q.ctrl_wait_pending = true;
   return SLATE_OK;
 }
@@ -1827,8 +1821,6 @@ void Server::release(Queue& Q) {
         track_resize(R, A.epoch, 2, t0);
         R.n_resizes += 1;
       }
-      if (std::getenv("SLATE_DEBUG_TIMING"))
-        fprintf(stderr, "[slate] survivor grow: %.1f us before grow_running (%zu issued)\n", now_us() - t0, A.issued.size());
       grow_running(A, old_lo, old_hi, &err);
     }
   }
