@@ -115,6 +115,26 @@ def test_shrink_then_grow_latency(sess):
     assert len(lat) == 2 and all(0 < v < 5000 for v in lat), lat
 
 
+def test_shrink_latency_inside_a_batch(sess):
+    """Resize accounting in a batched job (reading Q50 era fix): the finished
+    members of a batch stay issued until the batch's end event, and a shrink
+    used to be 'resolved' by the end stamp of one that had finished before the
+    resize (0 us).  Shrink the queue in the middle of a 200-launch triad job:
+    the shrink is timed from the call to the out-of-range workers' retirement
+    -- above 0, and well under a launch of the job."""
+    n = sess.info()["num_sms"]
+    t = make_triad(1 << 24, 208)
+    k = sess.register_kernel(t.kind)
+    ids = sess.launch_n(k, t.args, t.grid, 200, placement=S.PLACE_CORUN, sm=(0, n - 1))
+    time.sleep(0.003)                     # well into the job: many members already finished
+    st = sess.resize(ids[0], 0, n // 2 - 1)
+    sess.sync(0)
+    lats = [v for i in ids for kd, v in zip(sess.query(i)["resize_kind"], sess.query(i)["resize_us"]) if kd == "shrink"]
+    if st == S.DONE or not lats:
+        pytest.skip("the job ended before the resize landed")
+    assert all(0 < v < 200 for v in lats), lats
+
+
 def test_resize_storm_gemm_abandons_tiles(sess):
     """tcgen05 GEMM under a resize storm: workers leaving the range abandon their
     tile mid-K and give it back (Q28); every tile is still stored exactly once,
