@@ -454,12 +454,14 @@ def flush_l2(buf):
     torch.cuda.synchronize()
 
 
-def median_schedule(name, w, sA, sB, kA, kB, S, flush, reps):
+def median_schedule(name, w, sA, sB, kA, kB, S, flush, reps, spread=None):
     rs = []
     for _ in range(reps):
         flush_l2(flush)
         rs.append(run_schedule(name, w, sA, sB, kA, kB, S))
     rs.sort(key=lambda r: r[0])
+    if spread is not None:   # makespan min / max over the timed runs
+        spread[name] = {"runs": len(rs), "min_ms": round(rs[0][0], 3), "max_ms": round(rs[-1][0], 3)}
     return rs[len(rs) // 2]
 
 
@@ -515,6 +517,7 @@ def prof_view(p):
 def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     """Profiles, baselines and (if `timed` is None) `steps` timed Slate co-run steps.
     Returns a dict of results; `timed(callback)` lets the caller bracket the timed loop."""
+    import torch
     info = sA.info()
     kA, kB = sA.register_kernel(w.a.kind), sA.register_kernel(w.b.kind)
     pa = sA.profile(kA, w.a.args, w.a.grid, S.PROF_CURVE)
@@ -532,11 +535,19 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     jb = {k: v * w.b.reps for k, v in cb.items()}
     w.split, _ = S.choose_split(ja, jb, w.n_sms, 2, lo_b, hi_b)
     w.arrival_ms = w.arrival_frac * pa["solo_ms"] * w.a.reps
-    base = {}
+    base, spread = {}, {}
+    # every schedule gets 3 warm-up runs, then 10 timed runs; the
+    # median is reported with the min and max.  Each schedule starts from an
+    # idle GPU (a 0.2-s pause): back to back, ~100 runs of a 1-kW GEMM pair
+    # (C3) left the co-run measured last in a lower-clock state (1.86 ms
+    # against 1.74 ms; tools/c3_repeat.py showed the same drift in long series)
     for name in ("seq_cuda", "seq_cuda_ba", "seq_slate", "seq_slate_ba", "streams", "slate_table", "slate_forced",
                  "slate_antt"):
-        run_schedule(name, w, sA, sB, kA, kB, S)
-        base[name] = median_schedule(name, w, sA, sB, kA, kB, S, flush, 3)
+        torch.cuda.synchronize()
+        time.sleep(0.2)
+        for _ in range(3):
+            run_schedule(name, w, sA, sB, kA, kB, S)
+        base[name] = median_schedule(name, w, sA, sB, kA, kB, S, flush, 10, spread)
     # every job's solo time: alone on the whole GPU, as original kernels or as
     # workers (Slate-solo), whichever is faster, in either order -- the best
     # sequential schedule is the baseline of every gain
@@ -553,6 +564,8 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     # A first (B arriving at `arr` waits for A), or B first (as if B were there at 0)
     seq_orders = {"a_first": stp_antt([solo_a, solo_b], [solo_a, max(solo_a + solo_b - arr, 1e-9)]),
                   "b_first": stp_antt([solo_a, solo_b], [solo_a + solo_b, solo_b])}
+    torch.cuda.synchronize()
+    time.sleep(0.2)                       # the co-run starts from an idle GPU too
     for _ in range(max(3, warmup)):
         flush_l2(flush)
         run_schedule("slate", w, sA, sB, kA, kB, S)
@@ -584,6 +597,10 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
 
     sched = {k: summary(v) for k, v in base.items()}
     sched["slate_corun"] = summary(med)
+    for k in base:
+        sched[k]["makespan_spread"] = spread[k]
+    sched["slate_corun"]["makespan_spread"] = {"runs": len(steps_out), "min_ms": round(min(r[0] for r in steps_out), 3),
+                                               "max_ms": round(max(r[0] for r in steps_out), 3)}
     qa, qb = med[3], med[4]
     # resize latencies of every timed step (the median step alone holds two)
     resize = [v for r in steps_out for q in r[3] + r[4] for v in q["resize_us"]]
