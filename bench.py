@@ -660,6 +660,20 @@ def evaluate(w, S, sA, sB, flush, steps, warmup, peaks, timed=None):
     roof["solo"] = {"avg_launch_ms": round(solo_avg, 5),
                     "achieved": round(roof["achieved"] * avg / solo_avg, 3 if roof["unit"] != "GB/s" else 1),
                     "frac": round(roof["frac"] * avg / solo_avg, 4)}
+    if roof["kernel"] == "spmv::spmv_worker":
+        # the bound per SM (profiles/r2_spmv_limits.md): the worker's compute
+        # goes through the SM's shared-memory SRAM -- 0.25 LSU wavefronts (32 B)
+        # per nonzero measured by ncu, plus the bulk copies' 8 B per nonzero
+        # written into it -- against 128 B/clk: 3.2 nonzeros per clock, ~55 GB/s
+        # of SpMV traffic per SM; on its co-run share the HBM fraction is not
+        # its roofline position
+        ceil_gbs = 128.0 / 40.0 * 1.965e9 * (147e6 / 16.78e6) / 1e9
+        per_sm = roof["achieved"] / max(share, 1)
+        roof["per_sm"] = {"achieved_gbs": round(per_sm, 1), "ceiling_gbs": round(ceil_gbs, 1),
+                          "frac": round(per_sm / ceil_gbs, 4),
+                          "ceiling_source": "shared-memory SRAM: 40 B per nonzero (32 B LSU wavefronts, ncu, + 8 B "
+                                            "bulk-copy writes) at 128 B/clk x 1.965 GHz; 8.76 B of SpMV traffic per "
+                                            "nonzero (profiles/r2_spmv_limits.md)"}
     roof["traffic"] = None
     ncu_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(ncu_path):
